@@ -1,0 +1,194 @@
+"""Python face of the C oracle (oracle/ffsva_oracle.c) — TEST INFRASTRUCTURE ONLY.
+
+Only tests/, __graft_entry__.smoke() and bench.py's CPU-baseline leg
+(``cpu_baseline`` and ``--impl reference``) import this module. It is ctypes
+marshalling around the plain single-threaded C definitions plus
+``filter_frames``, which applies them frame by frame in the paper's order
+(SDD: downsample -> distance -> threshold; survivors in order,
+L143; SNM -> Eq. (2) decision, L159-L165, L193).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+u8p = ctypes.c_void_p
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} missing: run __graft_entry__.build()")
+        L = ctypes.CDLL(LIB_PATH)
+        L.orc_box_downsample.argtypes = [u8p, ctypes.c_int32, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32,
+                                         ctypes.c_int32, u8p]
+        L.orc_reference.argtypes = [u8p, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
+                                    ctypes.c_int64, ctypes.c_int32, ctypes.c_int32, u8p]
+        L.orc_ssd.argtypes = [u8p, u8p, ctypes.c_int64]
+        L.orc_ssd.restype = ctypes.c_uint64
+        L.orc_threshold.argtypes = [ctypes.c_double, ctypes.c_int64]
+        L.orc_threshold.restype = ctypes.c_uint64
+        L.orc_sdd_pass.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
+        L.orc_sdd_pass.restype = ctypes.c_int32
+        L.orc_compact.argtypes = [u8p, ctypes.c_int32, u8p]
+        L.orc_compact.restype = ctypes.c_int32
+        L.orc_round_bf16.argtypes = [ctypes.c_double]
+        L.orc_round_bf16.restype = ctypes.c_double
+        L.orc_conv3x3.argtypes = [u8p, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, u8p, u8p, ctypes.c_int32, u8p]
+        L.orc_maxpool2.argtypes = [u8p, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, u8p]
+        L.orc_snm_forward.argtypes = [u8p, ctypes.c_int32, ctypes.c_int32, u8p, ctypes.c_int32, ctypes.c_int32,
+                                      ctypes.c_int32]
+        L.orc_snm_forward.restype = ctypes.c_double
+        L.orc_snm_n_params.argtypes = [ctypes.c_int32] * 4
+        L.orc_snm_n_params.restype = ctypes.c_int64
+        L.orc_tpre.argtypes = [ctypes.c_double] * 3
+        L.orc_tpre.restype = ctypes.c_double
+        L.orc_logit.argtypes = [ctypes.c_double]
+        L.orc_logit.restype = ctypes.c_double
+        L.orc_decide.argtypes = [ctypes.c_double, ctypes.c_double, ctypes.c_double, ctypes.c_double, u8p, u8p]
+        _lib = L
+    return _lib
+
+
+def _c(a, dtype):
+    return np.ascontiguousarray(a, dtype=dtype)
+
+
+def box_downsample(frame: np.ndarray, width: int, dw: int, dh: int) -> np.ndarray:
+    """C1. frame: (H, pitch) uint8 with 3*width <= pitch. Returns (dh, dw, 3) uint8."""
+    f = _c(frame, np.uint8)
+    H, pitch = f.shape
+    out = np.zeros((dh, dw, 3), dtype=np.uint8)
+    lib().orc_box_downsample(f.ctypes.data, width, H, pitch, dw, dh, out.ctypes.data)
+    return out
+
+
+def reference(frames: np.ndarray, width: int, dw: int, dh: int) -> np.ndarray:
+    """C2. frames: (K, H, pitch) uint8 background frames. Returns (dh, dw, 3) uint8."""
+    f = _c(frames, np.uint8)
+    K, H, pitch = f.shape
+    out = np.zeros((dh, dw, 3), dtype=np.uint8)
+    lib().orc_reference(f.ctypes.data, K, H * pitch, width, H, pitch, dw, dh, out.ctypes.data)
+    return out
+
+
+def ssd(a: np.ndarray, b: np.ndarray) -> int:
+    """C3 sum of squared differences (u64)."""
+    a = _c(a, np.uint8).ravel()
+    b = _c(b, np.uint8).ravel()
+    assert a.size == b.size
+    return int(lib().orc_ssd(a.ctypes.data, b.ctypes.data, a.size))
+
+
+def threshold(delta_diff: float, n_values: int) -> int:
+    """C3 T = floor(delta_diff * N)."""
+    return int(lib().orc_threshold(delta_diff, n_values))
+
+
+def sdd_pass(ssd_value: int, T: int) -> int:
+    return int(lib().orc_sdd_pass(ssd_value, T))
+
+
+def compact(pass_mask) -> np.ndarray:
+    """C4 survivors in batch order."""
+    p = _c(pass_mask, np.uint8)
+    idx = np.zeros(max(1, p.size), dtype=np.int32)
+    m = lib().orc_compact(p.ctypes.data, p.size, idx.ctypes.data)
+    return idx[:m].copy()
+
+
+def round_bf16(x: float) -> float:
+    return float(lib().orc_round_bf16(x))
+
+
+def conv3x3(inp: np.ndarray, w: np.ndarray, b: np.ndarray | None = None) -> np.ndarray:
+    """C6 single conv layer. inp (C, H, W), w (K, C, 3, 3), b (K,) -> (K, H, W) float64."""
+    x = _c(inp, np.float64)
+    wt = _c(w, np.float64)
+    C, H, W = x.shape
+    K = wt.shape[0]
+    out = np.zeros((K, H, W), dtype=np.float64)
+    bb = _c(b, np.float64) if b is not None else None
+    lib().orc_conv3x3(x.ctypes.data, C, H, W, wt.ctypes.data, bb.ctypes.data if bb is not None else None, K,
+                      out.ctypes.data)
+    return out
+
+
+def maxpool2(inp: np.ndarray) -> np.ndarray:
+    x = _c(inp, np.float64)
+    C, H, W = x.shape
+    out = np.zeros((C, H // 2, W // 2), dtype=np.float64)
+    lib().orc_maxpool2(x.ctypes.data, C, H, W, out.ctypes.data)
+    return out
+
+
+def snm_n_params(h: int = 50, w: int = 50, c1: int = 16, c2: int = 32) -> int:
+    return int(lib().orc_snm_n_params(h, w, c1, c2))
+
+
+def snm_forward(d50: np.ndarray, params: np.ndarray, c1: int = 16, c2: int = 32, bf16_emul: bool = False) -> float:
+    """C5 + C6. d50: (h, w, 3) uint8; params packed float32 (C6 order). Returns the fp64 logit."""
+    d = _c(d50, np.uint8)
+    h, w, _ = d.shape
+    p = _c(params, np.float32)
+    assert p.size == snm_n_params(h, w, c1, c2)
+    return float(lib().orc_snm_forward(d.ctypes.data, h, w, p.ctypes.data, c1, c2, int(bf16_emul)))
+
+
+def tpre(c_low: float, c_high: float, filter_degree: float) -> float:
+    """PAPER.md L193 Eq. (2)."""
+    return float(lib().orc_tpre(c_low, c_high, filter_degree))
+
+
+def logit(t: float) -> float:
+    return float(lib().orc_logit(t))
+
+
+def decide(logit_value: float, c_low: float, c_high: float, filter_degree: float):
+    """C7 -> (pass, class)."""
+    p = np.zeros(1, dtype=np.uint8)
+    c = np.zeros(1, dtype=np.uint8)
+    lib().orc_decide(logit_value, c_low, c_high, filter_degree, p.ctypes.data, c.ctypes.data)
+    return int(p[0]), int(c[0])
+
+
+def filter_frames(frames, width: int, refs, deltas, snm_params, c_low, c_high, filter_degree,
+                  sdd_grid=(100, 100), snm_grid=(50, 50), bf16_emul: bool = False, run_snm: bool = True):
+    """The whole cascade on a list of frames, one frame at a time (no batching: C8 says batching never
+    changes per-frame results).
+
+    frames[i]: (H, pitch) uint8; refs[i]: (sdd_h, sdd_w, 3) reference of frame i's stream; deltas[i]:
+    delta_diff; snm_params[i]: packed params (or None); c_low/c_high/filter_degree: per-frame sequences.
+    Returns dict of per-frame arrays: d100, d50, ssd, sdd_pass, survivor_idx, logit, snm_pass, snm_class."""
+    n = len(frames)
+    dw, dh = sdd_grid
+    sw, sh = snm_grid
+    N = dw * dh * 3
+    d100 = np.zeros((n, dh, dw, 3), np.uint8)
+    d50 = np.zeros((n, sh, sw, 3), np.uint8)
+    ssd_v = np.zeros(n, np.uint64)
+    sp = np.zeros(n, np.uint8)
+    for i in range(n):
+        d100[i] = box_downsample(frames[i], width, dw, dh)
+        d50[i] = box_downsample(frames[i], width, sw, sh)
+        ssd_v[i] = ssd(d100[i], refs[i])
+        sp[i] = sdd_pass(int(ssd_v[i]), threshold(deltas[i], N))
+    surv = compact(sp)
+    sidx = np.full(n, -1, np.int32)
+    sidx[surv] = np.arange(surv.size, dtype=np.int32)
+    lg = np.full(n, np.nan, np.float64)
+    npass = np.zeros(n, np.uint8)
+    ncls = np.zeros(n, np.uint8)
+    if run_snm:
+        for i in surv:
+            lg[i] = snm_forward(d50[i], snm_params[i], bf16_emul=bf16_emul)
+            npass[i], ncls[i] = decide(lg[i], c_low[i], c_high[i], filter_degree[i])
+    return dict(d100=d100, d50=d50, ssd=ssd_v, sdd_pass=sp, survivors=surv, survivor_idx=sidx, logit=lg,
+                snm_pass=npass, snm_class=ncls)
