@@ -1,0 +1,195 @@
+/*
+ * ffsva.h — C-ABI of the B200-native FFS-VA prepositive filter cascade (SDD + SNM).
+ *
+ * The method (Zhang et al., "FFS-VA: A Fast Filtering System for Large-scale Video Analytics", ICPP 2018;
+ * /root/reference/PAPER.md line numbers) filters the frames of many concurrent surveillance streams:
+ *   SDD  (§3.2.1): downsample each frame to 100x100 (L155, L187), distance to the stream's
+ *        reference image (average of background frames, L151) by MSE, drop the frame if MSE <= delta_diff;
+ *   queue (L143 §3.1.2): survivors go to the stream's SNM queue in arrival order;
+ *   SNM  (L157-L167 §3.2.2): a per-stream three-layer CNN (CONV, CONV, FC; L159) on a 50x50 resize (L167)
+ *        outputs the probability c of the target; frames with c >= t_pre pass (L165), where
+ *        t_pre = (c_high - c_low) * FilterDegree + c_low (Eq. (2));
+ *   dynamic batching (L219-L223 §4.3.2): each SNM cycle pops min(BatchSize, queue depth) frames of a stream.
+ * Exact readings of what the paper leaves open are in DESIGN.md "Readings".
+ *
+ * Conventions for every function:
+ *   - returns ffsva_status: FFSVA_OK (0) or a negative error; ffsva_last_error() describes the last error of
+ *     the calling thread;
+ *   - all argument validation happens before any GPU work; on error nothing is written to outputs;
+ *   - FFSVA_ECUDA is sticky per device: after it the caller should close that device's streams;
+ *   - calls for one device are serialised by a per-device mutex; a stream handle must not be closed while a
+ *     batch that uses it is in flight. Handles are owned by the library.
+ *   - frame pixels are RGB8, HWC interleaved, `height` rows of 3*width bytes, rows `row_pitch` bytes apart.
+ *     When row_pitch and the pixel pointer are both multiples of 16 the kernels use 16-byte loads and may read
+ *     up to row_pitch bytes of every row (so the buffer must hold height*row_pitch bytes); otherwise a
+ *     byte-load path reads exactly 3*width bytes per row.
+ * The library has no CPU fallback: without a usable sm_100 device every compute call returns FFSVA_ECUDA.
+ */
+#ifndef FFSVA_H
+#define FFSVA_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#define FFSVA_API __attribute__((visibility("default")))
+#else
+#define FFSVA_API
+#endif
+
+typedef enum {
+  FFSVA_OK = 0,
+  FFSVA_EINVAL = -1,  /* bad argument or descriptor */
+  FFSVA_ENOMEM = -2,  /* device or pinned host allocation failed */
+  FFSVA_ECUDA = -3,   /* CUDA error (sticky per device) or no usable device */
+  FFSVA_ESTATE = -4,  /* a frame's stream has no reference image or no SNM loaded */
+  FFSVA_EAGAIN = -5,  /* online mode: the stream's SDD queue is over its feedback threshold (L209, L217) */
+  FFSVA_EDEVICE = -6  /* frames of one batch live on different devices */
+} ffsva_status;
+
+typedef struct ffsva_stream ffsva_stream; /* opaque, owned by the library */
+typedef struct ffsva_batch ffsva_batch;   /* opaque prepared batch, owned by the library */
+
+/* Per-stream configuration (SDD and SNM are specialised per stream; L183 thresholds per stream). */
+typedef struct {
+  int32_t device;          /* CUDA ordinal holding the stream's state and frames */
+  int32_t width, height;   /* raw frame size; sdd_w <= width <= 16384, sdd_h <= height <= 256*sdd_h */
+  int64_t row_pitch;       /* bytes between rows, >= 3*width */
+  int32_t sdd_w, sdd_h;    /* SDD grid, 100 x 100 (L155); even, 2 <= sdd <= 4096 */
+  int32_t snm_w, snm_h;    /* SNM grid, 50 x 50 (L167); must equal sdd/2 (the 50-grid cells are unions of
+                              2x2 100-grid cells, so one pass produces both resizes) */
+  double delta_diff;       /* MSE threshold (L151): pass iff SSD > floor(delta_diff * 3*sdd_w*sdd_h), i.e. iff
+                              MSE > delta_diff exactly; delta_diff >= 0 */
+  float c_low, c_high;     /* SNM class thresholds (L159), 0 <= c_low <= c_high <= 1 */
+  float filter_degree;     /* Eq. (2) (L193); must lie in [0, 1] ("cases t_pre < c_low, t_pre > c_high are not
+                              considered") */
+  int32_t snm_batch;       /* BatchSize (L219-L223), >= 1; default 30 */
+  int32_t q_sdd, q_snm;    /* feedback-queue depth thresholds in frames (L217), default 2 and 10 */
+} ffsva_stream_desc;
+
+/* SNM topology (L159: CONV, CONV, FC). The kernels implement c1 = 16, c2 = 32 on a 50x50 input. */
+typedef struct {
+  int32_t c1, c2;
+} ffsva_snm_desc;
+
+/* One input frame of a batch. `pixels` is a device pointer on the stream's device. */
+typedef struct {
+  ffsva_stream* stream;
+  const uint8_t* pixels;
+  int64_t frame_no;        /* caller's frame number (carried through, not interpreted) */
+} ffsva_frame;
+
+/* Per-frame result, in input order. */
+typedef struct {
+  uint64_t ssd;            /* sum over the 3*sdd_w*sdd_h values of (D100 - R)^2; MSE = ssd / (3*sdd_w*sdd_h) */
+  uint8_t sdd_pass;        /* 1 iff MSE > delta_diff (L151) */
+  uint8_t snm_pass;        /* 1 iff sdd_pass and c >= t_pre (L165) */
+  uint8_t snm_class;       /* 0: c < c_low, 1: unsure, 2: c > c_high (L159); 0 if !sdd_pass */
+  uint8_t pad;
+  float logit;             /* SNM output logit, c = 1/(1+exp(-logit)); NaN if !sdd_pass */
+  int32_t survivor_idx;    /* rank among this batch's SDD survivors in input order, -1 if !sdd_pass */
+} ffsva_result;
+
+/* Counters per stream slot, ffsva_stats_copy() layout: u64[slots][FFSVA_NSTAT]. */
+enum {
+  FFSVA_STAT_FRAMES = 0,   /* frames through SDD */
+  FFSVA_STAT_SDD_PASS = 1, /* SDD survivors */
+  FFSVA_STAT_SNM_PASS = 2, /* SNM survivors (c >= t_pre) */
+  FFSVA_STAT_SSD_SUM = 3,  /* sum of SSD over all frames */
+  FFSVA_STAT_CLASS0 = 4,   /* SNM class counts (L159) */
+  FFSVA_STAT_CLASS1 = 5,
+  FFSVA_STAT_CLASS2 = 6,
+  FFSVA_STAT_SNM_BATCHES = 7, /* SNM weight loads = dynamic batches executed (L219) */
+  FFSVA_NSTAT = 8
+};
+
+/* Create a stream (a camera) with its own SDD/SNM state on desc->device. The first stream of a device creates
+ * the device context (lazy); the last close destroys it. *out receives the handle. Errors: EINVAL (bad desc,
+ * out NULL), ECUDA, ENOMEM. */
+FFSVA_API ffsva_status ffsva_open_stream(const ffsva_stream_desc* desc, ffsva_stream** out);
+
+/* Build the stream's SDD reference image R ("average of dozens of background frames"): k >= 1
+ * background frames, frame j at frames + j*frame_stride (host or device memory; frame_stride >= height*pitch;
+ * each frame laid out like the stream's frames). R = round-half-up of the mean over all k*box samples of each
+ * 100-grid cell (one rounding). The input is copied; the caller may free it on return. Synchronous. */
+FFSVA_API ffsva_status ffsva_set_reference(ffsva_stream* s, const uint8_t* frames, int32_t k, int64_t frame_stride);
+
+/* Load the stream's SNM parameters (host fp32, packed w1[c1][3][3][3], b1[c1], w2[c2][c1][3][3], b2[c2],
+ * wfc[c2*12*12], bfc[1]; n_params = 27c1 + c1 + 9c1c2 + c2 + 144c2 + 1 = 9697 for 16/32). The weights w1, w2,
+ * wfc are rounded to bf16 (RNE) at load; biases stay fp32. Copied; synchronous. Errors: EINVAL (d not 16/32,
+ * n_params mismatch, NULL). */
+FFSVA_API ffsva_status ffsva_snm_load(ffsva_stream* s, const ffsva_snm_desc* d, const float* params,
+                                      int64_t n_params);
+
+/* Run the whole cascade on n frames and write n results (host memory, input order). Synchronous on
+ * cuda_stream (NULL = legacy default stream). Frames may come from any mix of open streams of ONE device and
+ * any mix of resolutions; survivors of one stream are scored in dynamic batches of at most snm_batch frames
+ * (L223). Errors: EINVAL, ESTATE, EDEVICE, ECUDA, ENOMEM. n = 0 is a no-op. */
+FFSVA_API ffsva_status ffsva_filter_batch(const ffsva_frame* frames, int32_t n, ffsva_result* results,
+                                          void* cuda_stream);
+
+/* Same cascade for frames held in HOST memory (`pixels` host pointers, pinned or pageable): the library stages
+ * them through a device ring with copies overlapped against the kernels. Synchronous. */
+FFSVA_API ffsva_status ffsva_filter_batch_host(const ffsva_frame* frames, int32_t n, ffsva_result* results,
+                                               void* cuda_stream);
+
+/* Prepared batches: upload the descriptors of n device frames once, then launch the cascade asynchronously
+ * any number of times (the kernel sequence is captured into a CUDA graph on the first launch and replayed),
+ * and fetch results when needed. The frames' bytes may change between launches; their addresses may not.
+ * ffsva_batch_launch enqueues on cuda_stream and returns immediately; ffsva_batch_fetch copies the results of
+ * the last launch to host (results may be NULL) and synchronises cuda_stream. */
+FFSVA_API ffsva_status ffsva_batch_prepare(const ffsva_frame* frames, int32_t n, ffsva_batch** out);
+FFSVA_API ffsva_status ffsva_batch_launch(ffsva_batch* b, void* cuda_stream);
+FFSVA_API ffsva_status ffsva_batch_fetch(ffsva_batch* b, ffsva_result* results, void* cuda_stream);
+/* Device views of a prepared batch's outputs (valid until destroy): ssd u64[n], sdd_pass u8[n], survivor_idx
+ * i32[n], logit f32[n], snm_pass u8[n], snm_class u8[n], d50 u8[n][snm_h][snm_w][3] (stride d50_stride bytes),
+ * survivor count i32[1]. Any pointer argument may be NULL. */
+FFSVA_API ffsva_status ffsva_batch_device_outputs(ffsva_batch* b, uint64_t** ssd, uint8_t** sdd_pass,
+                                                  int32_t** survivor_idx, float** logit, uint8_t** snm_pass,
+                                                  uint8_t** snm_class, uint8_t** d50, int64_t* d50_stride,
+                                                  int32_t** n_survivors);
+FFSVA_API ffsva_status ffsva_batch_destroy(ffsva_batch* b);
+
+/* Measurement hook: launch the cascade of each of the nb prepared batches in turn, iters times over the list,
+ * directly (no graph) with CUDA events recorded on cuda_stream around every kernel; ms_out[0..2] receive the
+ * mean device time per launch of K1 (ingest/downsample/SDD), K3 (compaction) and K4 (SNM). Synchronous. */
+FFSVA_API ffsva_status ffsva_batch_profile(ffsva_batch* const* batches, int32_t nb, int32_t iters,
+                                           float* ms_out, void* cuda_stream);
+
+/* SDD stage alone (for inspection and tests): D100 (sdd_h*sdd_w*3 u8 per frame, may be NULL), D50
+ * (snm_h*snm_w*3 per frame, may be NULL), SSD and pass per frame, written to HOST arrays in input order.
+ * Needs only a reference image (no SNM). Synchronous. */
+FFSVA_API ffsva_status ffsva_sdd_batch(const ffsva_frame* frames, int32_t n, uint8_t* d100, uint8_t* d50,
+                                       uint64_t* ssd, uint8_t* sdd_pass, void* cuda_stream);
+
+/* Copy the stream's reference image R (sdd_h*sdd_w*3 u8) to host memory. */
+FFSVA_API ffsva_status ffsva_get_reference(ffsva_stream* s, uint8_t* out);
+
+/* Stream slot id (index into the device's stats table) and device ordinal. */
+FFSVA_API ffsva_status ffsva_stream_info(ffsva_stream* s, int32_t* slot, int32_t* device);
+
+/* Per-stream statistics of `device` (a8): copy u64[slots][FFSVA_NSTAT] to dst (device memory on `device`, e.g.
+ * a torch tensor later all-gathered over NCCL, or host memory if dst_is_host). *slots receives the table size
+ * (max slot + 1); dst must hold max_slots*FFSVA_NSTAT values. reset != 0 zeroes the table afterwards. */
+FFSVA_API ffsva_status ffsva_stats_copy(int32_t device, uint64_t* dst, int32_t max_slots, int32_t* slots,
+                                        int32_t dst_is_host, int32_t reset, void* cuda_stream);
+
+/* Close a stream (NULL is a no-op). */
+FFSVA_API ffsva_status ffsva_close(ffsva_stream* s);
+
+/* Human-readable description of the calling thread's last error ("" if none). */
+FFSVA_API const char* ffsva_last_error(void);
+
+/* Number of kernels this process has launched through the library (all devices), for launch accounting. */
+FFSVA_API uint64_t ffsva_kernel_launches(void);
+
+/* Library version string. */
+FFSVA_API const char* ffsva_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* FFSVA_H */

@@ -1,0 +1,112 @@
+// ffsva_internal.h — shared declarations of the product library (kernels <-> host runtime).
+// Not part of the public ABI (include/ffsva.h is). Nothing here is shared with oracle/.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace ffsva {
+
+// ------------------------------------------------------------------ per-frame descriptor (device, 64 B)
+struct FrameDesc {
+  const uint8_t* pixels;   // raw RGB8 frame
+  const uint8_t* ref;      // stream's reference image R [sdd_h][sdd_w][3]
+  const uint8_t* snm;      // stream's packed SNM weight image (SnmLayout), nullptr for SDD-only batches
+  int64_t pitch;           // row pitch in bytes
+  uint64_t T;              // SDD threshold: pass iff SSD > T
+  int32_t W, H;            // raw size
+  float L_t;               // logit threshold for t_pre (Eq. (2)); pass iff logit >= L_t
+  float L_low, L_high;     // logit(c_low), logit(c_high) for the class (L159)
+  int32_t slot;            // stream slot (stats row)
+};
+static_assert(sizeof(FrameDesc) == 64, "FrameDesc must stay 64 B");
+
+// ------------------------------------------------------------------ SNM packed weight image (global + smem)
+// Exactly the shared-memory image the SNM kernel copies in once per stream change (dynamic batch, L219).
+// bf16 B operands are in the tcgen05 K-major no-swizzle canonical layout: [mma][khalf][n][8 k] (16 B rows).
+namespace snm {
+constexpr int C1 = 16, C2 = 32;
+constexpr int IN = 50, P1 = 25, P2 = 12;             // input, pooled conv1, pooled conv2 (floor)
+constexpr int NF = C2 * P2 * P2;                    // 4608 FC inputs
+constexpr int N_PARAMS = 27 * C1 + C1 + 9 * C1 * C2 + C2 + NF + 1;  // 9697
+constexpr int CONV1_MMAS = 5;                       // 9 taps x 8 channel slots paired into 5 K=16 MMAs
+constexpr int W1_BYTES = CONV1_MMAS * 2 * C1 * 16;  // 2560
+constexpr int W2_BYTES = 9 * 2 * C2 * 16;           // 9216
+constexpr int OFF_W1 = 0;
+constexpr int OFF_W2 = OFF_W1 + W1_BYTES;           // 2560
+constexpr int OFF_B1 = OFF_W2 + W2_BYTES;           // 11776 (fp32[16])
+constexpr int OFF_B2 = OFF_B1 + C1 * 4;             // 11840 (fp32[32])
+constexpr int OFF_BFC = OFF_B2 + C2 * 4;            // 11968 (fp32[1] + pad to 16)
+constexpr int OFF_WFC = OFF_BFC + 16;               // 11984 (fp32[4608], bf16-exact values)
+constexpr int BLOB_BYTES = OFF_WFC + NF * 4;        // 30416
+static_assert(BLOB_BYTES % 16 == 0, "blob must be 16-B granular");
+// conv1 MMA j pairs two taps (dy, dx) into the two K-halves of one K=16 MMA: {start tap, second tap, LBO}.
+// j = 4's first half is tap (2,1) again with zero weights (its second half carries tap (2,2)).
+}  // namespace snm
+
+// ------------------------------------------------------------------ launchers (defined in the .cu files)
+struct SddArgs {
+  const FrameDesc* frames;
+  int32_t n;
+  int32_t sdd_w, sdd_h;      // grid (uniform over the batch)
+  uint8_t* d50;              // [n][d50_stride]
+  int64_t d50_stride;
+  uint8_t* d100;             // optional [n][sdd_h*sdd_w*3]
+  uint32_t* partial;         // [n][sdd_h/2]
+  uint32_t* counter;         // [n], zero on entry, left zero
+  uint64_t* ssd;             // [n]
+  uint8_t* pass;             // [n]
+  unsigned long long* stats; // [slots][NSTAT] or nullptr
+  int32_t max_chunks;        // max over frames of ceil(3W/16)
+  bool vec16;                // all frames 16-B aligned with 16-B pitch
+};
+cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st);
+size_t sdd_smem_bytes(int max_chunks, int sdd_w);
+cudaError_t sdd_configure(size_t smem);  // raise the kernels' dynamic smem limit (outside graph capture)
+int sdd_threads(int max_chunks);
+
+struct CompactArgs {
+  const uint8_t* pass;       // [n] frame order
+  int32_t n;
+  const int32_t* perm;       // [n] work (stream-major, stable) order -> frame index
+  const int32_t* seg_lo;     // [n_seg + 1] segment boundaries in perm order (one segment per stream)
+  int32_t n_seg;
+  const int32_t* seg_batch;  // [n_seg] BatchSize of the segment's stream
+  int32_t* survivor_idx;     // [n] out
+  int32_t* work;             // [n] out: survivors in work order (frame indices)
+  int32_t* posw;             // [n + 1] scratch: exclusive survivor count in perm order
+  int32_t* chunks;           // [n + 1] out: chunk k = work[chunks[k] .. chunks[k+1]) (one stream, <= BatchSize)
+  int32_t* counts;           // [4] out: m, n_chunks, chunk cursor (reset 0), pad
+  float* logit;              // [n] initialised here: NaN / 0 / 0 (the SNM kernel overwrites survivors)
+  uint8_t* snm_pass;
+  uint8_t* snm_class;
+};
+cudaError_t launch_compact(const CompactArgs& a, cudaStream_t st);
+
+struct SnmArgs {
+  const FrameDesc* frames;
+  const uint8_t* d50;
+  int64_t d50_stride;
+  const int32_t* work;
+  const int32_t* chunks;
+  int32_t* counts;           // m, n_chunks, cursor
+  float* logit;              // [n] (frame order)
+  uint8_t* snm_pass;
+  uint8_t* snm_class;
+  unsigned long long* stats;
+  int32_t grid;
+  // debug taps (nullptr in production): pooled conv1 (bf16 as u16 [m][25][25][16]) and the pre-FC features
+  uint16_t* dbg_p1;
+  float* dbg_p2;             // [m][32][12][12]
+};
+cudaError_t launch_snm(const SnmArgs& a, cudaStream_t st);
+int snm_smem_bytes();
+cudaError_t snm_configure();
+
+cudaError_t launch_fill_nan(float* p, int32_t n, cudaStream_t st);
+cudaError_t launch_reference(const uint8_t* frames, int32_t k, int64_t frame_stride, int32_t W, int32_t H,
+                             int64_t pitch, int32_t sdd_w, int32_t sdd_h, uint8_t* out, cudaStream_t st);
+
+constexpr int NSTAT = 8;
+
+}  // namespace ffsva

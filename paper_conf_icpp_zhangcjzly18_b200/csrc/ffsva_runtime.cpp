@@ -1,0 +1,508 @@
+// ffsva_runtime.cpp — host runtime: device contexts, pointer validation, SNM weight packing, prepared
+// batches (descriptor upload, stream-major work order, CUDA-graph capture of K1 -> K3 -> K4).
+#include "ffsva_runtime.h"
+
+#include <cuda.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+
+namespace ffsva {
+
+std::atomic<uint64_t> g_launches{0};
+static thread_local std::string t_err;
+static std::mutex g_mu;
+static DeviceCtx* g_ctx[64] = {nullptr};
+constexpr int32_t kMaxSlots = 65536;  // stats table rows per device (fixed so graphs never see a realloc)
+
+void set_error(const std::string& msg) { t_err = msg; }
+const char* last_error() { return t_err.c_str(); }
+
+ffsva_status fail(ffsva_status st, const std::string& msg) {
+  t_err = msg;
+  return st;
+}
+
+ffsva_status cuda_fail(DeviceCtx* ctx, cudaError_t e, const char* what) {
+  if (ctx) ctx->sticky = true;
+  t_err = std::string(what) + ": " + cudaGetErrorString(e);
+  return e == cudaErrorMemoryAllocation ? FFSVA_ENOMEM : FFSVA_ECUDA;
+}
+
+#define FF_CUDA(ctx, call)                                  \
+  do {                                                      \
+    cudaError_t _e = (call);                                \
+    if (_e != cudaSuccess) return cuda_fail(ctx, _e, #call); \
+  } while (0)
+
+// ------------------------------------------------------------------ device contexts
+DeviceCtx* ctx_acquire(int device, ffsva_status* st) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  *st = FFSVA_OK;
+  if (device < 0 || device >= 64) {
+    *st = fail(FFSVA_EINVAL, "device ordinal out of range");
+    return nullptr;
+  }
+  int count = 0;
+  cudaError_t e = cudaGetDeviceCount(&count);
+  if (e != cudaSuccess || count == 0) {
+    *st = fail(FFSVA_ECUDA, std::string("no CUDA device: ") + cudaGetErrorString(e));
+    return nullptr;
+  }
+  if (device >= count) {
+    *st = fail(FFSVA_EINVAL, "device ordinal >= device count");
+    return nullptr;
+  }
+  DeviceCtx* c = g_ctx[device];
+  if (!c) {
+    DeviceGuard g(device);
+    cudaDeviceProp prop;
+    if ((e = cudaGetDeviceProperties(&prop, device)) != cudaSuccess) {
+      *st = fail(FFSVA_ECUDA, cudaGetErrorString(e));
+      return nullptr;
+    }
+    if (prop.major != 10) {
+      *st = fail(FFSVA_ECUDA, "the kernels are built for sm_100a (B200); device is sm_" +
+                                  std::to_string(prop.major) + std::to_string(prop.minor));
+      return nullptr;
+    }
+    c = new DeviceCtx();
+    c->device = device;
+    c->num_sms = prop.multiProcessorCount;
+    c->stats_cap = kMaxSlots;
+    if ((e = cudaMalloc(&c->d_stats, sizeof(unsigned long long) * NSTAT * kMaxSlots)) != cudaSuccess ||
+        (e = cudaMemset(c->d_stats, 0, sizeof(unsigned long long) * NSTAT * kMaxSlots)) != cudaSuccess ||
+        (e = cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking)) != cudaSuccess ||
+        (e = snm_configure()) != cudaSuccess) {
+      *st = cuda_fail(nullptr, e, "device context init");
+      delete c;
+      return nullptr;
+    }
+    g_ctx[device] = c;
+  }
+  c->nstreams++;
+  return c;
+}
+
+void ctx_release(DeviceCtx* c) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  if (--c->nstreams > 0) return;
+  DeviceGuard g(c->device);
+  cudaDeviceSynchronize();
+  if (c->scratch) {
+    batch_free(c->scratch);
+    delete c->scratch;
+  }
+  cudaFree(c->d_stats);
+  cudaFree(c->d_ring);
+  cudaStreamDestroy(c->copy_stream);
+  g_ctx[c->device] = nullptr;
+  delete c;
+}
+
+// A device pointer must lie inside a device allocation of the context's device. Allocation ranges are cached
+// so a batch of frames from one pool costs one driver query.
+ffsva_status check_device_ptr(DeviceCtx* ctx, const void* p, size_t bytes) {
+  if (!p) return fail(FFSVA_EINVAL, "NULL frame pointer");
+  const uintptr_t a = (uintptr_t)p;
+  for (auto& r : ctx->ranges)
+    if (a >= r.first && a + bytes <= r.first + r.second) return FFSVA_OK;
+  cudaPointerAttributes attr;
+  cudaError_t e = cudaPointerGetAttributes(&attr, p);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(FFSVA_EINVAL, "pixels is not a CUDA pointer");
+  }
+  if (attr.type != cudaMemoryTypeDevice && attr.type != cudaMemoryTypeManaged)
+    return fail(FFSVA_EINVAL, "pixels must be device memory (use ffsva_filter_batch_host for host frames)");
+  if (attr.device != ctx->device) return fail(FFSVA_EDEVICE, "frame pixels live on another device");
+  // driver entry point fetched through the runtime, so the library does not link libcuda (it must load on
+  // GPU-less hosts, where every compute call then reports FFSVA_ECUDA)
+  using GetRange = CUresult (*)(CUdeviceptr*, size_t*, CUdeviceptr);
+  static GetRange get_range = [] {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) != cudaSuccess) fn = nullptr;
+    return (GetRange)fn;
+  }();
+  CUdeviceptr base = 0;
+  size_t size = 0;
+  if (get_range && get_range(&base, &size, (CUdeviceptr)a) == CUDA_SUCCESS) {
+    if (a + bytes > (uintptr_t)base + size) return fail(FFSVA_EINVAL, "frame extends past its allocation");
+    if (ctx->ranges.size() >= 64) ctx->ranges.erase(ctx->ranges.begin());
+    ctx->ranges.emplace_back((uintptr_t)base, size);
+  }
+  return FFSVA_OK;
+}
+
+// ------------------------------------------------------------------ host arithmetic
+// floor(delta * n) with the product taken exactly: delta = mant * 2^e2 (IEEE-754 fields).
+uint64_t exact_threshold(double delta, uint64_t n) {
+  uint64_t bits;
+  std::memcpy(&bits, &delta, 8);
+  const int expf = (int)((bits >> 52) & 0x7FF);
+  const uint64_t frac = bits & ((1ull << 52) - 1);
+  if ((bits >> 63) || (expf == 0 && frac == 0)) return 0;
+  const uint64_t mant = expf ? (frac | (1ull << 52)) : frac;
+  const int e2 = expf ? expf - 1075 : -1074;
+  const unsigned __int128 prod = (unsigned __int128)mant * n;
+  if (e2 >= 0) {
+    if (e2 >= 64) return UINT64_MAX;
+    const unsigned __int128 v = prod << e2;
+    if ((v >> e2) != prod || (v >> 64) != 0) return UINT64_MAX;
+    return (uint64_t)v;
+  }
+  if (-e2 >= 128) return 0;
+  const unsigned __int128 v = prod >> (-e2);
+  return (v >> 64) ? UINT64_MAX : (uint64_t)v;
+}
+
+uint16_t bf16_bits_rne(float x) {
+  uint32_t u;
+  std::memcpy(&u, &x, 4);
+  if ((u & 0x7F800000u) == 0x7F800000u && (u & 0x007FFFFFu)) return 0x7FC0;  // NaN
+  return (uint16_t)((u + 0x7FFFu + ((u >> 16) & 1u)) >> 16);
+}
+
+static float bf16_value(float x) {
+  uint32_t u = (uint32_t)bf16_bits_rne(x) << 16;
+  float f;
+  std::memcpy(&f, &u, 4);
+  return f;
+}
+
+float logit_of(double t) {
+  if (t <= 0.0) return -INFINITY;
+  if (t >= 1.0) return INFINITY;
+  return (float)std::log(t / (1.0 - t));
+}
+
+// SNM weight image (see ffsva_internal.h snm::*). params = w1[16][3][3][3], b1[16], w2[32][16][3][3], b2[32],
+// wfc[4608], bfc.
+void pack_snm_blob(const float* params, uint8_t* blob) {
+  using namespace snm;
+  std::memset(blob, 0, BLOB_BYTES);
+  const float* w1 = params;
+  const float* b1 = w1 + 27 * C1;
+  const float* w2 = b1 + C1;
+  const float* b2 = w2 + 9 * C1 * C2;
+  const float* wfc = b2 + C2;
+  const float* bfc = wfc + NF;
+  // conv1: MMA j, K-half h carries tap (dy, dx) (channels 0..2 of the 8 slots); -1 = zero half
+  static const int tap_dy[5][2] = {{0, 0}, {1, 1}, {2, 2}, {0, 1}, {-1, 2}};
+  static const int tap_dx[5][2] = {{0, 1}, {0, 1}, {0, 1}, {2, 2}, {-1, 2}};
+  uint16_t* W1 = reinterpret_cast<uint16_t*>(blob + OFF_W1);
+  for (int j = 0; j < CONV1_MMAS; ++j)
+    for (int h = 0; h < 2; ++h) {
+      const int dy = tap_dy[j][h], dx = tap_dx[j][h];
+      if (dy < 0) continue;
+      for (int n = 0; n < C1; ++n)
+        for (int c = 0; c < 3; ++c)
+          W1[((j * 2 + h) * C1 + n) * 8 + c] = bf16_bits_rne(w1[((n * 3 + c) * 3 + dy) * 3 + dx]);
+    }
+  // conv2: tap t, K-half h = input channels 8h..8h+7
+  uint16_t* W2 = reinterpret_cast<uint16_t*>(blob + OFF_W2);
+  for (int t = 0; t < 9; ++t)
+    for (int h = 0; h < 2; ++h)
+      for (int n = 0; n < C2; ++n)
+        for (int c = 0; c < 8; ++c)
+          W2[((t * 2 + h) * C2 + n) * 8 + c] = bf16_bits_rne(w2[((n * C1 + 8 * h + c) * 3 + t / 3) * 3 + t % 3]);
+  std::memcpy(blob + OFF_B1, b1, C1 * 4);
+  std::memcpy(blob + OFF_B2, b2, C2 * 4);
+  std::memcpy(blob + OFF_BFC, bfc, 4);
+  float* F = reinterpret_cast<float*>(blob + OFF_WFC);
+  for (int i = 0; i < NF; ++i) F[i] = bf16_value(wfc[i]);
+}
+
+// ------------------------------------------------------------------ batches
+static size_t al(size_t x) { return (x + 255) & ~(size_t)255; }
+
+void batch_free(Batch* b) {
+  if (b->graph) cudaGraphExecDestroy(b->graph);
+  b->graph = nullptr;
+  cudaFree(b->d_mem);
+  cudaFreeHost(b->h_in);
+  cudaFreeHost(b->h_out);
+  b->d_mem = nullptr;
+  b->h_in = b->h_out = nullptr;
+  b->cap = 0;
+}
+
+static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t sdd_w, int32_t sdd_h, bool d100) {
+  batch_free(b);
+  const size_t n = (size_t)cap;
+  b->d50_stride = (int64_t)((3 * (sdd_w / 2) * (sdd_h / 2) + 15) & ~15);
+  // input block (mirrors h_in)
+  size_t off = 0;
+  const size_t o_desc = off; off += al(64 * n);
+  const size_t o_perm = off; off += al(4 * n);
+  const size_t o_seg = off; off += al(4 * (n + 1));
+  const size_t o_segb = off; off += al(4 * n);
+  b->in_bytes = off;
+  const size_t o_d50 = off; off += al((size_t)b->d50_stride * n);
+  const size_t o_d100 = off; off += d100 ? al((size_t)3 * sdd_w * sdd_h * n) : 0;
+  const size_t o_part = off; off += al(4 * n * (size_t)(sdd_h / 2));
+  const size_t o_cnt = off; off += al(4 * n);
+  const size_t o_work = off; off += al(4 * n);
+  const size_t o_posw = off; off += al(4 * (n + 1));
+  const size_t o_chunks = off; off += al(4 * (n + 1));
+  const size_t o_counts = off; off += al(16);
+  const size_t o_out = off;
+  const size_t out_bytes = 8 * n + 4 * n + 4 * n + 3 * n;
+  off += al(out_bytes);
+  b->d_bytes = off;
+  cudaError_t e = cudaMalloc(&b->d_mem, off);
+  if (e != cudaSuccess) return cuda_fail(nullptr, e, "cudaMalloc(batch)");
+  uint8_t* base = (uint8_t*)b->d_mem;
+  b->d_desc = (FrameDesc*)(base + o_desc);
+  b->d_perm = (int32_t*)(base + o_perm);
+  b->d_seg_lo = (int32_t*)(base + o_seg);
+  b->d_seg_batch = (int32_t*)(base + o_segb);
+  b->d_d50 = base + o_d50;
+  b->d_d100 = d100 ? base + o_d100 : nullptr;
+  b->d_partial = (uint32_t*)(base + o_part);
+  b->d_counter = (uint32_t*)(base + o_cnt);
+  b->d_work = (int32_t*)(base + o_work);
+  b->d_posw = (int32_t*)(base + o_posw);
+  b->d_chunks = (int32_t*)(base + o_chunks);
+  b->d_counts = (int32_t*)(base + o_counts);
+  b->d_out = base + o_out;
+  b->d_ssd = (uint64_t*)(b->d_out);
+  b->d_logit = (float*)(b->d_out + 8 * n);
+  b->d_surv = (int32_t*)(b->d_out + 12 * n);
+  b->d_pass = b->d_out + 16 * n;
+  b->d_snm_pass = b->d_out + 17 * n;
+  b->d_snm_class = b->d_out + 18 * n;
+  b->out_bytes = out_bytes;
+  if ((e = cudaMemset(b->d_counter, 0, 4 * n)) != cudaSuccess) return cuda_fail(ctx, e, "cudaMemset(counter)");
+  if ((e = cudaMemset(b->d_counts, 0, 16)) != cudaSuccess) return cuda_fail(ctx, e, "cudaMemset(counts)");
+  if ((e = cudaMallocHost(&b->h_in, b->in_bytes)) != cudaSuccess) return cuda_fail(nullptr, e, "cudaMallocHost");
+  if ((e = cudaMallocHost(&b->h_out, out_bytes)) != cudaSuccess) return cuda_fail(nullptr, e, "cudaMallocHost");
+  b->cap = cap;
+  b->sdd_w = sdd_w;
+  b->sdd_h = sdd_h;
+  b->want_d100 = d100;
+  b->ctx = ctx;
+  return FFSVA_OK;
+}
+
+ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, int32_t n, bool sdd_only,
+                         bool want_d100, cudaStream_t st) {
+  const StreamState* s0 = frames[0].stream;
+  const int32_t sdd_w = s0->desc.sdd_w, sdd_h = s0->desc.sdd_h;
+  bool vec16 = true;
+  int32_t max_chunks = 1;
+  for (int32_t i = 0; i < n; ++i) {
+    const StreamState* s = frames[i].stream;
+    if (s->desc.sdd_w != sdd_w || s->desc.sdd_h != sdd_h)
+      return fail(FFSVA_EINVAL, "all frames of a batch must share the SDD grid");
+    const int64_t bytes = (int64_t)(s->desc.height - 1) * s->desc.row_pitch + 3 * s->desc.width;
+    ffsva_status cs = check_device_ptr(ctx, frames[i].pixels, (size_t)bytes);
+    if (cs != FFSVA_OK) return cs;
+    if ((s->desc.row_pitch & 15) || ((uintptr_t)frames[i].pixels & 15)) vec16 = false;
+    max_chunks = std::max(max_chunks, (3 * s->desc.width + 15) / 16);
+  }
+  if (b->cap < n || b->sdd_w != sdd_w || b->sdd_h != sdd_h || (want_d100 && !b->want_d100)) {
+    ffsva_status as = batch_alloc(ctx, b, std::max(n, b->cap), sdd_w, sdd_h, want_d100 || b->want_d100);
+    if (as != FFSVA_OK) return as;
+  }
+  if (b->graph) {
+    cudaGraphExecDestroy(b->graph);
+    b->graph = nullptr;
+  }
+  cudaError_t e = sdd_configure(sdd_smem_bytes(max_chunks, sdd_w));
+  if (e != cudaSuccess) return cuda_fail(ctx, e, "sdd_configure");
+  b->n = n;
+  b->vec16 = vec16;
+  b->max_chunks = max_chunks;
+  b->sdd_only = sdd_only;
+  // ---- host staging: descriptors, stream-major permutation, segments
+  const size_t cap = (size_t)b->cap;
+  FrameDesc* hd = (FrameDesc*)b->h_in;
+  int32_t* hperm = (int32_t*)(b->h_in + al(64 * cap));
+  int32_t* hseg = (int32_t*)(b->h_in + al(64 * cap) + al(4 * cap));
+  int32_t* hsegb = (int32_t*)(b->h_in + al(64 * cap) + al(4 * cap) + al(4 * (cap + 1)));
+  bool sorted = true;
+  for (int32_t i = 0; i < n; ++i) {
+    const StreamState* s = frames[i].stream;
+    FrameDesc& d = hd[i];
+    d.pixels = frames[i].pixels;
+    d.ref = s->d_ref;
+    d.snm = s->d_snm;
+    d.pitch = s->desc.row_pitch;
+    d.T = s->T;
+    d.W = s->desc.width;
+    d.H = s->desc.height;
+    d.L_t = s->L_t;
+    d.L_low = s->L_low;
+    d.L_high = s->L_high;
+    d.slot = s->slot;
+    hperm[i] = i;
+    if (i && s->slot < frames[i - 1].stream->slot) sorted = false;
+  }
+  if (!sorted)
+    std::stable_sort(hperm, hperm + n, [&](int32_t x, int32_t y) { return hd[x].slot < hd[y].slot; });
+  int32_t nseg = 0;
+  for (int32_t k = 0; k < n; ++k)
+    if (k == 0 || hd[hperm[k]].slot != hd[hperm[k - 1]].slot) {
+      hseg[nseg] = k;
+      hsegb[nseg] = frames[hperm[k]].stream->desc.snm_batch;
+      ++nseg;
+    }
+  hseg[nseg] = n;
+  b->n_seg = nseg;
+  e = cudaMemcpyAsync(b->d_mem, b->h_in, b->in_bytes, cudaMemcpyHostToDevice, st);
+  if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaMemcpyAsync(descriptors)");
+  // the staging buffer is reused by the next build: make sure this copy has consumed it
+  e = cudaStreamSynchronize(st);
+  if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaStreamSynchronize(descriptors)");
+  return FFSVA_OK;
+}
+
+static ffsva_status batch_launch_kernels(Batch* b, cudaStream_t st, int* nk, cudaEvent_t* ev = nullptr) {
+  DeviceCtx* ctx = b->ctx;
+  SddArgs sa{};
+  sa.frames = b->d_desc;
+  sa.n = b->n;
+  sa.sdd_w = b->sdd_w;
+  sa.sdd_h = b->sdd_h;
+  sa.d50 = b->d_d50;
+  sa.d50_stride = b->d50_stride;
+  sa.d100 = b->want_d100 ? b->d_d100 : nullptr;
+  sa.partial = b->d_partial;
+  sa.counter = b->d_counter;
+  sa.ssd = b->d_ssd;
+  sa.pass = b->d_pass;
+  sa.stats = ctx->d_stats;
+  sa.max_chunks = b->max_chunks;
+  sa.vec16 = b->vec16;
+  if (ev) cudaEventRecord(ev[0], st);
+  FF_CUDA(ctx, launch_sdd(sa, st));
+  if (ev) cudaEventRecord(ev[1], st);
+  CompactArgs ca{};
+  ca.pass = b->d_pass;
+  ca.n = b->n;
+  ca.perm = b->d_perm;
+  ca.seg_lo = b->d_seg_lo;
+  ca.n_seg = b->n_seg;
+  ca.seg_batch = b->d_seg_batch;
+  ca.survivor_idx = b->d_surv;
+  ca.work = b->d_work;
+  ca.posw = b->d_posw;
+  ca.chunks = b->d_chunks;
+  ca.counts = b->d_counts;
+  ca.logit = b->d_logit;
+  ca.snm_pass = b->d_snm_pass;
+  ca.snm_class = b->d_snm_class;
+  FF_CUDA(ctx, launch_compact(ca, st));
+  if (ev) cudaEventRecord(ev[2], st);
+  *nk = 2;
+  if (!b->sdd_only) {
+    SnmArgs na{};
+    na.frames = b->d_desc;
+    na.d50 = b->d_d50;
+    na.d50_stride = b->d50_stride;
+    na.work = b->d_work;
+    na.chunks = b->d_chunks;
+    na.counts = b->d_counts;
+    na.logit = b->d_logit;
+    na.snm_pass = b->d_snm_pass;
+    na.snm_class = b->d_snm_class;
+    na.stats = ctx->d_stats;
+    na.grid = std::max(1, std::min(b->n, 2 * ctx->num_sms));
+    FF_CUDA(ctx, launch_snm(na, st));
+    *nk = 3;
+  }
+  if (ev) cudaEventRecord(ev[3], st);
+  return FFSVA_OK;
+}
+
+ffsva_status batch_profile(Batch* const* batches, int32_t nb, int32_t iters, float* ms_out, cudaStream_t st) {
+  DeviceCtx* ctx = batches[0]->ctx;
+  cudaEvent_t ev[4];
+  for (auto& e : ev) FF_CUDA(ctx, cudaEventCreate(&e));
+  double acc[3] = {0, 0, 0};
+  int count = 0;
+  ffsva_status s = FFSVA_OK;
+  for (int it = 0; it < iters && s == FFSVA_OK; ++it)
+    for (int32_t j = 0; j < nb && s == FFSVA_OK; ++j) {
+      int nk = 0;
+      s = batch_launch_kernels(batches[j], st, &nk, ev);
+      g_launches += nk;
+      if (s != FFSVA_OK) break;
+      cudaError_t e = cudaEventSynchronize(ev[3]);
+      if (e != cudaSuccess) {
+        s = cuda_fail(ctx, e, "cudaEventSynchronize(profile)");
+        break;
+      }
+      float t[3];
+      cudaEventElapsedTime(&t[0], ev[0], ev[1]);
+      cudaEventElapsedTime(&t[1], ev[1], ev[2]);
+      cudaEventElapsedTime(&t[2], ev[2], ev[3]);
+      for (int k = 0; k < 3; ++k) acc[k] += t[k];
+      ++count;
+    }
+  for (auto& e : ev) cudaEventDestroy(e);
+  if (s != FFSVA_OK) return s;
+  for (int k = 0; k < 3; ++k) ms_out[k] = count ? (float)(acc[k] / count) : 0.f;
+  return FFSVA_OK;
+}
+
+ffsva_status batch_run(Batch* b, cudaStream_t st, bool use_graph) {
+  DeviceCtx* ctx = b->ctx;
+  if (b->n == 0) return FFSVA_OK;
+  if (!use_graph || st == nullptr) {
+    int nk = 0;
+    ffsva_status s = batch_launch_kernels(b, st, &nk);
+    g_launches += nk;
+    return s;
+  }
+  if (!b->graph) {
+    cudaGraph_t g = nullptr;
+    FF_CUDA(ctx, cudaStreamBeginCapture(st, cudaStreamCaptureModeThreadLocal));
+    int nk = 0;
+    ffsva_status s = batch_launch_kernels(b, st, &nk);
+    cudaError_t e = cudaStreamEndCapture(st, &g);
+    if (s != FFSVA_OK) return s;
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaStreamEndCapture");
+    e = cudaGraphInstantiate(&b->graph, g, 0);
+    cudaGraphDestroy(g);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaGraphInstantiate");
+    b->graph_kernels = nk;
+  }
+  FF_CUDA(ctx, cudaGraphLaunch(b->graph, st));
+  g_launches += b->graph_kernels;
+  return FFSVA_OK;
+}
+
+ffsva_status batch_fetch(Batch* b, ffsva_result* results, cudaStream_t st) {
+  DeviceCtx* ctx = b->ctx;
+  const int32_t n = b->n;
+  if (n == 0) return FFSVA_OK;
+  if (results) {
+    FF_CUDA(ctx, cudaMemcpyAsync(b->h_out, b->d_out, b->out_bytes, cudaMemcpyDeviceToHost, st));
+  }
+  FF_CUDA(ctx, cudaStreamSynchronize(st));
+  if (!results) return FFSVA_OK;
+  const size_t cap = (size_t)b->cap;
+  const uint64_t* ssd = (const uint64_t*)b->h_out;
+  const float* lg = (const float*)(b->h_out + 8 * cap);
+  const int32_t* sv = (const int32_t*)(b->h_out + 12 * cap);
+  const uint8_t* ps = b->h_out + 16 * cap;
+  const uint8_t* sp = b->h_out + 17 * cap;
+  const uint8_t* sc = b->h_out + 18 * cap;
+  for (int32_t i = 0; i < n; ++i) {
+    ffsva_result& r = results[i];
+    r.ssd = ssd[i];
+    r.sdd_pass = ps[i];
+    r.snm_pass = sp[i];
+    r.snm_class = sc[i];
+    r.pad = 0;
+    r.logit = lg[i];
+    r.survivor_idx = sv[i];
+  }
+  return FFSVA_OK;
+}
+
+}  // namespace ffsva

@@ -1,0 +1,123 @@
+// ffsva_runtime.h — host runtime of the product library (internal).
+#pragma once
+
+#include <atomic>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "ffsva.h"
+#include "ffsva_internal.h"
+
+namespace ffsva {
+
+struct DeviceCtx;
+
+// Error reporting: every public entry point funnels through these.
+void set_error(const std::string& msg);
+ffsva_status fail(ffsva_status st, const std::string& msg);
+ffsva_status cuda_fail(DeviceCtx* ctx, cudaError_t e, const char* what);
+extern std::atomic<uint64_t> g_launches;
+
+// One camera stream (SDD and SNM are specialised per stream).
+struct StreamState {
+  ffsva_stream_desc desc{};
+  DeviceCtx* ctx = nullptr;
+  int32_t slot = -1;
+  uint8_t* d_ref = nullptr;   // R [sdd_h][sdd_w][3]
+  uint8_t* d_snm = nullptr;   // packed SNM weight image (snm::BLOB_BYTES)
+  bool has_ref = false, has_snm = false;
+  uint64_t T = 0;             // SDD threshold on SSD
+  float L_t = 0.f, L_low = 0.f, L_high = 0.f;
+};
+
+// A prepared batch: device descriptors + all per-batch device buffers; owns a CUDA graph of its kernels.
+struct Batch {
+  DeviceCtx* ctx = nullptr;
+  int32_t n = 0, cap = 0;
+  int32_t sdd_w = 0, sdd_h = 0, max_chunks = 0, n_seg = 0;
+  bool vec16 = true, sdd_only = false, want_d100 = false;
+  int64_t d50_stride = 0;
+  // device buffers (carved from one allocation)
+  void* d_mem = nullptr;
+  size_t d_bytes = 0;
+  FrameDesc* d_desc = nullptr;
+  int32_t *d_perm = nullptr, *d_seg_lo = nullptr, *d_seg_batch = nullptr;
+  uint8_t* d_d50 = nullptr;
+  uint8_t* d_d100 = nullptr;
+  uint32_t *d_partial = nullptr, *d_counter = nullptr;
+  int32_t *d_work = nullptr, *d_posw = nullptr, *d_chunks = nullptr, *d_counts = nullptr;
+  // output block (one D2H): ssd u64[n] | logit f32[n] | survivor_idx i32[n] | sdd_pass u8[n] | snm_pass u8[n] |
+  // snm_class u8[n]
+  uint8_t* d_out = nullptr;
+  uint64_t* d_ssd = nullptr;
+  float* d_logit = nullptr;
+  int32_t* d_surv = nullptr;
+  uint8_t *d_pass = nullptr, *d_snm_pass = nullptr, *d_snm_class = nullptr;
+  size_t out_bytes = 0;
+  // host pinned staging: inputs (desc|perm|seg_lo|seg_batch) and outputs
+  uint8_t* h_in = nullptr;
+  size_t in_bytes = 0;
+  uint8_t* h_out = nullptr;
+  // graph
+  cudaGraphExec_t graph = nullptr;
+  int graph_kernels = 0;
+};
+
+struct DeviceCtx {
+  int device = 0;
+  std::mutex mu;
+  int num_sms = 148;
+  int nstreams = 0;
+  std::vector<int32_t> free_slots;
+  int32_t next_slot = 0;
+  unsigned long long* d_stats = nullptr;  // [stats_cap][NSTAT]
+  int32_t stats_cap = 0;
+  bool sticky = false;
+  Batch* scratch = nullptr;  // reusable batch for ffsva_filter_batch / ffsva_sdd_batch
+  // staging ring for host-resident frames (ffsva_filter_batch_host)
+  uint8_t* d_ring = nullptr;
+  size_t ring_bytes = 0;
+  cudaStream_t copy_stream = nullptr;
+  // known device allocations [base, base + size) on this device (pointer validation cache)
+  std::vector<std::pair<uintptr_t, size_t>> ranges;
+};
+
+// device context registry
+DeviceCtx* ctx_acquire(int device, ffsva_status* st);  // creates lazily, increments nstreams
+void ctx_release(DeviceCtx* ctx);                       // decrements; destroys at 0
+
+// helpers
+ffsva_status check_device_ptr(DeviceCtx* ctx, const void* p, size_t bytes);
+ffsva_status ensure_stats(DeviceCtx* ctx, int32_t slots);
+uint64_t exact_threshold(double delta, uint64_t n_values);
+uint16_t bf16_bits_rne(float x);
+void pack_snm_blob(const float* params, uint8_t* blob);
+float logit_of(double t);
+
+// batches
+ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, int32_t n, bool sdd_only,
+                         bool want_d100, cudaStream_t st);
+ffsva_status batch_run(Batch* b, cudaStream_t st, bool use_graph);
+ffsva_status batch_fetch(Batch* b, ffsva_result* results, cudaStream_t st);
+ffsva_status batch_profile(Batch* const* batches, int32_t nb, int32_t iters, float* ms_out, cudaStream_t st);
+void batch_free(Batch* b);
+
+// RAII device switch
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+}  // namespace ffsva
+
+struct ffsva_stream : ffsva::StreamState {};
+struct ffsva_batch : ffsva::Batch {};

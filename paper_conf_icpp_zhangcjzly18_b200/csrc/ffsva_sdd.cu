@@ -1,0 +1,241 @@
+// ffsva_sdd.cu — K1: frame ingest + integer box downsample (D100 and D50 in one pass) + SDD distance and
+// threshold, for many frames of many streams in one launch.
+//
+// Method: raw frames are resized to each filter's feature size before the filter runs (L187;
+// SDD 100x100 L155, SNM 50x50 L167); SDD computes the distance of the 100x100 image to the stream's
+// reference image by MSE and keeps the frame iff MSE > delta_diff (L151). Readings: integer
+// box filter with round-half-up (Q1, Q2), RGB kept (Q3), SSD in integers with an exact threshold (Q4, Q5),
+// D50 from the raw frame = union of 2x2 D100 cells (Q8).
+//
+// B200 mapping. One CTA per (frame, 50-grid row band) = two 100-grid rows of source pixels. The band is a set
+// of whole source rows, streamed once from HBM with coalesced 16-byte non-allocating loads (each warp load
+// covers 512 contiguous bytes of a row); up to 8 rows are in flight per thread before any arithmetic.
+// Column sums are kept as packed 2x16-bit SIMD lanes in registers (1.25 integer ops per byte), written once
+// to shared memory, then summed per cell. Each CTA emits 2 rows of D100 cells (SSD against R from L2), one
+// row of D50, and a partial SSD; the last CTA of a frame (ticket counter, self-resetting) adds the partials
+// in u64, applies the threshold and updates the per-stream stats. HBM traffic = the raw frame bytes once +
+// 7.5 KB of D50 (+ 30 KB of D100 when requested) per frame.
+#include "ffsva_internal.h"
+
+namespace ffsva {
+namespace {
+
+__device__ __forceinline__ uint4 ld_stream16(const uint8_t* p) {
+  uint4 r;
+  asm("ld.global.nc.L1::no_allocate.v4.u32 {%0, %1, %2, %3}, [%4];"
+      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+      : "l"(p));
+  return r;
+}
+
+// Bytes 0..15 of a 16-byte chunk -> 8 accumulators of two 16-bit lanes:
+// a[2k] holds bytes (4k, 4k+2), a[2k+1] holds bytes (4k+1, 4k+3).
+__device__ __forceinline__ void acc16(uint32_t (&a)[8], const uint4& v) {
+  a[0] += v.x & 0x00FF00FFu; a[1] += (v.x >> 8) & 0x00FF00FFu;
+  a[2] += v.y & 0x00FF00FFu; a[3] += (v.y >> 8) & 0x00FF00FFu;
+  a[4] += v.z & 0x00FF00FFu; a[5] += (v.z >> 8) & 0x00FF00FFu;
+  a[6] += v.w & 0x00FF00FFu; a[7] += (v.w >> 8) & 0x00FF00FFu;
+}
+
+__device__ __forceinline__ uint4 load_chunk(const uint8_t* row, int c, int rowbytes, bool vec16) {
+  if (vec16) return ld_stream16(row + 16 * c);
+  uint32_t w[4] = {0u, 0u, 0u, 0u};
+#pragma unroll
+  for (int j = 0; j < 16; ++j) {
+    int b = 16 * c + j;
+    uint32_t v = b < rowbytes ? (uint32_t)__ldg(row + b) : 0u;
+    w[j >> 2] |= v << (8 * (j & 3));
+  }
+  return make_uint4(w[0], w[1], w[2], w[3]);
+}
+
+// Store the 16 column sums of chunk c (u16 each) for one 100-grid row.
+__device__ __forceinline__ void store_colsum(uint32_t* colw, int c, const uint32_t (&a)[8]) {
+  uint4 lo, hi;
+  lo.x = __byte_perm(a[0], a[1], 0x5410); lo.y = __byte_perm(a[0], a[1], 0x7632);
+  lo.z = __byte_perm(a[2], a[3], 0x5410); lo.w = __byte_perm(a[2], a[3], 0x7632);
+  hi.x = __byte_perm(a[4], a[5], 0x5410); hi.y = __byte_perm(a[4], a[5], 0x7632);
+  hi.z = __byte_perm(a[6], a[7], 0x5410); hi.w = __byte_perm(a[6], a[7], 0x7632);
+  reinterpret_cast<uint4*>(colw)[2 * c] = lo;
+  reinterpret_cast<uint4*>(colw)[2 * c + 1] = hi;
+}
+
+template <bool kD100>
+__global__ void __launch_bounds__(512) sdd_kernel(SddArgs a) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int nb = a.sdd_h >> 1;  // bands per frame
+  const int f = blockIdx.x / nb;
+  const int band = blockIdx.x - f * nb;
+  const FrameDesc fd = a.frames[f];
+  const int W = fd.W, H = fd.H, sdd_w = a.sdd_w, sdd_h = a.sdd_h;
+  const int rowbytes = 3 * W;
+  const int nchunk = (rowbytes + 15) >> 4;
+  const int cs = nchunk * 16;  // u16 column sums per 100-grid row
+  uint16_t* colsum = reinterpret_cast<uint16_t*>(smem);                  // [2][cs]
+  uint32_t* cell = reinterpret_cast<uint32_t*>(smem + 4 * (size_t)cs);   // [2][3*sdd_w]
+  __shared__ uint32_t red[32];
+  __shared__ int s_last;
+
+  // Source rows of the two 100-grid rows of this band: [ya0, ya1) and [ya1, yb1).
+  const int ya0 = (int)(((int64_t)(2 * band) * H) / sdd_h);
+  const int ya1 = (int)(((int64_t)(2 * band + 1) * H) / sdd_h);
+  const int yb1 = (int)(((int64_t)(2 * band + 2) * H) / sdd_h);
+  const int rows = yb1 - ya0, split = ya1 - ya0;
+
+  // ---- phase 1: stream the band's rows, vertical column sums in registers
+  for (int c = threadIdx.x; c < nchunk; c += blockDim.x) {
+    uint32_t accA[8] = {0, 0, 0, 0, 0, 0, 0, 0}, accB[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    const uint8_t* base = fd.pixels + (int64_t)ya0 * fd.pitch;
+    for (int r0 = 0; r0 < rows; r0 += 8) {
+      uint4 v[8];
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+        v[i] = (r0 + i < rows) ? load_chunk(base + (int64_t)(r0 + i) * fd.pitch, c, rowbytes, a.vec16)
+                               : make_uint4(0u, 0u, 0u, 0u);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        if (r0 + i < split) acc16(accA, v[i]);
+        else acc16(accB, v[i]);
+      }
+    }
+    store_colsum(reinterpret_cast<uint32_t*>(colsum), c, accA);
+    store_colsum(reinterpret_cast<uint32_t*>(colsum + cs), c, accB);
+  }
+  __syncthreads();
+
+  // ---- phase 2: 100-grid cell sums, D100, SSD against R
+  const int row3 = 3 * sdd_w;
+  uint32_t ssd_local = 0;
+  for (int o = threadIdx.x; o < 2 * row3; o += blockDim.x) {
+    const int sub = o >= row3;
+    const int r = o - sub * row3;
+    const int cx = r / 3, ch = r - 3 * cx;
+    const int x0 = (int)(((int64_t)cx * W) / sdd_w), x1 = (int)(((int64_t)(cx + 1) * W) / sdd_w);
+    const uint16_t* col = colsum + sub * cs + ch;
+    uint32_t s = 0;
+    for (int x = x0; x < x1; ++x) s += col[3 * x];
+    cell[o] = s;
+    const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)(sub ? rows - split : split);
+    const uint32_t d = (s + (n >> 1)) / n;
+    const int yrow = 2 * band + sub;
+    if (kD100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)yrow * row3 + r] = (uint8_t)d;
+    const int diff = (int)d - (int)__ldg(fd.ref + (int64_t)yrow * row3 + r);
+    ssd_local += (uint32_t)(diff * diff);
+  }
+  __syncthreads();
+
+  // ---- phase 3: D50 row from the four 100-cell sums of each 50-cell
+  const int half3 = 3 * (sdd_w >> 1);
+  for (int o = threadIdx.x; o < half3; o += blockDim.x) {
+    const int cx = o / 3, ch = o - 3 * cx;
+    const uint32_t s = cell[6 * cx + ch] + cell[6 * cx + 3 + ch] + cell[row3 + 6 * cx + ch] +
+                       cell[row3 + 6 * cx + 3 + ch];
+    const int x0 = (int)(((int64_t)(2 * cx) * W) / sdd_w), x1 = (int)(((int64_t)(2 * cx + 2) * W) / sdd_w);
+    const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)rows;
+    a.d50[(int64_t)f * a.d50_stride + (int64_t)band * half3 + o] = (uint8_t)((s + (n >> 1)) / n);
+  }
+
+  // ---- block SSD partial, then the frame's last CTA finalises
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) ssd_local += __shfl_xor_sync(0xffffffffu, ssd_local, off);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) red[warp] = ssd_local;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t t = 0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += red[w];
+    a.partial[(int64_t)f * nb + band] = t;
+    __threadfence();
+    const unsigned ticket = atomicAdd(a.counter + f, 1u);
+    s_last = (ticket == (unsigned)(nb - 1));
+  }
+  __syncthreads();
+  if (s_last && warp == 0) {
+    __threadfence();
+    unsigned long long sum = 0;
+    for (int b = lane; b < nb; b += 32) sum += __ldcg(a.partial + (int64_t)f * nb + b);
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, off);
+    if (lane == 0) {
+      const uint8_t p = sum > fd.T ? 1 : 0;
+      a.ssd[f] = sum;
+      a.pass[f] = p;
+      a.counter[f] = 0u;
+      if (a.stats) {  // a8: per-stream counters
+        unsigned long long* st = a.stats + (int64_t)fd.slot * NSTAT;
+        atomicAdd(st + 0, 1ull);
+        atomicAdd(st + 1, (unsigned long long)p);
+        atomicAdd(st + 3, sum);
+      }
+    }
+  }
+}
+
+// Reference image R: one rounding of the mean over k frames x box. One thread per value.
+__global__ void reference_kernel(const uint8_t* __restrict__ frames, int32_t k, int64_t frame_stride, int32_t W,
+                                 int32_t H, int64_t pitch, int32_t sdd_w, int32_t sdd_h, uint8_t* __restrict__ out) {
+  const int o = blockIdx.x * blockDim.x + threadIdx.x;
+  if (o >= 3 * sdd_w * sdd_h) return;
+  const int oy = o / (3 * sdd_w), r = o - oy * 3 * sdd_w, ox = r / 3, ch = r - 3 * ox;
+  const int64_t y0 = ((int64_t)oy * H) / sdd_h, y1 = ((int64_t)(oy + 1) * H) / sdd_h;
+  const int64_t x0 = ((int64_t)ox * W) / sdd_w, x1 = ((int64_t)(ox + 1) * W) / sdd_w;
+  unsigned long long s = 0;
+  for (int j = 0; j < k; ++j)
+    for (int64_t y = y0; y < y1; ++y) {
+      const uint8_t* row = frames + (int64_t)j * frame_stride + y * pitch + ch;
+      for (int64_t x = x0; x < x1; ++x) s += row[3 * x];
+    }
+  const unsigned long long n = (unsigned long long)k * (unsigned long long)((y1 - y0) * (x1 - x0));
+  out[o] = (uint8_t)((s + n / 2) / n);
+}
+
+__global__ void fill_nan_kernel(float* p, int32_t n) {
+  int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < n) p[i] = __int_as_float(0x7fc00000);
+}
+
+}  // namespace
+
+size_t sdd_smem_bytes(int max_chunks, int sdd_w) { return (size_t)4 * 16 * max_chunks + (size_t)8 * 3 * sdd_w; }
+
+int sdd_threads(int max_chunks) {
+  int t = ((max_chunks + 31) / 32) * 32;
+  if (t < 64) t = 64;
+  if (t > 512) t = 512;
+  return t;
+}
+
+cudaError_t sdd_configure(size_t smem) {
+  static size_t configured = 0;
+  if (smem <= configured) return cudaSuccess;
+  cudaError_t e = cudaFuncSetAttribute(sdd_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(sdd_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess) configured = smem;
+  return e;
+}
+
+cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st) {
+  if (a.n <= 0) return cudaSuccess;
+  const size_t smem = sdd_smem_bytes(a.max_chunks, a.sdd_w);
+  const int threads = sdd_threads(a.max_chunks);
+  const unsigned grid = (unsigned)a.n * (unsigned)(a.sdd_h / 2);
+  if (a.d100) sdd_kernel<true><<<grid, threads, smem, st>>>(a);
+  else sdd_kernel<false><<<grid, threads, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_reference(const uint8_t* frames, int32_t k, int64_t frame_stride, int32_t W, int32_t H,
+                             int64_t pitch, int32_t sdd_w, int32_t sdd_h, uint8_t* out, cudaStream_t st) {
+  const int n = 3 * sdd_w * sdd_h;
+  reference_kernel<<<(n + 127) / 128, 128, 0, st>>>(frames, k, frame_stride, W, H, pitch, sdd_w, sdd_h, out);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_fill_nan(float* p, int32_t n, cudaStream_t st) {
+  if (n <= 0) return cudaSuccess;
+  fill_nan_kernel<<<(n + 255) / 256, 256, 0, st>>>(p, n);
+  return cudaGetLastError();
+}
+
+}  // namespace ffsva

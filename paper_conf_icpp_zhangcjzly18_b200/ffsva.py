@@ -1,0 +1,359 @@
+"""Thin Python binding of the C-ABI in include/ffsva.h (ctypes argument marshalling only).
+
+Every function named ``ffsva_*`` here is the C entry point of the same name; every step of the filter
+cascade runs in the library's sm_100a kernels (paper_conf_icpp_zhangcjzly18_b200/lib/libffsva.so). There is
+no CPU fallback: if the library is missing this module raises at import of the library, and on a machine
+without a B200 every compute call fails with FFSVA_ECUDA.
+
+The small convenience layer (``Context``, ``Stream``, ``PreparedBatch``) converts torch tensors / numpy
+arrays to pointers and results to numpy arrays.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "lib", "libffsva.so")
+
+FFSVA_OK, FFSVA_EINVAL, FFSVA_ENOMEM, FFSVA_ECUDA, FFSVA_ESTATE, FFSVA_EAGAIN, FFSVA_EDEVICE = 0, -1, -2, -3, -4, -5, -6
+STATUS_NAMES = {0: "FFSVA_OK", -1: "FFSVA_EINVAL", -2: "FFSVA_ENOMEM", -3: "FFSVA_ECUDA", -4: "FFSVA_ESTATE",
+                -5: "FFSVA_EAGAIN", -6: "FFSVA_EDEVICE"}
+STAT_NAMES = ["frames", "sdd_pass", "snm_pass", "ssd_sum", "class0", "class1", "class2", "snm_batches"]
+NSTAT = len(STAT_NAMES)
+
+# Every symbol include/ffsva.h declares (checked by tests/test_abi.py).
+EXPORTS = ["ffsva_open_stream", "ffsva_set_reference", "ffsva_snm_load", "ffsva_filter_batch",
+           "ffsva_filter_batch_host", "ffsva_batch_prepare", "ffsva_batch_launch", "ffsva_batch_fetch",
+           "ffsva_batch_device_outputs", "ffsva_batch_destroy", "ffsva_batch_profile", "ffsva_sdd_batch",
+           "ffsva_get_reference",
+           "ffsva_stream_info", "ffsva_stats_copy", "ffsva_close", "ffsva_last_error", "ffsva_kernel_launches",
+           "ffsva_version"]
+
+
+class StreamDesc(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int32), ("width", ctypes.c_int32), ("height", ctypes.c_int32),
+                ("row_pitch", ctypes.c_int64), ("sdd_w", ctypes.c_int32), ("sdd_h", ctypes.c_int32),
+                ("snm_w", ctypes.c_int32), ("snm_h", ctypes.c_int32), ("delta_diff", ctypes.c_double),
+                ("c_low", ctypes.c_float), ("c_high", ctypes.c_float), ("filter_degree", ctypes.c_float),
+                ("snm_batch", ctypes.c_int32), ("q_sdd", ctypes.c_int32), ("q_snm", ctypes.c_int32)]
+
+
+class SnmDesc(ctypes.Structure):
+    _fields_ = [("c1", ctypes.c_int32), ("c2", ctypes.c_int32)]
+
+
+class Frame(ctypes.Structure):
+    _fields_ = [("stream", ctypes.c_void_p), ("pixels", ctypes.c_void_p), ("frame_no", ctypes.c_int64)]
+
+
+class Result(ctypes.Structure):
+    _fields_ = [("ssd", ctypes.c_uint64), ("sdd_pass", ctypes.c_uint8), ("snm_pass", ctypes.c_uint8),
+                ("snm_class", ctypes.c_uint8), ("pad", ctypes.c_uint8), ("logit", ctypes.c_float),
+                ("survivor_idx", ctypes.c_int32)]
+
+
+RESULT_DTYPE = np.dtype([("ssd", "<u8"), ("sdd_pass", "u1"), ("snm_pass", "u1"), ("snm_class", "u1"),
+                         ("pad", "u1"), ("logit", "<f4"), ("survivor_idx", "<i4")], align=True)
+assert RESULT_DTYPE.itemsize == ctypes.sizeof(Result) == 24
+
+_lib = None
+
+
+def lib():
+    """Load libffsva.so (fails loudly if the extension was not built: there is no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: run `python __graft_entry__.py` (build) first; "
+                               "the filter cascade has no CPU fallback")
+        L = ctypes.CDLL(LIB_PATH)
+        vp, i32, i64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+        sig = {
+            "ffsva_open_stream": [ctypes.POINTER(StreamDesc), ctypes.POINTER(vp)],
+            "ffsva_set_reference": [vp, vp, i32, i64],
+            "ffsva_snm_load": [vp, ctypes.POINTER(SnmDesc), vp, i64],
+            "ffsva_filter_batch": [vp, i32, vp, vp],
+            "ffsva_filter_batch_host": [vp, i32, vp, vp],
+            "ffsva_batch_prepare": [vp, i32, ctypes.POINTER(vp)],
+            "ffsva_batch_launch": [vp, vp],
+            "ffsva_batch_fetch": [vp, vp, vp],
+            "ffsva_batch_device_outputs": [vp] + [ctypes.POINTER(vp)] * 7 + [ctypes.POINTER(i64), ctypes.POINTER(vp)],
+            "ffsva_batch_destroy": [vp],
+            "ffsva_batch_profile": [vp, i32, i32, vp, vp],
+            "ffsva_sdd_batch": [vp, i32, vp, vp, vp, vp, vp],
+            "ffsva_get_reference": [vp, vp],
+            "ffsva_stream_info": [vp, ctypes.POINTER(i32), ctypes.POINTER(i32)],
+            "ffsva_stats_copy": [i32, vp, i32, ctypes.POINTER(i32), i32, i32, vp],
+            "ffsva_close": [vp],
+        }
+        for name, args in sig.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = ctypes.c_int
+        L.ffsva_last_error.restype = ctypes.c_char_p
+        L.ffsva_last_error.argtypes = []
+        L.ffsva_version.restype = ctypes.c_char_p
+        L.ffsva_version.argtypes = []
+        L.ffsva_kernel_launches.restype = ctypes.c_uint64
+        L.ffsva_kernel_launches.argtypes = []
+        _lib = L
+    return _lib
+
+
+class FfsvaError(RuntimeError):
+    def __init__(self, status: int, where: str):
+        self.status = status
+        msg = lib().ffsva_last_error().decode()
+        super().__init__(f"{where}: {STATUS_NAMES.get(status, status)}: {msg}")
+
+
+def _check(status: int, where: str) -> None:
+    if status != FFSVA_OK:
+        raise FfsvaError(status, where)
+
+
+# ------------------------------------------------------------------ C entry points, same names
+
+def ffsva_open_stream(desc: StreamDesc):
+    h = ctypes.c_void_p()
+    _check(lib().ffsva_open_stream(ctypes.byref(desc), ctypes.byref(h)), "ffsva_open_stream")
+    return h.value
+
+
+def ffsva_set_reference(stream, frames_ptr: int, k: int, frame_stride: int) -> None:
+    _check(lib().ffsva_set_reference(stream, frames_ptr, k, frame_stride), "ffsva_set_reference")
+
+
+def ffsva_snm_load(stream, params: np.ndarray, c1: int = 16, c2: int = 32) -> None:
+    p = np.ascontiguousarray(params, dtype=np.float32)
+    d = SnmDesc(c1, c2)
+    _check(lib().ffsva_snm_load(stream, ctypes.byref(d), p.ctypes.data, p.size), "ffsva_snm_load")
+
+
+def _frames_array(frames):
+    arr = (Frame * max(1, len(frames)))()
+    for i, (s, ptr, no) in enumerate(frames):
+        arr[i].stream = s
+        arr[i].pixels = ptr
+        arr[i].frame_no = no
+    return arr
+
+
+def ffsva_filter_batch(frames, cuda_stream: int = 0, host: bool = False) -> np.ndarray:
+    """frames: list of (stream handle, pixels pointer, frame_no). Returns a RESULT_DTYPE array."""
+    n = len(frames)
+    arr = _frames_array(frames)
+    out = np.zeros(max(1, n), dtype=RESULT_DTYPE)
+    fn = lib().ffsva_filter_batch_host if host else lib().ffsva_filter_batch
+    _check(fn(arr, n, out.ctypes.data, cuda_stream), "ffsva_filter_batch_host" if host else "ffsva_filter_batch")
+    return out[:n]
+
+
+def ffsva_sdd_batch(frames, sdd_w: int, sdd_h: int, want_d100: bool = True, cuda_stream: int = 0):
+    n = len(frames)
+    arr = _frames_array(frames)
+    d100 = np.zeros((max(1, n), sdd_h, sdd_w, 3), np.uint8) if want_d100 else None
+    d50 = np.zeros((max(1, n), sdd_h // 2, sdd_w // 2, 3), np.uint8)
+    ssd = np.zeros(max(1, n), np.uint64)
+    ps = np.zeros(max(1, n), np.uint8)
+    _check(lib().ffsva_sdd_batch(arr, n, d100.ctypes.data if want_d100 else None, d50.ctypes.data,
+                                 ssd.ctypes.data, ps.ctypes.data, cuda_stream), "ffsva_sdd_batch")
+    return dict(d100=d100[:n] if want_d100 else None, d50=d50[:n], ssd=ssd[:n], sdd_pass=ps[:n])
+
+
+def ffsva_batch_prepare(frames):
+    arr = _frames_array(frames)
+    h = ctypes.c_void_p()
+    _check(lib().ffsva_batch_prepare(arr, len(frames), ctypes.byref(h)), "ffsva_batch_prepare")
+    return h.value
+
+
+def ffsva_batch_launch(batch, cuda_stream: int) -> None:
+    _check(lib().ffsva_batch_launch(batch, cuda_stream), "ffsva_batch_launch")
+
+
+def ffsva_batch_fetch(batch, n: int | None, cuda_stream: int):
+    if n is None:
+        _check(lib().ffsva_batch_fetch(batch, None, cuda_stream), "ffsva_batch_fetch")
+        return None
+    out = np.zeros(max(1, n), dtype=RESULT_DTYPE)
+    _check(lib().ffsva_batch_fetch(batch, out.ctypes.data, cuda_stream), "ffsva_batch_fetch")
+    return out[:n]
+
+
+def ffsva_batch_device_outputs(batch) -> dict:
+    ptrs = [ctypes.c_void_p() for _ in range(7)]
+    stride = ctypes.c_int64()
+    cnt = ctypes.c_void_p()
+    _check(lib().ffsva_batch_device_outputs(batch, *[ctypes.byref(p) for p in ptrs], ctypes.byref(stride),
+                                            ctypes.byref(cnt)), "ffsva_batch_device_outputs")
+    names = ["ssd", "sdd_pass", "survivor_idx", "logit", "snm_pass", "snm_class", "d50"]
+    d = {k: p.value for k, p in zip(names, ptrs)}
+    d["d50_stride"] = stride.value
+    d["n_survivors"] = cnt.value
+    return d
+
+
+def ffsva_batch_destroy(batch) -> None:
+    _check(lib().ffsva_batch_destroy(batch), "ffsva_batch_destroy")
+
+
+def ffsva_batch_profile(batches, iters: int, cuda_stream: int) -> list:
+    """Mean device ms per launch of [K1, K3, K4] over iters passes of the prepared batches."""
+    arr = (ctypes.c_void_p * len(batches))(*batches)
+    ms = (ctypes.c_float * 3)()
+    _check(lib().ffsva_batch_profile(arr, len(batches), iters, ms, cuda_stream), "ffsva_batch_profile")
+    return [float(x) for x in ms]
+
+
+def ffsva_get_reference(stream, sdd_w: int, sdd_h: int) -> np.ndarray:
+    out = np.zeros((sdd_h, sdd_w, 3), np.uint8)
+    _check(lib().ffsva_get_reference(stream, out.ctypes.data), "ffsva_get_reference")
+    return out
+
+
+def ffsva_stream_info(stream):
+    slot, dev = ctypes.c_int32(), ctypes.c_int32()
+    _check(lib().ffsva_stream_info(stream, ctypes.byref(slot), ctypes.byref(dev)), "ffsva_stream_info")
+    return slot.value, dev.value
+
+
+def ffsva_stats_copy(device: int, dst_ptr: int, max_slots: int, dst_is_host: bool, reset: bool = False,
+                     cuda_stream: int = 0) -> int:
+    slots = ctypes.c_int32()
+    _check(lib().ffsva_stats_copy(device, dst_ptr, max_slots, ctypes.byref(slots), int(dst_is_host), int(reset),
+                                  cuda_stream), "ffsva_stats_copy")
+    return slots.value
+
+
+def ffsva_close(stream) -> None:
+    _check(lib().ffsva_close(stream), "ffsva_close")
+
+
+def ffsva_kernel_launches() -> int:
+    return int(lib().ffsva_kernel_launches())
+
+
+def ffsva_version() -> str:
+    return lib().ffsva_version().decode()
+
+
+# ------------------------------------------------------------------ convenience layer
+
+def _stream_handle(stream):
+    """torch.cuda.Stream / int / None -> cudaStream_t value."""
+    if stream is None:
+        return 0
+    if isinstance(stream, int):
+        return stream
+    return int(stream.cuda_stream)
+
+
+class Stream:
+    """One camera stream (per-stream SDD + SNM)."""
+
+    def __init__(self, ctx: "Context", desc: StreamDesc):
+        self.ctx = ctx
+        self.desc = desc
+        self.handle = ffsva_open_stream(desc)
+        self.slot, self.device = ffsva_stream_info(self.handle)
+
+    def set_reference(self, frames, k: int | None = None, frame_stride: int | None = None) -> None:
+        """frames: torch tensor (device or host) or numpy array of k background frames (k, H, pitch)."""
+        if isinstance(frames, np.ndarray):
+            frames = np.ascontiguousarray(frames)
+            k = frames.shape[0] if k is None else k
+            stride = frames[0].nbytes if frame_stride is None else frame_stride
+            ffsva_set_reference(self.handle, frames.ctypes.data, k, stride)
+        else:
+            frames = frames.contiguous()
+            k = frames.shape[0] if k is None else k
+            stride = frames[0].numel() * frames.element_size() if frame_stride is None else frame_stride
+            ffsva_set_reference(self.handle, frames.data_ptr(), k, stride)
+
+    def snm_load(self, params: np.ndarray) -> None:
+        ffsva_snm_load(self.handle, params)
+
+    def reference(self) -> np.ndarray:
+        return ffsva_get_reference(self.handle, self.desc.sdd_w, self.desc.sdd_h)
+
+    def close(self) -> None:
+        if self.handle:
+            ffsva_close(self.handle)
+            self.handle = None
+
+
+class Context:
+    """Per-device convenience wrapper; the device context itself lives inside the library."""
+
+    def __init__(self, device=0):
+        self.device = device.index if hasattr(device, "index") and device.index is not None else int(
+            getattr(device, "index", device) or 0)
+        self.streams: list[Stream] = []
+
+    def open_stream(self, width: int, height: int, row_pitch: int | None = None, delta_diff: float = 24.0,
+                    c_low: float = 0.2, c_high: float = 0.8, filter_degree: float = 0.5, snm_batch: int = 30,
+                    q_sdd: int = 2, q_snm: int = 10, sdd=(100, 100)) -> Stream:
+        d = StreamDesc(self.device, width, height, 3 * width if row_pitch is None else row_pitch, sdd[0], sdd[1],
+                       sdd[0] // 2, sdd[1] // 2, delta_diff, c_low, c_high, filter_degree, snm_batch, q_sdd, q_snm)
+        s = Stream(self, d)
+        self.streams.append(s)
+        return s
+
+    @staticmethod
+    def _frames(items):
+        out = []
+        for s, px, no in items:
+            ptr = px if isinstance(px, int) else (px.ctypes.data if isinstance(px, np.ndarray) else px.data_ptr())
+            out.append((s.handle, ptr, no))
+        return out
+
+    def filter_batch(self, items, stream=None, host: bool = False) -> dict:
+        """items: list of (Stream, pixels tensor/pointer, frame_no). Returns dict of per-frame numpy arrays."""
+        r = ffsva_filter_batch(self._frames(items), _stream_handle(stream), host=host)
+        return {k: r[k].copy() for k in ("ssd", "sdd_pass", "snm_pass", "snm_class", "logit", "survivor_idx")}
+
+    def sdd_batch(self, items, want_d100: bool = True, stream=None) -> dict:
+        s0 = items[0][0].desc
+        return ffsva_sdd_batch(self._frames(items), s0.sdd_w, s0.sdd_h, want_d100, _stream_handle(stream))
+
+    def prepare(self, items) -> "PreparedBatch":
+        return PreparedBatch(self._frames(items))
+
+    def stats(self, max_slots: int = 1024, reset: bool = False) -> np.ndarray:
+        out = np.zeros((max_slots, NSTAT), np.uint64)
+        slots = ffsva_stats_copy(self.device, out.ctypes.data, max_slots, True, reset)
+        return out[:min(slots, max_slots)]
+
+    def close(self) -> None:
+        for s in self.streams:
+            s.close()
+        self.streams = []
+
+
+class PreparedBatch:
+    """ffsva_batch_prepare / launch (CUDA graph replay) / fetch."""
+
+    def __init__(self, frames):
+        self.n = len(frames)
+        self.handle = ffsva_batch_prepare(frames)
+
+    def launch(self, stream=None) -> None:
+        ffsva_batch_launch(self.handle, _stream_handle(stream))
+
+    def fetch(self, stream=None, results: bool = True):
+        r = ffsva_batch_fetch(self.handle, self.n if results else None, _stream_handle(stream))
+        if r is None:
+            return None
+        return {k: r[k].copy() for k in ("ssd", "sdd_pass", "snm_pass", "snm_class", "logit", "survivor_idx")}
+
+    def device_outputs(self) -> dict:
+        return ffsva_batch_device_outputs(self.handle)
+
+    def destroy(self) -> None:
+        if self.handle:
+            ffsva_batch_destroy(self.handle)
+            self.handle = None

@@ -1,0 +1,89 @@
+"""Helpers shared by the GPU parity tests (tests/ only): set up streams through the C-ABI binding and run the
+same seeded inputs through the oracle."""
+from __future__ import annotations
+
+import numpy as np
+
+from oracle import oracle as orc
+from synth import synth
+
+SNM_TOL = 2e-2        # north_star: SNM logits within 2e-2 absolute of the oracle
+SNM_TOL_BF16 = 2e-3   # vs the oracle's bf16-emulation mode (same operand rounding as the kernel)
+F32 = np.float32
+
+
+def f32(x: float) -> float:
+    """The float32 value the C-ABI stores for a threshold, as a double for the oracle."""
+    return float(np.float32(x))
+
+
+class Cam:
+    """One synthetic camera: its video, its reference frames and its SNM weights."""
+
+    def __init__(self, ctx, video: synth.Video, stream_id: int, dev, delta=24.0, c_low=0.2, c_high=0.8, fd=0.5,
+                 snm_batch=30, pitch=None, k_ref=8, bias_std=0.05, load_snm=True):
+        import torch
+        self.video, self.sid, self.dev = video, stream_id, dev
+        self.pitch = 3 * video.width if pitch is None else pitch
+        self.delta, self.c_low, self.c_high, self.fd = delta, c_low, c_high, fd
+        self.st = ctx.open_stream(width=video.width, height=video.height, row_pitch=self.pitch, delta_diff=delta,
+                                  c_low=c_low, c_high=c_high, filter_degree=fd, snm_batch=snm_batch)
+        self.refs = synth.frames(video, [stream_id] * k_ref, list(range(k_ref)), ref=True, pitch=self.pitch)
+        self.st.set_reference(torch.from_numpy(self.refs).to(dev))
+        self.R = orc.reference(self.refs, video.width, 100, 100)
+        self.params = synth.snm_weights(video.seed, stream_id, bias_std=bias_std)
+        if load_snm:
+            self.st.snm_load(self.params)
+
+    def host_frames(self, ts):
+        return synth.frames(self.video, [self.sid] * len(ts), ts, pitch=self.pitch)
+
+
+def oracle_for(cams_and_frames, run_snm=True, bf16_emul=False):
+    """cams_and_frames: list of (Cam, host frame (H, pitch)). Runs the oracle cascade in batch order."""
+    frames = [f for _, f in cams_and_frames]
+    cams = [c for c, _ in cams_and_frames]
+    # all cameras of one call must share the frame width for filter_frames; group by width
+    widths = {c.video.width for c in cams}
+    assert len(widths) == 1
+    return orc.filter_frames(frames, cams[0].video.width, [c.R for c in cams], [c.delta for c in cams],
+                             [c.params for c in cams], [f32(c.c_low) for c in cams], [f32(c.c_high) for c in cams],
+                             [f32(c.fd) for c in cams], bf16_emul=bf16_emul, run_snm=run_snm)
+
+
+def oracle_mixed(cams_and_frames, run_snm=True, bf16_emul=False):
+    """Like oracle_for but frame by frame (any mix of resolutions)."""
+    outs = [oracle_for([cf], run_snm=False) for cf in cams_and_frames]
+    n = len(outs)
+    res = {k: np.concatenate([o[k] for o in outs]) for k in ("ssd", "sdd_pass")}
+    surv = orc.compact(res["sdd_pass"])
+    sidx = np.full(n, -1, np.int32)
+    sidx[surv] = np.arange(surv.size, dtype=np.int32)
+    res["survivors"], res["survivor_idx"] = surv, sidx
+    res["d50"] = [o["d50"][0] for o in outs]
+    res["d100"] = [o["d100"][0] for o in outs]
+    lg = np.full(n, np.nan)
+    if run_snm:
+        for i in surv:
+            lg[i] = orc.snm_forward(res["d50"][i], cams_and_frames[i][0].params, bf16_emul=bf16_emul)
+    res["logit"] = lg
+    return res
+
+
+def check_snm(got_logit, got_pass, got_cls, want_logit, cams, survivors, tol=SNM_TOL):
+    """Logits within tol; decisions identical except where the oracle logit is within tol of a threshold."""
+    if survivors.size == 0:
+        return 0.0
+    err = np.abs(got_logit[survivors].astype(np.float64) - want_logit[survivors])
+    assert np.all(np.isfinite(got_logit[survivors]))
+    assert err.max() <= tol, f"max |dlogit| {err.max():.3e} > {tol}"
+    for i in survivors:
+        c = cams[i]
+        lt = orc.logit(orc.tpre(f32(c.c_low), f32(c.c_high), f32(c.fd)))
+        p, k = orc.decide(want_logit[i], f32(c.c_low), f32(c.c_high), f32(c.fd))
+        near = min(abs(want_logit[i] - lt), abs(want_logit[i] - orc.logit(f32(c.c_low))),
+                   abs(want_logit[i] - orc.logit(f32(c.c_high))))
+        if near > tol:
+            assert got_pass[i] == p, (i, want_logit[i], got_logit[i])
+            assert got_cls[i] == k, (i, want_logit[i], got_logit[i])
+    return float(err.max())

@@ -1,0 +1,340 @@
+"""GPU parity: the sm_100a path through the C-ABI vs the CPU oracle on the same seeded inputs.
+
+Bars: D100, D50, SSD, SDD pass and survivor order bit-exact; SNM logits within 2e-2 of the
+fp64 oracle (and within 2e-3 of its bf16-emulation mode); SNM decisions identical except for frames whose
+oracle logit lies within 2e-2 of a threshold (north_star).
+"""
+import numpy as np
+import pytest
+
+from gpu_util import SNM_TOL, SNM_TOL_BF16, Cam, check_snm, f32, oracle_for, oracle_mixed
+from oracle import oracle as orc
+from synth import synth
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def env():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    import __graft_entry__ as ge
+    ge.build()
+    import paper_conf_icpp_zhangcjzly18_b200 as ff
+    dev = torch.device("cuda:0")
+    ctx = ff.Context(dev)
+    yield ff, ctx, dev
+    ctx.close()
+
+
+def _dev(x, dev):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(x)).to(dev)
+
+
+# ------------------------------------------------------------------ reference image (C2)
+
+@pytest.mark.parametrize("W,H,k", [(640, 360, 8), (101, 103, 3), (1920, 1080, 2), (600, 400, 5)])
+def test_reference_parity(env, W, H, k):
+    ff, ctx, dev = env
+    v = synth.Video(seed=31, width=W, height=H)
+    refs = synth.frames(v, [0] * k, list(range(k)), ref=True)
+    want = orc.reference(refs, W, 100, 100)
+    st = ctx.open_stream(width=W, height=H)
+    st.set_reference(_dev(refs, dev))
+    assert np.array_equal(st.reference(), want)
+    st.set_reference(refs)  # host input path
+    assert np.array_equal(st.reference(), want)
+    st.close()
+
+
+# ------------------------------------------------------------------ SDD stage (C1, C3)
+
+def test_sdd_config1_all_frames(env):
+    """Config 1: 1 stream, 300 frames 640x360, 10% target rate: every frame bit-exact; pass count = planted."""
+    ff, ctx, dev = env
+    v = synth.Video(seed=1001, width=640, height=360, period=300, on_len=30)
+    cam = Cam(ctx, v, 0, dev, k_ref=32, load_snm=False)
+    host = cam.host_frames(list(range(300)))
+    d = _dev(host, dev)
+    got = ctx.sdd_batch([(cam.st, d[i], i) for i in range(300)])
+    want = oracle_for([(cam, host[i]) for i in range(300)], run_snm=False)
+    assert np.array_equal(got["d100"], want["d100"])
+    assert np.array_equal(got["d50"], want["d50"])
+    assert np.array_equal(got["ssd"], want["ssd"])
+    assert np.array_equal(got["sdd_pass"], want["sdd_pass"])
+    assert int(got["sdd_pass"].sum()) == synth.planted(v, 0, 0, 300) == 30
+    cam.st.close()
+
+
+@pytest.mark.parametrize("W,H,pitch", [(100, 100, 300), (641, 361, 1923), (640, 360, 2048), (1280, 720, 3840),
+                                       (1920, 1080, 5760), (600, 400, 1800), (600, 400, 1808), (101, 103, 303),
+                                       (3840, 2160, 11520)])
+def test_sdd_edge_shapes(env, W, H, pitch):
+    ff, ctx, dev = env
+    v = synth.Video(seed=W + H, width=W, height=H, period=4, on_len=2)
+    cam = Cam(ctx, v, 3, dev, pitch=pitch, k_ref=2, load_snm=False)
+    ts = list(range(5))
+    host = cam.host_frames(ts)
+    d = _dev(host, dev)
+    got = ctx.sdd_batch([(cam.st, d[i], t) for i, t in enumerate(ts)])
+    want = oracle_for([(cam, host[i]) for i in range(len(ts))], run_snm=False)
+    for k in ("d100", "d50", "ssd", "sdd_pass"):
+        assert np.array_equal(got[k], want[k]), k
+    cam.st.close()
+
+
+def test_sdd_random_bytes_extreme_values(env):
+    """Uniform random bytes (every value 0..255, far from the synthetic recipe) and constant 0/255 frames."""
+    ff, ctx, dev = env
+    rng = np.random.default_rng(77)
+    W, H = 1280, 720
+    st = ctx.open_stream(width=W, height=H, delta_diff=0.0)
+    refs = rng.integers(0, 256, size=(3, H, 3 * W), dtype=np.uint8)
+    st.set_reference(refs)
+    R = orc.reference(refs, W, 100, 100)
+    frames = np.concatenate([rng.integers(0, 256, size=(4, H, 3 * W), dtype=np.uint8),
+                             np.zeros((1, H, 3 * W), np.uint8), np.full((1, H, 3 * W), 255, np.uint8)])
+    d = _dev(frames, dev)
+    got = ctx.sdd_batch([(st, d[i], i) for i in range(len(frames))])
+    for i, f in enumerate(frames):
+        d100 = orc.box_downsample(f, W, 100, 100)
+        assert np.array_equal(got["d100"][i], d100)
+        assert np.array_equal(got["d50"][i], orc.box_downsample(f, W, 50, 50))
+        assert int(got["ssd"][i]) == orc.ssd(d100, R)
+    st.close()
+
+
+def test_mixed_resolutions_and_streams_in_one_batch(env):
+    ff, ctx, dev = env
+    cams = [Cam(ctx, synth.Video(seed=5, width=W, height=H, period=6, on_len=3), s, dev, k_ref=2, load_snm=False)
+            for s, (W, H) in enumerate([(640, 360), (1280, 720), (641, 361)])]
+    items, pairs, keep = [], [], []
+    for t in range(6):
+        for c in cams:
+            h = c.host_frames([t])[0]
+            dd = _dev(h, dev)
+            keep.append(dd)
+            items.append((c.st, dd, t))
+            pairs.append((c, h))
+    got = ctx.sdd_batch(items)
+    want = oracle_mixed(pairs, run_snm=False)
+    assert np.array_equal(got["ssd"], want["ssd"])
+    assert np.array_equal(got["sdd_pass"], want["sdd_pass"])
+    for i in range(len(items)):
+        assert np.array_equal(got["d100"][i], want["d100"][i])
+        assert np.array_equal(got["d50"][i], want["d50"][i])
+    for c in cams:
+        c.st.close()
+
+
+# ------------------------------------------------------------------ compaction (C4) + SNM (C5-C7)
+
+def _run_full(ctx, dev, pairs, host=False):
+    keep = [_dev(h, dev) for _, h in pairs]
+    items = [(c.st, keep[i] if not host else np.ascontiguousarray(h), i) for i, (c, h) in enumerate(pairs)]
+    return ctx.filter_batch(items, host=host)
+
+
+def test_snm_parity_interleaved_streams(env):
+    """3 streams with different weights and nonzero biases, frames interleaved, BatchSize 4 (several dynamic
+    batches per stream), TOR 50%."""
+    ff, ctx, dev = env
+    cams = [Cam(ctx, synth.Video(seed=11, width=640, height=360, period=10, on_len=5), s, dev, snm_batch=4, k_ref=4,
+                bias_std=0.1) for s in range(3)]
+    pairs = [(c, c.host_frames([t])[0]) for t in range(20) for c in cams]
+    got = _run_full(ctx, dev, pairs)
+    want = oracle_for(pairs)
+    assert np.array_equal(got["ssd"], want["ssd"])
+    assert np.array_equal(got["sdd_pass"], want["sdd_pass"])
+    assert np.array_equal(got["survivor_idx"], want["survivor_idx"])
+    surv = want["survivors"]
+    assert surv.size == sum(synth.planted(c.video, c.sid, 0, 20) for c in cams)
+    camlist = [c for c, _ in pairs]
+    err = check_snm(got["logit"], got["snm_pass"], got["snm_class"], want["logit"], camlist, surv, SNM_TOL)
+    want16 = oracle_for(pairs, bf16_emul=True)
+    err16 = np.abs(got["logit"][surv] - want16["logit"][surv]).max()
+    assert err16 <= SNM_TOL_BF16, err16
+    nonsurv = np.setdiff1d(np.arange(len(pairs)), surv)
+    assert np.all(np.isnan(got["logit"][nonsurv]))
+    assert np.all(got["snm_pass"][nonsurv] == 0)
+    print(f"SNM max |dlogit| vs fp64 {err:.3e}, vs bf16-emulated {err16:.3e}, survivors {surv.size}")
+    for c in cams:
+        c.st.close()
+
+
+def test_snm_closed_forms_on_gpu(env):
+    """P10 on the kernel: zero weights -> logit = b_fc exactly; w2 = 0, wfc = 1 -> b_fc + 144 * sum ReLU(b2)."""
+    ff, ctx, dev = env
+    v = synth.Video(seed=2, width=640, height=360, period=2, on_len=2)  # every frame a target frame
+    cam = Cam(ctx, v, 0, dev, k_ref=2)
+    p = np.zeros(orc.snm_n_params(), np.float32)
+    p[-1] = 0.375
+    cam.st.snm_load(p)
+    pairs = [(cam, cam.host_frames([t])[0]) for t in range(4)]
+    got = _run_full(ctx, dev, pairs)
+    assert np.all(got["sdd_pass"] == 1)
+    assert np.all(got["logit"] == np.float32(0.375))
+    rng = np.random.default_rng(3)
+    p = rng.normal(0, 1, orc.snm_n_params()).astype(np.float32)
+    o_w2 = 27 * 16 + 16
+    o_b2 = o_w2 + 9 * 16 * 32
+    p[o_w2:o_b2] = 0
+    p[o_b2 + 32:-1] = 1.0
+    p = synth.to_bf16_values(p)
+    cam.st.snm_load(p)
+    got = _run_full(ctx, dev, pairs)
+    want = float(p[-1]) + 144.0 * float(np.maximum(p[o_b2:o_b2 + 32].astype(np.float64), 0).sum())
+    assert np.all(np.abs(got["logit"] - want) <= 1e-4 * max(1.0, abs(want)))
+    cam.st.close()
+
+
+@pytest.mark.parametrize("delta,expect", [(0.0, "all"), (1e9, "none")])
+def test_compaction_extremes(env, delta, expect):
+    ff, ctx, dev = env
+    v = synth.Video(seed=8, width=128, height=104, period=10, on_len=1)
+    cam = Cam(ctx, v, 0, dev, delta=delta, k_ref=1)
+    pairs = [(cam, cam.host_frames([t])[0]) for t in range(1, 40)]
+    got = _run_full(ctx, dev, pairs)
+    want = oracle_for(pairs)
+    assert np.array_equal(got["sdd_pass"], want["sdd_pass"])
+    assert np.array_equal(got["survivor_idx"], want["survivor_idx"])
+    if expect == "none":
+        assert got["sdd_pass"].sum() == 0 and np.all(got["survivor_idx"] == -1)
+    else:
+        assert got["sdd_pass"].sum() == len(pairs)  # noise makes every SSD > 0
+        check_snm(got["logit"], got["snm_pass"], got["snm_class"], want["logit"], [cam] * len(pairs),
+                  want["survivors"])
+    cam.st.close()
+
+
+def test_compaction_across_scan_tiles(env):
+    """n = 4097 + 4096 frames crosses two 4096-flag scan tiles; 2 streams interleaved in blocks."""
+    ff, ctx, dev = env
+    import torch
+    cams = [Cam(ctx, synth.Video(seed=21 + s, width=100, height=100, period=7, on_len=2), s, dev, k_ref=1,
+                snm_batch=30) for s in range(2)]
+    n = 8193
+    sid = (np.arange(n) // 100) % 2
+    ts = np.arange(n)
+    host = np.stack([cams[s].host_frames([int(t)])[0] for s, t in zip(sid, ts)])
+    d = torch.from_numpy(host).to(dev)
+    got = ctx.filter_batch([(cams[s].st, d[i], int(ts[i])) for i, s in enumerate(sid)])
+    want_pass = np.array([orc.sdd_pass(orc.ssd(orc.box_downsample(host[i], 100, 100, 100), cams[s].R),
+                                       orc.threshold(24.0, 30000)) for i, s in enumerate(sid)], np.uint8)
+    assert np.array_equal(got["sdd_pass"], want_pass)
+    surv = orc.compact(want_pass)
+    sidx = np.full(n, -1, np.int32)
+    sidx[surv] = np.arange(surv.size)
+    assert np.array_equal(got["survivor_idx"], sidx)
+    # SNM on a sample of survivors
+    for i in surv[:: max(1, surv.size // 40)]:
+        lg = orc.snm_forward(orc.box_downsample(host[i], 100, 50, 50), cams[sid[i]].params)
+        assert abs(got["logit"][i] - lg) <= SNM_TOL
+    for c in cams:
+        c.st.close()
+
+
+def test_prepared_batch_graph_replay_and_host_path(env):
+    ff, ctx, dev = env
+    import torch
+    cams = [Cam(ctx, synth.Video(seed=41, width=1280, height=720, period=10, on_len=3), s, dev, k_ref=2,
+                snm_batch=5) for s in range(2)]
+    pairs = [(c, c.host_frames([t])[0]) for c in cams for t in range(12)]
+    keep = [_dev(h, dev) for _, h in pairs]
+    items = [(c.st, keep[i], i) for i, (c, _) in enumerate(pairs)]
+    ref = ctx.filter_batch(items)
+    pb = ctx.prepare(items)
+    s = torch.cuda.Stream()
+    for _ in range(3):
+        pb.launch(s)
+    got = pb.fetch(s)
+    for k in ref:
+        assert np.array_equal(got[k], ref[k], equal_nan=True), k
+    pb.destroy()
+    pinned = [torch.from_numpy(h).pin_memory() for _, h in pairs]
+    host_items = [(c.st, pinned[i].data_ptr(), i) for i, (c, _) in enumerate(pairs)]
+    got_h = ctx.filter_batch(host_items, host=True)
+    for k in ref:
+        assert np.array_equal(got_h[k], ref[k], equal_nan=True), k
+    want = oracle_for(pairs)
+    assert np.array_equal(ref["ssd"], want["ssd"])
+    check_snm(ref["logit"], ref["snm_pass"], ref["snm_class"], want["logit"], [c for c, _ in pairs],
+              want["survivors"])
+    for c in cams:
+        c.st.close()
+
+
+def test_stats_counters(env):
+    ff, ctx, dev = env
+    cams = [Cam(ctx, synth.Video(seed=51, width=640, height=360, period=10, on_len=4), s, dev, snm_batch=3, k_ref=2)
+            for s in range(2)]
+    ctx.stats(reset=True)
+    pairs = [(c, c.host_frames([t])[0]) for t in range(10) for c in cams]
+    got = _run_full(ctx, dev, pairs)
+    st = ctx.stats()
+    for c in cams:
+        idx = np.array([i for i, (cc, _) in enumerate(pairs) if cc is c])
+        row = st[c.st.slot]
+        assert row[0] == idx.size
+        assert row[1] == got["sdd_pass"][idx].sum()
+        assert row[2] == got["snm_pass"][idx].sum()
+        assert row[3] == got["ssd"][idx].sum()
+        assert row[4] + row[5] + row[6] == got["sdd_pass"][idx].sum()
+        q = int(got["sdd_pass"][idx].sum())
+        assert row[7] == (q + 2) // 3  # dynamic batches of <= BatchSize 3 (L223)
+    for c in cams:
+        c.st.close()
+
+
+def test_synth_device_generator_matches_host(env):
+    ff, ctx, dev = env
+    import torch
+    v = synth.Video(seed=9, width=1280, height=720, period=10, on_len=4)
+    s = torch.tensor([0, 1, 2, 5], dtype=torch.int32, device=dev)
+    t = torch.tensor([0, 3, 4, 100], dtype=torch.int64, device=dev)
+    out = torch.empty((4, 720, 3840), dtype=torch.uint8, device=dev)
+    synth.frames_cuda(v, s, t, out, 720 * 3840, 3840)
+    torch.cuda.synchronize()
+    want = synth.frames(v, [0, 1, 2, 5], [0, 3, 4, 100])
+    assert np.array_equal(out.cpu().numpy(), want)
+
+
+def test_full_size_config2_sampled(env):
+    """Config 2 at full size in the bench's launch configuration: 30 streams x 30 frames of 720p (one second of
+    video), prepared batch + graph replay. Property at full size: SDD pass count == planted count; sampled
+    frames checked element by element against the oracle."""
+    ff, ctx, dev = env
+    import torch
+    S, F, W, H = 30, 30, 1280, 720
+    v = synth.Video(seed=1002, width=W, height=H, period=300, on_len=30)
+    cams = [Cam(ctx, v, s, dev, k_ref=8, snm_batch=30) for s in range(S)]
+    sid = torch.arange(S, dtype=torch.int32, device=dev).repeat_interleave(F)
+    t0 = 120
+    ts = (torch.arange(F, dtype=torch.int64, device=dev) + t0).repeat(S)
+    pool = torch.empty((S * F, H, 3 * W), dtype=torch.uint8, device=dev)
+    synth.frames_cuda(v, sid, ts, pool, H * 3 * W, 3 * W)
+    torch.cuda.synchronize()
+    items = [(cams[i // F].st, pool[i], t0 + i % F) for i in range(S * F)]
+    pb = ctx.prepare(items)
+    s = torch.cuda.Stream()
+    pb.launch(s)
+    pb.launch(s)
+    got = pb.fetch(s)
+    planted = sum(synth.planted(v, k, t0, t0 + F) for k in range(S))
+    assert int(got["sdd_pass"].sum()) == planted
+    sid_h, ts_h = sid.cpu().numpy(), ts.cpu().numpy()
+    for i in range(S * F):
+        assert got["sdd_pass"][i] == int(synth.is_target(v, int(sid_h[i]), int(ts_h[i])))
+    sample = [i for i in range(S * F) if i % 61 == 0] + [int(i) for i in np.flatnonzero(got["sdd_pass"])[:8]]
+    for i in sample:
+        c = cams[i // F]
+        h = c.host_frames([int(ts_h[i])])[0]
+        w = oracle_for([(c, h)])
+        assert int(got["ssd"][i]) == int(w["ssd"][0])
+        if w["sdd_pass"][0]:
+            assert abs(got["logit"][i] - w["logit"][0]) <= SNM_TOL
+    pb.destroy()
+    for c in cams:
+        c.st.close()
