@@ -150,20 +150,32 @@ __global__ void __launch_bounds__(kThreads) compact_kernel(CompactArgs a) {
   if (threadIdx.x == 0) a.posw[n] = carry;
   __syncthreads();
 
-  // ---------------- pass 3: per-stream pops of <= BatchSize (dynamic batching, L223)
+  // ---------------- pass 3: per-stream pops of <= BatchSize (dynamic batching, L223), each pop split into
+  // SNM work units of U frames so that small batches still spread over the SNM grid (U = m / snm_ctas,
+  // clamped to [1, BatchSize]; a unit never crosses a pop, so a pop's frames share one stream's weights)
+  const int m_all = carry;
   int chunk_carry = 0;
   for (int base = 0; base < a.n_seg; base += kThreads) {
     const int s = base + threadIdx.x;
-    int q = 0, B = 1, lo_pos = 0;
+    int q = 0, B = 1, lo_pos = 0, U = 1;
     if (s < a.n_seg) {
       lo_pos = a.posw[a.seg_lo[s]];
       q = a.posw[a.seg_lo[s + 1]] - lo_pos;  // this stream's SNM queue depth
       B = a.seg_batch[s];
+      U = a.snm_ctas > 0 ? m_all / a.snm_ctas : B;
+      U = U < 1 ? 1 : (U > B ? B : U);
+      if (a.stats && q > 0) atomicAdd(a.stats + (int64_t)a.seg_slot[s] * NSTAT + 7, (unsigned long long)((q + B - 1) / B));
     }
-    const int nch = (q + B - 1) / B;
+    const int full = q / B, rest = q - full * B;
+    const int per_full = (B + U - 1) / U;
+    const int nch = full * per_full + (rest + U - 1) / U;
     int total;
     const int off = chunk_carry + block_exclusive_scan(nch, s_warp, &total);
-    for (int j = 0; j < nch; ++j) a.chunks[off + j] = lo_pos + j * B;
+    int k = off;
+    for (int p = 0; p <= full; ++p) {
+      const int plen = p < full ? B : rest;
+      for (int u = 0; u < plen; u += U) a.chunks[k++] = lo_pos + p * B + u;
+    }
     chunk_carry += total;
   }
   if (threadIdx.x == 0) {

@@ -97,13 +97,15 @@ extern "C" FFSVA_API ffsva_status ffsva_filter_batch_host(const ffsva_frame* fra
     sa.d50 = b->d_d50 + (size_t)i0 * b->d50_stride;
     sa.d50_stride = b->d50_stride;
     sa.d100 = nullptr;
-    sa.partial = b->d_partial + (size_t)i0 * nb;
+    sa.partial = b->d_partial + (size_t)i0 * 2 * nb;
     sa.counter = b->d_counter + i0;
     sa.ssd = b->d_ssd + i0;
     sa.pass = b->d_pass + i0;
     sa.stats = ctx->d_stats;
     sa.max_chunks = b->max_chunks;
     sa.vec16 = b->vec16;
+    sa.bulk = b->bulk;
+    sa.stage_bytes = b->stage_bytes;
     if ((e = launch_sdd(sa, cs)) != cudaSuccess) st = cuda_fail(ctx, e, "launch_sdd");
     g_launches += 1;
     cudaEventRecord(ev_done[k], cs);
@@ -117,6 +119,9 @@ extern "C" FFSVA_API ffsva_status ffsva_filter_batch_host(const ffsva_frame* fra
     ca.seg_lo = b->d_seg_lo;
     ca.n_seg = b->n_seg;
     ca.seg_batch = b->d_seg_batch;
+    ca.seg_slot = b->d_seg_batch + b->cap;
+    ca.stats = ctx->d_stats;
+    ca.snm_ctas = std::max(1, std::min(n, 2 * ctx->num_sms));
     ca.survivor_idx = b->d_surv;
     ca.work = b->d_work;
     ca.posw = b->d_posw;

@@ -59,9 +59,14 @@ struct SddArgs {
   unsigned long long* stats; // [slots][NSTAT] or nullptr
   int32_t max_chunks;        // max over frames of ceil(3W/16)
   bool vec16;                // all frames 16-B aligned with 16-B pitch
+  bool bulk;                 // use the bulk-async (TMA engine) + cluster kernel (partial is then [n][sdd_h])
+  int32_t stage_bytes;       // bulk: shared-memory bytes for one 100-grid row's source rows (max over frames)
 };
 cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st);
 size_t sdd_smem_bytes(int max_chunks, int sdd_w);
+size_t sdd_bulk_smem_bytes(int stage_bytes, int sdd_w);
+int sdd_bulk_stage_bytes(int W, int H, int sdd_h);
+bool sdd_bulk_ok(int max_chunks, int stage_bytes);
 cudaError_t sdd_configure(size_t smem);  // raise the kernels' dynamic smem limit (outside graph capture)
 int sdd_threads(int max_chunks);
 
@@ -72,6 +77,9 @@ struct CompactArgs {
   const int32_t* seg_lo;     // [n_seg + 1] segment boundaries in perm order (one segment per stream)
   int32_t n_seg;
   const int32_t* seg_batch;  // [n_seg] BatchSize of the segment's stream
+  const int32_t* seg_slot;   // [n_seg] stats slot of the segment's stream
+  unsigned long long* stats; // SNM_BATCHES (pops) counted here; may be nullptr
+  int32_t snm_ctas;          // SNM grid size: pops are split into work units of ~m/snm_ctas frames
   int32_t* survivor_idx;     // [n] out
   int32_t* work;             // [n] out: survivors in work order (frame indices)
   int32_t* posw;             // [n + 1] scratch: exclusive survivor count in perm order

@@ -6,6 +6,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 
 namespace ffsva {
@@ -238,11 +239,11 @@ static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t s
   const size_t o_desc = off; off += al(64 * n);
   const size_t o_perm = off; off += al(4 * n);
   const size_t o_seg = off; off += al(4 * (n + 1));
-  const size_t o_segb = off; off += al(4 * n);
+  const size_t o_segb = off; off += al(8 * n);  // seg_batch[cap] then seg_slot[cap]
   b->in_bytes = off;
   const size_t o_d50 = off; off += al((size_t)b->d50_stride * n);
   const size_t o_d100 = off; off += d100 ? al((size_t)3 * sdd_w * sdd_h * n) : 0;
-  const size_t o_part = off; off += al(4 * n * (size_t)(sdd_h / 2));
+  const size_t o_part = off; off += al(4 * n * (size_t)sdd_h);
   const size_t o_cnt = off; off += al(4 * n);
   const size_t o_work = off; off += al(4 * n);
   const size_t o_posw = off; off += al(4 * (n + 1));
@@ -292,7 +293,7 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
   const StreamState* s0 = frames[0].stream;
   const int32_t sdd_w = s0->desc.sdd_w, sdd_h = s0->desc.sdd_h;
   bool vec16 = true;
-  int32_t max_chunks = 1;
+  int32_t max_chunks = 1, stage_bytes = 0;
   for (int32_t i = 0; i < n; ++i) {
     const StreamState* s = frames[i].stream;
     if (s->desc.sdd_w != sdd_w || s->desc.sdd_h != sdd_h)
@@ -302,7 +303,12 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     if (cs != FFSVA_OK) return cs;
     if ((s->desc.row_pitch & 15) || ((uintptr_t)frames[i].pixels & 15)) vec16 = false;
     max_chunks = std::max(max_chunks, (3 * s->desc.width + 15) / 16);
+    stage_bytes = std::max(stage_bytes, sdd_bulk_stage_bytes(s->desc.width, s->desc.height, sdd_h));
   }
+  // K1 variant: the bulk-async/cluster kernel needs 16-B aligned rows that fit the shared-memory stage;
+  // FFSVA_SDD_KERNEL=stream forces the register-streaming kernel (tests exercise both)
+  const char* force = std::getenv("FFSVA_SDD_KERNEL");
+  const bool bulk = vec16 && sdd_bulk_ok(max_chunks, stage_bytes) && !(force && std::strcmp(force, "stream") == 0);
   if (b->cap < n || b->sdd_w != sdd_w || b->sdd_h != sdd_h || (want_d100 && !b->want_d100)) {
     ffsva_status as = batch_alloc(ctx, b, std::max(n, b->cap), sdd_w, sdd_h, want_d100 || b->want_d100);
     if (as != FFSVA_OK) return as;
@@ -311,10 +317,12 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     cudaGraphExecDestroy(b->graph);
     b->graph = nullptr;
   }
-  cudaError_t e = sdd_configure(sdd_smem_bytes(max_chunks, sdd_w));
+  cudaError_t e = sdd_configure(bulk ? sdd_bulk_smem_bytes(stage_bytes, sdd_w) : sdd_smem_bytes(max_chunks, sdd_w));
   if (e != cudaSuccess) return cuda_fail(ctx, e, "sdd_configure");
   b->n = n;
   b->vec16 = vec16;
+  b->bulk = bulk;
+  b->stage_bytes = stage_bytes;
   b->max_chunks = max_chunks;
   b->sdd_only = sdd_only;
   // ---- host staging: descriptors, stream-major permutation, segments
@@ -348,6 +356,7 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     if (k == 0 || hd[hperm[k]].slot != hd[hperm[k - 1]].slot) {
       hseg[nseg] = k;
       hsegb[nseg] = frames[hperm[k]].stream->desc.snm_batch;
+      hsegb[cap + nseg] = frames[hperm[k]].stream->slot;
       ++nseg;
     }
   hseg[nseg] = n;
@@ -377,6 +386,8 @@ static ffsva_status batch_launch_kernels(Batch* b, cudaStream_t st, int* nk, cud
   sa.stats = ctx->d_stats;
   sa.max_chunks = b->max_chunks;
   sa.vec16 = b->vec16;
+  sa.bulk = b->bulk;
+  sa.stage_bytes = b->stage_bytes;
   if (ev) cudaEventRecord(ev[0], st);
   FF_CUDA(ctx, launch_sdd(sa, st));
   if (ev) cudaEventRecord(ev[1], st);
@@ -387,6 +398,9 @@ static ffsva_status batch_launch_kernels(Batch* b, cudaStream_t st, int* nk, cud
   ca.seg_lo = b->d_seg_lo;
   ca.n_seg = b->n_seg;
   ca.seg_batch = b->d_seg_batch;
+  ca.seg_slot = b->d_seg_batch + b->cap;
+  ca.stats = ctx->d_stats;
+  ca.snm_ctas = b->sdd_only ? 0 : std::max(1, std::min(b->n, 2 * ctx->num_sms));
   ca.survivor_idx = b->d_surv;
   ca.work = b->d_work;
   ca.posw = b->d_posw;

@@ -37,6 +37,8 @@ struct Batch {
   int32_t n = 0, cap = 0;
   int32_t sdd_w = 0, sdd_h = 0, max_chunks = 0, n_seg = 0;
   bool vec16 = true, sdd_only = false, want_d100 = false;
+  bool bulk = false;          // K1 variant: bulk-async + cluster (aligned frames) or register streaming
+  int32_t stage_bytes = 0;
   int64_t d50_stride = 0;
   // device buffers (carved from one allocation)
   void* d_mem = nullptr;

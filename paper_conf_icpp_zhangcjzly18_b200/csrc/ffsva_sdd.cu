@@ -15,7 +15,11 @@
 // row of D50, and a partial SSD; the last CTA of a frame (ticket counter, self-resetting) adds the partials
 // in u64, applies the threshold and updates the per-stream stats. HBM traffic = the raw frame bytes once +
 // 7.5 KB of D50 (+ 30 KB of D100 when requested) per frame.
+#include <cooperative_groups.h>
+
 #include "ffsva_internal.h"
+
+namespace cg = cooperative_groups;
 
 namespace ffsva {
 namespace {
@@ -171,6 +175,175 @@ __global__ void __launch_bounds__(512) sdd_kernel(SddArgs a) {
   }
 }
 
+// ------------------------------------------------------------------ bulk-async (TMA engine) variant
+// One CTA per (frame, 100-grid row); the two CTAs of a 50-grid row form a thread-block cluster.
+//   1. one thread arms an mbarrier with the row's byte count and issues cp.async.bulk copies (TMA engine,
+//      L2 evict-first) of the row's source rows into shared memory — the SM's whole share of the frame is in
+//      flight at once and no register is tied up waiting for it;
+//   2. column sums from shared memory (16-byte LDS, packed 2x16-bit SIMD adds), 100-grid cell sums, D100,
+//      SSD against R;
+//   3. the odd CTA of the pair pushes its 2-cell horizontal sums into the even CTA's shared memory (DSMEM)
+//      and the cluster barrier publishes them; the even CTA emits the D50 row from the four 100-cell sums;
+//   4. per-frame SSD partials + ticket, as in the fallback kernel.
+__device__ __forceinline__ void mbar_init_cta(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_parity(uint32_t bar, uint32_t parity) {
+  uint32_t done = 0;
+  while (!done) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}\n"
+        : "=r"(done)
+        : "r"(bar), "r"(parity)
+        : "memory");
+  }
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar, uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::
+          "r"(dst),
+      "l"(src), "r"(bytes), "r"(bar), "l"(pol)
+      : "memory");
+}
+
+constexpr int kBulkThreads = 256;
+constexpr int kBulkMaxStage = 160 * 1024;  // larger rows (e.g. 4K) take the register-streaming kernel
+
+template <bool kD100>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads) sdd_bulk_kernel(SddArgs a) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ __align__(8) uint64_t bar;
+  __shared__ uint32_t red[kBulkThreads / 32];
+  __shared__ int s_last;
+  cg::cluster_group cluster = cg::this_cluster();
+  const int sdd_w = a.sdd_w, sdd_h = a.sdd_h;
+  const int f = blockIdx.x / sdd_h;
+  const int r = blockIdx.x - f * sdd_h;  // 100-grid row; the cluster pairs rows 2b and 2b+1
+  const unsigned rank = cluster.block_rank();
+  const FrameDesc fd = a.frames[f];
+  const int W = fd.W, H = fd.H;
+  const int rb16 = (3 * W + 15) & ~15;
+  const int nchunk = rb16 >> 4;
+  const int y0 = (int)(((int64_t)r * H) / sdd_h), y1 = (int)(((int64_t)(r + 1) * H) / sdd_h);
+  const int rows = y1 - y0;
+  uint32_t* cell = reinterpret_cast<uint32_t*>(smem + a.stage_bytes);            // [3*sdd_w]
+  uint32_t* pair_in = cell + 3 * sdd_w;                                           // [3*sdd_w/2]
+  const uint32_t bar_a = (uint32_t)__cvta_generic_to_shared(&bar);
+
+  if (threadIdx.x == 0) {
+    mbar_init_cta(bar_a, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    mbar_expect_tx(bar_a, (uint32_t)(rows * rb16));
+    const uint32_t dst = (uint32_t)__cvta_generic_to_shared(smem);
+    const uint8_t* src = fd.pixels + (int64_t)y0 * fd.pitch;
+    if (fd.pitch == rb16) {
+      bulk_g2s(dst, src, (uint32_t)(rows * rb16), bar_a, pol);
+    } else {
+      for (int y = 0; y < rows; ++y) bulk_g2s(dst + y * rb16, src + (int64_t)y * fd.pitch, (uint32_t)rb16, bar_a, pol);
+    }
+  }
+  __syncthreads();
+  mbar_wait_parity(bar_a, 0);
+
+  // ---- column sums of the row's source rows (<= 2 16-byte chunks per thread)
+  uint32_t acc[2][8];
+#pragma unroll
+  for (int k = 0; k < 2; ++k) {
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[k][j] = 0u;
+    const int c = threadIdx.x + k * kBulkThreads;
+    if (c < nchunk)
+      for (int y = 0; y < rows; ++y) acc16(acc[k], *reinterpret_cast<const uint4*>(smem + y * rb16 + 16 * c));
+  }
+  __syncthreads();  // the stage is consumed; its first 2*rb16 bytes now hold the u16 column sums
+  uint16_t* colsum = reinterpret_cast<uint16_t*>(smem);
+#pragma unroll
+  for (int k = 0; k < 2; ++k) {
+    const int c = threadIdx.x + k * kBulkThreads;
+    if (c < nchunk) store_colsum(reinterpret_cast<uint32_t*>(colsum), c, acc[k]);
+  }
+  __syncthreads();
+
+  // ---- 100-grid cells of this row: D100, SSD vs R
+  const int row3 = 3 * sdd_w;
+  uint32_t ssd_local = 0;
+  for (int o = threadIdx.x; o < row3; o += kBulkThreads) {
+    const int cx = o / 3, ch = o - 3 * cx;
+    const int x0 = (int)(((int64_t)cx * W) / sdd_w), x1 = (int)(((int64_t)(cx + 1) * W) / sdd_w);
+    uint32_t s = 0;
+    for (int x = x0; x < x1; ++x) s += colsum[3 * x + ch];
+    cell[o] = s;
+    const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)rows;
+    const uint32_t d = (s + (n >> 1)) / n;
+    if (kD100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)r * row3 + o] = (uint8_t)d;
+    const int diff = (int)d - (int)__ldg(fd.ref + (int64_t)r * row3 + o);
+    ssd_local += (uint32_t)(diff * diff);
+  }
+  __syncthreads();
+
+  // ---- D50 row: odd CTA -> even CTA over DSMEM, then the even CTA combines the 2x2 cells
+  const int half3 = 3 * (sdd_w >> 1);
+  if (rank == 1) {
+    uint32_t* remote = cluster.map_shared_rank(pair_in, 0);
+    for (int o = threadIdx.x; o < half3; o += kBulkThreads) {
+      const int cx = o / 3, ch = o - 3 * cx;
+      remote[o] = cell[6 * cx + ch] + cell[6 * cx + 3 + ch];
+    }
+  }
+  cluster.sync();
+  if (rank == 0) {
+    const int yb = (int)(((int64_t)(r + 2) * H) / sdd_h);
+    for (int o = threadIdx.x; o < half3; o += kBulkThreads) {
+      const int cx = o / 3, ch = o - 3 * cx;
+      const uint32_t s = cell[6 * cx + ch] + cell[6 * cx + 3 + ch] + pair_in[o];
+      const int x0 = (int)(((int64_t)(2 * cx) * W) / sdd_w), x1 = (int)(((int64_t)(2 * cx + 2) * W) / sdd_w);
+      const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)(yb - y0);
+      a.d50[(int64_t)f * a.d50_stride + (int64_t)(r >> 1) * half3 + o] = (uint8_t)((s + (n >> 1)) / n);
+    }
+  }
+
+  // ---- SSD partial of this row, frame ticket, last CTA finalises
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) ssd_local += __shfl_xor_sync(0xffffffffu, ssd_local, off);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) red[warp] = ssd_local;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t t = 0;
+#pragma unroll
+    for (int w = 0; w < kBulkThreads / 32; ++w) t += red[w];
+    a.partial[(int64_t)f * sdd_h + r] = t;
+    __threadfence();
+    const unsigned ticket = atomicAdd(a.counter + f, 1u);
+    s_last = (ticket == (unsigned)(sdd_h - 1));
+  }
+  __syncthreads();
+  if (s_last && warp == 0) {
+    __threadfence();
+    unsigned long long sum = 0;
+    for (int b = lane; b < sdd_h; b += 32) sum += __ldcg(a.partial + (int64_t)f * sdd_h + b);
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, off);
+    if (lane == 0) {
+      const uint8_t p = sum > fd.T ? 1 : 0;
+      a.ssd[f] = sum;
+      a.pass[f] = p;
+      a.counter[f] = 0u;
+      if (a.stats) {
+        unsigned long long* st = a.stats + (int64_t)fd.slot * NSTAT;
+        atomicAdd(st + 0, 1ull);
+        atomicAdd(st + 1, (unsigned long long)p);
+        atomicAdd(st + 3, sum);
+      }
+    }
+  }
+}
+
 // Reference image R: one rounding of the mean over k frames x box. One thread per value.
 __global__ void reference_kernel(const uint8_t* __restrict__ frames, int32_t k, int64_t frame_stride, int32_t W,
                                  int32_t H, int64_t pitch, int32_t sdd_w, int32_t sdd_h, uint8_t* __restrict__ out) {
@@ -205,18 +378,44 @@ int sdd_threads(int max_chunks) {
   return t;
 }
 
+size_t sdd_bulk_smem_bytes(int stage_bytes, int sdd_w) {
+  return (size_t)stage_bytes + (size_t)4 * (3 * sdd_w + 3 * (sdd_w / 2));
+}
+
+int sdd_bulk_stage_bytes(int W, int H, int sdd_h) {
+  const int rb16 = (3 * W + 15) & ~15;
+  int rows = (H + sdd_h - 1) / sdd_h;  // max source rows of one 100-grid row
+  if (rows < 2) rows = 2;              // the stage also holds the 2*rb16-byte column sums
+  return rows * rb16;
+}
+
+bool sdd_bulk_ok(int max_chunks, int stage_bytes) {
+  return max_chunks <= 2 * kBulkThreads && stage_bytes <= kBulkMaxStage;
+}
+
 cudaError_t sdd_configure(size_t smem) {
   static size_t configured = 0;
   if (smem <= configured) return cudaSuccess;
   cudaError_t e = cudaFuncSetAttribute(sdd_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(sdd_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(sdd_bulk_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(sdd_bulk_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e == cudaSuccess) configured = smem;
   return e;
 }
 
 cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st) {
   if (a.n <= 0) return cudaSuccess;
+  if (a.bulk) {
+    const size_t smem = sdd_bulk_smem_bytes(a.stage_bytes, a.sdd_w);
+    const unsigned grid = (unsigned)a.n * (unsigned)a.sdd_h;
+    if (a.d100) sdd_bulk_kernel<true><<<grid, kBulkThreads, smem, st>>>(a);
+    else sdd_bulk_kernel<false><<<grid, kBulkThreads, smem, st>>>(a);
+    return cudaGetLastError();
+  }
   const size_t smem = sdd_smem_bytes(a.max_chunks, a.sdd_w);
   const int threads = sdd_threads(a.max_chunks);
   const unsigned grid = (unsigned)a.n * (unsigned)(a.sdd_h / 2);

@@ -341,7 +341,6 @@ __global__ void __launch_bounds__(kThreads, 2) snm_kernel(SnmArgs a) {
       atomicAdd(st + 4, (unsigned long long)cnt_c0);
       atomicAdd(st + 5, (unsigned long long)cnt_c1);
       atomicAdd(st + 6, (unsigned long long)cnt_c2);
-      atomicAdd(st + 7, 1ull);
     }
     __syncthreads();
   }
