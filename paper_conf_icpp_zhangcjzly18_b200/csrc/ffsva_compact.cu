@@ -70,13 +70,22 @@ __global__ void __launch_bounds__(kThreads) compact_kernel(CompactArgs a) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int n = a.n;
 
-  // ---------------- pass 1: ranks in input order
+  // ---------------- pass 1: SDD threshold (L151: MSE > delta_diff <=> SSD > T) and ranks in input order
   int carry = 0;
   for (int base = 0; base < n; base += 4 * kThreads) {
     const int i0 = base + 4 * threadIdx.x;
     bool f[4];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) f[j] = (i0 + j < n) && a.pass[i0 + j];
+    for (int j = 0; j < 4; ++j) {
+      f[j] = false;
+      if (i0 + j < n) {
+        const unsigned long long s = a.acc_ssd[i0 + j];
+        f[j] = s > a.frames[i0 + j].T;
+        a.ssd[i0 + j] = s;
+        a.pass[i0 + j] = f[j] ? 1 : 0;
+        a.acc_ssd[i0 + j] = 0ull;  // ready for the next launch of this batch
+      }
+    }
     int wtot;
     const int wr = warp_rank4(f, &wtot);
     if (lane == 0) s_wbase[warp] = wtot;
@@ -164,7 +173,11 @@ __global__ void __launch_bounds__(kThreads) compact_kernel(CompactArgs a) {
       B = a.seg_batch[s];
       U = a.snm_ctas > 0 ? m_all / a.snm_ctas : B;
       U = U < 1 ? 1 : (U > B ? B : U);
-      if (a.stats && q > 0) atomicAdd(a.stats + (int64_t)a.seg_slot[s] * NSTAT + 7, (unsigned long long)((q + B - 1) / B));
+      if (a.stats && q > 0) {
+        unsigned long long* st = a.stats + (int64_t)a.seg_slot[s] * NSTAT;
+        atomicAdd(st + 1, (unsigned long long)q);                    // SDD survivors
+        if (a.snm_ctas > 0) atomicAdd(st + 7, (unsigned long long)((q + B - 1) / B));  // dynamic batches
+      }
     }
     const int full = q / B, rest = q - full * B;
     const int per_full = (B + U - 1) / U;

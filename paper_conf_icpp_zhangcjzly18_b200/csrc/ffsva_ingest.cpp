@@ -71,7 +71,7 @@ extern "C" FFSVA_API ffsva_status ffsva_filter_batch_host(const ffsva_frame* fra
   cudaEventRecord(ev_done[0], cs);
   cudaEventRecord(ev_done[1], cs);
   const int nchunks = (n + kChunk - 1) / kChunk;
-  const int nb = b->sdd_h / 2;
+
   st = FFSVA_OK;
   for (int c = 0; c < nchunks && st == FFSVA_OK; ++c) {
     const int k = c & 1, i0 = c * kChunk, cnt = std::min(kChunk, n - i0);
@@ -89,61 +89,14 @@ extern "C" FFSVA_API ffsva_status ffsva_filter_batch_host(const ffsva_frame* fra
     if (st != FFSVA_OK) break;
     cudaEventRecord(ev_copy[k], ctx->copy_stream);
     cudaStreamWaitEvent(cs, ev_copy[k], 0);
-    SddArgs sa{};
-    sa.frames = b->d_desc + i0;
-    sa.n = cnt;
-    sa.sdd_w = b->sdd_w;
-    sa.sdd_h = b->sdd_h;
-    sa.d50 = b->d_d50 + (size_t)i0 * b->d50_stride;
-    sa.d50_stride = b->d50_stride;
-    sa.d100 = nullptr;
-    sa.partial = b->d_partial + (size_t)i0 * 2 * nb;
-    sa.counter = b->d_counter + i0;
-    sa.ssd = b->d_ssd + i0;
-    sa.pass = b->d_pass + i0;
-    sa.stats = ctx->d_stats;
-    sa.max_chunks = b->max_chunks;
-    sa.vec16 = b->vec16;
-    sa.bulk = b->bulk;
-    sa.stage_bytes = b->stage_bytes;
-    if ((e = launch_sdd(sa, cs)) != cudaSuccess) st = cuda_fail(ctx, e, "launch_sdd");
+    if ((e = launch_sdd(make_sdd_args(b, i0, cnt), cs)) != cudaSuccess) st = cuda_fail(ctx, e, "launch_sdd");
     g_launches += 1;
     cudaEventRecord(ev_done[k], cs);
   }
   if (st == FFSVA_OK) {
-    // K3 + K4 over the whole batch (run the prepared batch minus its SDD stage)
-    CompactArgs ca{};
-    ca.pass = b->d_pass;
-    ca.n = n;
-    ca.perm = b->d_perm;
-    ca.seg_lo = b->d_seg_lo;
-    ca.n_seg = b->n_seg;
-    ca.seg_batch = b->d_seg_batch;
-    ca.seg_slot = b->d_seg_batch + b->cap;
-    ca.stats = ctx->d_stats;
-    ca.snm_ctas = std::max(1, std::min(n, 2 * ctx->num_sms));
-    ca.survivor_idx = b->d_surv;
-    ca.work = b->d_work;
-    ca.posw = b->d_posw;
-    ca.chunks = b->d_chunks;
-    ca.counts = b->d_counts;
-    ca.logit = b->d_logit;
-    ca.snm_pass = b->d_snm_pass;
-    ca.snm_class = b->d_snm_class;
-    if ((e = launch_compact(ca, cs)) != cudaSuccess) st = cuda_fail(ctx, e, "launch_compact");
-    SnmArgs na{};
-    na.frames = b->d_desc;
-    na.d50 = b->d_d50;
-    na.d50_stride = b->d50_stride;
-    na.work = b->d_work;
-    na.chunks = b->d_chunks;
-    na.counts = b->d_counts;
-    na.logit = b->d_logit;
-    na.snm_pass = b->d_snm_pass;
-    na.snm_class = b->d_snm_class;
-    na.stats = ctx->d_stats;
-    na.grid = std::max(1, std::min(n, 2 * ctx->num_sms));
-    if (st == FFSVA_OK && (e = launch_snm(na, cs)) != cudaSuccess) st = cuda_fail(ctx, e, "launch_snm");
+    // K3 + K4 over the whole batch (they only touch the 7.5 KB D50 images, not the staged frames)
+    if ((e = launch_compact(make_compact_args(b), cs)) != cudaSuccess) st = cuda_fail(ctx, e, "launch_compact");
+    if (st == FFSVA_OK && (e = launch_snm(make_snm_args(b), cs)) != cudaSuccess) st = cuda_fail(ctx, e, "launch_snm");
     g_launches += 2;
   }
   if (st == FFSVA_OK) st = batch_fetch(b, results, cs);

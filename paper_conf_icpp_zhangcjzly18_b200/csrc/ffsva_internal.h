@@ -52,14 +52,11 @@ struct SddArgs {
   uint8_t* d50;              // [n][d50_stride]
   int64_t d50_stride;
   uint8_t* d100;             // optional [n][sdd_h*sdd_w*3]
-  uint32_t* partial;         // [n][sdd_h/2]
-  uint32_t* counter;         // [n], zero on entry, left zero
-  uint64_t* ssd;             // [n]
-  uint8_t* pass;             // [n]
+  unsigned long long* acc_ssd; // [n] per-frame SSD accumulator: zero on entry; K3 reads it and re-zeroes it
   unsigned long long* stats; // [slots][NSTAT] or nullptr
   int32_t max_chunks;        // max over frames of ceil(3W/16)
   bool vec16;                // all frames 16-B aligned with 16-B pitch
-  bool bulk;                 // use the bulk-async (TMA engine) + cluster kernel (partial is then [n][sdd_h])
+  bool bulk;                 // use the bulk-async (TMA engine) + cluster kernel
   int32_t stage_bytes;       // bulk: shared-memory bytes for one 100-grid row's source rows (max over frames)
 };
 cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st);
@@ -71,7 +68,10 @@ cudaError_t sdd_configure(size_t smem);  // raise the kernels' dynamic smem limi
 int sdd_threads(int max_chunks);
 
 struct CompactArgs {
-  const uint8_t* pass;       // [n] frame order
+  const FrameDesc* frames;   // [n] (threshold T per frame)
+  unsigned long long* acc_ssd; // [n] K1's SSD accumulators (read, then re-zeroed for the next launch)
+  uint64_t* ssd;             // [n] out
+  uint8_t* pass;             // [n] out: SSD > T
   int32_t n;
   const int32_t* perm;       // [n] work (stream-major, stable) order -> frame index
   const int32_t* seg_lo;     // [n_seg + 1] segment boundaries in perm order (one segment per stream)

@@ -243,8 +243,7 @@ static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t s
   b->in_bytes = off;
   const size_t o_d50 = off; off += al((size_t)b->d50_stride * n);
   const size_t o_d100 = off; off += d100 ? al((size_t)3 * sdd_w * sdd_h * n) : 0;
-  const size_t o_part = off; off += al(4 * n * (size_t)sdd_h);
-  const size_t o_cnt = off; off += al(4 * n);
+  const size_t o_acc = off; off += al(8 * n);
   const size_t o_work = off; off += al(4 * n);
   const size_t o_posw = off; off += al(4 * (n + 1));
   const size_t o_chunks = off; off += al(4 * (n + 1));
@@ -262,8 +261,7 @@ static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t s
   b->d_seg_batch = (int32_t*)(base + o_segb);
   b->d_d50 = base + o_d50;
   b->d_d100 = d100 ? base + o_d100 : nullptr;
-  b->d_partial = (uint32_t*)(base + o_part);
-  b->d_counter = (uint32_t*)(base + o_cnt);
+  b->d_acc = (unsigned long long*)(base + o_acc);
   b->d_work = (int32_t*)(base + o_work);
   b->d_posw = (int32_t*)(base + o_posw);
   b->d_chunks = (int32_t*)(base + o_chunks);
@@ -276,7 +274,7 @@ static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t s
   b->d_snm_pass = b->d_out + 17 * n;
   b->d_snm_class = b->d_out + 18 * n;
   b->out_bytes = out_bytes;
-  if ((e = cudaMemset(b->d_counter, 0, 4 * n)) != cudaSuccess) return cuda_fail(ctx, e, "cudaMemset(counter)");
+  if ((e = cudaMemset(b->d_acc, 0, 8 * n)) != cudaSuccess) return cuda_fail(ctx, e, "cudaMemset(acc_ssd)");
   if ((e = cudaMemset(b->d_counts, 0, 16)) != cudaSuccess) return cuda_fail(ctx, e, "cudaMemset(counts)");
   if ((e = cudaMallocHost(&b->h_in, b->in_bytes)) != cudaSuccess) return cuda_fail(nullptr, e, "cudaMallocHost");
   if ((e = cudaMallocHost(&b->h_out, out_bytes)) != cudaSuccess) return cuda_fail(nullptr, e, "cudaMallocHost");
@@ -369,29 +367,30 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
   return FFSVA_OK;
 }
 
-static ffsva_status batch_launch_kernels(Batch* b, cudaStream_t st, int* nk, cudaEvent_t* ev = nullptr) {
-  DeviceCtx* ctx = b->ctx;
+SddArgs make_sdd_args(Batch* b, int32_t i0, int32_t cnt) {
   SddArgs sa{};
-  sa.frames = b->d_desc;
-  sa.n = b->n;
+  sa.frames = b->d_desc + i0;
+  sa.n = cnt;
   sa.sdd_w = b->sdd_w;
   sa.sdd_h = b->sdd_h;
-  sa.d50 = b->d_d50;
+  sa.d50 = b->d_d50 + (size_t)i0 * b->d50_stride;
   sa.d50_stride = b->d50_stride;
-  sa.d100 = b->want_d100 ? b->d_d100 : nullptr;
-  sa.partial = b->d_partial;
-  sa.counter = b->d_counter;
-  sa.ssd = b->d_ssd;
-  sa.pass = b->d_pass;
-  sa.stats = ctx->d_stats;
+  sa.d100 = b->want_d100 ? b->d_d100 + (size_t)i0 * 3 * b->sdd_w * b->sdd_h : nullptr;
+  sa.acc_ssd = b->d_acc + i0;
+  sa.stats = b->ctx->d_stats;
   sa.max_chunks = b->max_chunks;
   sa.vec16 = b->vec16;
   sa.bulk = b->bulk;
   sa.stage_bytes = b->stage_bytes;
-  if (ev) cudaEventRecord(ev[0], st);
-  FF_CUDA(ctx, launch_sdd(sa, st));
-  if (ev) cudaEventRecord(ev[1], st);
+  return sa;
+}
+
+CompactArgs make_compact_args(Batch* b) {
+  DeviceCtx* ctx = b->ctx;
   CompactArgs ca{};
+  ca.frames = b->d_desc;
+  ca.acc_ssd = b->d_acc;
+  ca.ssd = b->d_ssd;
   ca.pass = b->d_pass;
   ca.n = b->n;
   ca.perm = b->d_perm;
@@ -409,23 +408,35 @@ static ffsva_status batch_launch_kernels(Batch* b, cudaStream_t st, int* nk, cud
   ca.logit = b->d_logit;
   ca.snm_pass = b->d_snm_pass;
   ca.snm_class = b->d_snm_class;
-  FF_CUDA(ctx, launch_compact(ca, st));
+  return ca;
+}
+
+SnmArgs make_snm_args(Batch* b) {
+  SnmArgs na{};
+  na.frames = b->d_desc;
+  na.d50 = b->d_d50;
+  na.d50_stride = b->d50_stride;
+  na.work = b->d_work;
+  na.chunks = b->d_chunks;
+  na.counts = b->d_counts;
+  na.logit = b->d_logit;
+  na.snm_pass = b->d_snm_pass;
+  na.snm_class = b->d_snm_class;
+  na.stats = b->ctx->d_stats;
+  na.grid = std::max(1, std::min(b->n, 2 * b->ctx->num_sms));
+  return na;
+}
+
+static ffsva_status batch_launch_kernels(Batch* b, cudaStream_t st, int* nk, cudaEvent_t* ev = nullptr) {
+  DeviceCtx* ctx = b->ctx;
+  if (ev) cudaEventRecord(ev[0], st);
+  FF_CUDA(ctx, launch_sdd(make_sdd_args(b, 0, b->n), st));
+  if (ev) cudaEventRecord(ev[1], st);
+  FF_CUDA(ctx, launch_compact(make_compact_args(b), st));
   if (ev) cudaEventRecord(ev[2], st);
   *nk = 2;
   if (!b->sdd_only) {
-    SnmArgs na{};
-    na.frames = b->d_desc;
-    na.d50 = b->d_d50;
-    na.d50_stride = b->d50_stride;
-    na.work = b->d_work;
-    na.chunks = b->d_chunks;
-    na.counts = b->d_counts;
-    na.logit = b->d_logit;
-    na.snm_pass = b->d_snm_pass;
-    na.snm_class = b->d_snm_class;
-    na.stats = ctx->d_stats;
-    na.grid = std::max(1, std::min(b->n, 2 * ctx->num_sms));
-    FF_CUDA(ctx, launch_snm(na, st));
+    FF_CUDA(ctx, launch_snm(make_snm_args(b), st));
     *nk = 3;
   }
   if (ev) cudaEventRecord(ev[3], st);

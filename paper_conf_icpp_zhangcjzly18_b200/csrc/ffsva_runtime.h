@@ -47,7 +47,7 @@ struct Batch {
   int32_t *d_perm = nullptr, *d_seg_lo = nullptr, *d_seg_batch = nullptr;
   uint8_t* d_d50 = nullptr;
   uint8_t* d_d100 = nullptr;
-  uint32_t *d_partial = nullptr, *d_counter = nullptr;
+  unsigned long long* d_acc = nullptr;  // per-frame SSD accumulators (K1 adds, K3 reads + re-zeroes)
   int32_t *d_work = nullptr, *d_posw = nullptr, *d_chunks = nullptr, *d_counts = nullptr;
   // output block (one D2H): ssd u64[n] | logit f32[n] | survivor_idx i32[n] | sdd_pass u8[n] | snm_pass u8[n] |
   // snm_class u8[n]
@@ -104,6 +104,9 @@ ffsva_status batch_run(Batch* b, cudaStream_t st, bool use_graph);
 ffsva_status batch_fetch(Batch* b, ffsva_result* results, cudaStream_t st);
 ffsva_status batch_profile(Batch* const* batches, int32_t nb, int32_t iters, float* ms_out, cudaStream_t st);
 void batch_free(Batch* b);
+SddArgs make_sdd_args(Batch* b, int32_t i0, int32_t cnt);  // K1 over frames [i0, i0 + cnt) of the batch
+CompactArgs make_compact_args(Batch* b);
+SnmArgs make_snm_args(Batch* b);
 
 // RAII device switch
 struct DeviceGuard {

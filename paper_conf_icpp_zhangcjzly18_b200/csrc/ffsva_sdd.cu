@@ -1,5 +1,6 @@
-// ffsva_sdd.cu — K1: frame ingest + integer box downsample (D100 and D50 in one pass) + SDD distance and
-// threshold, for many frames of many streams in one launch.
+// ffsva_sdd.cu — K1: frame ingest + integer box downsample (D100 and D50 in one pass) + SDD distance, for many
+// frames of many streams in one launch. (The threshold of the summed distance happens in K3, after the kernel
+// boundary has made every partial sum visible — no grid-scope fences here.)
 //
 // Method: raw frames are resized to each filter's feature size before the filter runs (L187;
 // SDD 100x100 L155, SNM 50x50 L167); SDD computes the distance of the 100x100 image to the stream's
@@ -7,14 +8,18 @@
 // box filter with round-half-up (Q1, Q2), RGB kept (Q3), SSD in integers with an exact threshold (Q4, Q5),
 // D50 from the raw frame = union of 2x2 D100 cells (Q8).
 //
-// B200 mapping. One CTA per (frame, 50-grid row band) = two 100-grid rows of source pixels. The band is a set
-// of whole source rows, streamed once from HBM with coalesced 16-byte non-allocating loads (each warp load
-// covers 512 contiguous bytes of a row); up to 8 rows are in flight per thread before any arithmetic.
-// Column sums are kept as packed 2x16-bit SIMD lanes in registers (1.25 integer ops per byte), written once
-// to shared memory, then summed per cell. Each CTA emits 2 rows of D100 cells (SSD against R from L2), one
-// row of D50, and a partial SSD; the last CTA of a frame (ticket counter, self-resetting) adds the partials
-// in u64, applies the threshold and updates the per-stream stats. HBM traffic = the raw frame bytes once +
-// 7.5 KB of D50 (+ 30 KB of D100 when requested) per frame.
+// Two variants, chosen per batch by the host:
+//  * sdd_bulk_kernel (rows 16-B aligned, one 100-grid row fits in shared memory — every workload of the
+//    benchmark): one CTA per (frame, 100-grid row), CTA pairs form thread-block clusters. One thread issues
+//    cp.async.bulk copies (TMA engine, L2 evict-first) of the row's source rows into shared memory against an
+//    mbarrier, so the SM's whole share of the frame is in flight without tying up registers; column sums are
+//    packed 2x16-bit SIMD adds of 16-byte shared loads; the odd CTA of a pair pushes its horizontal 2-cell sums
+//    into the even CTA's shared memory with st.async (DSMEM, mbarrier transaction completion, no fence) and
+//    the even CTA emits the D50 row from the four 100-cell sums.
+//  * sdd_kernel (any alignment / very wide rows): one CTA per (frame, 50-grid row), rows streamed straight to
+//    registers with 16-byte non-allocating loads (or byte loads for unaligned rows), 8 rows in flight.
+// Both add their row's squared-difference sum to a per-frame u64 accumulator (relaxed atomic) and count the
+// frame in the per-stream statistics.
 #include <cooperative_groups.h>
 
 #include "ffsva_internal.h"
@@ -64,6 +69,31 @@ __device__ __forceinline__ void store_colsum(uint32_t* colw, int c, const uint32
   reinterpret_cast<uint4*>(colw)[2 * c + 1] = hi;
 }
 
+// x boundaries of the 100-grid cells of a W-pixel row: xb[i] = floor(i*W/sdd_w), i = 0..sdd_w.
+__device__ __forceinline__ void fill_xbounds(int* xb, int W, int sdd_w) {
+  for (int i = threadIdx.x; i <= sdd_w; i += blockDim.x) xb[i] = (int)(((uint32_t)i * (uint32_t)W) / (uint32_t)sdd_w);
+}
+
+// Block-reduce this thread's SSD share; thread 0 adds it to the frame's accumulator and the stream's stats.
+__device__ __forceinline__ void ssd_commit(uint32_t v, uint32_t* red, const SddArgs& a, int f, int slot,
+                                           bool count_frame) {
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = v;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long t = 0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += red[w];
+    atomicAdd(a.acc_ssd + f, t);
+    if (a.stats) {
+      unsigned long long* st = a.stats + (int64_t)slot * NSTAT;
+      atomicAdd(st + 3, t);
+      if (count_frame) atomicAdd(st + 0, 1ull);
+    }
+  }
+}
+
+// ------------------------------------------------------------------ register-streaming variant
 template <bool kD100>
 __global__ void __launch_bounds__(512) sdd_kernel(SddArgs a) {
   extern __shared__ __align__(16) uint8_t smem[];
@@ -77,14 +107,15 @@ __global__ void __launch_bounds__(512) sdd_kernel(SddArgs a) {
   const int cs = nchunk * 16;  // u16 column sums per 100-grid row
   uint16_t* colsum = reinterpret_cast<uint16_t*>(smem);                  // [2][cs]
   uint32_t* cell = reinterpret_cast<uint32_t*>(smem + 4 * (size_t)cs);   // [2][3*sdd_w]
-  __shared__ uint32_t red[32];
-  __shared__ int s_last;
+  int* xb = reinterpret_cast<int*>(cell + 6 * sdd_w);                    // [sdd_w + 1]
+  __shared__ uint32_t red[16];
 
   // Source rows of the two 100-grid rows of this band: [ya0, ya1) and [ya1, yb1).
   const int ya0 = (int)(((int64_t)(2 * band) * H) / sdd_h);
   const int ya1 = (int)(((int64_t)(2 * band + 1) * H) / sdd_h);
   const int yb1 = (int)(((int64_t)(2 * band + 2) * H) / sdd_h);
   const int rows = yb1 - ya0, split = ya1 - ya0;
+  fill_xbounds(xb, W, sdd_w);
 
   // ---- phase 1: stream the band's rows, vertical column sums in registers
   for (int c = threadIdx.x; c < nchunk; c += blockDim.x) {
@@ -114,7 +145,7 @@ __global__ void __launch_bounds__(512) sdd_kernel(SddArgs a) {
     const int sub = o >= row3;
     const int r = o - sub * row3;
     const int cx = r / 3, ch = r - 3 * cx;
-    const int x0 = (int)(((int64_t)cx * W) / sdd_w), x1 = (int)(((int64_t)(cx + 1) * W) / sdd_w);
+    const int x0 = xb[cx], x1 = xb[cx + 1];
     const uint16_t* col = colsum + sub * cs + ch;
     uint32_t s = 0;
     for (int x = x0; x < x1; ++x) s += col[3 * x];
@@ -134,57 +165,13 @@ __global__ void __launch_bounds__(512) sdd_kernel(SddArgs a) {
     const int cx = o / 3, ch = o - 3 * cx;
     const uint32_t s = cell[6 * cx + ch] + cell[6 * cx + 3 + ch] + cell[row3 + 6 * cx + ch] +
                        cell[row3 + 6 * cx + 3 + ch];
-    const int x0 = (int)(((int64_t)(2 * cx) * W) / sdd_w), x1 = (int)(((int64_t)(2 * cx + 2) * W) / sdd_w);
-    const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)rows;
+    const uint32_t n = (uint32_t)(xb[2 * cx + 2] - xb[2 * cx]) * (uint32_t)rows;
     a.d50[(int64_t)f * a.d50_stride + (int64_t)band * half3 + o] = (uint8_t)((s + (n >> 1)) / n);
   }
-
-  // ---- block SSD partial, then the frame's last CTA finalises
-#pragma unroll
-  for (int off = 16; off > 0; off >>= 1) ssd_local += __shfl_xor_sync(0xffffffffu, ssd_local, off);
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  if (lane == 0) red[warp] = ssd_local;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    uint32_t t = 0;
-    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += red[w];
-    a.partial[(int64_t)f * nb + band] = t;
-    __threadfence();
-    const unsigned ticket = atomicAdd(a.counter + f, 1u);
-    s_last = (ticket == (unsigned)(nb - 1));
-  }
-  __syncthreads();
-  if (s_last && warp == 0) {
-    __threadfence();
-    unsigned long long sum = 0;
-    for (int b = lane; b < nb; b += 32) sum += __ldcg(a.partial + (int64_t)f * nb + b);
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, off);
-    if (lane == 0) {
-      const uint8_t p = sum > fd.T ? 1 : 0;
-      a.ssd[f] = sum;
-      a.pass[f] = p;
-      a.counter[f] = 0u;
-      if (a.stats) {  // a8: per-stream counters
-        unsigned long long* st = a.stats + (int64_t)fd.slot * NSTAT;
-        atomicAdd(st + 0, 1ull);
-        atomicAdd(st + 1, (unsigned long long)p);
-        atomicAdd(st + 3, sum);
-      }
-    }
-  }
+  ssd_commit(ssd_local, red, a, f, fd.slot, band == 0);
 }
 
-// ------------------------------------------------------------------ bulk-async (TMA engine) variant
-// One CTA per (frame, 100-grid row); the two CTAs of a 50-grid row form a thread-block cluster.
-//   1. one thread arms an mbarrier with the row's byte count and issues cp.async.bulk copies (TMA engine,
-//      L2 evict-first) of the row's source rows into shared memory — the SM's whole share of the frame is in
-//      flight at once and no register is tied up waiting for it;
-//   2. column sums from shared memory (16-byte LDS, packed 2x16-bit SIMD adds), 100-grid cell sums, D100,
-//      SSD against R;
-//   3. the odd CTA of the pair pushes its 2-cell horizontal sums into the even CTA's shared memory (DSMEM)
-//      and the cluster barrier publishes them; the even CTA emits the D50 row from the four 100-cell sums;
-//   4. per-frame SSD partials + ticket, as in the fallback kernel.
+// ------------------------------------------------------------------ bulk-async (TMA engine) + cluster variant
 __device__ __forceinline__ void mbar_init_cta(uint32_t bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
 }
@@ -208,6 +195,17 @@ __device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t
       "l"(src), "r"(bytes), "r"(bar), "l"(pol)
       : "memory");
 }
+__device__ __forceinline__ uint32_t map_to_rank(uint32_t saddr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
+  return r;
+}
+// Remote store of one u32 into a cluster peer's shared memory, completing bytes on the peer's mbarrier.
+__device__ __forceinline__ void st_async_u32(uint32_t raddr, uint32_t v, uint32_t rbar) {
+  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b32 [%0], %1, [%2];" ::"r"(raddr), "r"(v),
+               "r"(rbar)
+               : "memory");
+}
 
 constexpr int kBulkThreads = 256;
 constexpr int kBulkMaxStage = 160 * 1024;  // larger rows (e.g. 4K) take the register-streaming kernel
@@ -215,40 +213,48 @@ constexpr int kBulkMaxStage = 160 * 1024;  // larger rows (e.g. 4K) take the reg
 template <bool kD100>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads) sdd_bulk_kernel(SddArgs a) {
   extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ __align__(8) uint64_t bar;
+  __shared__ __align__(8) uint64_t bar_data;   // this row's source bytes have landed
+  __shared__ __align__(8) uint64_t bar_pair;   // (even CTA) the odd CTA's 2-cell sums have landed
   __shared__ uint32_t red[kBulkThreads / 32];
-  __shared__ int s_last;
-  cg::cluster_group cluster = cg::this_cluster();
   const int sdd_w = a.sdd_w, sdd_h = a.sdd_h;
   const int f = blockIdx.x / sdd_h;
   const int r = blockIdx.x - f * sdd_h;  // 100-grid row; the cluster pairs rows 2b and 2b+1
-  const unsigned rank = cluster.block_rank();
+  const uint32_t rank = (uint32_t)r & 1u;
   const FrameDesc fd = a.frames[f];
   const int W = fd.W, H = fd.H;
   const int rb16 = (3 * W + 15) & ~15;
   const int nchunk = rb16 >> 4;
   const int y0 = (int)(((int64_t)r * H) / sdd_h), y1 = (int)(((int64_t)(r + 1) * H) / sdd_h);
   const int rows = y1 - y0;
-  uint32_t* cell = reinterpret_cast<uint32_t*>(smem + a.stage_bytes);            // [3*sdd_w]
-  uint32_t* pair_in = cell + 3 * sdd_w;                                           // [3*sdd_w/2]
-  const uint32_t bar_a = (uint32_t)__cvta_generic_to_shared(&bar);
+  const int half3 = 3 * (sdd_w >> 1);
+  uint32_t* cell = reinterpret_cast<uint32_t*>(smem + a.stage_bytes);  // [3*sdd_w]
+  uint32_t* pair_in = cell + 3 * sdd_w;                                // [half3]
+  int* xb = reinterpret_cast<int*>(pair_in + half3);                   // [sdd_w + 1]
+  const uint32_t bar_d = (uint32_t)__cvta_generic_to_shared(&bar_data);
+  const uint32_t bar_p = (uint32_t)__cvta_generic_to_shared(&bar_pair);
 
   if (threadIdx.x == 0) {
-    mbar_init_cta(bar_a, 1);
+    mbar_init_cta(bar_d, 1);
+    mbar_init_cta(bar_p, 1);
+    if (rank == 0) mbar_expect_tx(bar_p, (uint32_t)(4 * half3));  // our own arrival + the peer's bytes
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     uint64_t pol;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-    mbar_expect_tx(bar_a, (uint32_t)(rows * rb16));
+    mbar_expect_tx(bar_d, (uint32_t)(rows * rb16));
     const uint32_t dst = (uint32_t)__cvta_generic_to_shared(smem);
     const uint8_t* src = fd.pixels + (int64_t)y0 * fd.pitch;
     if (fd.pitch == rb16) {
-      bulk_g2s(dst, src, (uint32_t)(rows * rb16), bar_a, pol);
+      bulk_g2s(dst, src, (uint32_t)(rows * rb16), bar_d, pol);
     } else {
-      for (int y = 0; y < rows; ++y) bulk_g2s(dst + y * rb16, src + (int64_t)y * fd.pitch, (uint32_t)rb16, bar_a, pol);
+      for (int y = 0; y < rows; ++y) bulk_g2s(dst + y * rb16, src + (int64_t)y * fd.pitch, (uint32_t)rb16, bar_d, pol);
     }
   }
+  // publish the peer's mbarrier before any remote st.async (relaxed: no memory fence needed beyond
+  // fence.mbarrier_init); the matching wait comes right before the DSMEM exchange
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
+  fill_xbounds(xb, W, sdd_w);
   __syncthreads();
-  mbar_wait_parity(bar_a, 0);
+  mbar_wait_parity(bar_d, 0);
 
   // ---- column sums of the row's source rows (<= 2 16-byte chunks per thread)
   uint32_t acc[2][8];
@@ -274,7 +280,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads) sdd_bu
   uint32_t ssd_local = 0;
   for (int o = threadIdx.x; o < row3; o += kBulkThreads) {
     const int cx = o / 3, ch = o - 3 * cx;
-    const int x0 = (int)(((int64_t)cx * W) / sdd_w), x1 = (int)(((int64_t)(cx + 1) * W) / sdd_w);
+    const int x0 = xb[cx], x1 = xb[cx + 1];
     uint32_t s = 0;
     for (int x = x0; x < x1; ++x) s += colsum[3 * x + ch];
     cell[o] = s;
@@ -286,62 +292,26 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads) sdd_bu
   }
   __syncthreads();
 
-  // ---- D50 row: odd CTA -> even CTA over DSMEM, then the even CTA combines the 2x2 cells
-  const int half3 = 3 * (sdd_w >> 1);
+  // ---- D50 row: odd CTA -> even CTA (st.async into the peer's shared memory), even CTA combines 2x2 cells
+  asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
   if (rank == 1) {
-    uint32_t* remote = cluster.map_shared_rank(pair_in, 0);
+    const uint32_t rbase = map_to_rank((uint32_t)__cvta_generic_to_shared(pair_in), 0);
+    const uint32_t rbar = map_to_rank(bar_p, 0);
     for (int o = threadIdx.x; o < half3; o += kBulkThreads) {
       const int cx = o / 3, ch = o - 3 * cx;
-      remote[o] = cell[6 * cx + ch] + cell[6 * cx + 3 + ch];
+      st_async_u32(rbase + 4u * (uint32_t)o, cell[6 * cx + ch] + cell[6 * cx + 3 + ch], rbar);
     }
-  }
-  cluster.sync();
-  if (rank == 0) {
+  } else {
     const int yb = (int)(((int64_t)(r + 2) * H) / sdd_h);
+    mbar_wait_parity(bar_p, 0);
     for (int o = threadIdx.x; o < half3; o += kBulkThreads) {
       const int cx = o / 3, ch = o - 3 * cx;
       const uint32_t s = cell[6 * cx + ch] + cell[6 * cx + 3 + ch] + pair_in[o];
-      const int x0 = (int)(((int64_t)(2 * cx) * W) / sdd_w), x1 = (int)(((int64_t)(2 * cx + 2) * W) / sdd_w);
-      const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)(yb - y0);
+      const uint32_t n = (uint32_t)(xb[2 * cx + 2] - xb[2 * cx]) * (uint32_t)(yb - y0);
       a.d50[(int64_t)f * a.d50_stride + (int64_t)(r >> 1) * half3 + o] = (uint8_t)((s + (n >> 1)) / n);
     }
   }
-
-  // ---- SSD partial of this row, frame ticket, last CTA finalises
-#pragma unroll
-  for (int off = 16; off > 0; off >>= 1) ssd_local += __shfl_xor_sync(0xffffffffu, ssd_local, off);
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  if (lane == 0) red[warp] = ssd_local;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    uint32_t t = 0;
-#pragma unroll
-    for (int w = 0; w < kBulkThreads / 32; ++w) t += red[w];
-    a.partial[(int64_t)f * sdd_h + r] = t;
-    __threadfence();
-    const unsigned ticket = atomicAdd(a.counter + f, 1u);
-    s_last = (ticket == (unsigned)(sdd_h - 1));
-  }
-  __syncthreads();
-  if (s_last && warp == 0) {
-    __threadfence();
-    unsigned long long sum = 0;
-    for (int b = lane; b < sdd_h; b += 32) sum += __ldcg(a.partial + (int64_t)f * sdd_h + b);
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) sum += __shfl_xor_sync(0xffffffffu, sum, off);
-    if (lane == 0) {
-      const uint8_t p = sum > fd.T ? 1 : 0;
-      a.ssd[f] = sum;
-      a.pass[f] = p;
-      a.counter[f] = 0u;
-      if (a.stats) {
-        unsigned long long* st = a.stats + (int64_t)fd.slot * NSTAT;
-        atomicAdd(st + 0, 1ull);
-        atomicAdd(st + 1, (unsigned long long)p);
-        atomicAdd(st + 3, sum);
-      }
-    }
-  }
+  ssd_commit(ssd_local, red, a, f, fd.slot, r == 0);
 }
 
 // Reference image R: one rounding of the mean over k frames x box. One thread per value.
@@ -369,7 +339,9 @@ __global__ void fill_nan_kernel(float* p, int32_t n) {
 
 }  // namespace
 
-size_t sdd_smem_bytes(int max_chunks, int sdd_w) { return (size_t)4 * 16 * max_chunks + (size_t)8 * 3 * sdd_w; }
+size_t sdd_smem_bytes(int max_chunks, int sdd_w) {
+  return (size_t)4 * 16 * max_chunks + (size_t)8 * 3 * sdd_w + (size_t)4 * (sdd_w + 1);
+}
 
 int sdd_threads(int max_chunks) {
   int t = ((max_chunks + 31) / 32) * 32;
@@ -379,7 +351,7 @@ int sdd_threads(int max_chunks) {
 }
 
 size_t sdd_bulk_smem_bytes(int stage_bytes, int sdd_w) {
-  return (size_t)stage_bytes + (size_t)4 * (3 * sdd_w + 3 * (sdd_w / 2));
+  return (size_t)stage_bytes + (size_t)4 * (3 * sdd_w + 3 * (sdd_w / 2) + sdd_w + 1);
 }
 
 int sdd_bulk_stage_bytes(int W, int H, int sdd_h) {
