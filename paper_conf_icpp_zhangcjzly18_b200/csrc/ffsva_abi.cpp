@@ -24,6 +24,7 @@ ffsva_status validate_desc(const ffsva_stream_desc* d) {
   if (d->width < d->sdd_w || d->height < d->sdd_h) return fail(FFSVA_EINVAL, "frame smaller than the SDD grid");
   if (d->width > 16384) return fail(FFSVA_EINVAL, "width > 16384");
   if ((int64_t)d->height > 256LL * d->sdd_h) return fail(FFSVA_EINVAL, "height > 256 * sdd_h");
+  if (d->height > 65535) return fail(FFSVA_EINVAL, "height > 65535");
   if (d->row_pitch < 3LL * d->width) return fail(FFSVA_EINVAL, "row_pitch < 3 * width");
   if (!(d->delta_diff >= 0.0) || !std::isfinite(d->delta_diff)) return fail(FFSVA_EINVAL, "delta_diff < 0");
   if (!(d->c_low >= 0.f && d->c_low <= d->c_high && d->c_high <= 1.f))
