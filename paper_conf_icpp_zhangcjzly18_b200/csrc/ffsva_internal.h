@@ -58,6 +58,9 @@ struct SddArgs {
   bool vec16;                // all frames 16-B aligned with 16-B pitch
   bool bulk;                 // use the bulk-async (TMA engine) + cluster kernel
   int32_t stage_bytes;       // bulk: shared-memory bytes for one 100-grid row's source rows (max over frames)
+  const int32_t* xbounds;    // [sdd_w + 1] floor(i*uni_W/sdd_w) for frames of width uni_W, or nullptr
+  const int32_t* ybounds;    // [sdd_h + 1] floor(i*uni_H/sdd_h) for frames of height uni_H, or nullptr
+  int32_t uni_W, uni_H;
 };
 cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st);
 size_t sdd_smem_bytes(int max_chunks, int sdd_w);

@@ -240,6 +240,8 @@ static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t s
   const size_t o_perm = off; off += al(4 * n);
   const size_t o_seg = off; off += al(4 * (n + 1));
   const size_t o_segb = off; off += al(8 * n);  // seg_batch[cap] then seg_slot[cap]
+  const size_t o_xb = off; off += al(4 * (size_t)(sdd_w + 1));
+  const size_t o_yb = off; off += al(4 * (size_t)(sdd_h + 1));
   b->in_bytes = off;
   const size_t o_d50 = off; off += al((size_t)b->d50_stride * n);
   const size_t o_d100 = off; off += d100 ? al((size_t)3 * sdd_w * sdd_h * n) : 0;
@@ -259,6 +261,8 @@ static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t s
   b->d_perm = (int32_t*)(base + o_perm);
   b->d_seg_lo = (int32_t*)(base + o_seg);
   b->d_seg_batch = (int32_t*)(base + o_segb);
+  b->d_xb = (int32_t*)(base + o_xb);
+  b->d_yb = (int32_t*)(base + o_yb);
   b->d_d50 = base + o_d50;
   b->d_d100 = d100 ? base + o_d100 : nullptr;
   b->d_acc = (unsigned long long*)(base + o_acc);
@@ -359,6 +363,19 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     }
   hseg[nseg] = n;
   b->n_seg = nseg;
+  // cell boundary tables (C1: cell i covers [floor(i*S/D), floor((i+1)*S/D))) when the batch shares W / H
+  int32_t* hxb = (int32_t*)((uint8_t*)b->h_in + ((uint8_t*)b->d_xb - (uint8_t*)b->d_mem));
+  int32_t* hyb = (int32_t*)((uint8_t*)b->h_in + ((uint8_t*)b->d_yb - (uint8_t*)b->d_mem));
+  b->uni_W = hd[0].W;
+  b->uni_H = hd[0].H;
+  for (int32_t i = 1; i < n; ++i) {
+    if (hd[i].W != b->uni_W) b->uni_W = -1;
+    if (hd[i].H != b->uni_H) b->uni_H = -1;
+  }
+  if (b->uni_W > 0)
+    for (int32_t i = 0; i <= sdd_w; ++i) hxb[i] = (int32_t)(((int64_t)i * b->uni_W) / sdd_w);
+  if (b->uni_H > 0)
+    for (int32_t i = 0; i <= sdd_h; ++i) hyb[i] = (int32_t)(((int64_t)i * b->uni_H) / sdd_h);
   e = cudaMemcpyAsync(b->d_mem, b->h_in, b->in_bytes, cudaMemcpyHostToDevice, st);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "cudaMemcpyAsync(descriptors)");
   // the staging buffer is reused by the next build: make sure this copy has consumed it
@@ -382,6 +399,10 @@ SddArgs make_sdd_args(Batch* b, int32_t i0, int32_t cnt) {
   sa.vec16 = b->vec16;
   sa.bulk = b->bulk;
   sa.stage_bytes = b->stage_bytes;
+  sa.uni_W = b->uni_W;
+  sa.uni_H = b->uni_H;
+  sa.xbounds = b->uni_W > 0 ? b->d_xb : nullptr;
+  sa.ybounds = b->uni_H > 0 ? b->d_yb : nullptr;
   return sa;
 }
 

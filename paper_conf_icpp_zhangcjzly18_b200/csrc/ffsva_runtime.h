@@ -39,6 +39,8 @@ struct Batch {
   bool vec16 = true, sdd_only = false, want_d100 = false;
   bool bulk = false;          // K1 variant: bulk-async + cluster (aligned frames) or register streaming
   int32_t stage_bytes = 0;
+  int32_t uni_W = -1, uni_H = -1;        // common frame size of the batch (-1: mixed)
+  int32_t *d_xb = nullptr, *d_yb = nullptr;  // cell boundary tables for uni_W / uni_H (in the input block)
   int64_t d50_stride = 0;
   // device buffers (carved from one allocation)
   void* d_mem = nullptr;

@@ -85,6 +85,40 @@ __device__ __forceinline__ uint32_t cell_sum(const uint16_t* col, int x0, int x1
   return s;
 }
 
+// All three channel sums of one 100-grid cell whose interleaved u16 column sums occupy [u0, u1) of colsum
+// (u0 = 3*x0, u1 = 3*x1), read as packed u32 words. u16 index u has channel u % 3, so word k = (2k, 2k+1)
+// carries channels (0,1), (2,0), (1,2) for k % 3 = 0, 1, 2: three packed accumulators by word class, then
+// ch0 = lo(S0) + hi(S1), ch1 = hi(S0) + lo(S2), ch2 = lo(S1) + hi(S2). The caller guarantees no 16-bit lane
+// overflows ((x1 - x0 + 2) * rows * 255 / 2 < 65536).
+__device__ __forceinline__ void cell_sum3_packed(const uint32_t* cw, int u0, int u1, uint32_t& c0, uint32_t& c1,
+                                                 uint32_t& c2) {
+  const int k0 = u0 >> 1, k1 = (u1 + 1) >> 1;  // words [k0, k1)
+  uint32_t a = 0, b = 0, c = 0;                // classes (k0 + 0, 1, 2) % 3
+  int k = k0;
+  for (; k + 3 <= k1; k += 3) {
+    a += cw[k];
+    b += cw[k + 1];
+    c += cw[k + 2];
+  }
+  if (k < k1) a += cw[k];
+  if (k + 1 < k1) b += cw[k + 1];
+  if (u0 & 1) a -= cw[k0] & 0xFFFFu;  // first word: its low half belongs to the previous cell
+  if (u1 & 1) {                        // last word: its high half belongs to the next cell
+    const uint32_t hi = cw[k1 - 1] & 0xFFFF0000u;
+    const int j = (k1 - 1 - k0) % 3;
+    if (j == 0) a -= hi;
+    else if (j == 1) b -= hi;
+    else c -= hi;
+  }
+  const int cls = k0 % 3;  // rotate (a, b, c) to word classes (S0, S1, S2)
+  const uint32_t S0 = cls == 0 ? a : (cls == 1 ? c : b);
+  const uint32_t S1 = cls == 0 ? b : (cls == 1 ? a : c);
+  const uint32_t S2 = cls == 0 ? c : (cls == 1 ? b : a);
+  c0 = (S0 & 0xFFFFu) + (S1 >> 16);
+  c1 = (S0 >> 16) + (S2 & 0xFFFFu);
+  c2 = (S1 & 0xFFFFu) + (S2 >> 16);
+}
+
 // Store the 16 column sums of chunk c (u16 each) for one 100-grid row.
 __device__ __forceinline__ void store_colsum(uint32_t* colw, int c, const uint32_t (&a)[8]) {
   uint4 lo, hi;
@@ -238,7 +272,7 @@ constexpr int kBulkThreads = 256;
 constexpr int kBulkMaxStage = 160 * 1024;  // larger rows (e.g. 4K) take the register-streaming kernel
 
 template <bool kD100>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads) sdd_bulk_kernel(SddArgs a) {
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, 6) sdd_bulk_kernel(SddArgs a) {
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t bar_data;   // this row's source bytes have landed
   __shared__ __align__(8) uint64_t bar_pair;   // (even CTA) the odd CTA's 2-cell sums have landed
@@ -251,14 +285,17 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads) sdd_bu
   const int W = fd.W, H = fd.H;
   const int rb16 = (3 * W + 15) & ~15;
   const int nchunk = rb16 >> 4;
-  // row boundaries in 32-bit (H <= 65535 and sdd_h <= 4096 are validated, so r*H < 2^28)
-  const int y0 = (int)(((uint32_t)r * (uint32_t)H) / (uint32_t)sdd_h);
-  const int y1 = (int)(((uint32_t)(r + 1) * (uint32_t)H) / (uint32_t)sdd_h);
+  // row boundaries: host table when every frame of the batch has this height, else 32-bit division
+  // (H <= 65535 and sdd_h <= 4096 are validated, so r*H < 2^28)
+  const bool uni_h = a.ybounds != nullptr && H == a.uni_H;
+  const int y0 = uni_h ? __ldg(a.ybounds + r) : (int)(((uint32_t)r * (uint32_t)H) / (uint32_t)sdd_h);
+  const int y1 = uni_h ? __ldg(a.ybounds + r + 1) : (int)(((uint32_t)(r + 1) * (uint32_t)H) / (uint32_t)sdd_h);
   const int rows = y1 - y0;
   const int half3 = 3 * (sdd_w >> 1);
   uint32_t* cell = reinterpret_cast<uint32_t*>(smem + a.stage_bytes);  // [3*sdd_w]
   uint32_t* pair_in = cell + 3 * sdd_w;                                // [half3]
-  int* xb = reinterpret_cast<int*>(pair_in + half3);                   // [sdd_w + 1]
+  const bool uni_w = a.xbounds != nullptr && W == a.uni_W;
+  const int* xb = uni_w ? a.xbounds : reinterpret_cast<int*>(pair_in + half3);  // [sdd_w + 1]
   const uint32_t bar_d = (uint32_t)__cvta_generic_to_shared(&bar_data);
   const uint32_t bar_p = (uint32_t)__cvta_generic_to_shared(&bar_pair);
 
@@ -281,7 +318,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads) sdd_bu
   // publish the peer's mbarrier before any remote st.async (relaxed: no memory fence needed beyond
   // fence.mbarrier_init); the matching wait comes right before the DSMEM exchange
   asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
-  fill_xbounds(xb, W, sdd_w);
+  if (!uni_w) fill_xbounds(const_cast<int*>(xb), W, sdd_w);
   __syncthreads();
   mbar_wait_parity(bar_d, 0);
 
@@ -309,19 +346,30 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads) sdd_bu
   }
   __syncthreads();
 
-  // ---- 100-grid cells of this row: D100, SSD vs R
+  // ---- 100-grid cells of this row (one thread per cell, all three channels): D100, SSD vs R
   const int row3 = 3 * sdd_w;
+  const bool packed = ((W + sdd_w - 1) / sdd_w + 2) * rows * 255 < 131072;  // no 16-bit lane overflow
   uint32_t ssd_local = 0;
-  for (int o = threadIdx.x; o < row3; o += kBulkThreads) {
-    const int cx = o / 3, ch = o - 3 * cx;
+  for (int cx = threadIdx.x; cx < sdd_w; cx += kBulkThreads) {
     const int x0 = xb[cx], x1 = xb[cx + 1];
-    const uint32_t s = cell_sum(colsum + ch, x0, x1);
-    cell[o] = s;
+    uint32_t s[3];
+    if (packed) {
+      cell_sum3_packed(reinterpret_cast<const uint32_t*>(colsum), 3 * x0, 3 * x1, s[0], s[1], s[2]);
+    } else {
+#pragma unroll
+      for (int ch = 0; ch < 3; ++ch) s[ch] = cell_sum(colsum + ch, x0, x1);
+    }
     const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)rows;
-    const uint32_t d = (s + (n >> 1)) / n;
-    if (kD100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)r * row3 + o] = (uint8_t)d;
-    const int diff = (int)d - (int)__ldg(fd.ref + (int64_t)r * row3 + o);
-    ssd_local += (uint32_t)(diff * diff);
+    const uchar3 ref = *reinterpret_cast<const uchar3*>(fd.ref + (int64_t)r * row3 + 3 * cx);
+    const int rv[3] = {ref.x, ref.y, ref.z};
+#pragma unroll
+    for (int ch = 0; ch < 3; ++ch) {
+      cell[3 * cx + ch] = s[ch];
+      const uint32_t d = (s[ch] + (n >> 1)) / n;
+      if (kD100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)r * row3 + 3 * cx + ch] = (uint8_t)d;
+      const int diff = (int)d - rv[ch];
+      ssd_local += (uint32_t)(diff * diff);
+    }
   }
   __syncthreads();
 
@@ -337,7 +385,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads) sdd_bu
       st_async_u32(rbase + 4u * (uint32_t)o, cell[6 * cx + ch] + cell[6 * cx + 3 + ch], rbar);
     }
   } else {
-    const int yb = (int)(((uint32_t)(r + 2) * (uint32_t)H) / (uint32_t)sdd_h);
+    const int yb = uni_h ? __ldg(a.ybounds + r + 2) : (int)(((uint32_t)(r + 2) * (uint32_t)H) / (uint32_t)sdd_h);
     mbar_wait_parity(bar_p, 0);
     for (int o = threadIdx.x; o < half3; o += kBulkThreads) {
       const int cx = o / 3, ch = o - 3 * cx;
