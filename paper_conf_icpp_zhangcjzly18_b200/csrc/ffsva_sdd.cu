@@ -85,6 +85,18 @@ __device__ __forceinline__ uint32_t cell_sum(const uint16_t* col, int x0, int x1
   return s;
 }
 
+// Sum of col[3x], x in [x0, x1) with x1 - x0 <= N: fully unrolled, predicated.
+template <int N>
+__device__ __forceinline__ uint32_t cell_sum_n(const uint16_t* col, int x0, int x1) {
+  uint32_t s = 0;
+  const uint16_t* p = col + 3 * x0;
+  const int w = x1 - x0;
+#pragma unroll
+  for (int k = 0; k < N; ++k)
+    if (k < w) s += p[3 * k];
+  return s;
+}
+
 // All three channel sums of one 100-grid cell whose interleaved u16 column sums occupy [u0, u1) of colsum
 // (u0 = 3*x0, u1 = 3*x1), read as packed u32 words. u16 index u has channel u % 3, so word k = (2k, 2k+1)
 // carries channels (0,1), (2,0), (1,2) for k % 3 = 0, 1, 2: three packed accumulators by word class, then
@@ -272,7 +284,11 @@ constexpr int kBulkThreads = 256;
 constexpr int kBulkMaxStage = 160 * 1024;  // larger rows (e.g. 4K) take the register-streaming kernel
 
 template <bool kD100>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, 6) sdd_bulk_kernel(SddArgs a) {
+#ifndef FFSVA_K1_MINBLOCKS
+#define FFSVA_K1_MINBLOCKS 1  // A/B knob: 6 caps registers at 40 (6 CTAs/SM) at the cost of small spills
+#endif
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_K1_MINBLOCKS)
+    sdd_bulk_kernel(SddArgs a) {
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t bar_data;   // this row's source bytes have landed
   __shared__ __align__(8) uint64_t bar_pair;   // (even CTA) the odd CTA's 2-cell sums have landed
@@ -346,30 +362,25 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, 6) sdd
   }
   __syncthreads();
 
-  // ---- 100-grid cells of this row (one thread per cell, all three channels): D100, SSD vs R
+  // ---- 100-grid cells of this row (one thread per cell and channel): D100, SSD vs R
   const int row3 = 3 * sdd_w;
-  const bool packed = ((W + sdd_w - 1) / sdd_w + 2) * rows * 255 < 131072;  // no 16-bit lane overflow
+  const int cellw = (W + sdd_w - 1) / sdd_w;  // widest cell of this frame (uniform over the CTA)
   uint32_t ssd_local = 0;
-  for (int cx = threadIdx.x; cx < sdd_w; cx += kBulkThreads) {
+  for (int o = threadIdx.x; o < row3; o += kBulkThreads) {
+    const int cx = o / 3, ch = o - 3 * cx;
     const int x0 = xb[cx], x1 = xb[cx + 1];
-    uint32_t s[3];
-    if (packed) {
-      cell_sum3_packed(reinterpret_cast<const uint32_t*>(colsum), 3 * x0, 3 * x1, s[0], s[1], s[2]);
-    } else {
-#pragma unroll
-      for (int ch = 0; ch < 3; ++ch) s[ch] = cell_sum(colsum + ch, x0, x1);
-    }
+    const uint16_t* col = colsum + ch;
+    uint32_t s;
+    if (cellw <= 8) s = cell_sum_n<8>(col, x0, x1);
+    else if (cellw <= 16) s = cell_sum_n<16>(col, x0, x1);
+    else if (cellw <= 24) s = cell_sum_n<24>(col, x0, x1);
+    else s = cell_sum(col, x0, x1);
+    cell[o] = s;
     const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)rows;
-    const uchar3 ref = *reinterpret_cast<const uchar3*>(fd.ref + (int64_t)r * row3 + 3 * cx);
-    const int rv[3] = {ref.x, ref.y, ref.z};
-#pragma unroll
-    for (int ch = 0; ch < 3; ++ch) {
-      cell[3 * cx + ch] = s[ch];
-      const uint32_t d = (s[ch] + (n >> 1)) / n;
-      if (kD100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)r * row3 + 3 * cx + ch] = (uint8_t)d;
-      const int diff = (int)d - rv[ch];
-      ssd_local += (uint32_t)(diff * diff);
-    }
+    const uint32_t d = (s + (n >> 1)) / n;
+    if (kD100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)r * row3 + o] = (uint8_t)d;
+    const int diff = (int)d - (int)__ldg(fd.ref + (int64_t)r * row3 + o);
+    ssd_local += (uint32_t)(diff * diff);
   }
   __syncthreads();
 

@@ -16,7 +16,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "lib", "libffsva.so")
+LIB_PATH = os.environ.get("FFSVA_LIB", os.path.join(_HERE, "lib", "libffsva.so"))  # FFSVA_LIB: A/B builds
 
 FFSVA_OK, FFSVA_EINVAL, FFSVA_ENOMEM, FFSVA_ECUDA, FFSVA_ESTATE, FFSVA_EAGAIN, FFSVA_EDEVICE = 0, -1, -2, -3, -4, -5, -6
 STATUS_NAMES = {0: "FFSVA_OK", -1: "FFSVA_EINVAL", -2: "FFSVA_ENOMEM", -3: "FFSVA_ECUDA", -4: "FFSVA_ESTATE",
