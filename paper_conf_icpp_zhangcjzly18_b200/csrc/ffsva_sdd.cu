@@ -285,7 +285,10 @@ constexpr int kBulkMaxStage = 160 * 1024;  // larger rows (e.g. 4K) take the reg
 
 template <bool kD100>
 #ifndef FFSVA_K1_MINBLOCKS
-#define FFSVA_K1_MINBLOCKS 1  // A/B knob: 6 caps registers at 40 (6 CTAs/SM) at the cost of small spills
+#define FFSVA_K1_MINBLOCKS 6  // 6 CTAs/SM: caps registers at 40 (A/B knob)
+#endif
+#ifndef FFSVA_K1_CELL16
+#define FFSVA_K1_CELL16 0     // A/B knob: cell sums unrolled to 16 instead of 24
 #endif
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_K1_MINBLOCKS)
     sdd_bulk_kernel(SddArgs a) {
@@ -301,17 +304,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   const int W = fd.W, H = fd.H;
   const int rb16 = (3 * W + 15) & ~15;
   const int nchunk = rb16 >> 4;
-  // row boundaries: host table when every frame of the batch has this height, else 32-bit division
-  // (H <= 65535 and sdd_h <= 4096 are validated, so r*H < 2^28)
-  const bool uni_h = a.ybounds != nullptr && H == a.uni_H;
-  const int y0 = uni_h ? __ldg(a.ybounds + r) : (int)(((uint32_t)r * (uint32_t)H) / (uint32_t)sdd_h);
-  const int y1 = uni_h ? __ldg(a.ybounds + r + 1) : (int)(((uint32_t)(r + 1) * (uint32_t)H) / (uint32_t)sdd_h);
+  // row boundaries in 32-bit arithmetic (H <= 65535 and sdd_h <= 4096 are validated, so r*H < 2^28); no
+  // dependent global load may sit in front of the bulk-copy issue
+  const int y0 = (int)(((uint32_t)r * (uint32_t)H) / (uint32_t)sdd_h);
+  const int y1 = (int)(((uint32_t)(r + 1) * (uint32_t)H) / (uint32_t)sdd_h);
   const int rows = y1 - y0;
   const int half3 = 3 * (sdd_w >> 1);
   uint32_t* cell = reinterpret_cast<uint32_t*>(smem + a.stage_bytes);  // [3*sdd_w]
   uint32_t* pair_in = cell + 3 * sdd_w;                                // [half3]
-  const bool uni_w = a.xbounds != nullptr && W == a.uni_W;
-  const int* xb = uni_w ? a.xbounds : reinterpret_cast<int*>(pair_in + half3);  // [sdd_w + 1]
+  int* xb = reinterpret_cast<int*>(pair_in + half3);                   // [sdd_w + 1]
   const uint32_t bar_d = (uint32_t)__cvta_generic_to_shared(&bar_data);
   const uint32_t bar_p = (uint32_t)__cvta_generic_to_shared(&bar_pair);
 
@@ -334,7 +335,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   // publish the peer's mbarrier before any remote st.async (relaxed: no memory fence needed beyond
   // fence.mbarrier_init); the matching wait comes right before the DSMEM exchange
   asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
-  if (!uni_w) fill_xbounds(const_cast<int*>(xb), W, sdd_w);
+  fill_xbounds(xb, W, sdd_w);
   __syncthreads();
   mbar_wait_parity(bar_d, 0);
 
@@ -370,11 +371,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
     const int cx = o / 3, ch = o - 3 * cx;
     const int x0 = xb[cx], x1 = xb[cx + 1];
     const uint16_t* col = colsum + ch;
-    uint32_t s;
-    if (cellw <= 8) s = cell_sum_n<8>(col, x0, x1);
-    else if (cellw <= 16) s = cell_sum_n<16>(col, x0, x1);
-    else if (cellw <= 24) s = cell_sum_n<24>(col, x0, x1);
-    else s = cell_sum(col, x0, x1);
+#if FFSVA_K1_CELL16
+    const uint32_t s = cellw <= 16 ? cell_sum_n<16>(col, x0, x1) : cell_sum(col, x0, x1);
+#else
+    const uint32_t s = cell_sum(col, x0, x1);
+#endif
     cell[o] = s;
     const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)rows;
     const uint32_t d = (s + (n >> 1)) / n;
@@ -396,7 +397,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
       st_async_u32(rbase + 4u * (uint32_t)o, cell[6 * cx + ch] + cell[6 * cx + 3 + ch], rbar);
     }
   } else {
-    const int yb = uni_h ? __ldg(a.ybounds + r + 2) : (int)(((uint32_t)(r + 2) * (uint32_t)H) / (uint32_t)sdd_h);
+    const int yb = (int)(((uint32_t)(r + 2) * (uint32_t)H) / (uint32_t)sdd_h);
     mbar_wait_parity(bar_p, 0);
     for (int o = threadIdx.x; o < half3; o += kBulkThreads) {
       const int cx = o / 3, ch = o - 3 * cx;
