@@ -288,7 +288,7 @@ template <bool kD100>
 #define FFSVA_K1_MINBLOCKS 6  // 6 CTAs/SM: caps registers at 40 (A/B knob)
 #endif
 #ifndef FFSVA_K1_CELL16
-#define FFSVA_K1_CELL16 0     // A/B knob: cell sums unrolled to 16 instead of 24
+#define FFSVA_K1_CELL16 1     // cell sums unrolled to 16 (cells <= 16 px) instead of 24 (A/B knob)
 #endif
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_K1_MINBLOCKS)
     sdd_bulk_kernel(SddArgs a) {
