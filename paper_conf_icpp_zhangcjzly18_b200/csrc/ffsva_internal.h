@@ -29,19 +29,20 @@ constexpr int C1 = 16, C2 = 32;
 constexpr int IN = 50, P1 = 25, P2 = 12;             // input, pooled conv1, pooled conv2 (floor)
 constexpr int NF = C2 * P2 * P2;                    // 4608 FC inputs
 constexpr int N_PARAMS = 27 * C1 + C1 + 9 * C1 * C2 + C2 + NF + 1;  // 9697
-constexpr int CONV1_MMAS = 5;                       // 9 taps x 8 channel slots paired into 5 K=16 MMAs
-constexpr int W1_BYTES = CONV1_MMAS * 2 * C1 * 16;  // 2560
-constexpr int W2_BYTES = 9 * 2 * C2 * 16;           // 9216
+// conv1 B operands: for pool column offset b in {0,1} and tap row dy in {0,1,2}: [0] the pair of taps dx in
+// {0,1} (K-half 0 = the tap in the x-even parity plane: dx = b; K-half 1 = dx = 1 - b), [1] tap dx = 2 in
+// K-half 0 and zero weights in K-half 1. Each is [2 K-halves][16 n][8 channel slots] bf16 (3 slots used).
+constexpr int CONV1_B = 12;
+constexpr int W1_BYTES = CONV1_B * 2 * C1 * 16;     // 6144
+constexpr int W2_BYTES = 9 * 2 * C2 * 16;           // 9216: [tap][channel half][32 n][8] bf16
 constexpr int OFF_W1 = 0;
-constexpr int OFF_W2 = OFF_W1 + W1_BYTES;           // 2560
-constexpr int OFF_B1 = OFF_W2 + W2_BYTES;           // 11776 (fp32[16])
-constexpr int OFF_B2 = OFF_B1 + C1 * 4;             // 11840 (fp32[32])
-constexpr int OFF_BFC = OFF_B2 + C2 * 4;            // 11968 (fp32[1] + pad to 16)
-constexpr int OFF_WFC = OFF_BFC + 16;               // 11984 (fp32[4608], bf16-exact values)
-constexpr int BLOB_BYTES = OFF_WFC + NF * 4;        // 30416
+constexpr int OFF_W2 = OFF_W1 + W1_BYTES;           // 6144
+constexpr int OFF_B1 = OFF_W2 + W2_BYTES;           // 15360 (fp32[16])
+constexpr int OFF_B2 = OFF_B1 + C1 * 4;             // 15424 (fp32[32])
+constexpr int OFF_BFC = OFF_B2 + C2 * 4;            // 15552 (fp32[1] + pad to 16)
+constexpr int OFF_WFC = OFF_BFC + 16;               // 15568 (fp32[4608], bf16-exact values)
+constexpr int BLOB_BYTES = OFF_WFC + NF * 4;        // 34000
 static_assert(BLOB_BYTES % 16 == 0, "blob must be 16-B granular");
-// conv1 MMA j pairs two taps (dy, dx) into the two K-halves of one K=16 MMA: {start tap, second tap, LBO}.
-// j = 4's first half is tap (2,1) again with zero weights (its second half carries tap (2,2)).
 }  // namespace snm
 
 // ------------------------------------------------------------------ launchers (defined in the .cu files)

@@ -190,18 +190,20 @@ void pack_snm_blob(const float* params, uint8_t* blob) {
   const float* b2 = w2 + 9 * C1 * C2;
   const float* wfc = b2 + C2;
   const float* bfc = wfc + NF;
-  // conv1: MMA j, K-half h carries tap (dy, dx) (channels 0..2 of the 8 slots); -1 = zero half
-  static const int tap_dy[5][2] = {{0, 0}, {1, 1}, {2, 2}, {0, 1}, {-1, 2}};
-  static const int tap_dx[5][2] = {{0, 1}, {0, 1}, {0, 1}, {2, 2}, {-1, 2}};
+  // conv1: B matrix (b, dy, kind); kind 0 = taps (dx = b, dx = 1 - b) in K-halves (0, 1); kind 1 = tap dx = 2
+  // in K-half 0, zero K-half 1. Channels 0..2 of the 8 slots.
   uint16_t* W1 = reinterpret_cast<uint16_t*>(blob + OFF_W1);
-  for (int j = 0; j < CONV1_MMAS; ++j)
-    for (int h = 0; h < 2; ++h) {
-      const int dy = tap_dy[j][h], dx = tap_dx[j][h];
-      if (dy < 0) continue;
-      for (int n = 0; n < C1; ++n)
-        for (int c = 0; c < 3; ++c)
-          W1[((j * 2 + h) * C1 + n) * 8 + c] = bf16_bits_rne(w1[((n * 3 + c) * 3 + dy) * 3 + dx]);
-    }
+  for (int b = 0; b < 2; ++b)
+    for (int dy = 0; dy < 3; ++dy)
+      for (int kind = 0; kind < 2; ++kind)
+        for (int h = 0; h < 2; ++h) {
+          const int dx = kind == 0 ? (h == 0 ? b : 1 - b) : (h == 0 ? 2 : -1);
+          if (dx < 0) continue;
+          const int m = (b * 3 + dy) * 2 + kind;
+          for (int n = 0; n < C1; ++n)
+            for (int c = 0; c < 3; ++c)
+              W1[((m * 2 + h) * C1 + n) * 8 + c] = bf16_bits_rne(w1[((n * 3 + c) * 3 + dy) * 3 + dx]);
+        }
   // conv2: tap t, K-half h = input channels 8h..8h+7
   uint16_t* W2 = reinterpret_cast<uint16_t*>(blob + OFF_W2);
   for (int t = 0; t < 9; ++t)
@@ -384,6 +386,9 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
   return FFSVA_OK;
 }
 
+// SNM grid: one persistent CTA per SM (the kernel holds all 512 TMEM columns), no more CTAs than frames.
+int snm_grid(const Batch* b) { return std::max(1, std::min(b->n, b->ctx->num_sms)); }
+
 SddArgs make_sdd_args(Batch* b, int32_t i0, int32_t cnt) {
   SddArgs sa{};
   sa.frames = b->d_desc + i0;
@@ -420,7 +425,7 @@ CompactArgs make_compact_args(Batch* b) {
   ca.seg_batch = b->d_seg_batch;
   ca.seg_slot = b->d_seg_batch + b->cap;
   ca.stats = ctx->d_stats;
-  ca.snm_ctas = b->sdd_only ? 0 : std::max(1, std::min(b->n, 2 * ctx->num_sms));
+  ca.snm_ctas = b->sdd_only ? 0 : snm_grid(b);
   ca.survivor_idx = b->d_surv;
   ca.work = b->d_work;
   ca.posw = b->d_posw;
@@ -444,7 +449,7 @@ SnmArgs make_snm_args(Batch* b) {
   na.snm_pass = b->d_snm_pass;
   na.snm_class = b->d_snm_class;
   na.stats = b->ctx->d_stats;
-  na.grid = std::max(1, std::min(b->n, 2 * b->ctx->num_sms));
+  na.grid = snm_grid(b);
   return na;
 }
 

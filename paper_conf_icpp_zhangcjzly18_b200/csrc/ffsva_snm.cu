@@ -7,24 +7,28 @@
 // 4608->1 logit (Q9, Q11); input (v-128)/128 (Q10); bf16 operands, fp32 accumulation, pooled conv1 rounded
 // to bf16, conv2 output and FC in fp32 (Q15).
 //
-// B200 mapping — implicit GEMM with no im2col: every 3x3 tap is a shifted view of one shared-memory image.
-//   * Activations are stored pixel-major with 8 channels per 16-byte row, which is exactly a row of a tcgen05
-//     K-major no-swizzle core matrix. An M=128 tile is a 16-row x 8-column patch of output pixels: core
-//     matrix j (8 rows of the MMA) = image row y0+j, so SBO = one padded image row; a tap (dy, dx) is the
-//     same descriptor shifted by (dy*Wp + dx)*16 bytes.
-//   * conv1 (K = 9 taps x 3 channels): each K=16 MMA carries two taps (one per 8-channel K-half, LBO = the
-//     byte distance between them) -> 5 MMAs of N=16 per tile, 28 tiles per frame (4 row strips x 7 column
-//     strips, the last strip of each overlapping so the 50x50 output is covered exactly).
-//   * conv2 (K = 9 taps x 16 channels): the two K-halves are two 8-channel planes (LBO = plane size) ->
-//     9 MMAs of N=32 per tile, 6 tiles (24x24 outputs survive the floor pooling; row/col 24 are skipped).
-//   * Accumulators live in TMEM (M=128 lanes x N fp32 columns per tile). The tile shape puts each 2x2
-//     pooling quad in lanes {l, l^1, l^8, l^9} of one warp, so max-pooling is two shuffles per value right
-//     after tcgen05.ld; bias and ReLU commute with max and are applied after pooling.
-//   * conv1's epilogue writes bf16 pooled activations straight into conv2's operand image; conv2's epilogue
+// B200 mapping — implicit GEMM, no im2col, pooling folded into the N dimension:
+//   * GEMM rows are POOLED output pixels. For each of the four 2x2-pool positions q = (a, b) the conv
+//     output (2py+a, 2px+b) is one MMA chain into its own TMEM column group, so the max-pool is an in-register
+//     max over four column groups of the same TMEM lane (no cross-lane shuffles); bias and ReLU commute with
+//     max and are applied once after it.
+//   * Inputs live in shared memory as four parity planes (even/odd padded row x even/odd padded column),
+//     pixel-major with 8 channels per 16-byte row (one K-major no-swizzle core-matrix row). The input pixel
+//     of pooled row py, column px, pool position (a,b), tap (dy,dx) is (2py+a+dy, 2px+b+dx) = parity plane
+//     ((a+dy)&1, (b+dx)&1), plane pixel (py + (a+dy)>>1, px + (b+dx)>>1): a constant-stride view, so each tap
+//     of each pool position is the same UMMA descriptor shifted by a few bytes (SBO = 8 pixels = 128 B; plane
+//     rows are 32 (conv1) / 16 (conv2) pixels so rows continue the 128-B core-matrix stride).
+//   * conv1 (3 channels in 8 slots): two taps that sit in the two x-parity planes share one K=16 MMA (LBO =
+//     the plane distance); 24 MMAs (M128, N16) per tile x 7 tiles of 4 pooled rows x 32 px.
+//     conv2 (16 channels = two 8-channel planes, LBO = plane distance): 36 MMAs (M128, N32) per tile x 2 tiles
+//     of 8 pooled rows x 16 px.
+//   * conv1's epilogue writes bf16 pooled activations straight into conv2's parity planes; conv2's epilogue
 //     multiplies the pooled features by the FC weights in fp32 and reduces to one logit per frame.
-// One CTA (128 threads, 4 warps = the 4 TMEM lane quadrants) per SM-half, persistent over dynamic batches
-// (chunks of <= BatchSize survivors of one stream): the stream's 30 KB weight image is copied into shared
-// memory once per chunk. Thread 0 issues all MMAs and commits them to one mbarrier.
+// One persistent CTA per SM (8 warps; warp w reads TMEM lane quadrant w%4, warp groups split the tiles), all
+// 512 TMEM columns; thread 0 issues every MMA and commits each tile to its own mbarrier so epilogues start as
+// soon as a tile lands. Work = dynamic-batch units (<= BatchSize survivors of one stream, split further when
+// the batch is small); the stream's 34 KB weight image is copied into shared memory once per unit (skipped when
+// the previous unit was the same stream), and the next frame's D50 image is prefetched with a bulk copy.
 #include <cuda_bf16.h>
 
 #include "ffsva_internal.h"
@@ -34,29 +38,29 @@ namespace {
 
 using namespace snm;
 
-constexpr int kThreads = 128;
-constexpr int X1W = 52, X1H = 52;                    // conv1 operand image: 50x50 + zero border, 8 ch (3 used)
-constexpr int X1_BYTES = X1W * X1H * 16;             // 43264
-constexpr int X2W = 26, X2H = 26;                    // conv2 operand image: 25x25 + zero border, 2 planes x 8 ch
-constexpr int X2_PLANE = X2W * X2H * 16;             // 10816
-constexpr int X2_BYTES = 2 * X2_PLANE;               // 21632
-constexpr int OFF_X1 = 0;
-constexpr int OFF_X2 = OFF_X1 + X1_BYTES;            // 43264
-constexpr int OFF_WB = OFF_X2 + X2_BYTES;            // 64896
-constexpr int OFF_RED = OFF_WB + BLOB_BYTES;         // 95312
-constexpr int OFF_BAR = OFF_RED + 64;                // 95376
-constexpr int OFF_TMEM = OFF_BAR + 8;                // 95384
-constexpr int SMEM_BYTES = OFF_TMEM + 8;             // 95392
-constexpr uint32_t kTmemCols = 256;
+constexpr int kThreads = 256;
+// conv1 operand: 4 parity planes [ypar][xpar] x 27 rows x 32 px x 16 B (padded input 52x52, 3 of 8 channels)
+constexpr int A1_COLS = 32, A1_ROWS = 27;
+constexpr int A1_PLANE = A1_ROWS * A1_COLS * 16;            // 13824
+constexpr int A1_BYTES = 4 * A1_PLANE;                      // 55296
+// conv2 operand: 8 planes [ypar][xpar][chalf] x 14 rows x 16 px x 16 B (padded pooled conv1 27x27, 16 ch)
+constexpr int A2_COLS = 16, A2_ROWS = 14;
+constexpr int A2_PLANE = A2_ROWS * A2_COLS * 16;            // 3584
+constexpr int A2_BYTES = 8 * A2_PLANE + 512;                // + zero tail read by junk rows of the last tile
+constexpr int D50_BYTES = 7504;                             // staged D50 image (one frame)
+constexpr int OFF_A1 = 0;
+constexpr int OFF_A2 = OFF_A1 + A1_BYTES;                   // 55296
+constexpr int OFF_WB = OFF_A2 + A2_BYTES;                   // 84480
+constexpr int OFF_IN = OFF_WB + BLOB_BYTES;                 // 2 staging buffers
+constexpr int OFF_RED = OFF_IN + 2 * D50_BYTES;
+constexpr int OFF_BAR = OFF_RED + 64;                       // 7 conv1 + 2 conv2 + 2 input mbarriers
+constexpr int OFF_TMEM = OFF_BAR + 16 * 8;
+constexpr int SMEM_BYTES = OFF_TMEM + 16;
+static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
+constexpr uint32_t kTmemCols = 512;
 
-constexpr int kConv1Tiles = 28;
-constexpr int kConv1Half = 14;
-__constant__ int8_t c1_y0[4] = {0, 16, 32, 34};
-__constant__ int8_t c1_x0[7] = {0, 8, 16, 24, 32, 40, 42};
-// conv1 MMA j: A starts at tap (dy, dx); the second K-half is LBO bytes further.
-__constant__ int8_t c1_dy[5] = {0, 1, 2, 0, 2};
-__constant__ int8_t c1_dx[5] = {0, 0, 0, 2, 1};
-__constant__ int16_t c1_lbo[5] = {16, 16, 16, X1W * 16, 16};
+constexpr int kTiles1 = 7, kTiles2 = 2;
+__constant__ int8_t c1_py0[kTiles1] = {0, 4, 8, 12, 16, 20, 21};  // last tile overlaps (idempotent writes)
 
 // ---------------------------------------------------------------- PTX wrappers (sm_100a)
 __device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -105,22 +109,49 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   }
 }
 
-__device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
-  uint32_t r[16];
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(bar)
+               : "memory");
+}
+
+// 32 lanes x 16 columns of fp32 from TMEM (asynchronous: the registers are valid after tmem_wait)
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
   asm volatile(
       "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
       : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
         "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
       : "r"(taddr));
-  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-#pragma unroll
-  for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+}
+// tcgen05.wait::ld, with the loaded registers as in/out operands so no use can be scheduled above it
+__device__ __forceinline__ void tmem_wait(uint32_t (&r)[16], uint32_t (&s)[16]) {
+  asm volatile("tcgen05.wait::ld.sync.aligned;"
+               : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]), "+r"(r[6]), "+r"(r[7]),
+                 "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11]), "+r"(r[12]), "+r"(r[13]), "+r"(r[14]),
+                 "+r"(r[15]), "+r"(s[0]), "+r"(s[1]), "+r"(s[2]), "+r"(s[3]), "+r"(s[4]), "+r"(s[5]), "+r"(s[6]),
+                 "+r"(s[7]), "+r"(s[8]), "+r"(s[9]), "+r"(s[10]), "+r"(s[11]), "+r"(s[12]), "+r"(s[13]),
+                 "+r"(s[14]), "+r"(s[15])
+               :
+               : "memory");
 }
 
-// 2x2 max over the pooling quad {l, l^1, l^8, l^9}.
-__device__ __forceinline__ float quad_max(float x) {
-  x = fmaxf(x, __shfl_xor_sync(0xffffffffu, x, 1));
-  return fmaxf(x, __shfl_xor_sync(0xffffffffu, x, 8));
+// max over the four pool positions: 16 consecutive channels starting at column col of each position group
+__device__ __forceinline__ void pooled16(uint32_t taddr, int col, int group_cols, float (&v)[16]) {
+  uint32_t r0[16], r1[16], r2[16], r3[16];
+  tmem_ld16(taddr + (uint32_t)col, r0);
+  tmem_ld16(taddr + (uint32_t)(col + group_cols), r1);
+  tmem_ld16(taddr + (uint32_t)(col + 2 * group_cols), r2);
+  tmem_ld16(taddr + (uint32_t)(col + 3 * group_cols), r3);
+  tmem_wait(r0, r1);
+  tmem_wait(r2, r3);
+#pragma unroll
+  for (int i = 0; i < 16; ++i)
+    v[i] = fmaxf(fmaxf(__uint_as_float(r0[i]), __uint_as_float(r1[i])),
+                 fmaxf(__uint_as_float(r2[i]), __uint_as_float(r3[i])));
 }
 
 __device__ __forceinline__ uint32_t pack_bf16(float lo, float hi) {
@@ -132,54 +163,87 @@ __device__ __forceinline__ uint32_t u8_to_bf16(uint32_t v) {  // (v - 128) / 128
   return (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(((float)v - 128.0f) * 0.0078125f));
 }
 
-// ---------------------------------------------------------------- per-tile epilogues
-// conv1 tile: TMEM columns [col, col+16) hold the 128x16 fp32 accumulator of the 16x8 output patch at
-// (y0, x0). Pool, add bias, ReLU, round to bf16, store into conv2's operand image X2.
-__device__ __forceinline__ void conv1_epilogue(uint32_t tmem, int col, int y0, int x0, uint8_t* X2,
-                                               const float* b1, uint16_t* dbg) {
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  float v[16];
-  tmem_ld16(tmem + ((uint32_t)(32 * warp) << 16) + (uint32_t)col, v);
+// ---------------------------------------------------------------- MMA issue (thread 0)
+__device__ __forceinline__ void issue_conv1_tile(uint32_t tmem, int t, uint32_t a1, uint32_t w1) {
+  const int py0 = c1_py0[t];
+  const uint32_t idesc = idesc_bf16(128, 16);
 #pragma unroll
-  for (int c = 0; c < 16; ++c) v[c] = quad_max(v[c]);
-  const int q = (lane & 1) | ((lane >> 2) & 2);  // which 4 channels this quad lane writes
-  const int y = y0 + 4 * warp + (lane >> 3), x = x0 + (lane & 7);
-  const int py = y >> 1, px = x >> 1;
-  float o[4];
+  for (int q = 0; q < 4; ++q) {
+    const int a = q >> 1, b = q & 1;
+    const uint32_t d = tmem + (uint32_t)(t * 64 + q * 16);
 #pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const float s = q == 0 ? v[i] : q == 1 ? v[4 + i] : q == 2 ? v[8 + i] : v[12 + i];
-    o[i] = fmaxf(s + b1[4 * q + i], 0.0f);
+    for (int dy = 0; dy < 3; ++dy) {
+      const int ypar = (a + dy) & 1, roff = (a + dy) >> 1;
+      const uint32_t rowbase = a1 + (uint32_t)(ypar * 2 * A1_PLANE + (py0 + roff) * A1_COLS * 16);
+      // taps dx = 0, 1 (one in each x-parity plane) share one MMA: the x-even tap is the first K-half
+      const int coff = b;  // x-even tap sits one plane column further right when b = 1
+      const uint64_t ad_pair = umma_desc(rowbase + (uint32_t)(coff * 16), (uint32_t)(A1_PLANE - 16 * coff), 128);
+      const uint64_t bd_pair = umma_desc(w1 + (uint32_t)(((b * 3 + dy) * 2 + 0) * 512), C1 * 16, 128);
+      mma_bf16(d, ad_pair, bd_pair, idesc, dy > 0 ? 1u : 0u);
+      // tap dx = 2: x-parity b, plane column 1; second K-half carries zero weights
+      const uint64_t ad_one = umma_desc(rowbase + (uint32_t)(b * A1_PLANE + 16), 16, 128);
+      const uint64_t bd_one = umma_desc(w1 + (uint32_t)(((b * 3 + dy) * 2 + 1) * 512), C1 * 16, 128);
+      mma_bf16(d, ad_one, bd_one, idesc, 1u);
+    }
   }
-  uint2 w;
-  w.x = pack_bf16(o[0], o[1]);
-  w.y = pack_bf16(o[2], o[3]);
-  *reinterpret_cast<uint2*>(X2 + (q >> 1) * X2_PLANE + ((py + 1) * X2W + (px + 1)) * 16 + (q & 1) * 8) = w;
-  if (dbg) *reinterpret_cast<uint2*>(dbg + (py * P1 + px) * 16 + 4 * q) = w;
 }
 
-// conv2 tile: 128x32 fp32 accumulator of the 16x8 patch at (y0, x0); returns this thread's FC partial sum.
-__device__ __forceinline__ float conv2_epilogue(uint32_t tmem, int col, int y0, int x0, const float* b2,
-                                                const float* wfc, float* dbg) {
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int q = (lane & 1) | ((lane >> 2) & 2);
-  const int y = y0 + 4 * warp + (lane >> 3), x = x0 + (lane & 7);
-  const int py = y >> 1, px = x >> 1;
-  const bool own = (y0 == 0) || (py >= 8);  // pooled rows 4..7 belong to the y0 = 0 tile
-  float acc = 0.0f;
+__device__ __forceinline__ void issue_conv2_tile(uint32_t tmem, int u, uint32_t a2, uint32_t w2) {
+  const int py0 = 4 * u;
+  const uint32_t idesc = idesc_bf16(128, 32);
 #pragma unroll
-  for (int h = 0; h < 2; ++h) {  // channels 16h .. 16h+15
+  for (int q = 0; q < 4; ++q) {
+    const int a = q >> 1, b = q & 1;
+    const uint32_t d = tmem + (uint32_t)(u * 128 + q * 32);
+#pragma unroll
+    for (int tap = 0; tap < 9; ++tap) {
+      const int dy = tap / 3, dx = tap % 3;
+      const int ypar = (a + dy) & 1, roff = (a + dy) >> 1, xpar = (b + dx) & 1, coff = (b + dx) >> 1;
+      const uint32_t addr = a2 + (uint32_t)(((ypar * 2 + xpar) * 2) * A2_PLANE + ((py0 + roff) * A2_COLS + coff) * 16);
+      mma_bf16(d, umma_desc(addr, A2_PLANE, 128), umma_desc(w2 + (uint32_t)(tap * 2 * C2 * 16), C2 * 16, 128), idesc,
+               tap > 0 ? 1u : 0u);
+    }
+  }
+}
+
+// ---------------------------------------------------------------- epilogues
+// conv1 tile t: lane (quadrant qd, l) = pooled pixel (py0 + qd, l); bias, ReLU, bf16 into conv2's planes.
+__device__ __forceinline__ void conv1_epilogue(uint32_t tmem, int t, uint8_t* A2, const float* b1, uint16_t* dbg) {
+  const int qd = (threadIdx.x >> 5) & 3, l = threadIdx.x & 31;
+  float v[16];
+  pooled16(tmem + ((uint32_t)(32 * qd) << 16), t * 64, 16, v);
+  const int py = c1_py0[t] + qd, px = l;
+  if (px < P1) {
+    uint32_t w[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) w[i] = pack_bf16(fmaxf(v[2 * i] + b1[2 * i], 0.f), fmaxf(v[2 * i + 1] + b1[2 * i + 1], 0.f));
+    const int Y = py + 1, X = px + 1;
+    uint8_t* p = A2 + ((((Y & 1) * 2 + (X & 1)) * 2) * A2_PLANE + ((Y >> 1) * A2_COLS + (X >> 1)) * 16);
+    *reinterpret_cast<uint4*>(p) = make_uint4(w[0], w[1], w[2], w[3]);
+    *reinterpret_cast<uint4*>(p + A2_PLANE) = make_uint4(w[4], w[5], w[6], w[7]);
+    if (dbg) {
+      uint4* d = reinterpret_cast<uint4*>(dbg + (py * P1 + px) * 16);
+      d[0] = make_uint4(w[0], w[1], w[2], w[3]);
+      d[1] = make_uint4(w[4], w[5], w[6], w[7]);
+    }
+  }
+}
+
+// conv2 tile u: lane (qd, l) = pooled pixel (4u + 2qd + (l >> 4), l & 15); returns the FC partial sum.
+__device__ __forceinline__ float conv2_epilogue(uint32_t tmem, int u, const float* b2, const float* wfc, float* dbg) {
+  const int qd = (threadIdx.x >> 5) & 3, l = threadIdx.x & 31;
+  const int py = 4 * u + 2 * qd + (l >> 4), px = l & 15;
+  const bool own = px < P2 && (u == 0 ? py < 8 : py >= 8);
+  float acc = 0.f;
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
     float v[16];
-    tmem_ld16(tmem + ((uint32_t)(32 * warp) << 16) + (uint32_t)(col + 16 * h), v);
+    pooled16(tmem + ((uint32_t)(32 * qd) << 16), u * 128 + 16 * h, 32, v);
+    if (own) {
 #pragma unroll
-    for (int c = 0; c < 16; ++c) v[c] = quad_max(v[c]);
-    // this lane handles channels 16h + 4q .. 16h + 4q + 3
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const float s = q == 0 ? v[i] : q == 1 ? v[4 + i] : q == 2 ? v[8 + i] : v[12 + i];
-      const int c = 16 * h + 4 * q + i;
-      const float r = fmaxf(s + b2[c], 0.0f);
-      if (own) {
+      for (int i = 0; i < 16; ++i) {
+        const int c = 16 * h + i;
+        const float r = fmaxf(v[i] + b2[c], 0.f);
         acc = fmaf(r, wfc[c * (P2 * P2) + py * P2 + px], acc);
         if (dbg) dbg[c * (P2 * P2) + py * P2 + px] = r;
       }
@@ -188,24 +252,23 @@ __device__ __forceinline__ float conv2_epilogue(uint32_t tmem, int col, int y0, 
   return acc;
 }
 
-__global__ void __launch_bounds__(kThreads, 2) snm_kernel(SnmArgs a) {
-  extern __shared__ __align__(128) uint8_t sm[];
-  uint8_t* X1 = sm + OFF_X1;
-  uint8_t* X2 = sm + OFF_X2;
+__global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
+  extern __shared__ __align__(1024) uint8_t sm[];
+  uint8_t* A1 = sm + OFF_A1;
+  uint8_t* A2 = sm + OFF_A2;
   uint8_t* WB = sm + OFF_WB;
+  uint8_t* stage = sm + OFF_IN;
   float* red = reinterpret_cast<float*>(sm + OFF_RED);
   uint32_t* s_tmem = reinterpret_cast<uint32_t*>(sm + OFF_TMEM);
   __shared__ int s_chunk;
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const uint32_t bar = smem_addr(sm + OFF_BAR);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, grp = warp >> 2;
+  const uint32_t bar0 = smem_addr(sm + OFF_BAR);  // bar0 + 8*i: i < 7 conv1 tiles, 7..8 conv2 tiles, 9..10 input
+  const int n_chunks = a.counts[1];
+  if (n_chunks == 0) return;  // no survivors in this batch
 
-  if (a.counts[1] == 0) return;  // no survivors in this batch
-
-  // zero both operand images once: borders and unused channel slots stay zero for the whole kernel
-  for (int i = tid; i < (X1_BYTES + X2_BYTES) / 16; i += kThreads)
-    reinterpret_cast<uint4*>(sm)[i] = make_uint4(0u, 0u, 0u, 0u);
+  for (int i = tid; i < (A1_BYTES + A2_BYTES) / 16; i += kThreads) reinterpret_cast<uint4*>(sm)[i] = make_uint4(0, 0, 0, 0);
   if (tid == 0) {
-    mbar_init(bar, 1);
+    for (int i = 0; i < 11; ++i) mbar_init(bar0 + 8 * i, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 0) {
@@ -217,16 +280,14 @@ __global__ void __launch_bounds__(kThreads, 2) snm_kernel(SnmArgs a) {
   __syncthreads();
   fence_after();
   const uint32_t tmem = *s_tmem;
-  uint32_t phase = 0;
-
-  const uint32_t x1a = smem_addr(X1), x2a = smem_addr(X2);
-  const uint32_t w1a = smem_addr(WB + OFF_W1), w2a = smem_addr(WB + OFF_W2);
+  const uint32_t a1 = smem_addr(A1), a2 = smem_addr(A2);
+  const uint32_t w1 = smem_addr(WB + OFF_W1), w2 = smem_addr(WB + OFF_W2);
   const float* b1 = reinterpret_cast<const float*>(WB + OFF_B1);
   const float* b2 = reinterpret_cast<const float*>(WB + OFF_B2);
   const float* wfc = reinterpret_cast<const float*>(WB + OFF_WFC);
-  const float bfc = 0.0f;  // read per chunk below
-  (void)bfc;
-  const int n_chunks = a.counts[1];
+  uint32_t ph = 0;           // parity of the per-frame mbarriers (one phase per frame)
+  uint32_t in_ph = 0;        // bit i: parity of input staging buffer i
+  const uint8_t* loaded = nullptr;  // weight image currently in shared memory
 
   for (;;) {
     if (tid == 0) s_chunk = atomicAdd(a.counts + 2, 1);
@@ -235,94 +296,87 @@ __global__ void __launch_bounds__(kThreads, 2) snm_kernel(SnmArgs a) {
     if (k >= n_chunks) break;
     const int start = a.chunks[k], end = a.chunks[k + 1];
     const FrameDesc fd0 = a.frames[a.work[start]];
-    // dynamic batch: this stream's SNM weight image is loaded once for the whole chunk (L219)
-    {
+    if (fd0.snm != loaded) {  // dynamic batch: one weight load per batch of this stream (L219)
       const uint4* src = reinterpret_cast<const uint4*>(fd0.snm);
       uint4* dst = reinterpret_cast<uint4*>(WB);
       for (int i = tid; i < BLOB_BYTES / 16; i += kThreads) dst[i] = __ldg(src + i);
+      loaded = fd0.snm;
     }
     const float fc_bias = __ldg(reinterpret_cast<const float*>(fd0.snm + OFF_BFC));
     uint32_t cnt_pass = 0, cnt_c0 = 0, cnt_c1 = 0, cnt_c2 = 0;
-
+    if (tid == 0) {  // stage the unit's first D50 image
+      mbar_expect_tx(bar0 + 8 * 9, D50_BYTES);
+      bulk_g2s(smem_addr(stage), a.d50 + (int64_t)a.work[start] * a.d50_stride, D50_BYTES, bar0 + 8 * 9);
+    }
     for (int j = start; j < end; ++j) {
       const int f = a.work[j];
-      // ---- input: D50 u8 -> (v-128)/128 bf16 into X1 interior (pixel = 16 B: 3 channels + 5 zeros)
-      const uint8_t* d = a.d50 + (int64_t)f * a.d50_stride;
-      for (int p = tid; p < IN * IN; p += kThreads) {
-        const int y = p / IN, x = p - y * IN;
+      const int buf = (j - start) & 1;
+      if (tid == 0 && j + 1 < end) {  // prefetch the next frame of the unit
+        const uint32_t nb = bar0 + 8 * (9 + (buf ^ 1));
+        mbar_expect_tx(nb, D50_BYTES);
+        bulk_g2s(smem_addr(stage + (buf ^ 1) * D50_BYTES), a.d50 + (int64_t)a.work[j + 1] * a.d50_stride, D50_BYTES, nb);
+      }
+      mbar_wait(bar0 + 8 * (9 + buf), (in_ph >> buf) & 1u);
+      in_ph ^= 1u << buf;
+      // ---- D50 u8 -> (v-128)/128 bf16 into conv1's parity planes (pixel = 16 B: 3 channels + 5 zeros)
+      const uint8_t* d = stage + buf * D50_BYTES;
+      for (int p = tid; p < snm::IN * snm::IN; p += kThreads) {
+        const int y = p / snm::IN, x = p - y * snm::IN;
+        const int Y = y + 1, X = x + 1;
         const uint32_t c0 = d[3 * p], c1 = d[3 * p + 1], c2 = d[3 * p + 2];
         uint4 w;
         w.x = u8_to_bf16(c0) | (u8_to_bf16(c1) << 16);
         w.y = u8_to_bf16(c2);
         w.z = 0u;
         w.w = 0u;
-        *reinterpret_cast<uint4*>(X1 + ((y + 1) * X1W + (x + 1)) * 16) = w;
+        *reinterpret_cast<uint4*>(A1 + ((Y & 1) * 2 + (X & 1)) * A1_PLANE + ((Y >> 1) * A1_COLS + (X >> 1)) * 16) = w;
       }
       fence_proxy_async();
       fence_before();
       __syncthreads();
 
-      // ---- conv1, two halves of 14 tiles (224 TMEM columns each)
-      uint16_t* dbg1 = a.dbg_p1 ? a.dbg_p1 + (int64_t)j * (P1 * P1 * 16) : nullptr;
-      for (int half = 0; half < 2; ++half) {
-        if (tid == 0) {
-          fence_after();
-          for (int t = half * kConv1Half; t < (half + 1) * kConv1Half; ++t) {
-            const int y0 = c1_y0[t / 7], x0 = c1_x0[t % 7];
-            const uint32_t dcol = tmem + (uint32_t)((t - half * kConv1Half) * 16);
-#pragma unroll
-            for (int m = 0; m < CONV1_MMAS; ++m) {
-              const uint32_t aaddr = x1a + (uint32_t)(((y0 + c1_dy[m]) * X1W + (x0 + c1_dx[m])) * 16);
-              mma_bf16(dcol, umma_desc(aaddr, (uint32_t)c1_lbo[m], X1W * 16),
-                       umma_desc(w1a + (uint32_t)(m * 2 * C1 * 16), C1 * 16, 128), idesc_bf16(128, 16),
-                       m > 0 ? 1u : 0u);
-            }
-          }
-          mma_commit(bar);
-        }
-        __syncwarp();
-        mbar_wait(bar, phase);
-        phase ^= 1u;
-        fence_after();
-        for (int t = half * kConv1Half; t < (half + 1) * kConv1Half; ++t)
-          conv1_epilogue(tmem, (t - half * kConv1Half) * 16, c1_y0[t / 7], c1_x0[t % 7], X2, b1, dbg1);
-        fence_before();
-        __syncthreads();
-      }
-
-      // ---- conv2: 6 tiles x 9 taps, N = 32
-      fence_proxy_async();
-      __syncthreads();
+      // ---- conv1: 7 tiles, one commit each; epilogues start as tiles land
       if (tid == 0) {
         fence_after();
-        for (int t = 0; t < 6; ++t) {
-          const int y0 = (t / 3) * 8, x0 = (t % 3) * 8;
-          const uint32_t dcol = tmem + (uint32_t)(t * 32);
-#pragma unroll
-          for (int tap = 0; tap < 9; ++tap) {
-            const int dy = tap / 3, dx = tap % 3;
-            const uint32_t aaddr = x2a + (uint32_t)(((y0 + dy) * X2W + (x0 + dx)) * 16);
-            mma_bf16(dcol, umma_desc(aaddr, X2_PLANE, X2W * 16), umma_desc(w2a + (uint32_t)(tap * 2 * C2 * 16), C2 * 16, 128),
-                     idesc_bf16(128, 32), tap > 0 ? 1u : 0u);
-          }
+        for (int t = 0; t < kTiles1; ++t) {
+          issue_conv1_tile(tmem, t, a1, w1);
+          mma_commit(bar0 + 8 * t);
         }
-        mma_commit(bar);
       }
       __syncwarp();
-      mbar_wait(bar, phase);
-      phase ^= 1u;
+      uint16_t* dbg1 = a.dbg_p1 ? a.dbg_p1 + (int64_t)j * (P1 * P1 * 16) : nullptr;
+      for (int t = grp; t < kTiles1; t += 2) {
+        mbar_wait(bar0 + 8 * t, ph);
+        fence_after();
+        conv1_epilogue(tmem, t, A2, b1, dbg1);
+      }
+      fence_proxy_async();  // conv1's epilogue wrote conv2's operand through the generic proxy
+      fence_before();
+      __syncthreads();
+
+      // ---- conv2: 2 tiles (one per warp group), then the FC
+      if (tid == 0) {
+        fence_after();
+        for (int u = 0; u < kTiles2; ++u) {
+          issue_conv2_tile(tmem, u, a2, w2);
+          mma_commit(bar0 + 8 * (7 + u));
+        }
+      }
+      __syncwarp();
+      mbar_wait(bar0 + 8 * (7 + grp), ph);
       fence_after();
       float* dbg2 = a.dbg_p2 ? a.dbg_p2 + (int64_t)j * NF : nullptr;
-      float acc = 0.0f;
-      for (int t = 0; t < 6; ++t) acc += conv2_epilogue(tmem, t * 32, (t / 3) * 8, (t % 3) * 8, b2, wfc, dbg2);
-      // ---- FC reduction -> logit -> Eq. (2) decision
+      float acc = conv2_epilogue(tmem, grp, b2, wfc, dbg2);
+      ph ^= 1u;
 #pragma unroll
       for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
       if (lane == 0) red[warp] = acc;
       fence_before();
       __syncthreads();
       if (tid == 0) {
-        const float logit = fc_bias + ((red[0] + red[1]) + (red[2] + red[3]));
+        float logit = fc_bias;
+#pragma unroll
+        for (int w = 0; w < kThreads / 32; ++w) logit += red[w];
         const FrameDesc fd = a.frames[f];
         const uint8_t p = logit >= fd.L_t ? 1 : 0;
         const uint8_t cls = logit < fd.L_low ? 0 : (logit > fd.L_high ? 2 : 1);
