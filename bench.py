@@ -51,7 +51,13 @@ CONFIGS = {
                   step_frames=30, period=300, on_len=150, seed=1004),
     "m5": dict(desc="M5: 256 streams 1920x1080 sharded over the GPUs, 1 target frame in 10", streams=256,
                W=1920, H=1080, pool_frames=10, step_frames=10, period=10, on_len=1, seed=1005, shard=True),
+    # standalone SNM (K4) run for its tensor-pipe roofline: delta_diff = 0 lets every frame
+    # through SDD, so one step scores 65,536 survivors across 256 streams (100x100 frames keep K1 small)
+    "snm": dict(desc="SNM microbenchmark: 65,536 survivors/step across 256 streams (100x100 frames, "
+                     "delta_diff = 0 so every frame reaches the SNM)", streams=256, W=100, H=100, pool_frames=256,
+                step_frames=256, period=300, on_len=30, seed=1006, delta=0.0),
 }
+SNM_FLOP = 7_477_632  # algorithmic FLOP per survivor
 DELTA, C_LOW, C_HIGH, FD, BATCH = 24.0, 0.2, 0.8, 0.5, 30
 
 
@@ -149,7 +155,8 @@ def run_ours(args, cfg, ws, rank, local):
     ctx = ff.Context(dev)
     streams = []
     for s in sids:
-        st = ctx.open_stream(width=W, height=H, delta_diff=DELTA, c_low=C_LOW, c_high=C_HIGH, filter_degree=FD,
+        st = ctx.open_stream(width=W, height=H, delta_diff=cfg.get("delta", DELTA), c_low=C_LOW, c_high=C_HIGH,
+                             filter_degree=FD,
                              snm_batch=BATCH)
         refs = torch.empty((32, H, P), dtype=torch.uint8, device=dev)
         synth.frames_cuda(video, torch.full((32,), s, dtype=torch.int32, device=dev),
@@ -180,8 +187,10 @@ def run_ours(args, cfg, ws, rank, local):
     for j, b in enumerate(batches):
         b.launch(cs)
         r = b.fetch(cs)
-        if int(r["sdd_pass"].sum()) != planted[j]:
-            raise RuntimeError(f"batch {j}: SDD passed {int(r['sdd_pass'].sum())} != planted {planted[j]}")
+        expect = planted[j] if cfg.get("delta", DELTA) == DELTA else frames_per_step
+        if int(r["sdd_pass"].sum()) != expect:
+            raise RuntimeError(f"batch {j}: SDD passed {int(r['sdd_pass'].sum())} != expected {expect}")
+        planted[j] = expect
     ctx.stats(reset=True)
 
     def step(i):
@@ -287,6 +296,14 @@ def run_ours(args, cfg, ws, rank, local):
                          "algorithmic_bytes_per_launch": k1_bytes,
                          "kernel_ms": {"K1_sdd": k_ms[0], "K3_compact": k_ms[1], "K4_snm": k_ms[2]},
                          "k1_share_of_step": k_ms[0] / max(1e-9, sum(k_ms))},
+            # K4 against the tensor roofline (algorithmic SNM FLOPs of this step's survivors / K4 time); the
+            # burst bf16 peak applies because K4 is timed alone (ffsva_batch_profile)
+            "snm_roofline": {"bound": "tensor", "kernel": "K4 snm_kernel (tcgen05 bf16, fp32 accumulate)",
+                             "survivors_per_launch": m_avg,
+                             "achieved": m_avg * SNM_FLOP / (k_ms[2] / 1e3) / 1e12 if k_ms[2] > 0 else 0.0,
+                             "peak": tf_peak, "unit": "TFLOP/s",
+                             "frac": (m_avg * SNM_FLOP / (k_ms[2] / 1e3) / 1e12) / tf_peak if k_ms[2] > 0 else 0.0,
+                             "peak_source": peak_kind, "survivors_per_s": m_avg / (k_ms[2] / 1e3) if k_ms[2] else 0},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
         }
     for b in batches:
