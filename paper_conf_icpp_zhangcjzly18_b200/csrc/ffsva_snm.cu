@@ -52,7 +52,8 @@ constexpr int OFF_A1 = 0;
 constexpr int OFF_A2 = OFF_A1 + A1_BYTES;                   // 55296
 constexpr int OFF_WB = OFF_A2 + A2_BYTES;                   // 84480
 constexpr int OFF_IN = OFF_WB + BLOB_BYTES;                 // 2 staging buffers
-constexpr int OFF_RED = OFF_IN + 2 * D50_BYTES;
+constexpr int OFF_LUT = OFF_IN + 2 * D50_BYTES;             // u16[256]: bf16 bits of (v - 128) / 128
+constexpr int OFF_RED = OFF_LUT + 512;
 constexpr int OFF_BAR = OFF_RED + 64;                       // 7 conv1 + 2 conv2 + 2 input mbarriers
 constexpr int OFF_TMEM = OFF_BAR + 16 * 8;
 constexpr int SMEM_BYTES = OFF_TMEM + 16;
@@ -163,7 +164,30 @@ __device__ __forceinline__ uint32_t u8_to_bf16(uint32_t v) {  // (v - 128) / 128
   return (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(((float)v - 128.0f) * 0.0078125f));
 }
 
-// ---------------------------------------------------------------- MMA issue (thread 0)
+// ---------------------------------------------------------------- input staging
+// D50 (50x50x3 u8, row-major) -> (v-128)/128 bf16 (C5, exact) into conv1's parity planes. Groups of 4 pixels =
+// 12 bytes = three aligned 32-bit shared loads; each channel through a 256-entry bf16 table.
+__device__ __forceinline__ void convert_input(const uint8_t* d, uint8_t* A1, const uint16_t* lut) {
+  constexpr int kGroups = snm::IN * snm::IN / 4;  // 625
+  for (int g = threadIdx.x; g < kGroups; g += kThreads) {
+    const uint32_t* w = reinterpret_cast<const uint32_t*>(d + 12 * g);
+    const uint32_t w0 = w[0], w1 = w[1], w2 = w[2];
+    const uint32_t b[12] = {w0 & 255u, (w0 >> 8) & 255u, (w0 >> 16) & 255u, w0 >> 24,
+                            w1 & 255u, (w1 >> 8) & 255u, (w1 >> 16) & 255u, w1 >> 24,
+                            w2 & 255u, (w2 >> 8) & 255u, (w2 >> 16) & 255u, w2 >> 24};
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const int p = 4 * g + q;
+      const int y = p / snm::IN, x = p - y * snm::IN;
+      const int Y = y + 1, X = x + 1;
+      const uint4 v = make_uint4((uint32_t)lut[b[3 * q]] | ((uint32_t)lut[b[3 * q + 1]] << 16),
+                                 (uint32_t)lut[b[3 * q + 2]], 0u, 0u);
+      *reinterpret_cast<uint4*>(A1 + ((Y & 1) * 2 + (X & 1)) * A1_PLANE + ((Y >> 1) * A1_COLS + (X >> 1)) * 16) = v;
+    }
+  }
+}
+
+// ---------------------------------------------------------------- MMA issue (one thread per warp group)
 __device__ __forceinline__ void issue_conv1_tile(uint32_t tmem, int t, uint32_t a1, uint32_t w1) {
   const int py0 = c1_py0[t];
   const uint32_t idesc = idesc_bf16(128, 16);
@@ -267,6 +291,8 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
   if (n_chunks == 0) return;  // no survivors in this batch
 
   for (int i = tid; i < (A1_BYTES + A2_BYTES) / 16; i += kThreads) reinterpret_cast<uint4*>(sm)[i] = make_uint4(0, 0, 0, 0);
+  uint16_t* lut = reinterpret_cast<uint16_t*>(sm + OFF_LUT);
+  lut[tid] = (uint16_t)u8_to_bf16((uint32_t)tid);  // kThreads == 256 entries
   if (tid == 0) {
     for (int i = 0; i < 11; ++i) mbar_init(bar0 + 8 * i, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -304,41 +330,30 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
     }
     const float fc_bias = __ldg(reinterpret_cast<const float*>(fd0.snm + OFF_BFC));
     uint32_t cnt_pass = 0, cnt_c0 = 0, cnt_c1 = 0, cnt_c2 = 0;
-    if (tid == 0) {  // stage the unit's first D50 image
+    if (tid == 0) {  // stage the unit's first two D50 images
       mbar_expect_tx(bar0 + 8 * 9, D50_BYTES);
       bulk_g2s(smem_addr(stage), a.d50 + (int64_t)a.work[start] * a.d50_stride, D50_BYTES, bar0 + 8 * 9);
+      if (start + 1 < end) {
+        mbar_expect_tx(bar0 + 8 * 10, D50_BYTES);
+        bulk_g2s(smem_addr(stage + D50_BYTES), a.d50 + (int64_t)a.work[start + 1] * a.d50_stride, D50_BYTES,
+                 bar0 + 8 * 10);
+      }
     }
+    mbar_wait(bar0 + 8 * 9, in_ph & 1u);
+    in_ph ^= 1u;
+    convert_input(stage, A1, lut);
+    fence_proxy_async();
+    const bool issuer = lane == 0 && (warp & 3) == 0;  // warp 0 issues group 0's tiles, warp 4 group 1's
     for (int j = start; j < end; ++j) {
       const int f = a.work[j];
       const int buf = (j - start) & 1;
-      if (tid == 0 && j + 1 < end) {  // prefetch the next frame of the unit
-        const uint32_t nb = bar0 + 8 * (9 + (buf ^ 1));
-        mbar_expect_tx(nb, D50_BYTES);
-        bulk_g2s(smem_addr(stage + (buf ^ 1) * D50_BYTES), a.d50 + (int64_t)a.work[j + 1] * a.d50_stride, D50_BYTES, nb);
-      }
-      mbar_wait(bar0 + 8 * (9 + buf), (in_ph >> buf) & 1u);
-      in_ph ^= 1u << buf;
-      // ---- D50 u8 -> (v-128)/128 bf16 into conv1's parity planes (pixel = 16 B: 3 channels + 5 zeros)
-      const uint8_t* d = stage + buf * D50_BYTES;
-      for (int p = tid; p < snm::IN * snm::IN; p += kThreads) {
-        const int y = p / snm::IN, x = p - y * snm::IN;
-        const int Y = y + 1, X = x + 1;
-        const uint32_t c0 = d[3 * p], c1 = d[3 * p + 1], c2 = d[3 * p + 2];
-        uint4 w;
-        w.x = u8_to_bf16(c0) | (u8_to_bf16(c1) << 16);
-        w.y = u8_to_bf16(c2);
-        w.z = 0u;
-        w.w = 0u;
-        *reinterpret_cast<uint4*>(A1 + ((Y & 1) * 2 + (X & 1)) * A1_PLANE + ((Y >> 1) * A1_COLS + (X >> 1)) * 16) = w;
-      }
-      fence_proxy_async();
       fence_before();
-      __syncthreads();
+      __syncthreads();  // frame j's conv1 operand (and the unit's weights) are in shared memory
 
-      // ---- conv1: 7 tiles, one commit each; epilogues start as tiles land
-      if (tid == 0) {
+      // ---- conv1: 7 tiles, each warp group issues and drains its own (one commit per tile)
+      if (issuer) {
         fence_after();
-        for (int t = 0; t < kTiles1; ++t) {
+        for (int t = grp; t < kTiles1; t += 2) {
           issue_conv1_tile(tmem, t, a1, w1);
           mma_commit(bar0 + 8 * t);
         }
@@ -352,17 +367,27 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
       }
       fence_proxy_async();  // conv1's epilogue wrote conv2's operand through the generic proxy
       fence_before();
-      __syncthreads();
+      __syncthreads();  // every conv1 tile has landed: conv1's operand is free again
 
-      // ---- conv2: 2 tiles (one per warp group), then the FC
-      if (tid == 0) {
+      // ---- conv2: one tile per warp group; while its MMAs run, stage frame j+1's conv1 operand
+      if (issuer) {
         fence_after();
-        for (int u = 0; u < kTiles2; ++u) {
-          issue_conv2_tile(tmem, u, a2, w2);
-          mma_commit(bar0 + 8 * (7 + u));
-        }
+        issue_conv2_tile(tmem, grp, a2, w2);
+        mma_commit(bar0 + 8 * (7 + grp));
       }
       __syncwarp();
+      if (j + 1 < end) {
+        const int nb = buf ^ 1;
+        mbar_wait(bar0 + 8 * (9 + nb), (in_ph >> nb) & 1u);
+        in_ph ^= 1u << nb;
+        convert_input(stage + nb * D50_BYTES, A1, lut);
+        fence_proxy_async();
+      }
+      if (tid == 0 && j + 2 < end) {  // frame j's staging buffer is consumed: prefetch frame j+2 into it
+        mbar_expect_tx(bar0 + 8 * (9 + buf), D50_BYTES);
+        bulk_g2s(smem_addr(stage + buf * D50_BYTES), a.d50 + (int64_t)a.work[j + 2] * a.d50_stride, D50_BYTES,
+                 bar0 + 8 * (9 + buf));
+      }
       mbar_wait(bar0 + 8 * (7 + grp), ph);
       fence_after();
       float* dbg2 = a.dbg_p2 ? a.dbg_p2 + (int64_t)j * NF : nullptr;
