@@ -177,6 +177,45 @@ FFSVA_API ffsva_status ffsva_stream_info(ffsva_stream* s, int32_t* slot, int32_t
 FFSVA_API ffsva_status ffsva_stats_copy(int32_t device, uint64_t* dst, int32_t max_slots, int32_t* slots,
                                         int32_t dst_is_host, int32_t reset, void* cuda_stream);
 
+/* ---------------------------------------------------------------------------------------------------------
+ * Online runtime (§4.3): per-stream SDD and SNM queues (L143), the global feedback queue (L209, L217)
+ * and dynamic batching (L223), driving the same kernels cycle by cycle.
+ *   push  — a stream's prefetcher hands over frames; a frame is refused (accepted[i] = 0, the caller keeps it:
+ *           the prefetcher is "blocked") while that stream's SDD queue holds more than q_sdd frames;
+ *   tick  — one cycle: the SDD stage admits queued frames round-robin (at most max_frames_per_tick, at most the
+ *           free SNM slots), skipping a stream while its SNM queue holds more than q_snm frames; survivors join
+ *           the stream's SNM queue (their 50x50 images stay in a device slot pool); then every non-empty SNM
+ *           queue pops min(BatchSize, depth) frames and the SNM scores all pops in one launch. Frames whose fate
+ *           is decided (dropped by SDD, or scored by SNM) are reported as events, oldest first; events beyond
+ *           `cap` are kept for the next tick. Synchronous on cuda_stream.
+ * The SNM stage feeds T-YOLO in the paper, which is out of scope: nothing blocks it here. Frames must stay valid
+ * until their event is reported. Streams must be open on the scheduler's device and carry a reference and an
+ * SNM; a stream is attached on its first push and must not be closed while it has queued frames. */
+typedef struct ffsva_sched ffsva_sched;
+typedef struct {
+  ffsva_stream* stream;
+  int64_t frame_no;
+  ffsva_result result;       /* survivor_idx = -1 (ranks are a batch notion) */
+} ffsva_event;
+typedef struct {
+  int32_t admitted;          /* frames through SDD this cycle */
+  int32_t sdd_pass;          /* of which survivors */
+  int32_t snm_scored;        /* frames scored by the SNM this cycle */
+  int32_t snm_batches;       /* dynamic batches (pops) this cycle */
+  int32_t sdd_blocked;       /* streams skipped by the SDD stage because their SNM queue was over q_snm */
+  int64_t sdd_queued;        /* frames waiting in SDD queues after the cycle */
+  int64_t snm_queued;        /* frames waiting in SNM queues after the cycle */
+  int64_t events_pending;    /* events not yet returned */
+} ffsva_tick_info;
+
+FFSVA_API ffsva_status ffsva_sched_create(int32_t device, int32_t max_frames_per_tick, int32_t snm_slots,
+                                          ffsva_sched** out);
+FFSVA_API ffsva_status ffsva_sched_push(ffsva_sched* s, const ffsva_frame* frames, int32_t n, uint8_t* accepted);
+FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva_event* events, int32_t cap,
+                                        int32_t* n_events, ffsva_tick_info* info);
+FFSVA_API ffsva_status ffsva_sched_depth(ffsva_sched* s, ffsva_stream* st, int32_t* sdd_depth, int32_t* snm_depth);
+FFSVA_API ffsva_status ffsva_sched_destroy(ffsva_sched* s);
+
 /* Close a stream (NULL is a no-op). */
 FFSVA_API ffsva_status ffsva_close(ffsva_stream* s);
 

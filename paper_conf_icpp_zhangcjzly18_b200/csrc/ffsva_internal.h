@@ -50,8 +50,9 @@ struct SddArgs {
   const FrameDesc* frames;
   int32_t n;
   int32_t sdd_w, sdd_h;      // grid (uniform over the batch)
-  uint8_t* d50;              // [n][d50_stride]
+  uint8_t* d50;              // [n][d50_stride], or a slot pool addressed through d50_index
   int64_t d50_stride;
+  const int32_t* d50_index;  // optional [n]: frame f's D50 goes to slot d50_index[f] (online queues)
   uint8_t* d100;             // optional [n][sdd_h*sdd_w*3]
   unsigned long long* acc_ssd; // [n] per-frame SSD accumulator: zero on entry; K3 reads it and re-zeroes it
   unsigned long long* stats; // [slots][NSTAT] or nullptr
@@ -99,9 +100,12 @@ struct SnmArgs {
   const FrameDesc* frames;
   const uint8_t* d50;
   int64_t d50_stride;
+  const int32_t* d50_index;  // optional [n]: frame f's D50 image is slot d50_index[f]
   const int32_t* work;
   const int32_t* chunks;
   int32_t* counts;           // m, n_chunks, cursor
+  const uint8_t* pop_start;  // optional [n_chunks]: 1 if the unit opens a dynamic batch (online mode counts
+                             // SNM_BATCHES here; batch mode counts them in K3)
   float* logit;              // [n] (frame order)
   uint8_t* snm_pass;
   uint8_t* snm_class;

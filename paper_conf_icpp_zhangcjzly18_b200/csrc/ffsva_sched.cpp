@@ -1,0 +1,404 @@
+// ffsva_sched.cpp — online runtime: the FFS-VA queue policy (ffsva_sched_policy.h) driving K1 -> K3 -> K4.
+//
+// One tick = one SDD cycle + one SNM cycle (§4.3):
+//   1. admit SDD-queued frames (feedback: streams whose SNM queue is over q_snm wait), give each a D50 slot;
+//   2. K1 writes each admitted frame's 50x50 image into its slot, K3 thresholds the SSD per frame;
+//   3. survivors join their stream's SNM queue, dropped frames become events and free their slot;
+//   4. every non-empty SNM queue pops min(BatchSize, depth) (dynamic batching); K4 scores all pops in one
+//      launch, reading the images from their slots; scored frames become events and free their slots.
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <deque>
+#include <memory>
+#include <unordered_map>
+#include <vector>
+
+#include "ffsva_runtime.h"
+#include "ffsva_sched_policy.h"
+
+using namespace ffsva;
+
+namespace {
+constexpr int64_t kD50Stride = 7504;
+size_t al256(size_t x) { return (x + 255) & ~(size_t)255; }
+
+// Per-cycle staging: one pinned host block mirrored by one device block (a single H2D per stage).
+struct Layout {
+  size_t desc, index, work, chunks, counts, seg_lo, seg_batch, seg_slot, pop_start, total;
+  explicit Layout(size_t n) {
+    size_t o = 0;
+    desc = o; o += al256(64 * n);
+    index = o; o += al256(4 * n);
+    work = o; o += al256(4 * n);
+    chunks = o; o += al256(4 * (n + 1));
+    counts = o; o += al256(16);
+    seg_lo = o; o += al256(4 * (n + 1));
+    seg_batch = o; o += al256(4 * n);
+    seg_slot = o; o += al256(4 * n);
+    pop_start = o; o += al256(n);
+    total = o;
+  }
+};
+}  // namespace
+
+struct ffsva_sched {
+  DeviceCtx* ctx = nullptr;
+  std::mutex mu;
+  sched::Policy pol;
+  std::unordered_map<ffsva_stream*, int32_t> ids;
+  std::vector<ffsva_stream*> by_id;
+  int32_t max_frames = 0, slots = 0, cap = 0;
+  int32_t sdd_w = -1, sdd_h = -1;
+  std::vector<int32_t> free_slots;
+  uint8_t* d_pool = nullptr;  // [slots][7504] D50 images of frames between SDD and SNM
+  uint8_t* d_in = nullptr;    // Layout(cap) mirror of h_in
+  uint8_t* h_in = nullptr;
+  // device scratch / outputs
+  void* d_mem = nullptr;
+  int32_t *d_perm = nullptr, *d_posw = nullptr, *d_surv = nullptr;
+  unsigned long long* d_acc = nullptr;
+  uint8_t* d_out = nullptr;   // ssd u64[cap] | logit f32[cap] | pass u8[cap] | snm_pass u8[cap] | snm_class u8[cap]
+  uint8_t* h_out = nullptr;
+  std::deque<ffsva_event> pending;
+};
+
+namespace {
+
+void sched_free(ffsva_sched* s) {
+  cudaFree(s->d_pool);
+  cudaFree(s->d_in);
+  cudaFree(s->d_mem);
+  cudaFreeHost(s->h_in);
+  cudaFreeHost(s->h_out);
+}
+
+FrameDesc make_desc(const ffsva_stream* st, const void* pixels) {
+  FrameDesc d{};
+  d.pixels = (const uint8_t*)pixels;
+  d.ref = st->d_ref;
+  d.snm = st->d_snm;
+  d.pitch = st->desc.row_pitch;
+  d.T = st->T;
+  d.W = st->desc.width;
+  d.H = st->desc.height;
+  d.L_t = st->L_t;
+  d.L_low = st->L_low;
+  d.L_high = st->L_high;
+  d.slot = st->slot;
+  return d;
+}
+
+template <typename T>
+T* at(uint8_t* base, size_t off) { return reinterpret_cast<T*>(base + off); }
+
+}  // namespace
+
+extern "C" {
+
+FFSVA_API ffsva_status ffsva_sched_create(int32_t device, int32_t max_frames_per_tick, int32_t snm_slots,
+                                          ffsva_sched** out) {
+  if (!out || max_frames_per_tick < 1 || snm_slots < 1) return fail(FFSVA_EINVAL, "bad argument");
+  ffsva_status st;
+  DeviceCtx* ctx = ctx_acquire(device, &st);  // the scheduler holds a context reference until destroyed
+  if (!ctx) return st;
+  std::unique_ptr<ffsva_sched> s(new ffsva_sched());
+  s->ctx = ctx;
+  s->max_frames = max_frames_per_tick;
+  s->slots = snm_slots;
+  s->cap = std::max(max_frames_per_tick, snm_slots);
+  const size_t n = (size_t)s->cap;
+  const Layout L(n);
+  DeviceGuard g(device);
+  const size_t o_perm = 0, o_posw = al256(4 * n), o_surv = o_posw + al256(4 * (n + 1)),
+               o_acc = o_surv + al256(4 * n), o_out = o_acc + al256(8 * n), total = o_out + al256(15 * n);
+  cudaError_t e = cudaMalloc(&s->d_mem, total);
+  if (e == cudaSuccess) e = cudaMalloc(&s->d_pool, (size_t)snm_slots * kD50Stride);
+  if (e == cudaSuccess) e = cudaMalloc(&s->d_in, L.total);
+  if (e == cudaSuccess) e = cudaMallocHost(&s->h_in, L.total);
+  if (e == cudaSuccess) e = cudaMallocHost(&s->h_out, 15 * n);
+  if (e == cudaSuccess) {
+    uint8_t* b = (uint8_t*)s->d_mem;
+    s->d_perm = at<int32_t>(b, o_perm);
+    s->d_posw = at<int32_t>(b, o_posw);
+    s->d_surv = at<int32_t>(b, o_surv);
+    s->d_acc = at<unsigned long long>(b, o_acc);
+    s->d_out = b + o_out;
+    std::vector<int32_t> ident(n);
+    for (size_t i = 0; i < n; ++i) ident[i] = (int32_t)i;
+    e = cudaMemcpy(s->d_perm, ident.data(), 4 * n, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemset(s->d_acc, 0, 8 * n);
+  }
+  if (e != cudaSuccess) {
+    sched_free(s.get());
+    ctx_release(ctx);
+    return cuda_fail(nullptr, e, "ffsva_sched_create");
+  }
+  for (int32_t i = snm_slots - 1; i >= 0; --i) s->free_slots.push_back(i);
+  *out = s.release();
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_sched_destroy(ffsva_sched* s) {
+  if (!s) return FFSVA_OK;
+  DeviceCtx* ctx = s->ctx;
+  {
+    DeviceGuard g(ctx->device);
+    cudaDeviceSynchronize();
+    sched_free(s);
+  }
+  delete s;
+  ctx_release(ctx);
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_sched_push(ffsva_sched* s, const ffsva_frame* frames, int32_t n, uint8_t* accepted) {
+  if (!s || n < 0 || (n > 0 && (!frames || !accepted))) return fail(FFSVA_EINVAL, "bad argument");
+  std::lock_guard<std::mutex> lk(s->mu);
+  for (int32_t i = 0; i < n; ++i) {  // validate everything before queueing anything
+    ffsva_stream* st = frames[i].stream;
+    if (!st || !frames[i].pixels) return fail(FFSVA_EINVAL, "frame without stream or pixels");
+    if (st->ctx != s->ctx) return fail(FFSVA_EDEVICE, "stream lives on another device");
+    if (!st->has_ref || !st->has_snm) return fail(FFSVA_ESTATE, "stream has no reference image or no SNM");
+    if (st->desc.snm_w != snm::IN || st->desc.snm_h != snm::IN) return fail(FFSVA_EINVAL, "SNM grid must be 50x50");
+    if (s->sdd_w < 0) {  // one SDD grid per scheduler (one K1 launch per cycle)
+      s->sdd_w = st->desc.sdd_w;
+      s->sdd_h = st->desc.sdd_h;
+    }
+    if (st->desc.sdd_w != s->sdd_w || st->desc.sdd_h != s->sdd_h)
+      return fail(FFSVA_EINVAL, "streams of one scheduler must share the SDD grid");
+  }
+  for (int32_t i = 0; i < n; ++i) {
+    ffsva_stream* st = frames[i].stream;
+    auto it = s->ids.find(st);
+    int32_t id;
+    if (it == s->ids.end()) {
+      id = s->pol.add_stream(st->desc.q_sdd, st->desc.q_snm, st->desc.snm_batch);
+      s->ids[st] = id;
+      if ((int32_t)s->by_id.size() <= id) s->by_id.resize(id + 1, nullptr);
+      s->by_id[id] = st;
+    } else {
+      id = it->second;
+    }
+    sched::QFrame q;
+    q.frame_no = frames[i].frame_no;
+    q.pixels = frames[i].pixels;
+    accepted[i] = s->pol.push(id, q) ? 1 : 0;
+  }
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_sched_depth(ffsva_sched* s, ffsva_stream* st, int32_t* sdd_depth, int32_t* snm_depth) {
+  if (!s || !st) return fail(FFSVA_EINVAL, "bad argument");
+  std::lock_guard<std::mutex> lk(s->mu);
+  auto it = s->ids.find(st);
+  if (sdd_depth) *sdd_depth = it == s->ids.end() ? 0 : (int32_t)s->pol.stream(it->second).sdd.size();
+  if (snm_depth) *snm_depth = it == s->ids.end() ? 0 : (int32_t)s->pol.stream(it->second).snm.size();
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva_event* events, int32_t cap,
+                                        int32_t* n_events, ffsva_tick_info* info) {
+  if (!s || cap < 0 || (cap > 0 && !events) || !n_events) return fail(FFSVA_EINVAL, "bad argument");
+  std::lock_guard<std::mutex> lk(s->mu);
+  DeviceCtx* ctx = s->ctx;
+  if (ctx->sticky) return fail(FFSVA_ECUDA, "device is in a sticky CUDA error state");
+  std::lock_guard<std::mutex> dlk(ctx->mu);
+  DeviceGuard g(ctx->device);
+  cudaStream_t cs = (cudaStream_t)cuda_stream;
+  const size_t n = (size_t)s->cap;
+  const Layout L(n);
+  uint8_t* h = s->h_in;
+  ffsva_tick_info ti{};
+  uint64_t blocked0 = 0;
+  for (int32_t i = 0; i < s->pol.n_streams(); ++i) blocked0 += s->pol.stream(i).sdd_blocked;
+  cudaError_t e = cudaSuccess;
+  uint64_t* h_ssd = at<uint64_t>(s->h_out, 0);
+  float* h_logit = at<float>(s->h_out, 8 * n);
+  uint8_t* h_pass = s->h_out + 12 * n;
+  uint8_t* h_snm_pass = s->h_out + 13 * n;
+  uint8_t* h_snm_class = s->h_out + 14 * n;
+
+  // ---------------- SDD cycle (admitted frames arrive grouped by stream: one K3 segment per stream)
+  std::vector<sched::QFrame> adm = s->pol.admit_sdd(s->max_frames, (int32_t)s->free_slots.size());
+  const int32_t na = (int32_t)adm.size();
+  ti.admitted = na;
+  if (na > 0) {
+    FrameDesc* hd = at<FrameDesc>(h, L.desc);
+    int32_t* hidx = at<int32_t>(h, L.index);
+    int32_t* hseg = at<int32_t>(h, L.seg_lo);
+    int32_t* hsegb = at<int32_t>(h, L.seg_batch);
+    int32_t* hsegs = at<int32_t>(h, L.seg_slot);
+    int32_t max_chunks = 1, stage = 0, nseg = 0;
+    const int32_t sdd_w = s->by_id[adm[0].stream]->desc.sdd_w, sdd_h = s->by_id[adm[0].stream]->desc.sdd_h;
+    bool vec16 = true;
+    for (int32_t i = 0; i < na; ++i) {
+      const ffsva_stream* st = s->by_id[adm[i].stream];
+      adm[i].slot = s->free_slots.back();
+      s->free_slots.pop_back();
+      hd[i] = make_desc(st, adm[i].pixels);
+      hidx[i] = adm[i].slot;
+      if (i == 0 || adm[i].stream != adm[i - 1].stream) {
+        hseg[nseg] = i;
+        hsegb[nseg] = st->desc.snm_batch;
+        hsegs[nseg] = st->slot;
+        ++nseg;
+      }
+      max_chunks = std::max(max_chunks, (3 * st->desc.width + 15) / 16);
+      stage = std::max(stage, sdd_bulk_stage_bytes(st->desc.width, st->desc.height, sdd_h));
+      if ((st->desc.row_pitch & 15) || ((uintptr_t)adm[i].pixels & 15)) vec16 = false;
+    }
+    hseg[nseg] = na;
+    const bool bulk = vec16 && sdd_bulk_ok(max_chunks, stage);
+    e = sdd_configure(bulk ? sdd_bulk_smem_bytes(stage, sdd_w) : sdd_smem_bytes(max_chunks, sdd_w));
+    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in, h, L.total, cudaMemcpyHostToDevice, cs);
+    SddArgs sa{};
+    sa.frames = at<FrameDesc>(s->d_in, L.desc);
+    sa.n = na;
+    sa.sdd_w = sdd_w;
+    sa.sdd_h = sdd_h;
+    sa.d50 = s->d_pool;
+    sa.d50_stride = kD50Stride;
+    sa.d50_index = at<int32_t>(s->d_in, L.index);
+    sa.acc_ssd = s->d_acc;
+    sa.stats = ctx->d_stats;
+    sa.max_chunks = max_chunks;
+    sa.vec16 = vec16;
+    sa.bulk = bulk;
+    sa.stage_bytes = stage;
+    if (e == cudaSuccess) e = launch_sdd(sa, cs);
+    CompactArgs ca{};  // threshold + per-stream SDD-pass stats; no SNM work units (snm_ctas = 0)
+    ca.frames = sa.frames;
+    ca.acc_ssd = s->d_acc;
+    ca.ssd = at<uint64_t>(s->d_out, 0);
+    ca.pass = s->d_out + 12 * n;
+    ca.n = na;
+    ca.perm = s->d_perm;
+    ca.seg_lo = at<int32_t>(s->d_in, L.seg_lo);
+    ca.n_seg = nseg;
+    ca.seg_batch = at<int32_t>(s->d_in, L.seg_batch);
+    ca.seg_slot = at<int32_t>(s->d_in, L.seg_slot);
+    ca.stats = ctx->d_stats;
+    ca.snm_ctas = 0;
+    ca.survivor_idx = s->d_surv;
+    ca.work = at<int32_t>(s->d_in, L.work);
+    ca.posw = s->d_posw;
+    ca.chunks = at<int32_t>(s->d_in, L.chunks);
+    ca.counts = at<int32_t>(s->d_in, L.counts);
+    ca.logit = at<float>(s->d_out, 8 * n);
+    ca.snm_pass = s->d_out + 13 * n;
+    ca.snm_class = s->d_out + 14 * n;
+    if (e == cudaSuccess) e = launch_compact(ca, cs);
+    g_launches += 2;
+    if (e == cudaSuccess) e = cudaMemcpyAsync(h_ssd, ca.ssd, 8 * (size_t)na, cudaMemcpyDeviceToHost, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(h_pass, ca.pass, (size_t)na, cudaMemcpyDeviceToHost, cs);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (SDD cycle)");
+    for (int32_t i = 0; i < na; ++i) {
+      adm[i].ssd = h_ssd[i];
+      s->pol.sdd_done(adm[i], h_pass[i] != 0);
+      if (h_pass[i]) {
+        ++ti.sdd_pass;
+        continue;
+      }
+      ffsva_event ev{};
+      ev.stream = s->by_id[adm[i].stream];
+      ev.frame_no = adm[i].frame_no;
+      ev.result.ssd = h_ssd[i];
+      ev.result.logit = NAN;
+      ev.result.survivor_idx = -1;
+      s->pending.push_back(ev);
+      s->free_slots.push_back(adm[i].slot);
+    }
+  }
+
+  // ---------------- SNM cycle: dynamic batching (pops of min(BatchSize, depth) per stream)
+  std::vector<std::vector<sched::QFrame>> pops = s->pol.pop_snm();
+  int32_t m = 0;
+  for (auto& p : pops) m += (int32_t)p.size();
+  ti.snm_batches = (int32_t)pops.size();
+  ti.snm_scored = m;
+  if (m > 0) {
+    FrameDesc* hd = at<FrameDesc>(h, L.desc);
+    int32_t* hidx = at<int32_t>(h, L.index);
+    int32_t* hwork = at<int32_t>(h, L.work);
+    int32_t* hch = at<int32_t>(h, L.chunks);
+    int32_t* hcnt = at<int32_t>(h, L.counts);
+    uint8_t* hpop = h + L.pop_start;
+    std::vector<sched::QFrame> flat;
+    flat.reserve(m);
+    int32_t j = 0, nch = 0;
+    for (auto& p : pops) {
+      const ffsva_stream* st = s->by_id[p[0].stream];
+      // a pop is split into work units of U frames so small cycles still spread over the SMs
+      const int32_t U = std::max(1, std::min(st->desc.snm_batch, m / std::max(1, ctx->num_sms)));
+      for (int32_t k = 0; k < (int32_t)p.size(); ++k) {
+        if (k % U == 0) {
+          hpop[nch] = k == 0 ? 1 : 0;
+          hch[nch++] = j;
+        }
+        hd[j] = make_desc(st, nullptr);
+        hidx[j] = p[k].slot;
+        hwork[j] = j;
+        flat.push_back(p[k]);
+        ++j;
+      }
+    }
+    hch[nch] = m;
+    hcnt[0] = m;
+    hcnt[1] = nch;
+    hcnt[2] = 0;
+    hcnt[3] = 0;
+    e = cudaMemcpyAsync(s->d_in, h, L.total, cudaMemcpyHostToDevice, cs);
+    SnmArgs na{};
+    na.frames = at<FrameDesc>(s->d_in, L.desc);
+    na.d50 = s->d_pool;
+    na.d50_stride = kD50Stride;
+    na.d50_index = at<int32_t>(s->d_in, L.index);
+    na.work = at<int32_t>(s->d_in, L.work);
+    na.chunks = at<int32_t>(s->d_in, L.chunks);
+    na.counts = at<int32_t>(s->d_in, L.counts);
+    na.pop_start = s->d_in + L.pop_start;
+    na.logit = at<float>(s->d_out, 8 * n);
+    na.snm_pass = s->d_out + 13 * n;
+    na.snm_class = s->d_out + 14 * n;
+    na.stats = ctx->d_stats;
+    na.grid = std::max(1, std::min(nch, ctx->num_sms));
+    if (e == cudaSuccess) e = launch_snm(na, cs);
+    g_launches += 1;
+    if (e == cudaSuccess) e = cudaMemcpyAsync(h_logit, na.logit, 4 * (size_t)m, cudaMemcpyDeviceToHost, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(h_snm_pass, na.snm_pass, 2 * n, cudaMemcpyDeviceToHost, cs);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (SNM cycle)");
+    for (int32_t k = 0; k < m; ++k) {
+      ffsva_event ev{};
+      ev.stream = s->by_id[flat[k].stream];
+      ev.frame_no = flat[k].frame_no;
+      ev.result.ssd = flat[k].ssd;
+      ev.result.sdd_pass = 1;
+      ev.result.snm_pass = h_snm_pass[k];
+      ev.result.snm_class = h_snm_class[k];
+      ev.result.logit = h_logit[k];
+      ev.result.survivor_idx = -1;
+      s->pending.push_back(ev);
+      s->free_slots.push_back(flat[k].slot);
+    }
+  }
+
+  uint64_t blocked1 = 0;
+  for (int32_t i = 0; i < s->pol.n_streams(); ++i) blocked1 += s->pol.stream(i).sdd_blocked;
+  ti.sdd_blocked = (int32_t)(blocked1 - blocked0);
+  int32_t k = 0;
+  while (k < cap && !s->pending.empty()) {
+    events[k++] = s->pending.front();
+    s->pending.pop_front();
+  }
+  *n_events = k;
+  ti.sdd_queued = s->pol.queued_sdd();
+  ti.snm_queued = s->pol.queued_snm();
+  ti.events_pending = (int64_t)s->pending.size();
+  if (info) *info = ti;
+  return FFSVA_OK;
+}
+
+}  // extern "C"

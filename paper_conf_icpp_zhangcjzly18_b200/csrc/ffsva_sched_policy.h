@@ -1,0 +1,150 @@
+// ffsva_sched_policy.h — the online queue policy of FFS-VA (§4.3), host-only and CUDA-free (unit-tested
+// on CPU by tests/test_sched_policy.py through tests/sched_policy_test.cpp).
+//
+//   * per-stream queues between consecutive stages (L143): an SDD queue (frames waiting for SDD) and an SNM
+//     queue (SDD survivors waiting for the SNM);
+//   * global feedback queue (L209, L217): a stage stops pulling from its input while the queue of the stage
+//     after it holds more than that queue's depth threshold. Thresholds are per stream, in frames (reading
+//     Q18): the prefetcher is refused while the SDD queue holds more than q_sdd frames (default 2); the SDD
+//     stage skips a stream while its SNM queue holds more than q_snm frames (default 10). The SNM stage feeds
+//     T-YOLO, which is out of scope, so nothing blocks it;
+//   * dynamic batching (L223): each SNM cycle pops min(BatchSize, depth) frames of every non-empty stream.
+// Streams are visited round-robin (the start rotates every cycle) so a per-cycle frame budget is shared fairly.
+#pragma once
+
+#include <algorithm>
+#include <cstdint>
+#include <deque>
+#include <vector>
+
+namespace ffsva {
+namespace sched {
+
+struct QFrame {
+  int32_t stream = -1;        // policy stream id
+  int64_t frame_no = 0;       // caller's frame number
+  const void* pixels = nullptr;
+  int32_t slot = -1;          // device D50 slot while the frame sits in the SNM queue
+  uint64_t ssd = 0;           // SDD distance, carried to the frame's final event
+};
+
+struct StreamQ {
+  int32_t q_sdd = 2, q_snm = 10, batch = 30;
+  bool live = false;
+  std::deque<QFrame> sdd, snm;
+  uint64_t pushed = 0, refused = 0, sdd_blocked = 0;
+  int32_t max_sdd = 0, max_snm = 0;
+};
+
+class Policy {
+ public:
+  int32_t add_stream(int32_t q_sdd, int32_t q_snm, int32_t batch) {
+    int32_t id = -1;
+    for (int32_t i = 0; i < (int32_t)st_.size(); ++i)
+      if (!st_[i].live) { id = i; break; }
+    if (id < 0) { id = (int32_t)st_.size(); st_.emplace_back(); }
+    StreamQ& s = st_[id];
+    s = StreamQ();
+    s.q_sdd = q_sdd;
+    s.q_snm = q_snm;
+    s.batch = batch < 1 ? 1 : batch;
+    s.live = true;
+    return id;
+  }
+
+  // Frames still queued are returned so the caller can release their device slots.
+  std::vector<QFrame> remove_stream(int32_t id) {
+    std::vector<QFrame> out;
+    if (id < 0 || id >= (int32_t)st_.size()) return out;
+    StreamQ& s = st_[id];
+    out.insert(out.end(), s.sdd.begin(), s.sdd.end());
+    out.insert(out.end(), s.snm.begin(), s.snm.end());
+    s = StreamQ();
+    return out;
+  }
+
+  bool live(int32_t id) const { return id >= 0 && id < (int32_t)st_.size() && st_[id].live; }
+
+  // The prefetcher of a stream is blocked while its SDD queue holds more than q_sdd frames (L209, L217).
+  bool push(int32_t id, const QFrame& f) {
+    StreamQ& s = st_[id];
+    if ((int32_t)s.sdd.size() > s.q_sdd) {
+      ++s.refused;
+      return false;
+    }
+    QFrame g = f;
+    g.stream = id;
+    s.sdd.push_back(g);
+    ++s.pushed;
+    s.max_sdd = std::max(s.max_sdd, (int32_t)s.sdd.size());
+    return true;
+  }
+
+  // SDD stage of one cycle: round-robin over streams; a stream whose SNM queue holds more than q_snm frames is
+  // skipped (feedback, L209); otherwise its queued frames are admitted in order, at most `budget` in total and
+  // at most `snm_room` that could still land in the SNM queue (device D50 slots).
+  std::vector<QFrame> admit_sdd(int32_t budget, int32_t snm_room) {
+    std::vector<QFrame> out;
+    const int32_t n = (int32_t)st_.size();
+    if (n == 0) return out;
+    int32_t limit = std::min(budget, snm_room);
+    for (int32_t k = 0; k < n && limit > 0; ++k) {
+      StreamQ& s = st_[(rr_ + k) % n];
+      if (!s.live || s.sdd.empty()) continue;
+      if ((int32_t)s.snm.size() > s.q_snm) {
+        ++s.sdd_blocked;
+        continue;
+      }
+      while (!s.sdd.empty() && limit > 0) {
+        out.push_back(s.sdd.front());
+        s.sdd.pop_front();
+        --limit;
+      }
+    }
+    rr_ = (rr_ + 1) % n;
+    return out;
+  }
+
+  // An admitted frame's SDD verdict: survivors join their stream's SNM queue in arrival order (L143).
+  void sdd_done(const QFrame& f, bool pass) {
+    if (!pass) return;
+    StreamQ& s = st_[f.stream];
+    s.snm.push_back(f);
+    s.max_snm = std::max(s.max_snm, (int32_t)s.snm.size());
+  }
+
+  // SNM stage of one cycle (dynamic batching, L223): every non-empty stream pops min(BatchSize, depth).
+  std::vector<std::vector<QFrame>> pop_snm() {
+    std::vector<std::vector<QFrame>> pops;
+    const int32_t n = (int32_t)st_.size();
+    for (int32_t k = 0; k < n; ++k) {
+      StreamQ& s = st_[k];
+      if (!s.live || s.snm.empty()) continue;
+      const int32_t take = std::min<int32_t>(s.batch, (int32_t)s.snm.size());
+      std::vector<QFrame> pop(s.snm.begin(), s.snm.begin() + take);
+      s.snm.erase(s.snm.begin(), s.snm.begin() + take);
+      pops.push_back(std::move(pop));
+    }
+    return pops;
+  }
+
+  const StreamQ& stream(int32_t id) const { return st_[id]; }
+  int32_t n_streams() const { return (int32_t)st_.size(); }
+  int64_t queued_sdd() const {
+    int64_t q = 0;
+    for (auto& s : st_) q += (int64_t)s.sdd.size();
+    return q;
+  }
+  int64_t queued_snm() const {
+    int64_t q = 0;
+    for (auto& s : st_) q += (int64_t)s.snm.size();
+    return q;
+  }
+
+ private:
+  std::vector<StreamQ> st_;
+  int32_t rr_ = 0;
+};
+
+}  // namespace sched
+}  // namespace ffsva

@@ -239,7 +239,8 @@ __global__ void __launch_bounds__(512) sdd_kernel(SddArgs a) {
     const uint32_t s = cell[6 * cx + ch] + cell[6 * cx + 3 + ch] + cell[row3 + 6 * cx + ch] +
                        cell[row3 + 6 * cx + 3 + ch];
     const uint32_t n = (uint32_t)(xb[2 * cx + 2] - xb[2 * cx]) * (uint32_t)rows;
-    a.d50[(int64_t)f * a.d50_stride + (int64_t)band * half3 + o] = (uint8_t)((s + (n >> 1)) / n);
+    const int64_t slot = a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f;
+    a.d50[slot * a.d50_stride + (int64_t)band * half3 + o] = (uint8_t)((s + (n >> 1)) / n);
   }
   ssd_commit(ssd_local, red, a, f, fd.slot, band == 0);
 }
@@ -403,7 +404,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
       const int cx = o / 3, ch = o - 3 * cx;
       const uint32_t s = cell[6 * cx + ch] + cell[6 * cx + 3 + ch] + pair_in[o];
       const uint32_t n = (uint32_t)(xb[2 * cx + 2] - xb[2 * cx]) * (uint32_t)(yb - y0);
-      a.d50[(int64_t)f * a.d50_stride + (int64_t)(r >> 1) * half3 + o] = (uint8_t)((s + (n >> 1)) / n);
+      const int64_t slot = a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f;
+      a.d50[slot * a.d50_stride + (int64_t)(r >> 1) * half3 + o] = (uint8_t)((s + (n >> 1)) / n);
     }
   }
   ssd_commit(ssd_local, red, a, f, fd.slot, r == 0);

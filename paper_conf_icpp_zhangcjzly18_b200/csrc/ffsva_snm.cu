@@ -164,6 +164,10 @@ __device__ __forceinline__ uint32_t u8_to_bf16(uint32_t v) {  // (v - 128) / 128
   return (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(((float)v - 128.0f) * 0.0078125f));
 }
 
+__device__ __forceinline__ const uint8_t* d50_of(const SnmArgs& a, int f) {
+  return a.d50 + (a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f) * a.d50_stride;
+}
+
 // ---------------------------------------------------------------- input staging
 // D50 (50x50x3 u8, row-major) -> (v-128)/128 bf16 (C5, exact) into conv1's parity planes. Groups of 4 pixels =
 // 12 bytes = three aligned 32-bit shared loads; each channel through a 256-entry bf16 table.
@@ -332,11 +336,10 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
     uint32_t cnt_pass = 0, cnt_c0 = 0, cnt_c1 = 0, cnt_c2 = 0;
     if (tid == 0) {  // stage the unit's first two D50 images
       mbar_expect_tx(bar0 + 8 * 9, D50_BYTES);
-      bulk_g2s(smem_addr(stage), a.d50 + (int64_t)a.work[start] * a.d50_stride, D50_BYTES, bar0 + 8 * 9);
+      bulk_g2s(smem_addr(stage), d50_of(a, a.work[start]), D50_BYTES, bar0 + 8 * 9);
       if (start + 1 < end) {
         mbar_expect_tx(bar0 + 8 * 10, D50_BYTES);
-        bulk_g2s(smem_addr(stage + D50_BYTES), a.d50 + (int64_t)a.work[start + 1] * a.d50_stride, D50_BYTES,
-                 bar0 + 8 * 10);
+        bulk_g2s(smem_addr(stage + D50_BYTES), d50_of(a, a.work[start + 1]), D50_BYTES, bar0 + 8 * 10);
       }
     }
     mbar_wait(bar0 + 8 * 9, in_ph & 1u);
@@ -385,8 +388,7 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
       }
       if (tid == 0 && j + 2 < end) {  // frame j's staging buffer is consumed: prefetch frame j+2 into it
         mbar_expect_tx(bar0 + 8 * (9 + buf), D50_BYTES);
-        bulk_g2s(smem_addr(stage + buf * D50_BYTES), a.d50 + (int64_t)a.work[j + 2] * a.d50_stride, D50_BYTES,
-                 bar0 + 8 * (9 + buf));
+        bulk_g2s(smem_addr(stage + buf * D50_BYTES), d50_of(a, a.work[j + 2]), D50_BYTES, bar0 + 8 * (9 + buf));
       }
       mbar_wait(bar0 + 8 * (7 + grp), ph);
       fence_after();
@@ -420,6 +422,7 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
       atomicAdd(st + 4, (unsigned long long)cnt_c0);
       atomicAdd(st + 5, (unsigned long long)cnt_c1);
       atomicAdd(st + 6, (unsigned long long)cnt_c2);
+      if (a.pop_start && a.pop_start[k]) atomicAdd(st + 7, 1ull);
     }
     __syncthreads();
   }

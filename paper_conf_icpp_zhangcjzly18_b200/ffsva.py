@@ -30,7 +30,8 @@ EXPORTS = ["ffsva_open_stream", "ffsva_set_reference", "ffsva_snm_load", "ffsva_
            "ffsva_batch_device_outputs", "ffsva_batch_destroy", "ffsva_batch_profile", "ffsva_sdd_batch",
            "ffsva_get_reference",
            "ffsva_stream_info", "ffsva_stats_copy", "ffsva_close", "ffsva_last_error", "ffsva_kernel_launches",
-           "ffsva_version"]
+           "ffsva_version", "ffsva_sched_create", "ffsva_sched_push", "ffsva_sched_tick", "ffsva_sched_depth",
+           "ffsva_sched_destroy"]
 
 
 class StreamDesc(ctypes.Structure):
@@ -58,6 +59,17 @@ class Result(ctypes.Structure):
 RESULT_DTYPE = np.dtype([("ssd", "<u8"), ("sdd_pass", "u1"), ("snm_pass", "u1"), ("snm_class", "u1"),
                          ("pad", "u1"), ("logit", "<f4"), ("survivor_idx", "<i4")], align=True)
 assert RESULT_DTYPE.itemsize == ctypes.sizeof(Result) == 24
+
+EVENT_DTYPE = np.dtype([("stream", "<u8"), ("frame_no", "<i8"), ("result", RESULT_DTYPE)], align=True)
+
+
+class TickInfo(ctypes.Structure):
+    _fields_ = [("admitted", ctypes.c_int32), ("sdd_pass", ctypes.c_int32), ("snm_scored", ctypes.c_int32),
+                ("snm_batches", ctypes.c_int32), ("sdd_blocked", ctypes.c_int32), ("sdd_queued", ctypes.c_int64),
+                ("snm_queued", ctypes.c_int64), ("events_pending", ctypes.c_int64)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
 
 _lib = None
 
@@ -88,6 +100,11 @@ def lib():
             "ffsva_stream_info": [vp, ctypes.POINTER(i32), ctypes.POINTER(i32)],
             "ffsva_stats_copy": [i32, vp, i32, ctypes.POINTER(i32), i32, i32, vp],
             "ffsva_close": [vp],
+            "ffsva_sched_create": [i32, i32, i32, ctypes.POINTER(vp)],
+            "ffsva_sched_push": [vp, vp, i32, vp],
+            "ffsva_sched_tick": [vp, vp, vp, i32, ctypes.POINTER(i32), ctypes.POINTER(TickInfo)],
+            "ffsva_sched_depth": [vp, vp, ctypes.POINTER(i32), ctypes.POINTER(i32)],
+            "ffsva_sched_destroy": [vp],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -332,6 +349,76 @@ class Context:
         for s in self.streams:
             s.close()
         self.streams = []
+
+
+def ffsva_sched_create(device: int, max_frames_per_tick: int, snm_slots: int):
+    h = ctypes.c_void_p()
+    _check(lib().ffsva_sched_create(device, max_frames_per_tick, snm_slots, ctypes.byref(h)), "ffsva_sched_create")
+    return h.value
+
+
+def ffsva_sched_push(sched, frames) -> np.ndarray:
+    """frames: list of (stream handle, device pointer, frame_no) or a structured array. Returns accepted (u8)."""
+    arr = _frames_array(frames)
+    acc = np.zeros(max(1, len(frames)), np.uint8)
+    _check(lib().ffsva_sched_push(sched, arr, len(frames), acc.ctypes.data), "ffsva_sched_push")
+    return acc[:len(frames)]
+
+
+def ffsva_sched_push_array(sched, frames: np.ndarray) -> np.ndarray:
+    """Vectorised push: frames is a FRAME_DTYPE array (stream handle, pixels pointer, frame_no)."""
+    f = np.ascontiguousarray(frames, dtype=FRAME_DTYPE)
+    acc = np.zeros(max(1, f.size), np.uint8)
+    _check(lib().ffsva_sched_push(sched, f.ctypes.data, f.size, acc.ctypes.data), "ffsva_sched_push")
+    return acc[:f.size]
+
+
+def ffsva_sched_tick(sched, cuda_stream: int, cap: int):
+    ev = np.zeros(max(1, cap), EVENT_DTYPE)
+    n = ctypes.c_int32()
+    info = TickInfo()
+    _check(lib().ffsva_sched_tick(sched, cuda_stream, ev.ctypes.data, cap, ctypes.byref(n), ctypes.byref(info)),
+           "ffsva_sched_tick")
+    return ev[:n.value], info.as_dict()
+
+
+def ffsva_sched_depth(sched, stream):
+    a, b = ctypes.c_int32(), ctypes.c_int32()
+    _check(lib().ffsva_sched_depth(sched, stream, ctypes.byref(a), ctypes.byref(b)), "ffsva_sched_depth")
+    return a.value, b.value
+
+
+def ffsva_sched_destroy(sched) -> None:
+    _check(lib().ffsva_sched_destroy(sched), "ffsva_sched_destroy")
+
+
+FRAME_DTYPE = np.dtype([("stream", "<u8"), ("pixels", "<u8"), ("frame_no", "<i8")], align=True)
+
+
+class Scheduler:
+    """Online runtime (§4.3): per-stream queues, feedback thresholds, dynamic batching."""
+
+    def __init__(self, ctx: "Context", max_frames_per_tick: int = 65536, snm_slots: int = 65536):
+        self.ctx = ctx
+        self.handle = ffsva_sched_create(ctx.device, max_frames_per_tick, snm_slots)
+        self.cap = max_frames_per_tick + snm_slots
+
+    def push(self, items) -> np.ndarray:
+        return ffsva_sched_push(self.handle, Context._frames(items))
+
+    def push_array(self, frames: np.ndarray) -> np.ndarray:
+        return ffsva_sched_push_array(self.handle, frames)
+
+    def tick(self, stream=None):
+        return ffsva_sched_tick(self.handle, _stream_handle(stream), self.cap)
+
+    def depth(self, st: "Stream"):
+        return ffsva_sched_depth(self.handle, st.handle)
+
+    def destroy(self) -> None:
+        if self.handle:
+            ffsva_sched_destroy(self.handle)
+            self.handle = None
 
 
 class PreparedBatch:

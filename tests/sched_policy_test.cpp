@@ -1,0 +1,103 @@
+// Hand traces of the online queue policy (§4.3: feedback queue L209/L217, dynamic batching L223).
+// Built and run by tests/test_sched_policy.py with g++ (no CUDA).
+#include <cstdio>
+#include <cstdlib>
+
+#include "../paper_conf_icpp_zhangcjzly18_b200/csrc/ffsva_sched_policy.h"
+
+using ffsva::sched::Policy;
+using ffsva::sched::QFrame;
+
+static int failures = 0;
+#define CHECK(c)                                                      \
+  do {                                                                \
+    if (!(c)) {                                                       \
+      std::printf("FAIL line %d: %s\n", __LINE__, #c);                \
+      ++failures;                                                     \
+    }                                                                 \
+  } while (0)
+
+static QFrame fr(int64_t no) {
+  QFrame q;
+  q.frame_no = no;
+  q.pixels = (const void*)0x1000;
+  return q;
+}
+
+int main() {
+  {  // the prefetcher is refused while the SDD queue holds more than q_sdd = 2 frames
+    Policy p;
+    int s = p.add_stream(2, 10, 30);
+    CHECK(p.push(s, fr(0)) && p.push(s, fr(1)) && p.push(s, fr(2)));
+    CHECK(!p.push(s, fr(3)));                      // depth 3 > 2: blocked
+    CHECK(p.stream(s).refused == 1 && p.stream(s).max_sdd == 3);
+    auto a = p.admit_sdd(100, 100);
+    CHECK(a.size() == 3 && a[0].frame_no == 0 && a[2].frame_no == 2);  // arrival order
+    CHECK(p.push(s, fr(3)));                       // drained: accepted again
+  }
+  {  // the SDD stage skips a stream while its SNM queue holds more than q_snm = 2 frames
+    Policy p;
+    int s = p.add_stream(100, 2, 2);
+    for (int i = 0; i < 5; ++i) p.push(s, fr(i));
+    auto a = p.admit_sdd(100, 100);
+    CHECK(a.size() == 5);
+    for (auto& f : a) p.sdd_done(f, true);         // all survive: SNM depth 5
+    CHECK(p.stream(s).snm.size() == 5);
+    p.push(s, fr(5));
+    CHECK(p.admit_sdd(100, 100).empty());          // 5 > 2: blocked
+    CHECK(p.stream(s).sdd_blocked == 1);
+    auto pops = p.pop_snm();                       // BatchSize 2
+    CHECK(pops.size() == 1 && pops[0].size() == 2 && pops[0][0].frame_no == 0);
+    CHECK(p.admit_sdd(100, 100).empty());          // depth 3 > 2: still blocked
+    p.pop_snm();                                   // depth 1
+    auto b = p.admit_sdd(100, 100);
+    CHECK(b.size() == 1 && b[0].frame_no == 5);    // resumes once depth <= threshold
+  }
+  {  // dynamic batching: each cycle pops min(BatchSize, depth), survivors in order, dropped frames never queue
+    Policy p;
+    int s = p.add_stream(100, 100, 3);
+    for (int i = 0; i < 9; ++i) p.push(s, fr(i));
+    auto a = p.admit_sdd(100, 100);
+    for (auto& f : a) p.sdd_done(f, f.frame_no % 4 != 0);  // frames 0, 4, 8 dropped: 6 survivors
+    CHECK(p.queued_snm() == 6);
+    auto p1 = p.pop_snm();
+    CHECK(p1.size() == 1 && p1[0].size() == 3 && p1[0][0].frame_no == 1 && p1[0][2].frame_no == 3);
+    auto p2 = p.pop_snm();
+    CHECK(p2[0].size() == 3 && p2[0][0].frame_no == 5 && p2[0][2].frame_no == 7);
+    CHECK(p.pop_snm().empty());
+  }
+  {  // a per-cycle budget is shared round-robin; the start stream rotates every cycle
+    Policy p;
+    int s0 = p.add_stream(100, 100, 30), s1 = p.add_stream(100, 100, 30), s2 = p.add_stream(100, 100, 30);
+    for (int i = 0; i < 2; ++i) {
+      p.push(s0, fr(i));
+      p.push(s1, fr(10 + i));
+      p.push(s2, fr(20 + i));
+    }
+    auto c1 = p.admit_sdd(3, 100);
+    CHECK(c1.size() == 3 && c1[0].stream == s0 && c1[1].stream == s0 && c1[2].stream == s1);
+    auto c2 = p.admit_sdd(3, 100);
+    CHECK(c2.size() == 3 && c2[0].stream == s1 && c2[1].stream == s2 && c2[2].stream == s2);
+    CHECK(p.queued_sdd() == 0);
+  }
+  {  // admission never exceeds the free SNM slots
+    Policy p;
+    int s = p.add_stream(100, 100, 30);
+    for (int i = 0; i < 10; ++i) p.push(s, fr(i));
+    CHECK(p.admit_sdd(100, 4).size() == 4);
+    CHECK(p.queued_sdd() == 6);
+  }
+  {  // removing a stream hands back its queued frames; its id is reused
+    Policy p;
+    int s = p.add_stream(100, 100, 30);
+    p.push(s, fr(0));
+    auto a = p.admit_sdd(100, 100);
+    p.sdd_done(a[0], true);
+    p.push(s, fr(1));
+    auto left = p.remove_stream(s);
+    CHECK(left.size() == 2 && !p.live(s));
+    CHECK(p.add_stream(1, 1, 1) == s);
+  }
+  if (failures == 0) std::printf("ALL PASS\n");
+  return failures == 0 ? 0 : 1;
+}

@@ -1,0 +1,92 @@
+"""GPU test of the online runtime (§4.3): per-stream queues, feedback thresholds, dynamic batching.
+
+Every accepted frame must come back exactly once with the same SDD result as the oracle (bit-exact) and an
+SNM logit within tolerance; the feedback queue must actually engage (refused pushes, blocked SDD admissions)
+and the queue depths must respect their thresholds at every cycle."""
+import numpy as np
+import pytest
+
+from gpu_util import SNM_TOL, Cam, f32
+from oracle import oracle as orc
+from synth import synth
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def env():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    import __graft_entry__ as ge
+    ge.build()
+    import paper_conf_icpp_zhangcjzly18_b200 as ff
+    dev = torch.device("cuda:0")
+    ctx = ff.Context(dev)
+    yield ff, ctx, dev
+    ctx.close()
+
+
+def test_online_feedback_queue_and_dynamic_batching(env):
+    ff, ctx, dev = env
+    import torch
+    from paper_conf_icpp_zhangcjzly18_b200.ffsva import Scheduler
+    q_sdd, q_snm, B = 2, 3, 1
+    v = synth.Video(seed=61, width=640, height=360, period=10, on_len=5)
+    cams = []
+    for s in range(3):
+        c = Cam(ctx, v, s, dev, k_ref=2, snm_batch=B)
+        cams.append(c)
+    # rebuild the streams with the online thresholds (Cam opens with the defaults)
+    for c in cams:
+        c.st.close()
+        c.st = ctx.open_stream(width=640, height=360, delta_diff=24.0, snm_batch=B, q_sdd=q_sdd, q_snm=q_snm)
+        c.st.set_reference(torch.from_numpy(c.refs).to(dev))
+        c.st.snm_load(c.params)
+    T = 24
+    host = {s: c.host_frames(list(range(T))) for s, c in enumerate(cams)}
+    dev_frames = {s: torch.from_numpy(host[s]).to(dev) for s in host}
+    sched = Scheduler(ctx, max_frames_per_tick=64, snm_slots=64)
+    handle_to_s = {c.st.handle: s for s, c in enumerate(cams)}
+    backlog = {s: list(range(T)) for s in range(3)}
+    got = {}
+    refused = blocked = 0
+    cs = torch.cuda.Stream()
+    for step in range(200):
+        items = []
+        for s in range(3):  # each prefetcher offers its next 3 frames; refused frames stay in its backlog
+            for t in backlog[s][:3]:
+                items.append((cams[s].st, dev_frames[s][t], t))
+        if items:
+            acc = sched.push(items)
+            refused += int((acc == 0).sum())
+            for (st, _, t), a in zip(items, acc):
+                if a:
+                    backlog[handle_to_s[st.handle]].remove(t)
+        ev, info = sched.tick(cs)
+        blocked += info["sdd_blocked"]
+        for c in cams:
+            d_sdd, d_snm = sched.depth(c.st)
+            assert d_sdd <= q_sdd + 1, "SDD queue grew past its threshold + 1"
+            assert d_snm <= q_snm + 3, "SNM queue grew past threshold + one cycle's admissions"
+        for e in ev:
+            key = (handle_to_s[int(e["stream"])], int(e["frame_no"]))
+            assert key not in got, "frame reported twice"
+            got[key] = e["result"]
+        if all(not b for b in backlog.values()) and info["sdd_queued"] == 0 and info["snm_queued"] == 0 \
+                and info["events_pending"] == 0:
+            break
+    sched.destroy()
+    assert len(got) == 3 * T, f"{len(got)} of {3 * T} frames reported"
+    assert refused > 0, "the SDD-queue threshold never refused a push"
+    assert blocked > 0, "the SNM-queue threshold never blocked the SDD stage"
+    for (s, t), r in got.items():
+        c = cams[s]
+        w = orc.filter_frames([host[s][t]], 640, [c.R], [24.0], [c.params], [f32(0.2)], [f32(0.8)], [f32(0.5)])
+        assert int(r["ssd"]) == int(w["ssd"][0]), (s, t)
+        assert int(r["sdd_pass"]) == int(w["sdd_pass"][0]), (s, t)
+        assert r["sdd_pass"] == int(synth.is_target(v, s, t))
+        if w["sdd_pass"][0]:
+            assert abs(float(r["logit"]) - w["logit"][0]) <= SNM_TOL, (s, t)
+        else:
+            assert np.isnan(r["logit"])
