@@ -274,6 +274,11 @@ def run_ours(args, cfg, ws, rank, local):
     if rank == 0 and ws == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(cfg, video, sids, pool, args.cpu_frames)
 
+    # ---- online validation of "sustained 30-FPS streams" (paced arrivals through the online runtime)
+    online = None
+    if args.online and args.config == "m2":
+        online = online_validation(args, ctx, video, sids, pool, value, dev, cs)
+
     out = None
     if rank == 0:
         out = {
@@ -305,6 +310,7 @@ def run_ours(args, cfg, ws, rank, local):
                              "frac": (m_avg * SNM_FLOP / (k_ms[2] / 1e3) / 1e12) / tf_peak if k_ms[2] > 0 else 0.0,
                              "peak_source": peak_kind, "survivors_per_s": m_avg / (k_ms[2] / 1e3) if k_ms[2] else 0},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
+            "online": online,
         }
     for b in batches:
         b.destroy()
@@ -312,6 +318,52 @@ def run_ours(args, cfg, ws, rank, local):
     if ws > 1:
         dist.destroy_process_group()
     return out
+
+
+def online_validation(args, ctx, video, sids, pool, value, dev, cs):
+    """Paced 30-FPS streams through the online runtime (feedback queue + dynamic batching, §4.3).
+    Stream i replays content stream i % len(sids) of the pool with its own reference image and SNM."""
+    import torch
+
+    from paper_conf_icpp_zhangcjzly18_b200.online import run_paced
+    from synth import synth
+    W, H, P = video.width, video.height, 3 * video.width
+    counts = []
+    for tok in args.online.split(","):
+        tok = tok.strip()
+        if tok == "auto":
+            counts.append(max(31, int(0.7 * value / 30)))
+        elif tok:
+            counts.append(int(tok))
+    nc = len(sids)
+    refs = []
+    for k, s in enumerate(sids):
+        r = torch.empty((32, H, P), dtype=torch.uint8, device=dev)
+        synth.frames_cuda(video, torch.full((32,), s, dtype=torch.int32, device=dev),
+                          torch.arange(32, dtype=torch.int64, device=dev), r, H * P, P, ref=True)
+        refs.append(r)
+    results = []
+    opened = []
+    for S in counts:
+        t_setup = time.perf_counter()
+        while len(opened) < S:
+            i = len(opened)
+            st = ctx.open_stream(width=W, height=H, delta_diff=DELTA, c_low=C_LOW, c_high=C_HIGH, filter_degree=FD,
+                                 snm_batch=BATCH, q_sdd=2, q_snm=10)
+            st.set_reference(refs[i % nc])
+            st.snm_load(synth.snm_weights(video.seed, 100000 + i))
+            opened.append(st)
+        setup_s = time.perf_counter() - t_setup
+        res = run_paced(ctx, opened[:S], [pool[i % nc] for i in range(S)], pool.shape[1], args.online_seconds,
+                        cuda_stream=cs)
+        res["stream_setup_s"] = setup_s
+        results.append(res)
+    for st in opened:
+        st.close()
+        ctx.streams.remove(st)
+    best = max([r["streams"] for r in results if r["sustained"]], default=0)
+    return {"runs": results, "max_sustained_streams_validated": best,
+            "policy": "q_sdd 2, q_snm 10, BatchSize 30 (PAPER.md L217, L219); latency budget p99 <= 1 s"}
 
 
 def cpu_baseline(cfg, video, sids, pool, n_frames):
@@ -407,6 +459,10 @@ def main():
     ap.add_argument("--cpu-frames", type=int, default=480)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--online", default="30,auto",
+                    help="comma-separated stream counts for the paced online validation (config m2); 'auto' = "
+                         "70%% of the measured frames/s / 30; empty to skip")
+    ap.add_argument("--online-seconds", type=float, default=4.0)
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")

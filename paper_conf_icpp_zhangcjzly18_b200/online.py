@@ -1,0 +1,90 @@
+"""Paced online driver: S cameras at 30 FPS through the online runtime (ffsva_sched_*), for validating
+"sustained 30-FPS streams": frame k of stream s becomes available at t0 + phi_s + k/30
+(phi_s spreads the streams over one frame period); each cycle pushes every frame that has arrived (frames the
+feedback queue refuses stay in the camera's backlog and are offered again next cycle), runs one scheduler tick
+and records arrival->decision latency for every reported frame. A stream count is sustained when the p99
+latency stays within the budget (the paper tolerates seconds) and no backlog accumulates.
+
+The frames' bytes live in a device pool (the online measurement covers scheduling + kernels, not ingest I/O);
+stream s replays content stream s % n_content with its own reference image and SNM."""
+from __future__ import annotations
+
+import time
+
+import numpy as np
+
+
+def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s=0.010, cuda_stream=None,
+              latency_budget_s=1.0):
+    """streams[i]: ff.Stream; content[i]: (device frame tensor [n_content_frames, H, pitch]).
+
+    Returns a dict of latency percentiles, refusals, backlog and throughput."""
+    import torch
+
+    from .ffsva import FRAME_DTYPE, Scheduler
+
+    S = len(streams)
+    handles = np.array([s.handle for s in streams], dtype=np.uint64)
+    order = np.argsort(handles)
+    sorted_handles = handles[order]
+    base_ptr = np.array([c.data_ptr() for c in content], dtype=np.uint64)
+    fbytes = np.array([c[0].numel() for c in content], dtype=np.uint64)
+    phase = (np.arange(S) * (1.0 / fps) / S).astype(np.float64)
+    start_frame = (np.arange(S) * 37) % n_content_frames
+    pushed = np.zeros(S, np.int64)          # frames handed to (and accepted by) the scheduler
+    max_frames_tick = max(1024, int(S * fps * 0.25))
+    sched = Scheduler(ctx, max_frames_per_tick=max_frames_tick, snm_slots=max(4096, S * 12))
+    lat = []
+    refused = 0
+    done = 0
+    max_backlog = 0
+    ticks = 0
+    try:
+        torch.cuda.synchronize()
+        t0 = time.perf_counter() + 0.05
+        while True:
+            now = time.perf_counter()
+            el = now - t0
+            if el > seconds:
+                break
+            due = np.floor((el - phase) * fps).astype(np.int64) + 1
+            due = np.maximum(due, 0)
+            want = due - pushed
+            max_backlog = max(max_backlog, int(want.max(initial=0)))
+            n_off = int(want.sum())
+            if n_off > 0:
+                # offer at most q_sdd + 1 frames per stream per cycle (the rest would be refused anyway)
+                take = np.minimum(want, 3)
+                idx = np.repeat(np.arange(S), take)
+                k = pushed[idx] + (np.arange(idx.size) - np.repeat(np.cumsum(take) - take, take))
+                fr = np.zeros(idx.size, dtype=FRAME_DTYPE)
+                fr["stream"] = handles[idx]
+                fr["pixels"] = base_ptr[idx] + ((start_frame[idx] + k) % n_content_frames).astype(np.uint64) * fbytes[idx]
+                fr["frame_no"] = k
+                acc = sched.push_array(fr)
+                refused += int((acc == 0).sum())
+                # accepted frames are a prefix per stream (a refusal stops the camera this cycle)
+                np.add.at(pushed, idx[acc == 1], 1)
+            ev, info = sched.tick(cuda_stream)
+            ticks += 1
+            t_done = time.perf_counter()
+            if ev.size:
+                si = order[np.searchsorted(sorted_handles, ev["stream"])]
+                arrival = t0 + phase[si] + ev["frame_no"].astype(np.float64) / fps
+                lat.append(t_done - arrival)
+                done += ev.size
+            rest = tick_s - (time.perf_counter() - now)
+            if rest > 0:
+                time.sleep(rest)
+        backlog_end = int((np.maximum(np.floor((time.perf_counter() - t0 - phase) * fps) + 1, 0) - pushed).sum())
+    finally:
+        sched.destroy()
+    L = np.concatenate(lat) if lat else np.zeros(1)
+    res = {"streams": S, "seconds": seconds, "ticks": ticks, "frames_decided": int(done),
+           "decided_fps": done / seconds, "offered_fps": S * fps, "refused_pushes": refused,
+           "max_backlog_frames_per_stream": max_backlog, "backlog_frames_at_end": backlog_end,
+           "latency_p50_s": float(np.percentile(L, 50)), "latency_p99_s": float(np.percentile(L, 99)),
+           "latency_max_s": float(L.max())}
+    res["sustained"] = bool(res["latency_p99_s"] <= latency_budget_s and backlog_end <= S * 2
+                            and done >= 0.9 * S * fps * (seconds - latency_budget_s))
+    return res

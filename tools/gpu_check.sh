@@ -2,14 +2,14 @@
 # One gpurun call: build, GPU tests, smoke, bench, ncu launch list + full captures of K1 and K4.
 #   BENCH="--steps 2000 --warmup 10"  run bench.py with these args
 #   NCU=1                              ncu launch list + --set full captures (profiles come back in gpurun_out/)
-#   PYTEST_ARGS="-k ..."               subset of GPU tests
+#   PYTEST_K="expr"                    subset of GPU tests (pytest -k)
 #   SKIP_TESTS=1                       skip pytest + smoke
 cd "$(dirname "$0")/.."
 mkdir -p gpurun_out
 nvidia-smi > gpurun_out/nvidia-smi.txt 2>&1
 timeout 600 python __graft_entry__.py > gpurun_out/build.log 2>&1 || { echo BUILD FAILED; tail -30 gpurun_out/build.log; exit 1; }
 if [ -z "$SKIP_TESTS" ]; then
-  timeout 1200 python -m pytest tests -m gpu -x -q ${PYTEST_ARGS} > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"
+  timeout 1200 python -m pytest tests -m gpu -x -q ${PYTEST_K:+-k "$PYTEST_K"} > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"
   tail -25 gpurun_out/pytest_gpu.log
   timeout 300 python __graft_entry__.py smoke > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"; tail -3 gpurun_out/smoke.log
 fi
