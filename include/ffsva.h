@@ -206,6 +206,9 @@ typedef struct {
   int64_t sdd_queued;        /* frames waiting in SDD queues after the cycle */
   int64_t snm_queued;        /* frames waiting in SNM queues after the cycle */
   int64_t events_pending;    /* events not yet returned */
+  float sdd_ms, snm_ms;      /* wall time of the SDD / SNM cycle (host work + kernels + copies) */
+  float host_ms;             /* wall time of the whole tick */
+  int32_t pad;
 } ffsva_tick_info;
 
 FFSVA_API ffsva_status ffsva_sched_create(int32_t device, int32_t max_frames_per_tick, int32_t snm_slots,

@@ -7,6 +7,7 @@
 //   4. every non-empty SNM queue pops min(BatchSize, depth) (dynamic batching); K4 scores all pops in one
 //      launch, reading the images from their slots; scored frames become events and free their slots.
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstring>
 #include <deque>
@@ -61,6 +62,8 @@ struct ffsva_sched {
   uint8_t* d_out = nullptr;   // ssd u64[cap] | logit f32[cap] | pass u8[cap] | snm_pass u8[cap] | snm_class u8[cap]
   uint8_t* h_out = nullptr;
   std::deque<ffsva_event> pending;
+  std::vector<sched::QFrame> flat;  // this cycle's SNM pops, reused
+  std::vector<int32_t> starts;
 };
 
 namespace {
@@ -210,6 +213,7 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
   const Layout L(n);
   uint8_t* h = s->h_in;
   ffsva_tick_info ti{};
+  const auto t_tick0 = std::chrono::steady_clock::now();
   uint64_t blocked0 = 0;
   for (int32_t i = 0; i < s->pol.n_streams(); ++i) blocked0 += s->pol.stream(i).sdd_blocked;
   cudaError_t e = cudaSuccess;
@@ -251,7 +255,15 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
     hseg[nseg] = na;
     const bool bulk = vec16 && sdd_bulk_ok(max_chunks, stage);
     e = sdd_configure(bulk ? sdd_bulk_smem_bytes(stage, sdd_w) : sdd_smem_bytes(max_chunks, sdd_w));
-    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in, h, L.total, cudaMemcpyHostToDevice, cs);
+    // upload only the used part of each staging region
+    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in + L.desc, h + L.desc, 64 * (size_t)na, cudaMemcpyHostToDevice, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in + L.index, h + L.index, 4 * (size_t)na, cudaMemcpyHostToDevice, cs);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(s->d_in + L.seg_lo, h + L.seg_lo, 4 * (size_t)(nseg + 1), cudaMemcpyHostToDevice, cs);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(s->d_in + L.seg_batch, h + L.seg_batch, 4 * (size_t)nseg, cudaMemcpyHostToDevice, cs);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(s->d_in + L.seg_slot, h + L.seg_slot, 4 * (size_t)nseg, cudaMemcpyHostToDevice, cs);
     SddArgs sa{};
     sa.frames = at<FrameDesc>(s->d_in, L.desc);
     sa.n = na;
@@ -313,10 +325,12 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
   }
 
   // ---------------- SNM cycle: dynamic batching (pops of min(BatchSize, depth) per stream)
-  std::vector<std::vector<sched::QFrame>> pops = s->pol.pop_snm();
-  int32_t m = 0;
-  for (auto& p : pops) m += (int32_t)p.size();
-  ti.snm_batches = (int32_t)pops.size();
+  const auto t_snm0 = std::chrono::steady_clock::now();
+  std::vector<sched::QFrame>& flat = s->flat;
+  std::vector<int32_t>& starts = s->starts;
+  s->pol.pop_snm(flat, starts);
+  const int32_t m = (int32_t)flat.size();
+  ti.snm_batches = (int32_t)starts.size() - 1;
   ti.snm_scored = m;
   if (m > 0) {
     FrameDesc* hd = at<FrameDesc>(h, L.desc);
@@ -325,23 +339,21 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
     int32_t* hch = at<int32_t>(h, L.chunks);
     int32_t* hcnt = at<int32_t>(h, L.counts);
     uint8_t* hpop = h + L.pop_start;
-    std::vector<sched::QFrame> flat;
-    flat.reserve(m);
-    int32_t j = 0, nch = 0;
-    for (auto& p : pops) {
-      const ffsva_stream* st = s->by_id[p[0].stream];
+    int32_t nch = 0;
+    for (size_t p = 0; p + 1 < starts.size(); ++p) {
+      const ffsva_stream* st = s->by_id[flat[starts[p]].stream];
       // a pop is split into work units of U frames so small cycles still spread over the SMs
       const int32_t U = std::max(1, std::min(st->desc.snm_batch, m / std::max(1, ctx->num_sms)));
-      for (int32_t k = 0; k < (int32_t)p.size(); ++k) {
+      const FrameDesc d = make_desc(st, nullptr);
+      for (int32_t j = starts[p]; j < starts[p + 1]; ++j) {
+        const int32_t k = j - starts[p];
         if (k % U == 0) {
           hpop[nch] = k == 0 ? 1 : 0;
           hch[nch++] = j;
         }
-        hd[j] = make_desc(st, nullptr);
-        hidx[j] = p[k].slot;
+        hd[j] = d;
+        hidx[j] = flat[j].slot;
         hwork[j] = j;
-        flat.push_back(p[k]);
-        ++j;
       }
     }
     hch[nch] = m;
@@ -349,7 +361,15 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
     hcnt[1] = nch;
     hcnt[2] = 0;
     hcnt[3] = 0;
-    e = cudaMemcpyAsync(s->d_in, h, L.total, cudaMemcpyHostToDevice, cs);
+    // upload only the used part of each staging region
+    e = cudaMemcpyAsync(s->d_in + L.desc, h + L.desc, 64 * (size_t)m, cudaMemcpyHostToDevice, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in + L.index, h + L.index, 4 * (size_t)m, cudaMemcpyHostToDevice, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in + L.work, h + L.work, 4 * (size_t)m, cudaMemcpyHostToDevice, cs);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(s->d_in + L.chunks, h + L.chunks, 4 * (size_t)(nch + 1), cudaMemcpyHostToDevice, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in + L.counts, h + L.counts, 16, cudaMemcpyHostToDevice, cs);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(s->d_in + L.pop_start, h + L.pop_start, (size_t)nch, cudaMemcpyHostToDevice, cs);
     SnmArgs na{};
     na.frames = at<FrameDesc>(s->d_in, L.desc);
     na.d50 = s->d_pool;
@@ -367,7 +387,8 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
     if (e == cudaSuccess) e = launch_snm(na, cs);
     g_launches += 1;
     if (e == cudaSuccess) e = cudaMemcpyAsync(h_logit, na.logit, 4 * (size_t)m, cudaMemcpyDeviceToHost, cs);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(h_snm_pass, na.snm_pass, 2 * n, cudaMemcpyDeviceToHost, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(h_snm_pass, na.snm_pass, (size_t)m, cudaMemcpyDeviceToHost, cs);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(h_snm_class, na.snm_class, (size_t)m, cudaMemcpyDeviceToHost, cs);
     if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
     if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (SNM cycle)");
     for (int32_t k = 0; k < m; ++k) {
@@ -397,6 +418,10 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
   ti.sdd_queued = s->pol.queued_sdd();
   ti.snm_queued = s->pol.queued_snm();
   ti.events_pending = (int64_t)s->pending.size();
+  const auto t_end = std::chrono::steady_clock::now();
+  ti.sdd_ms = std::chrono::duration<float, std::milli>(t_snm0 - t_tick0).count();
+  ti.snm_ms = std::chrono::duration<float, std::milli>(t_end - t_snm0).count();
+  ti.host_ms = std::chrono::duration<float, std::milli>(t_end - t_tick0).count();
   if (info) *info = ti;
   return FFSVA_OK;
 }

@@ -114,17 +114,29 @@ class Policy {
   }
 
   // SNM stage of one cycle (dynamic batching, L223): every non-empty stream pops min(BatchSize, depth).
-  std::vector<std::vector<QFrame>> pop_snm() {
-    std::vector<std::vector<QFrame>> pops;
+  // The pops are appended to `flat`; pop p is flat[starts[p] .. starts[p+1]) (starts gets a final sentinel).
+  void pop_snm(std::vector<QFrame>& flat, std::vector<int32_t>& starts) {
+    flat.clear();
+    starts.clear();
     const int32_t n = (int32_t)st_.size();
     for (int32_t k = 0; k < n; ++k) {
       StreamQ& s = st_[k];
       if (!s.live || s.snm.empty()) continue;
       const int32_t take = std::min<int32_t>(s.batch, (int32_t)s.snm.size());
-      std::vector<QFrame> pop(s.snm.begin(), s.snm.begin() + take);
+      starts.push_back((int32_t)flat.size());
+      flat.insert(flat.end(), s.snm.begin(), s.snm.begin() + take);
       s.snm.erase(s.snm.begin(), s.snm.begin() + take);
-      pops.push_back(std::move(pop));
     }
+    starts.push_back((int32_t)flat.size());
+  }
+
+  std::vector<std::vector<QFrame>> pop_snm() {  // convenience form for tests
+    std::vector<QFrame> flat;
+    std::vector<int32_t> starts;
+    pop_snm(flat, starts);
+    std::vector<std::vector<QFrame>> pops;
+    for (size_t p = 0; p + 1 < starts.size(); ++p)
+      pops.emplace_back(flat.begin() + starts[p], flat.begin() + starts[p + 1]);
     return pops;
   }
 

@@ -66,7 +66,8 @@ EVENT_DTYPE = np.dtype([("stream", "<u8"), ("frame_no", "<i8"), ("result", RESUL
 class TickInfo(ctypes.Structure):
     _fields_ = [("admitted", ctypes.c_int32), ("sdd_pass", ctypes.c_int32), ("snm_scored", ctypes.c_int32),
                 ("snm_batches", ctypes.c_int32), ("sdd_blocked", ctypes.c_int32), ("sdd_queued", ctypes.c_int64),
-                ("snm_queued", ctypes.c_int64), ("events_pending", ctypes.c_int64)]
+                ("snm_queued", ctypes.c_int64), ("events_pending", ctypes.c_int64), ("sdd_ms", ctypes.c_float),
+                ("snm_ms", ctypes.c_float), ("host_ms", ctypes.c_float), ("pad", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -402,6 +403,9 @@ class Scheduler:
         self.ctx = ctx
         self.handle = ffsva_sched_create(ctx.device, max_frames_per_tick, snm_slots)
         self.cap = max_frames_per_tick + snm_slots
+        self._events = np.zeros(self.cap, EVENT_DTYPE)  # reused every tick
+        self._n = ctypes.c_int32()
+        self._info = TickInfo()
 
     def push(self, items) -> np.ndarray:
         return ffsva_sched_push(self.handle, Context._frames(items))
@@ -410,7 +414,10 @@ class Scheduler:
         return ffsva_sched_push_array(self.handle, frames)
 
     def tick(self, stream=None):
-        return ffsva_sched_tick(self.handle, _stream_handle(stream), self.cap)
+        """One cycle; returns (events copied out of a reused buffer, info dict)."""
+        _check(lib().ffsva_sched_tick(self.handle, _stream_handle(stream), self._events.ctypes.data, self.cap,
+                                      ctypes.byref(self._n), ctypes.byref(self._info)), "ffsva_sched_tick")
+        return self._events[:self._n.value].copy(), self._info.as_dict()
 
     def depth(self, st: "Stream"):
         return ffsva_sched_depth(self.handle, st.handle)

@@ -39,6 +39,7 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
     done = 0
     max_backlog = 0
     ticks = 0
+    tim = [0.0, 0.0, 0.0, 0.0]  # python push, SDD cycle, SNM cycle, whole tick call (s)
     try:
         torch.cuda.synchronize()
         t0 = time.perf_counter() + 0.05
@@ -65,9 +66,14 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
                 refused += int((acc == 0).sum())
                 # accepted frames are a prefix per stream (a refusal stops the camera this cycle)
                 np.add.at(pushed, idx[acc == 1], 1)
+            t_push = time.perf_counter()
             ev, info = sched.tick(cuda_stream)
             ticks += 1
             t_done = time.perf_counter()
+            tim[0] += t_push - now
+            tim[1] += info["sdd_ms"] / 1e3
+            tim[2] += info["snm_ms"] / 1e3
+            tim[3] += t_done - t_push
             if ev.size:
                 si = order[np.searchsorted(sorted_handles, ev["stream"])]
                 arrival = t0 + phase[si] + ev["frame_no"].astype(np.float64) / fps
@@ -84,7 +90,9 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
            "decided_fps": done / seconds, "offered_fps": S * fps, "refused_pushes": refused,
            "max_backlog_frames_per_stream": max_backlog, "backlog_frames_at_end": backlog_end,
            "latency_p50_s": float(np.percentile(L, 50)), "latency_p99_s": float(np.percentile(L, 99)),
-           "latency_max_s": float(L.max())}
+           "latency_max_s": float(L.max()),
+           "mean_ms_per_tick": {"push_py": 1e3 * tim[0] / max(1, ticks), "sdd_cycle": 1e3 * tim[1] / max(1, ticks),
+                                "snm_cycle": 1e3 * tim[2] / max(1, ticks), "tick_call": 1e3 * tim[3] / max(1, ticks)}}
     res["sustained"] = bool(res["latency_p99_s"] <= latency_budget_s and backlog_end <= S * 2
                             and done >= 0.9 * S * fps * (seconds - latency_budget_s))
     return res
