@@ -47,8 +47,13 @@ struct ffsva_sched {
   DeviceCtx* ctx = nullptr;
   std::mutex mu;
   sched::Policy pol;
-  std::unordered_map<ffsva_stream*, int32_t> ids;
+  std::vector<int32_t> id_of_slot;  // stream slot -> policy id (O(1) per pushed frame)
   std::vector<ffsva_stream*> by_id;
+  int32_t lookup(const ffsva_stream* st) const {
+    if (st->slot < 0 || st->slot >= (int32_t)id_of_slot.size()) return -1;
+    const int32_t id = id_of_slot[st->slot];
+    return (id >= 0 && id < (int32_t)by_id.size() && by_id[id] == st) ? id : -1;
+  }
   int32_t max_frames = 0, slots = 0, cap = 0;
   int32_t sdd_w = -1, sdd_h = -1;
   std::vector<int32_t> free_slots;
@@ -173,15 +178,13 @@ FFSVA_API ffsva_status ffsva_sched_push(ffsva_sched* s, const ffsva_frame* frame
   }
   for (int32_t i = 0; i < n; ++i) {
     ffsva_stream* st = frames[i].stream;
-    auto it = s->ids.find(st);
-    int32_t id;
-    if (it == s->ids.end()) {
+    int32_t id = s->lookup(st);
+    if (id < 0) {
       id = s->pol.add_stream(st->desc.q_sdd, st->desc.q_snm, st->desc.snm_batch);
-      s->ids[st] = id;
       if ((int32_t)s->by_id.size() <= id) s->by_id.resize(id + 1, nullptr);
       s->by_id[id] = st;
-    } else {
-      id = it->second;
+      if ((int32_t)s->id_of_slot.size() <= st->slot) s->id_of_slot.resize(st->slot + 1, -1);
+      s->id_of_slot[st->slot] = id;
     }
     sched::QFrame q;
     q.frame_no = frames[i].frame_no;
@@ -194,9 +197,9 @@ FFSVA_API ffsva_status ffsva_sched_push(ffsva_sched* s, const ffsva_frame* frame
 FFSVA_API ffsva_status ffsva_sched_depth(ffsva_sched* s, ffsva_stream* st, int32_t* sdd_depth, int32_t* snm_depth) {
   if (!s || !st) return fail(FFSVA_EINVAL, "bad argument");
   std::lock_guard<std::mutex> lk(s->mu);
-  auto it = s->ids.find(st);
-  if (sdd_depth) *sdd_depth = it == s->ids.end() ? 0 : (int32_t)s->pol.stream(it->second).sdd.size();
-  if (snm_depth) *snm_depth = it == s->ids.end() ? 0 : (int32_t)s->pol.stream(it->second).snm.size();
+  const int32_t id = s->lookup(st);
+  if (sdd_depth) *sdd_depth = id < 0 ? 0 : (int32_t)s->pol.stream(id).sdd.size();
+  if (snm_depth) *snm_depth = id < 0 ? 0 : (int32_t)s->pol.stream(id).snm.size();
   return FFSVA_OK;
 }
 

@@ -65,7 +65,7 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
                 acc = sched.push_array(fr)
                 refused += int((acc == 0).sum())
                 # accepted frames are a prefix per stream (a refusal stops the camera this cycle)
-                np.add.at(pushed, idx[acc == 1], 1)
+                pushed += np.bincount(idx[acc == 1], minlength=S)
             t_push = time.perf_counter()
             ev, info = sched.tick(cuda_stream)
             ticks += 1
