@@ -331,8 +331,8 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
     counts = []
     for tok in args.online.split(","):
         tok = tok.strip()
-        if tok == "auto":
-            counts.append(max(31, int(0.7 * value / 30)))
+        if tok == "auto":  # 55% of the offline capacity: the online cycle runs host work and kernels serially
+            counts.append(max(31, int(0.55 * value / 30)))
         elif tok:
             counts.append(int(tok))
     nc = len(sids)
@@ -461,7 +461,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--online", default="30,auto",
                     help="comma-separated stream counts for the paced online validation (config m2); 'auto' = "
-                         "70%% of the measured frames/s / 30; empty to skip")
+                         "55%% of the measured frames/s / 30; empty to skip")
     ap.add_argument("--online-seconds", type=float, default=4.0)
     args = ap.parse_args()
     if args.warmup < 3:
