@@ -1,0 +1,26 @@
+#!/bin/bash
+# Round evidence on one B200: GPU tests, smoke, default bench, ncu launch list + full captures, sanitizers.
+# Everything lands in gpurun_out/; tools/summarize_evidence.py turns it into profiles/<round>/.
+cd "$(dirname "$0")/.."
+mkdir -p gpurun_out
+nvidia-smi > gpurun_out/nvidia-smi.txt 2>&1
+timeout 600 python __graft_entry__.py > gpurun_out/build.log 2>&1 || { echo BUILD FAILED; tail -30 gpurun_out/build.log; exit 1; }
+timeout 1200 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/pytest_gpu.log
+timeout 300 python __graft_entry__.py smoke > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"; tail -1 gpurun_out/smoke.log
+timeout 1200 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?"
+for tool in memcheck racecheck synccheck; do
+  timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_run.py > gpurun_out/sanitize_$tool.log 2>&1
+  echo "sanitize $tool rc=$?"; tail -2 gpurun_out/sanitize_$tool.log
+done
+for CFG in m2 m3; do
+  timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"sdd|compact|snm" -s 60 -c 60 --csv \
+    --log-file gpurun_out/launches_${CFG}.csv \
+    python bench.py --config $CFG --steps 40 --warmup 3 --no-e2e --no-cpu-baseline --online "" > gpurun_out/ncu_list_${CFG}.log 2>&1
+  echo "ncu list $CFG rc=$?"
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:sdd -s 40 -c 1 -o gpurun_out/prof_k1_${CFG} -f \
+    python bench.py --config $CFG --steps 20 --warmup 3 --no-e2e --no-cpu-baseline --online "" > gpurun_out/ncu_full_k1_${CFG}.log 2>&1
+  echo "ncu full k1 $CFG rc=$?"
+done
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:snm_kernel -s 10 -c 1 -o gpurun_out/prof_k4_snm -f \
+  python bench.py --config snm --steps 20 --warmup 3 --no-e2e --no-cpu-baseline --online "" > gpurun_out/ncu_full_k4.log 2>&1
+echo "ncu full k4 rc=$?"

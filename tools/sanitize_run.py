@@ -1,0 +1,54 @@
+"""Small run through every kernel path (K1 bulk + stream variants, K3, K4, reference, online scheduler) for
+compute-sanitizer (memcheck / racecheck / synccheck / initcheck). Prints OK at the end."""
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_icpp_zhangcjzly18_b200 as ff  # noqa: E402
+from paper_conf_icpp_zhangcjzly18_b200.ffsva import Scheduler  # noqa: E402
+from synth import synth  # noqa: E402
+
+
+def main():
+    dev = torch.device("cuda:0")
+    ctx = ff.Context(dev)
+    v = synth.Video(seed=5, width=640, height=360, period=4, on_len=2)
+    streams = []
+    for s in range(2):
+        st = ctx.open_stream(width=640, height=360, snm_batch=2, q_sdd=2, q_snm=3)
+        st.set_reference(torch.from_numpy(synth.frames(v, [s] * 2, [0, 1], ref=True)).to(dev))
+        st.snm_load(synth.snm_weights(5, s, bias_std=0.1))
+        streams.append(st)
+    host = synth.frames(v, [0, 1] * 4, [0, 0, 1, 1, 2, 2, 3, 3])
+    d = torch.from_numpy(host).to(dev)
+    items = [(streams[i % 2], d[i], i) for i in range(8)]
+    r1 = ctx.filter_batch(items)
+    os.environ["FFSVA_SDD_KERNEL"] = "stream"
+    r2 = ctx.filter_batch(items)
+    del os.environ["FFSVA_SDD_KERNEL"]
+    assert np.array_equal(r1["ssd"], r2["ssd"])
+    pb = ctx.prepare(items)
+    s = torch.cuda.Stream()
+    pb.launch(s)
+    pb.launch(s)
+    r3 = pb.fetch(s)
+    assert np.array_equal(r1["ssd"], r3["ssd"])
+    pb.destroy()
+    pinned = [torch.from_numpy(h).pin_memory() for h in host]
+    r4 = ctx.filter_batch([(streams[i % 2], pinned[i].data_ptr(), i) for i in range(8)], host=True)
+    assert np.array_equal(r1["ssd"], r4["ssd"])
+    sched = Scheduler(ctx, max_frames_per_tick=4, snm_slots=8)
+    for t in range(6):
+        sched.push([(streams[i % 2], d[i], i) for i in range(8)])
+        sched.tick(s)
+    sched.destroy()
+    ctx.close()
+    torch.cuda.synchronize()
+    print("OK")
+
+
+if __name__ == "__main__":
+    main()
