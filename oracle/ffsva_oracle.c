@@ -85,6 +85,26 @@ uint64_t orc_threshold(double delta_diff, int64_t N) {
 
 int32_t orc_sdd_pass(uint64_t ssd, uint64_t T) { return ssd > T ? 1 : 0; }
 
+/* "The distance between two video frames can be characterized by ... Sum of Absolute
+ * Differences (SAD)". SAD = sum |a - b| over the N values, in u64 (reading Q23: pass iff
+ * SAD > delta_diff, i.e. SAD > floor(delta_diff) = orc_threshold(delta_diff, 1)). */
+uint64_t orc_sad(const uint8_t* a, const uint8_t* b, int64_t N) {
+  uint64_t s = 0;
+  for (int64_t i = 0; i < N; ++i) {
+    int64_t d = (int64_t)a[i] - (int64_t)b[i];
+    s += (uint64_t)(d < 0 ? -d : d);
+  }
+  return s;
+}
+
+/* PAPER.md L151 NRMSE (reading Q24: Euclidean normalisation, NRMSE = sqrt(SSD / sum R^2)):
+ * the normaliser sum of squares of the reference image, in u64. */
+uint64_t orc_sum_sq(const uint8_t* a, int64_t N) {
+  uint64_t s = 0;
+  for (int64_t i = 0; i < N; ++i) s += (uint64_t)a[i] * (uint64_t)a[i];
+  return s;
+}
+
 /* SDD survivors are pushed to the SNM queue in arrival order. */
 int32_t orc_compact(const uint8_t* pass, int32_t n, int32_t* idx) {
   int32_t m = 0;

@@ -36,6 +36,13 @@ uint64_t orc_ssd(const uint8_t* a, const uint8_t* b, int64_t N);
 uint64_t orc_threshold(double delta_diff, int64_t N);
 int32_t orc_sdd_pass(uint64_t ssd, uint64_t T);
 
+/* f3 SDD variants ("MSE, NRMSE, or SAD"; readings Q23, Q24):
+ * SAD = sum |a - b| (u64); pass iff SAD > floor(delta_diff).
+ * NRMSE = sqrt(SSD / sum R^2); pass iff NRMSE > delta_diff <=> SSD > floor(delta_diff^2 * sum R^2), the product
+ * taken exactly (oracle.nrmse_threshold, Python fractions). */
+uint64_t orc_sad(const uint8_t* a, const uint8_t* b, int64_t N);
+uint64_t orc_sum_sq(const uint8_t* a, int64_t N);
+
 /* C4 (PAPER.md L143 survivors forwarded in order; Q16): idx[0..m) = passing indices in batch order. */
 int32_t orc_compact(const uint8_t* pass, int32_t n, int32_t* idx);
 

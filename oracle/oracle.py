@@ -35,6 +35,10 @@ def lib():
         L.orc_ssd.restype = ctypes.c_uint64
         L.orc_threshold.argtypes = [ctypes.c_double, ctypes.c_int64]
         L.orc_threshold.restype = ctypes.c_uint64
+        L.orc_sad.argtypes = [u8p, u8p, ctypes.c_int64]
+        L.orc_sad.restype = ctypes.c_uint64
+        L.orc_sum_sq.argtypes = [u8p, ctypes.c_int64]
+        L.orc_sum_sq.restype = ctypes.c_uint64
         L.orc_sdd_pass.argtypes = [ctypes.c_uint64, ctypes.c_uint64]
         L.orc_sdd_pass.restype = ctypes.c_int32
         L.orc_compact.argtypes = [u8p, ctypes.c_int32, u8p]
@@ -90,6 +94,51 @@ def ssd(a: np.ndarray, b: np.ndarray) -> int:
 def threshold(delta_diff: float, n_values: int) -> int:
     """C3 T = floor(delta_diff * N)."""
     return int(lib().orc_threshold(delta_diff, n_values))
+
+
+def sad(a: np.ndarray, b: np.ndarray) -> int:
+    """f3 sum of absolute differences (reading Q23)."""
+    a = _c(a, np.uint8).ravel()
+    b = _c(b, np.uint8).ravel()
+    assert a.size == b.size
+    return int(lib().orc_sad(a.ctypes.data, b.ctypes.data, a.size))
+
+
+def sum_sq(a: np.ndarray) -> int:
+    """f3 NRMSE normaliser: sum of squares of the reference image (reading Q24)."""
+    a = _c(a, np.uint8).ravel()
+    return int(lib().orc_sum_sq(a.ctypes.data, a.size))
+
+
+def sad_threshold(delta_diff: float) -> int:
+    """f3 SAD: pass iff SAD > delta_diff <=> SAD > floor(delta_diff) (reading Q23)."""
+    return threshold(delta_diff, 1)
+
+
+def nrmse_threshold(delta_diff: float, ref_sum_sq: int) -> int:
+    """f3 NRMSE = sqrt(SSD / sum R^2) (reading Q24). NRMSE > delta <=> SSD > delta^2 * sum R^2
+    <=> SSD > floor(delta^2 * sum R^2), delta taken as the exact rational value of the double. Clamped to u64."""
+    from fractions import Fraction
+    if not delta_diff > 0:
+        return 0
+    t = (Fraction(delta_diff) ** 2 * ref_sum_sq).__floor__()
+    return min(int(t), 2 ** 64 - 1)
+
+
+def distance(metric: str, d100: np.ndarray, ref: np.ndarray) -> int:
+    """The SDD distance numerator K1 reports in `ssd`: SSD for MSE and NRMSE, SAD for SAD."""
+    return sad(d100, ref) if metric == "sad" else ssd(d100, ref)
+
+
+def sdd_threshold(metric: str, delta_diff: float, ref: np.ndarray) -> int:
+    """T of the strict test distance > T for each metric (readings Q5, Q23, Q24)."""
+    if metric == "mse":
+        return threshold(delta_diff, int(np.asarray(ref).size))
+    if metric == "sad":
+        return sad_threshold(delta_diff)
+    if metric == "nrmse":
+        return nrmse_threshold(delta_diff, sum_sq(ref))
+    raise ValueError(metric)
 
 
 def sdd_pass(ssd_value: int, T: int) -> int:
@@ -160,26 +209,37 @@ def decide(logit_value: float, c_low: float, c_high: float, filter_degree: float
 
 
 def filter_frames(frames, width: int, refs, deltas, snm_params, c_low, c_high, filter_degree,
-                  sdd_grid=(100, 100), snm_grid=(50, 50), bf16_emul: bool = False, run_snm: bool = True):
+                  sdd_grid=(100, 100), snm_grid=(50, 50), bf16_emul: bool = False, run_snm: bool = True,
+                  metrics=None, ref_modes=None, stream_ids=None):
     """The whole cascade on a list of frames, one frame at a time (no batching: C8 says batching never
     changes per-frame results).
 
     frames[i]: (H, pitch) uint8; refs[i]: (sdd_h, sdd_w, 3) reference of frame i's stream; deltas[i]:
     delta_diff; snm_params[i]: packed params (or None); c_low/c_high/filter_degree: per-frame sequences.
-    Returns dict of per-frame arrays: d100, d50, ssd, sdd_pass, survivor_idx, logit, snm_pass, snm_class."""
+    f3 variants (optional per-frame sequences): metrics[i] in {"mse", "sad", "nrmse"} (PAPER.md L151);
+    ref_modes[i] in {"background", "previous"} with stream_ids[i]: in "previous" mode a frame is compared with
+    the D100 of its stream's previous frame in list order, the first one with refs[i] (reading Q25).
+    Returns dict of per-frame arrays: d100, d50, ssd, sdd_pass, survivor_idx, logit, snm_pass, snm_class, and
+    last_ref: {stream id: reference after the list} for "previous"-mode streams."""
     n = len(frames)
     dw, dh = sdd_grid
     sw, sh = snm_grid
-    N = dw * dh * 3
+    metrics = metrics if metrics is not None else ["mse"] * n
+    ref_modes = ref_modes if ref_modes is not None else ["background"] * n
     d100 = np.zeros((n, dh, dw, 3), np.uint8)
     d50 = np.zeros((n, sh, sw, 3), np.uint8)
     ssd_v = np.zeros(n, np.uint64)
     sp = np.zeros(n, np.uint8)
+    last_ref = {}
     for i in range(n):
         d100[i] = box_downsample(frames[i], width, dw, dh)
         d50[i] = box_downsample(frames[i], width, sw, sh)
-        ssd_v[i] = ssd(d100[i], refs[i])
-        sp[i] = sdd_pass(int(ssd_v[i]), threshold(deltas[i], N))
+        ref = refs[i]
+        if ref_modes[i] == "previous":
+            ref = last_ref.get(stream_ids[i], refs[i])
+            last_ref[stream_ids[i]] = d100[i]
+        ssd_v[i] = distance(metrics[i], d100[i], ref)
+        sp[i] = sdd_pass(int(ssd_v[i]), sdd_threshold(metrics[i], deltas[i], ref))
     surv = compact(sp)
     sidx = np.full(n, -1, np.int32)
     sidx[surv] = np.arange(surv.size, dtype=np.int32)
@@ -191,4 +251,4 @@ def filter_frames(frames, width: int, refs, deltas, snm_params, c_low, c_high, f
             lg[i] = snm_forward(d50[i], snm_params[i], bf16_emul=bf16_emul)
             npass[i], ncls[i] = decide(lg[i], c_low[i], c_high[i], filter_degree[i])
     return dict(d100=d100, d50=d50, ssd=ssd_v, sdd_pass=sp, survivors=surv, survivor_idx=sidx, logit=lg,
-                snm_pass=npass, snm_class=ncls)
+                snm_pass=npass, snm_class=ncls, last_ref=last_ref)

@@ -332,3 +332,115 @@ def test_decision_boundaries():
     # t_pre = 0 -> everything passes; t_pre = 1 -> nothing passes
     assert orc.decide(-1e30, 0.0, 1.0, 0.0)[0] == 1
     assert orc.decide(1e30, 0.0, 1.0, 1.0)[0] == 0
+
+
+# ------------------------------------------------------------------ f3 SDD variants: SAD, NRMSE (P13), previous-frame reference
+
+def _d_from_channel0(ch0):
+    a = np.asarray(ch0, dtype=np.uint8)
+    d = np.zeros(a.shape + (3,), np.uint8)
+    d[:, :, 0] = a
+    return d
+
+
+def test_p13_sad_hand_example():
+    g = _gold("p13_sad_nrmse.json")
+    d = _d_from_channel0(g["d_channel0"])
+    assert orc.sad(d, np.zeros_like(d)) == g["expected_sad_vs_zero"]
+    assert orc.sad(np.zeros_like(d), d) == g["expected_sad_vs_zero"]
+    assert orc.sum_sq(d) == g["expected_sum_sq"]
+
+
+def test_sad_invariants():
+    """Invariants SAD must satisfy whatever its implementation: symmetry, triangle inequality, SAD == SSD when
+    every |a - b| <= 1, and SSD <= SAD^2 <= N * SSD (Cauchy-Schwarz); closed form 255 * N."""
+    rng = np.random.default_rng(13)
+    N = 3000
+    assert orc.sad(np.full(N, 255, np.uint8), np.zeros(N, np.uint8)) == 255 * N
+    for _ in range(20):
+        a, b, c = (rng.integers(0, 256, N, dtype=np.uint8) for _ in range(3))
+        s_ab, s_bc, s_ac = orc.sad(a, b), orc.sad(b, c), orc.sad(a, c)
+        assert s_ab == orc.sad(b, a)
+        assert s_ac <= s_ab + s_bc
+        q = orc.ssd(a, b)
+        assert q <= s_ab * s_ab <= N * q
+        e = np.clip(a.astype(np.int64) + rng.integers(-1, 2, N), 0, 255).astype(np.uint8)
+        assert orc.sad(a, e) == orc.ssd(a, e)
+
+
+def test_p13_nrmse_exact_boundary():
+    """NRMSE(0, R=D) = 1 exactly (hand value): 'larger than' is strict, so delta = 1 drops the frame and the
+    next double below 1 keeps it; 2D vs D gives the hand SSD 58."""
+    g = _gold("p13_sad_nrmse.json")
+    d = _d_from_channel0(g["d_channel0"])
+    z = np.zeros_like(d)
+    Q = orc.sum_sq(d)
+    s = orc.ssd(z, d)
+    assert s == Q == g["expected_sum_sq"]
+    assert orc.sdd_pass(s, orc.sdd_threshold("nrmse", 1.0, d)) == 0
+    assert orc.sdd_pass(s, orc.sdd_threshold("nrmse", math.nextafter(1.0, 0.0), d)) == 1
+    d2 = np.clip(2 * d.astype(np.int64), 0, 255).astype(np.uint8)
+    s2 = orc.ssd(d2, d)
+    assert s2 == g["expected_ssd_2d_vs_d"]
+    r = math.sqrt(s2 / Q)
+    assert orc.sdd_pass(s2, orc.sdd_threshold("nrmse", r * (1 - 1e-12), d)) == 1
+    assert orc.sdd_pass(s2, orc.sdd_threshold("nrmse", r * (1 + 1e-12), d)) == 0
+
+
+def test_nrmse_threshold_against_float_definition():
+    """Away from the boundary the exact test agrees with sqrt(SSD / sum R^2) > delta in floating point;
+    constant reference v: sum R^2 = N v^2 (closed form); black reference: any change passes."""
+    rng = np.random.default_rng(24)
+    N = 30000
+    for v in [0, 1, 100, 255]:
+        assert orc.sum_sq(np.full(N, v, np.uint8)) == N * v * v
+    assert orc.nrmse_threshold(0.5, 0) == 0
+    for _ in range(200):
+        ref = rng.integers(0, 256, N, dtype=np.uint8)
+        Q = orc.sum_sq(ref)
+        delta = float(rng.uniform(0.0, 1.5))
+        T = orc.nrmse_threshold(delta, Q)
+        for s in [int(rng.integers(0, 2 * Q)), T, T + 1]:
+            val = math.sqrt(s / Q)
+            if abs(val - delta) < 1e-9:
+                continue
+            assert orc.sdd_pass(s, T) == int(val > delta), (s, T, delta)
+
+
+def test_sad_threshold_strict():
+    for delta, T in [(0.0, 0), (264.0, 264), (264.5, 264), (265.0, 265)]:
+        assert orc.sad_threshold(delta) == T
+    assert orc.sdd_pass(265, orc.sad_threshold(264.99)) == 1
+    assert orc.sdd_pass(265, orc.sad_threshold(265.0)) == 0
+
+
+def test_previous_frame_reference_mode():
+    """Reading Q25 ('previous' mode): frame t of a stream is compared with D100 of frame t-1 of the same
+    stream, the first frame with the stream's reference. A static sequence is background after its first
+    frame (P1 applied frame to frame); an A, B, A, B sequence has the same distance at every step (symmetry);
+    two interleaved streams do not see each other's frames."""
+    v = synth.Video(seed=77, width=200, height=120, period=6, on_len=3)
+    W = 200
+    a = synth.frame(v, 0, 0)
+    b = synth.frame(v, 0, 3)  # a target frame (object planted)
+    R = orc.reference(synth.frames(v, [0] * 4, list(range(4)), ref=True), W, 100, 100)
+    p = synth.snm_weights(1, 0)
+    n = 6
+
+    def run(frames, sids, metric):
+        return orc.filter_frames(frames, W, [R] * len(frames), [24.0 if metric != "sad" else 1000.0] * len(frames),
+                                 [p] * len(frames), [0.2] * len(frames), [0.8] * len(frames), [0.5] * len(frames),
+                                 run_snm=False, metrics=[metric] * len(frames),
+                                 ref_modes=["previous"] * len(frames), stream_ids=sids)
+
+    for metric in ["mse", "sad"]:
+        r = run([a] * n, [0] * n, metric)
+        assert (r["ssd"][1:] == 0).all() and (r["sdd_pass"][1:] == 0).all()
+        assert r["ssd"][0] == orc.distance(metric, orc.box_downsample(a, W, 100, 100), R)
+        r = run([a, b] * 3, [0] * n, metric)
+        dab = orc.distance(metric, orc.box_downsample(a, W, 100, 100), orc.box_downsample(b, W, 100, 100))
+        assert dab > 0 and (r["ssd"][1:] == dab).all() and (r["sdd_pass"][1:] == 1).all()
+        assert np.array_equal(r["last_ref"][0], orc.box_downsample(b, W, 100, 100))
+        # streams 0 and 1 interleaved, each static: only the first frame of each stream may differ from 0
+        r = run([a, b, a, b, a, b], [0, 1, 0, 1, 0, 1], metric)
+        assert (r["ssd"][2:] == 0).all()
