@@ -61,14 +61,38 @@ typedef struct {
   int32_t sdd_w, sdd_h;    /* SDD grid, 100 x 100 (L155); even, 2 <= sdd <= 4096 */
   int32_t snm_w, snm_h;    /* SNM grid, 50 x 50 (L167); must equal sdd/2 (the 50-grid cells are unions of
                               2x2 100-grid cells, so one pass produces both resizes) */
-  double delta_diff;       /* MSE threshold (L151): pass iff SSD > floor(delta_diff * 3*sdd_w*sdd_h), i.e. iff
-                              MSE > delta_diff exactly; delta_diff >= 0 */
+  double delta_diff;       /* distance threshold (L151), >= 0; for MSE: pass iff SSD > floor(delta_diff * 3*sdd_w*sdd_h),
+                              i.e. iff MSE > delta_diff exactly (other metrics: ffsva_distance) */
   float c_low, c_high;     /* SNM class thresholds (L159), 0 <= c_low <= c_high <= 1 */
   float filter_degree;     /* Eq. (2) (L193); must lie in [0, 1] ("cases t_pre < c_low, t_pre > c_high are not
                               considered") */
   int32_t snm_batch;       /* BatchSize (L219-L223), >= 1; default 30 */
   int32_t q_sdd, q_snm;    /* feedback-queue depth thresholds in frames (L217), default 2 and 10 */
+  int32_t distance;        /* SDD distance (L151 "MSE, NRMSE, or SAD"), an ffsva_distance; 0 = MSE */
+  int32_t ref_mode;        /* SDD reference (L151), an ffsva_ref_mode; 0 = background reference image */
 } ffsva_stream_desc;
+
+/* SDD distance metrics ("The distance between two video frames can be characterized by Mean
+ * Square Error (MSE), Normalized Root Mean Square Error (NRMSE), or Sum of Absolute Differences (SAD)").
+ * D = the frame's sdd_h x sdd_w x 3 resize, R = the reference, N = 3*sdd_w*sdd_h values. ffsva_result.ssd
+ * carries the integer distance numerator the threshold is applied to; every test is exact (Q5,
+ * Q23, Q24):
+ *   MSE   : ssd = sum (D-R)^2;  pass iff ssd/N > delta_diff          <=> ssd > floor(delta_diff * N)
+ *   SAD   : ssd = sum |D-R|;    pass iff ssd > delta_diff            <=> ssd > floor(delta_diff)
+ *   NRMSE : ssd = sum (D-R)^2;  pass iff sqrt(ssd / sum R^2) > delta_diff <=> ssd > floor(delta_diff^2 * sum R^2)
+ *           (Euclidean normalisation; the threshold is recomputed by every ffsva_set_reference. Prepared batches
+ *           snapshot it at ffsva_batch_prepare.) */
+typedef enum { FFSVA_DIST_MSE = 0, FFSVA_DIST_SAD = 1, FFSVA_DIST_NRMSE = 2 } ffsva_distance;
+
+/* SDD reference (the reference image "is usually computed as the average of dozens of background
+ * frames"; Q25 for the alternative):
+ *   BACKGROUND: R is the image ffsva_set_reference built; it changes only when that is called again.
+ *   PREVIOUS  : each frame is compared with the resize of its stream's previous frame. Within a batch
+ *               "previous" follows input order among the stream's frames; the first frame of a batch uses R,
+ *               and after the batch R holds the resize of the stream's last frame of that batch (so consecutive
+ *               batches chain, and ffsva_set_reference seeds the first comparison). MSE and SAD only (NRMSE's
+ *               normaliser would change per frame: EINVAL); batch API only (the online scheduler rejects it). */
+typedef enum { FFSVA_REF_BACKGROUND = 0, FFSVA_REF_PREVIOUS = 1 } ffsva_ref_mode;
 
 /* SNM topology (L159: CONV, CONV, FC). The kernels implement c1 = 16, c2 = 32 on a 50x50 input. */
 typedef struct {
@@ -84,8 +108,9 @@ typedef struct {
 
 /* Per-frame result, in input order. */
 typedef struct {
-  uint64_t ssd;            /* sum over the 3*sdd_w*sdd_h values of (D100 - R)^2; MSE = ssd / (3*sdd_w*sdd_h) */
-  uint8_t sdd_pass;        /* 1 iff MSE > delta_diff (L151) */
+  uint64_t ssd;            /* SDD distance numerator over the 3*sdd_w*sdd_h values: sum (D100 - R)^2 (MSE, NRMSE;
+                              MSE = ssd / (3*sdd_w*sdd_h)) or sum |D100 - R| (SAD) — see ffsva_distance */
+  uint8_t sdd_pass;        /* 1 iff the distance exceeds delta_diff (L151), e.g. MSE > delta_diff */
   uint8_t snm_pass;        /* 1 iff sdd_pass and c >= t_pre (L165) */
   uint8_t snm_class;       /* 0: c < c_low, 1: unsure, 2: c > c_high (L159); 0 if !sdd_pass */
   uint8_t pad;

@@ -33,6 +33,12 @@ ffsva_status validate_desc(const ffsva_stream_desc* d) {
     return fail(FFSVA_EINVAL, "filter_degree must lie in [0, 1] (PAPER.md L193)");
   if (d->snm_batch < 1) return fail(FFSVA_EINVAL, "snm_batch < 1");
   if (d->q_sdd < 0 || d->q_snm < 0) return fail(FFSVA_EINVAL, "negative queue threshold");
+  if (d->distance < FFSVA_DIST_MSE || d->distance > FFSVA_DIST_NRMSE)
+    return fail(FFSVA_EINVAL, "distance must be FFSVA_DIST_MSE, _SAD or _NRMSE");
+  if (d->ref_mode != FFSVA_REF_BACKGROUND && d->ref_mode != FFSVA_REF_PREVIOUS)
+    return fail(FFSVA_EINVAL, "ref_mode must be FFSVA_REF_BACKGROUND or FFSVA_REF_PREVIOUS");
+  if (d->ref_mode == FFSVA_REF_PREVIOUS && d->distance == FFSVA_DIST_NRMSE)
+    return fail(FFSVA_EINVAL, "NRMSE needs a fixed reference (its normaliser is sum R^2)");
   return FFSVA_OK;
 }
 
@@ -86,7 +92,7 @@ FFSVA_API ffsva_status ffsva_open_stream(const ffsva_stream_desc* desc, ffsva_st
     return fail(FFSVA_ENOMEM, "too many open streams on this device");
   }
   const uint64_t nvals = 3ull * (uint64_t)desc->sdd_w * (uint64_t)desc->sdd_h;
-  s->T = exact_threshold(desc->delta_diff, nvals);
+  s->T = stream_threshold(*desc, 0);  // NRMSE: recomputed from sum R^2 by ffsva_set_reference
   const double tpre = ((double)desc->c_high - (double)desc->c_low) * (double)desc->filter_degree + (double)desc->c_low;
   s->L_t = logit_of(tpre);
   s->L_low = logit_of(desc->c_low);
@@ -163,6 +169,16 @@ FFSVA_API ffsva_status ffsva_set_reference(ffsva_stream* s, const uint8_t* frame
   if (e == cudaSuccess) e = cudaDeviceSynchronize();
   cudaFree(tmp);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "reference kernel");
+  if (d.distance == FFSVA_DIST_NRMSE) {
+    // the NRMSE threshold floor(delta^2 * sum R^2) (Q24) depends on R: one 30 KB read-back per call
+    std::vector<uint8_t> r(3ull * d.sdd_w * d.sdd_h);
+    if ((e = cudaMemcpy(r.data(), s->d_ref, r.size(), cudaMemcpyDeviceToHost)) != cudaSuccess)
+      return cuda_fail(ctx, e, "cudaMemcpy(reference sum of squares)");
+    uint64_t q = 0;
+    for (uint8_t v : r) q += (uint64_t)v * v;
+    s->ref_sum_sq = q;
+    s->T = stream_threshold(d, q);
+  }
   s->has_ref = true;
   return FFSVA_OK;
 }

@@ -94,8 +94,11 @@ extern "C" FFSVA_API ffsva_status ffsva_filter_batch_host(const ffsva_frame* fra
     cudaEventRecord(ev_done[k], cs);
   }
   if (st == FFSVA_OK) {
-    // K3 + K4 over the whole batch (they only touch the 7.5 KB D50 images, not the staged frames)
-    if ((e = launch_compact(make_compact_args(b), cs)) != cudaSuccess) st = cuda_fail(ctx, e, "launch_compact");
+    // K2 (PREVIOUS-mode streams) + K3 + K4 over the whole batch (they only touch D100 / D50, not the staged frames)
+    if ((e = launch_prev(make_prev_args(b), cs)) != cudaSuccess) st = cuda_fail(ctx, e, "launch_prev");
+    g_launches += prev_launches(b);
+    if (st == FFSVA_OK && (e = launch_compact(make_compact_args(b), cs)) != cudaSuccess)
+      st = cuda_fail(ctx, e, "launch_compact");
     if (st == FFSVA_OK && (e = launch_snm(make_snm_args(b), cs)) != cudaSuccess) st = cuda_fail(ctx, e, "launch_snm");
     g_launches += 2;
   }

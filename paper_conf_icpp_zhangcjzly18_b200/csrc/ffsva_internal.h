@@ -17,8 +17,12 @@ struct FrameDesc {
   int32_t W, H;            // raw size
   float L_t;               // logit threshold for t_pre (Eq. (2)); pass iff logit >= L_t
   float L_low, L_high;     // logit(c_low), logit(c_high) for the class (L159)
-  int32_t slot;            // stream slot (stats row)
+  uint16_t slot;           // stream slot (stats row; < 65536 slots per device)
+  uint8_t metric;          // SDD distance: kDistMse / kDistSad / kDistNrmse (ffsva_distance)
+  uint8_t mode;            // SDD reference: kRefBackground / kRefPrevious (ffsva_ref_mode)
 };
+constexpr uint8_t kDistMse = 0, kDistSad = 1, kDistNrmse = 2;
+constexpr uint8_t kRefBackground = 0, kRefPrevious = 1;
 static_assert(sizeof(FrameDesc) == 64, "FrameDesc must stay 64 B");
 
 // ------------------------------------------------------------------ SNM packed weight image (global + smem)
@@ -118,6 +122,23 @@ struct SnmArgs {
 cudaError_t launch_snm(const SnmArgs& a, cudaStream_t st);
 int snm_smem_bytes();
 cudaError_t snm_configure();
+
+// Previous-frame reference (ffsva_ref_mode PREVIOUS, Q25). After K1 has written every frame's D100:
+//  K2 sdd_prev_kernel: one CTA per listed frame f, distance of D100[f] against D100[prev] (prev >= 0: the
+//     stream's previous frame in the batch) or the stream's R (prev = -1), added to acc_ssd[f] (K1 added 0);
+//  K2b ref_update_kernel: R of each listed stream <- D100 of its last frame in the batch.
+struct PrevArgs {
+  const FrameDesc* frames;
+  const uint8_t* d100;       // [n][3*sdd_w*sdd_h]
+  int32_t n_values;          // 3*sdd_w*sdd_h
+  const int32_t* pairs;      // [n_pm][2]: (frame, prev frame or -1)
+  int32_t n_pm;
+  const int32_t* last;       // [n_last]: last frame of each PREVIOUS-mode stream (its R is frames[f].ref)
+  int32_t n_last;
+  unsigned long long* acc_ssd;
+  unsigned long long* stats;
+};
+cudaError_t launch_prev(const PrevArgs& a, cudaStream_t st);  // K2 then K2b (2 launches if n_pm > 0)
 
 cudaError_t launch_fill_nan(float* p, int32_t n, cudaStream_t st);
 cudaError_t launch_reference(const uint8_t* frames, int32_t k, int64_t frame_stride, int32_t W, int32_t H,

@@ -159,6 +159,49 @@ uint64_t exact_threshold(double delta, uint64_t n) {
   return (v >> 64) ? UINT64_MAX : (uint64_t)v;
 }
 
+// floor(delta^2 * q) with the product taken exactly: delta = mant * 2^e2, so delta^2 * q = mant^2 * q * 2^(2 e2)
+// with mant^2 < 2^106 and q < 2^64: a 170-bit product held in three 64-bit limbs.
+uint64_t exact_threshold_sq(double delta, uint64_t q) {
+  uint64_t bits;
+  std::memcpy(&bits, &delta, 8);
+  const int expf = (int)((bits >> 52) & 0x7FF);
+  const uint64_t frac = bits & ((1ull << 52) - 1);
+  if ((bits >> 63) || (expf == 0 && frac == 0) || q == 0) return 0;
+  const uint64_t mant = expf ? (frac | (1ull << 52)) : frac;
+  const int e2 = expf ? expf - 1075 : -1074;
+  const unsigned __int128 m2 = (unsigned __int128)mant * mant;  // < 2^106
+  const unsigned __int128 lo = (unsigned __int128)(uint64_t)m2 * q;
+  const unsigned __int128 hi = (unsigned __int128)(uint64_t)(m2 >> 64) * q;  // weight 2^64
+  uint64_t w[3];  // little-endian limbs of m2 * q
+  w[0] = (uint64_t)lo;
+  const unsigned __int128 mid = (lo >> 64) + (uint64_t)hi;
+  w[1] = (uint64_t)mid;
+  w[2] = (uint64_t)(hi >> 64) + (uint64_t)(mid >> 64);
+  const int sh = 2 * e2;  // value = w * 2^sh
+  if (sh >= 0) {
+    if (w[2] || w[1] || sh >= 64 || (sh > 0 && (w[0] >> (64 - sh)))) return UINT64_MAX;
+    return w[0] << sh;
+  }
+  const int r = -sh;
+  if (r >= 192) return 0;
+  // floor(w / 2^r): shift the 192-bit value right by r and saturate to 64 bits
+  uint64_t out[3] = {0, 0, 0};
+  const int limb = r / 64, bit = r % 64;
+  for (int k = 0; k + limb < 3; ++k) {
+    out[k] = w[k + limb] >> bit;
+    if (bit && k + limb + 1 < 3) out[k] |= w[k + limb + 1] << (64 - bit);
+  }
+  return (out[1] || out[2]) ? UINT64_MAX : out[0];
+}
+
+uint64_t stream_threshold(const ffsva_stream_desc& d, uint64_t ref_sum_sq) {
+  switch (d.distance) {
+    case FFSVA_DIST_SAD: return exact_threshold(d.delta_diff, 1);
+    case FFSVA_DIST_NRMSE: return exact_threshold_sq(d.delta_diff, ref_sum_sq);
+    default: return exact_threshold(d.delta_diff, 3ull * (uint64_t)d.sdd_w * (uint64_t)d.sdd_h);
+  }
+}
+
 uint16_t bf16_bits_rne(float x) {
   uint32_t u;
   std::memcpy(&u, &x, 4);
@@ -244,6 +287,8 @@ static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t s
   const size_t o_segb = off; off += al(8 * n);  // seg_batch[cap] then seg_slot[cap]
   const size_t o_xb = off; off += al(4 * (size_t)(sdd_w + 1));
   const size_t o_yb = off; off += al(4 * (size_t)(sdd_h + 1));
+  const size_t o_pm = off; off += al(8 * n);    // PREVIOUS-mode (frame, prev) pairs
+  const size_t o_last = off; off += al(4 * n);  // PREVIOUS-mode streams' last frames
   b->in_bytes = off;
   const size_t o_d50 = off; off += al((size_t)b->d50_stride * n);
   const size_t o_d100 = off; off += d100 ? al((size_t)3 * sdd_w * sdd_h * n) : 0;
@@ -265,6 +310,8 @@ static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t s
   b->d_seg_batch = (int32_t*)(base + o_segb);
   b->d_xb = (int32_t*)(base + o_xb);
   b->d_yb = (int32_t*)(base + o_yb);
+  b->d_pm = (int32_t*)(base + o_pm);
+  b->d_last = (int32_t*)(base + o_last);
   b->d_d50 = base + o_d50;
   b->d_d100 = d100 ? base + o_d100 : nullptr;
   b->d_acc = (unsigned long long*)(base + o_acc);
@@ -308,6 +355,7 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     if ((s->desc.row_pitch & 15) || ((uintptr_t)frames[i].pixels & 15)) vec16 = false;
     max_chunks = std::max(max_chunks, (3 * s->desc.width + 15) / 16);
     stage_bytes = std::max(stage_bytes, sdd_bulk_stage_bytes(s->desc.width, s->desc.height, sdd_h));
+    if (s->desc.ref_mode == FFSVA_REF_PREVIOUS) want_d100 = true;  // K2 reads every frame's D100
   }
   // K1 variant: the bulk-async/cluster kernel needs 16-B aligned rows that fit the shared-memory stage;
   // FFSVA_SDD_KERNEL=stream forces the register-streaming kernel (tests exercise both)
@@ -349,7 +397,9 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     d.L_t = s->L_t;
     d.L_low = s->L_low;
     d.L_high = s->L_high;
-    d.slot = s->slot;
+    d.slot = (uint16_t)s->slot;
+    d.metric = (uint8_t)s->desc.distance;
+    d.mode = (uint8_t)s->desc.ref_mode;
     hperm[i] = i;
     if (i && s->slot < frames[i - 1].stream->slot) sorted = false;
   }
@@ -365,6 +415,32 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     }
   hseg[nseg] = n;
   b->n_seg = nseg;
+  // PREVIOUS-mode plan (Q25): each such frame's previous frame of its stream in input order (-1: the
+  // stream's R), and each such stream's last frame (its D100 becomes the stream's R after the batch)
+  {
+    int32_t* hpm = (int32_t*)(b->h_in + ((uint8_t*)b->d_pm - (uint8_t*)b->d_mem));
+    int32_t* hlast = (int32_t*)(b->h_in + ((uint8_t*)b->d_last - (uint8_t*)b->d_mem));
+    std::vector<std::pair<int32_t, int32_t>> last;  // (slot, latest frame) per PREVIOUS-mode stream
+    int32_t npm = 0;
+    for (int32_t i = 0; i < n; ++i) {
+      if (hd[i].mode != kRefPrevious) continue;
+      auto it = std::find_if(last.begin(), last.end(),
+                             [&](const std::pair<int32_t, int32_t>& p) { return p.first == hd[i].slot; });
+      int32_t prev = -1;
+      if (it != last.end()) {
+        prev = it->second;
+        it->second = i;
+      } else {
+        last.emplace_back(hd[i].slot, i);
+      }
+      hpm[2 * npm] = i;
+      hpm[2 * npm + 1] = prev;
+      ++npm;
+    }
+    for (size_t k = 0; k < last.size(); ++k) hlast[k] = last[k].second;
+    b->n_pm = npm;
+    b->n_last = (int32_t)last.size();
+  }
   // cell boundary tables (C1: cell i covers [floor(i*S/D), floor((i+1)*S/D))) when the batch shares W / H
   int32_t* hxb = (int32_t*)((uint8_t*)b->h_in + ((uint8_t*)b->d_xb - (uint8_t*)b->d_mem));
   int32_t* hyb = (int32_t*)((uint8_t*)b->h_in + ((uint8_t*)b->d_yb - (uint8_t*)b->d_mem));
@@ -453,17 +529,34 @@ SnmArgs make_snm_args(Batch* b) {
   return na;
 }
 
+PrevArgs make_prev_args(Batch* b) {
+  PrevArgs pa{};
+  pa.frames = b->d_desc;
+  pa.d100 = b->d_d100;
+  pa.n_values = 3 * b->sdd_w * b->sdd_h;
+  pa.pairs = b->d_pm;
+  pa.n_pm = b->n_pm;
+  pa.last = b->d_last;
+  pa.n_last = b->n_last;
+  pa.acc_ssd = b->d_acc;
+  pa.stats = b->ctx->d_stats;
+  return pa;
+}
+
+int prev_launches(const Batch* b) { return b->n_pm > 0 ? (b->n_last > 0 ? 2 : 1) : 0; }
+
 static ffsva_status batch_launch_kernels(Batch* b, cudaStream_t st, int* nk, cudaEvent_t* ev = nullptr) {
   DeviceCtx* ctx = b->ctx;
   if (ev) cudaEventRecord(ev[0], st);
   FF_CUDA(ctx, launch_sdd(make_sdd_args(b, 0, b->n), st));
+  FF_CUDA(ctx, launch_prev(make_prev_args(b), st));
   if (ev) cudaEventRecord(ev[1], st);
   FF_CUDA(ctx, launch_compact(make_compact_args(b), st));
   if (ev) cudaEventRecord(ev[2], st);
-  *nk = 2;
+  *nk = 2 + prev_launches(b);
   if (!b->sdd_only) {
     FF_CUDA(ctx, launch_snm(make_snm_args(b), st));
-    *nk = 3;
+    *nk += 1;
   }
   if (ev) cudaEventRecord(ev[3], st);
   return FFSVA_OK;

@@ -27,7 +27,8 @@ struct StreamState {
   uint8_t* d_ref = nullptr;   // R [sdd_h][sdd_w][3]
   uint8_t* d_snm = nullptr;   // packed SNM weight image (snm::BLOB_BYTES)
   bool has_ref = false, has_snm = false;
-  uint64_t T = 0;             // SDD threshold on SSD
+  uint64_t T = 0;             // SDD threshold on the distance numerator (ffsva_distance)
+  uint64_t ref_sum_sq = 0;    // sum R^2 of the reference (NRMSE normaliser)
   float L_t = 0.f, L_low = 0.f, L_high = 0.f;
 };
 
@@ -41,6 +42,8 @@ struct Batch {
   int32_t stage_bytes = 0;
   int32_t uni_W = -1, uni_H = -1;        // common frame size of the batch (-1: mixed)
   int32_t *d_xb = nullptr, *d_yb = nullptr;  // cell boundary tables for uni_W / uni_H (in the input block)
+  int32_t *d_pm = nullptr, *d_last = nullptr;  // PREVIOUS-mode plan (input block): (frame, prev) pairs, last frames
+  int32_t n_pm = 0, n_last = 0;
   int64_t d50_stride = 0;
   // device buffers (carved from one allocation)
   void* d_mem = nullptr;
@@ -95,6 +98,8 @@ void ctx_release(DeviceCtx* ctx);                       // decrements; destroys 
 ffsva_status check_device_ptr(DeviceCtx* ctx, const void* p, size_t bytes);
 ffsva_status ensure_stats(DeviceCtx* ctx, int32_t slots);
 uint64_t exact_threshold(double delta, uint64_t n_values);
+uint64_t exact_threshold_sq(double delta, uint64_t q);  // floor(delta^2 * q), exact (NRMSE, Q24)
+uint64_t stream_threshold(const ffsva_stream_desc& d, uint64_t ref_sum_sq);  // T of the stream's metric
 uint16_t bf16_bits_rne(float x);
 void pack_snm_blob(const float* params, uint8_t* blob);
 float logit_of(double t);
@@ -109,6 +114,8 @@ void batch_free(Batch* b);
 SddArgs make_sdd_args(Batch* b, int32_t i0, int32_t cnt);  // K1 over frames [i0, i0 + cnt) of the batch
 CompactArgs make_compact_args(Batch* b);
 SnmArgs make_snm_args(Batch* b);
+PrevArgs make_prev_args(Batch* b);
+int prev_launches(const Batch* b);  // kernels launch_prev issues for this batch (0, 1 or 2)
 
 // RAII device switch
 struct DeviceGuard {

@@ -93,7 +93,9 @@ FrameDesc make_desc(const ffsva_stream* st, const void* pixels) {
   d.L_t = st->L_t;
   d.L_low = st->L_low;
   d.L_high = st->L_high;
-  d.slot = st->slot;
+  d.slot = (uint16_t)st->slot;
+  d.metric = (uint8_t)st->desc.distance;
+  d.mode = (uint8_t)st->desc.ref_mode;
   return d;
 }
 
@@ -169,6 +171,8 @@ FFSVA_API ffsva_status ffsva_sched_push(ffsva_sched* s, const ffsva_frame* frame
     if (st->ctx != s->ctx) return fail(FFSVA_EDEVICE, "stream lives on another device");
     if (!st->has_ref || !st->has_snm) return fail(FFSVA_ESTATE, "stream has no reference image or no SNM");
     if (st->desc.snm_w != snm::IN || st->desc.snm_h != snm::IN) return fail(FFSVA_EINVAL, "SNM grid must be 50x50");
+    if (st->desc.ref_mode != FFSVA_REF_BACKGROUND)
+      return fail(FFSVA_EINVAL, "the online scheduler takes background-reference streams only");
     if (s->sdd_w < 0) {  // one SDD grid per scheduler (one K1 launch per cycle)
       s->sdd_w = st->desc.sdd_w;
       s->sdd_h = st->desc.sdd_h;

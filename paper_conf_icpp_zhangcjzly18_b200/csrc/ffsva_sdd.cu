@@ -147,6 +147,11 @@ __device__ __forceinline__ void fill_xbounds(int* xb, int W, int sdd_w) {
   for (int i = threadIdx.x; i <= sdd_w; i += blockDim.x) xb[i] = (int)(((uint32_t)i * (uint32_t)W) / (uint32_t)sdd_w);
 }
 
+// One value's share of the SDD distance: (D - R)^2 for MSE and NRMSE, |D - R| for SAD.
+__device__ __forceinline__ uint32_t dist_term(int diff, uint8_t metric) {
+  return metric == kDistSad ? (uint32_t)abs(diff) : (uint32_t)(diff * diff);
+}
+
 // Block-reduce this thread's SSD share; thread 0 adds it to the frame's accumulator and the stream's stats.
 __device__ __forceinline__ void ssd_commit(uint32_t v, uint32_t* red, const SddArgs& a, int f, int slot,
                                            bool count_frame) {
@@ -228,8 +233,9 @@ __global__ void __launch_bounds__(512) sdd_kernel(SddArgs a) {
     const int yrow = 2 * band + sub;
     if (kD100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)yrow * row3 + r] = (uint8_t)d;
     const int diff = (int)d - (int)__ldg(fd.ref + (int64_t)yrow * row3 + r);
-    ssd_local += (uint32_t)(diff * diff);
+    ssd_local += dist_term(diff, fd.metric);
   }
+  if (fd.mode == kRefPrevious) ssd_local = 0;  // K2 measures against the previous frame's D100
   __syncthreads();
 
   // ---- phase 3: D50 row from the four 100-cell sums of each 50-cell
@@ -382,8 +388,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
     const uint32_t d = (s + (n >> 1)) / n;
     if (kD100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)r * row3 + o] = (uint8_t)d;
     const int diff = (int)d - (int)__ldg(fd.ref + (int64_t)r * row3 + o);
-    ssd_local += (uint32_t)(diff * diff);
+    ssd_local += dist_term(diff, fd.metric);
   }
+  if (fd.mode == kRefPrevious) ssd_local = 0;  // K2 measures against the previous frame's D100
   __syncthreads();
 
   // ---- D50 row: odd CTA -> even CTA (st.async into the peer's shared memory), even CTA combines 2x2 cells.
@@ -427,6 +434,63 @@ __global__ void reference_kernel(const uint8_t* __restrict__ frames, int32_t k, 
     }
   const unsigned long long n = (unsigned long long)k * (unsigned long long)((y1 - y0) * (x1 - x0));
   out[o] = (uint8_t)((s + n / 2) / n);
+}
+
+// K2: distance of a PREVIOUS-mode frame's D100 to its stream's previous D100 (or R for the stream's first frame
+// of the batch). One CTA per frame; 16-byte loads of two L2-resident 30 KB images (K1 wrote them just before).
+constexpr int kPrevThreads = 256;
+__global__ void __launch_bounds__(kPrevThreads) sdd_prev_kernel(PrevArgs a) {
+  __shared__ uint32_t red[kPrevThreads / 32];
+  const int f = a.pairs[2 * blockIdx.x], prev = a.pairs[2 * blockIdx.x + 1];
+  const FrameDesc& fd = a.frames[f];
+  const uint8_t* x = a.d100 + (int64_t)f * a.n_values;
+  const uint8_t* r = prev >= 0 ? a.d100 + (int64_t)prev * a.n_values : fd.ref;
+  const bool sad = fd.metric == kDistSad;
+  uint32_t acc = 0;
+  const int nv16 = a.n_values >> 4;  // n_values = 3*sdd_w*sdd_h, sdd_w and sdd_h even: a multiple of 4 only
+  if ((a.n_values & 15) == 0) {
+    for (int i = threadIdx.x; i < nv16; i += kPrevThreads) {
+      const uint4 u = reinterpret_cast<const uint4*>(x)[i], v = reinterpret_cast<const uint4*>(r)[i];
+      const uint32_t uw[4] = {u.x, u.y, u.z, u.w}, vw[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        if (sad) {
+          acc = __vsadu4(uw[k], vw[k]) + acc;
+        } else {
+#pragma unroll
+          for (int b = 0; b < 4; ++b) {
+            const int d = (int)((uw[k] >> (8 * b)) & 255u) - (int)((vw[k] >> (8 * b)) & 255u);
+            acc += (uint32_t)(d * d);
+          }
+        }
+      }
+    }
+  } else {
+    for (int i = threadIdx.x; i < a.n_values; i += kPrevThreads) acc += dist_term((int)x[i] - (int)r[i], fd.metric);
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = acc;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long t = 0;
+    for (int w = 0; w < kPrevThreads / 32; ++w) t += red[w];
+    atomicAdd(a.acc_ssd + f, t);
+    if (a.stats) atomicAdd(a.stats + (int64_t)fd.slot * NSTAT + 3, t);
+  }
+}
+
+// K2b: the stream's reference becomes the D100 of its last frame in the batch (runs after every K2 read of R).
+__global__ void __launch_bounds__(kPrevThreads) ref_update_kernel(PrevArgs a) {
+  const int f = a.last[blockIdx.x];
+  const uint8_t* src = a.d100 + (int64_t)f * a.n_values;
+  uint8_t* dst = const_cast<uint8_t*>(a.frames[f].ref);
+  if ((a.n_values & 15) == 0) {
+    for (int i = threadIdx.x; i < (a.n_values >> 4); i += kPrevThreads)
+      reinterpret_cast<uint4*>(dst)[i] = reinterpret_cast<const uint4*>(src)[i];
+  } else {
+    for (int i = threadIdx.x; i < a.n_values; i += kPrevThreads) dst[i] = src[i];
+  }
 }
 
 __global__ void fill_nan_kernel(float* p, int32_t n) {
@@ -497,6 +561,15 @@ cudaError_t launch_reference(const uint8_t* frames, int32_t k, int64_t frame_str
                              int64_t pitch, int32_t sdd_w, int32_t sdd_h, uint8_t* out, cudaStream_t st) {
   const int n = 3 * sdd_w * sdd_h;
   reference_kernel<<<(n + 127) / 128, 128, 0, st>>>(frames, k, frame_stride, W, H, pitch, sdd_w, sdd_h, out);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_prev(const PrevArgs& a, cudaStream_t st) {
+  if (a.n_pm <= 0) return cudaSuccess;
+  sdd_prev_kernel<<<a.n_pm, kPrevThreads, 0, st>>>(a);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess || a.n_last <= 0) return e;
+  ref_update_kernel<<<a.n_last, kPrevThreads, 0, st>>>(a);
   return cudaGetLastError();
 }
 

@@ -39,7 +39,13 @@ class StreamDesc(ctypes.Structure):
                 ("row_pitch", ctypes.c_int64), ("sdd_w", ctypes.c_int32), ("sdd_h", ctypes.c_int32),
                 ("snm_w", ctypes.c_int32), ("snm_h", ctypes.c_int32), ("delta_diff", ctypes.c_double),
                 ("c_low", ctypes.c_float), ("c_high", ctypes.c_float), ("filter_degree", ctypes.c_float),
-                ("snm_batch", ctypes.c_int32), ("q_sdd", ctypes.c_int32), ("q_snm", ctypes.c_int32)]
+                ("snm_batch", ctypes.c_int32), ("q_sdd", ctypes.c_int32), ("q_snm", ctypes.c_int32),
+                ("distance", ctypes.c_int32), ("ref_mode", ctypes.c_int32)]
+
+
+# ffsva_distance / ffsva_ref_mode (include/ffsva.h)
+DISTANCES = {"mse": 0, "sad": 1, "nrmse": 2}
+REF_MODES = {"background": 0, "previous": 1}
 
 
 class SnmDesc(ctypes.Structure):
@@ -314,9 +320,11 @@ class Context:
 
     def open_stream(self, width: int, height: int, row_pitch: int | None = None, delta_diff: float = 24.0,
                     c_low: float = 0.2, c_high: float = 0.8, filter_degree: float = 0.5, snm_batch: int = 30,
-                    q_sdd: int = 2, q_snm: int = 10, sdd=(100, 100)) -> Stream:
+                    q_sdd: int = 2, q_snm: int = 10, sdd=(100, 100), distance: str = "mse",
+                    ref_mode: str = "background") -> Stream:
         d = StreamDesc(self.device, width, height, 3 * width if row_pitch is None else row_pitch, sdd[0], sdd[1],
-                       sdd[0] // 2, sdd[1] // 2, delta_diff, c_low, c_high, filter_degree, snm_batch, q_sdd, q_snm)
+                       sdd[0] // 2, sdd[1] // 2, delta_diff, c_low, c_high, filter_degree, snm_batch, q_sdd, q_snm,
+                       DISTANCES[distance], REF_MODES[ref_mode])
         s = Stream(self, d)
         self.streams.append(s)
         return s

@@ -21,13 +21,16 @@ class Cam:
     """One synthetic camera: its video, its reference frames and its SNM weights."""
 
     def __init__(self, ctx, video: synth.Video, stream_id: int, dev, delta=24.0, c_low=0.2, c_high=0.8, fd=0.5,
-                 snm_batch=30, pitch=None, k_ref=8, bias_std=0.05, load_snm=True):
+                 snm_batch=30, pitch=None, k_ref=8, bias_std=0.05, load_snm=True, distance="mse",
+                 ref_mode="background"):
         import torch
         self.video, self.sid, self.dev = video, stream_id, dev
         self.pitch = 3 * video.width if pitch is None else pitch
         self.delta, self.c_low, self.c_high, self.fd = delta, c_low, c_high, fd
+        self.distance, self.ref_mode = distance, ref_mode
         self.st = ctx.open_stream(width=video.width, height=video.height, row_pitch=self.pitch, delta_diff=delta,
-                                  c_low=c_low, c_high=c_high, filter_degree=fd, snm_batch=snm_batch)
+                                  c_low=c_low, c_high=c_high, filter_degree=fd, snm_batch=snm_batch,
+                                  distance=distance, ref_mode=ref_mode)
         self.refs = synth.frames(video, [stream_id] * k_ref, list(range(k_ref)), ref=True, pitch=self.pitch)
         self.st.set_reference(torch.from_numpy(self.refs).to(dev))
         self.R = orc.reference(self.refs, video.width, 100, 100)
@@ -48,7 +51,9 @@ def oracle_for(cams_and_frames, run_snm=True, bf16_emul=False):
     assert len(widths) == 1
     return orc.filter_frames(frames, cams[0].video.width, [c.R for c in cams], [c.delta for c in cams],
                              [c.params for c in cams], [f32(c.c_low) for c in cams], [f32(c.c_high) for c in cams],
-                             [f32(c.fd) for c in cams], bf16_emul=bf16_emul, run_snm=run_snm)
+                             [f32(c.fd) for c in cams], bf16_emul=bf16_emul, run_snm=run_snm,
+                             metrics=[c.distance for c in cams], ref_modes=[c.ref_mode for c in cams],
+                             stream_ids=[id(c) for c in cams])
 
 
 def oracle_mixed(cams_and_frames, run_snm=True, bf16_emul=False):
