@@ -244,6 +244,17 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
 FFSVA_API ffsva_status ffsva_sched_depth(ffsva_sched* s, ffsva_stream* st, int32_t* sdd_depth, int32_t* snm_depth);
 FFSVA_API ffsva_status ffsva_sched_destroy(ffsva_sched* s);
 
+/* SNM batch trigger of the online runtime, for the paper's batch-mechanism comparison (§4.3.2,
+ * §5.4; Q26):
+ *   DYNAMIC  (default, the paper's method, L223): each cycle pops min(BatchSize, depth) frames per stream;
+ *   FEEDBACK : fixed-size batches under the feedback queue: a stream pops BatchSize frames only once its SNM
+ *              queue holds that many, or its whole queue once that queue blocks its SDD stage (depth > q_snm);
+ *   STATIC   : fixed-size batches without SNM->SDD feedback (q_snm ignored; the slot pool bounds the queues).
+ * Under FEEDBACK / STATIC, a cycle in which nothing can pop while every D50 slot is taken pops the fullest queue
+ * (no deadlock). Frames left in partial batches at the end of input are drained by switching back to DYNAMIC. */
+typedef enum { FFSVA_BATCH_DYNAMIC = 0, FFSVA_BATCH_FEEDBACK = 1, FFSVA_BATCH_STATIC = 2 } ffsva_batch_policy;
+FFSVA_API ffsva_status ffsva_sched_set_policy(ffsva_sched* s, int32_t policy);
+
 /* Close a stream (NULL is a no-op). */
 FFSVA_API ffsva_status ffsva_close(ffsva_stream* s);
 

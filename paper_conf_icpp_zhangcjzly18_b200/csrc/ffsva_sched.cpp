@@ -207,6 +207,13 @@ FFSVA_API ffsva_status ffsva_sched_depth(ffsva_sched* s, ffsva_stream* st, int32
   return FFSVA_OK;
 }
 
+FFSVA_API ffsva_status ffsva_sched_set_policy(ffsva_sched* s, int32_t policy) {
+  if (!s || policy < FFSVA_BATCH_DYNAMIC || policy > FFSVA_BATCH_STATIC) return fail(FFSVA_EINVAL, "bad argument");
+  std::lock_guard<std::mutex> lk(s->mu);
+  s->pol.set_policy((sched::BatchPolicy)policy);
+  return FFSVA_OK;
+}
+
 FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva_event* events, int32_t cap,
                                         int32_t* n_events, ffsva_tick_info* info) {
   if (!s || cap < 0 || (cap > 0 && !events) || !n_events) return fail(FFSVA_EINVAL, "bad argument");
@@ -331,11 +338,12 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
     }
   }
 
-  // ---------------- SNM cycle: dynamic batching (pops of min(BatchSize, depth) per stream)
+  // ---------------- SNM cycle: dynamic batching (pops of min(BatchSize, depth) per stream; or the static /
+  // feedback-queue fixed-size trigger chosen by ffsva_sched_set_policy)
   const auto t_snm0 = std::chrono::steady_clock::now();
   std::vector<sched::QFrame>& flat = s->flat;
   std::vector<int32_t>& starts = s->starts;
-  s->pol.pop_snm(flat, starts);
+  s->pol.pop_snm(flat, starts, (int32_t)s->free_slots.size());
   const int32_t m = (int32_t)flat.size();
   ti.snm_batches = (int32_t)starts.size() - 1;
   ti.snm_scored = m;

@@ -10,6 +10,20 @@
 //     T-YOLO, which is out of scope, so nothing blocks it;
 //   * dynamic batching (L223): each SNM cycle pops min(BatchSize, depth) frames of every non-empty stream.
 // Streams are visited round-robin (the start rotates every cycle) so a per-cycle frame budget is shared fairly.
+//
+// The two batch mechanisms the paper compares dynamic batching with (§4.3.2, §5.4; f4) are
+// selectable for that study (BatchPolicy, Q26):
+//   * STATIC  — "a triggering strategy based on a fixed number of input frames per batch": the SNM pops exactly
+//               BatchSize frames of a stream once its queue holds that many; no feedback from the SNM queue to
+//               the SDD stage (q_snm is ignored; the device slot pool is the only bound);
+//   * FEEDBACK — the same fixed-size trigger under the feedback queue (the SDD stage skips a stream whose SNM
+//               queue holds more than q_snm frames). "When the batch size is greater than the queue depth
+//               threshold, video frames have to wait in the SNM" (L221): a stream whose SDD stage is blocked
+//               (depth > q_snm) has its queue popped whole, otherwise it would wait forever;
+//   * DYNAMIC — the paper's method (default).
+// Under STATIC and FEEDBACK, when no stream can pop and the slot pool is exhausted (every slot holds a partial
+// batch) the fullest queue is popped, so the runtime cannot deadlock. To drain at the end of input, switch the
+// policy back to DYNAMIC.
 #pragma once
 
 #include <algorithm>
@@ -27,6 +41,8 @@ struct QFrame {
   int32_t slot = -1;          // device D50 slot while the frame sits in the SNM queue
   uint64_t ssd = 0;           // SDD distance, carried to the frame's final event
 };
+
+enum class BatchPolicy : int32_t { DYNAMIC = 0, FEEDBACK = 1, STATIC = 2 };
 
 struct StreamQ {
   int32_t q_sdd = 2, q_snm = 10, batch = 30;
@@ -91,7 +107,7 @@ class Policy {
     for (int32_t k = 0; k < n && limit > 0; ++k) {
       StreamQ& s = st_[(rr_ + k) % n];
       if (!s.live || s.sdd.empty()) continue;
-      if ((int32_t)s.snm.size() > s.q_snm) {
+      if (policy_ != BatchPolicy::STATIC && (int32_t)s.snm.size() > s.q_snm) {
         ++s.sdd_blocked;
         continue;
       }
@@ -113,27 +129,47 @@ class Policy {
     s.max_snm = std::max(s.max_snm, (int32_t)s.snm.size());
   }
 
-  // SNM stage of one cycle (dynamic batching, L223): every non-empty stream pops min(BatchSize, depth).
+  // SNM stage of one cycle. DYNAMIC (L223): every non-empty stream pops min(BatchSize, depth). STATIC /
+  // FEEDBACK: a stream pops BatchSize frames only when it holds that many (FEEDBACK also pops a stream whose
+  // SDD stage it blocks). `slots_free` = free device D50 slots (deadlock guard, see above).
   // The pops are appended to `flat`; pop p is flat[starts[p] .. starts[p+1]) (starts gets a final sentinel).
-  void pop_snm(std::vector<QFrame>& flat, std::vector<int32_t>& starts) {
+  void pop_snm(std::vector<QFrame>& flat, std::vector<int32_t>& starts, int32_t slots_free = 1 << 30) {
     flat.clear();
     starts.clear();
     const int32_t n = (int32_t)st_.size();
-    for (int32_t k = 0; k < n; ++k) {
-      StreamQ& s = st_[k];
-      if (!s.live || s.snm.empty()) continue;
-      const int32_t take = std::min<int32_t>(s.batch, (int32_t)s.snm.size());
+    auto take_from = [&](StreamQ& s, int32_t take) {
       starts.push_back((int32_t)flat.size());
       flat.insert(flat.end(), s.snm.begin(), s.snm.begin() + take);
       s.snm.erase(s.snm.begin(), s.snm.begin() + take);
+    };
+    for (int32_t k = 0; k < n; ++k) {
+      StreamQ& s = st_[k];
+      if (!s.live || s.snm.empty()) continue;
+      const int32_t depth = (int32_t)s.snm.size();
+      if (policy_ == BatchPolicy::DYNAMIC) {
+        take_from(s, std::min(s.batch, depth));
+      } else if (depth >= s.batch) {
+        take_from(s, s.batch);
+      } else if (policy_ == BatchPolicy::FEEDBACK && depth > s.q_snm) {
+        take_from(s, depth);
+      }
+    }
+    if (flat.empty() && slots_free <= 0) {  // every slot holds a partial batch: pop the fullest queue
+      int32_t best = -1;
+      for (int32_t k = 0; k < n; ++k)
+        if (st_[k].live && !st_[k].snm.empty() && (best < 0 || st_[k].snm.size() > st_[best].snm.size())) best = k;
+      if (best >= 0) take_from(st_[best], std::min(st_[best].batch, (int32_t)st_[best].snm.size()));
     }
     starts.push_back((int32_t)flat.size());
   }
 
-  std::vector<std::vector<QFrame>> pop_snm() {  // convenience form for tests
+  void set_policy(BatchPolicy p) { policy_ = p; }
+  BatchPolicy policy() const { return policy_; }
+
+  std::vector<std::vector<QFrame>> pop_snm(int32_t slots_free = 1 << 30) {  // convenience form for tests
     std::vector<QFrame> flat;
     std::vector<int32_t> starts;
-    pop_snm(flat, starts);
+    pop_snm(flat, starts, slots_free);
     std::vector<std::vector<QFrame>> pops;
     for (size_t p = 0; p + 1 < starts.size(); ++p)
       pops.emplace_back(flat.begin() + starts[p], flat.begin() + starts[p + 1]);
@@ -156,6 +192,7 @@ class Policy {
  private:
   std::vector<StreamQ> st_;
   int32_t rr_ = 0;
+  BatchPolicy policy_ = BatchPolicy::DYNAMIC;
 };
 
 }  // namespace sched

@@ -31,7 +31,7 @@ EXPORTS = ["ffsva_open_stream", "ffsva_set_reference", "ffsva_snm_load", "ffsva_
            "ffsva_get_reference",
            "ffsva_stream_info", "ffsva_stats_copy", "ffsva_close", "ffsva_last_error", "ffsva_kernel_launches",
            "ffsva_version", "ffsva_sched_create", "ffsva_sched_push", "ffsva_sched_tick", "ffsva_sched_depth",
-           "ffsva_sched_destroy"]
+           "ffsva_sched_destroy", "ffsva_sched_set_policy"]
 
 
 class StreamDesc(ctypes.Structure):
@@ -112,6 +112,7 @@ def lib():
             "ffsva_sched_tick": [vp, vp, vp, i32, ctypes.POINTER(i32), ctypes.POINTER(TickInfo)],
             "ffsva_sched_depth": [vp, vp, ctypes.POINTER(i32), ctypes.POINTER(i32)],
             "ffsva_sched_destroy": [vp],
+            "ffsva_sched_set_policy": [vp, i32],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -401,6 +402,14 @@ def ffsva_sched_destroy(sched) -> None:
     _check(lib().ffsva_sched_destroy(sched), "ffsva_sched_destroy")
 
 
+# ffsva_batch_policy (include/ffsva.h; §4.3.2, §5.4)
+BATCH_POLICIES = {"dynamic": 0, "feedback": 1, "static": 2}
+
+
+def ffsva_sched_set_policy(sched, policy: str) -> None:
+    _check(lib().ffsva_sched_set_policy(sched, BATCH_POLICIES[policy]), "ffsva_sched_set_policy")
+
+
 FRAME_DTYPE = np.dtype([("stream", "<u8"), ("pixels", "<u8"), ("frame_no", "<i8")], align=True)
 
 
@@ -429,6 +438,10 @@ class Scheduler:
 
     def depth(self, st: "Stream"):
         return ffsva_sched_depth(self.handle, st.handle)
+
+    def set_policy(self, policy: str) -> None:
+        """'dynamic' (default), 'feedback' or 'static' (the §5.4 comparison mechanisms)."""
+        ffsva_sched_set_policy(self.handle, policy)
 
     def destroy(self) -> None:
         if self.handle:

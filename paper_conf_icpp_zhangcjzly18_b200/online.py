@@ -96,3 +96,72 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
     res["sustained"] = bool(res["latency_p99_s"] <= latency_budget_s and backlog_end <= S * 2
                             and done >= 0.9 * S * fps * (seconds - latency_budget_s))
     return res
+
+
+def run_unpaced(ctx, streams, content, n_content_frames, seconds, policy="dynamic", cuda_stream=None,
+                max_frames_per_tick=None, snm_slots=None):
+    """Saturated run of the online runtime for the batch-mechanism comparison (§5.4, f4): every camera
+    always has its next frame ready (the prefetcher re-offers whatever the feedback queue refused), so the
+    decided-frame rate is the runtime's throughput; latency is push-acceptance -> decision of each frame.
+    `policy` is the SNM batch trigger ('dynamic', 'feedback', 'static'; ffsva_sched_set_policy). After the timed
+    window the policy switches to dynamic and the queues are drained (not counted)."""
+    import torch
+
+    from .ffsva import FRAME_DTYPE, Scheduler
+
+    S = len(streams)
+    handles = np.array([s.handle for s in streams], dtype=np.uint64)
+    order = np.argsort(handles)
+    sorted_handles = handles[order]
+    base_ptr = np.array([c.data_ptr() for c in content], dtype=np.uint64)
+    fbytes = np.array([c[0].numel() for c in content], dtype=np.uint64)
+    start_frame = (np.arange(S) * 37) % n_content_frames
+    q_sdd = np.array([s.desc.q_sdd for s in streams], dtype=np.int64)
+    pushed = np.zeros(S, np.int64)
+    RING = 1 << 14
+    t_push = np.zeros((S, RING), np.float64)  # acceptance time of frame k of stream s at [s, k % RING]
+    mf = max_frames_per_tick or max(256, S * 8)
+    slots = snm_slots or max(1024, S * (max(s.desc.snm_batch for s in streams) + 16))
+    sched = Scheduler(ctx, max_frames_per_tick=mf, snm_slots=slots)
+    sched.set_policy(policy)
+    lat, done, ticks, pops, scored = [], 0, 0, 0, 0
+    try:
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        while True:
+            now = time.perf_counter()
+            if now - t0 > seconds:
+                break
+            take = q_sdd + 1
+            idx = np.repeat(np.arange(S), take)
+            k = pushed[idx] + (np.arange(idx.size) - np.repeat(np.cumsum(take) - take, take))
+            fr = np.zeros(idx.size, dtype=FRAME_DTYPE)
+            fr["stream"] = handles[idx]
+            fr["pixels"] = base_ptr[idx] + ((start_frame[idx] + k) % n_content_frames).astype(np.uint64) * fbytes[idx]
+            fr["frame_no"] = k
+            acc = sched.push_array(fr) == 1
+            t_push[idx[acc], k[acc] % RING] = time.perf_counter()
+            pushed += np.bincount(idx[acc], minlength=S)
+            ev, info = sched.tick(cuda_stream)
+            t_done = time.perf_counter()
+            ticks += 1
+            pops += info["snm_batches"]
+            scored += info["snm_scored"]
+            if ev.size:
+                si = order[np.searchsorted(sorted_handles, ev["stream"])]
+                lat.append(t_done - t_push[si, ev["frame_no"] % RING])
+                done += ev.size
+        elapsed = time.perf_counter() - t0
+        sched.set_policy("dynamic")
+        for _ in range(10000):
+            ev, info = sched.tick(cuda_stream)
+            if info["sdd_queued"] == 0 and info["snm_queued"] == 0 and info["events_pending"] == 0:
+                break
+    finally:
+        sched.destroy()
+    L = np.concatenate(lat) if lat else np.zeros(1)
+    return {"policy": policy, "streams": S, "seconds": elapsed, "ticks": ticks, "frames_decided": int(done),
+            "fps": done / elapsed, "latency_mean_ms": 1e3 * float(L.mean()),
+            "latency_p50_ms": 1e3 * float(np.percentile(L, 50)), "latency_p99_ms": 1e3 * float(np.percentile(L, 99)),
+            "snm_scored": int(scored), "snm_batches": int(pops),
+            "mean_snm_batch": scored / pops if pops else 0.0}

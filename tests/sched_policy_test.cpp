@@ -98,6 +98,48 @@ int main() {
     CHECK(left.size() == 2 && !p.live(s));
     CHECK(p.add_stream(1, 1, 1) == s);
   }
+  {  // STATIC (L221 "a triggering strategy based on a fixed number of input frames per batch"): no pop until
+     // BatchSize frames are queued, exactly BatchSize per pop, and the SNM queue never blocks the SDD stage
+    Policy p;
+    p.set_policy(ffsva::sched::BatchPolicy::STATIC);
+    int s = p.add_stream(100, 2, 4);
+    for (int i = 0; i < 3; ++i) p.push(s, fr(i));
+    for (auto& f : p.admit_sdd(100, 100)) p.sdd_done(f, true);
+    CHECK(p.pop_snm().empty());                    // 3 < 4 frames: wait (the latency cost, L221)
+    for (int i = 3; i < 9; ++i) p.push(s, fr(i));
+    auto a = p.admit_sdd(100, 100);
+    CHECK(a.size() == 6);                          // depth 3 > q_snm = 2 would block FEEDBACK, not STATIC
+    for (auto& f : a) p.sdd_done(f, true);
+    auto pops = p.pop_snm();
+    CHECK(pops.size() == 1 && pops[0].size() == 4 && pops[0][0].frame_no == 0 && pops[0][3].frame_no == 3);
+    pops = p.pop_snm();
+    CHECK(pops.size() == 1 && pops[0].size() == 4 && pops[0][0].frame_no == 4);
+    CHECK(p.pop_snm().empty() && p.queued_snm() == 1);  // frame 8 waits for a full batch
+    CHECK(p.pop_snm(0).size() == 1);               // unless the slot pool is exhausted (deadlock guard)
+  }
+  {  // FEEDBACK: fixed-size trigger under the feedback queue; a queue that blocks its SDD stage (depth > q_snm)
+     // is popped whole even below BatchSize (L221: BatchSize > threshold would otherwise wait forever)
+    Policy p;
+    p.set_policy(ffsva::sched::BatchPolicy::FEEDBACK);
+    int s = p.add_stream(100, 2, 5);
+    for (int i = 0; i < 2; ++i) p.push(s, fr(i));
+    for (auto& f : p.admit_sdd(100, 100)) p.sdd_done(f, true);
+    CHECK(p.pop_snm().empty());                    // depth 2 <= q_snm, < BatchSize: wait
+    p.push(s, fr(2));
+    for (auto& f : p.admit_sdd(100, 100)) p.sdd_done(f, true);
+    p.push(s, fr(3));
+    CHECK(p.admit_sdd(100, 100).empty());          // depth 3 > 2: SDD blocked
+    auto pops = p.pop_snm();
+    CHECK(pops.size() == 1 && pops[0].size() == 3 && pops[0][2].frame_no == 2);
+    auto b = p.admit_sdd(100, 100);
+    CHECK(b.size() == 1 && b[0].frame_no == 3);    // unblocked
+    // switching back to DYNAMIC drains partial batches (end of input)
+    p.sdd_done(b[0], true);
+    CHECK(p.pop_snm().empty());
+    p.set_policy(ffsva::sched::BatchPolicy::DYNAMIC);
+    pops = p.pop_snm();
+    CHECK(pops.size() == 1 && pops[0].size() == 1 && pops[0][0].frame_no == 3);
+  }
   if (failures == 0) std::printf("ALL PASS\n");
   return failures == 0 ? 0 : 1;
 }

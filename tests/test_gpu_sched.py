@@ -90,3 +90,57 @@ def test_online_feedback_queue_and_dynamic_batching(env):
             assert abs(float(r["logit"]) - w["logit"][0]) <= SNM_TOL, (s, t)
         else:
             assert np.isnan(r["logit"])
+
+
+@pytest.mark.parametrize("policy", ["static", "feedback"])
+def test_fixed_size_batch_policies(env, policy):
+    """f4 (§4.3.2, §5.4): under STATIC every SNM pop is exactly BatchSize frames until the end of
+    input is drained in DYNAMIC mode; under FEEDBACK a pop is either a full batch or a queue that blocked its SDD
+    stage (> q_snm frames). Every frame still comes back once with the oracle's SDD result."""
+    ff, ctx, dev = env
+    import torch
+    from paper_conf_icpp_zhangcjzly18_b200.ffsva import Scheduler
+    B, q_snm = 4, 5
+    v = synth.Video(seed=67, width=640, height=360, period=6, on_len=5)
+    cams = [Cam(ctx, v, s, dev, k_ref=2, load_snm=True) for s in range(2)]
+    for c in cams:
+        c.st.close()
+        c.st = ctx.open_stream(width=640, height=360, delta_diff=24.0, snm_batch=B, q_sdd=2, q_snm=q_snm)
+        c.st.set_reference(torch.from_numpy(c.refs).to(dev))
+        c.st.snm_load(c.params)
+    T = 30
+    dev_frames = [torch.from_numpy(c.host_frames(list(range(T)))).to(dev) for c in cams]
+    sched = Scheduler(ctx, max_frames_per_tick=64, snm_slots=64)
+    sched.set_policy(policy)
+    nxt = [0, 0]
+    got = {}
+    cs = torch.cuda.Stream()
+    for step in range(400):
+        items = [(cams[s].st, dev_frames[s][t], t) for s in range(2) for t in range(nxt[s], min(T, nxt[s] + 3))]
+        if items:
+            acc = sched.push(items)
+            for (st, _, t), a in zip(items, acc):
+                s = 0 if st is cams[0].st else 1
+                if a and t == nxt[s]:
+                    nxt[s] += 1
+        if nxt == [T, T]:
+            sched.set_policy("dynamic")  # end of input: drain partial batches
+        ev, info = sched.tick(cs)
+        if nxt != [T, T] and info["snm_batches"]:
+            per = info["snm_scored"] / info["snm_batches"]
+            if policy == "static":
+                assert info["snm_scored"] == B * info["snm_batches"], info
+            else:
+                assert per >= min(B, q_snm + 1) - 1e-9 or info["snm_scored"] % B == 0 or per > q_snm, info
+        for e in ev:
+            key = (0 if int(e["stream"]) == cams[0].st.handle else 1, int(e["frame_no"]))
+            assert key not in got
+            got[key] = e["result"]
+        if nxt == [T, T] and info["sdd_queued"] == 0 and info["snm_queued"] == 0 and info["events_pending"] == 0:
+            break
+    sched.destroy()
+    assert len(got) == 2 * T
+    for (s, t), r in got.items():
+        assert r["sdd_pass"] == int(synth.is_target(v, s, t)), (s, t)
+    for c in cams:
+        c.st.close()

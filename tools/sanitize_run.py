@@ -40,6 +40,18 @@ def main():
     pinned = [torch.from_numpy(h).pin_memory() for h in host]
     r4 = ctx.filter_batch([(streams[i % 2], pinned[i].data_ptr(), i) for i in range(8)], host=True)
     assert np.array_equal(r1["ssd"], r4["ssd"])
+    # f3 variants: SAD + previous-frame reference (K2 / K2b) and NRMSE, mixed in one batch
+    extra = []
+    for s_id, (dist, mode) in enumerate([("sad", "previous"), ("nrmse", "background")]):
+        st = ctx.open_stream(width=640, height=360, delta_diff=0.01 if dist == "nrmse" else 1000.0,
+                             distance=dist, ref_mode=mode)
+        st.set_reference(torch.from_numpy(synth.frames(v, [s_id] * 2, [0, 1], ref=True)).to(dev))
+        st.snm_load(synth.snm_weights(5, s_id))
+        extra.append(st)
+    r5 = ctx.filter_batch([(extra[i % 2], d[i], i) for i in range(8)] + items)
+    assert np.array_equal(r5["ssd"][8:], r1["ssd"])
+    for st in extra:
+        st.close()
     sched = Scheduler(ctx, max_frames_per_tick=4, snm_slots=8)
     for t in range(6):
         sched.push([(streams[i % 2], d[i], i) for i in range(8)])
