@@ -255,6 +255,43 @@ FFSVA_API ffsva_status ffsva_sched_destroy(ffsva_sched* s);
 typedef enum { FFSVA_BATCH_DYNAMIC = 0, FFSVA_BATCH_FEEDBACK = 1, FFSVA_BATCH_STATIC = 2 } ffsva_batch_policy;
 FFSVA_API ffsva_status ffsva_sched_set_policy(ffsva_sched* s, int32_t policy);
 
+/* ---------------------------------------------------------------------------------------------------------
+ * Admission control and stream re-forwarding between instances (§4.3.1: "when any queue of
+ * T-YOLO or SNM is longer than its predefined threshold ... the corresponding video stream is re-forwarded to
+ * another FFS-VA instance with spare capacity immediately"; L225: "load balancing can also be achieved by the
+ * re-forwarding of video streams between FFS-VAs instances"). One instance = one GPU process; the decision logic
+ * and the transport (NCCL point-to-point over NVLink) live in the Python layer (dist.py); these calls move a
+ * stream's whole state and report the per-stream overload signals.
+ *
+ * Stream image: a self-contained byte image of a stream — its descriptor, thresholds, reference image R, packed
+ * SNM weights and its per-stream statistics row — so the stream continues bit-identically elsewhere.
+ *   ffsva_stream_image_bytes: size of s's image (64,320 B at the default 100x100 grid);
+ *   ffsva_stream_export: write the image to dst (host memory, or device memory on s's device when dst_is_host
+ *     is 0 — e.g. a buffer about to be sent over NCCL); synchronous on cuda_stream;
+ *   ffsva_stream_import: open a new stream on `device` from an image (host memory, or device memory on `device`
+ *     when src_is_host is 0); the stream's statistics row continues from the exported counters. The source
+ *     stream is untouched (close it after the handover). Errors: EINVAL (bad image, version or descriptor). */
+FFSVA_API ffsva_status ffsva_stream_image_bytes(ffsva_stream* s, int64_t* bytes);
+FFSVA_API ffsva_status ffsva_stream_export(ffsva_stream* s, void* dst, int64_t cap, int32_t dst_is_host,
+                                           void* cuda_stream);
+FFSVA_API ffsva_status ffsva_stream_import(int32_t device, const void* src, int64_t bytes, int32_t src_is_host,
+                                           ffsva_stream** out);
+
+/* Per-stream overload signals of the online runtime since the previous reset (L213): a stream is overloaded
+ * when its SNM queue went over q_snm (the SDD stage had to skip it: sdd_blocked > 0) or its prefetcher was
+ * refused (SDD queue over q_sdd: refused > 0). */
+typedef struct {
+  int32_t sdd_depth, snm_depth;   /* current queue depths (frames) */
+  int32_t max_sdd, max_snm;       /* maxima since the reset */
+  uint64_t pushed, refused;       /* frames accepted / refused by the SDD queue since the reset */
+  uint64_t sdd_blocked;           /* SDD cycles that skipped the stream (SNM queue over q_snm) since the reset */
+} ffsva_stream_load;
+FFSVA_API ffsva_status ffsva_sched_stream_load(ffsva_sched* s, ffsva_stream* st, int32_t reset,
+                                               ffsva_stream_load* out);
+/* Detach a stream from the scheduler (before re-forwarding or closing it): FFSVA_EAGAIN while it still has
+ * queued frames or unreported events (keep ticking), FFSVA_OK once removed (or if it was never attached). */
+FFSVA_API ffsva_status ffsva_sched_detach(ffsva_sched* s, ffsva_stream* st);
+
 /* Close a stream (NULL is a no-op). */
 FFSVA_API ffsva_status ffsva_close(ffsva_stream* s);
 

@@ -369,6 +369,122 @@ FFSVA_API ffsva_status ffsva_stats_copy(int32_t device, uint64_t* dst, int32_t m
   return out;
 }
 
+// ---------------------------------------------------------------- stream images (re-forwarding)
+namespace {
+constexpr uint32_t kImageMagic = 0x56534646u;  // "FFSV"
+constexpr uint32_t kImageVersion = 1;
+constexpr int64_t kImageHeader = 256;
+struct ImageHeader {
+  uint32_t magic, version;
+  ffsva_stream_desc desc;
+  uint64_t T, ref_sum_sq;
+  int64_t ref_bytes, snm_bytes, stats_bytes, total;
+  uint8_t has_ref, has_snm, pad[6];
+};
+static_assert(sizeof(ImageHeader) <= kImageHeader, "image header");
+int64_t al16(int64_t x) { return (x + 15) & ~(int64_t)15; }
+int64_t image_bytes(const ffsva_stream_desc& d) {
+  return kImageHeader + al16(3LL * d.sdd_w * d.sdd_h) + al16(snm::BLOB_BYTES) + 8LL * NSTAT;
+}
+}  // namespace
+
+FFSVA_API ffsva_status ffsva_stream_image_bytes(ffsva_stream* s, int64_t* bytes) {
+  if (!s || !bytes) return fail(FFSVA_EINVAL, "NULL argument");
+  *bytes = image_bytes(s->desc);
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_stream_export(ffsva_stream* s, void* dst, int64_t cap, int32_t dst_is_host,
+                                           void* cuda_stream) {
+  if (!s || !dst) return fail(FFSVA_EINVAL, "NULL argument");
+  const int64_t total = image_bytes(s->desc);
+  if (cap < total) return fail(FFSVA_EINVAL, "destination smaller than ffsva_stream_image_bytes");
+  DeviceCtx* ctx = s->ctx;
+  if (ctx->sticky) return fail(FFSVA_ECUDA, "device is in a sticky CUDA error state");
+  std::lock_guard<std::mutex> lk(ctx->mu);
+  DeviceGuard g(ctx->device);
+  if (!dst_is_host) {
+    ffsva_status cs = check_device_ptr(ctx, dst, (size_t)total);
+    if (cs != FFSVA_OK) return cs;
+  }
+  ImageHeader h{};
+  h.magic = kImageMagic;
+  h.version = kImageVersion;
+  h.desc = s->desc;
+  h.T = s->T;
+  h.ref_sum_sq = s->ref_sum_sq;
+  h.ref_bytes = 3LL * s->desc.sdd_w * s->desc.sdd_h;
+  h.snm_bytes = snm::BLOB_BYTES;
+  h.stats_bytes = 8LL * NSTAT;
+  h.total = total;
+  h.has_ref = s->has_ref;
+  h.has_snm = s->has_snm;
+  uint8_t* d = (uint8_t*)dst;
+  const int64_t o_ref = kImageHeader, o_snm = o_ref + al16(h.ref_bytes), o_st = o_snm + al16(h.snm_bytes);
+  cudaStream_t cs = (cudaStream_t)cuda_stream;
+  const cudaMemcpyKind from_dev = dst_is_host ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice;
+  std::vector<uint8_t> hdr(kImageHeader, 0);
+  std::memcpy(hdr.data(), &h, sizeof(h));
+  cudaError_t e = cudaMemcpyAsync(d, hdr.data(), kImageHeader, dst_is_host ? cudaMemcpyHostToHost : cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(d + o_ref, s->d_ref, (size_t)h.ref_bytes, from_dev, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(d + o_snm, s->d_snm, (size_t)h.snm_bytes, from_dev, cs);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(d + o_st, ctx->d_stats + (size_t)s->slot * NSTAT, (size_t)h.stats_bytes, from_dev, cs);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(cs);  // hdr is a local buffer
+  if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_stream_export");
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_stream_import(int32_t device, const void* src, int64_t bytes, int32_t src_is_host,
+                                           ffsva_stream** out) {
+  if (!src || !out || bytes < kImageHeader) return fail(FFSVA_EINVAL, "bad argument");
+  ImageHeader h{};
+  if (src_is_host) {
+    std::memcpy(&h, src, sizeof(h));
+  } else {
+    DeviceGuard g(device);
+    cudaError_t e = cudaMemcpy(&h, src, sizeof(h), cudaMemcpyDeviceToHost);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return fail(FFSVA_EINVAL, std::string("cannot read the image header: ") + cudaGetErrorString(e));
+    }
+  }
+  if (h.magic != kImageMagic || h.version != kImageVersion) return fail(FFSVA_EINVAL, "not a stream image");
+  h.desc.device = device;
+  if (h.total != image_bytes(h.desc) || bytes < h.total || h.ref_bytes != 3LL * h.desc.sdd_w * h.desc.sdd_h ||
+      h.snm_bytes != snm::BLOB_BYTES || h.stats_bytes != 8LL * NSTAT)
+    return fail(FFSVA_EINVAL, "stream image sizes do not match its descriptor");
+  ffsva_stream* s = nullptr;
+  ffsva_status st = ffsva_open_stream(&h.desc, &s);  // validates the descriptor
+  if (st != FFSVA_OK) return st;
+  DeviceCtx* ctx = s->ctx;
+  bool ok = true;
+  {
+    std::lock_guard<std::mutex> lk(ctx->mu);
+    DeviceGuard g(device);
+    const uint8_t* p = (const uint8_t*)src;
+    const int64_t o_ref = kImageHeader, o_snm = o_ref + al16(h.ref_bytes), o_st = o_snm + al16(h.snm_bytes);
+    const cudaMemcpyKind to_dev = src_is_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+    cudaError_t e = cudaMemcpy(s->d_ref, p + o_ref, (size_t)h.ref_bytes, to_dev);
+    if (e == cudaSuccess) e = cudaMemcpy(s->d_snm, p + o_snm, (size_t)h.snm_bytes, to_dev);
+    if (e == cudaSuccess) e = cudaMemcpy(ctx->d_stats + (size_t)s->slot * NSTAT, p + o_st, (size_t)h.stats_bytes, to_dev);
+    if (e != cudaSuccess) {
+      cuda_fail(ctx, e, "ffsva_stream_import");
+      ok = false;
+    }
+    s->T = h.T;
+    s->ref_sum_sq = h.ref_sum_sq;
+    s->has_ref = h.has_ref != 0;
+    s->has_snm = h.has_snm != 0;
+  }
+  if (!ok) {
+    ffsva_close(s);
+    return FFSVA_ECUDA;
+  }
+  *out = s;
+  return FFSVA_OK;
+}
+
 FFSVA_API ffsva_status ffsva_filter_batch_host(const ffsva_frame* frames, int32_t n, ffsva_result* results,
                                                void* cuda_stream);
 

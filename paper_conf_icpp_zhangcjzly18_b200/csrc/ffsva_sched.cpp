@@ -207,6 +207,40 @@ FFSVA_API ffsva_status ffsva_sched_depth(ffsva_sched* s, ffsva_stream* st, int32
   return FFSVA_OK;
 }
 
+FFSVA_API ffsva_status ffsva_sched_stream_load(ffsva_sched* s, ffsva_stream* st, int32_t reset,
+                                               ffsva_stream_load* out) {
+  if (!s || !st || !out) return fail(FFSVA_EINVAL, "bad argument");
+  std::lock_guard<std::mutex> lk(s->mu);
+  std::memset(out, 0, sizeof(*out));
+  const int32_t id = s->lookup(st);
+  if (id < 0) return FFSVA_OK;  // not attached: idle
+  const sched::StreamQ& q = s->pol.stream(id);
+  out->sdd_depth = (int32_t)q.sdd.size();
+  out->snm_depth = (int32_t)q.snm.size();
+  out->max_sdd = q.max_sdd;
+  out->max_snm = q.max_snm;
+  out->pushed = q.pushed;
+  out->refused = q.refused;
+  out->sdd_blocked = q.sdd_blocked;
+  if (reset) s->pol.reset_counters(id);
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_sched_detach(ffsva_sched* s, ffsva_stream* st) {
+  if (!s || !st) return fail(FFSVA_EINVAL, "bad argument");
+  std::lock_guard<std::mutex> lk(s->mu);
+  const int32_t id = s->lookup(st);
+  if (id < 0) return FFSVA_OK;
+  const sched::StreamQ& q = s->pol.stream(id);
+  if (!q.sdd.empty() || !q.snm.empty()) return fail(FFSVA_EAGAIN, "stream still has queued frames");
+  for (const ffsva_event& e : s->pending)
+    if (e.stream == st) return fail(FFSVA_EAGAIN, "stream still has unreported events");
+  s->pol.remove_stream(id);
+  s->by_id[id] = nullptr;
+  s->id_of_slot[st->slot] = -1;
+  return FFSVA_OK;
+}
+
 FFSVA_API ffsva_status ffsva_sched_set_policy(ffsva_sched* s, int32_t policy) {
   if (!s || policy < FFSVA_BATCH_DYNAMIC || policy > FFSVA_BATCH_STATIC) return fail(FFSVA_EINVAL, "bad argument");
   std::lock_guard<std::mutex> lk(s->mu);

@@ -177,6 +177,13 @@ class Policy {
   }
 
   const StreamQ& stream(int32_t id) const { return st_[id]; }
+  // Zero a stream's overload counters (re-forwarding window, L213); depths are state, not counters.
+  void reset_counters(int32_t id) {
+    StreamQ& s = st_[id];
+    s.pushed = s.refused = s.sdd_blocked = 0;
+    s.max_sdd = (int32_t)s.sdd.size();
+    s.max_snm = (int32_t)s.snm.size();
+  }
   int32_t n_streams() const { return (int32_t)st_.size(); }
   int64_t queued_sdd() const {
     int64_t q = 0;

@@ -31,7 +31,8 @@ EXPORTS = ["ffsva_open_stream", "ffsva_set_reference", "ffsva_snm_load", "ffsva_
            "ffsva_get_reference",
            "ffsva_stream_info", "ffsva_stats_copy", "ffsva_close", "ffsva_last_error", "ffsva_kernel_launches",
            "ffsva_version", "ffsva_sched_create", "ffsva_sched_push", "ffsva_sched_tick", "ffsva_sched_depth",
-           "ffsva_sched_destroy", "ffsva_sched_set_policy"]
+           "ffsva_sched_destroy", "ffsva_sched_set_policy", "ffsva_stream_image_bytes", "ffsva_stream_export",
+           "ffsva_stream_import", "ffsva_sched_stream_load", "ffsva_sched_detach"]
 
 
 class StreamDesc(ctypes.Structure):
@@ -78,6 +79,19 @@ class TickInfo(ctypes.Structure):
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
+
+class StreamLoad(ctypes.Structure):
+    """ffsva_stream_load: per-stream overload signals of the online runtime."""
+    _fields_ = [("sdd_depth", ctypes.c_int32), ("snm_depth", ctypes.c_int32), ("max_sdd", ctypes.c_int32),
+                ("max_snm", ctypes.c_int32), ("pushed", ctypes.c_uint64), ("refused", ctypes.c_uint64),
+                ("sdd_blocked", ctypes.c_uint64)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+IMAGE_DESC_OFFSET = 8  # ffsva_stream_desc inside a stream image header (after magic, version)
+
 _lib = None
 
 
@@ -113,6 +127,11 @@ def lib():
             "ffsva_sched_depth": [vp, vp, ctypes.POINTER(i32), ctypes.POINTER(i32)],
             "ffsva_sched_destroy": [vp],
             "ffsva_sched_set_policy": [vp, i32],
+            "ffsva_stream_image_bytes": [vp, ctypes.POINTER(i64)],
+            "ffsva_stream_export": [vp, vp, i64, i32, vp],
+            "ffsva_stream_import": [i32, vp, i64, i32, ctypes.POINTER(vp)],
+            "ffsva_sched_stream_load": [vp, vp, i32, ctypes.POINTER(StreamLoad)],
+            "ffsva_sched_detach": [vp, vp],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -305,6 +324,25 @@ class Stream:
     def reference(self) -> np.ndarray:
         return ffsva_get_reference(self.handle, self.desc.sdd_w, self.desc.sdd_h)
 
+    def image_bytes(self) -> int:
+        n = ctypes.c_int64()
+        _check(lib().ffsva_stream_image_bytes(self.handle, ctypes.byref(n)), "ffsva_stream_image_bytes")
+        return n.value
+
+    def export(self, out=None, stream=None):
+        """The stream's image (f2 re-forwarding): a numpy uint8 array (host), or written into
+        `out`, a uint8 torch tensor (device tensors must live on the stream's device). Returns the buffer."""
+        n = self.image_bytes()
+        if out is None:
+            out = np.zeros(n, np.uint8)
+        if isinstance(out, np.ndarray):
+            assert out.dtype == np.uint8 and out.flags["C_CONTIGUOUS"]
+            ptr, cap, host = out.ctypes.data, out.nbytes, 1
+        else:
+            ptr, cap, host = out.data_ptr(), out.numel() * out.element_size(), 0 if out.is_cuda else 1
+        _check(lib().ffsva_stream_export(self.handle, ptr, cap, host, _stream_handle(stream)), "ffsva_stream_export")
+        return out
+
     def close(self) -> None:
         if self.handle:
             ffsva_close(self.handle)
@@ -359,6 +397,26 @@ class Context:
         for s in self.streams:
             s.close()
         self.streams = []
+
+    def import_stream(self, image) -> Stream:
+        """Open a stream on this device from an image made by Stream.export (numpy host array or uint8 torch
+        tensor on this device)."""
+        if isinstance(image, np.ndarray):
+            buf = np.ascontiguousarray(image, dtype=np.uint8)
+            ptr, n, host, hdr = buf.ctypes.data, buf.nbytes, 1, buf[:256].tobytes()
+        else:
+            ptr, n = image.data_ptr(), image.numel()
+            host = 0 if image.is_cuda else 1
+            hdr = image[:256].cpu().numpy().tobytes()
+        h = ctypes.c_void_p()
+        _check(lib().ffsva_stream_import(self.device, ptr, n, host, ctypes.byref(h)), "ffsva_stream_import")
+        desc = StreamDesc.from_buffer_copy(hdr, IMAGE_DESC_OFFSET)
+        desc.device = self.device
+        st = Stream.__new__(Stream)
+        st.ctx, st.desc, st.handle = self, desc, h.value
+        st.slot, st.device = ffsva_stream_info(st.handle)
+        self.streams.append(st)
+        return st
 
 
 def ffsva_sched_create(device: int, max_frames_per_tick: int, snm_slots: int):
@@ -438,6 +496,21 @@ class Scheduler:
 
     def depth(self, st: "Stream"):
         return ffsva_sched_depth(self.handle, st.handle)
+
+    def stream_load(self, st: "Stream", reset: bool = False) -> dict:
+        """Overload signals of one stream since the last reset (ffsva_sched_stream_load)."""
+        out = StreamLoad()
+        _check(lib().ffsva_sched_stream_load(self.handle, st.handle, int(reset), ctypes.byref(out)),
+               "ffsva_sched_stream_load")
+        return out.as_dict()
+
+    def detach(self, st: "Stream") -> bool:
+        """True once the stream is detached; False while it still has queued frames / unreported events."""
+        r = lib().ffsva_sched_detach(self.handle, st.handle)
+        if r == FFSVA_EAGAIN:
+            return False
+        _check(r, "ffsva_sched_detach")
+        return True
 
     def set_policy(self, policy: str) -> None:
         """'dynamic' (default), 'feedback' or 'static' (the §5.4 comparison mechanisms)."""
