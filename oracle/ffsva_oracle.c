@@ -235,3 +235,132 @@ void orc_decide(double logit, double c_low, double c_high, double filter_degree,
   else if (logit > orc_logit(c_high)) *cls = 2;
   else *cls = 1;
 }
+
+/* ===================================================================================== f1: T-YOLO (L169-L175) */
+
+/* Q28: cell i covers [floor(iS/D), max(floor((i+1)S/D), floor(iS/D) + 1)). */
+void orc_resize(const uint8_t* frame, int32_t W, int32_t H, int64_t pitch, int32_t Dw, int32_t Dh, uint8_t* out) {
+  for (int32_t oy = 0; oy < Dh; ++oy) {
+    int64_t y0 = cell_lo(oy, H, Dh), y1 = cell_lo(oy + 1, H, Dh);
+    if (y1 <= y0) y1 = y0 + 1;
+    for (int32_t ox = 0; ox < Dw; ++ox) {
+      int64_t x0 = cell_lo(ox, W, Dw), x1 = cell_lo(ox + 1, W, Dw);
+      if (x1 <= x0) x1 = x0 + 1;
+      int64_t n = (y1 - y0) * (x1 - x0);
+      for (int32_t c = 0; c < 3; ++c) {
+        int64_t sum = 0;
+        for (int64_t y = y0; y < y1; ++y)
+          for (int64_t x = x0; x < x1; ++x) sum += frame[y * pitch + 3 * x + c];
+        out[((int64_t)oy * Dw + ox) * 3 + c] = (uint8_t)((sum + n / 2) / n);
+      }
+    }
+  }
+}
+
+void orc_conv1x1(const double* in, int32_t C, int32_t H, int32_t W, const double* w, const double* b, int32_t K,
+                 double* out) {
+  for (int32_t k = 0; k < K; ++k)
+    for (int64_t p = 0; p < (int64_t)H * W; ++p) {
+      double s = b ? b[k] : 0.0;
+      for (int32_t c = 0; c < C; ++c) s += in[(int64_t)c * H * W + p] * w[(int64_t)k * C + c];
+      out[(int64_t)k * H * W + p] = s;
+    }
+}
+
+void orc_leaky(double* v, int64_t n) {
+  for (int64_t i = 0; i < n; ++i)
+    if (v[i] < 0.0) v[i] *= 0.1;
+}
+
+void orc_maxpool2_s1(const double* in, int32_t C, int32_t H, int32_t W, double* out) {
+  for (int32_t c = 0; c < C; ++c)
+    for (int32_t y = 0; y < H; ++y)
+      for (int32_t x = 0; x < W; ++x) {
+        double m = in[((int64_t)c * H + y) * W + x];
+        for (int32_t dy = 0; dy < 2; ++dy)
+          for (int32_t dx = 0; dx < 2; ++dx) {
+            if (y + dy >= H || x + dx >= W) continue;
+            double v = in[((int64_t)c * H + y + dy) * W + x + dx];
+            if (v > m) m = v;
+          }
+        out[((int64_t)c * H + y) * W + x] = m;
+      }
+}
+
+/* tiny-yolo-voc topology: (Cin, Cout, kernel, pool after: 0 none, 1 = 2x2/2, 2 = 2x2/1) */
+static const int32_t kTyolo[9][4] = {{3, 16, 3, 1},     {16, 32, 3, 1},     {32, 64, 3, 1},
+                                     {64, 128, 3, 1},   {128, 256, 3, 1},   {256, 512, 3, 2},
+                                     {512, 1024, 3, 0}, {1024, 1024, 3, 0}, {1024, 125, 1, 0}};
+
+int64_t orc_tyolo_n_params(void) {
+  int64_t n = 0;
+  for (int l = 0; l < 9; ++l) n += (int64_t)kTyolo[l][1] * kTyolo[l][0] * kTyolo[l][2] * kTyolo[l][2] + kTyolo[l][1];
+  return n;
+}
+
+/* 9 CONV + 6 POOL layers on 416x416 input; L171: 13x13 grid x 5 boxes. */
+int32_t orc_tyolo_forward(const uint8_t* img, int32_t S, const float* params, int32_t bf16_emul, double* out) {
+  if (S <= 0 || S % 32) return -1;
+  int32_t H = S, W = S;
+  double* x = malloc(sizeof(double) * 3 * (size_t)S * S);
+  for (int32_t c = 0; c < 3; ++c) /* Q29: x = v / 256, CHW */
+    for (int64_t p = 0; p < (int64_t)S * S; ++p) x[(int64_t)c * S * S + p] = (double)img[p * 3 + c] / 256.0;
+  const float* pp = params;
+  for (int l = 0; l < 9; ++l) {
+    const int32_t C = kTyolo[l][0], K = kTyolo[l][1], k = kTyolo[l][2], pool = kTyolo[l][3];
+    const int64_t nw = (int64_t)K * C * k * k;
+    double* w = malloc(sizeof(double) * nw);
+    double* b = malloc(sizeof(double) * K);
+    for (int64_t i = 0; i < nw; ++i) w[i] = bf16_emul ? orc_round_bf16(pp[i]) : (double)pp[i];
+    for (int32_t i = 0; i < K; ++i) b[i] = pp[nw + i];
+    pp += nw + K;
+    double* y = malloc(sizeof(double) * K * (size_t)H * W);
+    if (k == 3)
+      orc_conv3x3(x, C, H, W, w, b, K, y);
+    else
+      orc_conv1x1(x, C, H, W, w, b, K, y);
+    if (l < 8) orc_leaky(y, (int64_t)K * H * W);
+    free(x);
+    free(w);
+    free(b);
+    if (pool == 1) {
+      double* z = malloc(sizeof(double) * K * (size_t)(H / 2) * (W / 2));
+      orc_maxpool2(y, K, H, W, z);
+      free(y);
+      y = z;
+      H /= 2;
+      W /= 2;
+    } else if (pool == 2) {
+      double* z = malloc(sizeof(double) * K * (size_t)H * W);
+      orc_maxpool2_s1(y, K, H, W, z);
+      free(y);
+      y = z;
+    }
+    if (bf16_emul && l < 8)
+      for (int64_t i = 0; i < (int64_t)K * H * W; ++i) y[i] = orc_round_bf16(y[i]);
+    x = y;
+  }
+  /* CHW -> HWC */
+  for (int32_t c = 0; c < 125; ++c)
+    for (int64_t p = 0; p < (int64_t)H * W; ++p) out[p * 125 + c] = x[(int64_t)c * H * W + p];
+  free(x);
+  return 0;
+}
+
+/* L171 "If the confidence score exceeds the threshold (e.g., 0.2), one target object is considered to appear";
+ * L195 NumberofObjects. Confidence of box b = sigmoid(objectness) * softmax(class logits)[target] (Q31). */
+int32_t orc_tyolo_count(const double* out, int32_t cells, int32_t target_class, double thresh) {
+  int32_t n = 0;
+  for (int32_t p = 0; p < cells; ++p)
+    for (int32_t b = 0; b < 5; ++b) {
+      const double* v = out + (int64_t)p * 125 + 25 * b;
+      double mx = v[5];
+      for (int32_t k = 1; k < 20; ++k)
+        if (v[5 + k] > mx) mx = v[5 + k];
+      double z = 0.0;
+      for (int32_t k = 0; k < 20; ++k) z += exp(v[5 + k] - mx);
+      const double score = 1.0 / (1.0 + exp(-v[4])) * exp(v[5 + target_class] - mx) / z;
+      if (score > thresh) ++n;
+    }
+  return n;
+}

@@ -73,4 +73,41 @@ double orc_logit(double t);
  * pass iff c >= t_pre; cls = 0 if c < c_low, 2 if c > c_high, else 1. All compared in logit space. */
 void orc_decide(double logit, double c_low, double c_high, double filter_degree, uint8_t* pass, uint8_t* cls);
 
+/* ---------------------------------------------------------------------------------------------------------
+ * f1: Tiny-YOLO-VOC (T-YOLO) stage + NumberofObjects (§3.2.3, §4.2.2; DESIGN.md
+ * readings Q28-Q32).
+ * "T-YOLO consists of 9 CONV layers and 6 POOL layers" on "416*416 pixel images" (L169), trained on VOC's 20
+ * classes; "divides the input image into a 13*13 grid ... Each grid cell predicts 5 bounding boxes and confidence
+ * scores ... If the confidence score exceeds the threshold (e.g., 0.2), one target object is considered to
+ * appear" (L171). The layers are those of tiny-yolo-voc (L169's [44]):
+ *   conv3x3 3->16, pool2/2, 16->32, pool2/2, 32->64, pool2/2, 64->128, pool2/2, 128->256, pool2/2, 256->512,
+ *   pool2/1, 512->1024, 1024->1024 (each conv + bias, leaky ReLU 0.1; batch norm folded into the bias),
+ *   conv1x1 1024->125 linear = 5 boxes x (tx, ty, tw, th, objectness, 20 class logits) per cell.
+ * Params packed per layer: w[Cout][Cin][k][k] then b[Cout] (9 layers, 15,858,717 floats). */
+
+/* Resize for filters whose feature size may exceed the frame (T-YOLO's 416 vs 360-row frames; Q28): cell i of a
+ * dimension S split in D covers [floor(iS/D), max(floor((i+1)S/D), floor(iS/D) + 1)) -- the C1 box when S >= D,
+ * one source pixel per cell otherwise; value = (s + n/2) / n. */
+void orc_resize(const uint8_t* frame, int32_t W, int32_t H, int64_t pitch, int32_t Dw, int32_t Dh, uint8_t* out);
+
+/* 1x1 convolution (C -> K), CHW fp64; b may be NULL. */
+void orc_conv1x1(const double* in, int32_t C, int32_t H, int32_t W, const double* w, const double* b, int32_t K,
+                 double* out);
+/* leaky ReLU, slope 0.1 for x < 0 (darknet's "leaky") */
+void orc_leaky(double* v, int64_t n);
+/* 2x2 max-pool, stride 1, output H x W: out[y][x] = max over the in-bounds of (y..y+1, x..x+1) (darknet pads the
+ * right/bottom border with -inf, Q30). */
+void orc_maxpool2_s1(const double* in, int32_t C, int32_t H, int32_t W, double* out);
+
+/* T-YOLO forward on a S x S x 3 u8 image (S = 416; any multiple of 32 for tests): x = v / 256 (Q29), the nine
+ * layers above; bf16_emul = 1 rounds every weight and every layer's output activation to bf16 (the kernel's
+ * operand precision). out = (S/32) x (S/32) x 125 doubles, HWC. Returns 0, or -1 if S is not a multiple of 32. */
+int32_t orc_tyolo_forward(const uint8_t* img, int32_t S, const float* params, int32_t bf16_emul, double* out);
+int64_t orc_tyolo_n_params(void);
+
+/* L171 + L195 (NumberofObjects): score of box b of a cell = sigmoid(objectness) * softmax(class logits)[target];
+ * a target object appears in the box iff score > thresh (strict, "exceeds"); returns the count over all cells and
+ * boxes (Q31: no non-maximum suppression). A frame passes T-YOLO iff count >= NumberofObjects. */
+int32_t orc_tyolo_count(const double* out, int32_t cells, int32_t target_class, double thresh);
+
 #endif

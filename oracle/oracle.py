@@ -57,6 +57,17 @@ def lib():
         L.orc_logit.argtypes = [ctypes.c_double]
         L.orc_logit.restype = ctypes.c_double
         L.orc_decide.argtypes = [ctypes.c_double, ctypes.c_double, ctypes.c_double, ctypes.c_double, u8p, u8p]
+        L.orc_resize.argtypes = [u8p, ctypes.c_int32, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32, ctypes.c_int32,
+                                 u8p]
+        L.orc_conv1x1.argtypes = [u8p, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, u8p, u8p, ctypes.c_int32, u8p]
+        L.orc_leaky.argtypes = [u8p, ctypes.c_int64]
+        L.orc_maxpool2_s1.argtypes = [u8p, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, u8p]
+        L.orc_tyolo_forward.argtypes = [u8p, ctypes.c_int32, u8p, ctypes.c_int32, u8p]
+        L.orc_tyolo_forward.restype = ctypes.c_int32
+        L.orc_tyolo_n_params.argtypes = []
+        L.orc_tyolo_n_params.restype = ctypes.c_int64
+        L.orc_tyolo_count.argtypes = [u8p, ctypes.c_int32, ctypes.c_int32, ctypes.c_double]
+        L.orc_tyolo_count.restype = ctypes.c_int32
         _lib = L
     return _lib
 
@@ -252,3 +263,70 @@ def filter_frames(frames, width: int, refs, deltas, snm_params, c_low, c_high, f
             npass[i], ncls[i] = decide(lg[i], c_low[i], c_high[i], filter_degree[i])
     return dict(d100=d100, d50=d50, ssd=ssd_v, sdd_pass=sp, survivors=surv, survivor_idx=sidx, logit=lg,
                 snm_pass=npass, snm_class=ncls, last_ref=last_ref)
+
+
+# ------------------------------------------------------------------ f1: T-YOLO + NumberofObjects (L169-L175, L195)
+
+def resize(frame: np.ndarray, width: int, dw: int, dh: int) -> np.ndarray:
+    """Q28 resize (C1 box when the frame is larger, one source pixel per cell when smaller). -> (dh, dw, 3) u8."""
+    f = _c(frame, np.uint8)
+    H, pitch = f.shape
+    out = np.zeros((dh, dw, 3), dtype=np.uint8)
+    lib().orc_resize(f.ctypes.data, width, H, pitch, dw, dh, out.ctypes.data)
+    return out
+
+
+def conv1x1(inp: np.ndarray, w: np.ndarray, b: np.ndarray | None = None) -> np.ndarray:
+    x = _c(inp, np.float64)
+    wt = _c(w, np.float64)
+    C, H, W = x.shape
+    K = wt.shape[0]
+    out = np.zeros((K, H, W), dtype=np.float64)
+    bb = _c(b, np.float64) if b is not None else None
+    lib().orc_conv1x1(x.ctypes.data, C, H, W, wt.ctypes.data, bb.ctypes.data if bb is not None else None, K,
+                      out.ctypes.data)
+    return out
+
+
+def leaky(v: np.ndarray) -> np.ndarray:
+    x = np.array(v, dtype=np.float64, copy=True, order="C")
+    lib().orc_leaky(x.ctypes.data, x.size)
+    return x
+
+
+def maxpool2_s1(inp: np.ndarray) -> np.ndarray:
+    x = _c(inp, np.float64)
+    C, H, W = x.shape
+    out = np.zeros_like(x)
+    lib().orc_maxpool2_s1(x.ctypes.data, C, H, W, out.ctypes.data)
+    return out
+
+
+def tyolo_n_params() -> int:
+    return int(lib().orc_tyolo_n_params())
+
+
+def tyolo_forward(img: np.ndarray, params: np.ndarray, bf16_emul: bool = False) -> np.ndarray:
+    """T-YOLO on an (S, S, 3) u8 image (S = 416, or any multiple of 32). Returns (S/32, S/32, 125) float64."""
+    im = _c(img, np.uint8)
+    S = im.shape[0]
+    assert im.shape == (S, S, 3)
+    p = _c(params, np.float32)
+    assert p.size == tyolo_n_params()
+    out = np.zeros((S // 32, S // 32, 125), np.float64)
+    assert lib().orc_tyolo_forward(im.ctypes.data, S, p.ctypes.data, int(bf16_emul), out.ctypes.data) == 0
+    return out
+
+
+def tyolo_count(out: np.ndarray, target_class: int, thresh: float = 0.2) -> int:
+    """L171 + Q31: boxes whose sigmoid(objectness) * softmax(classes)[target] exceeds thresh."""
+    o = _c(out, np.float64)
+    return int(lib().orc_tyolo_count(o.ctypes.data, o.size // 125, target_class, thresh))
+
+
+def tyolo_scores(out: np.ndarray, target_class: int) -> np.ndarray:
+    """Per-box scores (cells x 5) by the same definition, for near-threshold exemptions in parity tests."""
+    o = np.asarray(out, np.float64).reshape(-1, 5, 25)
+    cls = o[:, :, 5:]
+    e = np.exp(cls - cls.max(axis=2, keepdims=True))
+    return 1.0 / (1.0 + np.exp(-o[:, :, 4])) * e[:, :, target_class] / e.sum(axis=2)

@@ -163,3 +163,30 @@ def snm_weights(seed: int, stream: int, c1: int = 16, c2: int = 32, h: int = 50,
     bfc = rng.normal(0.0, bias_std, size=(1,)) if bias_std else np.zeros(1)
     packed = np.concatenate([w1.ravel(), b1, w2.ravel(), b2, wfc, bfc]).astype(np.float32)
     return to_bf16_values(packed)
+
+
+# tiny-yolo-voc layer table (Cin, Cout, kernel): the shape of the random-init weights the T-YOLO stage takes
+TYOLO_LAYERS = [(3, 16, 3), (16, 32, 3), (32, 64, 3), (64, 128, 3), (128, 256, 3), (256, 512, 3), (512, 1024, 3),
+                (1024, 1024, 3), (1024, 125, 1)]
+
+
+def tyolo_weights(seed: int, target_class: int = 6, class_bias: float = 3.0, bias_std: float = 0.05,
+                  out_gain: float = 1.0) -> np.ndarray:
+    """Seeded random T-YOLO params (no trained VOC weights exist here): per layer w[Cout][Cin][k][k] (He normal,
+    N(0, 2/fan_in); the last layer N(0, out_gain^2/fan_in)) then b[Cout] (N(0, bias_std^2); the last layer 0 except
+    +class_bias on target_class's logit of every box, so scores straddle the 0.2 threshold). float32, bf16-exact."""
+    rng = np.random.default_rng([seed, 0x59_4F_4C_4F])
+    parts = []
+    for i, (cin, cout, k) in enumerate(TYOLO_LAYERS):
+        fan = cin * k * k
+        last = i == len(TYOLO_LAYERS) - 1
+        std = out_gain / np.sqrt(fan) if last else np.sqrt(2.0 / fan)
+        w = rng.standard_normal(size=cout * fan, dtype=np.float32) * np.float32(std)
+        if last:
+            b = np.zeros(cout, np.float32)
+            for box in range(5):
+                b[25 * box + 5 + target_class] = class_bias
+        else:
+            b = (rng.standard_normal(size=cout, dtype=np.float32) * np.float32(bias_std)).astype(np.float32)
+        parts += [w, b]
+    return to_bf16_values(np.concatenate(parts).astype(np.float32))

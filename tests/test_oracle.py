@@ -444,3 +444,136 @@ def test_previous_frame_reference_mode():
         # streams 0 and 1 interleaved, each static: only the first frame of each stream may differ from 0
         r = run([a, b, a, b, a, b], [0, 1, 0, 1, 0, 1], metric)
         assert (r["ssd"][2:] == 0).all()
+
+
+# ------------------------------------------------------------------ f1: T-YOLO + NumberofObjects (P14-P17)
+
+def test_p14_tyolo_count_hand_example():
+    g = _gold("p14_tyolo_count.json")
+    ln = {"0": 0.0, "ln3": math.log(3), "-ln3": -math.log(3), "ln19": math.log(19),
+          "ln(19*0.4/0.6)": math.log(19 * 0.4 / 0.6)}
+    out = np.zeros((1, 1, 125))
+    for b in range(5):
+        out[0, 0, 25 * b + 4] = ln[g["objectness"][b]]
+        out[0, 0, 25 * b + 5 + 6] = ln[g["target_logit"][b]]
+    s = orc.tyolo_scores(out, 6)[0]
+    assert np.allclose(s, g["expected_scores"], rtol=0, atol=1e-12)
+    # box 3 sits at 0.2 up to rounding of the logs: the hand count avoids relying on which side it lands
+    assert orc.tyolo_count(out, 6, 0.2 + 1e-9) == g["expected_count_at_0.2"]
+    assert orc.tyolo_count(out, 6, 0.1) == g["expected_count_at_0.1"]
+    assert orc.tyolo_count(out, 7, 0.2) == 0  # another class: 1/38 at best
+
+
+def test_p15_resize_upsampling_and_pool_s1_hand():
+    g = _gold("p15_resize_pool.json")
+    f, W = _frame_from_channel0(g["resize"]["channel0"])
+    d = orc.resize(f, W, *g["resize"]["grid"])
+    assert d[:, :, 0].tolist() == g["resize"]["expected_channel0"]
+    x = np.asarray(g["pool_s1"]["input"], np.float64)[None]
+    assert orc.maxpool2_s1(x)[0].tolist() == g["pool_s1"]["expected"]
+
+
+@pytest.mark.parametrize("W,H,D", [(640, 360, 100), (1280, 720, 416), (1920, 1080, 416), (416, 416, 416)])
+def test_resize_reduces_to_box_downsample_when_downscaling(W, H, D):
+    f = np.random.default_rng(W).integers(0, 256, size=(H, 3 * W), dtype=np.uint8)
+    if W >= D and H >= D:
+        assert np.array_equal(orc.resize(f, W, D, D), orc.box_downsample(f, W, D, D))
+
+
+def test_resize_mixed_up_and_down():
+    """640x360 -> 416x416: x downsamples (boxes of 1-2 px), y upsamples (one source row per cell, row
+    floor(j*360/416)); checked against a brute-force restatement on both axes."""
+    W, H, D = 640, 360, 416
+    f = np.random.default_rng(1).integers(0, 256, size=(H, 3 * W), dtype=np.uint8)
+    got = orc.resize(f, W, D, D)
+    img = f.reshape(H, W, 3).astype(np.int64)
+    for j in [0, 1, 2, 207, 415]:
+        y = j * H // D
+        for i in [0, 1, 100, 415]:
+            x0, x1 = i * W // D, (i + 1) * W // D
+            s = img[y, x0:x1].sum(axis=0)
+            n = x1 - x0
+            assert (got[j, i] == (2 * s + n) // (2 * n)).all()
+
+
+def test_leaky_closed_form():
+    v = np.array([-2.0, -0.5, 0.0, 0.25, 3.0])
+    assert orc.leaky(v).tolist() == [-0.2, -0.05, 0.0, 0.25, 3.0]
+
+
+def _torch_tyolo(img, params, bf16=False):
+    """T-YOLO restated with torch fp64 library ops (conv2d, leaky_relu, max_pool2d) — independent of the oracle."""
+    import torch
+    import torch.nn.functional as F
+    from synth.synth import TYOLO_LAYERS
+    x = torch.from_numpy(img.astype(np.float64) / 256.0).permute(2, 0, 1)[None]
+    p = torch.from_numpy(params.astype(np.float64))
+    o = 0
+    pools = [1, 1, 1, 1, 1, 2, 0, 0, 0]
+    for i, (cin, cout, k) in enumerate(TYOLO_LAYERS):
+        w = p[o:o + cout * cin * k * k].reshape(cout, cin, k, k)
+        o += w.numel()
+        b = p[o:o + cout]
+        o += cout
+        if bf16:
+            w = w.to(torch.bfloat16).to(torch.float64)
+        x = F.conv2d(x, w, b, padding=k // 2)
+        if i < 8:
+            x = F.leaky_relu(x, 0.1)
+        if pools[i] == 1:
+            x = F.max_pool2d(x, 2, 2)
+        elif pools[i] == 2:
+            x = F.max_pool2d(F.pad(x, (0, 1, 0, 1), value=-float("inf")), 2, 1)
+        if bf16 and i < 8:
+            x = x.to(torch.bfloat16).to(torch.float64)
+    return x[0].permute(1, 2, 0).numpy()
+
+
+@pytest.mark.parametrize("S", [32, 64])
+def test_p16_tyolo_forward_vs_torch_fp64(S):
+    from synth import synth as sy
+    rng = np.random.default_rng(S)
+    img = rng.integers(0, 256, size=(S, S, 3), dtype=np.uint8)
+    params = sy.tyolo_weights(S)
+    got = orc.tyolo_forward(img, params)
+    want = _torch_tyolo(img, params)
+    assert got.shape == (S // 32, S // 32, 125)
+    assert np.allclose(got, want, rtol=1e-9, atol=1e-9)
+    got_b = orc.tyolo_forward(img, params, bf16_emul=True)
+    want_b = _torch_tyolo(img, params, bf16=True)
+    assert np.allclose(got_b, want_b, rtol=0, atol=5e-2)  # bf16 rounding flips from summation order only
+    assert np.median(np.abs(got_b - want_b)) < 1e-3
+
+
+def test_p17_tyolo_zero_weight_closed_form():
+    """All conv weights 0, biases b_l: every layer outputs leaky(b_l) per channel (pooling keeps constants), so
+    the output is b9 + W9 . leaky(b8) at every cell."""
+    from synth import synth as sy
+    params = np.zeros(orc.tyolo_n_params(), np.float32)
+    rng = np.random.default_rng(17)
+    o = 0
+    b8 = w9 = b9 = None
+    for i, (cin, cout, k) in enumerate(sy.TYOLO_LAYERS):
+        nw = cout * cin * k * k
+        if i == 8:
+            w9 = rng.normal(0, 0.05, size=(cout, cin)).astype(np.float32)
+            params[o:o + nw] = w9.ravel()
+        o += nw
+        b = rng.normal(0, 1, size=cout).astype(np.float32)
+        params[o:o + cout] = b
+        o += cout
+        if i == 7:
+            b8 = b
+        if i == 8:
+            b9 = b
+    img = rng.integers(0, 256, size=(64, 64, 3), dtype=np.uint8)
+    got = orc.tyolo_forward(img, params)
+    lb8 = np.where(b8 < 0, 0.1 * b8.astype(np.float64), b8.astype(np.float64))
+    want = b9.astype(np.float64) + w9.astype(np.float64) @ lb8
+    assert np.allclose(got, np.broadcast_to(want, got.shape), rtol=1e-12, atol=1e-12)
+
+
+def test_tyolo_n_params_tiny_yolo_voc():
+    """tiny-yolo-voc: 15,858,717 parameters (conv weights + folded BN biases), hand sum over the nine layers."""
+    assert orc.tyolo_n_params() == 448 + 4640 + 18496 + 73856 + 295168 + 1180160 + 4719616 + 9438208 + 128125
+    assert orc.tyolo_n_params() == 15_858_717
