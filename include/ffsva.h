@@ -292,6 +292,33 @@ FFSVA_API ffsva_status ffsva_sched_stream_load(ffsva_sched* s, ffsva_stream* st,
  * queued frames or unreported events (keep ticking), FFSVA_OK once removed (or if it was never attached). */
 FFSVA_API ffsva_status ffsva_sched_detach(ffsva_sched* s, ffsva_stream* st);
 
+/* ---------------------------------------------------------------------------------------------------------
+ * T-YOLO stage (§3.2.3, §4.2.2). The third filter: Tiny-YOLO-VOC
+ * ("9 CONV layers and 6 POOL layers", 416x416 input, VOC's 20 classes; L169), one model shared by all streams of a
+ * device (L175). Each frame is resized to 416x416 (Q28), scaled by 1/256 (Q29) and run through the nine
+ * layers on tcgen05 tensor cores (bf16 operands, fp32 accumulation, bf16 activations between layers: Q32). The
+ * 13x13x125 head is decoded per box as score = sigmoid(objectness) * softmax(class logits)[target_class]; a box
+ * whose score exceeds `thresh` (0.2 in the paper, L171) is one target object (Q31, no NMS), and a frame passes
+ * iff its count >= number_of_objects (NumberofObjects, L195).
+ *   ffsva_tyolo_load: params = the nine layers' w[Cout][Cin][k][k] then b[Cout] (fp32, batch norm folded into b;
+ *     15,858,717 values); weights are rounded to bf16 at load. The model holds a reference on the device context.
+ *   ffsva_tyolo_run: n frames (device pixels; each frame's stream supplies its geometry); outputs (host, may be
+ *     NULL, not all): counts[n], pass[n], raw[n][13][13][125] fp32 head outputs. Synchronous on cuda_stream.
+ *   ffsva_tyolo_layer_output (diagnostic): run the resize and layers 0..layer on n <= 256 frames and copy that
+ *     layer's bf16 NHWC activation (layer -1: the resized input, 416x416x4) to host `out` (bf16 bit patterns).
+ *   ffsva_tyolo_profile (measurement): mean device ms of the resize and of each of the nine layers over iters runs
+ *     of n <= 256 frames, CUDA events on cuda_stream; ms_out[10]. */
+typedef struct ffsva_tyolo ffsva_tyolo;
+FFSVA_API ffsva_status ffsva_tyolo_load(int32_t device, const float* params, int64_t n_params, ffsva_tyolo** out);
+FFSVA_API ffsva_status ffsva_tyolo_run(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, int32_t target_class,
+                                       float thresh, int32_t number_of_objects, int32_t* counts, uint8_t* pass,
+                                       float* raw, void* cuda_stream);
+FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, int32_t layer,
+                                                uint16_t* out, void* cuda_stream);
+FFSVA_API ffsva_status ffsva_tyolo_profile(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, int32_t iters,
+                                           float* ms_out, void* cuda_stream);
+FFSVA_API ffsva_status ffsva_tyolo_destroy(ffsva_tyolo* m);
+
 /* Close a stream (NULL is a no-op). */
 FFSVA_API ffsva_status ffsva_close(ffsva_stream* s);
 

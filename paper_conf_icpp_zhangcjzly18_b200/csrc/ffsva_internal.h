@@ -2,6 +2,7 @@
 // Not part of the public ABI (include/ffsva.h is). Nothing here is shared with oracle/.
 #pragma once
 
+#include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -139,6 +140,33 @@ struct PrevArgs {
   unsigned long long* stats;
 };
 cudaError_t launch_prev(const PrevArgs& a, cudaStream_t st);  // K2 then K2b (2 launches if n_pm > 0)
+
+// ------------------------------------------------------------------ T-YOLO (f1, ffsva_tyolo.cu)
+struct TyFrame {           // raw frame geometry for the 416x416 resize
+  const uint8_t* pixels;
+  int64_t pitch;
+  int32_t W, H;
+};
+struct TyConvArgs {
+  const __nv_bfloat16* in;   // NHWC [N][H][W][Cp] bf16 (conv input; 'same' convolution keeps H x W)
+  __nv_bfloat16* out;        // NHWC [N][Ho][Wo][Cout] bf16 (hidden layers)
+  float* out_f32;            // [M][Cout] fp32 (head)
+  const uint8_t* wpk;        // weights packed per (N tile, K step) in the UMMA B layout
+  const float* bias;         // [Cout] fp32 (zero-padded)
+  int32_t N, H, W, Cp;       // batch, conv spatial size, padded input channels (4, 16, 32 or a multiple of 64)
+  int32_t Ho, Wo;            // output spatial size (after pooling)
+  int32_t Cout, NT, Cout_tiles;  // output channels (row stride of out), N tile, number of N tiles
+  int32_t nq, pool, ksize;   // accumulator chains (4 for pool layers), pool 0/1 (2x2/2)/2 (2x2/1), kernel 3 or 1
+  int32_t kchunks, ksteps;   // K steps of 64 channels, MMA K16 steps per K step
+  int32_t stages, tmem_cols, leaky, M;
+  int32_t head, target;      // head: count boxes of class `target` scoring > thresh into counts[frame]
+  float thresh;
+  int32_t* counts;
+};
+cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st);
+cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, __nv_bfloat16* out, cudaStream_t st);
+int tyolo_conv_smem_bytes(int stages, int nq, int NT);
+cudaError_t tyolo_configure();
 
 cudaError_t launch_fill_nan(float* p, int32_t n, cudaStream_t st);
 cudaError_t launch_reference(const uint8_t* frames, int32_t k, int64_t frame_stride, int32_t W, int32_t H,

@@ -1,0 +1,313 @@
+// ffsva_tyolo.cu — K5: the T-YOLO stage on tcgen05 tensor cores.
+//
+// Method (§3.2.3, §4.2.2): the third filter is Tiny-YOLO-VOC — "9 CONV layers and 6 POOL
+// layers" on 416x416 images — shared by all streams; it "divides the input image into a 13*13 grid", "each grid
+// cell predicts 5 bounding boxes and confidence scores", a box whose confidence exceeds the threshold (0.2) is one
+// target object, and frames with fewer than NumberofObjects targets are filtered out. Readings (DESIGN.md
+// Q28-Q32): Q28 resize, x = v/256 (Q29), -inf border of the stride-1 pool (Q30), score = sigmoid(objectness) *
+// softmax(classes)[target] without NMS (Q31), bf16 operands / fp32 accumulation / bf16 activations between
+// layers (Q32).
+//
+// B200 mapping — one implicit-GEMM kernel for every layer, activations NHWC bf16 in HBM/L2:
+//   * GEMM rows = OUTPUT pixels of the layer (pooled pixels for the pool layers) of the whole batch, 128 per CTA;
+//     N = output channels (tile NT <= 256); K = taps x input channels, staged 64 bf16 (128 B) per pipeline step.
+//   * Pooling is folded into the MMA like the SNM: for a pool layer the four 2x2 positions are four accumulator
+//     chains in four TMEM column groups, so the epilogue max-pools in registers (bias and leaky ReLU commute
+//     with max and are applied once after it). The 2x2/1 pool of layer 6 uses the same four chains with the
+//     border positions excluded (Q30).
+//   * A operands are gathered (im2col on the fly) by 128 producer threads with cp.async zero-fill (padding and
+//     K padding are zeros), written straight into the UMMA K-major no-swizzle core-matrix layout; B operands
+//     (weights, pre-packed on the host in exactly that layout per (N tile, K step)) arrive by one bulk copy per
+//     step. A 2- or 4-stage mbarrier ring overlaps copies with the MMAs, issued by one thread.
+//   * The 1x1 head (1024 -> 125) writes its fp32 outputs and counts, per row, the boxes whose score exceeds the
+//     threshold into the frame's counter (L171).
+#include "ffsva_internal.h"
+#include "ffsva_ptx.h"
+
+namespace ffsva {
+namespace {
+
+using namespace ptx;
+
+constexpr int kConvThreads = 192;  // warps 0-3: A gather + epilogue, warp 4: TMEM + MMA issue, warp 5: B copies
+constexpr int kATile = 128 * 128;  // one stage of A for one chain: 128 rows x 64 bf16
+
+// byte offset of (K group g of 8 bf16, row r) in a 128-row K-major no-swizzle tile: core matrices of 8 rows x 16 B,
+// K-adjacent core matrices 2048 B apart (LBO), 8-row groups 128 B apart (SBO)
+__device__ __forceinline__ uint32_t a_off(int g, int r) {
+  return (uint32_t)(g * 2048 + (r >> 3) * 128 + (r & 7) * 16);
+}
+
+// The A rows of one K step (chunk j) for output row r whose conv pixel is (cy, cx).
+__device__ __forceinline__ void gather(const TyConvArgs& a, const __nv_bfloat16* img, bool rv, int cy, int cx, int j,
+                                       uint32_t dst, int r) {
+  const int H = a.H, W = a.W, Cp = a.Cp;
+  if (Cp >= 64) {
+    int t, c0;
+    if (a.ksize == 3) {
+      const int cpt = Cp >> 6;
+      t = j / cpt;
+      c0 = (j - t * cpt) << 6;
+    } else {
+      t = 4;
+      c0 = j << 6;
+    }
+    const int sy = cy + t / 3 - 1, sx = cx + t % 3 - 1;
+    const bool v = rv && sy >= 0 && sy < H && sx >= 0 && sx < W;
+    const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * Cp + c0 : a.in;
+#pragma unroll
+    for (int g = 0; g < 8; ++g) cp_async16(dst + a_off(g, r), src + 8 * g, v);
+  } else if (Cp >= 16) {  // 16 or 32 channels: 4 or 2 taps per K step
+    const int tpc = 64 / Cp, upt = Cp >> 3;
+    for (int i = 0; i < tpc; ++i) {
+      const int t = j * tpc + i;
+      const int sy = cy + t / 3 - 1, sx = cx + t % 3 - 1;
+      const bool v = rv && t < 9 && sy >= 0 && sy < H && sx >= 0 && sx < W;
+      const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * Cp : a.in;
+      for (int u = 0; u < upt; ++u) cp_async16(dst + a_off(i * upt + u, r), src + 8 * u, v);
+    }
+  } else {  // 4 channels (RGB + zero): two taps per 16-byte K group, all nine taps in one step
+#pragma unroll
+    for (int g = 0; g < 8; ++g)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int t = 2 * g + h;
+        const int sy = cy + t / 3 - 1, sx = cx + t % 3 - 1;
+        const bool v = rv && t < 9 && sy >= 0 && sy < H && sx >= 0 && sx < W;
+        const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * 4 : a.in;
+        cp_async8(dst + a_off(g, r) + 8 * h, src, v);
+      }
+  }
+}
+
+__device__ __forceinline__ void conv_pixel(const TyConvArgs& a, int oy, int ox, int q, int& cy, int& cx) {
+  if (a.pool == 1) {
+    cy = 2 * oy + (q >> 1);
+    cx = 2 * ox + (q & 1);
+  } else if (a.pool == 2) {
+    cy = oy + (q >> 1);
+    cx = ox + (q & 1);
+  } else {
+    cy = oy;
+    cx = ox;
+  }
+}
+
+__global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs a) {
+  extern __shared__ __align__(1024) uint8_t sm[];
+  const int S = a.stages, nq = a.nq, NT = a.NT, KC = a.kchunks;
+  const uint32_t stage_a = (uint32_t)nq * kATile;
+  const uint32_t b_bytes = (uint32_t)NT * 128;
+  uint8_t* As = sm;
+  uint8_t* Bs = sm + (size_t)S * stage_a;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(Bs + (size_t)S * b_bytes);
+  uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 2 * S + 1);
+  const uint32_t full0 = smem_addr(bars), empty0 = full0 + 8 * S, done = full0 + 16 * S;
+  const uint32_t As0 = smem_addr(As), Bs0 = smem_addr(Bs);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int m0 = blockIdx.x * 128, nt = blockIdx.y;
+
+  if (tid == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(full0 + 8 * s, 129);  // 128 gather threads + the weight copy's expect_tx arrival
+      mbar_init(empty0 + 8 * s, 1);
+    }
+    mbar_init(done, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 4) tmem_alloc(smem_addr(s_tmem), (uint32_t)a.tmem_cols);
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *s_tmem;
+
+  const int r = tid;  // warps 0-3: tile row = TMEM lane
+  const int m = m0 + (r & 127);
+  const bool rv = warp < 4 && m < a.M;
+  int n = 0, oy = 0, ox = 0;
+  if (rv) {
+    const int hw = a.Ho * a.Wo;
+    n = m / hw;
+    const int rem = m - n * hw;
+    oy = rem / a.Wo;
+    ox = rem - oy * a.Wo;
+  }
+
+  if (warp < 4) {
+    // ---------------- A producers
+    const __nv_bfloat16* img = a.in + (int64_t)n * a.H * a.W * a.Cp;
+    for (int j = 0; j < KC; ++j) {
+      const int s = j % S;
+      mbar_wait(empty0 + 8 * s, ((j / S) & 1) ^ 1);
+      for (int q = 0; q < nq; ++q) {
+        int cy, cx;
+        conv_pixel(a, oy, ox, q, cy, cx);
+        gather(a, img, rv, cy, cx, j, As0 + (uint32_t)(s * nq + q) * kATile, r);
+      }
+      cp_async_commit();
+      if (j > 0) {  // the previous step's copies have landed: publish them to the tensor core (async proxy)
+        cp_async_wait<1>();
+        fence_proxy_async();
+        mbar_arrive(full0 + 8 * ((j - 1) % S));
+      }
+    }
+    cp_async_wait<0>();
+    fence_proxy_async();
+    mbar_arrive(full0 + 8 * ((KC - 1) % S));
+  } else if (warp == 4) {
+    // ---------------- MMA issue (one thread)
+    if (lane == 0) {
+      const uint32_t idesc = idesc_bf16(128, NT);
+      for (int j = 0; j < KC; ++j) {
+        const int s = j % S;
+        mbar_wait(full0 + 8 * s, (j / S) & 1);
+        fence_after();
+        for (int q = 0; q < nq; ++q)
+          for (int ks = 0; ks < a.ksteps; ++ks) {
+            const uint64_t ad = umma_desc(As0 + (uint32_t)(s * nq + q) * kATile + (uint32_t)ks * 4096u, 2048, 128);
+            const uint64_t bd = umma_desc(Bs0 + (uint32_t)s * b_bytes + (uint32_t)(ks * 2 * NT * 16), NT * 16, 128);
+            mma_bf16(tmem + (uint32_t)(q * NT), ad, bd, idesc, (j > 0 || ks > 0) ? 1u : 0u);
+          }
+        mma_commit(empty0 + 8 * s);
+      }
+      mma_commit(done);
+    }
+  } else {
+    // ---------------- weight copies (one thread)
+    if (lane == 0) {
+      const uint8_t* wsrc = a.wpk + (int64_t)nt * KC * b_bytes;
+      for (int j = 0; j < KC; ++j) {
+        const int s = j % S;
+        mbar_wait(empty0 + 8 * s, ((j / S) & 1) ^ 1);
+        mbar_expect_tx(full0 + 8 * s, b_bytes);
+        bulk_g2s(Bs0 + (uint32_t)s * b_bytes, wsrc + (int64_t)j * b_bytes, b_bytes, full0 + 8 * s);
+      }
+    }
+  }
+
+  // ---------------- epilogue (warps 0-3): TMEM lane = tile row
+  if (warp < 4) {
+    mbar_wait(done, 0);
+    fence_after();
+    const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
+    bool qv[4] = {true, true, true, true};
+    if (a.pool == 2)
+      for (int q = 0; q < 4; ++q) qv[q] = (oy + (q >> 1) < a.H) && (ox + (q & 1) < a.W);
+    const int cbase = nt * NT;
+    for (int c0 = 0; c0 < NT; c0 += 16) {
+      uint32_t rr[16];
+      float v[16];
+      tmem_ld16(trow + (uint32_t)c0, rr);
+      tmem_wait_ld(rr);
+#pragma unroll
+      for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(rr[i]);
+      for (int q = 1; q < nq; ++q) {
+        tmem_ld16(trow + (uint32_t)(q * NT + c0), rr);
+        tmem_wait_ld(rr);
+        if (qv[q]) {
+#pragma unroll
+          for (int i = 0; i < 16; ++i) v[i] = fmaxf(v[i], __uint_as_float(rr[i]));
+        }
+      }
+      if (!rv) continue;
+      if (a.head) {
+        float* o = a.out_f32 + (int64_t)m * a.Cout + cbase + c0;
+#pragma unroll
+        for (int i = 0; i < 16; i += 4)
+          *reinterpret_cast<float4*>(o + i) = make_float4(v[i] + a.bias[cbase + c0 + i], v[i + 1] + a.bias[cbase + c0 + i + 1],
+                                                          v[i + 2] + a.bias[cbase + c0 + i + 2],
+                                                          v[i + 3] + a.bias[cbase + c0 + i + 3]);
+      } else {
+        uint32_t w[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          float x0 = v[2 * i] + a.bias[cbase + c0 + 2 * i], x1 = v[2 * i + 1] + a.bias[cbase + c0 + 2 * i + 1];
+          if (a.leaky) {
+            x0 = x0 < 0.f ? 0.1f * x0 : x0;
+            x1 = x1 < 0.f ? 0.1f * x1 : x1;
+          }
+          w[i] = pack_bf16(x0, x1);
+        }
+        uint4* o = reinterpret_cast<uint4*>(a.out + (int64_t)m * a.Cout + cbase + c0);
+        o[0] = make_uint4(w[0], w[1], w[2], w[3]);
+        o[1] = make_uint4(w[4], w[5], w[6], w[7]);
+      }
+    }
+    if (a.head && rv) {  // L171: count this cell's boxes whose score exceeds the threshold (Q31)
+      const float* o = a.out_f32 + (int64_t)m * a.Cout;
+      int cnt = 0;
+      for (int b = 0; b < 5; ++b) {
+        const float* p = o + 25 * b;
+        float mx = p[5];
+        for (int k = 1; k < 20; ++k) mx = fmaxf(mx, p[5 + k]);
+        float z = 0.f;
+        for (int k = 0; k < 20; ++k) z += __expf(p[5 + k] - mx);
+        const float score = __expf(p[5 + a.target] - mx) / z / (1.f + __expf(-p[4]));
+        cnt += score > a.thresh ? 1 : 0;
+      }
+      if (cnt) atomicAdd(a.counts + n, cnt);
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == 4) {
+    fence_after();
+    tmem_dealloc(tmem, (uint32_t)a.tmem_cols);
+  }
+}
+
+// Q28 resize of each raw RGB8 frame to 416x416, x = v / 256 (Q29) as bf16 NHWC with a zero 4th channel.
+__global__ void tyolo_resize_kernel(const TyFrame* frames, int32_t n, int32_t D, __nv_bfloat16* out) {
+  const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t per = (int64_t)D * D;
+  if (idx >= per * n) return;
+  const int f = (int)(idx / per);
+  const int p = (int)(idx - (int64_t)f * per);
+  const int oy = p / D, ox = p - oy * D;
+  const TyFrame fr = frames[f];
+  int y0 = (int)(((int64_t)oy * fr.H) / D), y1 = (int)(((int64_t)(oy + 1) * fr.H) / D);
+  int x0 = (int)(((int64_t)ox * fr.W) / D), x1 = (int)(((int64_t)(ox + 1) * fr.W) / D);
+  if (y1 <= y0) y1 = y0 + 1;
+  if (x1 <= x0) x1 = x0 + 1;
+  uint32_t s0 = 0, s1 = 0, s2 = 0;
+  for (int y = y0; y < y1; ++y) {
+    const uint8_t* row = fr.pixels + (int64_t)y * fr.pitch + 3 * x0;
+    for (int x = 0; x < x1 - x0; ++x) {
+      s0 += row[3 * x];
+      s1 += row[3 * x + 1];
+      s2 += row[3 * x + 2];
+    }
+  }
+  const uint32_t nn = (uint32_t)((y1 - y0) * (x1 - x0));
+  const float inv = 1.f / 256.f;
+  const float v0 = (float)((s0 + nn / 2) / nn) * inv, v1 = (float)((s1 + nn / 2) / nn) * inv,
+              v2 = (float)((s2 + nn / 2) / nn) * inv;
+  uint2 w;
+  w.x = pack_bf16(v0, v1);
+  w.y = pack_bf16(v2, 0.f);
+  *reinterpret_cast<uint2*>(out + idx * 4) = w;
+}
+
+}  // namespace
+
+int tyolo_conv_smem_bytes(int stages, int nq, int NT) {
+  return stages * (nq * kATile + NT * 128) + 8 * (2 * stages + 1) + 16;
+}
+
+cudaError_t tyolo_configure() {
+  return cudaFuncSetAttribute(tyolo_conv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+}
+
+cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st) {
+  const dim3 grid((unsigned)((a.M + 127) / 128), (unsigned)(a.Cout_tiles));
+  tyolo_conv_kernel<<<grid, kConvThreads, tyolo_conv_smem_bytes(a.stages, a.nq, a.NT), st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, __nv_bfloat16* out, cudaStream_t st) {
+  const int64_t total = (int64_t)n * D * D;
+  tyolo_resize_kernel<<<(unsigned)((total + 255) / 256), 256, 0, st>>>(frames, n, D, out);
+  return cudaGetLastError();
+}
+
+}  // namespace ffsva

@@ -1,0 +1,382 @@
+// ffsva_tyolo_host.cpp — the shared T-YOLO model of a device (f1; one model "shared by all
+// streams", L175) and its C-ABI: weight packing into the kernel's UMMA B layout, workspace, the layer sequence.
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <memory>
+#include <vector>
+
+#include "ffsva_runtime.h"
+
+using namespace ffsva;
+
+namespace {
+
+constexpr int kIn = 416;      // T-YOLO input size (L169)
+constexpr int kGrid = 13;     // output grid (L171)
+constexpr int kHeadPad = 128; // 125 outputs padded to a 128-column tile
+constexpr int kMaxChunk = 256;
+
+// tiny-yolo-voc: (Cin, Cout, kernel, pool after: 0 none, 1 2x2/2, 2 2x2/1)
+constexpr int kNet[9][4] = {{3, 16, 3, 1},     {16, 32, 3, 1},     {32, 64, 3, 1},
+                            {64, 128, 3, 1},   {128, 256, 3, 1},   {256, 512, 3, 2},
+                            {512, 1024, 3, 0}, {1024, 1024, 3, 0}, {1024, 125, 1, 0}};
+
+struct Layer {
+  int Cin, Cout, k, pool;
+  int Cp, Cout_pad, NT, nq, kchunks, ksteps, stages, tmem_cols;
+  int H;                      // conv spatial size (input = output before pooling)
+  int Ho;                     // after pooling
+  size_t w_off, b_off;        // into the packed weight / bias blobs (bytes / floats)
+  size_t w_bytes;
+};
+
+uint16_t bf16_bits(float x) { return bf16_bits_rne(x); }
+
+int pow2_at_least(int v) {
+  int p = 32;
+  while (p < v) p <<= 1;
+  return p;
+}
+
+}  // namespace
+
+struct ffsva_tyolo {
+  DeviceCtx* ctx = nullptr;
+  Layer L[9];
+  uint8_t* d_w = nullptr;
+  float* d_b = nullptr;
+  // workspace for up to `cap` frames per chunk
+  int cap = 0;
+  __nv_bfloat16* d_act[2] = {nullptr, nullptr};
+  float* d_raw = nullptr;
+  int32_t* d_counts = nullptr;
+  TyFrame* d_frames = nullptr;
+  TyFrame* h_frames = nullptr;
+  int32_t* h_counts = nullptr;
+};
+
+namespace {
+
+void build_layers(ffsva_tyolo* m) {
+  int H = kIn;
+  size_t w_off = 0, b_off = 0;
+  for (int l = 0; l < 9; ++l) {
+    Layer& L = m->L[l];
+    L.Cin = kNet[l][0];
+    L.Cout = kNet[l][1];
+    L.k = kNet[l][2];
+    L.pool = kNet[l][3];
+    L.Cp = L.Cin == 3 ? 4 : L.Cin;
+    L.Cout_pad = l == 8 ? kHeadPad : L.Cout;
+    L.nq = L.pool ? 4 : 1;
+    L.NT = std::min(L.Cout_pad, L.pool ? 128 : 256);
+    if (L.k == 1) L.kchunks = L.Cp / 64;
+    else if (L.Cp >= 64) L.kchunks = 9 * L.Cp / 64;
+    else if (L.Cp == 4) L.kchunks = 1;
+    else L.kchunks = (9 + 64 / L.Cp - 1) / (64 / L.Cp);
+    L.ksteps = L.Cp == 4 ? 3 : 4;  // the first layer's 9 taps x 4 channels = 36 K fit in 3 MMA K16 steps
+    const int stage = L.nq * 128 * 128 + L.NT * 128;
+    L.stages = std::max(2, std::min(4, (227 * 1024 - 1024) / stage));
+    L.tmem_cols = pow2_at_least(L.nq * L.NT);
+    L.H = H;
+    L.Ho = L.pool == 1 ? H / 2 : H;
+    L.w_off = w_off;
+    L.w_bytes = (size_t)(L.Cout_pad / L.NT) * L.kchunks * L.NT * 128;
+    w_off += L.w_bytes;
+    L.b_off = b_off;
+    b_off += L.Cout_pad;
+    H = L.Ho;
+  }
+}
+
+// Pack layer l's weights w[Cout][Cin][k][k] into [N tile][K step][K group 8][NT rows][8 bf16] (the kernel's B
+// tile layout: K-adjacent core matrices NT*16 B apart, 8-row groups 128 B apart).
+void pack_layer(const Layer& L, const float* w, uint8_t* dst) {
+  uint16_t* out = reinterpret_cast<uint16_t*>(dst);
+  const int tiles = L.Cout_pad / L.NT;
+  for (int t = 0; t < tiles; ++t)
+    for (int j = 0; j < L.kchunks; ++j)
+      for (int g = 0; g < 8; ++g)
+        for (int nn = 0; nn < L.NT; ++nn)
+          for (int e = 0; e < 8; ++e) {
+            const int kk = g * 8 + e;
+            int tap, c;
+            if (L.k == 1) {
+              tap = 4;
+              c = j * 64 + kk;
+            } else if (L.Cp >= 64) {
+              const int cpt = L.Cp / 64;
+              tap = j / cpt;
+              c = (j % cpt) * 64 + kk;
+            } else {
+              const int tpc = 64 / L.Cp;
+              tap = j * tpc + kk / L.Cp;
+              c = kk % L.Cp;
+            }
+            const int co = t * L.NT + nn;
+            float v = 0.f;
+            if (tap < 9 && c < L.Cin && co < L.Cout)
+              v = L.k == 1 ? w[(size_t)co * L.Cin + c] : w[(((size_t)co * L.Cin + c) * 3 + tap / 3) * 3 + tap % 3];
+            const size_t o = (((size_t)(t * L.kchunks + j) * 8 + g) * L.NT + nn) * 8 + e;
+            out[o] = bf16_bits(v);
+          }
+}
+
+ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
+  if (m->cap >= std::min(n, kMaxChunk)) return FFSVA_OK;
+  const int cap = std::min(kMaxChunk, std::max(n, 16));
+  cudaFree(m->d_act[0]);
+  cudaFree(m->d_act[1]);
+  cudaFree(m->d_raw);
+  cudaFree(m->d_counts);
+  cudaFree(m->d_frames);
+  cudaFreeHost(m->h_frames);
+  cudaFreeHost(m->h_counts);
+  m->cap = 0;
+  size_t act = 0;  // largest activation per frame (bytes)
+  act = std::max(act, (size_t)kIn * kIn * 4 * 2);
+  for (int l = 0; l < 8; ++l) act = std::max(act, (size_t)m->L[l].Ho * m->L[l].Ho * m->L[l].Cout_pad * 2);
+  cudaError_t e = cudaMalloc(&m->d_act[0], act * cap);
+  if (e == cudaSuccess) e = cudaMalloc(&m->d_act[1], act * cap);
+  if (e == cudaSuccess) e = cudaMalloc(&m->d_raw, (size_t)cap * kGrid * kGrid * kHeadPad * 4);
+  if (e == cudaSuccess) e = cudaMalloc(&m->d_counts, (size_t)cap * 4);
+  if (e == cudaSuccess) e = cudaMalloc(&m->d_frames, (size_t)cap * sizeof(TyFrame));
+  if (e == cudaSuccess) e = cudaMallocHost(&m->h_frames, (size_t)cap * sizeof(TyFrame));
+  if (e == cudaSuccess) e = cudaMallocHost(&m->h_counts, (size_t)cap * 4);
+  if (e != cudaSuccess) return cuda_fail(nullptr, e, "T-YOLO workspace");
+  m->cap = cap;
+  return FFSVA_OK;
+}
+
+TyConvArgs layer_args(const ffsva_tyolo* m, int l, int n, const __nv_bfloat16* in, __nv_bfloat16* out,
+                      int target, float thresh) {
+  const Layer& L = m->L[l];
+  TyConvArgs a{};
+  a.in = in;
+  a.out = out;
+  a.out_f32 = l == 8 ? m->d_raw : nullptr;
+  a.wpk = m->d_w + L.w_off;
+  a.bias = m->d_b + L.b_off;
+  a.N = n;
+  a.H = a.W = L.H;
+  a.Cp = L.Cp;
+  a.Ho = a.Wo = L.Ho;
+  a.Cout = L.Cout_pad;
+  a.NT = L.NT;
+  a.Cout_tiles = L.Cout_pad / L.NT;
+  a.nq = L.nq;
+  a.pool = L.pool;
+  a.ksize = L.k;
+  a.kchunks = L.kchunks;
+  a.ksteps = L.ksteps;
+  a.stages = L.stages;
+  a.tmem_cols = L.tmem_cols;
+  a.leaky = l < 8 ? 1 : 0;
+  a.M = n * L.Ho * L.Ho;
+  a.head = l == 8 ? 1 : 0;
+  a.target = target;
+  a.thresh = thresh;
+  a.counts = m->d_counts;
+  return a;
+}
+
+// Resize + layers [0, upto] for frames [0, n) (n <= cap), on stream st. ev (optional): 11 events around the
+// resize and each layer.
+ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, int n, int upto, int target, float thresh,
+                       cudaStream_t st, cudaEvent_t* ev) {
+  DeviceCtx* ctx = m->ctx;
+  for (int i = 0; i < n; ++i) {
+    const ffsva_stream_desc& d = frames[i].stream->desc;
+    m->h_frames[i] = TyFrame{frames[i].pixels, d.row_pitch, d.width, d.height};
+  }
+  cudaError_t e = cudaMemcpyAsync(m->d_frames, m->h_frames, sizeof(TyFrame) * n, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemsetAsync(m->d_counts, 0, 4 * (size_t)n, st);
+  if (e != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO staging");
+  if (ev) cudaEventRecord(ev[0], st);
+  if ((e = launch_tyolo_resize(m->d_frames, n, kIn, m->d_act[0], st)) != cudaSuccess)
+    return cuda_fail(ctx, e, "T-YOLO resize");
+  g_launches += 1;
+  if (ev) cudaEventRecord(ev[1], st);
+  int cur = 0;
+  for (int l = 0; l <= upto; ++l) {
+    const TyConvArgs a = layer_args(m, l, n, m->d_act[cur], m->d_act[cur ^ 1], target, thresh);
+    if ((e = launch_tyolo_conv(a, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO conv layer");
+    g_launches += 1;
+    if (ev) cudaEventRecord(ev[2 + l], st);
+    cur ^= 1;
+  }
+  return FFSVA_OK;
+}
+
+ffsva_status validate(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n) {
+  if (!m || n < 0 || (n > 0 && !frames)) return fail(FFSVA_EINVAL, "bad argument");
+  for (int32_t i = 0; i < n; ++i) {
+    if (!frames[i].stream || !frames[i].pixels) return fail(FFSVA_EINVAL, "frame without stream or pixels");
+    if (frames[i].stream->ctx != m->ctx) return fail(FFSVA_EDEVICE, "frame lives on another device");
+    const ffsva_stream_desc& d = frames[i].stream->desc;
+    ffsva_status cs = check_device_ptr(m->ctx, frames[i].pixels, (size_t)(d.height - 1) * d.row_pitch + 3 * d.width);
+    if (cs != FFSVA_OK) return cs;
+  }
+  if (m->ctx->sticky) return fail(FFSVA_ECUDA, "device is in a sticky CUDA error state");
+  return FFSVA_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+FFSVA_API ffsva_status ffsva_tyolo_load(int32_t device, const float* params, int64_t n_params, ffsva_tyolo** out) {
+  if (!params || !out) return fail(FFSVA_EINVAL, "NULL argument");
+  std::unique_ptr<ffsva_tyolo> m(new ffsva_tyolo());
+  build_layers(m.get());
+  int64_t need = 0;
+  for (auto& L : m->L) need += (int64_t)L.Cout * L.Cin * L.k * L.k + L.Cout;
+  if (n_params != need) return fail(FFSVA_EINVAL, "n_params != 15,858,717 (tiny-yolo-voc)");
+  for (int64_t i = 0; i < n_params; ++i)
+    if (!std::isfinite(params[i])) return fail(FFSVA_EINVAL, "non-finite T-YOLO parameter");
+  ffsva_status st;
+  DeviceCtx* ctx = ctx_acquire(device, &st);
+  if (!ctx) return st;
+  m->ctx = ctx;
+  size_t wbytes = 0, nb = 0;
+  for (auto& L : m->L) {
+    wbytes += L.w_bytes;
+    nb += L.Cout_pad;
+  }
+  std::vector<uint8_t> hw(wbytes);
+  std::vector<float> hb(nb, 0.f);
+  const float* p = params;
+  for (auto& L : m->L) {
+    const size_t nw = (size_t)L.Cout * L.Cin * L.k * L.k;
+    pack_layer(L, p, hw.data() + L.w_off);
+    std::memcpy(hb.data() + L.b_off, p + nw, sizeof(float) * L.Cout);
+    p += nw + L.Cout;
+  }
+  {
+    std::lock_guard<std::mutex> lk(ctx->mu);
+    DeviceGuard g(device);
+    cudaError_t e = cudaMalloc(&m->d_w, wbytes);
+    if (e == cudaSuccess) e = cudaMalloc(&m->d_b, nb * 4);
+    if (e == cudaSuccess) e = cudaMemcpy(m->d_w, hw.data(), wbytes, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = cudaMemcpy(m->d_b, hb.data(), nb * 4, cudaMemcpyHostToDevice);
+    if (e == cudaSuccess) e = tyolo_configure();
+    if (e != cudaSuccess) {
+      cudaFree(m->d_w);
+      cudaFree(m->d_b);
+      ctx_release(ctx);
+      return cuda_fail(nullptr, e, "ffsva_tyolo_load");
+    }
+  }
+  *out = m.release();
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_tyolo_run(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, int32_t target_class,
+                                       float thresh, int32_t number_of_objects, int32_t* counts, uint8_t* pass,
+                                       float* raw, void* cuda_stream) {
+  if (target_class < 0 || target_class >= 20) return fail(FFSVA_EINVAL, "target_class must be a VOC class 0..19");
+  if (n > 0 && !counts && !pass && !raw) return fail(FFSVA_EINVAL, "no output requested");
+  ffsva_status st = validate(m, frames, n);
+  if (st != FFSVA_OK || n == 0) return st;
+  DeviceCtx* ctx = m->ctx;
+  std::lock_guard<std::mutex> lk(ctx->mu);
+  DeviceGuard g(ctx->device);
+  if ((st = ensure_workspace(m, n)) != FFSVA_OK) return st;
+  cudaStream_t cs = (cudaStream_t)cuda_stream;
+  for (int32_t i0 = 0; i0 < n; i0 += m->cap) {
+    const int cnt = std::min(m->cap, n - i0);
+    if ((st = run_chunk(m, frames + i0, cnt, 8, target_class, thresh, cs, nullptr)) != FFSVA_OK) return st;
+    cudaError_t e = cudaMemcpyAsync(m->h_counts, m->d_counts, 4 * (size_t)cnt, cudaMemcpyDeviceToHost, cs);
+    if (e == cudaSuccess && raw) {  // [cnt][13][13][125] from the 128-wide padded rows
+      e = cudaMemcpy2DAsync(raw + (size_t)i0 * kGrid * kGrid * 125, 125 * 4, m->d_raw, kHeadPad * 4, 125 * 4,
+                            (size_t)cnt * kGrid * kGrid, cudaMemcpyDeviceToHost, cs);
+    }
+    if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_tyolo_run");
+    for (int i = 0; i < cnt; ++i) {
+      if (counts) counts[i0 + i] = m->h_counts[i];
+      if (pass) pass[i0 + i] = m->h_counts[i] >= number_of_objects ? 1 : 0;  // L195 NumberofObjects
+    }
+  }
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, int32_t layer,
+                                                uint16_t* out, void* cuda_stream) {
+  if (layer < -1 || layer > 7 || !out) return fail(FFSVA_EINVAL, "layer must be -1 (resized input) .. 7");
+  ffsva_status st = validate(m, frames, n);
+  if (st != FFSVA_OK || n == 0) return st;
+  DeviceCtx* ctx = m->ctx;
+  std::lock_guard<std::mutex> lk(ctx->mu);
+  DeviceGuard g(ctx->device);
+  if (n > kMaxChunk) return fail(FFSVA_EINVAL, "at most 256 frames");
+  if ((st = ensure_workspace(m, n)) != FFSVA_OK) return st;
+  cudaStream_t cs = (cudaStream_t)cuda_stream;
+  if ((st = run_chunk(m, frames, n, layer, 0, 0.2f, cs, nullptr)) != FFSVA_OK) return st;
+  const size_t bytes = layer < 0 ? (size_t)n * kIn * kIn * 4 * 2
+                                 : (size_t)n * m->L[layer].Ho * m->L[layer].Ho * m->L[layer].Cout_pad * 2;
+  const int buf = (layer + 1) & 1;  // the resize writes act[0], layer l writes act[(l + 1) & 1]
+  cudaError_t e = cudaMemcpyAsync(out, m->d_act[buf], bytes, cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+  if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_tyolo_layer_output");
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_tyolo_profile(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, int32_t iters,
+                                           float* ms_out, void* cuda_stream) {
+  if (iters < 1 || !ms_out) return fail(FFSVA_EINVAL, "bad argument");
+  ffsva_status st = validate(m, frames, n);
+  if (st != FFSVA_OK || n == 0) return st;
+  if (n > kMaxChunk) return fail(FFSVA_EINVAL, "at most 256 frames per profiled chunk");
+  DeviceCtx* ctx = m->ctx;
+  std::lock_guard<std::mutex> lk(ctx->mu);
+  DeviceGuard g(ctx->device);
+  if ((st = ensure_workspace(m, n)) != FFSVA_OK) return st;
+  cudaStream_t cs = (cudaStream_t)cuda_stream;
+  cudaEvent_t ev[11];
+  for (auto& e : ev) cudaEventCreate(&e);
+  double acc[10] = {0};
+  for (int it = 0; it < iters && st == FFSVA_OK; ++it) {
+    st = run_chunk(m, frames, n, 8, 6, 0.2f, cs, ev);
+    if (st != FFSVA_OK) break;
+    cudaError_t e = cudaEventSynchronize(ev[10]);
+    if (e != cudaSuccess) {
+      st = cuda_fail(ctx, e, "ffsva_tyolo_profile");
+      break;
+    }
+    for (int k = 0; k < 10; ++k) {
+      float t = 0.f;
+      cudaEventElapsedTime(&t, ev[k], ev[k + 1]);
+      acc[k] += t;
+    }
+  }
+  for (auto& e : ev) cudaEventDestroy(e);
+  if (st != FFSVA_OK) return st;
+  for (int k = 0; k < 10; ++k) ms_out[k] = (float)(acc[k] / iters);
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_tyolo_destroy(ffsva_tyolo* m) {
+  if (!m) return FFSVA_OK;
+  DeviceCtx* ctx = m->ctx;
+  {
+    std::lock_guard<std::mutex> lk(ctx->mu);
+    DeviceGuard g(ctx->device);
+    cudaDeviceSynchronize();
+    cudaFree(m->d_w);
+    cudaFree(m->d_b);
+    cudaFree(m->d_act[0]);
+    cudaFree(m->d_act[1]);
+    cudaFree(m->d_raw);
+    cudaFree(m->d_counts);
+    cudaFree(m->d_frames);
+    cudaFreeHost(m->h_frames);
+    cudaFreeHost(m->h_counts);
+  }
+  delete m;
+  ctx_release(ctx);
+  return FFSVA_OK;
+}
+
+}  // extern "C"

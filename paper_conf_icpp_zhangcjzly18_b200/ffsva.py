@@ -32,7 +32,8 @@ EXPORTS = ["ffsva_open_stream", "ffsva_set_reference", "ffsva_snm_load", "ffsva_
            "ffsva_stream_info", "ffsva_stats_copy", "ffsva_close", "ffsva_last_error", "ffsva_kernel_launches",
            "ffsva_version", "ffsva_sched_create", "ffsva_sched_push", "ffsva_sched_tick", "ffsva_sched_depth",
            "ffsva_sched_destroy", "ffsva_sched_set_policy", "ffsva_stream_image_bytes", "ffsva_stream_export",
-           "ffsva_stream_import", "ffsva_sched_stream_load", "ffsva_sched_detach"]
+           "ffsva_stream_import", "ffsva_sched_stream_load", "ffsva_sched_detach", "ffsva_tyolo_load",
+           "ffsva_tyolo_run", "ffsva_tyolo_layer_output", "ffsva_tyolo_profile", "ffsva_tyolo_destroy"]
 
 
 class StreamDesc(ctypes.Structure):
@@ -132,6 +133,11 @@ def lib():
             "ffsva_stream_import": [i32, vp, i64, i32, ctypes.POINTER(vp)],
             "ffsva_sched_stream_load": [vp, vp, i32, ctypes.POINTER(StreamLoad)],
             "ffsva_sched_detach": [vp, vp],
+            "ffsva_tyolo_load": [i32, vp, i64, ctypes.POINTER(vp)],
+            "ffsva_tyolo_run": [vp, vp, i32, i32, ctypes.c_float, i32, vp, vp, vp, vp],
+            "ffsva_tyolo_layer_output": [vp, vp, i32, i32, vp, vp],
+            "ffsva_tyolo_profile": [vp, vp, i32, i32, vp, vp],
+            "ffsva_tyolo_destroy": [vp],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -544,4 +550,64 @@ class PreparedBatch:
     def destroy(self) -> None:
         if self.handle:
             ffsva_batch_destroy(self.handle)
+            self.handle = None
+
+
+# ---------------------------------------------------------------------------------------------- T-YOLO (f1)
+TYOLO_GRID = 13
+
+
+def _bf16_bits_to_f32(u16: np.ndarray) -> np.ndarray:
+    return (u16.astype(np.uint32) << 16).view(np.float32)
+
+
+class Tyolo:
+    """The shared T-YOLO stage of a device (NumberofObjects L195; include/ffsva.h)."""
+
+    def __init__(self, ctx: "Context", params: np.ndarray):
+        p = np.ascontiguousarray(params, dtype=np.float32)
+        h = ctypes.c_void_p()
+        _check(lib().ffsva_tyolo_load(ctx.device, p.ctypes.data, p.size, ctypes.byref(h)), "ffsva_tyolo_load")
+        self.ctx, self.handle = ctx, h.value
+
+    def run(self, items, target_class: int = 6, thresh: float = 0.2, number_of_objects: int = 1,
+            raw: bool = False, stream=None) -> dict:
+        """items: (Stream, device pixels, frame_no) as for Context.filter_batch. Returns counts, pass (and raw
+        head outputs [n, 13, 13, 125] fp32 when raw=True)."""
+        fr = _frames_array(Context._frames(items))
+        n = len(items)
+        counts = np.zeros(n, np.int32)
+        ok = np.zeros(n, np.uint8)
+        out = np.zeros((n, TYOLO_GRID, TYOLO_GRID, 125), np.float32) if raw else None
+        _check(lib().ffsva_tyolo_run(self.handle, ctypes.addressof(fr), n, target_class, thresh,
+                                     number_of_objects, counts.ctypes.data, ok.ctypes.data,
+                                     out.ctypes.data if raw else None, _stream_handle(stream)), "ffsva_tyolo_run")
+        res = {"counts": counts, "pass": ok}
+        if raw:
+            res["raw"] = out
+        return res
+
+    def layer_output(self, items, layer: int, stream=None) -> np.ndarray:
+        """Diagnostic: float32 copy of the bf16 NHWC activation after `layer` (-1 = resized input)."""
+        fr = _frames_array(Context._frames(items))
+        n = len(items)
+        shapes = {-1: (416, 4), 0: (208, 16), 1: (104, 32), 2: (52, 64), 3: (26, 128), 4: (13, 256), 5: (13, 512),
+                  6: (13, 1024), 7: (13, 1024)}
+        hw, c = shapes[layer]
+        out = np.zeros((n, hw, hw, c), np.uint16)
+        _check(lib().ffsva_tyolo_layer_output(self.handle, ctypes.addressof(fr), n, layer, out.ctypes.data,
+                                              _stream_handle(stream)), "ffsva_tyolo_layer_output")
+        return _bf16_bits_to_f32(out)
+
+    def profile(self, items, iters: int = 5, stream=None) -> list:
+        """Mean device ms of [resize, layer 1..9] over iters runs (CUDA events on the launching stream)."""
+        fr = _frames_array(Context._frames(items))
+        ms = (ctypes.c_float * 10)()
+        _check(lib().ffsva_tyolo_profile(self.handle, ctypes.addressof(fr), len(items), iters, ms, _stream_handle(stream)),
+               "ffsva_tyolo_profile")
+        return list(ms)
+
+    def destroy(self) -> None:
+        if self.handle:
+            _check(lib().ffsva_tyolo_destroy(self.handle), "ffsva_tyolo_destroy")
             self.handle = None
