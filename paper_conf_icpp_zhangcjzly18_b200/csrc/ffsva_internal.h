@@ -159,11 +159,14 @@ struct TyConvArgs {
   int32_t nq, pool, ksize;   // accumulator chains (4 for pool layers), pool 0/1 (2x2/2)/2 (2x2/1), kernel 3 or 1
   int32_t kchunks, ksteps;   // K steps of 64 channels, MMA K16 steps per K step
   int32_t stages, tmem_cols, leaky, M;
+  int32_t acc_bufs, grid;    // TMEM accumulator buffers (1 or 2), persistent grid size (CTAs)
   int32_t head, target;      // head: count boxes of class `target` scoring > thresh into counts[frame]
   float thresh;
   int32_t* counts;
 };
 cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st);
+cudaError_t launch_tyolo_pool_s1(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C,
+                                 cudaStream_t st);
 cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, __nv_bfloat16* out, cudaStream_t st);
 int tyolo_conv_smem_bytes(int stages, int nq, int NT);
 cudaError_t tyolo_configure();

@@ -29,7 +29,7 @@ namespace {
 
 using namespace ptx;
 
-constexpr int kConvThreads = 192;  // warps 0-3: A gather + epilogue, warp 4: TMEM + MMA issue, warp 5: B copies
+constexpr int kConvThreads = 320;  // warps 0-3: A gather, 4: TMEM + MMA issue, 5: B copies, 6-9: epilogue
 constexpr int kATile = 128 * 128;  // one stage of A for one chain: 128 rows x 64 bf16
 
 // byte offset of (K group g of 8 bf16, row r) in a 128-row K-major no-swizzle tile: core matrices of 8 rows x 16 B,
@@ -93,26 +93,42 @@ __device__ __forceinline__ void conv_pixel(const TyConvArgs& a, int oy, int ox, 
   }
 }
 
+// Decode output row m of the layer into (frame, oy, ox).
+__device__ __forceinline__ void decode_row(const TyConvArgs& a, int m, int& n, int& oy, int& ox) {
+  const int hw = a.Ho * a.Wo;
+  n = m / hw;
+  const int rem = m - n * hw;
+  oy = rem / a.Wo;
+  ox = rem - oy * a.Wo;
+}
+
+// Persistent, warp-specialised: each CTA walks tiles t = blockIdx.x, + gridDim.x, ... (tile = 128 output rows x NT
+// channels); one K-step ring (S stages) runs continuously across tiles, and the TMEM accumulator is double
+// buffered when 2 x nq x NT columns fit, so the epilogue of tile i overlaps the mainloop of tile i + 1.
 __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs a) {
   extern __shared__ __align__(1024) uint8_t sm[];
-  const int S = a.stages, nq = a.nq, NT = a.NT, KC = a.kchunks;
+  const int S = a.stages, nq = a.nq, NT = a.NT, KC = a.kchunks, NB = a.acc_bufs;
   const uint32_t stage_a = (uint32_t)nq * kATile;
   const uint32_t b_bytes = (uint32_t)NT * 128;
   uint8_t* As = sm;
   uint8_t* Bs = sm + (size_t)S * stage_a;
   uint64_t* bars = reinterpret_cast<uint64_t*>(Bs + (size_t)S * b_bytes);
-  uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 2 * S + 1);
-  const uint32_t full0 = smem_addr(bars), empty0 = full0 + 8 * S, done = full0 + 16 * S;
+  uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 2 * S + 4);
+  const uint32_t full0 = smem_addr(bars), empty0 = full0 + 8 * S;
+  const uint32_t accf0 = full0 + 16 * S, acce0 = accf0 + 16;  // acc_full[2], acc_empty[2]
   const uint32_t As0 = smem_addr(As), Bs0 = smem_addr(Bs);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int m0 = blockIdx.x * 128, nt = blockIdx.y;
+  const int n_tiles = a.Cout_tiles, tiles = ((a.M + 127) / 128) * n_tiles;
 
   if (tid == 0) {
     for (int s = 0; s < S; ++s) {
       mbar_init(full0 + 8 * s, 129);  // 128 gather threads + the weight copy's expect_tx arrival
       mbar_init(empty0 + 8 * s, 1);
     }
-    mbar_init(done, 1);
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(accf0 + 8 * b, 1);
+      mbar_init(acce0 + 8 * b, 128);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 4) tmem_alloc(smem_addr(s_tmem), (uint32_t)a.tmem_cols);
@@ -121,131 +137,143 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
   fence_after();
   const uint32_t tmem = *s_tmem;
 
-  const int r = tid;  // warps 0-3: tile row = TMEM lane
-  const int m = m0 + (r & 127);
-  const bool rv = warp < 4 && m < a.M;
-  int n = 0, oy = 0, ox = 0;
-  if (rv) {
-    const int hw = a.Ho * a.Wo;
-    n = m / hw;
-    const int rem = m - n * hw;
-    oy = rem / a.Wo;
-    ox = rem - oy * a.Wo;
-  }
-
   if (warp < 4) {
-    // ---------------- A producers
-    const __nv_bfloat16* img = a.in + (int64_t)n * a.H * a.W * a.Cp;
-    for (int j = 0; j < KC; ++j) {
-      const int s = j % S;
-      mbar_wait(empty0 + 8 * s, ((j / S) & 1) ^ 1);
-      for (int q = 0; q < nq; ++q) {
-        int cy, cx;
-        conv_pixel(a, oy, ox, q, cy, cx);
-        gather(a, img, rv, cy, cx, j, As0 + (uint32_t)(s * nq + q) * kATile, r);
-      }
-      cp_async_commit();
-      if (j > 0) {  // the previous step's copies have landed: publish them to the tensor core (async proxy)
-        cp_async_wait<1>();
-        fence_proxy_async();
-        mbar_arrive(full0 + 8 * ((j - 1) % S));
+    // ---------------- A producers: thread = tile row
+    const int r = tid;
+    int g = 0;  // global K-step counter (continues across tiles)
+    for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
+      const int m = (t / n_tiles) * 128 + r;
+      const bool rv = m < a.M;
+      int n = 0, oy = 0, ox = 0;
+      if (rv) decode_row(a, m, n, oy, ox);
+      const __nv_bfloat16* img = a.in + (int64_t)n * a.H * a.W * a.Cp;
+      for (int j = 0; j < KC; ++j, ++g) {
+        const int s = g % S;
+        mbar_wait(empty0 + 8 * s, ((g / S) & 1) ^ 1);
+        for (int q = 0; q < nq; ++q) {
+          int cy, cx;
+          conv_pixel(a, oy, ox, q, cy, cx);
+          gather(a, img, rv, cy, cx, j, As0 + (uint32_t)(s * nq + q) * kATile, r);
+        }
+        cp_async_commit();
+        if (g > 0) {  // the previous step's copies have landed: publish them to the tensor core (async proxy)
+          cp_async_wait<1>();
+          fence_proxy_async();
+          mbar_arrive(full0 + 8 * ((g - 1) % S));
+        }
       }
     }
-    cp_async_wait<0>();
-    fence_proxy_async();
-    mbar_arrive(full0 + 8 * ((KC - 1) % S));
+    if (g > 0) {
+      cp_async_wait<0>();
+      fence_proxy_async();
+      mbar_arrive(full0 + 8 * ((g - 1) % S));
+    }
   } else if (warp == 4) {
     // ---------------- MMA issue (one thread)
     if (lane == 0) {
       const uint32_t idesc = idesc_bf16(128, NT);
-      for (int j = 0; j < KC; ++j) {
-        const int s = j % S;
-        mbar_wait(full0 + 8 * s, (j / S) & 1);
+      int g = 0, i = 0;
+      for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++i) {
+        const int b = i % NB;
+        mbar_wait(acce0 + 8 * b, ((i / NB) & 1) ^ 1);  // the epilogue has drained this accumulator
         fence_after();
-        for (int q = 0; q < nq; ++q)
-          for (int ks = 0; ks < a.ksteps; ++ks) {
-            const uint64_t ad = umma_desc(As0 + (uint32_t)(s * nq + q) * kATile + (uint32_t)ks * 4096u, 2048, 128);
-            const uint64_t bd = umma_desc(Bs0 + (uint32_t)s * b_bytes + (uint32_t)(ks * 2 * NT * 16), NT * 16, 128);
-            mma_bf16(tmem + (uint32_t)(q * NT), ad, bd, idesc, (j > 0 || ks > 0) ? 1u : 0u);
-          }
-        mma_commit(empty0 + 8 * s);
+        const uint32_t acc = tmem + (uint32_t)(b * nq * NT);
+        for (int j = 0; j < KC; ++j, ++g) {
+          const int s = g % S;
+          mbar_wait(full0 + 8 * s, (g / S) & 1);
+          fence_after();
+          for (int q = 0; q < nq; ++q)
+            for (int ks = 0; ks < a.ksteps; ++ks) {
+              const uint64_t ad = umma_desc(As0 + (uint32_t)(s * nq + q) * kATile + (uint32_t)ks * 4096u, 2048, 128);
+              const uint64_t bd = umma_desc(Bs0 + (uint32_t)s * b_bytes + (uint32_t)(ks * 2 * NT * 16), NT * 16, 128);
+              mma_bf16(acc + (uint32_t)(q * NT), ad, bd, idesc, (j > 0 || ks > 0) ? 1u : 0u);
+            }
+          mma_commit(empty0 + 8 * s);
+        }
+        mma_commit(accf0 + 8 * b);
       }
-      mma_commit(done);
     }
-  } else {
+  } else if (warp == 5) {
     // ---------------- weight copies (one thread)
     if (lane == 0) {
-      const uint8_t* wsrc = a.wpk + (int64_t)nt * KC * b_bytes;
-      for (int j = 0; j < KC; ++j) {
-        const int s = j % S;
-        mbar_wait(empty0 + 8 * s, ((j / S) & 1) ^ 1);
-        mbar_expect_tx(full0 + 8 * s, b_bytes);
-        bulk_g2s(Bs0 + (uint32_t)s * b_bytes, wsrc + (int64_t)j * b_bytes, b_bytes, full0 + 8 * s);
+      int g = 0;
+      for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
+        const uint8_t* wsrc = a.wpk + (int64_t)(t % n_tiles) * KC * b_bytes;
+        for (int j = 0; j < KC; ++j, ++g) {
+          const int s = g % S;
+          mbar_wait(empty0 + 8 * s, ((g / S) & 1) ^ 1);
+          mbar_expect_tx(full0 + 8 * s, b_bytes);
+          bulk_g2s(Bs0 + (uint32_t)s * b_bytes, wsrc + (int64_t)j * b_bytes, b_bytes, full0 + 8 * s);
+        }
       }
     }
-  }
-
-  // ---------------- epilogue (warps 0-3): TMEM lane = tile row
-  if (warp < 4) {
-    mbar_wait(done, 0);
-    fence_after();
-    const uint32_t trow = tmem + ((uint32_t)(32 * warp) << 16);
-    bool qv[4] = {true, true, true, true};
-    if (a.pool == 2)
-      for (int q = 0; q < 4; ++q) qv[q] = (oy + (q >> 1) < a.H) && (ox + (q & 1) < a.W);
-    const int cbase = nt * NT;
-    for (int c0 = 0; c0 < NT; c0 += 16) {
-      uint32_t rr[16];
-      float v[16];
-      tmem_ld16(trow + (uint32_t)c0, rr);
-      tmem_wait_ld(rr);
-#pragma unroll
-      for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(rr[i]);
-      for (int q = 1; q < nq; ++q) {
-        tmem_ld16(trow + (uint32_t)(q * NT + c0), rr);
+  } else {
+    // ---------------- epilogue (warps 6-9): TMEM lane quadrant = warp % 4, row = 32 * quadrant + lane
+    const int qd = warp & 3, r = 32 * qd + lane;
+    int i = 0;
+    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++i) {
+      const int b = i % NB, nt = t % n_tiles;
+      const int m = (t / n_tiles) * 128 + r;
+      const bool rv = m < a.M;
+      int n = 0, oy = 0, ox = 0;
+      if (rv) decode_row(a, m, n, oy, ox);
+      mbar_wait(accf0 + 8 * b, (i / NB) & 1);
+      fence_after();
+      const uint32_t trow = tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(b * nq * NT);
+      const int cbase = nt * NT;
+      for (int c0 = 0; c0 < NT; c0 += 16) {
+        uint32_t rr[16];
+        float v[16];
+        tmem_ld16(trow + (uint32_t)c0, rr);
         tmem_wait_ld(rr);
-        if (qv[q]) {
 #pragma unroll
-          for (int i = 0; i < 16; ++i) v[i] = fmaxf(v[i], __uint_as_float(rr[i]));
+        for (int k = 0; k < 16; ++k) v[k] = __uint_as_float(rr[k]);
+        for (int q = 1; q < nq; ++q) {
+          tmem_ld16(trow + (uint32_t)(q * NT + c0), rr);
+          tmem_wait_ld(rr);
+#pragma unroll
+          for (int k = 0; k < 16; ++k) v[k] = fmaxf(v[k], __uint_as_float(rr[k]));
         }
-      }
-      if (!rv) continue;
-      if (a.head) {
-        float* o = a.out_f32 + (int64_t)m * a.Cout + cbase + c0;
+        if (!rv) continue;
+        const float* bias = a.bias + cbase + c0;
+        if (a.head) {
+          float* o = a.out_f32 + (int64_t)m * a.Cout + cbase + c0;
 #pragma unroll
-        for (int i = 0; i < 16; i += 4)
-          *reinterpret_cast<float4*>(o + i) = make_float4(v[i] + a.bias[cbase + c0 + i], v[i + 1] + a.bias[cbase + c0 + i + 1],
-                                                          v[i + 2] + a.bias[cbase + c0 + i + 2],
-                                                          v[i + 3] + a.bias[cbase + c0 + i + 3]);
-      } else {
-        uint32_t w[8];
+          for (int k = 0; k < 16; k += 4)
+            *reinterpret_cast<float4*>(o + k) =
+                make_float4(v[k] + bias[k], v[k + 1] + bias[k + 1], v[k + 2] + bias[k + 2], v[k + 3] + bias[k + 3]);
+        } else {
+          uint32_t w[8];
 #pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          float x0 = v[2 * i] + a.bias[cbase + c0 + 2 * i], x1 = v[2 * i + 1] + a.bias[cbase + c0 + 2 * i + 1];
-          if (a.leaky) {
-            x0 = x0 < 0.f ? 0.1f * x0 : x0;
-            x1 = x1 < 0.f ? 0.1f * x1 : x1;
+          for (int k = 0; k < 8; ++k) {
+            float x0 = v[2 * k] + bias[2 * k], x1 = v[2 * k + 1] + bias[2 * k + 1];
+            if (a.leaky) {
+              x0 = x0 < 0.f ? 0.1f * x0 : x0;
+              x1 = x1 < 0.f ? 0.1f * x1 : x1;
+            }
+            w[k] = pack_bf16(x0, x1);
           }
-          w[i] = pack_bf16(x0, x1);
+          uint4* o = reinterpret_cast<uint4*>(a.out + (int64_t)m * a.Cout + cbase + c0);
+          o[0] = make_uint4(w[0], w[1], w[2], w[3]);
+          o[1] = make_uint4(w[4], w[5], w[6], w[7]);
         }
-        uint4* o = reinterpret_cast<uint4*>(a.out + (int64_t)m * a.Cout + cbase + c0);
-        o[0] = make_uint4(w[0], w[1], w[2], w[3]);
-        o[1] = make_uint4(w[4], w[5], w[6], w[7]);
       }
-    }
-    if (a.head && rv) {  // L171: count this cell's boxes whose score exceeds the threshold (Q31)
-      const float* o = a.out_f32 + (int64_t)m * a.Cout;
-      int cnt = 0;
-      for (int b = 0; b < 5; ++b) {
-        const float* p = o + 25 * b;
-        float mx = p[5];
-        for (int k = 1; k < 20; ++k) mx = fmaxf(mx, p[5 + k]);
-        float z = 0.f;
-        for (int k = 0; k < 20; ++k) z += __expf(p[5 + k] - mx);
-        const float score = __expf(p[5 + a.target] - mx) / z / (1.f + __expf(-p[4]));
-        cnt += score > a.thresh ? 1 : 0;
+      fence_before();
+      mbar_arrive(acce0 + 8 * b);  // this accumulator may be overwritten
+      if (a.head && rv) {  // L171: count this cell's boxes whose score exceeds the threshold (Q31)
+        const float* o = a.out_f32 + (int64_t)m * a.Cout;
+        int cnt = 0;
+        for (int bx = 0; bx < 5; ++bx) {
+          const float* p = o + 25 * bx;
+          float mx = p[5];
+          for (int k = 1; k < 20; ++k) mx = fmaxf(mx, p[5 + k]);
+          float z = 0.f;
+          for (int k = 0; k < 20; ++k) z += __expf(p[5 + k] - mx);
+          const float score = __expf(p[5 + a.target] - mx) / z / (1.f + __expf(-p[4]));
+          cnt += score > a.thresh ? 1 : 0;
+        }
+        if (cnt) atomicAdd(a.counts + n, cnt);
       }
-      if (cnt) atomicAdd(a.counts + n, cnt);
     }
   }
   fence_before();
@@ -254,6 +282,41 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
     fence_after();
     tmem_dealloc(tmem, (uint32_t)a.tmem_cols);
   }
+}
+
+// 2x2 max-pool with stride 1 and a -inf right/bottom border (Q30) on bf16 NHWC, 8 channels per thread. Applied
+// after the layer-6 convolution (bf16 rounding is monotone, so pooling the rounded values equals rounding the
+// pooled ones).
+__global__ void tyolo_pool_s1_kernel(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C) {
+  const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int c8 = C >> 3;
+  const int64_t total = (int64_t)n * H * H * c8;
+  if (idx >= total) return;
+  const int cg = (int)(idx % c8);
+  const int64_t p = idx / c8;
+  const int x = (int)(p % H), y = (int)((p / H) % H);
+  const int64_t base = p - (int64_t)y * H - x;  // frame's first pixel
+  __nv_bfloat162 mx[4];
+  const uint4 v0 = *reinterpret_cast<const uint4*>(in + p * C + 8 * cg);
+  mx[0] = *reinterpret_cast<const __nv_bfloat162*>(&v0.x);
+  mx[1] = *reinterpret_cast<const __nv_bfloat162*>(&v0.y);
+  mx[2] = *reinterpret_cast<const __nv_bfloat162*>(&v0.z);
+  mx[3] = *reinterpret_cast<const __nv_bfloat162*>(&v0.w);
+  for (int d = 1; d < 4; ++d) {
+    const int yy = y + (d >> 1), xx = x + (d & 1);
+    if (yy >= H || xx >= H) continue;
+    const uint4 v = *reinterpret_cast<const uint4*>(in + (base + (int64_t)yy * H + xx) * C + 8 * cg);
+    mx[0] = __hmax2(mx[0], *reinterpret_cast<const __nv_bfloat162*>(&v.x));
+    mx[1] = __hmax2(mx[1], *reinterpret_cast<const __nv_bfloat162*>(&v.y));
+    mx[2] = __hmax2(mx[2], *reinterpret_cast<const __nv_bfloat162*>(&v.z));
+    mx[3] = __hmax2(mx[3], *reinterpret_cast<const __nv_bfloat162*>(&v.w));
+  }
+  uint4 o;
+  o.x = *reinterpret_cast<uint32_t*>(&mx[0]);
+  o.y = *reinterpret_cast<uint32_t*>(&mx[1]);
+  o.z = *reinterpret_cast<uint32_t*>(&mx[2]);
+  o.w = *reinterpret_cast<uint32_t*>(&mx[3]);
+  *reinterpret_cast<uint4*>(out + p * C + 8 * cg) = o;
 }
 
 // Q28 resize of each raw RGB8 frame to 416x416, x = v / 256 (Q29) as bf16 NHWC with a zero 4th channel.
@@ -291,7 +354,7 @@ __global__ void tyolo_resize_kernel(const TyFrame* frames, int32_t n, int32_t D,
 }  // namespace
 
 int tyolo_conv_smem_bytes(int stages, int nq, int NT) {
-  return stages * (nq * kATile + NT * 128) + 8 * (2 * stages + 1) + 16;
+  return stages * (nq * kATile + NT * 128) + 8 * (2 * stages + 4) + 16;
 }
 
 cudaError_t tyolo_configure() {
@@ -299,8 +362,16 @@ cudaError_t tyolo_configure() {
 }
 
 cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st) {
-  const dim3 grid((unsigned)((a.M + 127) / 128), (unsigned)(a.Cout_tiles));
+  const int tiles = ((a.M + 127) / 128) * a.Cout_tiles;
+  const unsigned grid = (unsigned)(tiles < a.grid ? tiles : a.grid);
   tyolo_conv_kernel<<<grid, kConvThreads, tyolo_conv_smem_bytes(a.stages, a.nq, a.NT), st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tyolo_pool_s1(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C,
+                                 cudaStream_t st) {
+  const int64_t total = (int64_t)n * H * H * (C / 8);
+  tyolo_pool_s1_kernel<<<(unsigned)((total + 255) / 256), 256, 0, st>>>(in, out, n, H, C);
   return cudaGetLastError();
 }
 

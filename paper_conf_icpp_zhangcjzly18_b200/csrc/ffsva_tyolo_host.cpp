@@ -23,8 +23,9 @@ constexpr int kNet[9][4] = {{3, 16, 3, 1},     {16, 32, 3, 1},     {32, 64, 3, 1
                             {512, 1024, 3, 0}, {1024, 1024, 3, 0}, {1024, 125, 1, 0}};
 
 struct Layer {
-  int Cin, Cout, k, pool;
-  int Cp, Cout_pad, NT, nq, kchunks, ksteps, stages, tmem_cols;
+  int Cin, Cout, k, pool;     // pool: the network's (0 none, 1 2x2/2, 2 2x2/1)
+  int conv_pool;              // pool folded into the conv kernel (the 2x2/2 layers); 2x2/1 runs as its own kernel
+  int Cp, Cout_pad, NT, nq, kchunks, ksteps, stages, tmem_cols, acc_bufs;
   int H;                      // conv spatial size (input = output before pooling)
   int Ho;                     // after pooling
   size_t w_off, b_off;        // into the packed weight / bias blobs (bytes / floats)
@@ -69,8 +70,9 @@ void build_layers(ffsva_tyolo* m) {
     L.pool = kNet[l][3];
     L.Cp = L.Cin == 3 ? 4 : L.Cin;
     L.Cout_pad = l == 8 ? kHeadPad : L.Cout;
-    L.nq = L.pool ? 4 : 1;
-    L.NT = std::min(L.Cout_pad, L.pool ? 128 : 256);
+    L.conv_pool = L.pool == 1 ? 1 : 0;
+    L.nq = L.conv_pool ? 4 : 1;
+    L.NT = std::min(L.Cout_pad, L.conv_pool ? 128 : 256);
     if (L.k == 1) L.kchunks = L.Cp / 64;
     else if (L.Cp >= 64) L.kchunks = 9 * L.Cp / 64;
     else if (L.Cp == 4) L.kchunks = 1;
@@ -78,7 +80,8 @@ void build_layers(ffsva_tyolo* m) {
     L.ksteps = L.Cp == 4 ? 3 : 4;  // the first layer's 9 taps x 4 channels = 36 K fit in 3 MMA K16 steps
     const int stage = L.nq * 128 * 128 + L.NT * 128;
     L.stages = std::max(2, std::min(4, (227 * 1024 - 1024) / stage));
-    L.tmem_cols = pow2_at_least(L.nq * L.NT);
+    L.acc_bufs = 2 * L.nq * L.NT <= 512 ? 2 : 1;  // double-buffered accumulator when it fits in TMEM
+    L.tmem_cols = pow2_at_least(L.acc_bufs * L.nq * L.NT);
     L.H = H;
     L.Ho = L.pool == 1 ? H / 2 : H;
     L.w_off = w_off;
@@ -166,12 +169,14 @@ TyConvArgs layer_args(const ffsva_tyolo* m, int l, int n, const __nv_bfloat16* i
   a.NT = L.NT;
   a.Cout_tiles = L.Cout_pad / L.NT;
   a.nq = L.nq;
-  a.pool = L.pool;
+  a.pool = L.conv_pool;
   a.ksize = L.k;
   a.kchunks = L.kchunks;
   a.ksteps = L.ksteps;
   a.stages = L.stages;
   a.tmem_cols = L.tmem_cols;
+  a.acc_bufs = L.acc_bufs;
+  a.grid = m->ctx->num_sms;
   a.leaky = l < 8 ? 1 : 0;
   a.M = n * L.Ho * L.Ho;
   a.head = l == 8 ? 1 : 0;
@@ -182,9 +187,9 @@ TyConvArgs layer_args(const ffsva_tyolo* m, int l, int n, const __nv_bfloat16* i
 }
 
 // Resize + layers [0, upto] for frames [0, n) (n <= cap), on stream st. ev (optional): 11 events around the
-// resize and each layer.
+// resize and each layer. *out_buf receives the activation buffer holding the last layer's output.
 ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, int n, int upto, int target, float thresh,
-                       cudaStream_t st, cudaEvent_t* ev) {
+                       cudaStream_t st, cudaEvent_t* ev, int* out_buf = nullptr) {
   DeviceCtx* ctx = m->ctx;
   for (int i = 0; i < n; ++i) {
     const ffsva_stream_desc& d = frames[i].stream->desc;
@@ -203,9 +208,17 @@ ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, int n, int upt
     const TyConvArgs a = layer_args(m, l, n, m->d_act[cur], m->d_act[cur ^ 1], target, thresh);
     if ((e = launch_tyolo_conv(a, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO conv layer");
     g_launches += 1;
-    if (ev) cudaEventRecord(ev[2 + l], st);
     cur ^= 1;
+    if (m->L[l].pool == 2) {  // 2x2/1 max-pool (Q30) back into the layer's input buffer
+      const Layer& L = m->L[l];
+      if ((e = launch_tyolo_pool_s1(m->d_act[cur], m->d_act[cur ^ 1], n, L.Ho, L.Cout_pad, st)) != cudaSuccess)
+        return cuda_fail(ctx, e, "T-YOLO 2x2/1 pool");
+      g_launches += 1;
+      cur ^= 1;
+    }
+    if (ev) cudaEventRecord(ev[2 + l], st);
   }
+  if (out_buf) *out_buf = cur;
   return FFSVA_OK;
 }
 
@@ -313,10 +326,10 @@ FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_fram
   if (n > kMaxChunk) return fail(FFSVA_EINVAL, "at most 256 frames");
   if ((st = ensure_workspace(m, n)) != FFSVA_OK) return st;
   cudaStream_t cs = (cudaStream_t)cuda_stream;
-  if ((st = run_chunk(m, frames, n, layer, 0, 0.2f, cs, nullptr)) != FFSVA_OK) return st;
+  int buf = 0;
+  if ((st = run_chunk(m, frames, n, layer, 0, 0.2f, cs, nullptr, &buf)) != FFSVA_OK) return st;
   const size_t bytes = layer < 0 ? (size_t)n * kIn * kIn * 4 * 2
                                  : (size_t)n * m->L[layer].Ho * m->L[layer].Ho * m->L[layer].Cout_pad * 2;
-  const int buf = (layer + 1) & 1;  // the resize writes act[0], layer l writes act[(l + 1) & 1]
   cudaError_t e = cudaMemcpyAsync(out, m->d_act[buf], bytes, cudaMemcpyDeviceToHost, cs);
   if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_tyolo_layer_output");
