@@ -51,6 +51,10 @@ CONFIGS = {
                   step_frames=30, period=300, on_len=150, seed=1004),
     "m5": dict(desc="M5: 256 streams 1920x1080 sharded over the GPUs, 1 target frame in 10", streams=256,
                W=1920, H=1080, pool_frames=10, step_frames=10, period=10, on_len=1, seed=1005, shard=True),
+    # f1: the T-YOLO stage on a batch of SNM survivors (random-init tiny-yolo-voc weights)
+    "tyolo": dict(desc="f1 T-YOLO stage: 256 SNM-surviving 1280x720 frames per step through tiny-yolo-voc at "
+                       "416x416 (random-init weights), NumberofObjects count", streams=1, W=1280, H=720,
+                  pool_frames=256, step_frames=256, period=4, on_len=2, seed=1007),
     # standalone SNM (K4) run for its tensor-pipe roofline: delta_diff = 0 lets every frame
     # through SDD, so one step scores 65,536 survivors across 256 streams (100x100 frames keep K1 small)
     "snm": dict(desc="SNM microbenchmark: 65,536 survivors/step across 256 streams (100x100 frames, "
@@ -320,6 +324,84 @@ def run_ours(args, cfg, ws, rank, local):
     return out
 
 
+# tiny-yolo-voc convolutions at 416x416: (H, Cin, Cout, k); algorithmic FLOPs = 2 x MACs at full resolution
+TYOLO_CONV = [(416, 3, 16, 3), (208, 16, 32, 3), (104, 32, 64, 3), (52, 64, 128, 3), (26, 128, 256, 3),
+              (13, 256, 512, 3), (13, 512, 1024, 3), (13, 1024, 1024, 3), (13, 1024, 125, 1)]
+TYOLO_FLOP = sum(2 * h * h * ci * co * k * k for h, ci, co, k in TYOLO_CONV)  # 6,971,041,792 per frame
+
+
+def run_tyolo(args, cfg, ws, rank, local):
+    """--config tyolo: the f1 stage alone. Device time per step = the mean CUDA-event time of the resize and the
+    nine layers over the timed steps (ffsva_tyolo_profile, events on the launching stream); e2e = wall time of
+    ffsva_tyolo_run (host call, counts copied back) per step."""
+    import torch
+    import paper_conf_icpp_zhangcjzly18_b200 as ff
+    from synth import synth
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    W, H, P, n = cfg["W"], cfg["H"], 3 * cfg["W"], cfg["step_frames"]
+    video = synth.Video(seed=cfg["seed"], width=W, height=H, period=cfg["period"], on_len=cfg["on_len"])
+    frames = torch.empty((n, H, P), dtype=torch.uint8, device=dev)
+    synth.frames_cuda(video, torch.zeros(n, dtype=torch.int32, device=dev), torch.arange(n, dtype=torch.int64,
+                      device=dev), frames, H * P, P)
+    ctx = ff.Context(dev)
+    st = ctx.open_stream(width=W, height=H)
+    params = synth.tyolo_weights(cfg["seed"])
+    ty = ff.Tyolo(ctx, params)
+    items = [(st, frames[i], i) for i in range(n)]
+    cs = torch.cuda.Stream(device=dev)
+    launches0 = ff.ffsva_kernel_launches()
+    ty.profile(items, args.warmup, stream=cs)
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)
+    ms = ty.profile(items, args.steps, stream=cs)
+    clk = clocks.stop()
+    launches = (ff.ffsva_kernel_launches() - launches0) * args.steps // (args.steps + args.warmup)
+    step_ms = sum(ms)
+    value = n / (step_ms / 1e3)
+    _, tf_peak, peak_kind = measured_peaks()
+    layer_tf = [TYOLO_CONV[i][0] ** 2 * 2 * TYOLO_CONV[i][1] * TYOLO_CONV[i][2] * TYOLO_CONV[i][3] ** 2 * n
+                / (ms[i + 1] / 1e3) / 1e12 for i in range(9)]
+    dom = max(range(9), key=lambda i: ms[i + 1])
+    achieved = TYOLO_FLOP * n / (step_ms / 1e3) / 1e12
+    t0 = time.perf_counter()
+    n_e2e = max(1, min(5, args.steps))
+    for _ in range(n_e2e):
+        res = ty.run(items, number_of_objects=2, stream=cs)
+    e2e = n * n_e2e / (time.perf_counter() - t0)
+    cpu = None
+    if not args.no_cpu_baseline:
+        from oracle import oracle as orc
+        host = frames[:2].cpu().numpy()
+        t0 = time.perf_counter()
+        for i in range(2):
+            orc.tyolo_forward(orc.resize(host[i], W, 416, 416), params, bf16_emul=False)
+        dt = time.perf_counter() - t0
+        cpu = {"value": 2 / dt, "unit": "frames/s", "cores": 1, "kind": "oracle",
+               "sample": "2 frames (resize + the nine layers in fp64 + count) of the same workload", "seconds": dt}
+    out = {"metric": "T-YOLO frames/sec (f1 stage, 416x416 tiny-yolo-voc)", "value": value, "unit": "frames/s",
+           "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": step_ms,
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16 (fp32 accumulate)",
+           "data": "synthetic",
+           "config": {"workload": cfg["desc"], "config_id": "tyolo", "frames_per_step": n, "seed": cfg["seed"],
+                      "l2": "activations of 256 frames (up to 354 MB per layer) exceed L2; weights 31.7 MB bf16"},
+           "roofline": {"bound": "tensor", "kernel": "K5 tyolo_conv_kernel (all nine layers)",
+                        "achieved": achieved, "peak": tf_peak, "unit": "TFLOP/s", "frac": achieved / tf_peak,
+                        "peak_source": peak_kind, "traffic": None, "flop_per_frame": TYOLO_FLOP,
+                        "dominant_layer": f"L{dom + 1}", "dominant_layer_tflops": layer_tf[dom],
+                        "layer_ms": {("resize" if i == 0 else f"L{i}"): ms[i] for i in range(10)},
+                        "layer_tflops": {f"L{i + 1}": layer_tf[i] for i in range(9)}},
+           "cpu_baseline": cpu,
+           "e2e": {"value": e2e, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 8 * n,
+                   "path": "ffsva_tyolo_run on device-resident frames (host call, counts + pass copied back)",
+                   "mean_count": float(np.mean(res["counts"]))},
+           "gpu_launches": int(launches), "clocks": clk}
+    ty.destroy()
+    ctx.close()
+    return out
+
+
 def online_validation(args, ctx, video, sids, pool, value, dev, cs):
     """Paced 30-FPS streams through the online runtime (feedback queue + dynamic batching, §4.3).
     Stream i replays content stream i % len(sids) of the pool with its own reference image and SNM."""
@@ -478,7 +560,7 @@ def main():
             # other ranks wait for rank 0's build (the .so must exist before they load it)
             while not os.path.exists(os.path.join(ROOT, "paper_conf_icpp_zhangcjzly18_b200", "lib", "libffsva.so")):
                 time.sleep(0.5)
-        out = run_ours(args, cfg, ws, rank, local)
+        out = run_tyolo(args, cfg, ws, rank, local) if args.config == "tyolo" else run_ours(args, cfg, ws, rank, local)
     if rank == 0 and out is not None:
         print(json.dumps(out))
 

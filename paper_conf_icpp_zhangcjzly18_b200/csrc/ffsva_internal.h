@@ -160,6 +160,8 @@ struct TyConvArgs {
   int32_t kchunks, ksteps;   // K steps of 64 channels, MMA K16 steps per K step
   int32_t stages, tmem_cols, leaky, M;
   int32_t acc_bufs, grid;    // TMEM accumulator buffers (1 or 2), persistent grid size (CTAs)
+  int32_t msub;              // 128-row halves per tile sharing each weight stage (1 or 2)
+  int32_t patch;             // pool layers: A row = the pooled pixel's 4x4 input patch, weights per pool position
   int32_t head, target;      // head: count boxes of class `target` scoring > thresh into counts[frame]
   float thresh;
   int32_t* counts;
@@ -168,7 +170,7 @@ cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st);
 cudaError_t launch_tyolo_pool_s1(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C,
                                  cudaStream_t st);
 cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, __nv_bfloat16* out, cudaStream_t st);
-int tyolo_conv_smem_bytes(int stages, int nq, int NT);
+int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT);
 cudaError_t tyolo_configure();
 
 cudaError_t launch_fill_nan(float* p, int32_t n, cudaStream_t st);

@@ -102,23 +102,55 @@ __device__ __forceinline__ void decode_row(const TyConvArgs& a, int m, int& n, i
   ox = rem - oy * a.Wo;
 }
 
-// Persistent, warp-specialised: each CTA walks tiles t = blockIdx.x, + gridDim.x, ... (tile = 128 output rows x NT
-// channels); one K-step ring (S stages) runs continuously across tiles, and the TMEM accumulator is double
-// buffered when 2 x nq x NT columns fit, so the epilogue of tile i overlaps the mainloop of tile i + 1.
+// Patch gather (pool layers with few input channels): the A row of pooled pixel (oy, ox) is its 4x4 input patch
+// (rows 2oy-1 .. 2oy+2, columns 2ox-1 .. 2ox+2) x Cp channels, pixel-major; K step j holds 64 of its values. The
+// four pool positions then differ only in their weights (the 3x3 kernel placed at offset (a, b) of the 4x4 patch),
+// so one A tile feeds all four accumulator chains.
+__device__ __forceinline__ void gather_patch(const TyConvArgs& a, const __nv_bfloat16* img, bool rv, int oy, int ox,
+                                             int j, uint32_t dst, int r) {
+  const int H = a.H, W = a.W, Cp = a.Cp;
+  if (Cp == 4) {  // all 16 patch pixels in one K step, two pixels per 16-byte K group
+#pragma unroll
+    for (int p = 0; p < 16; ++p) {
+      const int sy = 2 * oy - 1 + (p >> 2), sx = 2 * ox - 1 + (p & 3);
+      const bool v = rv && sy >= 0 && sy < H && sx >= 0 && sx < W;
+      cp_async8(dst + a_off(p >> 1, r) + 8 * (p & 1), v ? img + ((int64_t)sy * W + sx) * 4 : a.in, v);
+    }
+  } else {  // Cp = 8 * upp channels: 64 / Cp pixels per K step, upp 16-byte units each
+    const int ppc = 64 / Cp, upp = Cp >> 3;
+    for (int pl = 0; pl < ppc; ++pl) {
+      const int p = j * ppc + pl;
+      const int sy = 2 * oy - 1 + (p >> 2), sx = 2 * ox - 1 + (p & 3);
+      const bool v = rv && sy >= 0 && sy < H && sx >= 0 && sx < W;
+      const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * Cp : a.in;
+      for (int u = 0; u < upp; ++u) cp_async16(dst + a_off(pl * upp + u, r), src + 8 * u, v);
+    }
+  }
+}
+
+// Persistent, warp-specialised: each CTA walks tiles t = blockIdx.x, + gridDim.x, ... A tile = msub x 128 output
+// rows x NT channels (msub = 2 shares every weight stage between two 128-row halves: half the L2 weight traffic
+// per MAC for the wide 13x13 layers). One K-step ring (S stages) runs continuously across tiles; the TMEM
+// accumulators are double buffered when they fit twice, so the epilogue of tile i overlaps tile i + 1's mainloop.
+// Stage = a_tiles A tiles (msub x (patch ? 1 : nq)) + b_tiles B tiles (patch ? nq : 1).
 __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs a) {
   extern __shared__ __align__(1024) uint8_t sm[];
-  const int S = a.stages, nq = a.nq, NT = a.NT, KC = a.kchunks, NB = a.acc_bufs;
-  const uint32_t stage_a = (uint32_t)nq * kATile;
-  const uint32_t b_bytes = (uint32_t)NT * 128;
+  const int S = a.stages, nq = a.nq, NT = a.NT, KC = a.kchunks, NB = a.acc_bufs, MS = a.msub;
+  const int a_per_sub = a.patch ? 1 : nq;
+  const int b_tiles = a.patch ? nq : 1;
+  const uint32_t stage_a = (uint32_t)(MS * a_per_sub) * kATile;
+  const uint32_t b_tile = (uint32_t)NT * 128, stage_b = (uint32_t)b_tiles * b_tile;
+  const int acc_cols = MS * nq * NT;  // per accumulator buffer
   uint8_t* As = sm;
   uint8_t* Bs = sm + (size_t)S * stage_a;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(Bs + (size_t)S * b_bytes);
+  uint64_t* bars = reinterpret_cast<uint64_t*>(Bs + (size_t)S * stage_b);
   uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 2 * S + 4);
   const uint32_t full0 = smem_addr(bars), empty0 = full0 + 8 * S;
   const uint32_t accf0 = full0 + 16 * S, acce0 = accf0 + 16;  // acc_full[2], acc_empty[2]
   const uint32_t As0 = smem_addr(As), Bs0 = smem_addr(Bs);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-  const int n_tiles = a.Cout_tiles, tiles = ((a.M + 127) / 128) * n_tiles;
+  const int rows_per_tile = 128 * MS;
+  const int n_tiles = a.Cout_tiles, tiles = ((a.M + rows_per_tile - 1) / rows_per_tile) * n_tiles;
 
   if (tid == 0) {
     for (int s = 0; s < S; ++s) {
@@ -138,22 +170,32 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
   const uint32_t tmem = *s_tmem;
 
   if (warp < 4) {
-    // ---------------- A producers: thread = tile row
+    // ---------------- A producers: thread = row r of every 128-row half of the tile
     const int r = tid;
     int g = 0;  // global K-step counter (continues across tiles)
     for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
-      const int m = (t / n_tiles) * 128 + r;
-      const bool rv = m < a.M;
-      int n = 0, oy = 0, ox = 0;
-      if (rv) decode_row(a, m, n, oy, ox);
-      const __nv_bfloat16* img = a.in + (int64_t)n * a.H * a.W * a.Cp;
+      int n[2] = {0, 0}, oy[2] = {0, 0}, ox[2] = {0, 0};
+      bool rv[2] = {false, false};
+      for (int i = 0; i < MS; ++i) {
+        const int m = (t / n_tiles) * rows_per_tile + i * 128 + r;
+        rv[i] = m < a.M;
+        if (rv[i]) decode_row(a, m, n[i], oy[i], ox[i]);
+      }
       for (int j = 0; j < KC; ++j, ++g) {
         const int s = g % S;
         mbar_wait(empty0 + 8 * s, ((g / S) & 1) ^ 1);
-        for (int q = 0; q < nq; ++q) {
-          int cy, cx;
-          conv_pixel(a, oy, ox, q, cy, cx);
-          gather(a, img, rv, cy, cx, j, As0 + (uint32_t)(s * nq + q) * kATile, r);
+        for (int i = 0; i < MS; ++i) {
+          const __nv_bfloat16* img = a.in + (int64_t)n[i] * a.H * a.W * a.Cp;
+          const uint32_t base = As0 + (uint32_t)s * stage_a + (uint32_t)(i * a_per_sub) * kATile;
+          if (a.patch) {
+            gather_patch(a, img, rv[i], oy[i], ox[i], j, base, r);
+          } else {
+            for (int q = 0; q < nq; ++q) {
+              int cy, cx;
+              conv_pixel(a, oy[i], ox[i], q, cy, cx);
+              gather(a, img, rv[i], cy, cx, j, base + (uint32_t)q * kATile, r);
+            }
+          }
         }
         cp_async_commit();
         if (g > 0) {  // the previous step's copies have landed: publish them to the tensor core (async proxy)
@@ -172,21 +214,25 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
     // ---------------- MMA issue (one thread)
     if (lane == 0) {
       const uint32_t idesc = idesc_bf16(128, NT);
-      int g = 0, i = 0;
-      for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++i) {
-        const int b = i % NB;
-        mbar_wait(acce0 + 8 * b, ((i / NB) & 1) ^ 1);  // the epilogue has drained this accumulator
+      int g = 0, it = 0;
+      for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
+        const int b = it % NB;
+        mbar_wait(acce0 + 8 * b, ((it / NB) & 1) ^ 1);  // the epilogue has drained this accumulator
         fence_after();
-        const uint32_t acc = tmem + (uint32_t)(b * nq * NT);
+        const uint32_t acc = tmem + (uint32_t)(b * acc_cols);
         for (int j = 0; j < KC; ++j, ++g) {
           const int s = g % S;
           mbar_wait(full0 + 8 * s, (g / S) & 1);
           fence_after();
-          for (int q = 0; q < nq; ++q)
-            for (int ks = 0; ks < a.ksteps; ++ks) {
-              const uint64_t ad = umma_desc(As0 + (uint32_t)(s * nq + q) * kATile + (uint32_t)ks * 4096u, 2048, 128);
-              const uint64_t bd = umma_desc(Bs0 + (uint32_t)s * b_bytes + (uint32_t)(ks * 2 * NT * 16), NT * 16, 128);
-              mma_bf16(acc + (uint32_t)(q * NT), ad, bd, idesc, (j > 0 || ks > 0) ? 1u : 0u);
+          for (int i = 0; i < MS; ++i)
+            for (int q = 0; q < nq; ++q) {
+              const uint32_t at = As0 + (uint32_t)s * stage_a + (uint32_t)(i * a_per_sub + (a.patch ? 0 : q)) * kATile;
+              const uint32_t bt = Bs0 + (uint32_t)s * stage_b + (uint32_t)(a.patch ? q : 0) * b_tile;
+              for (int ks = 0; ks < a.ksteps; ++ks) {
+                const uint64_t ad = umma_desc(at + (uint32_t)ks * 4096u, 2048, 128);
+                const uint64_t bd = umma_desc(bt + (uint32_t)(ks * 2 * NT * 16), NT * 16, 128);
+                mma_bf16(acc + (uint32_t)((i * nq + q) * NT), ad, bd, idesc, (j > 0 || ks > 0) ? 1u : 0u);
+              }
             }
           mma_commit(empty0 + 8 * s);
         }
@@ -194,86 +240,88 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
       }
     }
   } else if (warp == 5) {
-    // ---------------- weight copies (one thread)
+    // ---------------- weight copies (one thread): all B tiles of a step are one contiguous block
     if (lane == 0) {
       int g = 0;
       for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
-        const uint8_t* wsrc = a.wpk + (int64_t)(t % n_tiles) * KC * b_bytes;
+        const uint8_t* wsrc = a.wpk + (int64_t)(t % n_tiles) * KC * stage_b;
         for (int j = 0; j < KC; ++j, ++g) {
           const int s = g % S;
           mbar_wait(empty0 + 8 * s, ((g / S) & 1) ^ 1);
-          mbar_expect_tx(full0 + 8 * s, b_bytes);
-          bulk_g2s(Bs0 + (uint32_t)s * b_bytes, wsrc + (int64_t)j * b_bytes, b_bytes, full0 + 8 * s);
+          mbar_expect_tx(full0 + 8 * s, stage_b);
+          bulk_g2s(Bs0 + (uint32_t)s * stage_b, wsrc + (int64_t)j * stage_b, stage_b, full0 + 8 * s);
         }
       }
     }
   } else {
     // ---------------- epilogue (warps 6-9): TMEM lane quadrant = warp % 4, row = 32 * quadrant + lane
     const int qd = warp & 3, r = 32 * qd + lane;
-    int i = 0;
-    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++i) {
-      const int b = i % NB, nt = t % n_tiles;
-      const int m = (t / n_tiles) * 128 + r;
-      const bool rv = m < a.M;
-      int n = 0, oy = 0, ox = 0;
-      if (rv) decode_row(a, m, n, oy, ox);
-      mbar_wait(accf0 + 8 * b, (i / NB) & 1);
+    int it = 0;
+    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
+      const int b = it % NB, nt = t % n_tiles;
+      mbar_wait(accf0 + 8 * b, (it / NB) & 1);
       fence_after();
-      const uint32_t trow = tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(b * nq * NT);
       const int cbase = nt * NT;
-      for (int c0 = 0; c0 < NT; c0 += 16) {
-        uint32_t rr[16];
-        float v[16];
-        tmem_ld16(trow + (uint32_t)c0, rr);
-        tmem_wait_ld(rr);
-#pragma unroll
-        for (int k = 0; k < 16; ++k) v[k] = __uint_as_float(rr[k]);
-        for (int q = 1; q < nq; ++q) {
-          tmem_ld16(trow + (uint32_t)(q * NT + c0), rr);
+      for (int i = 0; i < MS; ++i) {
+        const int m = (t / n_tiles) * rows_per_tile + i * 128 + r;
+        const bool rv = m < a.M;
+        int n = 0, oy = 0, ox = 0;
+        if (rv) decode_row(a, m, n, oy, ox);
+        const uint32_t trow = tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(b * acc_cols + i * nq * NT);
+        for (int c0 = 0; c0 < NT; c0 += 16) {
+          uint32_t rr[16];
+          float v[16];
+          tmem_ld16(trow + (uint32_t)c0, rr);
           tmem_wait_ld(rr);
 #pragma unroll
-          for (int k = 0; k < 16; ++k) v[k] = fmaxf(v[k], __uint_as_float(rr[k]));
-        }
-        if (!rv) continue;
-        const float* bias = a.bias + cbase + c0;
-        if (a.head) {
-          float* o = a.out_f32 + (int64_t)m * a.Cout + cbase + c0;
+          for (int k = 0; k < 16; ++k) v[k] = __uint_as_float(rr[k]);
+          for (int q = 1; q < nq; ++q) {
+            tmem_ld16(trow + (uint32_t)(q * NT + c0), rr);
+            tmem_wait_ld(rr);
 #pragma unroll
-          for (int k = 0; k < 16; k += 4)
-            *reinterpret_cast<float4*>(o + k) =
-                make_float4(v[k] + bias[k], v[k + 1] + bias[k + 1], v[k + 2] + bias[k + 2], v[k + 3] + bias[k + 3]);
-        } else {
-          uint32_t w[8];
-#pragma unroll
-          for (int k = 0; k < 8; ++k) {
-            float x0 = v[2 * k] + bias[2 * k], x1 = v[2 * k + 1] + bias[2 * k + 1];
-            if (a.leaky) {
-              x0 = x0 < 0.f ? 0.1f * x0 : x0;
-              x1 = x1 < 0.f ? 0.1f * x1 : x1;
-            }
-            w[k] = pack_bf16(x0, x1);
+            for (int k = 0; k < 16; ++k) v[k] = fmaxf(v[k], __uint_as_float(rr[k]));
           }
-          uint4* o = reinterpret_cast<uint4*>(a.out + (int64_t)m * a.Cout + cbase + c0);
-          o[0] = make_uint4(w[0], w[1], w[2], w[3]);
-          o[1] = make_uint4(w[4], w[5], w[6], w[7]);
+          if (!rv) continue;
+          const float* bias = a.bias + cbase + c0;
+          if (a.head) {
+            float* o = a.out_f32 + (int64_t)m * a.Cout + cbase + c0;
+#pragma unroll
+            for (int k = 0; k < 16; k += 4)
+              *reinterpret_cast<float4*>(o + k) =
+                  make_float4(v[k] + bias[k], v[k + 1] + bias[k + 1], v[k + 2] + bias[k + 2], v[k + 3] + bias[k + 3]);
+          } else {
+            uint32_t w[8];
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+              float x0 = v[2 * k] + bias[2 * k], x1 = v[2 * k + 1] + bias[2 * k + 1];
+              if (a.leaky) {
+                x0 = x0 < 0.f ? 0.1f * x0 : x0;
+                x1 = x1 < 0.f ? 0.1f * x1 : x1;
+              }
+              w[k] = pack_bf16(x0, x1);
+            }
+            uint4* o = reinterpret_cast<uint4*>(a.out + (int64_t)m * a.Cout + cbase + c0);
+            o[0] = make_uint4(w[0], w[1], w[2], w[3]);
+            o[1] = make_uint4(w[4], w[5], w[6], w[7]);
+          }
+        }
+        if (a.head && rv) {  // L171: count this cell's boxes whose score exceeds the threshold (Q31)
+          const float* o = a.out_f32 + (int64_t)m * a.Cout;
+          int cnt = 0;
+          for (int bx = 0; bx < 5; ++bx) {
+            const float* p = o + 25 * bx;
+            float mx = p[5];
+            for (int k = 1; k < 20; ++k) mx = fmaxf(mx, p[5 + k]);
+            float z = 0.f;
+            for (int k = 0; k < 20; ++k) z += __expf(p[5 + k] - mx);
+            const float score = __expf(p[5 + a.target] - mx) / z / (1.f + __expf(-p[4]));
+            cnt += score > a.thresh ? 1 : 0;
+          }
+          if (cnt) atomicAdd(a.counts + n, cnt);
         }
       }
       fence_before();
       mbar_arrive(acce0 + 8 * b);  // this accumulator may be overwritten
-      if (a.head && rv) {  // L171: count this cell's boxes whose score exceeds the threshold (Q31)
-        const float* o = a.out_f32 + (int64_t)m * a.Cout;
-        int cnt = 0;
-        for (int bx = 0; bx < 5; ++bx) {
-          const float* p = o + 25 * bx;
-          float mx = p[5];
-          for (int k = 1; k < 20; ++k) mx = fmaxf(mx, p[5 + k]);
-          float z = 0.f;
-          for (int k = 0; k < 20; ++k) z += __expf(p[5 + k] - mx);
-          const float score = __expf(p[5 + a.target] - mx) / z / (1.f + __expf(-p[4]));
-          cnt += score > a.thresh ? 1 : 0;
-        }
-        if (cnt) atomicAdd(a.counts + n, cnt);
-      }
     }
   }
   fence_before();
@@ -353,8 +401,8 @@ __global__ void tyolo_resize_kernel(const TyFrame* frames, int32_t n, int32_t D,
 
 }  // namespace
 
-int tyolo_conv_smem_bytes(int stages, int nq, int NT) {
-  return stages * (nq * kATile + NT * 128) + 8 * (2 * stages + 4) + 16;
+int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT) {
+  return stages * (a_tiles * kATile + b_tiles * NT * 128) + 8 * (2 * stages + 4) + 16;
 }
 
 cudaError_t tyolo_configure() {
@@ -362,9 +410,11 @@ cudaError_t tyolo_configure() {
 }
 
 cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st) {
-  const int tiles = ((a.M + 127) / 128) * a.Cout_tiles;
+  const int rows = 128 * a.msub;
+  const int tiles = ((a.M + rows - 1) / rows) * a.Cout_tiles;
   const unsigned grid = (unsigned)(tiles < a.grid ? tiles : a.grid);
-  tyolo_conv_kernel<<<grid, kConvThreads, tyolo_conv_smem_bytes(a.stages, a.nq, a.NT), st>>>(a);
+  const int a_tiles = a.msub * (a.patch ? 1 : a.nq), b_tiles = a.patch ? a.nq : 1;
+  tyolo_conv_kernel<<<grid, kConvThreads, tyolo_conv_smem_bytes(a.stages, a_tiles, b_tiles, a.NT), st>>>(a);
   return cudaGetLastError();
 }
 

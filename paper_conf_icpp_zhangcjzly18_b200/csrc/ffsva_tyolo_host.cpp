@@ -2,6 +2,7 @@
 // streams", L175) and its C-ABI: weight packing into the kernel's UMMA B layout, workspace, the layer sequence.
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <memory>
 #include <vector>
@@ -26,6 +27,7 @@ struct Layer {
   int Cin, Cout, k, pool;     // pool: the network's (0 none, 1 2x2/2, 2 2x2/1)
   int conv_pool;              // pool folded into the conv kernel (the 2x2/2 layers); 2x2/1 runs as its own kernel
   int Cp, Cout_pad, NT, nq, kchunks, ksteps, stages, tmem_cols, acc_bufs;
+  int patch, msub;            // kernel variants (see TyConvArgs)
   int H;                      // conv spatial size (input = output before pooling)
   int Ho;                     // after pooling
   size_t w_off, b_off;        // into the packed weight / bias blobs (bytes / floats)
@@ -59,7 +61,15 @@ struct ffsva_tyolo {
 
 namespace {
 
+int env_int(const char* name, int dflt) {
+  const char* v = std::getenv(name);
+  return v ? std::atoi(v) : dflt;
+}
+
 void build_layers(ffsva_tyolo* m) {
+  // A/B knobs: patch gather for pool layers with Cp <= FFSVA_TYOLO_PATCH_CP (default 32), and FFSVA_TYOLO_MSUB
+  // 128-row halves per tile for the non-pool layers (default 2)
+  const int patch_cp = env_int("FFSVA_TYOLO_PATCH_CP", 32), msub = env_int("FFSVA_TYOLO_MSUB", 2);
   int H = kIn;
   size_t w_off = 0, b_off = 0;
   for (int l = 0; l < 9; ++l) {
@@ -73,19 +83,24 @@ void build_layers(ffsva_tyolo* m) {
     L.conv_pool = L.pool == 1 ? 1 : 0;
     L.nq = L.conv_pool ? 4 : 1;
     L.NT = std::min(L.Cout_pad, L.conv_pool ? 128 : 256);
-    if (L.k == 1) L.kchunks = L.Cp / 64;
+    L.patch = L.conv_pool && L.Cp <= patch_cp ? 1 : 0;
+    L.msub = L.conv_pool ? 1 : std::max(1, std::min(2, msub));
+    if (L.patch) L.kchunks = 16 * L.Cp / 64 > 0 ? 16 * L.Cp / 64 : 1;  // 4x4 patch x Cp channels
+    else if (L.k == 1) L.kchunks = L.Cp / 64;
     else if (L.Cp >= 64) L.kchunks = 9 * L.Cp / 64;
     else if (L.Cp == 4) L.kchunks = 1;
     else L.kchunks = (9 + 64 / L.Cp - 1) / (64 / L.Cp);
-    L.ksteps = L.Cp == 4 ? 3 : 4;  // the first layer's 9 taps x 4 channels = 36 K fit in 3 MMA K16 steps
-    const int stage = L.nq * 128 * 128 + L.NT * 128;
-    L.stages = std::max(2, std::min(4, (227 * 1024 - 1024) / stage));
-    L.acc_bufs = 2 * L.nq * L.NT <= 512 ? 2 : 1;  // double-buffered accumulator when it fits in TMEM
-    L.tmem_cols = pow2_at_least(L.acc_bufs * L.nq * L.NT);
+    // the first layer's 9 taps x 4 channels = 36 K fit in 3 MMA K16 steps (the patch form uses all 64)
+    L.ksteps = (L.Cp == 4 && !L.patch) ? 3 : 4;
+    const int a_tiles = L.msub * (L.patch ? 1 : L.nq), b_tiles = L.patch ? L.nq : 1;
+    const int stage = a_tiles * 128 * 128 + b_tiles * L.NT * 128;
+    L.stages = std::max(2, std::min(8, (227 * 1024 - 1024) / stage));
+    L.acc_bufs = 2 * L.msub * L.nq * L.NT <= 512 ? 2 : 1;  // double-buffered accumulator when it fits in TMEM
+    L.tmem_cols = pow2_at_least(L.acc_bufs * L.msub * L.nq * L.NT);
     L.H = H;
     L.Ho = L.pool == 1 ? H / 2 : H;
     L.w_off = w_off;
-    L.w_bytes = (size_t)(L.Cout_pad / L.NT) * L.kchunks * L.NT * 128;
+    L.w_bytes = (size_t)(L.Cout_pad / L.NT) * L.kchunks * b_tiles * L.NT * 128;
     w_off += L.w_bytes;
     L.b_off = b_off;
     b_off += L.Cout_pad;
@@ -93,19 +108,25 @@ void build_layers(ffsva_tyolo* m) {
   }
 }
 
-// Pack layer l's weights w[Cout][Cin][k][k] into [N tile][K step][K group 8][NT rows][8 bf16] (the kernel's B
-// tile layout: K-adjacent core matrices NT*16 B apart, 8-row groups 128 B apart).
+// Pack layer l's weights w[Cout][Cin][k][k] into [N tile][K step][B tile][K group 8][NT rows][8 bf16] (the
+// kernel's B tile layout: K-adjacent core matrices NT*16 B apart, 8-row groups 128 B apart). Patch layers have one
+// B tile per pool position q = (a, b): patch pixel (u, v) carries tap (u - a, v - b) when that lies in the 3x3.
 void pack_layer(const Layer& L, const float* w, uint8_t* dst) {
   uint16_t* out = reinterpret_cast<uint16_t*>(dst);
-  const int tiles = L.Cout_pad / L.NT;
+  const int tiles = L.Cout_pad / L.NT, bt = L.patch ? L.nq : 1;
   for (int t = 0; t < tiles; ++t)
     for (int j = 0; j < L.kchunks; ++j)
+      for (int q = 0; q < bt; ++q)
       for (int g = 0; g < 8; ++g)
         for (int nn = 0; nn < L.NT; ++nn)
           for (int e = 0; e < 8; ++e) {
             const int kk = g * 8 + e;
             int tap, c;
-            if (L.k == 1) {
+            if (L.patch) {
+              const int k = j * 64 + kk, px = k / L.Cp, dy = (px >> 2) - (q >> 1), dx = (px & 3) - (q & 1);
+              c = k % L.Cp;
+              tap = (dy >= 0 && dy < 3 && dx >= 0 && dx < 3) ? dy * 3 + dx : 9;
+            } else if (L.k == 1) {
               tap = 4;
               c = j * 64 + kk;
             } else if (L.Cp >= 64) {
@@ -121,7 +142,7 @@ void pack_layer(const Layer& L, const float* w, uint8_t* dst) {
             float v = 0.f;
             if (tap < 9 && c < L.Cin && co < L.Cout)
               v = L.k == 1 ? w[(size_t)co * L.Cin + c] : w[(((size_t)co * L.Cin + c) * 3 + tap / 3) * 3 + tap % 3];
-            const size_t o = (((size_t)(t * L.kchunks + j) * 8 + g) * L.NT + nn) * 8 + e;
+            const size_t o = (((((size_t)t * L.kchunks + j) * bt + q) * 8 + g) * L.NT + nn) * 8 + e;
             out[o] = bf16_bits(v);
           }
 }
@@ -176,6 +197,8 @@ TyConvArgs layer_args(const ffsva_tyolo* m, int l, int n, const __nv_bfloat16* i
   a.stages = L.stages;
   a.tmem_cols = L.tmem_cols;
   a.acc_bufs = L.acc_bufs;
+  a.msub = L.msub;
+  a.patch = L.patch;
   a.grid = m->ctx->num_sms;
   a.leaky = l < 8 ? 1 : 0;
   a.M = n * L.Ho * L.Ho;
