@@ -133,9 +133,24 @@ __device__ __forceinline__ void gather_patch(const TyConvArgs& a, const __nv_bfl
 // per MAC for the wide 13x13 layers). One K-step ring (S stages) runs continuously across tiles; the TMEM
 // accumulators are double buffered when they fit twice, so the epilogue of tile i overlaps tile i + 1's mainloop.
 // Stage = a_tiles A tiles (msub x (patch ? 1 : nq)) + b_tiles B tiles (patch ? nq : 1).
+// cp.async.wait_group with a runtime count (the immediate must be a constant): at most n groups stay pending
+__device__ __forceinline__ void cp_async_wait_n(int n) {
+  switch (n) {
+    case 0: cp_async_wait<0>(); break;
+    case 1: cp_async_wait<1>(); break;
+    case 2: cp_async_wait<2>(); break;
+    case 3: cp_async_wait<3>(); break;
+    case 4: cp_async_wait<4>(); break;
+    case 5: cp_async_wait<5>(); break;
+    case 6: cp_async_wait<6>(); break;
+    default: cp_async_wait<7>(); break;
+  }
+}
+
+template <int MS>
 __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs a) {
   extern __shared__ __align__(1024) uint8_t sm[];
-  const int S = a.stages, nq = a.nq, NT = a.NT, KC = a.kchunks, NB = a.acc_bufs, MS = a.msub;
+  const int S = a.stages, nq = a.nq, NT = a.NT, KC = a.kchunks, NB = a.acc_bufs;
   const int a_per_sub = a.patch ? 1 : nq;
   const int b_tiles = a.patch ? nq : 1;
   const uint32_t stage_a = (uint32_t)(MS * a_per_sub) * kATile;
@@ -171,12 +186,17 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
 
   if (warp < 4) {
     // ---------------- A producers: thread = row r of every 128-row half of the tile
-    const int r = tid;
+    // Up to LAG = S - 1 steps of copies stay in flight per thread; step g is published (cp.async.wait_group, proxy
+    // fence, mbarrier arrive) once step g + LAG has been issued. Deadlock-free: the wait for slot g % S needs the
+    // MMA of step g - S, published after step g - S + LAG = g - 1 was issued.
+    const int r = tid, lag = S - 1;
     int g = 0;  // global K-step counter (continues across tiles)
     for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
-      int n[2] = {0, 0}, oy[2] = {0, 0}, ox[2] = {0, 0};
-      bool rv[2] = {false, false};
+      int n[MS], oy[MS], ox[MS];
+      bool rv[MS];
+#pragma unroll
       for (int i = 0; i < MS; ++i) {
+        n[i] = oy[i] = ox[i] = 0;
         const int m = (t / n_tiles) * rows_per_tile + i * 128 + r;
         rv[i] = m < a.M;
         if (rv[i]) decode_row(a, m, n[i], oy[i], ox[i]);
@@ -184,6 +204,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
       for (int j = 0; j < KC; ++j, ++g) {
         const int s = g % S;
         mbar_wait(empty0 + 8 * s, ((g / S) & 1) ^ 1);
+#pragma unroll
         for (int i = 0; i < MS; ++i) {
           const __nv_bfloat16* img = a.in + (int64_t)n[i] * a.H * a.W * a.Cp;
           const uint32_t base = As0 + (uint32_t)s * stage_a + (uint32_t)(i * a_per_sub) * kATile;
@@ -198,18 +219,16 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
           }
         }
         cp_async_commit();
-        if (g > 0) {  // the previous step's copies have landed: publish them to the tensor core (async proxy)
-          cp_async_wait<1>();
+        if (g >= lag) {  // step g - lag has landed: publish it to the tensor core (async proxy)
+          cp_async_wait_n(lag);
           fence_proxy_async();
-          mbar_arrive(full0 + 8 * ((g - 1) % S));
+          mbar_arrive(full0 + 8 * ((g - lag) % S));
         }
       }
     }
-    if (g > 0) {
-      cp_async_wait<0>();
-      fence_proxy_async();
-      mbar_arrive(full0 + 8 * ((g - 1) % S));
-    }
+    cp_async_wait<0>();
+    fence_proxy_async();
+    for (int h = g - lag < 0 ? 0 : g - lag; h < g; ++h) mbar_arrive(full0 + 8 * (h % S));
   } else if (warp == 4) {
     // ---------------- MMA issue (one thread)
     if (lane == 0) {
@@ -406,7 +425,10 @@ int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT) {
 }
 
 cudaError_t tyolo_configure() {
-  return cudaFuncSetAttribute(tyolo_conv_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+  cudaError_t e = cudaFuncSetAttribute(tyolo_conv_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tyolo_conv_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+  return e;
 }
 
 cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st) {
@@ -414,7 +436,9 @@ cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st) {
   const int tiles = ((a.M + rows - 1) / rows) * a.Cout_tiles;
   const unsigned grid = (unsigned)(tiles < a.grid ? tiles : a.grid);
   const int a_tiles = a.msub * (a.patch ? 1 : a.nq), b_tiles = a.patch ? a.nq : 1;
-  tyolo_conv_kernel<<<grid, kConvThreads, tyolo_conv_smem_bytes(a.stages, a_tiles, b_tiles, a.NT), st>>>(a);
+  const int smem = tyolo_conv_smem_bytes(a.stages, a_tiles, b_tiles, a.NT);
+  if (a.msub == 2) tyolo_conv_kernel<2><<<grid, kConvThreads, smem, st>>>(a);
+  else tyolo_conv_kernel<1><<<grid, kConvThreads, smem, st>>>(a);
   return cudaGetLastError();
 }
 
