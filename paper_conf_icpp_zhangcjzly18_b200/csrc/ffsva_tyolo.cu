@@ -186,10 +186,11 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
 
   if (warp < 4) {
     // ---------------- A producers: thread = row r of every 128-row half of the tile
-    // Up to LAG = S - 1 steps of copies stay in flight per thread; step g is published (cp.async.wait_group, proxy
-    // fence, mbarrier arrive) once step g + LAG has been issued. Deadlock-free: the wait for slot g % S needs the
-    // MMA of step g - S, published after step g - S + LAG = g - 1 was issued.
-    const int r = tid, lag = S - 1;
+    // Up to `lag` (<= S - 1) steps of copies stay in flight per thread; step g is published (cp.async.wait_group,
+    // proxy fence, mbarrier arrive) once step g + lag has been issued. Deadlock-free: the wait for slot g % S needs
+    // the MMA of step g - S, published after step g - S + lag <= g - 1 was issued. lag = S - 1 leaves the MMA no
+    // slack; lag = 1 measured best (profiles/r01/tyolo_ab.md).
+    const int r = tid, lag = a.lag < 1 ? 1 : (a.lag > S - 1 ? S - 1 : a.lag);
     int g = 0;  // global K-step counter (continues across tiles)
     for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
       int n[MS], oy[MS], ox[MS];

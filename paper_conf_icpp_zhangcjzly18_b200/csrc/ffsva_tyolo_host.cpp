@@ -199,6 +199,7 @@ TyConvArgs layer_args(const ffsva_tyolo* m, int l, int n, const __nv_bfloat16* i
   a.acc_bufs = L.acc_bufs;
   a.msub = L.msub;
   a.patch = L.patch;
+  a.lag = env_int("FFSVA_TYOLO_LAG", 1);
   a.grid = m->ctx->num_sms;
   a.leaky = l < 8 ? 1 : 0;
   a.M = n * L.Ho * L.Ho;
