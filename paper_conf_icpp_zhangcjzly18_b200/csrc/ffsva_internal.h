@@ -163,7 +163,6 @@ struct TyConvArgs {
   int32_t msub;              // 128-row halves per tile sharing each weight stage (1 or 2)
   int32_t patch;             // pool layers: A row = the pooled pixel's 4x4 input patch, weights per pool position
   int32_t lag;               // K steps of gathers in flight per producer thread before it publishes (1 .. S-1)
-  int32_t cp_shift;          // log2(Cp)
   int32_t head, target;      // head: count boxes of class `target` scoring > thresh into counts[frame]
   float thresh;
   int32_t* counts;

@@ -43,57 +43,82 @@ __device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr) {
          (2ull << 61);
 }
 
-// The source offset of one K group: pixel (du, dv) relative to the row's reference pixel, channel ch; ok = the
-// group holds real K (tap < 9). Uniform over the rows of a K step, so it is computed once per step per thread.
-struct Piece {
-  int du, dv, ch;
-  bool ok;
-};
+// Output row info packed in one word: valid (bit 31), frame (bits 20-30), oy (10-19), ox (0-9).
+__device__ __forceinline__ uint32_t pack_row(bool v, int n, int oy, int ox) {
+  return (v ? 0x80000000u : 0u) | ((uint32_t)n << 20) | ((uint32_t)oy << 10) | (uint32_t)ox;
+}
 
-// K group c of K step j. Reference pixel of a row: patch mode (2oy - 1, 2ox - 1); pool layers (2oy, 2ox) + the pool
-// position; otherwise (oy, ox). Cp = 1 << cp_shift. For Cp = 4, piece h = 0, 1 is the 8-byte half of the group.
-__device__ __forceinline__ Piece piece_of(const TyConvArgs& a, int j, int c, int h) {
-  Piece p;
-  const int cps = a.cp_shift;
-  if (a.Cp == 4) {
-    const int px = 2 * c + h;  // patch pixel or tap
-    if (a.patch) {
-      p.du = px >> 2;
-      p.dv = px & 3;
-      p.ok = true;
-    } else {
-      p.du = px / 3 - 1;
-      p.dv = px % 3 - 1;
-      p.ok = px < 9;
+// One 16-byte K group c of K step j for one output row (packed info) and pool position q, into the row's slot.
+__device__ __forceinline__ void gather_group(const TyConvArgs& a, uint32_t info, int q, int j, int c, uint32_t dst) {
+  const int H = a.H, W = a.W, Cp = a.Cp;
+  const bool rv = (info >> 31) != 0;
+  const int n = (int)((info >> 20) & 0x7FFu), oy = (int)((info >> 10) & 0x3FFu), ox = (int)(info & 0x3FFu);
+  const __nv_bfloat16* img = a.in + (int64_t)n * H * W * Cp;
+  if (Cp == 4) {  // two 8-byte pixels per K group: patch pixels 2c, 2c+1 or taps 2c, 2c+1
+    int cy = 0, cx = 0;
+    if (!a.patch) {
+      if (a.pool == 1) {
+        cy = 2 * oy + (q >> 1);
+        cx = 2 * ox + (q & 1);
+      } else {
+        cy = oy;
+        cx = ox;
+      }
     }
-    p.ch = 0;
-    return p;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const int p = 2 * c + h;
+      int sy, sx;
+      bool inb;
+      if (a.patch) {
+        sy = 2 * oy - 1 + (p >> 2);
+        sx = 2 * ox - 1 + (p & 3);
+        inb = true;
+      } else {
+        sy = cy + p / 3 - 1;
+        sx = cx + p % 3 - 1;
+        inb = p < 9;
+      }
+      const bool v = rv && inb && sy >= 0 && sy < H && sx >= 0 && sx < W;
+      cp_async8(dst + 8 * h, v ? img + ((int64_t)sy * W + sx) * 4 : a.in, v);
+    }
+    return;
   }
-  const int k = 64 * j + 8 * c;
+  int sy, sx, ch;
+  bool inb = true;
   if (a.patch) {
-    const int px = k >> cps;
-    p.du = px >> 2;
-    p.dv = px & 3;
-    p.ch = k & (a.Cp - 1);
-    p.ok = true;
-    return p;
-  }
-  int t;
-  if (a.ksize == 1) {
-    t = 4;
-    p.ch = k;
-  } else if (a.Cp >= 64) {
-    const int sh = cps - 6;  // K steps per tap = Cp / 64
-    t = j >> sh;
-    p.ch = ((j & ((1 << sh) - 1)) << 6) + 8 * c;
+    const int k = 64 * j + 8 * c, p = k / Cp;
+    ch = k - p * Cp;
+    sy = 2 * oy - 1 + (p >> 2);
+    sx = 2 * ox - 1 + (p & 3);
   } else {
-    t = k >> cps;
-    p.ch = k & (a.Cp - 1);
+    int cy, cx;
+    if (a.pool == 1) {
+      cy = 2 * oy + (q >> 1);
+      cx = 2 * ox + (q & 1);
+    } else {
+      cy = oy;
+      cx = ox;
+    }
+    int t;
+    if (a.ksize == 1) {
+      t = 4;
+      ch = 64 * j + 8 * c;
+    } else if (Cp >= 64) {
+      const int cpt = Cp >> 6;
+      t = j / cpt;
+      ch = ((j - t * cpt) << 6) + 8 * c;
+    } else {
+      const int k = 64 * j + 8 * c;
+      t = k / Cp;
+      ch = k - t * Cp;
+      inb = t < 9;
+    }
+    sy = cy + t / 3 - 1;
+    sx = cx + t % 3 - 1;
   }
-  p.ok = t < 9;
-  p.du = t / 3 - 1;
-  p.dv = t % 3 - 1;
-  return p;
+  const bool v = rv && inb && sy >= 0 && sy < H && sx >= 0 && sx < W;
+  cp_async16(dst, v ? img + ((int64_t)sy * W + sx) * Cp + ch : a.in, v);
 }
 
 // Decode output row m of the layer into (frame, oy, ox).
@@ -103,27 +128,6 @@ __device__ __forceinline__ void decode_row(const TyConvArgs& a, int m, int& n, i
   const int rem = m - n * hw;
   oy = rem / a.Wo;
   ox = rem - oy * a.Wo;
-}
-
-// Row state per producer thread and row: pixel index of the reference pixel ((n * H + ry) * W + rx; may lie one
-// pixel outside the image) and (valid, ry + 1, rx + 1) packed as 1 | 15 | 16 bits.
-__device__ __forceinline__ void row_ref(const TyConvArgs& a, int m, int& pix, uint32_t& yx) {
-  int n = 0, oy = 0, ox = 0;
-  const bool v = m < a.M;
-  if (v) decode_row(a, m, n, oy, ox);
-  const int sc = a.pool == 1 ? 2 : 1, off = a.patch ? -1 : 0;
-  const int ry = sc * oy + off, rx = sc * ox + off;
-  pix = (n * a.H + ry) * a.W + rx;
-  yx = (v ? 0x80000000u : 0u) | ((uint32_t)(ry + 1) << 16) | (uint32_t)(rx + 1);
-}
-
-__device__ __forceinline__ void gather_piece(const TyConvArgs& a, int pix, uint32_t yx, const Piece& p, int qa, int qb,
-                                             uint32_t dst, bool half) {
-  const int sy = (int)((yx >> 16) & 0x7FFFu) - 1 + p.du + qa, sx = (int)(yx & 0xFFFFu) - 1 + p.dv + qb;
-  const bool v = (yx >> 31) && p.ok && (unsigned)sy < (unsigned)a.H && (unsigned)sx < (unsigned)a.W;
-  const __nv_bfloat16* src = v ? a.in + (int64_t)(pix + (p.du + qa) * a.W + p.dv + qb) * a.Cp + p.ch : a.in;
-  if (half) cp_async8(dst, src, v);
-  else cp_async16(dst, src, v);
 }
 
 // Patch mode (pool layers with few input channels): the A row of pooled pixel (oy, ox) is its 4x4 input patch
@@ -198,28 +202,22 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
     const int a_tiles_sub = a.patch ? 1 : nq;
     int g = 0;  // global K-step counter (continues across tiles)
     for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
-      int pix[MS * 8];
-      uint32_t yx[MS * 8];
+      uint32_t info[MS * 8];
 #pragma unroll
-      for (int i = 0; i < MS * 8; ++i)
-        row_ref(a, (t / n_tiles) * rows_per_tile + (i >> 3) * 128 + (i & 7) * 16 + r0, pix[i], yx[i]);
+      for (int i = 0; i < MS * 8; ++i) {
+        const int m = (t / n_tiles) * rows_per_tile + (i >> 3) * 128 + (i & 7) * 16 + r0;
+        int n = 0, oy = 0, ox = 0;
+        if (m < a.M) decode_row(a, m, n, oy, ox);
+        info[i] = pack_row(m < a.M, n, oy, ox);
+      }
       for (int j = 0; j < KC; ++j, ++g) {
         const int s = g % S;
-        const Piece p0 = piece_of(a, j, c, 0), p1 = piece_of(a, j, c, 1);
         mbar_wait(empty0 + 8 * s, ((g / S) & 1) ^ 1);
-        const uint32_t stage = As0 + (uint32_t)s * stage_a;
-        for (int q = 0; q < a_tiles_sub; ++q) {
-          const int qa = a.patch ? 0 : (q >> 1), qb = a.patch ? 0 : (q & 1);
 #pragma unroll
-          for (int i = 0; i < MS * 8; ++i) {
-            const uint32_t dst = stage + (uint32_t)((i >> 3) * a_tiles_sub + q) * kATile + sw128_off((i & 7) * 16 + r0, c);
-            if (a.Cp == 4) {
-              gather_piece(a, pix[i], yx[i], p0, qa, qb, dst, true);
-              gather_piece(a, pix[i], yx[i], p1, qa, qb, dst + 8, true);
-            } else {
-              gather_piece(a, pix[i], yx[i], p0, qa, qb, dst, false);
-            }
-          }
+        for (int i = 0; i < MS * 8; ++i) {
+          const int R = (i & 7) * 16 + r0;
+          const uint32_t base = As0 + (uint32_t)s * stage_a + (uint32_t)((i >> 3) * a_tiles_sub) * kATile + sw128_off(R, c);
+          for (int q = 0; q < a_tiles_sub; ++q) gather_group(a, info[i], q, j, c, base + (uint32_t)q * kATile);
         }
         cp_async_commit();
         if (g >= lag) {  // step g - lag has landed: publish it to the tensor core (async proxy)
