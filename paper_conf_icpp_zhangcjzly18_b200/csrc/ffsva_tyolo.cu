@@ -13,10 +13,10 @@
 //     N = output channels (tile NT <= 256); K = taps x input channels, staged 64 bf16 (128 B) per pipeline step.
 //   * Pooling is folded into the MMA like the SNM: for a pool layer the four 2x2 positions are four accumulator
 //     chains in four TMEM column groups, so the epilogue max-pools in registers (bias and leaky ReLU commute
-//     with max and are applied once after it). The 2x2/1 pool of layer 6 (Q30) is a small separate kernel.
+//     with max and are applied once after it). The 2x2/1 pool of layer 6 uses the same four chains with the
+//     border positions excluded (Q30).
 //   * A operands are gathered (im2col on the fly) by 128 producer threads with cp.async zero-fill (padding and
-//     K padding are zeros), eight threads per 128-byte row, straight into the UMMA K-major SWIZZLE_128B layout;
-//     B operands
+//     K padding are zeros), written straight into the UMMA K-major no-swizzle core-matrix layout; B operands
 //     (weights, pre-packed on the host in exactly that layout per (N tile, K step)) arrive by one bulk copy per
 //     step. A 2- or 4-stage mbarrier ring overlaps copies with the MMAs, issued by one thread.
 //   * The 1x1 head (1024 -> 125) writes its fp32 outputs and counts, per row, the boxes whose score exceeds the
@@ -32,93 +32,65 @@ using namespace ptx;
 constexpr int kConvThreads = 320;  // warps 0-3: A gather, 4: TMEM + MMA issue, 5: B copies, 6-9: epilogue
 constexpr int kATile = 128 * 128;  // one stage of A for one chain: 128 rows x 64 bf16
 
-// A tiles use the UMMA K-major SWIZZLE_128B layout: row r (64 bf16 = 128 B) at r * 128, its 16-byte K group c at
-// position c ^ (r & 7); 8-row atoms of 1024 B (SBO), tiles 1024-B aligned. Eight consecutive producer threads fill
-// one row (one 128-byte line of the source pixel), so every warp-wide cp.async reads four full lines and writes
-// 512 contiguous, conflict-free bytes of shared memory.
-__device__ __forceinline__ uint32_t sw128_off(int r, int c) { return (uint32_t)(r * 128 + ((c ^ (r & 7)) << 4)); }
-
-__device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr) {
-  return (uint64_t)((saddr >> 4) & 0x3FFFu) | (1ull << 16) | ((uint64_t)(1024 >> 4) << 32) | (1ull << 46) |
-         (2ull << 61);
+// byte offset of (K group g of 8 bf16, row r) in a 128-row K-major no-swizzle tile: core matrices of 8 rows x 16 B,
+// K-adjacent core matrices 2048 B apart (LBO), 8-row groups 128 B apart (SBO)
+__device__ __forceinline__ uint32_t a_off(int g, int r) {
+  return (uint32_t)(g * 2048 + (r >> 3) * 128 + (r & 7) * 16);
 }
 
-// Output row info packed in one word: valid (bit 31), frame (bits 20-30), oy (10-19), ox (0-9).
-__device__ __forceinline__ uint32_t pack_row(bool v, int n, int oy, int ox) {
-  return (v ? 0x80000000u : 0u) | ((uint32_t)n << 20) | ((uint32_t)oy << 10) | (uint32_t)ox;
-}
-
-// One 16-byte K group c of K step j for one output row (packed info) and pool position q, into the row's slot.
-__device__ __forceinline__ void gather_group(const TyConvArgs& a, uint32_t info, int q, int j, int c, uint32_t dst) {
+// The A rows of one K step (chunk j) for output row r whose conv pixel is (cy, cx).
+__device__ __forceinline__ void gather(const TyConvArgs& a, const __nv_bfloat16* img, bool rv, int cy, int cx, int j,
+                                       uint32_t dst, int r) {
   const int H = a.H, W = a.W, Cp = a.Cp;
-  const bool rv = (info >> 31) != 0;
-  const int n = (int)((info >> 20) & 0x7FFu), oy = (int)((info >> 10) & 0x3FFu), ox = (int)(info & 0x3FFu);
-  const __nv_bfloat16* img = a.in + (int64_t)n * H * W * Cp;
-  if (Cp == 4) {  // two 8-byte pixels per K group: patch pixels 2c, 2c+1 or taps 2c, 2c+1
-    int cy = 0, cx = 0;
-    if (!a.patch) {
-      if (a.pool == 1) {
-        cy = 2 * oy + (q >> 1);
-        cx = 2 * ox + (q & 1);
-      } else {
-        cy = oy;
-        cx = ox;
-      }
-    }
-#pragma unroll
-    for (int h = 0; h < 2; ++h) {
-      const int p = 2 * c + h;
-      int sy, sx;
-      bool inb;
-      if (a.patch) {
-        sy = 2 * oy - 1 + (p >> 2);
-        sx = 2 * ox - 1 + (p & 3);
-        inb = true;
-      } else {
-        sy = cy + p / 3 - 1;
-        sx = cx + p % 3 - 1;
-        inb = p < 9;
-      }
-      const bool v = rv && inb && sy >= 0 && sy < H && sx >= 0 && sx < W;
-      cp_async8(dst + 8 * h, v ? img + ((int64_t)sy * W + sx) * 4 : a.in, v);
-    }
-    return;
-  }
-  int sy, sx, ch;
-  bool inb = true;
-  if (a.patch) {
-    const int k = 64 * j + 8 * c, p = k / Cp;
-    ch = k - p * Cp;
-    sy = 2 * oy - 1 + (p >> 2);
-    sx = 2 * ox - 1 + (p & 3);
-  } else {
-    int cy, cx;
-    if (a.pool == 1) {
-      cy = 2 * oy + (q >> 1);
-      cx = 2 * ox + (q & 1);
-    } else {
-      cy = oy;
-      cx = ox;
-    }
-    int t;
-    if (a.ksize == 1) {
-      t = 4;
-      ch = 64 * j + 8 * c;
-    } else if (Cp >= 64) {
+  if (Cp >= 64) {
+    int t, c0;
+    if (a.ksize == 3) {
       const int cpt = Cp >> 6;
       t = j / cpt;
-      ch = ((j - t * cpt) << 6) + 8 * c;
+      c0 = (j - t * cpt) << 6;
     } else {
-      const int k = 64 * j + 8 * c;
-      t = k / Cp;
-      ch = k - t * Cp;
-      inb = t < 9;
+      t = 4;
+      c0 = j << 6;
     }
-    sy = cy + t / 3 - 1;
-    sx = cx + t % 3 - 1;
+    const int sy = cy + t / 3 - 1, sx = cx + t % 3 - 1;
+    const bool v = rv && sy >= 0 && sy < H && sx >= 0 && sx < W;
+    const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * Cp + c0 : a.in;
+#pragma unroll
+    for (int g = 0; g < 8; ++g) cp_async16(dst + a_off(g, r), src + 8 * g, v);
+  } else if (Cp >= 16) {  // 16 or 32 channels: 4 or 2 taps per K step
+    const int tpc = 64 / Cp, upt = Cp >> 3;
+    for (int i = 0; i < tpc; ++i) {
+      const int t = j * tpc + i;
+      const int sy = cy + t / 3 - 1, sx = cx + t % 3 - 1;
+      const bool v = rv && t < 9 && sy >= 0 && sy < H && sx >= 0 && sx < W;
+      const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * Cp : a.in;
+      for (int u = 0; u < upt; ++u) cp_async16(dst + a_off(i * upt + u, r), src + 8 * u, v);
+    }
+  } else {  // 4 channels (RGB + zero): two taps per 16-byte K group, all nine taps in one step
+#pragma unroll
+    for (int g = 0; g < 8; ++g)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int t = 2 * g + h;
+        const int sy = cy + t / 3 - 1, sx = cx + t % 3 - 1;
+        const bool v = rv && t < 9 && sy >= 0 && sy < H && sx >= 0 && sx < W;
+        const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * 4 : a.in;
+        cp_async8(dst + a_off(g, r) + 8 * h, src, v);
+      }
   }
-  const bool v = rv && inb && sy >= 0 && sy < H && sx >= 0 && sx < W;
-  cp_async16(dst, v ? img + ((int64_t)sy * W + sx) * Cp + ch : a.in, v);
+}
+
+__device__ __forceinline__ void conv_pixel(const TyConvArgs& a, int oy, int ox, int q, int& cy, int& cx) {
+  if (a.pool == 1) {
+    cy = 2 * oy + (q >> 1);
+    cx = 2 * ox + (q & 1);
+  } else if (a.pool == 2) {
+    cy = oy + (q >> 1);
+    cx = ox + (q & 1);
+  } else {
+    cy = oy;
+    cx = ox;
+  }
 }
 
 // Decode output row m of the layer into (frame, oy, ox).
@@ -130,10 +102,31 @@ __device__ __forceinline__ void decode_row(const TyConvArgs& a, int m, int& n, i
   ox = rem - oy * a.Wo;
 }
 
-// Patch mode (pool layers with few input channels): the A row of pooled pixel (oy, ox) is its 4x4 input patch
+// Patch gather (pool layers with few input channels): the A row of pooled pixel (oy, ox) is its 4x4 input patch
 // (rows 2oy-1 .. 2oy+2, columns 2ox-1 .. 2ox+2) x Cp channels, pixel-major; K step j holds 64 of its values. The
 // four pool positions then differ only in their weights (the 3x3 kernel placed at offset (a, b) of the 4x4 patch),
 // so one A tile feeds all four accumulator chains.
+__device__ __forceinline__ void gather_patch(const TyConvArgs& a, const __nv_bfloat16* img, bool rv, int oy, int ox,
+                                             int j, uint32_t dst, int r) {
+  const int H = a.H, W = a.W, Cp = a.Cp;
+  if (Cp == 4) {  // all 16 patch pixels in one K step, two pixels per 16-byte K group
+#pragma unroll
+    for (int p = 0; p < 16; ++p) {
+      const int sy = 2 * oy - 1 + (p >> 2), sx = 2 * ox - 1 + (p & 3);
+      const bool v = rv && sy >= 0 && sy < H && sx >= 0 && sx < W;
+      cp_async8(dst + a_off(p >> 1, r) + 8 * (p & 1), v ? img + ((int64_t)sy * W + sx) * 4 : a.in, v);
+    }
+  } else {  // Cp = 8 * upp channels: 64 / Cp pixels per K step, upp 16-byte units each
+    const int ppc = 64 / Cp, upp = Cp >> 3;
+    for (int pl = 0; pl < ppc; ++pl) {
+      const int p = j * ppc + pl;
+      const int sy = 2 * oy - 1 + (p >> 2), sx = 2 * ox - 1 + (p & 3);
+      const bool v = rv && sy >= 0 && sy < H && sx >= 0 && sx < W;
+      const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * Cp : a.in;
+      for (int u = 0; u < upp; ++u) cp_async16(dst + a_off(pl * upp + u, r), src + 8 * u, v);
+    }
+  }
+}
 
 // Persistent, warp-specialised: each CTA walks tiles t = blockIdx.x, + gridDim.x, ... A tile = msub x 128 output
 // rows x NT channels (msub = 2 shares every weight stage between two 128-row halves: half the L2 weight traffic
@@ -197,27 +190,34 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
     // proxy fence, mbarrier arrive) once step g + lag has been issued. Deadlock-free: the wait for slot g % S needs
     // the MMA of step g - S, published after step g - S + lag <= g - 1 was issued. lag = S - 1 leaves the MMA no
     // slack; lag = 1 measured best (profiles/r01/tyolo_ab.md).
-    const int lag = a.lag < 1 ? 1 : (a.lag > S - 1 ? S - 1 : a.lag);
-    const int c = tid & 7, r0 = tid >> 3;  // this thread's K group, and its first row (rows r0 + 16 i)
-    const int a_tiles_sub = a.patch ? 1 : nq;
+    const int r = tid, lag = a.lag < 1 ? 1 : (a.lag > S - 1 ? S - 1 : a.lag);
     int g = 0;  // global K-step counter (continues across tiles)
     for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
-      uint32_t info[MS * 8];
+      int n[MS], oy[MS], ox[MS];
+      bool rv[MS];
 #pragma unroll
-      for (int i = 0; i < MS * 8; ++i) {
-        const int m = (t / n_tiles) * rows_per_tile + (i >> 3) * 128 + (i & 7) * 16 + r0;
-        int n = 0, oy = 0, ox = 0;
-        if (m < a.M) decode_row(a, m, n, oy, ox);
-        info[i] = pack_row(m < a.M, n, oy, ox);
+      for (int i = 0; i < MS; ++i) {
+        n[i] = oy[i] = ox[i] = 0;
+        const int m = (t / n_tiles) * rows_per_tile + i * 128 + r;
+        rv[i] = m < a.M;
+        if (rv[i]) decode_row(a, m, n[i], oy[i], ox[i]);
       }
       for (int j = 0; j < KC; ++j, ++g) {
         const int s = g % S;
         mbar_wait(empty0 + 8 * s, ((g / S) & 1) ^ 1);
 #pragma unroll
-        for (int i = 0; i < MS * 8; ++i) {
-          const int R = (i & 7) * 16 + r0;
-          const uint32_t base = As0 + (uint32_t)s * stage_a + (uint32_t)((i >> 3) * a_tiles_sub) * kATile + sw128_off(R, c);
-          for (int q = 0; q < a_tiles_sub; ++q) gather_group(a, info[i], q, j, c, base + (uint32_t)q * kATile);
+        for (int i = 0; i < MS; ++i) {
+          const __nv_bfloat16* img = a.in + (int64_t)n[i] * a.H * a.W * a.Cp;
+          const uint32_t base = As0 + (uint32_t)s * stage_a + (uint32_t)(i * a_per_sub) * kATile;
+          if (a.patch) {
+            gather_patch(a, img, rv[i], oy[i], ox[i], j, base, r);
+          } else {
+            for (int q = 0; q < nq; ++q) {
+              int cy, cx;
+              conv_pixel(a, oy[i], ox[i], q, cy, cx);
+              gather(a, img, rv[i], cy, cx, j, base + (uint32_t)q * kATile, r);
+            }
+          }
         }
         cp_async_commit();
         if (g >= lag) {  // step g - lag has landed: publish it to the tensor core (async proxy)
@@ -249,7 +249,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
               const uint32_t at = As0 + (uint32_t)s * stage_a + (uint32_t)(i * a_per_sub + (a.patch ? 0 : q)) * kATile;
               const uint32_t bt = Bs0 + (uint32_t)s * stage_b + (uint32_t)(a.patch ? q : 0) * b_tile;
               for (int ks = 0; ks < a.ksteps; ++ks) {
-                const uint64_t ad = umma_desc_sw128(at + (uint32_t)ks * 32u);
+                const uint64_t ad = umma_desc(at + (uint32_t)ks * 4096u, 2048, 128);
                 const uint64_t bd = umma_desc(bt + (uint32_t)(ks * 2 * NT * 16), NT * 16, 128);
                 mma_bf16(acc + (uint32_t)((i * nq + q) * NT), ad, bd, idesc, (j > 0 || ks > 0) ? 1u : 0u);
               }
