@@ -170,7 +170,8 @@ struct TyConvArgs {
 cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st);
 cudaError_t launch_tyolo_pool_s1(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C,
                                  cudaStream_t st);
-cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, __nv_bfloat16* out, cudaStream_t st);
+cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int32_t max_row_bytes,
+                                __nv_bfloat16* out, cudaStream_t st);
 int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT);
 cudaError_t tyolo_configure();
 

@@ -387,36 +387,50 @@ __global__ void tyolo_pool_s1_kernel(const __nv_bfloat16* in, __nv_bfloat16* out
   *reinterpret_cast<uint4*>(out + p * C + 8 * cg) = o;
 }
 
-// Q28 resize of each raw RGB8 frame to 416x416, x = v / 256 (Q29) as bf16 NHWC with a zero 4th channel.
-__global__ void tyolo_resize_kernel(const TyFrame* frames, int32_t n, int32_t D, __nv_bfloat16* out) {
-  const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const int64_t per = (int64_t)D * D;
-  if (idx >= per * n) return;
-  const int f = (int)(idx / per);
-  const int p = (int)(idx - (int64_t)f * per);
-  const int oy = p / D, ox = p - oy * D;
+// Q28 resize of each raw RGB8 frame to 416x416, x = v / 256 (Q29) as bf16 NHWC with a zero 4th channel. One CTA per
+// (frame, output row): the row's source rows are staged in shared memory with 16-byte loads (when the frame's rows
+// are 16-byte aligned), then each thread box-sums its output pixels from shared memory.
+constexpr int kResizeThreads = 256;
+constexpr int kResizeMaxRows = 4;  // source rows per output row: ceil(H / 416) + 1 <= 4 for H <= 1248
+
+__global__ void __launch_bounds__(kResizeThreads) tyolo_resize_kernel(const TyFrame* frames, int32_t D,
+                                                                     __nv_bfloat16* out) {
+  extern __shared__ __align__(16) uint8_t rows_sm[];
+  const int f = blockIdx.x / D, oy = blockIdx.x - f * D;
   const TyFrame fr = frames[f];
   int y0 = (int)(((int64_t)oy * fr.H) / D), y1 = (int)(((int64_t)(oy + 1) * fr.H) / D);
-  int x0 = (int)(((int64_t)ox * fr.W) / D), x1 = (int)(((int64_t)(ox + 1) * fr.W) / D);
   if (y1 <= y0) y1 = y0 + 1;
-  if (x1 <= x0) x1 = x0 + 1;
-  uint32_t s0 = 0, s1 = 0, s2 = 0;
-  for (int y = y0; y < y1; ++y) {
-    const uint8_t* row = fr.pixels + (int64_t)y * fr.pitch + 3 * x0;
-    for (int x = 0; x < x1 - x0; ++x) {
-      s0 += row[3 * x];
-      s1 += row[3 * x + 1];
-      s2 += row[3 * x + 2];
+  const int nrows = y1 - y0, rb = 3 * fr.W;
+  const int rb16 = (rb + 15) & ~15;
+  const bool staged = nrows <= kResizeMaxRows && ((fr.pitch & 15) == 0) && (((uintptr_t)fr.pixels & 15) == 0);
+  if (staged) {
+    const int chunks = rb16 >> 4;
+    for (int k = threadIdx.x; k < nrows * chunks; k += kResizeThreads) {
+      const int r = k / chunks, c = k - r * chunks;
+      reinterpret_cast<uint4*>(rows_sm + r * rb16)[c] =
+          __ldg(reinterpret_cast<const uint4*>(fr.pixels + (int64_t)(y0 + r) * fr.pitch) + c);
     }
+    __syncthreads();
   }
-  const uint32_t nn = (uint32_t)((y1 - y0) * (x1 - x0));
   const float inv = 1.f / 256.f;
-  const float v0 = (float)((s0 + nn / 2) / nn) * inv, v1 = (float)((s1 + nn / 2) / nn) * inv,
-              v2 = (float)((s2 + nn / 2) / nn) * inv;
-  uint2 w;
-  w.x = pack_bf16(v0, v1);
-  w.y = pack_bf16(v2, 0.f);
-  *reinterpret_cast<uint2*>(out + idx * 4) = w;
+  for (int ox = threadIdx.x; ox < D; ox += kResizeThreads) {
+    int x0 = (int)(((int64_t)ox * fr.W) / D), x1 = (int)(((int64_t)(ox + 1) * fr.W) / D);
+    if (x1 <= x0) x1 = x0 + 1;
+    uint32_t s0 = 0, s1 = 0, s2 = 0;
+    for (int r = 0; r < nrows; ++r) {
+      const uint8_t* row = staged ? rows_sm + r * rb16 : fr.pixels + (int64_t)(y0 + r) * fr.pitch;
+      for (int x = x0; x < x1; ++x) {
+        s0 += row[3 * x];
+        s1 += row[3 * x + 1];
+        s2 += row[3 * x + 2];
+      }
+    }
+    const uint32_t nn = (uint32_t)(nrows * (x1 - x0));
+    uint2 w;
+    w.x = pack_bf16((float)((s0 + nn / 2) / nn) * inv, (float)((s1 + nn / 2) / nn) * inv);
+    w.y = pack_bf16((float)((s2 + nn / 2) / nn) * inv, 0.f);
+    *reinterpret_cast<uint2*>(out + (((int64_t)f * D + oy) * D + ox) * 4) = w;
+  }
 }
 
 }  // namespace
@@ -450,9 +464,16 @@ cudaError_t launch_tyolo_pool_s1(const __nv_bfloat16* in, __nv_bfloat16* out, in
   return cudaGetLastError();
 }
 
-cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, __nv_bfloat16* out, cudaStream_t st) {
-  const int64_t total = (int64_t)n * D * D;
-  tyolo_resize_kernel<<<(unsigned)((total + 255) / 256), 256, 0, st>>>(frames, n, D, out);
+cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int32_t max_row_bytes,
+                                __nv_bfloat16* out, cudaStream_t st) {
+  const int smem = kResizeMaxRows * ((max_row_bytes + 15) & ~15);
+  static int configured = 0;
+  if (smem > 48 * 1024 && smem > configured) {
+    cudaError_t e = cudaFuncSetAttribute(tyolo_resize_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    configured = smem;
+  }
+  tyolo_resize_kernel<<<(unsigned)(n * D), kResizeThreads, smem, st>>>(frames, D, out);
   return cudaGetLastError();
 }
 

@@ -69,8 +69,10 @@ def _round_bf16_fast(x):
     return u.astype(np.uint32).view(np.float32).astype(np.float64)
 
 
-@pytest.mark.parametrize("W,H", [(640, 360), (1280, 720), (416, 416)])
+@pytest.mark.parametrize("W,H", [(640, 360), (1280, 720), (416, 416), (1920, 1080), (641, 361), (3840, 2160)])
 def test_resize_input_bit_exact(env, W, H):
+    """Row-staged path (16-byte aligned rows, <= 4 source rows per output row) and the direct path (641-wide
+    rows are unaligned; 2160 rows need 5-6 source rows per output row)."""
     ff, ctx, dev, ty, params = env
     st, host, d, items = _frames(ctx, dev, W, H, 3)
     got = ty.layer_output(items, -1)

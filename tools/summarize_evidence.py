@@ -27,9 +27,11 @@ OUT = os.path.join(ROOT, "gpurun_out")
 
 
 def short(name):
-    for k in ("sdd", "compact", "snm"):
+    for k, v in (("tyolo_conv", "K5 tyolo_conv"), ("tyolo_resize", "K5 tyolo_resize"), ("tyolo_pool", "K5 tyolo_pool_s1"),
+                 ("sdd_prev", "K2 sdd_prev"), ("ref_update", "K2b ref_update"), ("sdd", "K1 sdd"),
+                 ("compact", "K3 compact"), ("snm", "K4 snm")):
         if k in name:
-            return {"sdd": "K1 sdd", "compact": "K3 compact", "snm": "K4 snm"}[k]
+            return v
     return name[:40]
 
 
@@ -59,7 +61,8 @@ def main():
     rnd = sys.argv[1] if len(sys.argv) > 1 else "r01"
     dst = os.path.join(ROOT, "profiles", rnd)
     os.makedirs(dst, exist_ok=True)
-    for f in ["bench.json", "bench.err", "pytest_gpu.log", "smoke.log", "nvidia-smi.txt"] + \
+    for f in ["bench.json", "bench.err", "bench_tyolo.json", "tyolo_profile.json", "pytest_gpu.log", "smoke.log",
+              "nvidia-smi.txt"] + \
             [os.path.basename(p) for p in glob.glob(os.path.join(OUT, "sanitize_*.log"))]:
         p = os.path.join(OUT, f)
         if os.path.exists(p):
