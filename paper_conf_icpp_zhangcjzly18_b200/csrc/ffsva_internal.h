@@ -68,6 +68,7 @@ struct SddArgs {
   const int32_t* xbounds;    // [sdd_w + 1] floor(i*uni_W/sdd_w) for frames of width uni_W, or nullptr
   const int32_t* ybounds;    // [sdd_h + 1] floor(i*uni_H/sdd_h) for frames of height uni_H, or nullptr
   int32_t uni_W, uni_H;
+  int32_t cellw;             // widest 100-grid cell of uni_W-wide frames, ceil(uni_W / sdd_w) (0 if mixed)
 };
 cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st);
 size_t sdd_smem_bytes(int max_chunks, int sdd_w);

@@ -482,6 +482,7 @@ SddArgs make_sdd_args(Batch* b, int32_t i0, int32_t cnt) {
   sa.stage_bytes = b->stage_bytes;
   sa.uni_W = b->uni_W;
   sa.uni_H = b->uni_H;
+  sa.cellw = b->uni_W > 0 ? (b->uni_W + b->sdd_w - 1) / b->sdd_w : 0;
   sa.xbounds = b->uni_W > 0 ? b->d_xb : nullptr;
   sa.ybounds = b->uni_H > 0 ? b->d_yb : nullptr;
   return sa;

@@ -131,6 +131,28 @@ __device__ __forceinline__ void cell_sum3_packed(const uint32_t* cw, int u0, int
   c2 = (S1 & 0xFFFFu) + (S2 >> 16);
 }
 
+// floor(a / n) for a < 2^31 and a quotient below 2^16 (box means: <= 255), without the ~20-instruction integer
+// division: the float estimate (relative error < 2^-21, so off by at most one) and one remainder correction.
+__device__ __forceinline__ uint32_t udiv_small(uint32_t a, uint32_t n) {
+  uint32_t q = __float2uint_rz(__uint2float_rn(a) * __frcp_rn(__uint2float_rn(n)));
+  const int r = (int)(a - q * n);
+  if (r < 0) --q;
+  else if (r >= (int)n) ++q;
+  return q;
+}
+
+// Round-half-up mean (s + n/2) / n of a box (C1).
+__device__ __forceinline__ uint32_t box_mean(uint32_t s, uint32_t n) { return udiv_small(s + (n >> 1), n); }
+
+// Cell sum of one channel with the unroll matched to the frame's widest cell (cellw).
+__device__ __forceinline__ uint32_t cell_sum_w(const uint16_t* col, int x0, int x1, int cellw) {
+  if (cellw <= 8) return cell_sum_n<8>(col, x0, x1);
+  if (cellw <= 13) return cell_sum_n<13>(col, x0, x1);
+  if (cellw <= 16) return cell_sum_n<16>(col, x0, x1);
+  if (cellw <= 20) return cell_sum_n<20>(col, x0, x1);
+  return cell_sum(col, x0, x1);
+}
+
 // Store the 16 column sums of chunk c (u16 each) for one 100-grid row.
 __device__ __forceinline__ void store_colsum(uint32_t* colw, int c, const uint32_t (&a)[8]) {
   uint4 lo, hi;
@@ -229,7 +251,7 @@ __global__ void __launch_bounds__(512) sdd_kernel(SddArgs a) {
     for (int x = x0; x < x1; ++x) s += col[3 * x];
     cell[o] = s;
     const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)(sub ? rows - split : split);
-    const uint32_t d = (s + (n >> 1)) / n;
+    const uint32_t d = box_mean(s, n);
     const int yrow = 2 * band + sub;
     if (kD100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)yrow * row3 + r] = (uint8_t)d;
     const int diff = (int)d - (int)__ldg(fd.ref + (int64_t)yrow * row3 + r);
@@ -246,7 +268,7 @@ __global__ void __launch_bounds__(512) sdd_kernel(SddArgs a) {
                        cell[row3 + 6 * cx + 3 + ch];
     const uint32_t n = (uint32_t)(xb[2 * cx + 2] - xb[2 * cx]) * (uint32_t)rows;
     const int64_t slot = a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f;
-    a.d50[slot * a.d50_stride + (int64_t)band * half3 + o] = (uint8_t)((s + (n >> 1)) / n);
+    a.d50[slot * a.d50_stride + (int64_t)band * half3 + o] = (uint8_t)box_mean(s, n);
   }
   ssd_commit(ssd_local, red, a, f, fd.slot, band == 0);
 }
@@ -304,17 +326,18 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   __shared__ __align__(8) uint64_t bar_pair;   // (even CTA) the odd CTA's 2-cell sums have landed
   __shared__ uint32_t red[kBulkThreads / 32];
   const int sdd_w = a.sdd_w, sdd_h = a.sdd_h;
-  const int f = blockIdx.x / sdd_h;
-  const int r = blockIdx.x - f * sdd_h;  // 100-grid row; the cluster pairs rows 2b and 2b+1
+  const int f = blockIdx.y;              // frame (launches of > 65535 frames are split on the host)
+  const int r = blockIdx.x;              // 100-grid row; the cluster pairs rows 2b and 2b+1
   const uint32_t rank = (uint32_t)r & 1u;
   const FrameDesc fd = a.frames[f];
   const int W = fd.W, H = fd.H;
   const int rb16 = (3 * W + 15) & ~15;
   const int nchunk = rb16 >> 4;
-  // row boundaries in 32-bit arithmetic (H <= 65535 and sdd_h <= 4096 are validated, so r*H < 2^28); no
-  // dependent global load may sit in front of the bulk-copy issue
-  const int y0 = (int)(((uint32_t)r * (uint32_t)H) / (uint32_t)sdd_h);
-  const int y1 = (int)(((uint32_t)(r + 1) * (uint32_t)H) / (uint32_t)sdd_h);
+  // row boundaries: the host table when the batch shares H, else 32-bit division (H <= 65535, sdd_h <= 4096 are
+  // validated, so r*H < 2^28)
+  const bool ytab = a.ybounds && H == a.uni_H;
+  const int y0 = ytab ? __ldg(a.ybounds + r) : (int)(((uint32_t)r * (uint32_t)H) / (uint32_t)sdd_h);
+  const int y1 = ytab ? __ldg(a.ybounds + r + 1) : (int)(((uint32_t)(r + 1) * (uint32_t)H) / (uint32_t)sdd_h);
   const int rows = y1 - y0;
   const int half3 = 3 * (sdd_w >> 1);
   uint32_t* cell = reinterpret_cast<uint32_t*>(smem + a.stage_bytes);  // [3*sdd_w]
@@ -342,7 +365,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   // publish the peer's mbarrier before any remote st.async (relaxed: no memory fence needed beyond
   // fence.mbarrier_init); the matching wait comes right before the DSMEM exchange
   asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
-  fill_xbounds(xb, W, sdd_w);
+  if (a.xbounds && W == a.uni_W) {
+    for (int i = threadIdx.x; i <= sdd_w; i += blockDim.x) xb[i] = __ldg(a.xbounds + i);
+  } else {
+    fill_xbounds(xb, W, sdd_w);
+  }
   __syncthreads();
   mbar_wait_parity(bar_d, 0);
 
@@ -372,20 +399,16 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
 
   // ---- 100-grid cells of this row (one thread per cell and channel): D100, SSD vs R
   const int row3 = 3 * sdd_w;
-  const int cellw = (W + sdd_w - 1) / sdd_w;  // widest cell of this frame (uniform over the CTA)
+  const int cellw = W == a.uni_W ? a.cellw : (W + sdd_w - 1) / sdd_w;  // widest cell (uniform over the CTA)
   uint32_t ssd_local = 0;
   for (int o = threadIdx.x; o < row3; o += kBulkThreads) {
     const int cx = o / 3, ch = o - 3 * cx;
     const int x0 = xb[cx], x1 = xb[cx + 1];
     const uint16_t* col = colsum + ch;
-#if FFSVA_K1_CELL16
-    const uint32_t s = cellw <= 16 ? cell_sum_n<16>(col, x0, x1) : cell_sum(col, x0, x1);
-#else
-    const uint32_t s = cell_sum(col, x0, x1);
-#endif
+    const uint32_t s = cell_sum_w(col, x0, x1, cellw);
     cell[o] = s;
     const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)rows;
-    const uint32_t d = (s + (n >> 1)) / n;
+    const uint32_t d = box_mean(s, n);
     if (kD100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)r * row3 + o] = (uint8_t)d;
     const int diff = (int)d - (int)__ldg(fd.ref + (int64_t)r * row3 + o);
     ssd_local += dist_term(diff, fd.metric);
@@ -405,14 +428,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
       st_async_u32(rbase + 4u * (uint32_t)o, cell[6 * cx + ch] + cell[6 * cx + 3 + ch], rbar);
     }
   } else {
-    const int yb = (int)(((uint32_t)(r + 2) * (uint32_t)H) / (uint32_t)sdd_h);
+    const int yb = ytab ? __ldg(a.ybounds + r + 2) : (int)(((uint32_t)(r + 2) * (uint32_t)H) / (uint32_t)sdd_h);
+    const int64_t slot = a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f;
+    uint8_t* d50row = a.d50 + slot * a.d50_stride + (int64_t)(r >> 1) * half3;
     mbar_wait_parity(bar_p, 0);
     for (int o = threadIdx.x; o < half3; o += kBulkThreads) {
       const int cx = o / 3, ch = o - 3 * cx;
       const uint32_t s = cell[6 * cx + ch] + cell[6 * cx + 3 + ch] + pair_in[o];
       const uint32_t n = (uint32_t)(xb[2 * cx + 2] - xb[2 * cx]) * (uint32_t)(yb - y0);
-      const int64_t slot = a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f;
-      a.d50[slot * a.d50_stride + (int64_t)(r >> 1) * half3 + o] = (uint8_t)((s + (n >> 1)) / n);
+      d50row[o] = (uint8_t)box_mean(s, n);
     }
   }
   ssd_commit(ssd_local, red, a, f, fd.slot, r == 0);
@@ -544,9 +568,20 @@ cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st) {
   if (a.n <= 0) return cudaSuccess;
   if (a.bulk) {
     const size_t smem = sdd_bulk_smem_bytes(a.stage_bytes, a.sdd_w);
-    const unsigned grid = (unsigned)a.n * (unsigned)a.sdd_h;
-    if (a.d100) sdd_bulk_kernel<true><<<grid, kBulkThreads, smem, st>>>(a);
-    else sdd_bulk_kernel<false><<<grid, kBulkThreads, smem, st>>>(a);
+    // grid (row, frame); gridDim.y <= 65535, so very large batches take several launches
+    for (int32_t f0 = 0; f0 < a.n; f0 += 65535) {
+      SddArgs b = a;
+      const int32_t cnt = a.n - f0 < 65535 ? a.n - f0 : 65535;
+      b.frames += f0;
+      b.acc_ssd += f0;
+      b.n = cnt;
+      if (b.d50_index) b.d50_index += f0;
+      else b.d50 += (int64_t)f0 * a.d50_stride;
+      if (b.d100) b.d100 += (int64_t)f0 * a.sdd_w * a.sdd_h * 3;
+      const dim3 grid((unsigned)a.sdd_h, (unsigned)cnt);
+      if (b.d100) sdd_bulk_kernel<true><<<grid, kBulkThreads, smem, st>>>(b);
+      else sdd_bulk_kernel<false><<<grid, kBulkThreads, smem, st>>>(b);
+    }
     return cudaGetLastError();
   }
   const size_t smem = sdd_smem_bytes(a.max_chunks, a.sdd_w);
