@@ -335,9 +335,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   const int W = fd.W, H = fd.H;
   const int rb16 = (3 * W + 15) & ~15;
   const int nchunk = rb16 >> 4;
-  // row boundaries: the host table when the batch shares H, else 32-bit division (H <= 65535, sdd_h <= 4096 are
-  // validated, so r*H < 2^28)
-  const bool ytab = a.ybounds && H == a.uni_H;
+  // row boundaries: the host table (set only when every frame of the batch has height uni_H, so its loads do not
+  // wait for the frame descriptor), else 32-bit division (H <= 65535, sdd_h <= 4096 are validated: r*H < 2^28)
+  const bool ytab = a.ybounds != nullptr;
   const int y0 = ytab ? __ldg(a.ybounds + r) : (int)(((uint32_t)r * (uint32_t)H) / (uint32_t)sdd_h);
   const int y1 = ytab ? __ldg(a.ybounds + r + 1) : (int)(((uint32_t)(r + 1) * (uint32_t)H) / (uint32_t)sdd_h);
   const int rows = y1 - y0;
@@ -367,7 +367,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   // publish the peer's mbarrier before any remote st.async (relaxed: no memory fence needed beyond
   // fence.mbarrier_init); the matching wait comes right before the DSMEM exchange
   asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
-  if (a.xbounds && W == a.uni_W) {
+  if (a.xbounds) {  // set only for uniform-width batches
     for (int i = threadIdx.x; i <= sdd_w; i += blockDim.x) xb[i] = __ldg(a.xbounds + i);
   } else {
     fill_xbounds(xb, W, sdd_w);
@@ -401,7 +401,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
 
   // ---- 100-grid cells of this row (one thread per cell and channel): D100, SSD vs R
   const int row3 = 3 * sdd_w;
-  const int cellw = W == a.uni_W ? a.cellw : (W + sdd_w - 1) / sdd_w;  // widest cell (uniform over the CTA)
+  const int cellw = a.xbounds ? a.cellw : (W + sdd_w - 1) / sdd_w;  // widest cell (uniform over the CTA)
   uint32_t ssd_local = 0;
   for (int o = threadIdx.x; o < row3; o += kBulkThreads) {
     const int cx = o / 3, ch = o - 3 * cx;
