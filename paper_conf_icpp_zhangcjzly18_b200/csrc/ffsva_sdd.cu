@@ -418,6 +418,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   if (fd.mode == kRefPrevious) ssd_local = 0;  // K2 measures against the previous frame's D100
   __syncthreads();
 
+#ifndef FFSVA_K1_NO_D50
+#define FFSVA_K1_NO_D50 0  // timing probe only (A/B): skip the D50 pair exchange; D50 is left unwritten
+#endif
+  if (FFSVA_K1_NO_D50) {
+    ssd_commit(ssd_local, red, a, f, fd.slot, r == 0);
+    return;
+  }
   // ---- D50 row: odd CTA -> even CTA (st.async into the peer's shared memory), even CTA combines 2x2 cells.
   // Only the odd CTA touches its peer's memory, so only it waits on the cluster barrier (for the peer's
   // mbarrier init); the even CTA stays alive until the peer's bytes land on its mbarrier.
