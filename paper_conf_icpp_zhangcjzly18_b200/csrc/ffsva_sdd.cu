@@ -456,25 +456,27 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
 
 // Deferred D50 (C1 / Q8: every 50-cell is the union of 2x2 100-cells): from the per-row 2-cell sums K1 left in
 // `rowsum`, for the frames that need it — the SDD survivors in work order (after K3) or every frame (SDD-only
-// batches). One CTA per (listed frame, 50-grid band); the two rows of the band are added and rounded once.
-__global__ void __launch_bounds__(160) d50_kernel(D50Args a) {
-  const int nb = a.sdd_h >> 1;
-  const int idx = blockIdx.x / nb, b = blockIdx.x - idx * nb;
+// batches). One CTA per frame; the two rows of each band are added and rounded once.
+__global__ void __launch_bounds__(256) d50_kernel(D50Args a) {
+  const int idx = blockIdx.x;
   if (a.list_count && idx >= *a.list_count) return;
   const int f = a.list ? __ldg(a.list + idx) : idx;
-  const FrameDesc& fd = a.frames[f];
+  const FrameDesc fd = a.frames[f];
   const int W = fd.W, H = fd.H, sdd_w = a.sdd_w, sdd_h = a.sdd_h;
-  const int half3 = 3 * (sdd_w >> 1);
-  const int ya = a.ybounds ? __ldg(a.ybounds + 2 * b) : (int)(((uint32_t)(2 * b) * (uint32_t)H) / (uint32_t)sdd_h);
-  const int yb = a.ybounds ? __ldg(a.ybounds + 2 * b + 2) : (int)(((uint32_t)(2 * b + 2) * (uint32_t)H) / (uint32_t)sdd_h);
-  const uint32_t* rs = a.rowsum + ((int64_t)f * sdd_h + 2 * b) * half3;
+  const int half3 = 3 * (sdd_w >> 1), nb = sdd_h >> 1;
+  const uint32_t* rs = a.rowsum + (int64_t)f * sdd_h * half3;
   const int64_t slot = a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f;
-  uint8_t* out = a.d50 + slot * a.d50_stride + (int64_t)b * half3;
-  for (int k = threadIdx.x; k < half3; k += blockDim.x) {
-    const int cx = k / 3;
+  uint8_t* out = a.d50 + slot * a.d50_stride;
+  for (int o = threadIdx.x; o < nb * half3; o += blockDim.x) {
+    const int b = o / half3, k = o - b * half3, cx = k / 3;
+    const int ya = a.ybounds ? __ldg(a.ybounds + 2 * b) : (int)(((uint32_t)(2 * b) * (uint32_t)H) / (uint32_t)sdd_h);
+    const int yb = a.ybounds ? __ldg(a.ybounds + 2 * b + 2)
+                             : (int)(((uint32_t)(2 * b + 2) * (uint32_t)H) / (uint32_t)sdd_h);
     const int xa = a.xbounds ? __ldg(a.xbounds + 2 * cx) : (int)(((uint32_t)(2 * cx) * (uint32_t)W) / (uint32_t)sdd_w);
-    const int xc = a.xbounds ? __ldg(a.xbounds + 2 * cx + 2) : (int)(((uint32_t)(2 * cx + 2) * (uint32_t)W) / (uint32_t)sdd_w);
-    out[k] = (uint8_t)box_mean(rs[k] + rs[half3 + k], (uint32_t)(xc - xa) * (uint32_t)(yb - ya));
+    const int xc = a.xbounds ? __ldg(a.xbounds + 2 * cx + 2)
+                             : (int)(((uint32_t)(2 * cx + 2) * (uint32_t)W) / (uint32_t)sdd_w);
+    const uint32_t s = rs[(2 * b) * half3 + k] + rs[(2 * b + 1) * half3 + k];
+    out[o] = (uint8_t)box_mean(s, (uint32_t)(xc - xa) * (uint32_t)(yb - ya));
   }
 }
 
@@ -646,7 +648,7 @@ cudaError_t launch_prev(const PrevArgs& a, cudaStream_t st) {
 
 cudaError_t launch_d50(const D50Args& a, int32_t max_frames, cudaStream_t st) {
   if (max_frames <= 0) return cudaSuccess;
-  d50_kernel<<<(unsigned)(max_frames * (a.sdd_h / 2)), 160, 0, st>>>(a);
+  d50_kernel<<<(unsigned)max_frames, 256, 0, st>>>(a);
   return cudaGetLastError();
 }
 
