@@ -179,9 +179,8 @@ FFSVA_API ffsva_status ffsva_batch_device_outputs(ffsva_batch* b, uint64_t** ssd
 FFSVA_API ffsva_status ffsva_batch_destroy(ffsva_batch* b);
 
 /* Measurement hook: launch the cascade of each of the nb prepared batches in turn, iters times over the list,
- * directly (no graph) with CUDA events recorded on cuda_stream around every kernel; ms_out[0..3] receive the
- * mean device time per launch of K1 (ingest/downsample/SDD, with K2 for previous-frame streams), K3
- * (compaction), the deferred D50 kernel and K4 (SNM). Synchronous. */
+ * directly (no graph) with CUDA events recorded on cuda_stream around every kernel; ms_out[0..2] receive the
+ * mean device time per launch of K1 (ingest/downsample/SDD), K3 (compaction) and K4 (SNM). Synchronous. */
 FFSVA_API ffsva_status ffsva_batch_profile(ffsva_batch* const* batches, int32_t nb, int32_t iters,
                                            float* ms_out, void* cuda_stream);
 

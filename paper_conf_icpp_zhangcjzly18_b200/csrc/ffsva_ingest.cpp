@@ -99,10 +99,8 @@ extern "C" FFSVA_API ffsva_status ffsva_filter_batch_host(const ffsva_frame* fra
     g_launches += prev_launches(b);
     if (st == FFSVA_OK && (e = launch_compact(make_compact_args(b), cs)) != cudaSuccess)
       st = cuda_fail(ctx, e, "launch_compact");
-    g_launches += 1;
-    int nk = 0;
-    if (st == FFSVA_OK) st = launch_after_sdd(b, cs, &nk, nullptr, nullptr);
-    g_launches += nk;
+    if (st == FFSVA_OK && (e = launch_snm(make_snm_args(b), cs)) != cudaSuccess) st = cuda_fail(ctx, e, "launch_snm");
+    g_launches += 2;
   }
   if (st == FFSVA_OK) st = batch_fetch(b, results, cs);
   cudaStreamSynchronize(ctx->copy_stream);

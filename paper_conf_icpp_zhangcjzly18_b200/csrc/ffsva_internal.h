@@ -69,28 +69,16 @@ struct SddArgs {
   const int32_t* ybounds;    // [sdd_h + 1] floor(i*uni_H/sdd_h) for frames of height uni_H, or nullptr
   int32_t uni_W, uni_H;
   int32_t cellw;             // widest 100-grid cell of uni_W-wide frames, ceil(uni_W / sdd_w) (0 if mixed)
-  uint32_t* rowsum;          // bulk kernel: non-null = deferred D50 (per-row 2-cell sums [n][sdd_h][3*sdd_w/2] here,
-                             // d50_kernel finishes them); null = D50 by DSMEM exchange within each CTA pair
+  int32_t pipe_stages;       // > 0: persistent double-buffered kernel with this many stages per CTA
+  int32_t pipe_grid;         // its grid size (CTAs)
 };
 cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st);
 size_t sdd_smem_bytes(int max_chunks, int sdd_w);
 size_t sdd_bulk_smem_bytes(int stage_bytes, int sdd_w);
 int sdd_bulk_stage_bytes(int W, int H, int sdd_h);
 bool sdd_bulk_ok(int max_chunks, int stage_bytes);
-// Deferred D50 from K1's row sums, for the listed frames (survivors after K3) or all frames (list = nullptr).
-struct D50Args {
-  const FrameDesc* frames;
-  const uint32_t* rowsum;
-  const int32_t* list;       // frame indices, or nullptr = frames 0 .. grid-1
-  const int32_t* list_count; // device count of `list` (K3's survivor count), or nullptr
-  uint8_t* d50;
-  int64_t d50_stride;
-  const int32_t* d50_index;
-  const int32_t* xbounds;    // uniform-batch tables (or nullptr)
-  const int32_t* ybounds;
-  int32_t sdd_w, sdd_h;
-};
-cudaError_t launch_d50(const D50Args& a, int32_t max_frames, cudaStream_t st);
+size_t sdd_pipe_smem_bytes(int stages, int stage_bytes, int max_chunks, int sdd_w);
+void sdd_pipe_config(int stage_bytes, int max_chunks, int sdd_w, int num_sms, int* stages, int* grid);
 cudaError_t sdd_configure(size_t smem);  // raise the kernels' dynamic smem limit (outside graph capture)
 int sdd_threads(int max_chunks);
 

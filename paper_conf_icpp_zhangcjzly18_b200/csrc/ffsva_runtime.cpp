@@ -292,7 +292,6 @@ static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t s
   b->in_bytes = off;
   const size_t o_d50 = off; off += al((size_t)b->d50_stride * n);
   const size_t o_d100 = off; off += d100 ? al((size_t)3 * sdd_w * sdd_h * n) : 0;
-  const size_t o_rowsum = off; off += al((size_t)4 * sdd_h * (3 * (sdd_w / 2)) * n);  // deferred-D50 row sums
   const size_t o_acc = off; off += al(8 * n);
   const size_t o_work = off; off += al(4 * n);
   const size_t o_posw = off; off += al(4 * (n + 1));
@@ -315,7 +314,6 @@ static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t s
   b->d_last = (int32_t*)(base + o_last);
   b->d_d50 = base + o_d50;
   b->d_d100 = d100 ? base + o_d100 : nullptr;
-  b->d_rowsum = (uint32_t*)(base + o_rowsum);
   b->d_acc = (unsigned long long*)(base + o_acc);
   b->d_work = (int32_t*)(base + o_work);
   b->d_posw = (int32_t*)(base + o_posw);
@@ -371,11 +369,16 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     cudaGraphExecDestroy(b->graph);
     b->graph = nullptr;
   }
-  cudaError_t e = sdd_configure(bulk ? sdd_bulk_smem_bytes(stage_bytes, sdd_w) : sdd_smem_bytes(max_chunks, sdd_w));
+  // persistent double-buffered variant of the bulk kernel (FFSVA_SDD_KERNEL=bulk keeps the one-shot kernel)
+  int pipe_stages = 0, pipe_grid = 0;
+  if (bulk && !(force && std::strcmp(force, "bulk") == 0))
+    sdd_pipe_config(stage_bytes, max_chunks, sdd_w, ctx->num_sms, &pipe_stages, &pipe_grid);
+  size_t smem_need = bulk ? sdd_bulk_smem_bytes(stage_bytes, sdd_w) : sdd_smem_bytes(max_chunks, sdd_w);
+  if (pipe_stages) smem_need = std::max(smem_need, sdd_pipe_smem_bytes(pipe_stages, stage_bytes, max_chunks, sdd_w));
+  cudaError_t e = sdd_configure(smem_need);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "sdd_configure");
-  // the bulk kernel defers D50 to d50_kernel (no wait on the CTA pair); FFSVA_SDD_KERNEL=pair keeps the DSMEM
-  // exchange
-  b->deferred_d50 = bulk && !(force && std::strcmp(force, "pair") == 0);
+  b->pipe_stages = pipe_stages;
+  b->pipe_grid = pipe_grid;
   b->n = n;
   b->vec16 = vec16;
   b->bulk = bulk;
@@ -488,7 +491,8 @@ SddArgs make_sdd_args(Batch* b, int32_t i0, int32_t cnt) {
   sa.uni_W = b->uni_W;
   sa.uni_H = b->uni_H;
   sa.cellw = b->uni_W > 0 ? (b->uni_W + b->sdd_w - 1) / b->sdd_w : 0;
-  sa.rowsum = b->deferred_d50 ? b->d_rowsum + (size_t)i0 * b->sdd_h * (3 * (b->sdd_w / 2)) : nullptr;
+  sa.pipe_stages = b->pipe_stages;
+  sa.pipe_grid = b->pipe_grid;
   sa.xbounds = b->uni_W > 0 ? b->d_xb : nullptr;
   sa.ybounds = b->uni_H > 0 ? b->d_yb : nullptr;
   return sa;
@@ -552,37 +556,6 @@ PrevArgs make_prev_args(Batch* b) {
 
 int prev_launches(const Batch* b) { return b->n_pm > 0 ? (b->n_last > 0 ? 2 : 1) : 0; }
 
-D50Args make_d50_args(Batch* b) {
-  D50Args da{};
-  da.frames = b->d_desc;
-  da.rowsum = b->d_rowsum;
-  da.list = b->sdd_only ? nullptr : b->d_work;        // survivors in work order (K3), or every frame
-  da.list_count = b->sdd_only ? nullptr : b->d_counts;
-  da.d50 = b->d_d50;
-  da.d50_stride = b->d50_stride;
-  da.xbounds = b->uni_W > 0 ? b->d_xb : nullptr;
-  da.ybounds = b->uni_H > 0 ? b->d_yb : nullptr;
-  da.sdd_w = b->sdd_w;
-  da.sdd_h = b->sdd_h;
-  return da;
-}
-
-// K3 -> deferred D50 (if K1 left row sums) -> K4, shared by batches and the host-frame path.
-ffsva_status launch_after_sdd(Batch* b, cudaStream_t st, int* nk, cudaEvent_t ev_d50, cudaEvent_t ev_snm) {
-  DeviceCtx* ctx = b->ctx;
-  if (b->deferred_d50) {
-    FF_CUDA(ctx, launch_d50(make_d50_args(b), b->n, st));
-    *nk += 1;
-  }
-  if (ev_d50) cudaEventRecord(ev_d50, st);
-  if (!b->sdd_only) {
-    FF_CUDA(ctx, launch_snm(make_snm_args(b), st));
-    *nk += 1;
-  }
-  if (ev_snm) cudaEventRecord(ev_snm, st);
-  return FFSVA_OK;
-}
-
 static ffsva_status batch_launch_kernels(Batch* b, cudaStream_t st, int* nk, cudaEvent_t* ev = nullptr) {
   DeviceCtx* ctx = b->ctx;
   if (ev) cudaEventRecord(ev[0], st);
@@ -592,14 +565,19 @@ static ffsva_status batch_launch_kernels(Batch* b, cudaStream_t st, int* nk, cud
   FF_CUDA(ctx, launch_compact(make_compact_args(b), st));
   if (ev) cudaEventRecord(ev[2], st);
   *nk = 2 + prev_launches(b);
-  return launch_after_sdd(b, st, nk, ev ? ev[3] : nullptr, ev ? ev[4] : nullptr);
+  if (!b->sdd_only) {
+    FF_CUDA(ctx, launch_snm(make_snm_args(b), st));
+    *nk += 1;
+  }
+  if (ev) cudaEventRecord(ev[3], st);
+  return FFSVA_OK;
 }
 
 ffsva_status batch_profile(Batch* const* batches, int32_t nb, int32_t iters, float* ms_out, cudaStream_t st) {
   DeviceCtx* ctx = batches[0]->ctx;
-  cudaEvent_t ev[5];
+  cudaEvent_t ev[4];
   for (auto& e : ev) FF_CUDA(ctx, cudaEventCreate(&e));
-  double acc[4] = {0, 0, 0, 0};
+  double acc[3] = {0, 0, 0};
   int count = 0;
   ffsva_status s = FFSVA_OK;
   for (int it = 0; it < iters && s == FFSVA_OK; ++it)
@@ -608,19 +586,21 @@ ffsva_status batch_profile(Batch* const* batches, int32_t nb, int32_t iters, flo
       s = batch_launch_kernels(batches[j], st, &nk, ev);
       g_launches += nk;
       if (s != FFSVA_OK) break;
-      cudaError_t e = cudaEventSynchronize(ev[4]);
+      cudaError_t e = cudaEventSynchronize(ev[3]);
       if (e != cudaSuccess) {
         s = cuda_fail(ctx, e, "cudaEventSynchronize(profile)");
         break;
       }
-      float t[4];
-      for (int k = 0; k < 4; ++k) cudaEventElapsedTime(&t[k], ev[k], ev[k + 1]);
-      for (int k = 0; k < 4; ++k) acc[k] += t[k];
+      float t[3];
+      cudaEventElapsedTime(&t[0], ev[0], ev[1]);
+      cudaEventElapsedTime(&t[1], ev[1], ev[2]);
+      cudaEventElapsedTime(&t[2], ev[2], ev[3]);
+      for (int k = 0; k < 3; ++k) acc[k] += t[k];
       ++count;
     }
   for (auto& e : ev) cudaEventDestroy(e);
   if (s != FFSVA_OK) return s;
-  for (int k = 0; k < 4; ++k) ms_out[k] = count ? (float)(acc[k] / count) : 0.f;
+  for (int k = 0; k < 3; ++k) ms_out[k] = count ? (float)(acc[k] / count) : 0.f;
   return FFSVA_OK;
 }
 

@@ -40,7 +40,7 @@ struct Batch {
   bool vec16 = true, sdd_only = false, want_d100 = false;
   bool bulk = false;          // K1 variant: bulk-async + cluster (aligned frames) or register streaming
   int32_t stage_bytes = 0;
-  bool deferred_d50 = false;  // K1 leaves per-row 2-cell sums in d_rowsum; d50_kernel forms D50 after K3
+  int32_t pipe_stages = 0, pipe_grid = 0;  // persistent double-buffered K1 (0: one-shot kernels)
   int32_t uni_W = -1, uni_H = -1;        // common frame size of the batch (-1: mixed)
   int32_t *d_xb = nullptr, *d_yb = nullptr;  // cell boundary tables for uni_W / uni_H (in the input block)
   int32_t *d_pm = nullptr, *d_last = nullptr;  // PREVIOUS-mode plan (input block): (frame, prev) pairs, last frames
@@ -53,7 +53,6 @@ struct Batch {
   int32_t *d_perm = nullptr, *d_seg_lo = nullptr, *d_seg_batch = nullptr;
   uint8_t* d_d50 = nullptr;
   uint8_t* d_d100 = nullptr;
-  uint32_t* d_rowsum = nullptr;
   unsigned long long* d_acc = nullptr;  // per-frame SSD accumulators (K1 adds, K3 reads + re-zeroes)
   int32_t *d_work = nullptr, *d_posw = nullptr, *d_chunks = nullptr, *d_counts = nullptr;
   // output block (one D2H): ssd u64[n] | logit f32[n] | survivor_idx i32[n] | sdd_pass u8[n] | snm_pass u8[n] |
@@ -118,9 +117,6 @@ CompactArgs make_compact_args(Batch* b);
 SnmArgs make_snm_args(Batch* b);
 PrevArgs make_prev_args(Batch* b);
 int prev_launches(const Batch* b);  // kernels launch_prev issues for this batch (0, 1 or 2)
-D50Args make_d50_args(Batch* b);
-// after K1 (+ K2) and K3: the deferred D50 kernel and the SNM; *nk counts the launches; events optional
-ffsva_status launch_after_sdd(Batch* b, cudaStream_t st, int* nk, cudaEvent_t ev_d50, cudaEvent_t ev_snm);
 
 // RAII device switch
 struct DeviceGuard {

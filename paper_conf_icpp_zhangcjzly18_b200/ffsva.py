@@ -252,9 +252,9 @@ def ffsva_batch_destroy(batch) -> None:
 
 
 def ffsva_batch_profile(batches, iters: int, cuda_stream: int) -> list:
-    """Mean device ms per launch of [K1 (+K2), K3, D50, K4] over iters passes of the prepared batches."""
+    """Mean device ms per launch of [K1, K3, K4] over iters passes of the prepared batches."""
     arr = (ctypes.c_void_p * len(batches))(*batches)
-    ms = (ctypes.c_float * 4)()
+    ms = (ctypes.c_float * 3)()
     _check(lib().ffsva_batch_profile(arr, len(batches), iters, ms, cuda_stream), "ffsva_batch_profile")
     return [float(x) for x in ms]
 
