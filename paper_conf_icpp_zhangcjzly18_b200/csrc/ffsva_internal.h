@@ -69,16 +69,12 @@ struct SddArgs {
   const int32_t* ybounds;    // [sdd_h + 1] floor(i*uni_H/sdd_h) for frames of height uni_H, or nullptr
   int32_t uni_W, uni_H;
   int32_t cellw;             // widest 100-grid cell of uni_W-wide frames, ceil(uni_W / sdd_w) (0 if mixed)
-  int32_t pipe_stages;       // > 0: persistent double-buffered kernel with this many stages per CTA
-  int32_t pipe_grid;         // its grid size (CTAs)
 };
 cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st);
 size_t sdd_smem_bytes(int max_chunks, int sdd_w);
 size_t sdd_bulk_smem_bytes(int stage_bytes, int sdd_w);
 int sdd_bulk_stage_bytes(int W, int H, int sdd_h);
 bool sdd_bulk_ok(int max_chunks, int stage_bytes);
-size_t sdd_pipe_smem_bytes(int stages, int stage_bytes, int max_chunks, int sdd_w);
-void sdd_pipe_config(int stage_bytes, int max_chunks, int sdd_w, int num_sms, int* stages, int* grid);
 cudaError_t sdd_configure(size_t smem);  // raise the kernels' dynamic smem limit (outside graph capture)
 int sdd_threads(int max_chunks);
 

@@ -369,16 +369,8 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     cudaGraphExecDestroy(b->graph);
     b->graph = nullptr;
   }
-  // persistent double-buffered variant of the bulk kernel (FFSVA_SDD_KERNEL=bulk keeps the one-shot kernel)
-  int pipe_stages = 0, pipe_grid = 0;
-  if (bulk && !(force && std::strcmp(force, "bulk") == 0))
-    sdd_pipe_config(stage_bytes, max_chunks, sdd_w, ctx->num_sms, &pipe_stages, &pipe_grid);
-  size_t smem_need = bulk ? sdd_bulk_smem_bytes(stage_bytes, sdd_w) : sdd_smem_bytes(max_chunks, sdd_w);
-  if (pipe_stages) smem_need = std::max(smem_need, sdd_pipe_smem_bytes(pipe_stages, stage_bytes, max_chunks, sdd_w));
-  cudaError_t e = sdd_configure(smem_need);
+  cudaError_t e = sdd_configure(bulk ? sdd_bulk_smem_bytes(stage_bytes, sdd_w) : sdd_smem_bytes(max_chunks, sdd_w));
   if (e != cudaSuccess) return cuda_fail(ctx, e, "sdd_configure");
-  b->pipe_stages = pipe_stages;
-  b->pipe_grid = pipe_grid;
   b->n = n;
   b->vec16 = vec16;
   b->bulk = bulk;
@@ -491,8 +483,6 @@ SddArgs make_sdd_args(Batch* b, int32_t i0, int32_t cnt) {
   sa.uni_W = b->uni_W;
   sa.uni_H = b->uni_H;
   sa.cellw = b->uni_W > 0 ? (b->uni_W + b->sdd_w - 1) / b->sdd_w : 0;
-  sa.pipe_stages = b->pipe_stages;
-  sa.pipe_grid = b->pipe_grid;
   sa.xbounds = b->uni_W > 0 ? b->d_xb : nullptr;
   sa.ybounds = b->uni_H > 0 ? b->d_yb : nullptr;
   return sa;

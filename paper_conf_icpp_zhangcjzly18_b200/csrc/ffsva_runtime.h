@@ -40,7 +40,6 @@ struct Batch {
   bool vec16 = true, sdd_only = false, want_d100 = false;
   bool bulk = false;          // K1 variant: bulk-async + cluster (aligned frames) or register streaming
   int32_t stage_bytes = 0;
-  int32_t pipe_stages = 0, pipe_grid = 0;  // persistent double-buffered K1 (0: one-shot kernels)
   int32_t uni_W = -1, uni_H = -1;        // common frame size of the batch (-1: mixed)
   int32_t *d_xb = nullptr, *d_yb = nullptr;  // cell boundary tables for uni_W / uni_H (in the input block)
   int32_t *d_pm = nullptr, *d_last = nullptr;  // PREVIOUS-mode plan (input block): (frame, prev) pairs, last frames

@@ -418,13 +418,6 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   if (fd.mode == kRefPrevious) ssd_local = 0;  // K2 measures against the previous frame's D100
   __syncthreads();
 
-#ifndef FFSVA_K1_NO_D50
-#define FFSVA_K1_NO_D50 0  // timing probe only (A/B): skip the D50 pair exchange; D50 is left unwritten
-#endif
-  if (FFSVA_K1_NO_D50) {
-    ssd_commit(ssd_local, red, a, f, fd.slot, r == 0);
-    return;
-  }
   // ---- D50 row: odd CTA -> even CTA (st.async into the peer's shared memory), even CTA combines 2x2 cells.
   // Only the odd CTA touches its peer's memory, so only it waits on the cluster barrier (for the peer's
   // mbarrier init); the even CTA stays alive until the peer's bytes land on its mbarrier.
@@ -449,158 +442,6 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
     }
   }
   ssd_commit(ssd_local, red, a, f, fd.slot, r == 0);
-}
-
-// ------------------------------------------------------------------ persistent, double-buffered bulk variant
-// sdd_pipe_kernel (aligned rows; the default): a persistent grid walks (frame, 50-grid band) work items; each CTA
-// streams its bands' 100-grid rows through an S-stage ring of shared-memory buffers filled by cp.async.bulk (TMA
-// engine, L2 evict-first), so the copies of the next rows are in flight while the current row is reduced — the
-// one-shot kernel above leaves the SM's share of HBM idle while each CTA computes. Both rows of a band live in the
-// same CTA, so D50 (2x2 100-cells) needs no cluster exchange. Distances accumulate per band: one u64 atomic per
-// band and frame.
-constexpr int kPipeThreads = 256;
-constexpr int kPipeMaxStages = 4;
-
-struct PipeRow {  // where global row g of this CTA comes from (written by the issuing thread, read after the wait)
-  int32_t f, r, y0, rows;
-};
-
-__device__ __forceinline__ void pipe_row_of(const SddArgs& a, int g, int& f, int& r) {
-  const int nb = a.sdd_h >> 1;
-  const int w = blockIdx.x + (g >> 1) * gridDim.x;
-  f = w / nb;
-  r = 2 * (w - f * nb) + (g & 1);
-}
-
-__device__ __forceinline__ void pipe_issue(const SddArgs& a, int g, uint8_t* stage, uint32_t bar, PipeRow* meta,
-                                           uint64_t pol) {
-  int f, r;
-  pipe_row_of(a, g, f, r);
-  const FrameDesc& fd = a.frames[f];
-  const int H = fd.H, W = fd.W;
-  const bool ytab = a.ybounds && H == a.uni_H;
-  const int y0 = ytab ? __ldg(a.ybounds + r) : (int)(((uint32_t)r * (uint32_t)H) / (uint32_t)a.sdd_h);
-  const int y1 = ytab ? __ldg(a.ybounds + r + 1) : (int)(((uint32_t)(r + 1) * (uint32_t)H) / (uint32_t)a.sdd_h);
-  const int rows = y1 - y0, rb16 = (3 * W + 15) & ~15;
-  *meta = PipeRow{f, r, y0, rows};
-  mbar_expect_tx(bar, (uint32_t)(rows * rb16));
-  const uint32_t dst = (uint32_t)__cvta_generic_to_shared(stage);
-  const uint8_t* src = fd.pixels + (int64_t)y0 * fd.pitch;
-  if (fd.pitch == rb16) {
-    bulk_g2s(dst, src, (uint32_t)(rows * rb16), bar, pol);
-  } else {
-    for (int y = 0; y < rows; ++y) bulk_g2s(dst + y * rb16, src + (int64_t)y * fd.pitch, (uint32_t)rb16, bar, pol);
-  }
-}
-
-template <bool kD100>
-__global__ void __launch_bounds__(kPipeThreads, 3) sdd_pipe_kernel(SddArgs a) {
-  extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ __align__(8) uint64_t bars[kPipeMaxStages];
-  __shared__ PipeRow meta[kPipeMaxStages];
-  __shared__ uint32_t red[kPipeThreads / 32];
-  const int S = a.pipe_stages, sdd_w = a.sdd_w, row3 = 3 * sdd_w, half3 = 3 * (sdd_w >> 1);
-  const int tid = threadIdx.x;
-  uint16_t* colsum = reinterpret_cast<uint16_t*>(smem + (size_t)S * a.stage_bytes);  // [max rb16]
-  uint32_t* cellbuf = reinterpret_cast<uint32_t*>(colsum + a.max_chunks * 16);      // [2][row3]
-  int* xb = reinterpret_cast<int*>(cellbuf + 2 * row3);                              // [sdd_w + 1]
-  const int nb = a.sdd_h >> 1;
-  const int bands = a.n * nb;
-  const int my_bands = blockIdx.x < bands ? (bands - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
-  const int total = 2 * my_bands;
-  uint64_t pol = 0;
-  if (tid == 0) {
-    for (int s = 0; s < S; ++s) mbar_init_cta((uint32_t)__cvta_generic_to_shared(&bars[s]), 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-    for (int g = 0; g < S && g < total; ++g)
-      pipe_issue(a, g, smem + (size_t)g * a.stage_bytes, (uint32_t)__cvta_generic_to_shared(&bars[g]), &meta[g], pol);
-  }
-  int cur_W = -1, ya = 0;  // ya: first source row of the current band
-  uint32_t dist = 0;       // this thread's share of the current band's distance
-  for (int g = 0; g < total; ++g) {
-    const int s = g % S;
-    const int h = g & 1;  // row within the band
-    const uint32_t bar = (uint32_t)__cvta_generic_to_shared(&bars[s]);
-    int f, r;
-    pipe_row_of(a, g, f, r);
-    const FrameDesc fd = a.frames[f];
-    const int W = fd.W, H = fd.H;
-    const int rb16 = (3 * W + 15) & ~15, nchunk = rb16 >> 4;
-    if (h == 0 && W != cur_W) {  // cell boundaries of this frame width (the previous row's readers are done)
-      if (a.xbounds && W == a.uni_W) {
-        for (int i = tid; i <= sdd_w; i += kPipeThreads) xb[i] = __ldg(a.xbounds + i);
-      } else {
-        fill_xbounds(xb, W, sdd_w);
-      }
-      cur_W = W;
-    }
-    mbar_wait_parity(bar, (uint32_t)(g / S) & 1u);
-    const int rows = meta[s].rows, y0 = meta[s].y0;
-    if (h == 0) ya = y0;
-    const uint8_t* st = smem + (size_t)s * a.stage_bytes;
-    // ---- column sums (<= 2 16-byte chunks per thread)
-#pragma unroll
-    for (int k = 0; k < 2; ++k) {
-      const int c = tid + k * kPipeThreads;
-      if (c < nchunk) {
-        uint32_t acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-        const uint8_t* p = st + 16 * c;
-        int y = 0;
-        for (; y + 1 < rows; y += 2)
-          acc16x2(acc, *reinterpret_cast<const uint4*>(p + y * rb16), *reinterpret_cast<const uint4*>(p + (y + 1) * rb16));
-        if (y < rows) acc16(acc, *reinterpret_cast<const uint4*>(p + y * rb16));
-        store_colsum(reinterpret_cast<uint32_t*>(colsum), c, acc);
-      }
-    }
-    __syncthreads();  // stage s consumed, colsum (and xb) complete
-    if (tid == 0 && g + S < total) {
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic reads of the stage before the refill
-      pipe_issue(a, g + S, smem + (size_t)s * a.stage_bytes, bar, &meta[s], pol);
-    }
-    // ---- 100-grid cells of row r: D100, distance vs R, cell sums for D50
-    const int cellw = W == a.uni_W ? a.cellw : (W + sdd_w - 1) / sdd_w;
-    uint32_t* cell = cellbuf + h * row3;
-    for (int o = tid; o < row3; o += kPipeThreads) {
-      const int cx = o / 3, ch = o - 3 * cx;
-      const int x0 = xb[cx], x1 = xb[cx + 1];
-      const uint32_t sum = cell_sum_w(colsum + ch, x0, x1, cellw);
-      cell[o] = sum;
-      const uint32_t d = box_mean(sum, (uint32_t)(x1 - x0) * (uint32_t)rows);
-      if (kD100) a.d100[(int64_t)f * a.sdd_h * row3 + (int64_t)r * row3 + o] = (uint8_t)d;
-      dist += dist_term((int)d - (int)__ldg(fd.ref + (int64_t)r * row3 + o), fd.metric);
-    }
-    if (h == 1) {
-      __syncthreads();  // both rows' cell sums complete
-      const int64_t slot = a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f;
-      uint8_t* d50row = a.d50 + slot * a.d50_stride + (int64_t)(r >> 1) * half3;
-      const uint32_t bh = (uint32_t)(y0 + rows - ya);
-      for (int o = tid; o < half3; o += kPipeThreads) {
-        const int cx = o / 3, ch = o - 3 * cx;
-        const uint32_t sum = cellbuf[6 * cx + ch] + cellbuf[6 * cx + 3 + ch] + cellbuf[row3 + 6 * cx + ch] +
-                             cellbuf[row3 + 6 * cx + 3 + ch];
-        d50row[o] = (uint8_t)box_mean(sum, (uint32_t)(xb[2 * cx + 2] - xb[2 * cx]) * bh);
-      }
-      // ---- band done: its distance into the frame's accumulator (PREVIOUS-mode frames: K2 measures instead)
-      uint32_t v = fd.mode == kRefPrevious ? 0u : dist;
-      dist = 0;
-#pragma unroll
-      for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
-      if ((tid & 31) == 0) red[tid >> 5] = v;
-      __syncthreads();
-      if (tid == 0) {
-        unsigned long long t = 0;
-        for (int w = 0; w < kPipeThreads / 32; ++w) t += red[w];
-        atomicAdd(a.acc_ssd + f, t);
-        if (a.stats) {
-          unsigned long long* stt = a.stats + (int64_t)fd.slot * NSTAT;
-          atomicAdd(stt + 3, t);
-          if (r == 1) atomicAdd(stt + 0, 1ull);
-        }
-      }
-    }
-    __syncthreads();  // colsum / cellbuf / red reuse by the next row
-  }
 }
 
 // Reference image R: one rounding of the mean over k frames x box. One thread per value.
@@ -707,31 +548,6 @@ int sdd_bulk_stage_bytes(int W, int H, int sdd_h) {
   return rows * rb16;
 }
 
-size_t sdd_pipe_smem_bytes(int stages, int stage_bytes, int max_chunks, int sdd_w) {
-  return (size_t)stages * stage_bytes + (size_t)32 * max_chunks + (size_t)4 * (6 * sdd_w + sdd_w + 1);
-}
-
-// Pipelined variant: stages per CTA and CTAs per SM for this batch (0 stages: use the one-shot kernel).
-void sdd_pipe_config(int stage_bytes, int max_chunks, int sdd_w, int num_sms, int* stages, int* grid) {
-  *stages = 0;
-  *grid = 0;
-  if (max_chunks > 2 * kPipeThreads) return;
-  const size_t budget = 227 * 1024 - 2048;  // per SM, leaving room for the static barriers / metadata
-  // two stages and at least two CTAs per SM when they fit (720p: 3 CTAs); otherwise one CTA with three stages
-  // (1080p rows of 11 x 5760 B), or two
-  const int per_sm2 = (int)(budget / sdd_pipe_smem_bytes(2, stage_bytes, max_chunks, sdd_w));
-  if (per_sm2 >= 2) {
-    *stages = 2;
-    *grid = num_sms * std::min(per_sm2, 3);
-  } else if (budget >= sdd_pipe_smem_bytes(3, stage_bytes, max_chunks, sdd_w)) {
-    *stages = 3;
-    *grid = num_sms;
-  } else if (per_sm2 == 1) {
-    *stages = 2;
-    *grid = num_sms;
-  }
-}
-
 bool sdd_bulk_ok(int max_chunks, int stage_bytes) {
   return max_chunks <= 2 * kBulkThreads && stage_bytes <= kBulkMaxStage;
 }
@@ -739,11 +555,7 @@ bool sdd_bulk_ok(int max_chunks, int stage_bytes) {
 cudaError_t sdd_configure(size_t smem) {
   static size_t configured = 0;
   if (smem <= configured) return cudaSuccess;
-  cudaError_t e = cudaFuncSetAttribute(sdd_pipe_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(sdd_pipe_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(sdd_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  cudaError_t e = cudaFuncSetAttribute(sdd_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(sdd_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e == cudaSuccess)
@@ -756,14 +568,6 @@ cudaError_t sdd_configure(size_t smem) {
 
 cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st) {
   if (a.n <= 0) return cudaSuccess;
-  if (a.pipe_stages > 0) {
-    const size_t smem = sdd_pipe_smem_bytes(a.pipe_stages, a.stage_bytes, a.max_chunks, a.sdd_w);
-    const int bands = a.n * (a.sdd_h / 2);
-    const unsigned grid = (unsigned)(bands < a.pipe_grid ? bands : a.pipe_grid);
-    if (a.d100) sdd_pipe_kernel<true><<<grid, kPipeThreads, smem, st>>>(a);
-    else sdd_pipe_kernel<false><<<grid, kPipeThreads, smem, st>>>(a);
-    return cudaGetLastError();
-  }
   if (a.bulk) {
     const size_t smem = sdd_bulk_smem_bytes(a.stage_bytes, a.sdd_w);
     // grid (row, frame); gridDim.y <= 65535, so very large batches take several launches
