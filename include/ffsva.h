@@ -52,6 +52,7 @@ typedef enum {
 
 typedef struct ffsva_stream ffsva_stream; /* opaque, owned by the library */
 typedef struct ffsva_batch ffsva_batch;   /* opaque prepared batch, owned by the library */
+typedef struct ffsva_tyolo ffsva_tyolo;   /* opaque shared T-YOLO model of a device (f1) */
 
 /* Per-stream configuration (SDD and SNM are specialised per stream; L183 thresholds per stream). */
 typedef struct {
@@ -70,6 +71,11 @@ typedef struct {
   int32_t q_sdd, q_snm;    /* feedback-queue depth thresholds in frames (L217), default 2 and 10 */
   int32_t distance;        /* SDD distance (L151 "MSE, NRMSE, or SAD"), an ffsva_distance; 0 = MSE */
   int32_t ref_mode;        /* SDD reference (L151), an ffsva_ref_mode; 0 = background reference image */
+  int32_t number_of_objects; /* NumberofObjects (L195): the T-YOLO stage keeps a frame iff it counts at least this
+                                many target objects; >= 0 (online runtime with a T-YOLO model attached) */
+  int32_t target_class;    /* the stream's target object, a VOC class 0..19 for T-YOLO (L139: "the target events to
+                              detect, such as the occurrences of cars, persons, etc. ... are predefined by users") */
+  int32_t q_tyolo;         /* T-YOLO queue depth threshold in frames (L217), default 2 */
 } ffsva_stream_desc;
 
 /* SDD distance metrics ("The distance between two video frames can be characterized by Mean
@@ -113,9 +119,11 @@ typedef struct {
   uint8_t sdd_pass;        /* 1 iff the distance exceeds delta_diff (L151), e.g. MSE > delta_diff */
   uint8_t snm_pass;        /* 1 iff sdd_pass and c >= t_pre (L165) */
   uint8_t snm_class;       /* 0: c < c_low, 1: unsure, 2: c > c_high (L159); 0 if !sdd_pass */
-  uint8_t pad;
+  uint8_t tyolo_pass;      /* online runtime with T-YOLO: 1 iff tyolo_count >= NumberofObjects (L195); else 0 */
   float logit;             /* SNM output logit, c = 1/(1+exp(-logit)); NaN if !sdd_pass */
   int32_t survivor_idx;    /* rank among this batch's SDD survivors in input order, -1 if !sdd_pass */
+  int32_t tyolo_count;     /* target objects T-YOLO counted (L171); -1 if the frame did not reach T-YOLO */
+  int32_t reserved;
 } ffsva_result;
 
 /* Counters per stream slot, ffsva_stats_copy() layout: u64[slots][FFSVA_NSTAT]. */
@@ -234,6 +242,11 @@ typedef struct {
   float sdd_ms, snm_ms;      /* wall time of the SDD / SNM cycle (host work + kernels + copies) */
   float host_ms;             /* wall time of the whole tick */
   int32_t pad;
+  int32_t tyolo_scored;      /* frames T-YOLO scored this cycle (0 without a T-YOLO model) */
+  int32_t snm_blocked;       /* streams the SNM stage skipped because their T-YOLO queue was over q_tyolo (L209) */
+  int64_t tyolo_queued;      /* frames waiting in T-YOLO queues after the cycle */
+  float tyolo_ms;            /* wall time of the T-YOLO cycle */
+  int32_t pad2;
 } ffsva_tick_info;
 
 FFSVA_API ffsva_status ffsva_sched_create(int32_t device, int32_t max_frames_per_tick, int32_t snm_slots,
@@ -286,6 +299,14 @@ typedef struct {
   uint64_t pushed, refused;       /* frames accepted / refused by the SDD queue since the reset */
   uint64_t sdd_blocked;           /* SDD cycles that skipped the stream (SNM queue over q_snm) since the reset */
 } ffsva_stream_load;
+/* Attach the device's shared T-YOLO model (ffsva_tyolo_load) to the online runtime as its third stage (f1; NULL
+ * detaches): SNM survivors then wait in per-stream T-YOLO queues; the SNM stage skips a stream while its T-YOLO
+ * queue holds more than q_tyolo frames (L209); each tick ends with a T-YOLO cycle that takes at most num_tyolo
+ * frames from every non-empty T-YOLO queue (L173), counts each frame's target objects (its stream's
+ * target_class, boxes scoring > thresh) and reports tyolo_count / tyolo_pass in its event. The model must outlive
+ * the attachment and live on the scheduler's device. */
+FFSVA_API ffsva_status ffsva_sched_set_tyolo(ffsva_sched* s, ffsva_tyolo* m, int32_t num_tyolo, float thresh);
+
 FFSVA_API ffsva_status ffsva_sched_stream_load(ffsva_sched* s, ffsva_stream* st, int32_t reset,
                                                ffsva_stream_load* out);
 /* Detach a stream from the scheduler (before re-forwarding or closing it): FFSVA_EAGAIN while it still has
@@ -308,7 +329,6 @@ FFSVA_API ffsva_status ffsva_sched_detach(ffsva_sched* s, ffsva_stream* st);
  *     layer's bf16 NHWC activation (layer -1: the resized input, 416x416x4) to host `out` (bf16 bit patterns).
  *   ffsva_tyolo_profile (measurement): mean device ms of the resize and of each of the nine layers over iters runs
  *     of n <= 256 frames, CUDA events on cuda_stream; ms_out[10]. */
-typedef struct ffsva_tyolo ffsva_tyolo;
 FFSVA_API ffsva_status ffsva_tyolo_load(int32_t device, const float* params, int64_t n_params, ffsva_tyolo** out);
 FFSVA_API ffsva_status ffsva_tyolo_run(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, int32_t target_class,
                                        float thresh, int32_t number_of_objects, int32_t* counts, uint8_t* pass,

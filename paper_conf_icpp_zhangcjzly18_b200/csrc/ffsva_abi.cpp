@@ -37,6 +37,9 @@ ffsva_status validate_desc(const ffsva_stream_desc* d) {
     return fail(FFSVA_EINVAL, "distance must be FFSVA_DIST_MSE, _SAD or _NRMSE");
   if (d->ref_mode != FFSVA_REF_BACKGROUND && d->ref_mode != FFSVA_REF_PREVIOUS)
     return fail(FFSVA_EINVAL, "ref_mode must be FFSVA_REF_BACKGROUND or FFSVA_REF_PREVIOUS");
+  if (d->number_of_objects < 0) return fail(FFSVA_EINVAL, "number_of_objects < 0");
+  if (d->target_class < 0 || d->target_class >= 20) return fail(FFSVA_EINVAL, "target_class must be a VOC class 0..19");
+  if (d->q_tyolo < 0) return fail(FFSVA_EINVAL, "negative queue threshold");
   if (d->ref_mode == FFSVA_REF_PREVIOUS && d->distance == FFSVA_DIST_NRMSE)
     return fail(FFSVA_EINVAL, "NRMSE needs a fixed reference (its normaliser is sum R^2)");
   return FFSVA_OK;
@@ -372,7 +375,7 @@ FFSVA_API ffsva_status ffsva_stats_copy(int32_t device, uint64_t* dst, int32_t m
 // ---------------------------------------------------------------- stream images (re-forwarding)
 namespace {
 constexpr uint32_t kImageMagic = 0x56534646u;  // "FFSV"
-constexpr uint32_t kImageVersion = 1;
+constexpr uint32_t kImageVersion = 2;  // 2: descriptor with NumberofObjects, target class, q_tyolo
 constexpr int64_t kImageHeader = 256;
 struct ImageHeader {
   uint32_t magic, version;

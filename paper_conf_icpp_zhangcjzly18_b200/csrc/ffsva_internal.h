@@ -143,10 +143,11 @@ struct PrevArgs {
 cudaError_t launch_prev(const PrevArgs& a, cudaStream_t st);  // K2 then K2b (2 launches if n_pm > 0)
 
 // ------------------------------------------------------------------ T-YOLO (f1, ffsva_tyolo.cu)
-struct TyFrame {           // raw frame geometry for the 416x416 resize
+struct TyFrame {           // raw frame geometry for the 416x416 resize, and the frame's target class (head)
   const uint8_t* pixels;
   int64_t pitch;
   int32_t W, H;
+  int32_t target, pad;
 };
 struct TyConvArgs {
   const __nv_bfloat16* in;   // NHWC [N][H][W][Cp] bf16 (conv input; 'same' convolution keeps H x W)
@@ -164,7 +165,8 @@ struct TyConvArgs {
   int32_t msub;              // 128-row halves per tile sharing each weight stage (1 or 2)
   int32_t patch;             // pool layers: A row = the pooled pixel's 4x4 input patch, weights per pool position
   int32_t lag;               // K steps of gathers in flight per producer thread before it publishes (1 .. S-1)
-  int32_t head, target;      // head: count boxes of class `target` scoring > thresh into counts[frame]
+  int32_t head;              // head: count boxes of frame f's target class scoring > thresh into counts[f]
+  const TyFrame* frames;     // head: per-frame target classes
   float thresh;
   int32_t* counts;
 };

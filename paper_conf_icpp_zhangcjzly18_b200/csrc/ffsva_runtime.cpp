@@ -643,7 +643,9 @@ ffsva_status batch_fetch(Batch* b, ffsva_result* results, cudaStream_t st) {
     r.sdd_pass = ps[i];
     r.snm_pass = sp[i];
     r.snm_class = sc[i];
-    r.pad = 0;
+    r.tyolo_pass = 0;
+    r.tyolo_count = -1;  // the batch API stops after the SNM (T-YOLO: ffsva_tyolo_run / the online runtime)
+    r.reserved = 0;
     r.logit = lg[i];
     r.survivor_idx = sv[i];
   }

@@ -117,6 +117,13 @@ SnmArgs make_snm_args(Batch* b);
 PrevArgs make_prev_args(Batch* b);
 int prev_launches(const Batch* b);  // kernels launch_prev issues for this batch (0, 1 or 2)
 
+// T-YOLO (ffsva_tyolo_host.cpp): run the shared model on n frames with per-frame target classes; the caller holds
+// the device lock. counts / pass / raw (host) may be NULL.
+DeviceCtx* tyolo_device_ctx(const ffsva_tyolo* m);
+ffsva_status tyolo_run_unlocked(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, const int32_t* targets,
+                                float thresh, int32_t number_of_objects, int32_t* counts, uint8_t* pass, float* raw,
+                                cudaStream_t cs);
+
 // RAII device switch
 struct DeviceGuard {
   int prev = -1;

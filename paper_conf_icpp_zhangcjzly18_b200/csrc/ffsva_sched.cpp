@@ -69,6 +69,10 @@ struct ffsva_sched {
   std::deque<ffsva_event> pending;
   std::vector<sched::QFrame> flat;  // this cycle's SNM pops, reused
   std::vector<int32_t> starts;
+  // T-YOLO stage (f1): the device's shared model, its per-cycle extraction and score threshold
+  ffsva_tyolo* tyolo = nullptr;
+  float ty_thresh = 0.2f;
+  std::vector<sched::QFrame> tyflat;
 };
 
 namespace {
@@ -184,7 +188,7 @@ FFSVA_API ffsva_status ffsva_sched_push(ffsva_sched* s, const ffsva_frame* frame
     ffsva_stream* st = frames[i].stream;
     int32_t id = s->lookup(st);
     if (id < 0) {
-      id = s->pol.add_stream(st->desc.q_sdd, st->desc.q_snm, st->desc.snm_batch);
+      id = s->pol.add_stream(st->desc.q_sdd, st->desc.q_snm, st->desc.snm_batch, st->desc.q_tyolo);
       if ((int32_t)s->by_id.size() <= id) s->by_id.resize(id + 1, nullptr);
       s->by_id[id] = st;
       if ((int32_t)s->id_of_slot.size() <= st->slot) s->id_of_slot.resize(st->slot + 1, -1);
@@ -232,12 +236,23 @@ FFSVA_API ffsva_status ffsva_sched_detach(ffsva_sched* s, ffsva_stream* st) {
   const int32_t id = s->lookup(st);
   if (id < 0) return FFSVA_OK;
   const sched::StreamQ& q = s->pol.stream(id);
-  if (!q.sdd.empty() || !q.snm.empty()) return fail(FFSVA_EAGAIN, "stream still has queued frames");
+  if (!q.sdd.empty() || !q.snm.empty() || !q.ty.empty()) return fail(FFSVA_EAGAIN, "stream still has queued frames");
   for (const ffsva_event& e : s->pending)
     if (e.stream == st) return fail(FFSVA_EAGAIN, "stream still has unreported events");
   s->pol.remove_stream(id);
   s->by_id[id] = nullptr;
   s->id_of_slot[st->slot] = -1;
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_sched_set_tyolo(ffsva_sched* s, ffsva_tyolo* m, int32_t num_tyolo, float thresh) {
+  if (!s || (m && num_tyolo < 1) || !(thresh >= 0.f && thresh <= 1.f)) return fail(FFSVA_EINVAL, "bad argument");
+  if (m && tyolo_device_ctx(m) != s->ctx) return fail(FFSVA_EDEVICE, "T-YOLO model lives on another device");
+  std::lock_guard<std::mutex> lk(s->mu);
+  if (!m && s->pol.queued_ty() > 0) return fail(FFSVA_EAGAIN, "frames still wait in T-YOLO queues");
+  s->tyolo = m;
+  s->ty_thresh = thresh;
+  s->pol.set_tyolo(m != nullptr, num_tyolo);
   return FFSVA_OK;
 }
 
@@ -263,7 +278,11 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
   ffsva_tick_info ti{};
   const auto t_tick0 = std::chrono::steady_clock::now();
   uint64_t blocked0 = 0;
-  for (int32_t i = 0; i < s->pol.n_streams(); ++i) blocked0 += s->pol.stream(i).sdd_blocked;
+  int32_t snm_blocked0 = 0;
+  for (int32_t i = 0; i < s->pol.n_streams(); ++i) {
+    blocked0 += s->pol.stream(i).sdd_blocked;
+    snm_blocked0 += (int32_t)s->pol.stream(i).snm_blocked;
+  }
   cudaError_t e = cudaSuccess;
   uint64_t* h_ssd = at<uint64_t>(s->h_out, 0);
   float* h_logit = at<float>(s->h_out, 8 * n);
@@ -367,6 +386,7 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
       ev.result.ssd = h_ssd[i];
       ev.result.logit = NAN;
       ev.result.survivor_idx = -1;
+      ev.result.tyolo_count = -1;
       s->pending.push_back(ev);
       s->free_slots.push_back(adm[i].slot);
     }
@@ -441,6 +461,10 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
     if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
     if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (SNM cycle)");
     for (int32_t k = 0; k < m; ++k) {
+      s->free_slots.push_back(flat[k].slot);
+      flat[k].logit = h_logit[k];
+      flat[k].snm_class = h_snm_class[k];
+      if (s->pol.snm_done(flat[k], h_snm_pass[k] != 0)) continue;  // waits in the stream's T-YOLO queue
       ffsva_event ev{};
       ev.stream = s->by_id[flat[k].stream];
       ev.frame_no = flat[k].frame_no;
@@ -450,10 +474,48 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
       ev.result.snm_class = h_snm_class[k];
       ev.result.logit = h_logit[k];
       ev.result.survivor_idx = -1;
+      ev.result.tyolo_count = -1;
       s->pending.push_back(ev);
-      s->free_slots.push_back(flat[k].slot);
     }
   }
+
+  // ---------------- T-YOLO cycle (f1): at most num_t-yolo frames from each T-YOLO queue (L173), counted with
+  // the shared model; NumberofObjects per stream (L195)
+  const auto t_ty0 = std::chrono::steady_clock::now();
+  if (s->tyolo) {
+    std::vector<sched::QFrame>& tf = s->tyflat;
+    s->pol.pop_ty(tf);
+    const int32_t nt = (int32_t)tf.size();
+    ti.tyolo_scored = nt;
+    if (nt > 0) {
+      std::vector<ffsva_frame> fr((size_t)nt);
+      std::vector<int32_t> targets((size_t)nt), counts((size_t)nt);
+      for (int32_t i = 0; i < nt; ++i) {
+        ffsva_stream* st = s->by_id[tf[i].stream];
+        fr[i] = ffsva_frame{st, (const uint8_t*)tf[i].pixels, tf[i].frame_no};
+        targets[i] = st->desc.target_class;
+      }
+      ffsva_status ts = tyolo_run_unlocked(s->tyolo, fr.data(), nt, targets.data(), s->ty_thresh, 0, counts.data(),
+                                           nullptr, nullptr, cs);
+      if (ts != FFSVA_OK) return ts;
+      for (int32_t i = 0; i < nt; ++i) {
+        const ffsva_stream* st = s->by_id[tf[i].stream];
+        ffsva_event ev{};
+        ev.stream = s->by_id[tf[i].stream];
+        ev.frame_no = tf[i].frame_no;
+        ev.result.ssd = tf[i].ssd;
+        ev.result.sdd_pass = 1;
+        ev.result.snm_pass = 1;
+        ev.result.snm_class = tf[i].snm_class;
+        ev.result.logit = tf[i].logit;
+        ev.result.survivor_idx = -1;
+        ev.result.tyolo_count = counts[i];
+        ev.result.tyolo_pass = counts[i] >= st->desc.number_of_objects ? 1 : 0;
+        s->pending.push_back(ev);
+      }
+    }
+  }
+  const auto t_ty1 = std::chrono::steady_clock::now();
 
   uint64_t blocked1 = 0;
   for (int32_t i = 0; i < s->pol.n_streams(); ++i) blocked1 += s->pol.stream(i).sdd_blocked;
@@ -466,10 +528,14 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
   *n_events = k;
   ti.sdd_queued = s->pol.queued_sdd();
   ti.snm_queued = s->pol.queued_snm();
+  ti.tyolo_queued = s->pol.queued_ty();
+  for (int32_t i = 0; i < s->pol.n_streams(); ++i) ti.snm_blocked += (int32_t)s->pol.stream(i).snm_blocked;
+  ti.snm_blocked -= snm_blocked0;
+  ti.tyolo_ms = std::chrono::duration<float, std::milli>(t_ty1 - t_ty0).count();
   ti.events_pending = (int64_t)s->pending.size();
   const auto t_end = std::chrono::steady_clock::now();
   ti.sdd_ms = std::chrono::duration<float, std::milli>(t_snm0 - t_tick0).count();
-  ti.snm_ms = std::chrono::duration<float, std::milli>(t_end - t_snm0).count();
+  ti.snm_ms = std::chrono::duration<float, std::milli>(t_ty0 - t_snm0).count();
   ti.host_ms = std::chrono::duration<float, std::milli>(t_end - t_tick0).count();
   if (info) *info = ti;
   return FFSVA_OK;

@@ -8,7 +8,12 @@
 //     Q18): the prefetcher is refused while the SDD queue holds more than q_sdd frames (default 2); the SDD
 //     stage skips a stream while its SNM queue holds more than q_snm frames (default 10). The SNM stage feeds
 //     T-YOLO, which is out of scope, so nothing blocks it;
-//   * dynamic batching (L223): each SNM cycle pops min(BatchSize, depth) frames of every non-empty stream.
+//   * dynamic batching (L223): each SNM cycle pops min(BatchSize, depth) frames of every non-empty stream;
+//   * T-YOLO stage (f1, when a T-YOLO model is attached): SNM survivors join the stream's T-YOLO queue; the SNM
+//     stage skips a stream while its T-YOLO queue holds more than q_ty frames ("when the T-YOLO queue depth
+//     exceeds a threshold, the SNM thread ... stops pushing frames to the T-YOLO queue", L209; default 2, L217);
+//     each T-YOLO cycle traverses the streams' T-YOLO queues and extracts at most num_t-yolo frames from each,
+//     skipping empty queues (L173, L211).
 // Streams are visited round-robin (the start rotates every cycle) so a per-cycle frame budget is shared fairly.
 //
 // The two batch mechanisms the paper compares dynamic batching with (§4.3.2, §5.4; f4) are
@@ -40,21 +45,23 @@ struct QFrame {
   const void* pixels = nullptr;
   int32_t slot = -1;          // device D50 slot while the frame sits in the SNM queue
   uint64_t ssd = 0;           // SDD distance, carried to the frame's final event
+  float logit = 0.f;          // SNM result, carried through the T-YOLO queue
+  uint8_t snm_class = 0;
 };
 
 enum class BatchPolicy : int32_t { DYNAMIC = 0, FEEDBACK = 1, STATIC = 2 };
 
 struct StreamQ {
-  int32_t q_sdd = 2, q_snm = 10, batch = 30;
+  int32_t q_sdd = 2, q_snm = 10, batch = 30, q_ty = 2;
   bool live = false;
-  std::deque<QFrame> sdd, snm;
-  uint64_t pushed = 0, refused = 0, sdd_blocked = 0;
-  int32_t max_sdd = 0, max_snm = 0;
+  std::deque<QFrame> sdd, snm, ty;
+  uint64_t pushed = 0, refused = 0, sdd_blocked = 0, snm_blocked = 0;
+  int32_t max_sdd = 0, max_snm = 0, max_ty = 0;
 };
 
 class Policy {
  public:
-  int32_t add_stream(int32_t q_sdd, int32_t q_snm, int32_t batch) {
+  int32_t add_stream(int32_t q_sdd, int32_t q_snm, int32_t batch, int32_t q_ty = 2) {
     int32_t id = -1;
     for (int32_t i = 0; i < (int32_t)st_.size(); ++i)
       if (!st_[i].live) { id = i; break; }
@@ -63,6 +70,7 @@ class Policy {
     s = StreamQ();
     s.q_sdd = q_sdd;
     s.q_snm = q_snm;
+    s.q_ty = q_ty;
     s.batch = batch < 1 ? 1 : batch;
     s.live = true;
     return id;
@@ -75,6 +83,7 @@ class Policy {
     StreamQ& s = st_[id];
     out.insert(out.end(), s.sdd.begin(), s.sdd.end());
     out.insert(out.end(), s.snm.begin(), s.snm.end());
+    out.insert(out.end(), s.ty.begin(), s.ty.end());
     s = StreamQ();
     return out;
   }
@@ -145,6 +154,10 @@ class Policy {
     for (int32_t k = 0; k < n; ++k) {
       StreamQ& s = st_[k];
       if (!s.live || s.snm.empty()) continue;
+      if (tyolo_ && (int32_t)s.ty.size() > s.q_ty) {  // T-YOLO -> SNM feedback (L209)
+        ++s.snm_blocked;
+        continue;
+      }
       const int32_t depth = (int32_t)s.snm.size();
       if (policy_ == BatchPolicy::DYNAMIC) {
         take_from(s, std::min(s.batch, depth));
@@ -163,6 +176,33 @@ class Policy {
     starts.push_back((int32_t)flat.size());
   }
 
+  // An SNM-scored frame: with the T-YOLO stage attached, a survivor joins the stream's T-YOLO queue (returns true:
+  // its event waits for T-YOLO); otherwise its SNM result is final (false).
+  bool snm_done(const QFrame& f, bool pass) {
+    if (!tyolo_ || !pass) return false;
+    StreamQ& s = st_[f.stream];
+    s.ty.push_back(f);
+    s.max_ty = std::max(s.max_ty, (int32_t)s.ty.size());
+    return true;
+  }
+
+  // T-YOLO cycle (L173): every non-empty T-YOLO queue gives at most num_t-yolo frames, oldest first.
+  void pop_ty(std::vector<QFrame>& flat) {
+    flat.clear();
+    for (auto& s : st_) {
+      if (!s.live || s.ty.empty()) continue;
+      const int32_t take = std::min<int32_t>(ty_take_, (int32_t)s.ty.size());
+      flat.insert(flat.end(), s.ty.begin(), s.ty.begin() + take);
+      s.ty.erase(s.ty.begin(), s.ty.begin() + take);
+    }
+  }
+
+  void set_tyolo(bool on, int32_t per_stream) {
+    tyolo_ = on;
+    ty_take_ = per_stream < 1 ? 1 : per_stream;
+  }
+  bool tyolo() const { return tyolo_; }
+
   void set_policy(BatchPolicy p) { policy_ = p; }
   BatchPolicy policy() const { return policy_; }
 
@@ -180,9 +220,10 @@ class Policy {
   // Zero a stream's overload counters (re-forwarding window, L213); depths are state, not counters.
   void reset_counters(int32_t id) {
     StreamQ& s = st_[id];
-    s.pushed = s.refused = s.sdd_blocked = 0;
+    s.pushed = s.refused = s.sdd_blocked = s.snm_blocked = 0;
     s.max_sdd = (int32_t)s.sdd.size();
     s.max_snm = (int32_t)s.snm.size();
+    s.max_ty = (int32_t)s.ty.size();
   }
   int32_t n_streams() const { return (int32_t)st_.size(); }
   int64_t queued_sdd() const {
@@ -195,11 +236,18 @@ class Policy {
     for (auto& s : st_) q += (int64_t)s.snm.size();
     return q;
   }
+  int64_t queued_ty() const {
+    int64_t q = 0;
+    for (auto& s : st_) q += (int64_t)s.ty.size();
+    return q;
+  }
 
  private:
   std::vector<StreamQ> st_;
   int32_t rr_ = 0;
   BatchPolicy policy_ = BatchPolicy::DYNAMIC;
+  bool tyolo_ = false;
+  int32_t ty_take_ = 4;
 };
 
 }  // namespace sched

@@ -334,7 +334,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
             for (int k = 1; k < 20; ++k) mx = fmaxf(mx, p[5 + k]);
             float z = 0.f;
             for (int k = 0; k < 20; ++k) z += __expf(p[5 + k] - mx);
-            const float score = __expf(p[5 + a.target] - mx) / z / (1.f + __expf(-p[4]));
+            const float score = __expf(p[5 + a.frames[n].target] - mx) / z / (1.f + __expf(-p[4]));
             cnt += score > a.thresh ? 1 : 0;
           }
           if (cnt) atomicAdd(a.counts + n, cnt);

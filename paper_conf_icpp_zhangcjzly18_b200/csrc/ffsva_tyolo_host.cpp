@@ -174,7 +174,7 @@ ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
 }
 
 TyConvArgs layer_args(const ffsva_tyolo* m, int l, int n, const __nv_bfloat16* in, __nv_bfloat16* out,
-                      int target, float thresh) {
+                      float thresh) {
   const Layer& L = m->L[l];
   TyConvArgs a{};
   a.in = in;
@@ -204,7 +204,7 @@ TyConvArgs layer_args(const ffsva_tyolo* m, int l, int n, const __nv_bfloat16* i
   a.leaky = l < 8 ? 1 : 0;
   a.M = n * L.Ho * L.Ho;
   a.head = l == 8 ? 1 : 0;
-  a.target = target;
+  a.frames = m->d_frames;
   a.thresh = thresh;
   a.counts = m->d_counts;
   return a;
@@ -212,13 +212,13 @@ TyConvArgs layer_args(const ffsva_tyolo* m, int l, int n, const __nv_bfloat16* i
 
 // Resize + layers [0, upto] for frames [0, n) (n <= cap), on stream st. ev (optional): 11 events around the
 // resize and each layer. *out_buf receives the activation buffer holding the last layer's output.
-ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, int n, int upto, int target, float thresh,
-                       cudaStream_t st, cudaEvent_t* ev, int* out_buf = nullptr) {
+ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, const int32_t* targets, int n, int upto,
+                       float thresh, cudaStream_t st, cudaEvent_t* ev, int* out_buf = nullptr) {
   DeviceCtx* ctx = m->ctx;
   int max_row = 0;
   for (int i = 0; i < n; ++i) {
     const ffsva_stream_desc& d = frames[i].stream->desc;
-    m->h_frames[i] = TyFrame{frames[i].pixels, d.row_pitch, d.width, d.height};
+    m->h_frames[i] = TyFrame{frames[i].pixels, d.row_pitch, d.width, d.height, targets ? targets[i] : 0, 0};
     max_row = std::max(max_row, 3 * d.width);
   }
   cudaError_t e = cudaMemcpyAsync(m->d_frames, m->h_frames, sizeof(TyFrame) * n, cudaMemcpyHostToDevice, st);
@@ -231,7 +231,7 @@ ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, int n, int upt
   if (ev) cudaEventRecord(ev[1], st);
   int cur = 0;
   for (int l = 0; l <= upto; ++l) {
-    const TyConvArgs a = layer_args(m, l, n, m->d_act[cur], m->d_act[cur ^ 1], target, thresh);
+    const TyConvArgs a = layer_args(m, l, n, m->d_act[cur], m->d_act[cur ^ 1], thresh);
     if ((e = launch_tyolo_conv(a, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO conv layer");
     g_launches += 1;
     cur ^= 1;
@@ -321,11 +321,26 @@ FFSVA_API ffsva_status ffsva_tyolo_run(ffsva_tyolo* m, const ffsva_frame* frames
   DeviceCtx* ctx = m->ctx;
   std::lock_guard<std::mutex> lk(ctx->mu);
   DeviceGuard g(ctx->device);
-  if ((st = ensure_workspace(m, n)) != FFSVA_OK) return st;
-  cudaStream_t cs = (cudaStream_t)cuda_stream;
+  std::vector<int32_t> targets((size_t)n, target_class);
+  return tyolo_run_unlocked(m, frames, n, targets.data(), thresh, number_of_objects, counts, pass, raw,
+                            (cudaStream_t)cuda_stream);
+}
+
+}  // extern "C"
+
+DeviceCtx* ffsva::tyolo_device_ctx(const ffsva_tyolo* m) { return m->ctx; }
+
+// The run itself, for callers that already hold the device lock (ffsva_tyolo_run, the online runtime's T-YOLO
+// cycle): frames in chunks of the workspace capacity, per-frame target classes.
+ffsva_status ffsva::tyolo_run_unlocked(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, const int32_t* targets,
+                                       float thresh, int32_t number_of_objects, int32_t* counts, uint8_t* pass,
+                                       float* raw, cudaStream_t cs) {
+  DeviceCtx* ctx = m->ctx;
+  ffsva_status st = ensure_workspace(m, n);
+  if (st != FFSVA_OK) return st;
   for (int32_t i0 = 0; i0 < n; i0 += m->cap) {
     const int cnt = std::min(m->cap, n - i0);
-    if ((st = run_chunk(m, frames + i0, cnt, 8, target_class, thresh, cs, nullptr)) != FFSVA_OK) return st;
+    if ((st = run_chunk(m, frames + i0, targets + i0, cnt, 8, thresh, cs, nullptr)) != FFSVA_OK) return st;
     cudaError_t e = cudaMemcpyAsync(m->h_counts, m->d_counts, 4 * (size_t)cnt, cudaMemcpyDeviceToHost, cs);
     if (e == cudaSuccess && raw) {  // [cnt][13][13][125] from the 128-wide padded rows
       e = cudaMemcpy2DAsync(raw + (size_t)i0 * kGrid * kGrid * 125, 125 * 4, m->d_raw, kHeadPad * 4, 125 * 4,
@@ -341,6 +356,8 @@ FFSVA_API ffsva_status ffsva_tyolo_run(ffsva_tyolo* m, const ffsva_frame* frames
   return FFSVA_OK;
 }
 
+extern "C" {
+
 FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, int32_t layer,
                                                 uint16_t* out, void* cuda_stream) {
   if (layer < -1 || layer > 7 || !out) return fail(FFSVA_EINVAL, "layer must be -1 (resized input) .. 7");
@@ -353,7 +370,7 @@ FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_fram
   if ((st = ensure_workspace(m, n)) != FFSVA_OK) return st;
   cudaStream_t cs = (cudaStream_t)cuda_stream;
   int buf = 0;
-  if ((st = run_chunk(m, frames, n, layer, 0, 0.2f, cs, nullptr, &buf)) != FFSVA_OK) return st;
+  if ((st = run_chunk(m, frames, nullptr, n, layer, 0.2f, cs, nullptr, &buf)) != FFSVA_OK) return st;
   const size_t bytes = layer < 0 ? (size_t)n * kIn * kIn * 4 * 2
                                  : (size_t)n * m->L[layer].Ho * m->L[layer].Ho * m->L[layer].Cout_pad * 2;
   cudaError_t e = cudaMemcpyAsync(out, m->d_act[buf], bytes, cudaMemcpyDeviceToHost, cs);
@@ -377,7 +394,7 @@ FFSVA_API ffsva_status ffsva_tyolo_profile(ffsva_tyolo* m, const ffsva_frame* fr
   for (auto& e : ev) cudaEventCreate(&e);
   double acc[10] = {0};
   for (int it = 0; it < iters && st == FFSVA_OK; ++it) {
-    st = run_chunk(m, frames, n, 8, 6, 0.2f, cs, ev);
+    st = run_chunk(m, frames, nullptr, n, 8, 0.2f, cs, ev);
     if (st != FFSVA_OK) break;
     cudaError_t e = cudaEventSynchronize(ev[10]);
     if (e != cudaSuccess) {

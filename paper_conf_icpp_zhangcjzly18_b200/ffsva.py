@@ -33,7 +33,8 @@ EXPORTS = ["ffsva_open_stream", "ffsva_set_reference", "ffsva_snm_load", "ffsva_
            "ffsva_version", "ffsva_sched_create", "ffsva_sched_push", "ffsva_sched_tick", "ffsva_sched_depth",
            "ffsva_sched_destroy", "ffsva_sched_set_policy", "ffsva_stream_image_bytes", "ffsva_stream_export",
            "ffsva_stream_import", "ffsva_sched_stream_load", "ffsva_sched_detach", "ffsva_tyolo_load",
-           "ffsva_tyolo_run", "ffsva_tyolo_layer_output", "ffsva_tyolo_profile", "ffsva_tyolo_destroy"]
+           "ffsva_tyolo_run", "ffsva_tyolo_layer_output", "ffsva_tyolo_profile", "ffsva_tyolo_destroy",
+           "ffsva_sched_set_tyolo"]
 
 
 class StreamDesc(ctypes.Structure):
@@ -42,7 +43,8 @@ class StreamDesc(ctypes.Structure):
                 ("snm_w", ctypes.c_int32), ("snm_h", ctypes.c_int32), ("delta_diff", ctypes.c_double),
                 ("c_low", ctypes.c_float), ("c_high", ctypes.c_float), ("filter_degree", ctypes.c_float),
                 ("snm_batch", ctypes.c_int32), ("q_sdd", ctypes.c_int32), ("q_snm", ctypes.c_int32),
-                ("distance", ctypes.c_int32), ("ref_mode", ctypes.c_int32)]
+                ("distance", ctypes.c_int32), ("ref_mode", ctypes.c_int32),
+                ("number_of_objects", ctypes.c_int32), ("target_class", ctypes.c_int32), ("q_tyolo", ctypes.c_int32)]
 
 
 # ffsva_distance / ffsva_ref_mode (include/ffsva.h)
@@ -60,13 +62,14 @@ class Frame(ctypes.Structure):
 
 class Result(ctypes.Structure):
     _fields_ = [("ssd", ctypes.c_uint64), ("sdd_pass", ctypes.c_uint8), ("snm_pass", ctypes.c_uint8),
-                ("snm_class", ctypes.c_uint8), ("pad", ctypes.c_uint8), ("logit", ctypes.c_float),
-                ("survivor_idx", ctypes.c_int32)]
+                ("snm_class", ctypes.c_uint8), ("tyolo_pass", ctypes.c_uint8), ("logit", ctypes.c_float),
+                ("survivor_idx", ctypes.c_int32), ("tyolo_count", ctypes.c_int32), ("reserved", ctypes.c_int32)]
 
 
 RESULT_DTYPE = np.dtype([("ssd", "<u8"), ("sdd_pass", "u1"), ("snm_pass", "u1"), ("snm_class", "u1"),
-                         ("pad", "u1"), ("logit", "<f4"), ("survivor_idx", "<i4")], align=True)
-assert RESULT_DTYPE.itemsize == ctypes.sizeof(Result) == 24
+                         ("tyolo_pass", "u1"), ("logit", "<f4"), ("survivor_idx", "<i4"), ("tyolo_count", "<i4"),
+                         ("reserved", "<i4")], align=True)
+assert RESULT_DTYPE.itemsize == ctypes.sizeof(Result) == 32
 
 EVENT_DTYPE = np.dtype([("stream", "<u8"), ("frame_no", "<i8"), ("result", RESULT_DTYPE)], align=True)
 
@@ -75,7 +78,9 @@ class TickInfo(ctypes.Structure):
     _fields_ = [("admitted", ctypes.c_int32), ("sdd_pass", ctypes.c_int32), ("snm_scored", ctypes.c_int32),
                 ("snm_batches", ctypes.c_int32), ("sdd_blocked", ctypes.c_int32), ("sdd_queued", ctypes.c_int64),
                 ("snm_queued", ctypes.c_int64), ("events_pending", ctypes.c_int64), ("sdd_ms", ctypes.c_float),
-                ("snm_ms", ctypes.c_float), ("host_ms", ctypes.c_float), ("pad", ctypes.c_int32)]
+                ("snm_ms", ctypes.c_float), ("host_ms", ctypes.c_float), ("pad", ctypes.c_int32),
+                ("tyolo_scored", ctypes.c_int32), ("snm_blocked", ctypes.c_int32), ("tyolo_queued", ctypes.c_int64),
+                ("tyolo_ms", ctypes.c_float), ("pad2", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -138,6 +143,7 @@ def lib():
             "ffsva_tyolo_layer_output": [vp, vp, i32, i32, vp, vp],
             "ffsva_tyolo_profile": [vp, vp, i32, i32, vp, vp],
             "ffsva_tyolo_destroy": [vp],
+            "ffsva_sched_set_tyolo": [vp, vp, i32, ctypes.c_float],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -366,10 +372,11 @@ class Context:
     def open_stream(self, width: int, height: int, row_pitch: int | None = None, delta_diff: float = 24.0,
                     c_low: float = 0.2, c_high: float = 0.8, filter_degree: float = 0.5, snm_batch: int = 30,
                     q_sdd: int = 2, q_snm: int = 10, sdd=(100, 100), distance: str = "mse",
-                    ref_mode: str = "background") -> Stream:
+                    ref_mode: str = "background", number_of_objects: int = 1, target_class: int = 6,
+                    q_tyolo: int = 2) -> Stream:
         d = StreamDesc(self.device, width, height, 3 * width if row_pitch is None else row_pitch, sdd[0], sdd[1],
                        sdd[0] // 2, sdd[1] // 2, delta_diff, c_low, c_high, filter_degree, snm_batch, q_sdd, q_snm,
-                       DISTANCES[distance], REF_MODES[ref_mode])
+                       DISTANCES[distance], REF_MODES[ref_mode], number_of_objects, target_class, q_tyolo)
         s = Stream(self, d)
         self.streams.append(s)
         return s
@@ -517,6 +524,12 @@ class Scheduler:
             return False
         _check(r, "ffsva_sched_detach")
         return True
+
+    def set_tyolo(self, model, num_tyolo: int = 4, thresh: float = 0.2) -> None:
+        """Attach the device's shared T-YOLO stage (a Tyolo, or None to detach): SNM survivors then wait in per-
+        stream T-YOLO queues and each tick takes at most num_tyolo frames per stream."""
+        _check(lib().ffsva_sched_set_tyolo(self.handle, model.handle if model is not None else None, num_tyolo,
+                                           thresh), "ffsva_sched_set_tyolo")
 
     def set_policy(self, policy: str) -> None:
         """'dynamic' (default), 'feedback' or 'static' (the §5.4 comparison mechanisms)."""

@@ -140,6 +140,37 @@ int main() {
     pops = p.pop_snm();
     CHECK(pops.size() == 1 && pops[0].size() == 1 && pops[0][0].frame_no == 3);
   }
+  {  // T-YOLO stage (L173, L209, L217): survivors of the SNM wait in the T-YOLO queue; each cycle takes at most
+     // num_t-yolo per stream; the SNM stage skips a stream whose T-YOLO queue holds more than q_ty = 2 frames
+    Policy p;
+    p.set_tyolo(true, 2);
+    int s0 = p.add_stream(100, 100, 5, 2), s1 = p.add_stream(100, 100, 5, 2);
+    for (int i = 0; i < 5; ++i) p.push(s0, fr(i));
+    p.push(s1, fr(100));
+    for (auto& f : p.admit_sdd(100, 100)) p.sdd_done(f, true);
+    auto pops = p.pop_snm();                       // s0: 5 frames, s1: 1 frame
+    CHECK(pops.size() == 2 && pops[0].size() == 5 && pops[1].size() == 1);
+    for (auto& pop : pops)  // frame 3 is dropped by the SNM: its result is final, it never queues
+      for (auto& f : pop) CHECK(p.snm_done(f, f.frame_no != 3) == (f.frame_no != 3));
+    CHECK(p.queued_ty() == 5);                     // s0: 0, 1, 2, 4; s1: 100
+    std::vector<QFrame> ty;
+    p.pop_ty(ty);
+    CHECK(ty.size() == 3 && ty[0].frame_no == 0 && ty[1].frame_no == 1 && ty[2].frame_no == 100);
+    CHECK(p.queued_ty() == 2);                     // s0: 2, 4 (depth 2, not over q_ty)
+    for (int i = 5; i < 8; ++i) p.push(s0, fr(i));
+    for (auto& f : p.admit_sdd(100, 100)) p.sdd_done(f, true);
+    pops = p.pop_snm();                            // s0 T-YOLO depth 2 <= 2: may pop
+    CHECK(pops.size() == 1 && pops[0].size() == 3);
+    for (auto& f : pops[0]) p.snm_done(f, true);   // T-YOLO depth 5 > 2
+    p.push(s0, fr(8));
+    for (auto& f : p.admit_sdd(100, 100)) p.sdd_done(f, true);
+    CHECK(p.pop_snm().empty());                    // blocked by the T-YOLO queue (L209)
+    CHECK(p.stream(s0).snm_blocked == 1 && p.stream(s0).max_ty == 5);
+    p.pop_ty(ty);
+    CHECK(ty.size() == 2 && ty[0].frame_no == 2 && ty[1].frame_no == 4);
+    p.pop_ty(ty);                                  // depth 1 <= 2: unblocked
+    CHECK(p.pop_snm().size() == 1);
+  }
   if (failures == 0) std::printf("ALL PASS\n");
   return failures == 0 ? 0 : 1;
 }

@@ -46,15 +46,15 @@ def test_library_is_sm100a(ff):
 
 
 def test_struct_layouts(ff):
-    assert ctypes.sizeof(ff.StreamDesc) == 80
+    assert ctypes.sizeof(ff.StreamDesc) == 96
     assert ctypes.sizeof(ff.Frame) == 24
-    assert ctypes.sizeof(ff.Result) == 24
+    assert ctypes.sizeof(ff.Result) == 32
 
 
 def _desc(ff, **kw):
     d = dict(device=0, width=640, height=360, row_pitch=1920, sdd_w=100, sdd_h=100, snm_w=50, snm_h=50,
              delta_diff=24.0, c_low=0.2, c_high=0.8, filter_degree=0.5, snm_batch=30, q_sdd=2, q_snm=10,
-             distance=0, ref_mode=0)
+             distance=0, ref_mode=0, number_of_objects=1, target_class=6, q_tyolo=2)
     d.update(kw)
     return ff.StreamDesc(*[d[k] for k, _ in ff.StreamDesc._fields_])
 
@@ -64,7 +64,8 @@ def _desc(ff, **kw):
                                  dict(snm_w=40), dict(sdd_w=101, snm_w=50), dict(snm_batch=0),
                                  dict(height=360 * 100), dict(device=-1), dict(c_high=1.5),
                                  dict(distance=3), dict(distance=-1), dict(ref_mode=2),
-                                 dict(distance=2, ref_mode=1)])
+                                 dict(distance=2, ref_mode=1), dict(number_of_objects=-1), dict(target_class=20),
+                                 dict(target_class=-1), dict(q_tyolo=-1)])
 def test_open_stream_rejects_bad_descriptors_before_cuda(ff, bad):
     h = ctypes.c_void_p()
     st = ff.lib().ffsva_open_stream(ctypes.byref(_desc(ff, **bad)), ctypes.byref(h))

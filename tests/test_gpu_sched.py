@@ -143,3 +143,76 @@ def test_fixed_size_batch_policies(env, policy):
         assert r["sdd_pass"] == int(synth.is_target(v, s, t)), (s, t)
     for c in cams:
         c.st.close()
+
+
+def test_online_three_stage_cascade_with_tyolo(env):
+    """f1 in the online runtime (§3.1 Fig. 2): SDD -> SNM -> T-YOLO queue -> T-YOLO. Every frame comes back
+    once; SNM survivors carry a T-YOLO count equal to the standalone stage's on the same frame and target class
+    (one frame also against the fp64 oracle), tyolo_pass = count >= NumberofObjects (L195), everything else -1;
+    the T-YOLO queue threshold (q_tyolo = 1) blocks the SNM stage (L209)."""
+    ff, ctx, dev = env
+    import torch
+    from paper_conf_icpp_zhangcjzly18_b200.ffsva import Scheduler
+    v = synth.Video(seed=71, width=640, height=360, period=4, on_len=3)
+    params = synth.tyolo_weights(5, target_class=14)
+    ty = ff.Tyolo(ctx, params)
+    cams = [Cam(ctx, v, s, dev, k_ref=2) for s in range(2)]
+    targets, noo = [14, 6], [2, 150]
+    for s, c in enumerate(cams):  # reopen with the T-YOLO fields (c_low = 0: every SDD survivor passes the SNM)
+        c.st.close()
+        c.st = ctx.open_stream(width=640, height=360, delta_diff=24.0, c_low=0.0, c_high=0.0, filter_degree=0.0,
+                               snm_batch=4, q_sdd=2, q_snm=4, number_of_objects=noo[s], target_class=targets[s],
+                               q_tyolo=1)
+        c.st.set_reference(torch.from_numpy(c.refs).to(dev))
+        c.st.snm_load(c.params)
+    T = 16
+    host = {s: c.host_frames(list(range(T))) for s, c in enumerate(cams)}
+    frames = {s: torch.from_numpy(host[s]).to(dev) for s in host}
+    sched = Scheduler(ctx, max_frames_per_tick=64, snm_slots=64)
+    sched.set_tyolo(ty, num_tyolo=1, thresh=0.2)
+    h2s = {c.st.handle: s for s, c in enumerate(cams)}
+    nxt, got, snm_blocked, scored = [0, 0], {}, 0, 0
+    for step in range(400):
+        items = [(cams[s].st, frames[s][t], t) for s in range(2) for t in range(nxt[s], min(T, nxt[s] + 3))]
+        if items:
+            acc = sched.push(items)
+            for (st, _, t), a in zip(items, acc):
+                s = h2s[st.handle]
+                if a and t == nxt[s]:
+                    nxt[s] += 1
+        ev, info = sched.tick()
+        snm_blocked += info["snm_blocked"]
+        scored += info["tyolo_scored"]
+        for e in ev:
+            key = (h2s[int(e["stream"])], int(e["frame_no"]))
+            assert key not in got
+            got[key] = e["result"]
+        if nxt == [T, T] and info["sdd_queued"] == 0 and info["snm_queued"] == 0 and info["tyolo_queued"] == 0 \
+                and info["events_pending"] == 0:
+            break
+    sched.set_tyolo(None)
+    sched.destroy()
+    assert len(got) == 2 * T
+    assert snm_blocked > 0, "the T-YOLO queue threshold never blocked the SNM stage"
+    reached = [(s, t) for (s, t), r in got.items() if r["snm_pass"]]
+    assert scored == len(reached) > 0
+    for (s, t), r in got.items():
+        assert r["sdd_pass"] == int(synth.is_target(v, s, t))
+        if r["snm_pass"]:
+            assert r["tyolo_count"] >= 0 and r["tyolo_pass"] == int(r["tyolo_count"] >= noo[s])
+        else:
+            assert r["tyolo_count"] == -1 and r["tyolo_pass"] == 0
+    for s in range(2):
+        ts = [t for (ss, t) in reached if ss == s]
+        if not ts:
+            continue
+        alone = ty.run([(cams[s].st, frames[s][t], t) for t in ts], target_class=targets[s], thresh=0.2)
+        assert [int(got[(s, t)]["tyolo_count"]) for t in ts] == alone["counts"].tolist()
+    s, t = reached[0]
+    want = orc.tyolo_forward(orc.resize(host[s][t], 640, 416, 416), params, bf16_emul=True)
+    sc = orc.tyolo_scores(want, targets[s])
+    near = int((np.abs(sc - 0.2) <= 2e-2).sum())
+    assert abs(int(got[(s, t)]["tyolo_count"]) - orc.tyolo_count(want, targets[s], 0.2)) <= near
+    for c in cams:
+        c.st.close()
+    ty.destroy()
