@@ -424,9 +424,22 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
         synth.frames_cuda(video, torch.full((32,), s, dtype=torch.int32, device=dev),
                           torch.arange(32, dtype=torch.int64, device=dev), r, H * P, P, ref=True)
         refs.append(r)
+    # full three-filter cascade (f1: SDD -> SNM -> T-YOLO, random-init T-YOLO weights) at these stream counts
+    ty_counts = []
+    for tok in args.online_tyolo.split(","):
+        tok = tok.strip()
+        if tok == "auto":
+            ty_counts.append(max(31, int(0.25 * value / 30)))
+        elif tok:
+            ty_counts.append(int(tok))
     results = []
     opened = []
-    for S in counts:
+    runs = [(S, False) for S in counts] + [(S, True) for S in ty_counts]
+    ty = None
+    if ty_counts:
+        import paper_conf_icpp_zhangcjzly18_b200 as ff
+        ty = ff.Tyolo(ctx, synth.tyolo_weights(video.seed))
+    for S, with_ty in runs:
         t_setup = time.perf_counter()
         while len(opened) < S:
             i = len(opened)
@@ -437,15 +450,20 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
             opened.append(st)
         setup_s = time.perf_counter() - t_setup
         res = run_paced(ctx, opened[:S], [pool[i % nc] for i in range(S)], pool.shape[1], args.online_seconds,
-                        cuda_stream=cs)
+                        cuda_stream=cs, tyolo=ty if with_ty else None)
         res["stream_setup_s"] = setup_s
         results.append(res)
     for st in opened:
         st.close()
         ctx.streams.remove(st)
-    best = max([r["streams"] for r in results if r["sustained"]], default=0)
+    if ty is not None:
+        ty.destroy()
+    best = max([r["streams"] for r in results if r["sustained"] and "stages" not in r], default=0)
+    best_ty = max([r["streams"] for r in results if r["sustained"] and "stages" in r], default=0)
     return {"runs": results, "max_sustained_streams_validated": best,
-            "policy": "q_sdd 2, q_snm 10, BatchSize 30 (PAPER.md L217, L219); latency budget p99 <= 1 s"}
+            "max_sustained_streams_validated_with_tyolo": best_ty,
+            "policy": "q_sdd 2, q_snm 10, q_tyolo 2, BatchSize 30, num_t-yolo 4 (PAPER.md L173, L217, L219); "
+                      "latency budget p99 <= 1 s"}
 
 
 def cpu_baseline(cfg, video, sids, pool, n_frames):
@@ -545,6 +563,9 @@ def main():
                     help="comma-separated stream counts for the paced online validation (config m2); 'auto' = "
                          "55%% of the measured frames/s / 30; empty to skip")
     ap.add_argument("--online-seconds", type=float, default=4.0)
+    ap.add_argument("--online-tyolo", default="auto",
+                    help="stream counts for a paced run of the full cascade with the T-YOLO stage (f1); 'auto' = "
+                         "25%% of the measured frames/s / 30; empty to skip")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")

@@ -15,8 +15,9 @@ import numpy as np
 
 
 def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s=0.010, cuda_stream=None,
-              latency_budget_s=1.0):
-    """streams[i]: ff.Stream; content[i]: (device frame tensor [n_content_frames, H, pitch]).
+              latency_budget_s=1.0, tyolo=None, num_tyolo=4):
+    """streams[i]: ff.Stream; content[i]: (device frame tensor [n_content_frames, H, pitch]). tyolo: a Tyolo to run
+    the full three-filter cascade (SDD -> SNM -> T-YOLO, f1) instead of SDD -> SNM.
 
     Returns a dict of latency percentiles, refusals, backlog and throughput."""
     import torch
@@ -34,6 +35,9 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
     pushed = np.zeros(S, np.int64)          # frames handed to (and accepted by) the scheduler
     max_frames_tick = max(1024, int(S * fps * 0.25))
     sched = Scheduler(ctx, max_frames_per_tick=max_frames_tick, snm_slots=max(4096, S * 12))
+    if tyolo is not None:
+        sched.set_tyolo(tyolo, num_tyolo=num_tyolo)
+    ty_scored = 0
     lat = []
     refused = 0
     done = 0
@@ -69,6 +73,7 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
             t_push = time.perf_counter()
             ev, info = sched.tick(cuda_stream)
             ticks += 1
+            ty_scored += info["tyolo_scored"]
             t_done = time.perf_counter()
             tim[0] += t_push - now
             tim[1] += info["sdd_ms"] / 1e3
@@ -93,6 +98,9 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
            "latency_max_s": float(L.max()),
            "mean_ms_per_tick": {"push_py": 1e3 * tim[0] / max(1, ticks), "sdd_cycle": 1e3 * tim[1] / max(1, ticks),
                                 "snm_cycle": 1e3 * tim[2] / max(1, ticks), "tick_call": 1e3 * tim[3] / max(1, ticks)}}
+    if tyolo is not None:
+        res["stages"] = "SDD -> SNM -> T-YOLO (f1)"
+        res["tyolo_scored"] = int(ty_scored)
     res["sustained"] = bool(res["latency_p99_s"] <= latency_budget_s and backlog_end <= S * 2
                             and done >= 0.9 * S * fps * (seconds - latency_budget_s))
     return res
@@ -165,3 +173,4 @@ def run_unpaced(ctx, streams, content, n_content_frames, seconds, policy="dynami
             "latency_p50_ms": 1e3 * float(np.percentile(L, 50)), "latency_p99_ms": 1e3 * float(np.percentile(L, 99)),
             "snm_scored": int(scored), "snm_batches": int(pops),
             "mean_snm_batch": scored / pops if pops else 0.0}
+
