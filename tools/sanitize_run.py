@@ -52,11 +52,17 @@ def main():
     assert np.array_equal(r5["ssd"][8:], r1["ssd"])
     for st in extra:
         st.close()
+    # T-YOLO stage (f1): standalone on 3 frames, then attached to the online runtime (three-stage cascade)
+    ty = ff.Tyolo(ctx, synth.tyolo_weights(5))
+    r6 = ty.run([(streams[i % 2], d[i], i) for i in range(3)], raw=True)
+    assert r6["counts"].shape == (3,)
     sched = Scheduler(ctx, max_frames_per_tick=4, snm_slots=8)
+    sched.set_tyolo(ty, num_tyolo=1)
     for t in range(6):
         sched.push([(streams[i % 2], d[i], i) for i in range(8)])
         sched.tick(s)
     sched.destroy()
+    ty.destroy()
     ctx.close()
     torch.cuda.synchronize()
     print("OK")
