@@ -31,6 +31,7 @@ using namespace ptx;
 
 constexpr int kConvThreads = 320;  // warps 0-3: A gather, 4: TMEM + MMA issue, 5: B copies, 6-9: epilogue
 constexpr int kATile = 128 * 128;  // one stage of A for one chain: 128 rows x 64 bf16
+constexpr int kMaxAccBufs = 8;     // TMEM accumulator buffers (small N tiles keep several tiles in flight)
 
 // byte offset of (K group g of 8 bf16, row r) in a 128-row K-major no-swizzle tile: core matrices of 8 rows x 16 B,
 // K-adjacent core matrices 2048 B apart (LBO), 8-row groups 128 B apart (SBO)
@@ -159,9 +160,9 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
   uint8_t* As = sm;
   uint8_t* Bs = sm + (size_t)S * stage_a;
   uint64_t* bars = reinterpret_cast<uint64_t*>(Bs + (size_t)S * stage_b);
-  uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 2 * S + 4);
+  uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 2 * S + 2 * kMaxAccBufs);
   const uint32_t full0 = smem_addr(bars), empty0 = full0 + 8 * S;
-  const uint32_t accf0 = full0 + 16 * S, acce0 = accf0 + 16;  // acc_full[2], acc_empty[2]
+  const uint32_t accf0 = full0 + 16 * S, acce0 = accf0 + 8 * kMaxAccBufs;  // acc_full[NB], acc_empty[NB]
   const uint32_t As0 = smem_addr(As), Bs0 = smem_addr(Bs);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int rows_per_tile = 128 * MS;
@@ -172,7 +173,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
       mbar_init(full0 + 8 * s, 129);  // 128 gather threads + the weight copy's expect_tx arrival
       mbar_init(empty0 + 8 * s, 1);
     }
-    for (int b = 0; b < 2; ++b) {
+    for (int b = 0; b < NB; ++b) {
       mbar_init(accf0 + 8 * b, 1);
       mbar_init(acce0 + 8 * b, 128);
     }
@@ -289,17 +290,25 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
         if (rv) decode_row(a, m, n, oy, ox);
         const uint32_t trow = tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(b * acc_cols + i * nq * NT);
         for (int c0 = 0; c0 < NT; c0 += 16) {
-          uint32_t rr[16];
           float v[16];
-          tmem_ld16(trow + (uint32_t)c0, rr);
-          tmem_wait_ld(rr);
+          if (nq == 4) {  // the four pool chains: all four loads in flight, one wait
+            uint32_t r0[16], r1[16], r2[16], r3[16];
+            tmem_ld16(trow + (uint32_t)c0, r0);
+            tmem_ld16(trow + (uint32_t)(NT + c0), r1);
+            tmem_ld16(trow + (uint32_t)(2 * NT + c0), r2);
+            tmem_ld16(trow + (uint32_t)(3 * NT + c0), r3);
+            tmem_wait_ld2(r0, r1);
+            reg_fence2(r2, r3);
 #pragma unroll
-          for (int k = 0; k < 16; ++k) v[k] = __uint_as_float(rr[k]);
-          for (int q = 1; q < nq; ++q) {
-            tmem_ld16(trow + (uint32_t)(q * NT + c0), rr);
+            for (int k = 0; k < 16; ++k)
+              v[k] = fmaxf(fmaxf(__uint_as_float(r0[k]), __uint_as_float(r1[k])),
+                           fmaxf(__uint_as_float(r2[k]), __uint_as_float(r3[k])));
+          } else {
+            uint32_t rr[16];
+            tmem_ld16(trow + (uint32_t)c0, rr);
             tmem_wait_ld(rr);
 #pragma unroll
-            for (int k = 0; k < 16; ++k) v[k] = fmaxf(v[k], __uint_as_float(rr[k]));
+            for (int k = 0; k < 16; ++k) v[k] = __uint_as_float(rr[k]);
           }
           if (!rv) continue;
           const float* bias = a.bias + cbase + c0;
@@ -436,7 +445,7 @@ __global__ void __launch_bounds__(kResizeThreads) tyolo_resize_kernel(const TyFr
 }  // namespace
 
 int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT) {
-  return stages * (a_tiles * kATile + b_tiles * NT * 128) + 8 * (2 * stages + 4) + 16;
+  return stages * (a_tiles * kATile + b_tiles * NT * 128) + 8 * (2 * stages + 2 * kMaxAccBufs) + 16;
 }
 
 cudaError_t tyolo_configure() {

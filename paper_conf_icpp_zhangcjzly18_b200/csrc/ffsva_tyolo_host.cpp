@@ -95,7 +95,8 @@ void build_layers(ffsva_tyolo* m) {
     const int a_tiles = L.msub * (L.patch ? 1 : L.nq), b_tiles = L.patch ? L.nq : 1;
     const int stage = a_tiles * 128 * 128 + b_tiles * L.NT * 128;
     L.stages = std::max(2, std::min(8, (227 * 1024 - 1024) / stage));
-    L.acc_bufs = 2 * L.msub * L.nq * L.NT <= 512 ? 2 : 1;  // double-buffered accumulator when it fits in TMEM
+    // as many TMEM accumulator buffers as fit (up to 8): the epilogue of earlier tiles overlaps later mainloops
+    L.acc_bufs = std::max(1, std::min(8, 512 / (L.msub * L.nq * L.NT)));
     L.tmem_cols = pow2_at_least(L.acc_bufs * L.msub * L.nq * L.NT);
     L.H = H;
     L.Ho = L.pool == 1 ? H / 2 : H;
