@@ -148,12 +148,12 @@ __device__ __forceinline__ void cp_async_wait_n(int n) {
   }
 }
 
-template <int MS>
+template <int MS, int NQ, bool PATCH>
 __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs a) {
   extern __shared__ __align__(1024) uint8_t sm[];
-  const int S = a.stages, nq = a.nq, NT = a.NT, KC = a.kchunks, NB = a.acc_bufs;
-  const int a_per_sub = a.patch ? 1 : nq;
-  const int b_tiles = a.patch ? nq : 1;
+  const int S = a.stages, nq = NQ, NT = a.NT, KC = a.kchunks, NB = a.acc_bufs;
+  const int a_per_sub = PATCH ? 1 : nq;
+  const int b_tiles = PATCH ? nq : 1;
   const uint32_t stage_a = (uint32_t)(MS * a_per_sub) * kATile;
   const uint32_t b_tile = (uint32_t)NT * 128, stage_b = (uint32_t)b_tiles * b_tile;
   const int acc_cols = MS * nq * NT;  // per accumulator buffer
@@ -210,7 +210,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
         for (int i = 0; i < MS; ++i) {
           const __nv_bfloat16* img = a.in + (int64_t)n[i] * a.H * a.W * a.Cp;
           const uint32_t base = As0 + (uint32_t)s * stage_a + (uint32_t)(i * a_per_sub) * kATile;
-          if (a.patch) {
+          if (PATCH) {
             gather_patch(a, img, rv[i], oy[i], ox[i], j, base, r);
           } else {
             for (int q = 0; q < nq; ++q) {
@@ -233,8 +233,14 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
     for (int h = g - lag < 0 ? 0 : g - lag; h < g; ++h) mbar_arrive(full0 + 8 * (h % S));
   } else if (warp == 4) {
     // ---------------- MMA issue (one thread)
+    // Descriptors are built once; per MMA only their start-address fields advance (byte offset >> 4 added to the
+    // low 14 bits, which cannot carry: shared addresses stay below 256 KB), so the single issuing thread spends a
+    // few instructions per MMA instead of rebuilding two 64-bit descriptors.
     if (lane == 0) {
       const uint32_t idesc = idesc_bf16(128, NT);
+      const uint64_t a_base = umma_desc(As0, 2048, 128), b_base = umma_desc(Bs0, (uint32_t)NT * 16, 128);
+      const uint32_t a_tile16 = (uint32_t)kATile >> 4, b_tile16 = b_tile >> 4, b_ks16 = (uint32_t)(2 * NT * 16) >> 4;
+      const int ksteps = a.ksteps;
       int g = 0, it = 0;
       for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++it) {
         const int b = it % NB;
@@ -245,15 +251,18 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
           const int s = g % S;
           mbar_wait(full0 + 8 * s, (g / S) & 1);
           fence_after();
+          const uint64_t a_s = a_base + (((uint32_t)s * stage_a) >> 4), b_s = b_base + (((uint32_t)s * stage_b) >> 4);
+#pragma unroll
           for (int i = 0; i < MS; ++i)
-            for (int q = 0; q < nq; ++q) {
-              const uint32_t at = As0 + (uint32_t)s * stage_a + (uint32_t)(i * a_per_sub + (a.patch ? 0 : q)) * kATile;
-              const uint32_t bt = Bs0 + (uint32_t)s * stage_b + (uint32_t)(a.patch ? q : 0) * b_tile;
-              for (int ks = 0; ks < a.ksteps; ++ks) {
-                const uint64_t ad = umma_desc(at + (uint32_t)ks * 4096u, 2048, 128);
-                const uint64_t bd = umma_desc(bt + (uint32_t)(ks * 2 * NT * 16), NT * 16, 128);
-                mma_bf16(acc + (uint32_t)((i * nq + q) * NT), ad, bd, idesc, (j > 0 || ks > 0) ? 1u : 0u);
-              }
+#pragma unroll
+            for (int q = 0; q < NQ; ++q) {
+              const uint64_t ad = a_s + (uint64_t)((i * (PATCH ? 1 : NQ) + (PATCH ? 0 : q)) * a_tile16);
+              const uint64_t bd = b_s + (uint64_t)((PATCH ? q : 0) * b_tile16);
+              const uint32_t d = acc + (uint32_t)((i * NQ + q) * NT);
+#pragma unroll
+              for (int ks = 0; ks < 4; ++ks)
+                if (ks < ksteps)
+                  mma_bf16(d, ad + (uint64_t)(ks * 256), bd + (uint64_t)(ks * b_ks16), idesc, (j > 0 || ks > 0) ? 1u : 0u);
             }
           mma_commit(empty0 + 8 * s);
         }
@@ -291,7 +300,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
         const uint32_t trow = tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(b * acc_cols + i * nq * NT);
         for (int c0 = 0; c0 < NT; c0 += 16) {
           float v[16];
-          if (nq == 4) {  // the four pool chains: all four loads in flight, one wait
+          if (NQ == 4) {  // the four pool chains: all four loads in flight, one wait
             uint32_t r0[16], r1[16], r2[16], r3[16];
             tmem_ld16(trow + (uint32_t)c0, r0);
             tmem_ld16(trow + (uint32_t)(NT + c0), r1);
@@ -449,9 +458,14 @@ int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT) {
 }
 
 cudaError_t tyolo_configure() {
-  cudaError_t e = cudaFuncSetAttribute(tyolo_conv_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+  const int smem = 227 * 1024;
+  cudaError_t e = cudaFuncSetAttribute(tyolo_conv_kernel<1, 4, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(tyolo_conv_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    e = cudaFuncSetAttribute(tyolo_conv_kernel<1, 4, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tyolo_conv_kernel<2, 1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(tyolo_conv_kernel<1, 1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   return e;
 }
 
@@ -461,8 +475,12 @@ cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st) {
   const unsigned grid = (unsigned)(tiles < a.grid ? tiles : a.grid);
   const int a_tiles = a.msub * (a.patch ? 1 : a.nq), b_tiles = a.patch ? a.nq : 1;
   const int smem = tyolo_conv_smem_bytes(a.stages, a_tiles, b_tiles, a.NT);
-  if (a.msub == 2) tyolo_conv_kernel<2><<<grid, kConvThreads, smem, st>>>(a);
-  else tyolo_conv_kernel<1><<<grid, kConvThreads, smem, st>>>(a);
+  // the three shapes of tiny-yolo-voc: pool layers by patch (L1-L3) or per-position gather (L4, L5), and the 13x13
+  // layers with two row halves (L6-L9); msub 1 for the A/B knob
+  if (a.nq == 4 && a.patch) tyolo_conv_kernel<1, 4, true><<<grid, kConvThreads, smem, st>>>(a);
+  else if (a.nq == 4) tyolo_conv_kernel<1, 4, false><<<grid, kConvThreads, smem, st>>>(a);
+  else if (a.msub == 2) tyolo_conv_kernel<2, 1, false><<<grid, kConvThreads, smem, st>>>(a);
+  else tyolo_conv_kernel<1, 1, false><<<grid, kConvThreads, smem, st>>>(a);
   return cudaGetLastError();
 }
 
