@@ -1,16 +1,17 @@
 #!/bin/bash
-# Round evidence on one B200: GPU tests, smoke, default bench, ncu launch list + full captures, sanitizers.
-# Everything lands in gpurun_out/; tools/summarize_evidence.py turns it into profiles/<round>/.
+# Round evidence on one B200: GPU tests, smoke, default bench (M2) + M3 / SNM / T-YOLO configs, ncu launch lists and
+# --set full captures (K1 M2/M3, K4, T-YOLO layers), sanitizers. Everything lands in gpurun_out/;
+# tools/summarize_evidence.py turns it into profiles/<round>/.
 cd "$(dirname "$0")/.."
 mkdir -p gpurun_out
 nvidia-smi > gpurun_out/nvidia-smi.txt 2>&1
 timeout 600 python __graft_entry__.py > gpurun_out/build.log 2>&1 || { echo BUILD FAILED; tail -30 gpurun_out/build.log; exit 1; }
-timeout 1200 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/pytest_gpu.log
+timeout 1500 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/pytest_gpu.log
 timeout 300 python __graft_entry__.py smoke > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"; tail -1 gpurun_out/smoke.log
-timeout 1200 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?"
-for tool in memcheck racecheck synccheck; do
-  timeout 900 compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_run.py > gpurun_out/sanitize_$tool.log 2>&1
-  echo "sanitize $tool rc=$?"; tail -2 gpurun_out/sanitize_$tool.log
+timeout 1500 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?"
+for CFG in m3 snm tyolo; do
+  timeout 900 python bench.py --config $CFG --steps ${STEPS:-200} --warmup 5 --online "" > gpurun_out/bench_$CFG.json 2> gpurun_out/bench_$CFG.err
+  echo "bench $CFG rc=$?"
 done
 for CFG in m2 m3; do
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"sdd|compact|snm" -s 60 -c 60 --csv \
@@ -24,3 +25,11 @@ done
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:snm_kernel -s 10 -c 1 -o gpurun_out/prof_k4_snm -f \
   python bench.py --config snm --steps 20 --warmup 3 --no-e2e --no-cpu-baseline --online "" > gpurun_out/ncu_full_k4.log 2>&1
 echo "ncu full k4 rc=$?"
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:tyolo --csv --log-file gpurun_out/launches_tyolo.csv \
+  python tools/tyolo_profile.py --frames 256 --iters 1 > /dev/null 2>&1; echo "ncu list tyolo rc=$?"
+LAYERS="1 2 8" bash tools/tyolo_ncu.sh
+timeout 300 python tools/tyolo_profile.py --frames 256 --iters 10 > gpurun_out/tyolo_profile.log 2>&1
+for tool in memcheck synccheck racecheck; do
+  timeout ${SAN_TIMEOUT:-1200} compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_run.py > gpurun_out/sanitize_$tool.log 2>&1
+  echo "sanitize $tool rc=$?"; tail -2 gpurun_out/sanitize_$tool.log
+done

@@ -61,8 +61,8 @@ def main():
     rnd = sys.argv[1] if len(sys.argv) > 1 else "r01"
     dst = os.path.join(ROOT, "profiles", rnd)
     os.makedirs(dst, exist_ok=True)
-    for f in ["bench.json", "bench.err", "bench_tyolo.json", "tyolo_profile.json", "pytest_gpu.log", "smoke.log",
-              "nvidia-smi.txt"] + \
+    for f in ["bench.json", "bench.err", "bench_m3.json", "bench_snm.json", "bench_tyolo.json", "tyolo_profile.json",
+              "tyolo_profile.log", "pytest_gpu.log", "smoke.log", "nvidia-smi.txt"] + \
             [os.path.basename(p) for p in glob.glob(os.path.join(OUT, "sanitize_*.log"))]:
         p = os.path.join(OUT, f)
         if os.path.exists(p):
