@@ -509,6 +509,23 @@ def run_reference(args, cfg, ws, rank):
     from synth import synth
     W, H = cfg["W"], cfg["H"]
     video = synth.Video(seed=cfg["seed"], width=W, height=H, period=cfg["period"], on_len=cfg["on_len"])
+    if args.config == "tyolo":  # the f1 stage: one frame (resize + nine layers in fp64 + count) per step
+        params = synth.tyolo_weights(cfg["seed"])
+        imgs = [orc.resize(synth.frame(video, 0, t), W, 416, 416) for t in range(4)]
+        for i in range(args.warmup):
+            orc.tyolo_count(orc.tyolo_forward(imgs[i % 4], params), 6)
+        t0 = time.perf_counter()
+        for i in range(args.steps):
+            orc.tyolo_count(orc.tyolo_forward(imgs[i % 4], params), 6)
+        dt = time.perf_counter() - t0
+        value = args.steps / dt
+        return {"metric": "T-YOLO frames/sec (f1 stage, 416x416 tiny-yolo-voc)", "value": value, "unit": "frames/s",
+                "n_gpus": ws, "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3 / args.steps,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "impl": "reference", "config": {"workload": cfg["desc"], "config_id": args.config},
+                "cpu_baseline": {"value": value, "unit": "frames/s", "cores": 1, "kind": "oracle",
+                                 "sample": "1 frame per step (resize + nine layers in fp64 + count)"},
+                "e2e": {"value": value, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     S = min(cfg["streams"], 8)
     refs, params = {}, {}
     for s in range(S):

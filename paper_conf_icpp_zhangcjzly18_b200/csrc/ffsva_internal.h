@@ -165,6 +165,7 @@ struct TyConvArgs {
   int32_t msub;              // 128-row halves per tile sharing each weight stage (1 or 2)
   int32_t patch;             // pool layers: A row = the pooled pixel's 4x4 input patch, weights per pool position
   int32_t lag;               // K steps of gathers in flight per producer thread before it publishes (1 .. S-1)
+  int32_t cp_shift;          // log2(Cp)
   int32_t head;              // head: count boxes of frame f's target class scoring > thresh into counts[f]
   const TyFrame* frames;     // head: per-frame target classes
   float thresh;

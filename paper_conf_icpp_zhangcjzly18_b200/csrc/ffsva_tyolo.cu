@@ -39,61 +39,6 @@ __device__ __forceinline__ uint32_t a_off(int g, int r) {
   return (uint32_t)(g * 2048 + (r >> 3) * 128 + (r & 7) * 16);
 }
 
-// The A rows of one K step (chunk j) for output row r whose conv pixel is (cy, cx).
-__device__ __forceinline__ void gather(const TyConvArgs& a, const __nv_bfloat16* img, bool rv, int cy, int cx, int j,
-                                       uint32_t dst, int r) {
-  const int H = a.H, W = a.W, Cp = a.Cp;
-  if (Cp >= 64) {
-    int t, c0;
-    if (a.ksize == 3) {
-      const int cpt = Cp >> 6;
-      t = j / cpt;
-      c0 = (j - t * cpt) << 6;
-    } else {
-      t = 4;
-      c0 = j << 6;
-    }
-    const int sy = cy + t / 3 - 1, sx = cx + t % 3 - 1;
-    const bool v = rv && sy >= 0 && sy < H && sx >= 0 && sx < W;
-    const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * Cp + c0 : a.in;
-#pragma unroll
-    for (int g = 0; g < 8; ++g) cp_async16(dst + a_off(g, r), src + 8 * g, v);
-  } else if (Cp >= 16) {  // 16 or 32 channels: 4 or 2 taps per K step
-    const int tpc = 64 / Cp, upt = Cp >> 3;
-    for (int i = 0; i < tpc; ++i) {
-      const int t = j * tpc + i;
-      const int sy = cy + t / 3 - 1, sx = cx + t % 3 - 1;
-      const bool v = rv && t < 9 && sy >= 0 && sy < H && sx >= 0 && sx < W;
-      const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * Cp : a.in;
-      for (int u = 0; u < upt; ++u) cp_async16(dst + a_off(i * upt + u, r), src + 8 * u, v);
-    }
-  } else {  // 4 channels (RGB + zero): two taps per 16-byte K group, all nine taps in one step
-#pragma unroll
-    for (int g = 0; g < 8; ++g)
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        const int t = 2 * g + h;
-        const int sy = cy + t / 3 - 1, sx = cx + t % 3 - 1;
-        const bool v = rv && t < 9 && sy >= 0 && sy < H && sx >= 0 && sx < W;
-        const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * 4 : a.in;
-        cp_async8(dst + a_off(g, r) + 8 * h, src, v);
-      }
-  }
-}
-
-__device__ __forceinline__ void conv_pixel(const TyConvArgs& a, int oy, int ox, int q, int& cy, int& cx) {
-  if (a.pool == 1) {
-    cy = 2 * oy + (q >> 1);
-    cx = 2 * ox + (q & 1);
-  } else if (a.pool == 2) {
-    cy = oy + (q >> 1);
-    cx = ox + (q & 1);
-  } else {
-    cy = oy;
-    cx = ox;
-  }
-}
-
 // Decode output row m of the layer into (frame, oy, ox).
 __device__ __forceinline__ void decode_row(const TyConvArgs& a, int m, int& n, int& oy, int& ox) {
   const int hw = a.Ho * a.Wo;
@@ -103,30 +48,78 @@ __device__ __forceinline__ void decode_row(const TyConvArgs& a, int m, int& n, i
   ox = rem - oy * a.Wo;
 }
 
-// Patch gather (pool layers with few input channels): the A row of pooled pixel (oy, ox) is its 4x4 input patch
-// (rows 2oy-1 .. 2oy+2, columns 2ox-1 .. 2ox+2) x Cp channels, pixel-major; K step j holds 64 of its values. The
-// four pool positions then differ only in their weights (the 3x3 kernel placed at offset (a, b) of the 4x4 patch),
-// so one A tile feeds all four accumulator chains.
-__device__ __forceinline__ void gather_patch(const TyConvArgs& a, const __nv_bfloat16* img, bool rv, int oy, int ox,
-                                             int j, uint32_t dst, int r) {
-  const int H = a.H, W = a.W, Cp = a.Cp;
-  if (Cp == 4) {  // all 16 patch pixels in one K step, two pixels per 16-byte K group
+// Gather state of one output row for one tile: the address of its 4x4 input window's origin — rows ry0 .. ry0+3,
+// columns rx0 .. rx0+3 with (ry0, rx0) = (2oy-1, 2ox-1) for pool layers (the four pool positions' 3x3 taps and the
+// 4x4 patch all lie in it) and (oy-1, ox-1) otherwise — and which window rows / columns lie inside the image.
+// Every K group then costs a few instructions: validity = three mask bits, address = origin + two constant offsets.
+struct RowWin {
+  const char* p0;  // window origin (may point outside the image; only dereferenced for in-image pixels)
+  uint32_t mask;   // bit 16: row exists; bits 0-3: window rows inside; bits 4-7: window columns inside
+};
+
+__device__ __forceinline__ RowWin row_window(const TyConvArgs& a, int m) {
+  RowWin w{reinterpret_cast<const char*>(a.in), 0u};
+  if (m >= a.M) return w;
+  int n, oy, ox;
+  decode_row(a, m, n, oy, ox);
+  const int sc = a.pool == 1 ? 2 : 1, ry0 = sc * oy - 1, rx0 = sc * ox - 1;
+  uint32_t mask = 1u << 16;
 #pragma unroll
-    for (int p = 0; p < 16; ++p) {
-      const int sy = 2 * oy - 1 + (p >> 2), sx = 2 * ox - 1 + (p & 3);
-      const bool v = rv && sy >= 0 && sy < H && sx >= 0 && sx < W;
-      cp_async8(dst + a_off(p >> 1, r) + 8 * (p & 1), v ? img + ((int64_t)sy * W + sx) * 4 : a.in, v);
-    }
+  for (int u = 0; u < 4; ++u) {
+    if ((unsigned)(ry0 + u) < (unsigned)a.H) mask |= 1u << u;
+    if ((unsigned)(rx0 + u) < (unsigned)a.W) mask |= 1u << (4 + u);
+  }
+  w.p0 = reinterpret_cast<const char*>(a.in) + (((int64_t)n * a.H + ry0) * a.W + rx0) * a.Cp * 2;
+  w.mask = mask;
+  return w;
+}
+
+// One piece of a row's K step: window pixel (du, dv) at byte offset off within it.
+__device__ __forceinline__ void gather_piece(const TyConvArgs& a, const RowWin& w, int du, int dv, int off,
+                                             int64_t rowb, int pixb, uint32_t dst, bool half, bool ok = true) {
+  const bool v = ok && ((w.mask >> 16) & (w.mask >> du) & (w.mask >> (4 + dv)) & 1u);
+  const void* src = v ? (const void*)(w.p0 + du * rowb + dv * pixb + off) : (const void*)a.in;
+  if (half) cp_async8(dst, src, v);
+  else cp_async16(dst, src, v);
+}
+
+// Patch mode (pool layers with few input channels): the A row of pooled pixel (oy, ox) is its 4x4 input patch
+// (the window) x Cp channels, pixel-major; K step j holds 64 of its values. The four pool positions then differ
+// only in their weights (the 3x3 kernel placed at offset (a, b) of the patch), so one A tile feeds all four
+// accumulator chains.
+__device__ __forceinline__ void gather_patch(const TyConvArgs& a, const RowWin& w, int j, int64_t rowb, int pixb,
+                                             uint32_t dst, int r) {
+  if (a.Cp == 4) {  // all 16 patch pixels in one K step, two 8-byte pixels per 16-byte K group
+#pragma unroll
+    for (int p = 0; p < 16; ++p) gather_piece(a, w, p >> 2, p & 3, 0, rowb, pixb, dst + a_off(p >> 1, r) + 8 * (p & 1), true);
   } else {  // Cp = 8 * upp channels: 64 / Cp pixels per K step, upp 16-byte units each
-    const int ppc = 64 / Cp, upp = Cp >> 3;
+    const int ppc = 64 / a.Cp, upp = a.Cp >> 3;
     for (int pl = 0; pl < ppc; ++pl) {
       const int p = j * ppc + pl;
-      const int sy = 2 * oy - 1 + (p >> 2), sx = 2 * ox - 1 + (p & 3);
-      const bool v = rv && sy >= 0 && sy < H && sx >= 0 && sx < W;
-      const __nv_bfloat16* src = v ? img + ((int64_t)sy * W + sx) * Cp : a.in;
-      for (int u = 0; u < upp; ++u) cp_async16(dst + a_off(pl * upp + u, r), src + 8 * u, v);
+      for (int u = 0; u < upp; ++u)
+        gather_piece(a, w, p >> 2, p & 3, 16 * u, rowb, pixb, dst + a_off(pl * upp + u, r), false);
     }
   }
+}
+
+// Per-position / plain gather (Cp a multiple of 64): K step j is one tap (dy, dx) and 64 channels; pool position
+// (qa, qb) shifts it inside the window.
+__device__ __forceinline__ void gather_tap(const TyConvArgs& a, const RowWin& w, int j, int qa, int qb, int64_t rowb,
+                                           int pixb, uint32_t dst, int r) {
+  int t, c0;
+  if (a.ksize == 1) {
+    t = 4;
+    c0 = j << 6;
+  } else {
+    const int sh = a.cp_shift - 6;  // K steps per tap = Cp / 64
+    t = j >> sh;
+    c0 = (j - (t << sh)) << 6;
+  }
+  const int du = qa + t / 3, dv = qb + t % 3;
+  const bool v = (w.mask >> 16) & (w.mask >> du) & (w.mask >> (4 + dv)) & 1u;
+  const char* src = v ? w.p0 + du * rowb + dv * pixb + c0 * 2 : reinterpret_cast<const char*>(a.in);
+#pragma unroll
+  for (int g = 0; g < 8; ++g) cp_async16(dst + a_off(g, r), src + 16 * g, v);
 }
 
 // Persistent, warp-specialised: each CTA walks tiles t = blockIdx.x, + gridDim.x, ... A tile = msub x 128 output
@@ -193,31 +186,25 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
     // slack; lag = 1 measured best (profiles/r01/tyolo_ab.md).
     const int r = tid, lag = a.lag < 1 ? 1 : (a.lag > S - 1 ? S - 1 : a.lag);
     int g = 0;  // global K-step counter (continues across tiles)
+    const int64_t rowb = (int64_t)a.W * a.Cp * 2;
+    const int pixb = a.Cp * 2;
     for (int t = blockIdx.x; t < tiles; t += gridDim.x) {
-      int n[MS], oy[MS], ox[MS];
-      bool rv[MS];
+      RowWin w[MS];
 #pragma unroll
-      for (int i = 0; i < MS; ++i) {
-        n[i] = oy[i] = ox[i] = 0;
-        const int m = (t / n_tiles) * rows_per_tile + i * 128 + r;
-        rv[i] = m < a.M;
-        if (rv[i]) decode_row(a, m, n[i], oy[i], ox[i]);
-      }
+      for (int i = 0; i < MS; ++i) w[i] = row_window(a, (t / n_tiles) * rows_per_tile + i * 128 + r);
       for (int j = 0; j < KC; ++j, ++g) {
         const int s = g % S;
         mbar_wait(empty0 + 8 * s, ((g / S) & 1) ^ 1);
 #pragma unroll
         for (int i = 0; i < MS; ++i) {
-          const __nv_bfloat16* img = a.in + (int64_t)n[i] * a.H * a.W * a.Cp;
           const uint32_t base = As0 + (uint32_t)s * stage_a + (uint32_t)(i * a_per_sub) * kATile;
           if (PATCH) {
-            gather_patch(a, img, rv[i], oy[i], ox[i], j, base, r);
+            gather_patch(a, w[i], j, rowb, pixb, base, r);
           } else {
-            for (int q = 0; q < nq; ++q) {
-              int cy, cx;
-              conv_pixel(a, oy[i], ox[i], q, cy, cx);
-              gather(a, img, rv[i], cy, cx, j, base + (uint32_t)q * kATile, r);
-            }
+#pragma unroll
+            for (int q = 0; q < NQ; ++q)
+              gather_tap(a, w[i], j, NQ == 4 ? (q >> 1) : 0, NQ == 4 ? (q & 1) : 0, rowb, pixb,
+                         base + (uint32_t)q * kATile, r);
           }
         }
         cp_async_commit();

@@ -201,6 +201,8 @@ TyConvArgs layer_args(const ffsva_tyolo* m, int l, int n, const __nv_bfloat16* i
   a.msub = L.msub;
   a.patch = L.patch;
   a.lag = env_int("FFSVA_TYOLO_LAG", 1);
+  a.cp_shift = 0;
+  while ((1 << a.cp_shift) < L.Cp) ++a.cp_shift;
   a.grid = m->ctx->num_sms;
   a.leaky = l < 8 ? 1 : 0;
   a.M = n * L.Ho * L.Ho;
