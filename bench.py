@@ -410,11 +410,11 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
     from paper_conf_icpp_zhangcjzly18_b200.online import run_paced
     from synth import synth
     W, H, P = video.width, video.height, 3 * video.width
-    counts = []
+    counts, ladder = [], []
     for tok in args.online.split(","):
         tok = tok.strip()
-        if tok == "auto":  # 55% of the offline capacity: the online cycle runs host work and kernels serially
-            counts.append(max(31, int(0.55 * value / 30)))
+        if tok == "auto":  # a ladder of fractions of the offline capacity, climbed until a count is not sustained
+            ladder = [max(31, int(f * value / 30)) for f in (0.55, 0.7, 0.85)]
         elif tok:
             counts.append(int(tok))
     nc = len(sids)
@@ -434,12 +434,15 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
             ty_counts.append(int(tok))
     results = []
     opened = []
-    runs = [(S, False) for S in counts] + [(S, True) for S in ty_counts]
+    runs = [(S, False) for S in counts] + [(S, False) for S in ladder] + [(S, True) for S in ty_counts]
     ty = None
     if ty_counts:
         import paper_conf_icpp_zhangcjzly18_b200 as ff
         ty = ff.Tyolo(ctx, synth.tyolo_weights(video.seed))
+    ladder_failed = False
     for S, with_ty in runs:
+        if S in ladder and not with_ty and ladder_failed:
+            continue  # the ladder stops at its first count that is not sustained
         t_setup = time.perf_counter()
         while len(opened) < S:
             i = len(opened)
@@ -453,6 +456,8 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
                         cuda_stream=cs, tyolo=ty if with_ty else None)
         res["stream_setup_s"] = setup_s
         results.append(res)
+        if S in ladder and not with_ty and not res["sustained"]:
+            ladder_failed = True
     for st in opened:
         st.close()
         ctx.streams.remove(st)
@@ -578,7 +583,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--online", default="30,auto",
                     help="comma-separated stream counts for the paced online validation (config m2); 'auto' = "
-                         "55%% of the measured frames/s / 30; empty to skip")
+                         "a ladder of 55/70/85%% of the measured frames/s / 30, climbed until a count is not "
+                         "sustained; empty to skip")
     ap.add_argument("--online-seconds", type=float, default=4.0)
     ap.add_argument("--online-tyolo", default="2000,auto",
                     help="stream counts for a paced run of the full cascade with the T-YOLO stage (f1); 'auto' = "

@@ -268,6 +268,17 @@ FFSVA_API ffsva_status ffsva_sched_destroy(ffsva_sched* s);
 typedef enum { FFSVA_BATCH_DYNAMIC = 0, FFSVA_BATCH_FEEDBACK = 1, FFSVA_BATCH_STATIC = 2 } ffsva_batch_policy;
 FFSVA_API ffsva_status ffsva_sched_set_policy(ffsva_sched* s, int32_t policy);
 
+/* Pipelined ticks (on != 0; default off = synchronous ticks as described above). The paper runs its stages as
+ * concurrent threads linked by queues (§3.1.2); here the host half of a cycle (admission,
+ * batch assembly, event reporting) and the caller's work between ticks overlap the kernels of the previous cycle:
+ * tick k prepares cycle k on the host, waits for cycle k-1's kernels, harvests their results (events, SNM queue
+ * updates), runs the T-YOLO cycle, and launches cycle k's kernels without waiting for them. SNM pops of cycle k
+ * therefore see SDD survivors of cycles <= k-2 (survivors of cycle k-1 join the SNM queues at tick k's harvest),
+ * and every decision is reported one tick later than in synchronous mode; ffsva_tick_info.events_pending counts
+ * in-flight frames too. Frames in flight hold their D50 slots, so size snm_slots for two cycles. Turning the mode
+ * off while a cycle is in flight returns FFSVA_EAGAIN (tick once more first). Errors: EINVAL. */
+FFSVA_API ffsva_status ffsva_sched_set_pipeline(ffsva_sched* s, int32_t on);
+
 /* ---------------------------------------------------------------------------------------------------------
  * Admission control and stream re-forwarding between instances (§4.3.1: "when any queue of
  * T-YOLO or SNM is longer than its predefined threshold ... the corresponding video stream is re-forwarded to

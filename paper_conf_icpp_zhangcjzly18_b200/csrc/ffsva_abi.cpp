@@ -102,7 +102,7 @@ FFSVA_API ffsva_status ffsva_open_stream(const ffsva_stream_desc* desc, ffsva_st
   s->L_high = logit_of(desc->c_high);
   {
     DeviceGuard g(ctx->device);
-    const size_t rbytes = (size_t)nvals;
+    const size_t rbytes = ((size_t)nvals + 15) & ~(size_t)15;  // K1's band kernel bulk-copies 16-B aligned R spans
     cudaError_t e = cudaMalloc(&s->d_ref, rbytes);
     if (e == cudaSuccess) e = cudaMalloc(&s->d_snm, snm::BLOB_BYTES);
     if (e != cudaSuccess) {

@@ -70,6 +70,20 @@ struct SddArgs {
   int32_t uni_W, uni_H;
   int32_t cellw;             // widest 100-grid cell of uni_W-wide frames, ceil(uni_W / sdd_w) (0 if mixed)
 };
+
+// K1 variant choice for one batch (sdd_plan_add per frame, then sdd_plan_finish): the bulk-async CTA-pair kernel
+// for 16-B aligned rows whose 100-grid row fits the stage, the register-streaming kernel otherwise;
+// FFSVA_SDD_KERNEL=stream forces the latter (tests exercise both).
+enum SddVariant : int32_t { kSddStream = 0, kSddPair = 1 };
+struct SddPlan {
+  int32_t max_chunks = 1, pair_stage = 0;
+  bool vec16 = true;
+  int32_t variant = kSddStream, stage_bytes = 0;
+  size_t smem = 0;
+};
+void sdd_plan_add(SddPlan& p, int32_t W, int32_t H, int64_t pitch, const void* pixels, int32_t sdd_h);
+void sdd_plan_finish(SddPlan& p, int32_t sdd_w, int32_t sdd_h);
+void sdd_plan_apply(const SddPlan& p, SddArgs& a);
 cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st);
 size_t sdd_smem_bytes(int max_chunks, int sdd_w);
 size_t sdd_bulk_smem_bytes(int stage_bytes, int sdd_w);
@@ -174,7 +188,7 @@ struct TyConvArgs {
 cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st);
 cudaError_t launch_tyolo_pool_s1(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C,
                                  cudaStream_t st);
-cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int32_t max_row_bytes,
+cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int32_t max_row_bytes, int32_t max_H,
                                 __nv_bfloat16* out, cudaStream_t st);
 int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT);
 cudaError_t tyolo_configure();

@@ -343,8 +343,7 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
                          bool want_d100, cudaStream_t st) {
   const StreamState* s0 = frames[0].stream;
   const int32_t sdd_w = s0->desc.sdd_w, sdd_h = s0->desc.sdd_h;
-  bool vec16 = true;
-  int32_t max_chunks = 1, stage_bytes = 0;
+  SddPlan plan;
   for (int32_t i = 0; i < n; ++i) {
     const StreamState* s = frames[i].stream;
     if (s->desc.sdd_w != sdd_w || s->desc.sdd_h != sdd_h)
@@ -352,15 +351,11 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     const int64_t bytes = (int64_t)(s->desc.height - 1) * s->desc.row_pitch + 3 * s->desc.width;
     ffsva_status cs = check_device_ptr(ctx, frames[i].pixels, (size_t)bytes);
     if (cs != FFSVA_OK) return cs;
-    if ((s->desc.row_pitch & 15) || ((uintptr_t)frames[i].pixels & 15)) vec16 = false;
-    max_chunks = std::max(max_chunks, (3 * s->desc.width + 15) / 16);
-    stage_bytes = std::max(stage_bytes, sdd_bulk_stage_bytes(s->desc.width, s->desc.height, sdd_h));
+    sdd_plan_add(plan, s->desc.width, s->desc.height, s->desc.row_pitch, frames[i].pixels, sdd_h);
     if (s->desc.ref_mode == FFSVA_REF_PREVIOUS) want_d100 = true;  // K2 reads every frame's D100
   }
-  // K1 variant: the bulk-async/cluster kernel needs 16-B aligned rows that fit the shared-memory stage;
-  // FFSVA_SDD_KERNEL=stream forces the register-streaming kernel (tests exercise both)
-  const char* force = std::getenv("FFSVA_SDD_KERNEL");
-  const bool bulk = vec16 && sdd_bulk_ok(max_chunks, stage_bytes) && !(force && std::strcmp(force, "stream") == 0);
+  // K1 variant (band / CTA-pair cluster / register streaming) and its shared-memory layout
+  sdd_plan_finish(plan, sdd_w, sdd_h);
   if (b->cap < n || b->sdd_w != sdd_w || b->sdd_h != sdd_h || (want_d100 && !b->want_d100)) {
     ffsva_status as = batch_alloc(ctx, b, std::max(n, b->cap), sdd_w, sdd_h, want_d100 || b->want_d100);
     if (as != FFSVA_OK) return as;
@@ -369,13 +364,10 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     cudaGraphExecDestroy(b->graph);
     b->graph = nullptr;
   }
-  cudaError_t e = sdd_configure(bulk ? sdd_bulk_smem_bytes(stage_bytes, sdd_w) : sdd_smem_bytes(max_chunks, sdd_w));
+  cudaError_t e = sdd_configure(plan.smem);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "sdd_configure");
   b->n = n;
-  b->vec16 = vec16;
-  b->bulk = bulk;
-  b->stage_bytes = stage_bytes;
-  b->max_chunks = max_chunks;
+  b->plan = plan;
   b->sdd_only = sdd_only;
   // ---- host staging: descriptors, stream-major permutation, segments
   const size_t cap = (size_t)b->cap;
@@ -476,10 +468,7 @@ SddArgs make_sdd_args(Batch* b, int32_t i0, int32_t cnt) {
   sa.d100 = b->want_d100 ? b->d_d100 + (size_t)i0 * 3 * b->sdd_w * b->sdd_h : nullptr;
   sa.acc_ssd = b->d_acc + i0;
   sa.stats = b->ctx->d_stats;
-  sa.max_chunks = b->max_chunks;
-  sa.vec16 = b->vec16;
-  sa.bulk = b->bulk;
-  sa.stage_bytes = b->stage_bytes;
+  sdd_plan_apply(b->plan, sa);
   sa.uni_W = b->uni_W;
   sa.uni_H = b->uni_H;
   sa.cellw = b->uni_W > 0 ? (b->uni_W + b->sdd_w - 1) / b->sdd_w : 0;

@@ -36,10 +36,9 @@ struct StreamState {
 struct Batch {
   DeviceCtx* ctx = nullptr;
   int32_t n = 0, cap = 0;
-  int32_t sdd_w = 0, sdd_h = 0, max_chunks = 0, n_seg = 0;
-  bool vec16 = true, sdd_only = false, want_d100 = false;
-  bool bulk = false;          // K1 variant: bulk-async + cluster (aligned frames) or register streaming
-  int32_t stage_bytes = 0;
+  int32_t sdd_w = 0, sdd_h = 0, n_seg = 0;
+  bool sdd_only = false, want_d100 = false;
+  SddPlan plan;               // K1 variant and its shared-memory layout (sdd_plan_*)
   int32_t uni_W = -1, uni_H = -1;        // common frame size of the batch (-1: mixed)
   int32_t *d_xb = nullptr, *d_yb = nullptr;  // cell boundary tables for uni_W / uni_H (in the input block)
   int32_t *d_pm = nullptr, *d_last = nullptr;  // PREVIOUS-mode plan (input block): (frame, prev) pairs, last frames

@@ -67,8 +67,16 @@ struct ffsva_sched {
   uint8_t* d_out = nullptr;   // ssd u64[cap] | logit f32[cap] | pass u8[cap] | snm_pass u8[cap] | snm_class u8[cap]
   uint8_t* h_out = nullptr;
   std::deque<ffsva_event> pending;
+  std::vector<sched::QFrame> adm;   // this cycle's SDD admissions, reused
   std::vector<sched::QFrame> flat;  // this cycle's SNM pops, reused
   std::vector<int32_t> starts;
+  // pipelined mode (ffsva_sched_set_pipeline): the kernels tick k launches are harvested by tick k + 1, so the
+  // caller's work between ticks and the next cycle's host preparation overlap them. Host staging is double
+  // buffered (hb), the device staging holds separate SDD and SNM regions.
+  bool pipelined = false, inflight = false;
+  int32_t hb = 0;
+  cudaEvent_t done_ev = nullptr;
+  std::vector<sched::QFrame> f_adm, f_flat;  // the in-flight cycle's admissions and pops
   // T-YOLO stage (f1): the device's shared model, its per-cycle extraction and score threshold
   ffsva_tyolo* tyolo = nullptr;
   float ty_thresh = 0.2f;
@@ -78,6 +86,7 @@ struct ffsva_sched {
 namespace {
 
 void sched_free(ffsva_sched* s) {
+  if (s->done_ev) cudaEventDestroy(s->done_ev);
   cudaFree(s->d_pool);
   cudaFree(s->d_in);
   cudaFree(s->d_mem);
@@ -106,6 +115,269 @@ FrameDesc make_desc(const ffsva_stream* st, const void* pixels) {
 template <typename T>
 T* at(uint8_t* base, size_t off) { return reinterpret_cast<T*>(base + off); }
 
+// ---------------------------------------------------------------- cycle phases (shared by both tick modes)
+struct SddStage {
+  int32_t na = 0, nseg = 0, sdd_w = 0, sdd_h = 0;
+  SddPlan plan;
+};
+struct SnmStage {
+  int32_t m = 0, nch = 0;
+};
+
+// SDD admission (feedback: streams whose SNM queue is over q_snm wait) into host staging h: one D50 slot per
+// admitted frame, frame descriptors, per-stream segments (admitted frames arrive grouped by stream).
+SddStage prep_sdd(ffsva_sched* s, uint8_t* h, const Layout& L, std::vector<sched::QFrame>& adm) {
+  SddStage sd;
+  adm = s->pol.admit_sdd(s->max_frames, (int32_t)s->free_slots.size());
+  sd.na = (int32_t)adm.size();
+  if (sd.na == 0) return sd;
+  FrameDesc* hd = at<FrameDesc>(h, L.desc);
+  int32_t* hidx = at<int32_t>(h, L.index);
+  int32_t* hseg = at<int32_t>(h, L.seg_lo);
+  int32_t* hsegb = at<int32_t>(h, L.seg_batch);
+  int32_t* hsegs = at<int32_t>(h, L.seg_slot);
+  sd.sdd_w = s->by_id[adm[0].stream]->desc.sdd_w;
+  sd.sdd_h = s->by_id[adm[0].stream]->desc.sdd_h;
+  for (int32_t i = 0; i < sd.na; ++i) {
+    const ffsva_stream* st = s->by_id[adm[i].stream];
+    adm[i].slot = s->free_slots.back();
+    s->free_slots.pop_back();
+    hd[i] = make_desc(st, adm[i].pixels);
+    hidx[i] = adm[i].slot;
+    if (i == 0 || adm[i].stream != adm[i - 1].stream) {
+      hseg[sd.nseg] = i;
+      hsegb[sd.nseg] = st->desc.snm_batch;
+      hsegs[sd.nseg] = st->slot;
+      ++sd.nseg;
+    }
+    sdd_plan_add(sd.plan, st->desc.width, st->desc.height, st->desc.row_pitch, adm[i].pixels, sd.sdd_h);
+  }
+  hseg[sd.nseg] = sd.na;
+  sdd_plan_finish(sd.plan, sd.sdd_w, sd.sdd_h);
+  return sd;
+}
+
+// Upload the SDD staging (used parts only) into device region d, launch K1 (D50 into the slots) and K3 (threshold),
+// queue the D2H of distances and pass flags into h_out. Asynchronous on cs.
+cudaError_t launch_sdd_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layout& L, const SddStage& sd,
+                             cudaStream_t cs) {
+  DeviceCtx* ctx = s->ctx;
+  const size_t n = (size_t)s->cap;
+  const int32_t na = sd.na, nseg = sd.nseg;
+  cudaError_t e = sdd_configure(sd.plan.smem);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(d + L.desc, h + L.desc, 64 * (size_t)na, cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(d + L.index, h + L.index, 4 * (size_t)na, cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(d + L.seg_lo, h + L.seg_lo, 4 * (size_t)(nseg + 1), cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(d + L.seg_batch, h + L.seg_batch, 4 * (size_t)nseg, cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(d + L.seg_slot, h + L.seg_slot, 4 * (size_t)nseg, cudaMemcpyHostToDevice, cs);
+  SddArgs sa{};
+  sa.frames = at<FrameDesc>(d, L.desc);
+  sa.n = na;
+  sa.sdd_w = sd.sdd_w;
+  sa.sdd_h = sd.sdd_h;
+  sa.d50 = s->d_pool;
+  sa.d50_stride = kD50Stride;
+  sa.d50_index = at<int32_t>(d, L.index);
+  sa.acc_ssd = s->d_acc;
+  sa.stats = ctx->d_stats;
+  sdd_plan_apply(sd.plan, sa);
+  if (e == cudaSuccess) e = launch_sdd(sa, cs);
+  CompactArgs ca{};  // threshold + per-stream SDD-pass stats; no SNM work units (snm_ctas = 0)
+  ca.frames = sa.frames;
+  ca.acc_ssd = s->d_acc;
+  ca.ssd = at<uint64_t>(s->d_out, 0);
+  ca.pass = s->d_out + 12 * n;
+  ca.n = na;
+  ca.perm = s->d_perm;
+  ca.seg_lo = at<int32_t>(d, L.seg_lo);
+  ca.n_seg = nseg;
+  ca.seg_batch = at<int32_t>(d, L.seg_batch);
+  ca.seg_slot = at<int32_t>(d, L.seg_slot);
+  ca.stats = ctx->d_stats;
+  ca.snm_ctas = 0;
+  ca.survivor_idx = s->d_surv;
+  ca.work = at<int32_t>(d, L.work);
+  ca.posw = s->d_posw;
+  ca.chunks = at<int32_t>(d, L.chunks);
+  ca.counts = at<int32_t>(d, L.counts);
+  ca.logit = at<float>(s->d_out, 8 * n);
+  ca.snm_pass = s->d_out + 13 * n;
+  ca.snm_class = s->d_out + 14 * n;
+  if (e == cudaSuccess) e = launch_compact(ca, cs);
+  g_launches += 2;
+  if (e == cudaSuccess) e = cudaMemcpyAsync(at<uint64_t>(s->h_out, 0), ca.ssd, 8 * (size_t)na, cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(s->h_out + 12 * n, ca.pass, (size_t)na, cudaMemcpyDeviceToHost, cs);
+  return e;
+}
+
+// SDD results (in h_out) of admissions adm[0, na): survivors join their SNM queue, dropped frames become events.
+void harvest_sdd(ffsva_sched* s, std::vector<sched::QFrame>& adm, int32_t na, ffsva_tick_info& ti) {
+  const size_t n = (size_t)s->cap;
+  const uint64_t* h_ssd = at<uint64_t>(s->h_out, 0);
+  const uint8_t* h_pass = s->h_out + 12 * n;
+  for (int32_t i = 0; i < na; ++i) {
+    adm[i].ssd = h_ssd[i];
+    s->pol.sdd_done(adm[i], h_pass[i] != 0);
+    if (h_pass[i]) {
+      ++ti.sdd_pass;
+      continue;
+    }
+    ffsva_event ev{};
+    ev.stream = s->by_id[adm[i].stream];
+    ev.frame_no = adm[i].frame_no;
+    ev.result.ssd = h_ssd[i];
+    ev.result.logit = NAN;
+    ev.result.survivor_idx = -1;
+    ev.result.tyolo_count = -1;
+    s->pending.push_back(ev);
+    s->free_slots.push_back(adm[i].slot);
+  }
+}
+
+// SNM cycle: dynamic batching (pops of min(BatchSize, depth) per stream; or the static / feedback-queue fixed-size
+// trigger chosen by ffsva_sched_set_policy) into host staging h.
+SnmStage prep_snm(ffsva_sched* s, uint8_t* h, const Layout& L, std::vector<sched::QFrame>& flat,
+                  std::vector<int32_t>& starts, ffsva_tick_info& ti) {
+  SnmStage sn;
+  s->pol.pop_snm(flat, starts, (int32_t)s->free_slots.size());
+  sn.m = (int32_t)flat.size();
+  ti.snm_batches = (int32_t)starts.size() - 1;
+  ti.snm_scored = sn.m;
+  if (sn.m == 0) return sn;
+  const int32_t m = sn.m;
+  FrameDesc* hd = at<FrameDesc>(h, L.desc);
+  int32_t* hidx = at<int32_t>(h, L.index);
+  int32_t* hwork = at<int32_t>(h, L.work);
+  int32_t* hch = at<int32_t>(h, L.chunks);
+  int32_t* hcnt = at<int32_t>(h, L.counts);
+  uint8_t* hpop = h + L.pop_start;
+  int32_t nch = 0;
+  for (size_t p = 0; p + 1 < starts.size(); ++p) {
+    const ffsva_stream* st = s->by_id[flat[starts[p]].stream];
+    // a pop is split into work units of U frames so small cycles still spread over the SMs
+    const int32_t U = std::max(1, std::min(st->desc.snm_batch, m / std::max(1, s->ctx->num_sms)));
+    const FrameDesc d = make_desc(st, nullptr);
+    for (int32_t j = starts[p]; j < starts[p + 1]; ++j) {
+      const int32_t k = j - starts[p];
+      if (k % U == 0) {
+        hpop[nch] = k == 0 ? 1 : 0;
+        hch[nch++] = j;
+      }
+      hd[j] = d;
+      hidx[j] = flat[j].slot;
+      hwork[j] = j;
+    }
+  }
+  hch[nch] = m;
+  hcnt[0] = m;
+  hcnt[1] = nch;
+  hcnt[2] = 0;
+  hcnt[3] = 0;
+  sn.nch = nch;
+  return sn;
+}
+
+// Upload the SNM staging into device region d, launch K4 on the popped frames' slots, queue the D2H of logits,
+// decisions and classes into h_out. Asynchronous on cs.
+cudaError_t launch_snm_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layout& L, const SnmStage& sn,
+                             cudaStream_t cs) {
+  const size_t n = (size_t)s->cap;
+  const int32_t m = sn.m, nch = sn.nch;
+  cudaError_t e = cudaMemcpyAsync(d + L.desc, h + L.desc, 64 * (size_t)m, cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(d + L.index, h + L.index, 4 * (size_t)m, cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(d + L.work, h + L.work, 4 * (size_t)m, cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(d + L.chunks, h + L.chunks, 4 * (size_t)(nch + 1), cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(d + L.counts, h + L.counts, 16, cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(d + L.pop_start, h + L.pop_start, (size_t)nch, cudaMemcpyHostToDevice, cs);
+  SnmArgs na{};
+  na.frames = at<FrameDesc>(d, L.desc);
+  na.d50 = s->d_pool;
+  na.d50_stride = kD50Stride;
+  na.d50_index = at<int32_t>(d, L.index);
+  na.work = at<int32_t>(d, L.work);
+  na.chunks = at<int32_t>(d, L.chunks);
+  na.counts = at<int32_t>(d, L.counts);
+  na.pop_start = d + L.pop_start;
+  na.logit = at<float>(s->d_out, 8 * n);
+  na.snm_pass = s->d_out + 13 * n;
+  na.snm_class = s->d_out + 14 * n;
+  na.stats = s->ctx->d_stats;
+  na.grid = std::max(1, std::min(nch, s->ctx->num_sms));
+  if (e == cudaSuccess) e = launch_snm(na, cs);
+  g_launches += 1;
+  if (e == cudaSuccess) e = cudaMemcpyAsync(at<float>(s->h_out, 8 * n), na.logit, 4 * (size_t)m, cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(s->h_out + 13 * n, na.snm_pass, (size_t)m, cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(s->h_out + 14 * n, na.snm_class, (size_t)m, cudaMemcpyDeviceToHost, cs);
+  return e;
+}
+
+// SNM results (in h_out) of pops flat[0, m): slots are freed; survivors with a T-YOLO stage wait in its queue,
+// every other frame becomes an event.
+void harvest_snm(ffsva_sched* s, std::vector<sched::QFrame>& flat, int32_t m) {
+  const size_t n = (size_t)s->cap;
+  const float* h_logit = at<float>(s->h_out, 8 * n);
+  const uint8_t* h_snm_pass = s->h_out + 13 * n;
+  const uint8_t* h_snm_class = s->h_out + 14 * n;
+  for (int32_t k = 0; k < m; ++k) {
+    s->free_slots.push_back(flat[k].slot);
+    flat[k].logit = h_logit[k];
+    flat[k].snm_class = h_snm_class[k];
+    if (s->pol.snm_done(flat[k], h_snm_pass[k] != 0)) continue;  // waits in the stream's T-YOLO queue
+    ffsva_event ev{};
+    ev.stream = s->by_id[flat[k].stream];
+    ev.frame_no = flat[k].frame_no;
+    ev.result.ssd = flat[k].ssd;
+    ev.result.sdd_pass = 1;
+    ev.result.snm_pass = h_snm_pass[k];
+    ev.result.snm_class = h_snm_class[k];
+    ev.result.logit = h_logit[k];
+    ev.result.survivor_idx = -1;
+    ev.result.tyolo_count = -1;
+    s->pending.push_back(ev);
+  }
+}
+
+// T-YOLO cycle (f1): at most num_t-yolo frames from each T-YOLO queue (L173), counted with the shared model;
+// NumberofObjects per stream (L195). Synchronous on cs.
+ffsva_status tyolo_cycle(ffsva_sched* s, cudaStream_t cs, ffsva_tick_info& ti) {
+  if (!s->tyolo) return FFSVA_OK;
+  std::vector<sched::QFrame>& tf = s->tyflat;
+  s->pol.pop_ty(tf);
+  const int32_t nt = (int32_t)tf.size();
+  ti.tyolo_scored = nt;
+  if (nt == 0) return FFSVA_OK;
+  std::vector<ffsva_frame> fr((size_t)nt);
+  std::vector<int32_t> targets((size_t)nt), counts((size_t)nt);
+  for (int32_t i = 0; i < nt; ++i) {
+    ffsva_stream* st = s->by_id[tf[i].stream];
+    fr[i] = ffsva_frame{st, (const uint8_t*)tf[i].pixels, tf[i].frame_no};
+    targets[i] = st->desc.target_class;
+  }
+  ffsva_status ts = tyolo_run_unlocked(s->tyolo, fr.data(), nt, targets.data(), s->ty_thresh, 0, counts.data(),
+                                       nullptr, nullptr, cs);
+  if (ts != FFSVA_OK) return ts;
+  for (int32_t i = 0; i < nt; ++i) {
+    const ffsva_stream* st = s->by_id[tf[i].stream];
+    ffsva_event ev{};
+    ev.stream = s->by_id[tf[i].stream];
+    ev.frame_no = tf[i].frame_no;
+    ev.result.ssd = tf[i].ssd;
+    ev.result.sdd_pass = 1;
+    ev.result.snm_pass = 1;
+    ev.result.snm_class = tf[i].snm_class;
+    ev.result.logit = tf[i].logit;
+    ev.result.survivor_idx = -1;
+    ev.result.tyolo_count = counts[i];
+    ev.result.tyolo_pass = counts[i] >= st->desc.number_of_objects ? 1 : 0;
+    s->pending.push_back(ev);
+  }
+  return FFSVA_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -128,8 +400,9 @@ FFSVA_API ffsva_status ffsva_sched_create(int32_t device, int32_t max_frames_per
                o_acc = o_surv + al256(4 * n), o_out = o_acc + al256(8 * n), total = o_out + al256(15 * n);
   cudaError_t e = cudaMalloc(&s->d_mem, total);
   if (e == cudaSuccess) e = cudaMalloc(&s->d_pool, (size_t)snm_slots * kD50Stride);
-  if (e == cudaSuccess) e = cudaMalloc(&s->d_in, L.total);
-  if (e == cudaSuccess) e = cudaMallocHost(&s->h_in, L.total);
+  if (e == cudaSuccess) e = cudaMalloc(&s->d_in, 2 * L.total);       // SDD region | SNM region
+  if (e == cudaSuccess) e = cudaMallocHost(&s->h_in, 4 * L.total);   // 2 buffers x (SDD | SNM)
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&s->done_ev, cudaEventDisableTiming);
   if (e == cudaSuccess) e = cudaMallocHost(&s->h_out, 15 * n);
   if (e == cudaSuccess) {
     uint8_t* b = (uint8_t*)s->d_mem;
@@ -239,6 +512,12 @@ FFSVA_API ffsva_status ffsva_sched_detach(ffsva_sched* s, ffsva_stream* st) {
   if (!q.sdd.empty() || !q.snm.empty() || !q.ty.empty()) return fail(FFSVA_EAGAIN, "stream still has queued frames");
   for (const ffsva_event& e : s->pending)
     if (e.stream == st) return fail(FFSVA_EAGAIN, "stream still has unreported events");
+  if (s->inflight) {
+    for (const sched::QFrame& q : s->f_adm)
+      if (q.stream == id) return fail(FFSVA_EAGAIN, "stream has frames in flight");
+    for (const sched::QFrame& q : s->f_flat)
+      if (q.stream == id) return fail(FFSVA_EAGAIN, "stream has frames in flight");
+  }
   s->pol.remove_stream(id);
   s->by_id[id] = nullptr;
   s->id_of_slot[st->slot] = -1;
@@ -263,6 +542,14 @@ FFSVA_API ffsva_status ffsva_sched_set_policy(ffsva_sched* s, int32_t policy) {
   return FFSVA_OK;
 }
 
+FFSVA_API ffsva_status ffsva_sched_set_pipeline(ffsva_sched* s, int32_t on) {
+  if (!s) return fail(FFSVA_EINVAL, "bad argument");
+  std::lock_guard<std::mutex> lk(s->mu);
+  if (!on && s->inflight) return fail(FFSVA_EAGAIN, "a cycle is still in flight (tick once more)");
+  s->pipelined = on != 0;
+  return FFSVA_OK;
+}
+
 FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva_event* events, int32_t cap,
                                         int32_t* n_events, ffsva_tick_info* info) {
   if (!s || cap < 0 || (cap > 0 && !events) || !n_events) return fail(FFSVA_EINVAL, "bad argument");
@@ -272,254 +559,72 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
   std::lock_guard<std::mutex> dlk(ctx->mu);
   DeviceGuard g(ctx->device);
   cudaStream_t cs = (cudaStream_t)cuda_stream;
-  const size_t n = (size_t)s->cap;
-  const Layout L(n);
-  uint8_t* h = s->h_in;
+  const Layout L((size_t)s->cap);
   ffsva_tick_info ti{};
   const auto t_tick0 = std::chrono::steady_clock::now();
-  uint64_t blocked0 = 0;
-  int32_t snm_blocked0 = 0;
-  for (int32_t i = 0; i < s->pol.n_streams(); ++i) {
-    blocked0 += s->pol.stream(i).sdd_blocked;
-    snm_blocked0 += (int32_t)s->pol.stream(i).snm_blocked;
-  }
-  cudaError_t e = cudaSuccess;
-  uint64_t* h_ssd = at<uint64_t>(s->h_out, 0);
-  float* h_logit = at<float>(s->h_out, 8 * n);
-  uint8_t* h_pass = s->h_out + 12 * n;
-  uint8_t* h_snm_pass = s->h_out + 13 * n;
-  uint8_t* h_snm_class = s->h_out + 14 * n;
+  const uint64_t blocked0 = s->pol.total_sdd_blocked(), snm_blocked0 = s->pol.total_snm_blocked();
+  uint8_t* const d_sdd = s->d_in;
+  uint8_t* const d_snm = s->d_in + L.total;
+  ffsva_status st = FFSVA_OK;
+  std::chrono::steady_clock::time_point t_snm0, t_ty0;
 
-  // ---------------- SDD cycle (admitted frames arrive grouped by stream: one K3 segment per stream)
-  std::vector<sched::QFrame> adm = s->pol.admit_sdd(s->max_frames, (int32_t)s->free_slots.size());
-  const int32_t na = (int32_t)adm.size();
-  ti.admitted = na;
-  if (na > 0) {
-    FrameDesc* hd = at<FrameDesc>(h, L.desc);
-    int32_t* hidx = at<int32_t>(h, L.index);
-    int32_t* hseg = at<int32_t>(h, L.seg_lo);
-    int32_t* hsegb = at<int32_t>(h, L.seg_batch);
-    int32_t* hsegs = at<int32_t>(h, L.seg_slot);
-    int32_t max_chunks = 1, stage = 0, nseg = 0;
-    const int32_t sdd_w = s->by_id[adm[0].stream]->desc.sdd_w, sdd_h = s->by_id[adm[0].stream]->desc.sdd_h;
-    bool vec16 = true;
-    for (int32_t i = 0; i < na; ++i) {
-      const ffsva_stream* st = s->by_id[adm[i].stream];
-      adm[i].slot = s->free_slots.back();
-      s->free_slots.pop_back();
-      hd[i] = make_desc(st, adm[i].pixels);
-      hidx[i] = adm[i].slot;
-      if (i == 0 || adm[i].stream != adm[i - 1].stream) {
-        hseg[nseg] = i;
-        hsegb[nseg] = st->desc.snm_batch;
-        hsegs[nseg] = st->slot;
-        ++nseg;
-      }
-      max_chunks = std::max(max_chunks, (3 * st->desc.width + 15) / 16);
-      stage = std::max(stage, sdd_bulk_stage_bytes(st->desc.width, st->desc.height, sdd_h));
-      if ((st->desc.row_pitch & 15) || ((uintptr_t)adm[i].pixels & 15)) vec16 = false;
+  if (!s->pipelined) {
+    // ---------------- synchronous cycle: SDD (launch, wait, harvest), then SNM on the updated queues
+    uint8_t* hs = s->h_in;
+    uint8_t* hn = s->h_in + L.total;
+    SddStage sd = prep_sdd(s, hs, L, s->adm);
+    ti.admitted = sd.na;
+    if (sd.na > 0) {
+      cudaError_t e = launch_sdd_stage(s, hs, d_sdd, L, sd, cs);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+      if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (SDD cycle)");
+      harvest_sdd(s, s->adm, sd.na, ti);
     }
-    hseg[nseg] = na;
-    const bool bulk = vec16 && sdd_bulk_ok(max_chunks, stage);
-    e = sdd_configure(bulk ? sdd_bulk_smem_bytes(stage, sdd_w) : sdd_smem_bytes(max_chunks, sdd_w));
-    // upload only the used part of each staging region
-    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in + L.desc, h + L.desc, 64 * (size_t)na, cudaMemcpyHostToDevice, cs);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in + L.index, h + L.index, 4 * (size_t)na, cudaMemcpyHostToDevice, cs);
-    if (e == cudaSuccess)
-      e = cudaMemcpyAsync(s->d_in + L.seg_lo, h + L.seg_lo, 4 * (size_t)(nseg + 1), cudaMemcpyHostToDevice, cs);
-    if (e == cudaSuccess)
-      e = cudaMemcpyAsync(s->d_in + L.seg_batch, h + L.seg_batch, 4 * (size_t)nseg, cudaMemcpyHostToDevice, cs);
-    if (e == cudaSuccess)
-      e = cudaMemcpyAsync(s->d_in + L.seg_slot, h + L.seg_slot, 4 * (size_t)nseg, cudaMemcpyHostToDevice, cs);
-    SddArgs sa{};
-    sa.frames = at<FrameDesc>(s->d_in, L.desc);
-    sa.n = na;
-    sa.sdd_w = sdd_w;
-    sa.sdd_h = sdd_h;
-    sa.d50 = s->d_pool;
-    sa.d50_stride = kD50Stride;
-    sa.d50_index = at<int32_t>(s->d_in, L.index);
-    sa.acc_ssd = s->d_acc;
-    sa.stats = ctx->d_stats;
-    sa.max_chunks = max_chunks;
-    sa.vec16 = vec16;
-    sa.bulk = bulk;
-    sa.stage_bytes = stage;
-    if (e == cudaSuccess) e = launch_sdd(sa, cs);
-    CompactArgs ca{};  // threshold + per-stream SDD-pass stats; no SNM work units (snm_ctas = 0)
-    ca.frames = sa.frames;
-    ca.acc_ssd = s->d_acc;
-    ca.ssd = at<uint64_t>(s->d_out, 0);
-    ca.pass = s->d_out + 12 * n;
-    ca.n = na;
-    ca.perm = s->d_perm;
-    ca.seg_lo = at<int32_t>(s->d_in, L.seg_lo);
-    ca.n_seg = nseg;
-    ca.seg_batch = at<int32_t>(s->d_in, L.seg_batch);
-    ca.seg_slot = at<int32_t>(s->d_in, L.seg_slot);
-    ca.stats = ctx->d_stats;
-    ca.snm_ctas = 0;
-    ca.survivor_idx = s->d_surv;
-    ca.work = at<int32_t>(s->d_in, L.work);
-    ca.posw = s->d_posw;
-    ca.chunks = at<int32_t>(s->d_in, L.chunks);
-    ca.counts = at<int32_t>(s->d_in, L.counts);
-    ca.logit = at<float>(s->d_out, 8 * n);
-    ca.snm_pass = s->d_out + 13 * n;
-    ca.snm_class = s->d_out + 14 * n;
-    if (e == cudaSuccess) e = launch_compact(ca, cs);
-    g_launches += 2;
-    if (e == cudaSuccess) e = cudaMemcpyAsync(h_ssd, ca.ssd, 8 * (size_t)na, cudaMemcpyDeviceToHost, cs);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(h_pass, ca.pass, (size_t)na, cudaMemcpyDeviceToHost, cs);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
-    if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (SDD cycle)");
-    for (int32_t i = 0; i < na; ++i) {
-      adm[i].ssd = h_ssd[i];
-      s->pol.sdd_done(adm[i], h_pass[i] != 0);
-      if (h_pass[i]) {
-        ++ti.sdd_pass;
-        continue;
-      }
-      ffsva_event ev{};
-      ev.stream = s->by_id[adm[i].stream];
-      ev.frame_no = adm[i].frame_no;
-      ev.result.ssd = h_ssd[i];
-      ev.result.logit = NAN;
-      ev.result.survivor_idx = -1;
-      ev.result.tyolo_count = -1;
-      s->pending.push_back(ev);
-      s->free_slots.push_back(adm[i].slot);
+    t_snm0 = std::chrono::steady_clock::now();
+    SnmStage sn = prep_snm(s, hn, L, s->flat, s->starts, ti);
+    if (sn.m > 0) {
+      cudaError_t e = launch_snm_stage(s, hn, d_snm, L, sn, cs);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+      if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (SNM cycle)");
+      harvest_snm(s, s->flat, sn.m);
     }
-  }
-
-  // ---------------- SNM cycle: dynamic batching (pops of min(BatchSize, depth) per stream; or the static /
-  // feedback-queue fixed-size trigger chosen by ffsva_sched_set_policy)
-  const auto t_snm0 = std::chrono::steady_clock::now();
-  std::vector<sched::QFrame>& flat = s->flat;
-  std::vector<int32_t>& starts = s->starts;
-  s->pol.pop_snm(flat, starts, (int32_t)s->free_slots.size());
-  const int32_t m = (int32_t)flat.size();
-  ti.snm_batches = (int32_t)starts.size() - 1;
-  ti.snm_scored = m;
-  if (m > 0) {
-    FrameDesc* hd = at<FrameDesc>(h, L.desc);
-    int32_t* hidx = at<int32_t>(h, L.index);
-    int32_t* hwork = at<int32_t>(h, L.work);
-    int32_t* hch = at<int32_t>(h, L.chunks);
-    int32_t* hcnt = at<int32_t>(h, L.counts);
-    uint8_t* hpop = h + L.pop_start;
-    int32_t nch = 0;
-    for (size_t p = 0; p + 1 < starts.size(); ++p) {
-      const ffsva_stream* st = s->by_id[flat[starts[p]].stream];
-      // a pop is split into work units of U frames so small cycles still spread over the SMs
-      const int32_t U = std::max(1, std::min(st->desc.snm_batch, m / std::max(1, ctx->num_sms)));
-      const FrameDesc d = make_desc(st, nullptr);
-      for (int32_t j = starts[p]; j < starts[p + 1]; ++j) {
-        const int32_t k = j - starts[p];
-        if (k % U == 0) {
-          hpop[nch] = k == 0 ? 1 : 0;
-          hch[nch++] = j;
-        }
-        hd[j] = d;
-        hidx[j] = flat[j].slot;
-        hwork[j] = j;
-      }
+    t_ty0 = std::chrono::steady_clock::now();
+    if ((st = tyolo_cycle(s, cs, ti)) != FFSVA_OK) return st;
+  } else {
+    // ---------------- pipelined cycle: prepare this cycle on the host while the previous one runs, then harvest
+    // the previous one, run the T-YOLO cycle on its survivors, and launch this one without waiting for it
+    uint8_t* hs = s->h_in + (size_t)(2 * s->hb) * L.total;
+    uint8_t* hn = hs + L.total;
+    SddStage sd = prep_sdd(s, hs, L, s->adm);
+    ti.admitted = sd.na;
+    SnmStage sn = prep_snm(s, hn, L, s->flat, s->starts, ti);
+    if (s->inflight) {
+      cudaError_t e = cudaEventSynchronize(s->done_ev);
+      if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (in-flight cycle)");
+      harvest_sdd(s, s->f_adm, (int32_t)s->f_adm.size(), ti);
+      harvest_snm(s, s->f_flat, (int32_t)s->f_flat.size());
+      s->inflight = false;
     }
-    hch[nch] = m;
-    hcnt[0] = m;
-    hcnt[1] = nch;
-    hcnt[2] = 0;
-    hcnt[3] = 0;
-    // upload only the used part of each staging region
-    e = cudaMemcpyAsync(s->d_in + L.desc, h + L.desc, 64 * (size_t)m, cudaMemcpyHostToDevice, cs);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in + L.index, h + L.index, 4 * (size_t)m, cudaMemcpyHostToDevice, cs);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in + L.work, h + L.work, 4 * (size_t)m, cudaMemcpyHostToDevice, cs);
-    if (e == cudaSuccess)
-      e = cudaMemcpyAsync(s->d_in + L.chunks, h + L.chunks, 4 * (size_t)(nch + 1), cudaMemcpyHostToDevice, cs);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(s->d_in + L.counts, h + L.counts, 16, cudaMemcpyHostToDevice, cs);
-    if (e == cudaSuccess)
-      e = cudaMemcpyAsync(s->d_in + L.pop_start, h + L.pop_start, (size_t)nch, cudaMemcpyHostToDevice, cs);
-    SnmArgs na{};
-    na.frames = at<FrameDesc>(s->d_in, L.desc);
-    na.d50 = s->d_pool;
-    na.d50_stride = kD50Stride;
-    na.d50_index = at<int32_t>(s->d_in, L.index);
-    na.work = at<int32_t>(s->d_in, L.work);
-    na.chunks = at<int32_t>(s->d_in, L.chunks);
-    na.counts = at<int32_t>(s->d_in, L.counts);
-    na.pop_start = s->d_in + L.pop_start;
-    na.logit = at<float>(s->d_out, 8 * n);
-    na.snm_pass = s->d_out + 13 * n;
-    na.snm_class = s->d_out + 14 * n;
-    na.stats = ctx->d_stats;
-    na.grid = std::max(1, std::min(nch, ctx->num_sms));
-    if (e == cudaSuccess) e = launch_snm(na, cs);
-    g_launches += 1;
-    if (e == cudaSuccess) e = cudaMemcpyAsync(h_logit, na.logit, 4 * (size_t)m, cudaMemcpyDeviceToHost, cs);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(h_snm_pass, na.snm_pass, (size_t)m, cudaMemcpyDeviceToHost, cs);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(h_snm_class, na.snm_class, (size_t)m, cudaMemcpyDeviceToHost, cs);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
-    if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (SNM cycle)");
-    for (int32_t k = 0; k < m; ++k) {
-      s->free_slots.push_back(flat[k].slot);
-      flat[k].logit = h_logit[k];
-      flat[k].snm_class = h_snm_class[k];
-      if (s->pol.snm_done(flat[k], h_snm_pass[k] != 0)) continue;  // waits in the stream's T-YOLO queue
-      ffsva_event ev{};
-      ev.stream = s->by_id[flat[k].stream];
-      ev.frame_no = flat[k].frame_no;
-      ev.result.ssd = flat[k].ssd;
-      ev.result.sdd_pass = 1;
-      ev.result.snm_pass = h_snm_pass[k];
-      ev.result.snm_class = h_snm_class[k];
-      ev.result.logit = h_logit[k];
-      ev.result.survivor_idx = -1;
-      ev.result.tyolo_count = -1;
-      s->pending.push_back(ev);
-    }
-  }
-
-  // ---------------- T-YOLO cycle (f1): at most num_t-yolo frames from each T-YOLO queue (L173), counted with
-  // the shared model; NumberofObjects per stream (L195)
-  const auto t_ty0 = std::chrono::steady_clock::now();
-  if (s->tyolo) {
-    std::vector<sched::QFrame>& tf = s->tyflat;
-    s->pol.pop_ty(tf);
-    const int32_t nt = (int32_t)tf.size();
-    ti.tyolo_scored = nt;
-    if (nt > 0) {
-      std::vector<ffsva_frame> fr((size_t)nt);
-      std::vector<int32_t> targets((size_t)nt), counts((size_t)nt);
-      for (int32_t i = 0; i < nt; ++i) {
-        ffsva_stream* st = s->by_id[tf[i].stream];
-        fr[i] = ffsva_frame{st, (const uint8_t*)tf[i].pixels, tf[i].frame_no};
-        targets[i] = st->desc.target_class;
-      }
-      ffsva_status ts = tyolo_run_unlocked(s->tyolo, fr.data(), nt, targets.data(), s->ty_thresh, 0, counts.data(),
-                                           nullptr, nullptr, cs);
-      if (ts != FFSVA_OK) return ts;
-      for (int32_t i = 0; i < nt; ++i) {
-        const ffsva_stream* st = s->by_id[tf[i].stream];
-        ffsva_event ev{};
-        ev.stream = s->by_id[tf[i].stream];
-        ev.frame_no = tf[i].frame_no;
-        ev.result.ssd = tf[i].ssd;
-        ev.result.sdd_pass = 1;
-        ev.result.snm_pass = 1;
-        ev.result.snm_class = tf[i].snm_class;
-        ev.result.logit = tf[i].logit;
-        ev.result.survivor_idx = -1;
-        ev.result.tyolo_count = counts[i];
-        ev.result.tyolo_pass = counts[i] >= st->desc.number_of_objects ? 1 : 0;
-        s->pending.push_back(ev);
-      }
+    t_snm0 = std::chrono::steady_clock::now();
+    t_ty0 = t_snm0;
+    if ((st = tyolo_cycle(s, cs, ti)) != FFSVA_OK) return st;
+    if (sd.na > 0 || sn.m > 0) {
+      cudaError_t e = cudaSuccess;
+      if (sd.na > 0) e = launch_sdd_stage(s, hs, d_sdd, L, sd, cs);
+      if (e == cudaSuccess && sn.m > 0) e = launch_snm_stage(s, hn, d_snm, L, sn, cs);
+      if (e == cudaSuccess) e = cudaEventRecord(s->done_ev, cs);
+      if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (launch)");
+      s->f_adm.swap(s->adm);
+      s->f_adm.resize((size_t)sd.na);
+      s->f_flat.swap(s->flat);
+      s->f_flat.resize((size_t)sn.m);
+      s->inflight = true;
+      s->hb ^= 1;
     }
   }
   const auto t_ty1 = std::chrono::steady_clock::now();
 
-  uint64_t blocked1 = 0;
-  for (int32_t i = 0; i < s->pol.n_streams(); ++i) blocked1 += s->pol.stream(i).sdd_blocked;
-  ti.sdd_blocked = (int32_t)(blocked1 - blocked0);
+  ti.sdd_blocked = (int32_t)(s->pol.total_sdd_blocked() - blocked0);
   int32_t k = 0;
   while (k < cap && !s->pending.empty()) {
     events[k++] = s->pending.front();
@@ -529,10 +634,10 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
   ti.sdd_queued = s->pol.queued_sdd();
   ti.snm_queued = s->pol.queued_snm();
   ti.tyolo_queued = s->pol.queued_ty();
-  for (int32_t i = 0; i < s->pol.n_streams(); ++i) ti.snm_blocked += (int32_t)s->pol.stream(i).snm_blocked;
-  ti.snm_blocked -= snm_blocked0;
+  ti.snm_blocked = (int32_t)(s->pol.total_snm_blocked() - snm_blocked0);
   ti.tyolo_ms = std::chrono::duration<float, std::milli>(t_ty1 - t_ty0).count();
-  ti.events_pending = (int64_t)s->pending.size();
+  // in-flight frames count as pending events (they will be reported by a later tick)
+  ti.events_pending = (int64_t)s->pending.size() + (s->inflight ? (int64_t)(s->f_adm.size() + s->f_flat.size()) : 0);
   const auto t_end = std::chrono::steady_clock::now();
   ti.sdd_ms = std::chrono::duration<float, std::milli>(t_snm0 - t_tick0).count();
   ti.snm_ms = std::chrono::duration<float, std::milli>(t_ty0 - t_snm0).count();

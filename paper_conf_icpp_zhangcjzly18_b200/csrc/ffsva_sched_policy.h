@@ -65,7 +65,13 @@ class Policy {
     int32_t id = -1;
     for (int32_t i = 0; i < (int32_t)st_.size(); ++i)
       if (!st_[i].live) { id = i; break; }
-    if (id < 0) { id = (int32_t)st_.size(); st_.emplace_back(); }
+    if (id < 0) {
+      id = (int32_t)st_.size();
+      st_.emplace_back();
+      nsdd_.push_back(0);
+      nsnm_.push_back(0);
+      nty_.push_back(0);
+    }
     StreamQ& s = st_[id];
     s = StreamQ();
     s.q_sdd = q_sdd;
@@ -84,6 +90,10 @@ class Policy {
     out.insert(out.end(), s.sdd.begin(), s.sdd.end());
     out.insert(out.end(), s.snm.begin(), s.snm.end());
     out.insert(out.end(), s.ty.begin(), s.ty.end());
+    nq_sdd_ -= (int64_t)s.sdd.size();
+    nq_snm_ -= (int64_t)s.snm.size();
+    nq_ty_ -= (int64_t)s.ty.size();
+    nsdd_[id] = nsnm_[id] = nty_[id] = 0;
     s = StreamQ();
     return out;
   }
@@ -100,6 +110,8 @@ class Policy {
     QFrame g = f;
     g.stream = id;
     s.sdd.push_back(g);
+    ++nsdd_[id];
+    ++nq_sdd_;
     ++s.pushed;
     s.max_sdd = std::max(s.max_sdd, (int32_t)s.sdd.size());
     return true;
@@ -113,16 +125,19 @@ class Policy {
     const int32_t n = (int32_t)st_.size();
     if (n == 0) return out;
     int32_t limit = std::min(budget, snm_room);
-    for (int32_t k = 0; k < n && limit > 0; ++k) {
-      StreamQ& s = st_[(rr_ + k) % n];
-      if (!s.live || s.sdd.empty()) continue;
-      if (policy_ != BatchPolicy::STATIC && (int32_t)s.snm.size() > s.q_snm) {
+    for (int32_t k = 0, i = rr_; k < n && limit > 0; ++k, i = (i + 1 == n ? 0 : i + 1)) {
+      if (nsdd_[i] == 0) continue;  // compact depth mirror: idle streams cost 4 bytes of scan
+      StreamQ& s = st_[i];
+      if (policy_ != BatchPolicy::STATIC && nsnm_[i] > s.q_snm) {
         ++s.sdd_blocked;
+        ++tot_sdd_blocked_;
         continue;
       }
       while (!s.sdd.empty() && limit > 0) {
         out.push_back(s.sdd.front());
         s.sdd.pop_front();
+        --nsdd_[i];
+        --nq_sdd_;
         --limit;
       }
     }
@@ -135,6 +150,8 @@ class Policy {
     if (!pass) return;
     StreamQ& s = st_[f.stream];
     s.snm.push_back(f);
+    ++nsnm_[f.stream];
+    ++nq_snm_;
     s.max_snm = std::max(s.max_snm, (int32_t)s.snm.size());
   }
 
@@ -146,32 +163,36 @@ class Policy {
     flat.clear();
     starts.clear();
     const int32_t n = (int32_t)st_.size();
-    auto take_from = [&](StreamQ& s, int32_t take) {
+    auto take_from = [&](int32_t k, int32_t take) {
+      StreamQ& s = st_[k];
       starts.push_back((int32_t)flat.size());
       flat.insert(flat.end(), s.snm.begin(), s.snm.begin() + take);
       s.snm.erase(s.snm.begin(), s.snm.begin() + take);
+      nsnm_[k] -= take;
+      nq_snm_ -= take;
     };
     for (int32_t k = 0; k < n; ++k) {
+      if (nsnm_[k] == 0) continue;
       StreamQ& s = st_[k];
-      if (!s.live || s.snm.empty()) continue;
-      if (tyolo_ && (int32_t)s.ty.size() > s.q_ty) {  // T-YOLO -> SNM feedback (L209)
+      if (tyolo_ && nty_[k] > s.q_ty) {  // T-YOLO -> SNM feedback (L209)
         ++s.snm_blocked;
+        ++tot_snm_blocked_;
         continue;
       }
       const int32_t depth = (int32_t)s.snm.size();
       if (policy_ == BatchPolicy::DYNAMIC) {
-        take_from(s, std::min(s.batch, depth));
+        take_from(k, std::min(s.batch, depth));
       } else if (depth >= s.batch) {
-        take_from(s, s.batch);
+        take_from(k, s.batch);
       } else if (policy_ == BatchPolicy::FEEDBACK && depth > s.q_snm) {
-        take_from(s, depth);
+        take_from(k, depth);
       }
     }
     if (flat.empty() && slots_free <= 0) {  // every slot holds a partial batch: pop the fullest queue
       int32_t best = -1;
       for (int32_t k = 0; k < n; ++k)
         if (st_[k].live && !st_[k].snm.empty() && (best < 0 || st_[k].snm.size() > st_[best].snm.size())) best = k;
-      if (best >= 0) take_from(st_[best], std::min(st_[best].batch, (int32_t)st_[best].snm.size()));
+      if (best >= 0) take_from(best, std::min(st_[best].batch, (int32_t)st_[best].snm.size()));
     }
     starts.push_back((int32_t)flat.size());
   }
@@ -182,6 +203,8 @@ class Policy {
     if (!tyolo_ || !pass) return false;
     StreamQ& s = st_[f.stream];
     s.ty.push_back(f);
+    ++nty_[f.stream];
+    ++nq_ty_;
     s.max_ty = std::max(s.max_ty, (int32_t)s.ty.size());
     return true;
   }
@@ -189,11 +212,14 @@ class Policy {
   // T-YOLO cycle (L173): every non-empty T-YOLO queue gives at most num_t-yolo frames, oldest first.
   void pop_ty(std::vector<QFrame>& flat) {
     flat.clear();
-    for (auto& s : st_) {
-      if (!s.live || s.ty.empty()) continue;
+    for (int32_t k = 0; k < (int32_t)st_.size(); ++k) {
+      if (nty_[k] == 0) continue;
+      StreamQ& s = st_[k];
       const int32_t take = std::min<int32_t>(ty_take_, (int32_t)s.ty.size());
       flat.insert(flat.end(), s.ty.begin(), s.ty.begin() + take);
       s.ty.erase(s.ty.begin(), s.ty.begin() + take);
+      nty_[k] -= take;
+      nq_ty_ -= take;
     }
   }
 
@@ -226,24 +252,18 @@ class Policy {
     s.max_ty = (int32_t)s.ty.size();
   }
   int32_t n_streams() const { return (int32_t)st_.size(); }
-  int64_t queued_sdd() const {
-    int64_t q = 0;
-    for (auto& s : st_) q += (int64_t)s.sdd.size();
-    return q;
-  }
-  int64_t queued_snm() const {
-    int64_t q = 0;
-    for (auto& s : st_) q += (int64_t)s.snm.size();
-    return q;
-  }
-  int64_t queued_ty() const {
-    int64_t q = 0;
-    for (auto& s : st_) q += (int64_t)s.ty.size();
-    return q;
-  }
+  // queue totals and blocking counters over all streams, maintained incrementally (O(1) per tick)
+  int64_t queued_sdd() const { return nq_sdd_; }
+  int64_t queued_snm() const { return nq_snm_; }
+  int64_t queued_ty() const { return nq_ty_; }
+  uint64_t total_sdd_blocked() const { return tot_sdd_blocked_; }
+  uint64_t total_snm_blocked() const { return tot_snm_blocked_; }
 
  private:
   std::vector<StreamQ> st_;
+  std::vector<int32_t> nsdd_, nsnm_, nty_;  // per-stream queue depths (compact mirror of the deques)
+  int64_t nq_sdd_ = 0, nq_snm_ = 0, nq_ty_ = 0;
+  uint64_t tot_sdd_blocked_ = 0, tot_snm_blocked_ = 0;
   int32_t rr_ = 0;
   BatchPolicy policy_ = BatchPolicy::DYNAMIC;
   bool tyolo_ = false;

@@ -23,6 +23,8 @@
 #include <cooperative_groups.h>
 
 #include <algorithm>
+#include <cstdlib>
+#include <cstring>
 
 #include "ffsva_internal.h"
 
@@ -550,6 +552,34 @@ int sdd_bulk_stage_bytes(int W, int H, int sdd_h) {
 
 bool sdd_bulk_ok(int max_chunks, int stage_bytes) {
   return max_chunks <= 2 * kBulkThreads && stage_bytes <= kBulkMaxStage;
+}
+
+void sdd_plan_add(SddPlan& p, int32_t W, int32_t H, int64_t pitch, const void* pixels, int32_t sdd_h) {
+  const int rb16 = (3 * W + 15) & ~15;
+  p.max_chunks = std::max(p.max_chunks, rb16 >> 4);
+  p.pair_stage = std::max(p.pair_stage, sdd_bulk_stage_bytes(W, H, sdd_h));
+  if ((pitch & 15) || ((uintptr_t)pixels & 15)) p.vec16 = false;
+}
+
+void sdd_plan_finish(SddPlan& p, int32_t sdd_w, int32_t sdd_h) {
+  (void)sdd_h;
+  const char* force = std::getenv("FFSVA_SDD_KERNEL");
+  const bool pair_ok = p.vec16 && sdd_bulk_ok(p.max_chunks, p.pair_stage);
+  p.variant = pair_ok && !(force && !std::strcmp(force, "stream")) ? kSddPair : kSddStream;
+  if (p.variant == kSddPair) {
+    p.stage_bytes = p.pair_stage;
+    p.smem = sdd_bulk_smem_bytes(p.pair_stage, sdd_w);
+  } else {
+    p.stage_bytes = 0;
+    p.smem = sdd_smem_bytes(p.max_chunks, sdd_w);
+  }
+}
+
+void sdd_plan_apply(const SddPlan& p, SddArgs& a) {
+  a.max_chunks = p.max_chunks;
+  a.vec16 = p.vec16;
+  a.bulk = p.variant == kSddPair;
+  a.stage_bytes = p.stage_bytes;
 }
 
 cudaError_t sdd_configure(size_t smem) {

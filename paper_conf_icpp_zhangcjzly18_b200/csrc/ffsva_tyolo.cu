@@ -21,6 +21,9 @@
 //     step. A 2- or 4-stage mbarrier ring overlaps copies with the MMAs, issued by one thread.
 //   * The 1x1 head (1024 -> 125) writes its fp32 outputs and counts, per row, the boxes whose score exceeds the
 //     threshold into the frame's counter (L171).
+#include <algorithm>
+#include <cstdlib>
+
 #include "ffsva_internal.h"
 #include "ffsva_ptx.h"
 
@@ -393,48 +396,91 @@ __global__ void tyolo_pool_s1_kernel(const __nv_bfloat16* in, __nv_bfloat16* out
 }
 
 // Q28 resize of each raw RGB8 frame to 416x416, x = v / 256 (Q29) as bf16 NHWC with a zero 4th channel. One CTA per
-// (frame, output row): the row's source rows are staged in shared memory with 16-byte loads (when the frame's rows
-// are 16-byte aligned), then each thread box-sums its output pixels from shared memory.
+// (frame, group of R output rows): thread 0 bulk-copies the group's source rows (one contiguous span of the frame,
+// L2 evict-first) into shared memory against an mbarrier — R is sized on the host so several CTAs per SM keep tens
+// of KB each in flight — then each thread box-sums output pixels from shared memory. Frames whose rows are not
+// 16-byte aligned (or whose span exceeds the stage) read their bytes straight from global memory.
 constexpr int kResizeThreads = 256;
-constexpr int kResizeMaxRows = 4;  // source rows per output row: ceil(H / 416) + 1 <= 4 for H <= 1248
+constexpr int kResizeMaxD = 1024;  // output size bound of the column-bound table
 
-__global__ void __launch_bounds__(kResizeThreads) tyolo_resize_kernel(const TyFrame* frames, int32_t D,
-                                                                     __nv_bfloat16* out) {
+// Q28 cell bounds: [floor(i*S/D), max(floor((i+1)*S/D), floor(i*S/D) + 1))
+__device__ __forceinline__ int rs_lo(int i, int S, int D) { return (int)(((int64_t)i * S) / D); }
+__device__ __forceinline__ int rs_hi(int i, int S, int D) {
+  const int lo = rs_lo(i, S, D), hi = (int)(((int64_t)(i + 1) * S) / D);
+  return hi > lo ? hi : lo + 1;
+}
+
+// floor(a / n) for a < 2^31 with a quotient < 2^16: float estimate + one remainder correction (box means <= 255)
+__device__ __forceinline__ uint32_t rs_div(uint32_t a, uint32_t n) {
+  uint32_t q = __float2uint_rz(__uint2float_rn(a) * __frcp_rn(__uint2float_rn(n)));
+  const int r = (int)(a - q * n);
+  if (r < 0) --q;
+  else if (r >= (int)n) ++q;
+  return q;
+}
+
+__global__ void __launch_bounds__(kResizeThreads) tyolo_resize_kernel(const TyFrame* frames, int32_t D, int32_t R,
+                                                                     int32_t stage_bytes, __nv_bfloat16* out) {
   extern __shared__ __align__(16) uint8_t rows_sm[];
-  const int f = blockIdx.x / D, oy = blockIdx.x - f * D;
+  __shared__ __align__(8) uint64_t bar;
+  __shared__ int2 xcell[kResizeMaxD];  // Q28 column bounds of every output column (32-bit: i * W < 2^31)
+  const int f = blockIdx.y;
+  const int oy0 = blockIdx.x * R, oy1 = min(oy0 + R, D);
   const TyFrame fr = frames[f];
-  int y0 = (int)(((int64_t)oy * fr.H) / D), y1 = (int)(((int64_t)(oy + 1) * fr.H) / D);
-  if (y1 <= y0) y1 = y0 + 1;
-  const int nrows = y1 - y0, rb = 3 * fr.W;
-  const int rb16 = (rb + 15) & ~15;
-  const bool staged = nrows <= kResizeMaxRows && ((fr.pitch & 15) == 0) && (((uintptr_t)fr.pixels & 15) == 0);
-  if (staged) {
-    const int chunks = rb16 >> 4;
-    for (int k = threadIdx.x; k < nrows * chunks; k += kResizeThreads) {
-      const int r = k / chunks, c = k - r * chunks;
-      reinterpret_cast<uint4*>(rows_sm + r * rb16)[c] =
-          __ldg(reinterpret_cast<const uint4*>(fr.pixels + (int64_t)(y0 + r) * fr.pitch) + c);
+  const int ylo = rs_lo(oy0, fr.H, D), yhi = rs_hi(oy1 - 1, fr.H, D);
+  const int rb = 3 * fr.W, rb16 = (rb + 15) & ~15;
+  const bool staged = ((fr.pitch & 15) == 0) && (((uintptr_t)fr.pixels & 15) == 0) && (yhi - ylo) * rb16 <= stage_bytes;
+  const uint32_t b = smem_addr(&bar);
+  if (staged && threadIdx.x == 0) {
+    mbar_init(b, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    const uint32_t bytes = (uint32_t)((yhi - ylo) * rb16);
+    mbar_expect_tx(b, bytes);
+    const uint8_t* src = fr.pixels + (int64_t)ylo * fr.pitch;
+    if (fr.pitch == rb16) {
+      asm volatile(
+          "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+          ::"r"(smem_addr(rows_sm)), "l"(src), "r"(bytes), "r"(b), "l"(pol) : "memory");
+    } else {
+      for (int y = 0; y < yhi - ylo; ++y)
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+            ::"r"(smem_addr(rows_sm + y * rb16)), "l"(src + (int64_t)y * fr.pitch), "r"((uint32_t)rb16), "r"(b),
+            "l"(pol) : "memory");
     }
-    __syncthreads();
   }
+  for (int i = threadIdx.x; i < D; i += kResizeThreads) {
+    const int lo = (int)(((uint32_t)i * (uint32_t)fr.W) / (uint32_t)D);
+    const int hi = (int)(((uint32_t)(i + 1) * (uint32_t)fr.W) / (uint32_t)D);
+    xcell[i] = make_int2(lo, hi > lo ? hi : lo + 1);
+  }
+  __syncthreads();  // barrier initialised, column bounds ready
+  if (staged) mbar_wait(b, 0);
   const float inv = 1.f / 256.f;
-  for (int ox = threadIdx.x; ox < D; ox += kResizeThreads) {
-    int x0 = (int)(((int64_t)ox * fr.W) / D), x1 = (int)(((int64_t)(ox + 1) * fr.W) / D);
-    if (x1 <= x0) x1 = x0 + 1;
-    uint32_t s0 = 0, s1 = 0, s2 = 0;
-    for (int r = 0; r < nrows; ++r) {
-      const uint8_t* row = staged ? rows_sm + r * rb16 : fr.pixels + (int64_t)(y0 + r) * fr.pitch;
-      for (int x = x0; x < x1; ++x) {
-        s0 += row[3 * x];
-        s1 += row[3 * x + 1];
-        s2 += row[3 * x + 2];
+  for (int oy = oy0; oy < oy1; ++oy) {
+    const int y0 = (int)(((uint32_t)oy * (uint32_t)fr.H) / (uint32_t)D);
+    const int yh = (int)(((uint32_t)(oy + 1) * (uint32_t)fr.H) / (uint32_t)D);
+    const int y1 = yh > y0 ? yh : y0 + 1;
+    __nv_bfloat16* orow = out + ((int64_t)f * D + oy) * D * 4;
+    for (int ox = threadIdx.x; ox < D; ox += kResizeThreads) {
+      const int2 xc = xcell[ox];
+      uint32_t s0 = 0, s1 = 0, s2 = 0;
+      for (int y = y0; y < y1; ++y) {
+        const uint8_t* row = staged ? rows_sm + (y - ylo) * rb16 : fr.pixels + (int64_t)y * fr.pitch;
+        for (int x = xc.x; x < xc.y; ++x) {
+          s0 += row[3 * x];
+          s1 += row[3 * x + 1];
+          s2 += row[3 * x + 2];
+        }
       }
+      const uint32_t nn = (uint32_t)((y1 - y0) * (xc.y - xc.x));
+      uint2 w;
+      w.x = pack_bf16((float)rs_div(s0 + nn / 2, nn) * inv, (float)rs_div(s1 + nn / 2, nn) * inv);
+      w.y = pack_bf16((float)rs_div(s2 + nn / 2, nn) * inv, 0.f);
+      *reinterpret_cast<uint2*>(orow + ox * 4) = w;
     }
-    const uint32_t nn = (uint32_t)(nrows * (x1 - x0));
-    uint2 w;
-    w.x = pack_bf16((float)((s0 + nn / 2) / nn) * inv, (float)((s1 + nn / 2) / nn) * inv);
-    w.y = pack_bf16((float)((s2 + nn / 2) / nn) * inv, 0.f);
-    *reinterpret_cast<uint2*>(out + (((int64_t)f * D + oy) * D + ox) * 4) = w;
   }
 }
 
@@ -478,16 +524,27 @@ cudaError_t launch_tyolo_pool_s1(const __nv_bfloat16* in, __nv_bfloat16* out, in
   return cudaGetLastError();
 }
 
-cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int32_t max_row_bytes,
+cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int32_t max_row_bytes, int32_t max_H,
                                 __nv_bfloat16* out, cudaStream_t st) {
-  const int smem = kResizeMaxRows * ((max_row_bytes + 15) & ~15);
-  static int configured = 0;
-  if (smem > 48 * 1024 && smem > configured) {
-    cudaError_t e = cudaFuncSetAttribute(tyolo_resize_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  // R output rows per CTA: the largest with a stage of <= ~48 KB (4 CTAs per SM); a group of R rows spans at most
+  // ceil(R*H/D) + 1 source rows (or R rows when H < D)
+  const int rb16 = (max_row_bytes + 15) & ~15;
+  const char* renv = std::getenv("FFSVA_TYOLO_RESIZE_ROWS");
+  auto span = [&](int r) { return std::max((r * max_H + D - 1) / D + 1, r); };
+  int R = 1;
+  if (renv) R = std::max(1, std::atoi(renv));
+  else
+    while (R < D && span(R + 1) * rb16 <= 48 * 1024) ++R;
+  const int stage = span(R) * rb16;
+  if (D > kResizeMaxD || stage > 200 * 1024) return cudaErrorInvalidValue;
+  static bool configured = false;  // opt in once: the default 48 KB limit also covers static and reserved memory
+  if (!configured) {
+    cudaError_t e = cudaFuncSetAttribute(tyolo_resize_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     if (e != cudaSuccess) return e;
-    configured = smem;
+    configured = true;
   }
-  tyolo_resize_kernel<<<(unsigned)(n * D), kResizeThreads, smem, st>>>(frames, D, out);
+  const dim3 grid((unsigned)((D + R - 1) / R), (unsigned)n);
+  tyolo_resize_kernel<<<grid, kResizeThreads, stage, st>>>(frames, D, R, stage, out);
   return cudaGetLastError();
 }
 

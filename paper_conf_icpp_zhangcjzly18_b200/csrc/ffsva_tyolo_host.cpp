@@ -218,17 +218,18 @@ TyConvArgs layer_args(const ffsva_tyolo* m, int l, int n, const __nv_bfloat16* i
 ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, const int32_t* targets, int n, int upto,
                        float thresh, cudaStream_t st, cudaEvent_t* ev, int* out_buf = nullptr) {
   DeviceCtx* ctx = m->ctx;
-  int max_row = 0;
+  int max_row = 0, max_H = 0;
   for (int i = 0; i < n; ++i) {
     const ffsva_stream_desc& d = frames[i].stream->desc;
     m->h_frames[i] = TyFrame{frames[i].pixels, d.row_pitch, d.width, d.height, targets ? targets[i] : 0, 0};
     max_row = std::max(max_row, 3 * d.width);
+    max_H = std::max(max_H, d.height);
   }
   cudaError_t e = cudaMemcpyAsync(m->d_frames, m->h_frames, sizeof(TyFrame) * n, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemsetAsync(m->d_counts, 0, 4 * (size_t)n, st);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO staging");
   if (ev) cudaEventRecord(ev[0], st);
-  if ((e = launch_tyolo_resize(m->d_frames, n, kIn, max_row, m->d_act[0], st)) != cudaSuccess)
+  if ((e = launch_tyolo_resize(m->d_frames, n, kIn, max_row, max_H, m->d_act[0], st)) != cudaSuccess)
     return cuda_fail(ctx, e, "T-YOLO resize");
   g_launches += 1;
   if (ev) cudaEventRecord(ev[1], st);

@@ -31,7 +31,8 @@ EXPORTS = ["ffsva_open_stream", "ffsva_set_reference", "ffsva_snm_load", "ffsva_
            "ffsva_get_reference",
            "ffsva_stream_info", "ffsva_stats_copy", "ffsva_close", "ffsva_last_error", "ffsva_kernel_launches",
            "ffsva_version", "ffsva_sched_create", "ffsva_sched_push", "ffsva_sched_tick", "ffsva_sched_depth",
-           "ffsva_sched_destroy", "ffsva_sched_set_policy", "ffsva_stream_image_bytes", "ffsva_stream_export",
+           "ffsva_sched_destroy", "ffsva_sched_set_policy", "ffsva_sched_set_pipeline", "ffsva_stream_image_bytes",
+           "ffsva_stream_export",
            "ffsva_stream_import", "ffsva_sched_stream_load", "ffsva_sched_detach", "ffsva_tyolo_load",
            "ffsva_tyolo_run", "ffsva_tyolo_layer_output", "ffsva_tyolo_profile", "ffsva_tyolo_destroy",
            "ffsva_sched_set_tyolo"]
@@ -133,6 +134,7 @@ def lib():
             "ffsva_sched_depth": [vp, vp, ctypes.POINTER(i32), ctypes.POINTER(i32)],
             "ffsva_sched_destroy": [vp],
             "ffsva_sched_set_policy": [vp, i32],
+            "ffsva_sched_set_pipeline": [vp, i32],
             "ffsva_stream_image_bytes": [vp, ctypes.POINTER(i64)],
             "ffsva_stream_export": [vp, vp, i64, i32, vp],
             "ffsva_stream_import": [i32, vp, i64, i32, ctypes.POINTER(vp)],
@@ -534,6 +536,15 @@ class Scheduler:
     def set_policy(self, policy: str) -> None:
         """'dynamic' (default), 'feedback' or 'static' (the §5.4 comparison mechanisms)."""
         ffsva_sched_set_policy(self.handle, policy)
+
+    def set_pipeline(self, on: bool) -> bool:
+        """Pipelined ticks (ffsva_sched_set_pipeline): tick k harvests cycle k-1's kernels and launches cycle k's
+        without waiting. Returns False (mode unchanged) while a cycle is still in flight when switching off."""
+        r = lib().ffsva_sched_set_pipeline(self.handle, int(bool(on)))
+        if r == FFSVA_EAGAIN:
+            return False
+        _check(r, "ffsva_sched_set_pipeline")
+        return True
 
     def destroy(self) -> None:
         if self.handle:

@@ -15,9 +15,10 @@ import numpy as np
 
 
 def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s=0.010, cuda_stream=None,
-              latency_budget_s=1.0, tyolo=None, num_tyolo=4):
+              latency_budget_s=1.0, tyolo=None, num_tyolo=4, pipelined=True):
     """streams[i]: ff.Stream; content[i]: (device frame tensor [n_content_frames, H, pitch]). tyolo: a Tyolo to run
-    the full three-filter cascade (SDD -> SNM -> T-YOLO, f1) instead of SDD -> SNM.
+    the full three-filter cascade (SDD -> SNM -> T-YOLO, f1) instead of SDD -> SNM. pipelined: ticks overlap the
+    previous cycle's kernels with this driver's host work (ffsva_sched_set_pipeline).
 
     Returns a dict of latency percentiles, refusals, backlog and throughput."""
     import torch
@@ -37,6 +38,7 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
     sched = Scheduler(ctx, max_frames_per_tick=max_frames_tick, snm_slots=max(4096, S * 12))
     if tyolo is not None:
         sched.set_tyolo(tyolo, num_tyolo=num_tyolo)
+    sched.set_pipeline(pipelined)
     ty_scored = 0
     lat = []
     refused = 0
@@ -98,6 +100,7 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
            "latency_max_s": float(L.max()),
            "mean_ms_per_tick": {"push_py": 1e3 * tim[0] / max(1, ticks), "sdd_cycle": 1e3 * tim[1] / max(1, ticks),
                                 "snm_cycle": 1e3 * tim[2] / max(1, ticks), "tick_call": 1e3 * tim[3] / max(1, ticks)}}
+    res["pipelined"] = bool(pipelined)
     if tyolo is not None:
         res["stages"] = "SDD -> SNM -> T-YOLO (f1)"
         res["tyolo_scored"] = int(ty_scored)

@@ -2,6 +2,7 @@
 // Built and run by tests/test_sched_policy.py with g++ (no CUDA).
 #include <cstdio>
 #include <cstdlib>
+#include <vector>
 
 #include "../paper_conf_icpp_zhangcjzly18_b200/csrc/ffsva_sched_policy.h"
 
@@ -170,6 +171,33 @@ int main() {
     CHECK(ty.size() == 2 && ty[0].frame_no == 2 && ty[1].frame_no == 4);
     p.pop_ty(ty);                                  // depth 1 <= 2: unblocked
     CHECK(p.pop_snm().size() == 1);
+  }
+  {  // the incremental totals (queued_*, total_*_blocked) equal the per-stream sums after a random trace
+    Policy p;
+    p.set_tyolo(true, 2);
+    uint32_t h = 12345u;
+    auto rnd = [&](uint32_t m) { h = h * 1664525u + 1013904223u; return (h >> 8) % m; };
+    std::vector<int> ids;
+    for (int i = 0; i < 7; ++i) ids.push_back(p.add_stream(1 + (int)rnd(3), 1 + (int)rnd(4), 1 + (int)rnd(5), 1 + (int)rnd(2)));
+    int64_t no = 0;
+    for (int step = 0; step < 400; ++step) {
+      for (int k = 0; k < 6; ++k) p.push(ids[rnd(7)], fr(no++));
+      for (auto& f : p.admit_sdd(1 + (int)rnd(20), 1 + (int)rnd(30))) p.sdd_done(f, rnd(3) != 0);
+      for (auto& pop : p.pop_snm()) for (auto& f : pop) p.snm_done(f, rnd(2) != 0);
+      if (rnd(2)) { std::vector<QFrame> ty; p.pop_ty(ty); }
+      if (step == 200) { p.remove_stream(ids[3]); ids[3] = p.add_stream(2, 2, 3, 1); }
+      int64_t qs = 0, qn = 0, qt = 0;
+      uint64_t bs = 0, bn = 0;
+      for (int i = 0; i < p.n_streams(); ++i) {
+        qs += (int64_t)p.stream(i).sdd.size();
+        qn += (int64_t)p.stream(i).snm.size();
+        qt += (int64_t)p.stream(i).ty.size();
+        bs += p.stream(i).sdd_blocked;
+        bn += p.stream(i).snm_blocked;
+      }
+      CHECK(qs == p.queued_sdd() && qn == p.queued_snm() && qt == p.queued_ty());
+      if (step < 200) CHECK(bs == p.total_sdd_blocked() && bn == p.total_snm_blocked());  // until a removal
+    }
   }
   if (failures == 0) std::printf("ALL PASS\n");
   return failures == 0 ? 0 : 1;

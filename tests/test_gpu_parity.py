@@ -51,12 +51,21 @@ def test_reference_parity(env, W, H, k):
 
 # ------------------------------------------------------------------ SDD stage (C1, C3)
 
-@pytest.mark.parametrize("kernel", ["auto", "stream"])
+K1_VARIANTS = ["auto", "stream"]
+
+
+def _force_k1(kernel, monkeypatch):
+    """FFSVA_SDD_KERNEL=stream forces the register-streaming K1 (auto takes the bulk-async CTA-pair kernel for
+    aligned rows)."""
+    if kernel != "auto":
+        monkeypatch.setenv("FFSVA_SDD_KERNEL", kernel)
+
+
+@pytest.mark.parametrize("kernel", K1_VARIANTS)
 def test_sdd_config1_all_frames(env, kernel, monkeypatch):
     """Config 1: 1 stream, 300 frames 640x360, 10% target rate: every frame bit-exact; pass count = planted."""
     ff, ctx, dev = env
-    if kernel == "stream":
-        monkeypatch.setenv("FFSVA_SDD_KERNEL", "stream")
+    _force_k1(kernel, monkeypatch)
     v = synth.Video(seed=1001, width=640, height=360, period=300, on_len=30)
     cam = Cam(ctx, v, 0, dev, k_ref=32, load_snm=False)
     host = cam.host_frames(list(range(300)))
@@ -71,15 +80,14 @@ def test_sdd_config1_all_frames(env, kernel, monkeypatch):
     cam.st.close()
 
 
-@pytest.mark.parametrize("kernel", ["auto", "stream"])
+@pytest.mark.parametrize("kernel", K1_VARIANTS)
 @pytest.mark.parametrize("W,H,pitch", [(100, 100, 300), (641, 361, 1923), (640, 360, 2048), (1280, 720, 3840),
                                        (1920, 1080, 5760), (600, 400, 1800), (600, 400, 1808), (101, 103, 303),
                                        (3840, 2160, 11520), (112, 200, 336), (160, 100, 480)])
 def test_sdd_edge_shapes(env, W, H, pitch, kernel, monkeypatch):
-    """Both K1 variants (bulk-async + cluster for aligned rows, register streaming otherwise / when forced)."""
+    """Both K1 variants (bulk-async CTA pairs for aligned rows, register streaming otherwise / when forced)."""
     ff, ctx, dev = env
-    if kernel == "stream":
-        monkeypatch.setenv("FFSVA_SDD_KERNEL", "stream")
+    _force_k1(kernel, monkeypatch)
     v = synth.Video(seed=W + H, width=W, height=H, period=4, on_len=2)
     cam = Cam(ctx, v, 3, dev, pitch=pitch, k_ref=2, load_snm=False)
     ts = list(range(5))
@@ -113,10 +121,15 @@ def test_sdd_random_bytes_extreme_values(env):
     st.close()
 
 
-def test_mixed_resolutions_and_streams_in_one_batch(env):
+@pytest.mark.parametrize("shapes,kernel", [
+    ([(640, 360), (1280, 720), (641, 361)], "auto"),                   # unaligned member: register streaming
+    ([(640, 360), (1280, 720), (1920, 1080), (112, 200)], "auto"),     # aligned, mixed heights and widths
+    ([(640, 360), (1280, 720), (1920, 1080), (112, 200)], "stream")])
+def test_mixed_resolutions_and_streams_in_one_batch(env, shapes, kernel, monkeypatch):
     ff, ctx, dev = env
+    _force_k1(kernel, monkeypatch)
     cams = [Cam(ctx, synth.Video(seed=5, width=W, height=H, period=6, on_len=3), s, dev, k_ref=2, load_snm=False)
-            for s, (W, H) in enumerate([(640, 360), (1280, 720), (641, 361)])]
+            for s, (W, H) in enumerate(shapes)]
     items, pairs, keep = [], [], []
     for t in range(6):
         for c in cams:
