@@ -414,7 +414,7 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
     for tok in args.online.split(","):
         tok = tok.strip()
         if tok == "auto":  # a ladder of fractions of the offline capacity, climbed until a count is not sustained
-            ladder = [max(31, int(f * value / 30)) for f in (0.55, 0.7, 0.85)]
+            ladder = [max(31, int(f * value / 30)) for f in (0.55, 0.65, 0.75, 0.85)]
         elif tok:
             counts.append(int(tok))
     nc = len(sids)
@@ -439,6 +439,7 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
     if ty_counts:
         import paper_conf_icpp_zhangcjzly18_b200 as ff
         ty = ff.Tyolo(ctx, synth.tyolo_weights(video.seed))
+    ty_warm = False
     ladder_failed = False
     for S, with_ty in runs:
         if S in ladder and not with_ty and ladder_failed:
@@ -452,8 +453,12 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
             st.snm_load(synth.snm_weights(video.seed, 100000 + i))
             opened.append(st)
         setup_s = time.perf_counter() - t_setup
+        if with_ty and not ty_warm:  # outside the paced window: the first T-YOLO launches load their modules
+            ty.run([(opened[0], pool[0][t], t) for t in range(2)], target_class=14, thresh=0.2)
+            ty_warm = True
+        # cycles of 10 ms, 25 ms from 10 K streams on (the driver's per-cycle work over all cameras is amortised)
         res = run_paced(ctx, opened[:S], [pool[i % nc] for i in range(S)], pool.shape[1], args.online_seconds,
-                        cuda_stream=cs, tyolo=ty if with_ty else None)
+                        cuda_stream=cs, tyolo=ty if with_ty else None, tick_s=0.010 if S < 10000 else 0.025)
         res["stream_setup_s"] = setup_s
         results.append(res)
         if S in ladder and not with_ty and not res["sustained"]:
@@ -583,7 +588,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--online", default="30,auto",
                     help="comma-separated stream counts for the paced online validation (config m2); 'auto' = "
-                         "a ladder of 55/70/85%% of the measured frames/s / 30, climbed until a count is not "
+                         "a ladder of 55/65/75/85%% of the measured frames/s / 30, climbed until a count is not "
                          "sustained; empty to skip")
     ap.add_argument("--online-seconds", type=float, default=4.0)
     ap.add_argument("--online-tyolo", default="2000,auto",

@@ -33,7 +33,6 @@
 
 #include <algorithm>
 #include <cstdint>
-#include <deque>
 #include <vector>
 
 namespace ffsva {
@@ -51,10 +50,39 @@ struct QFrame {
 
 enum class BatchPolicy : int32_t { DYNAMIC = 0, FEEDBACK = 1, STATIC = 2 };
 
+// FIFO of frames: a vector with a head index (pops advance the head; the storage is reset when the queue empties
+// and compacted when the dead prefix dominates). An empty queue owns no memory, so tens of thousands of streams
+// cost a few cache lines each (std::deque allocates a 512-byte chunk per queue up front).
+class Fifo {
+ public:
+  using const_iterator = std::vector<QFrame>::const_iterator;
+  size_t size() const { return v_.size() - h_; }
+  bool empty() const { return h_ == v_.size(); }
+  const QFrame& front() const { return v_[h_]; }
+  void push_back(const QFrame& f) { v_.push_back(f); }
+  void pop_front() { erase_front(1); }
+  void erase_front(size_t n) {
+    h_ += n;
+    if (h_ == v_.size()) {
+      v_.clear();
+      h_ = 0;
+    } else if (h_ >= 64 && 2 * h_ >= v_.size()) {
+      v_.erase(v_.begin(), v_.begin() + (std::ptrdiff_t)h_);
+      h_ = 0;
+    }
+  }
+  const_iterator begin() const { return v_.begin() + (std::ptrdiff_t)h_; }
+  const_iterator end() const { return v_.end(); }
+
+ private:
+  std::vector<QFrame> v_;
+  size_t h_ = 0;
+};
+
 struct StreamQ {
   int32_t q_sdd = 2, q_snm = 10, batch = 30, q_ty = 2;
   bool live = false;
-  std::deque<QFrame> sdd, snm, ty;
+  Fifo sdd, snm, ty;
   uint64_t pushed = 0, refused = 0, sdd_blocked = 0, snm_blocked = 0;
   int32_t max_sdd = 0, max_snm = 0, max_ty = 0;
 };
@@ -167,7 +195,7 @@ class Policy {
       StreamQ& s = st_[k];
       starts.push_back((int32_t)flat.size());
       flat.insert(flat.end(), s.snm.begin(), s.snm.begin() + take);
-      s.snm.erase(s.snm.begin(), s.snm.begin() + take);
+      s.snm.erase_front((size_t)take);
       nsnm_[k] -= take;
       nq_snm_ -= take;
     };
@@ -217,7 +245,7 @@ class Policy {
       StreamQ& s = st_[k];
       const int32_t take = std::min<int32_t>(ty_take_, (int32_t)s.ty.size());
       flat.insert(flat.end(), s.ty.begin(), s.ty.begin() + take);
-      s.ty.erase(s.ty.begin(), s.ty.begin() + take);
+      s.ty.erase_front((size_t)take);
       nty_[k] -= take;
       nq_ty_ -= take;
     }

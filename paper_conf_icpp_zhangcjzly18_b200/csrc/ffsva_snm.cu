@@ -60,7 +60,7 @@ constexpr int SMEM_BYTES = OFF_TMEM + 16;
 static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
 constexpr uint32_t kTmemCols = 512;
 
-constexpr int kTiles1 = 7, kTiles2 = 2;
+constexpr int kTiles1 = 7;
 __constant__ int8_t c1_py0[kTiles1] = {0, 4, 8, 12, 16, 20, 21};  // last tile overlaps (idempotent writes)
 
 // ---------------------------------------------------------------- PTX wrappers (sm_100a)
@@ -79,16 +79,21 @@ __host__ __device__ constexpr uint32_t idesc_bf16(int M, int N) {
   return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }
 
+// Issued by a whole warp with warp-uniform operands; elect.sync picks the one lane that issues (the same lane for
+// the MMAs and their commit). Warp-uniform descriptors stay in uniform registers: no per-MMA R2UR waterfall loop,
+// which made a single divergent issuing thread the bottleneck of this kernel.
 __device__ __forceinline__ void mma_bf16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
   asm volatile(
-      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(d_tmem),
+      "{\n\t.reg .pred p, e;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(d_tmem),
       "l"(a), "l"(b), "r"(idesc), "r"(acc));
 }
 
 __device__ __forceinline__ void mma_commit(uint32_t bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar)
-               : "memory");
+  asm volatile(
+      "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}\n" ::"r"(bar)
+      : "memory");
 }
 
 __device__ __forceinline__ void fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
@@ -289,7 +294,8 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
   float* red = reinterpret_cast<float*>(sm + OFF_RED);
   uint32_t* s_tmem = reinterpret_cast<uint32_t*>(sm + OFF_TMEM);
   __shared__ int s_chunk;
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, grp = warp >> 2;
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0), grp = warp >> 2;  // warp-uniform (uniform registers)
   const uint32_t bar0 = smem_addr(sm + OFF_BAR);  // bar0 + 8*i: i < 7 conv1 tiles, 7..8 conv2 tiles, 9..10 input
   const int n_chunks = a.counts[1];
   if (n_chunks == 0) return;  // no survivors in this batch
@@ -346,7 +352,7 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
     in_ph ^= 1u;
     convert_input(stage, A1, lut);
     fence_proxy_async();
-    const bool issuer = lane == 0 && (warp & 3) == 0;  // warp 0 issues group 0's tiles, warp 4 group 1's
+    const bool issuer = (warp & 3) == 0;  // warp 0 issues group 0's tiles, warp 4 group 1's (one elected lane)
     for (int j = start; j < end; ++j) {
       const int f = a.work[j];
       const int buf = (j - start) & 1;

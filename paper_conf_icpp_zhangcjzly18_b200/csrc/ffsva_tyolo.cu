@@ -160,7 +160,8 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
   const uint32_t full0 = smem_addr(bars), empty0 = full0 + 8 * S;
   const uint32_t accf0 = full0 + 16 * S, acce0 = accf0 + 8 * kMaxAccBufs;  // acc_full[NB], acc_empty[NB]
   const uint32_t As0 = smem_addr(As), Bs0 = smem_addr(Bs);
-  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);  // warp-uniform (role branches, MMA issue)
   const int rows_per_tile = 128 * MS;
   const int n_tiles = a.Cout_tiles, tiles = ((a.M + rows_per_tile - 1) / rows_per_tile) * n_tiles;
 
@@ -222,11 +223,11 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
     fence_proxy_async();
     for (int h = g - lag < 0 ? 0 : g - lag; h < g; ++h) mbar_arrive(full0 + 8 * (h % S));
   } else if (warp == 4) {
-    // ---------------- MMA issue (one thread)
+    // ---------------- MMA issue (the whole warp, one elected lane issues: ffsva_ptx.h mma_bf16)
     // Descriptors are built once; per MMA only their start-address fields advance (byte offset >> 4 added to the
-    // low 14 bits, which cannot carry: shared addresses stay below 256 KB), so the single issuing thread spends a
-    // few instructions per MMA instead of rebuilding two 64-bit descriptors.
-    if (lane == 0) {
+    // low 14 bits, which cannot carry: shared addresses stay below 256 KB), so the issuing warp spends a few
+    // instructions per MMA instead of rebuilding two 64-bit descriptors.
+    {
       const uint32_t idesc = idesc_bf16(128, NT);
       const uint64_t a_base = umma_desc(As0, 2048, 128), b_base = umma_desc(Bs0, (uint32_t)NT * 16, 128);
       const uint32_t a_tile16 = (uint32_t)kATile >> 4, b_tile16 = b_tile >> 4, b_ks16 = (uint32_t)(2 * NT * 16) >> 4;

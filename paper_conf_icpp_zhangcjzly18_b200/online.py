@@ -45,7 +45,7 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
     done = 0
     max_backlog = 0
     ticks = 0
-    tim = [0.0, 0.0, 0.0, 0.0]  # python push, SDD cycle, SNM cycle, whole tick call (s)
+    tim = [0.0, 0.0, 0.0, 0.0, 0.0]  # python push, SDD cycle, SNM cycle, whole tick call, python events (s)
     try:
         torch.cuda.synchronize()
         t0 = time.perf_counter() + 0.05
@@ -86,6 +86,7 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
                 arrival = t0 + phase[si] + ev["frame_no"].astype(np.float64) / fps
                 lat.append(t_done - arrival)
                 done += ev.size
+            tim[4] += time.perf_counter() - t_done
             rest = tick_s - (time.perf_counter() - now)
             if rest > 0:
                 time.sleep(rest)
@@ -99,7 +100,8 @@ def run_paced(ctx, streams, content, n_content_frames, seconds, fps=30.0, tick_s
            "latency_p50_s": float(np.percentile(L, 50)), "latency_p99_s": float(np.percentile(L, 99)),
            "latency_max_s": float(L.max()),
            "mean_ms_per_tick": {"push_py": 1e3 * tim[0] / max(1, ticks), "sdd_cycle": 1e3 * tim[1] / max(1, ticks),
-                                "snm_cycle": 1e3 * tim[2] / max(1, ticks), "tick_call": 1e3 * tim[3] / max(1, ticks)}}
+                                "snm_cycle": 1e3 * tim[2] / max(1, ticks), "tick_call": 1e3 * tim[3] / max(1, ticks),
+                                "events_py": 1e3 * tim[4] / max(1, ticks)}}
     res["pipelined"] = bool(pipelined)
     if tyolo is not None:
         res["stages"] = "SDD -> SNM -> T-YOLO (f1)"
