@@ -289,7 +289,7 @@ FFSVA_API ffsva_status ffsva_sched_set_pipeline(ffsva_sched* s, int32_t on);
  *
  * Stream image: a self-contained byte image of a stream — its descriptor, thresholds, reference image R, packed
  * SNM weights and its per-stream statistics row — so the stream continues bit-identically elsewhere.
- *   ffsva_stream_image_bytes: size of s's image (64,320 B at the default 100x100 grid);
+ *   ffsva_stream_image_bytes: size of s's image (57,152 B at the default 100x100 grid);
  *   ffsva_stream_export: write the image to dst (host memory, or device memory on s's device when dst_is_host
  *     is 0 — e.g. a buffer about to be sent over NCCL); synchronous on cuda_stream;
  *   ffsva_stream_import: open a new stream on `device` from an image (host memory, or device memory on `device`

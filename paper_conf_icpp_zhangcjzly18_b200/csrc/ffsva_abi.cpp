@@ -375,7 +375,7 @@ FFSVA_API ffsva_status ffsva_stats_copy(int32_t device, uint64_t* dst, int32_t m
 // ---------------------------------------------------------------- stream images (re-forwarding)
 namespace {
 constexpr uint32_t kImageMagic = 0x56534646u;  // "FFSV"
-constexpr uint32_t kImageVersion = 2;  // 2: descriptor with NumberofObjects, target class, q_tyolo
+constexpr uint32_t kImageVersion = 3;  // 3: SNM image with patch-row conv1 operands and bf16 FC weights
 constexpr int64_t kImageHeader = 256;
 struct ImageHeader {
   uint32_t magic, version;

@@ -34,19 +34,19 @@ constexpr int C1 = 16, C2 = 32;
 constexpr int IN = 50, P1 = 25, P2 = 12;             // input, pooled conv1, pooled conv2 (floor)
 constexpr int NF = C2 * P2 * P2;                    // 4608 FC inputs
 constexpr int N_PARAMS = 27 * C1 + C1 + 9 * C1 * C2 + C2 + NF + 1;  // 9697
-// conv1 B operands: for pool column offset b in {0,1} and tap row dy in {0,1,2}: [0] the pair of taps dx in
-// {0,1} (K-half 0 = the tap in the x-even parity plane: dx = b; K-half 1 = dx = 1 - b), [1] tap dx = 2 in
-// K-half 0 and zero weights in K-half 1. Each is [2 K-halves][16 n][8 channel slots] bf16 (3 slots used).
-constexpr int CONV1_B = 12;
-constexpr int W1_BYTES = CONV1_B * 2 * C1 * 16;     // 6144
+// conv1 B operands, one per 4x4-patch row dy (the MMA's A rows are pooled pixels' 4x4 input patches, 4 channel
+// slots per pixel): N = 64 = [pool position q = 2a + b][16 output channels], K = 16 = [patch column u][4 channel
+// slots], value w1[oc][c][dy - a][u - b] where that tap exists (c < 3), else 0. Each is [2 K-halves][64 n][8 k] bf16.
+constexpr int W1_MMAS = 4;
+constexpr int W1_BYTES = W1_MMAS * 2 * 64 * 16;     // 8192
 constexpr int W2_BYTES = 9 * 2 * C2 * 16;           // 9216: [tap][channel half][32 n][8] bf16
 constexpr int OFF_W1 = 0;
-constexpr int OFF_W2 = OFF_W1 + W1_BYTES;           // 6144
-constexpr int OFF_B1 = OFF_W2 + W2_BYTES;           // 15360 (fp32[16])
-constexpr int OFF_B2 = OFF_B1 + C1 * 4;             // 15424 (fp32[32])
-constexpr int OFF_BFC = OFF_B2 + C2 * 4;            // 15552 (fp32[1] + pad to 16)
-constexpr int OFF_WFC = OFF_BFC + 16;               // 15568 (fp32[4608], bf16-exact values)
-constexpr int BLOB_BYTES = OFF_WFC + NF * 4;        // 34000
+constexpr int OFF_W2 = OFF_W1 + W1_BYTES;           // 8192
+constexpr int OFF_B1 = OFF_W2 + W2_BYTES;           // 17408 (fp32[16])
+constexpr int OFF_B2 = OFF_B1 + C1 * 4;             // 17472 (fp32[32])
+constexpr int OFF_BFC = OFF_B2 + C2 * 4;            // 17600 (fp32[1] + pad to 16)
+constexpr int OFF_WFC = OFF_BFC + 16;               // 17616 (bf16[4608]: the weights are bf16 values, L159 Q15)
+constexpr int BLOB_BYTES = OFF_WFC + NF * 2;        // 26832
 static_assert(BLOB_BYTES % 16 == 0, "blob must be 16-B granular");
 }  // namespace snm
 
@@ -136,6 +136,7 @@ struct SnmArgs {
   float* dbg_p2;             // [m][32][12][12]
 };
 cudaError_t launch_snm(const SnmArgs& a, cudaStream_t st);
+constexpr int kSnmCtasPerSm = 2;  // K4 is persistent with two CTAs per SM (256 TMEM columns, < 113 KB smem each)
 int snm_smem_bytes();
 cudaError_t snm_configure();
 

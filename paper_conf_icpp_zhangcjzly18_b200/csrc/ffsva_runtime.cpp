@@ -209,7 +209,7 @@ uint16_t bf16_bits_rne(float x) {
   return (uint16_t)((u + 0x7FFFu + ((u >> 16) & 1u)) >> 16);
 }
 
-static float bf16_value(float x) {
+[[maybe_unused]] static float bf16_value(float x) {
   uint32_t u = (uint32_t)bf16_bits_rne(x) << 16;
   float f;
   std::memcpy(&f, &u, 4);
@@ -233,20 +233,19 @@ void pack_snm_blob(const float* params, uint8_t* blob) {
   const float* b2 = w2 + 9 * C1 * C2;
   const float* wfc = b2 + C2;
   const float* bfc = wfc + NF;
-  // conv1: B matrix (b, dy, kind); kind 0 = taps (dx = b, dx = 1 - b) in K-halves (0, 1); kind 1 = tap dx = 2
-  // in K-half 0, zero K-half 1. Channels 0..2 of the 8 slots.
+  // conv1: B matrix of patch row dy: n = 16q + oc (q = 2a + b), k = 4u + c (patch column u, channel slot c);
+  // K-half h holds patch columns 2h, 2h+1. The 3x3 kernel of pool position (a, b) sits at offset (a, b) of the patch.
   uint16_t* W1 = reinterpret_cast<uint16_t*>(blob + OFF_W1);
-  for (int b = 0; b < 2; ++b)
-    for (int dy = 0; dy < 3; ++dy)
-      for (int kind = 0; kind < 2; ++kind)
-        for (int h = 0; h < 2; ++h) {
-          const int dx = kind == 0 ? (h == 0 ? b : 1 - b) : (h == 0 ? 2 : -1);
-          if (dx < 0) continue;
-          const int m = (b * 3 + dy) * 2 + kind;
-          for (int n = 0; n < C1; ++n)
-            for (int c = 0; c < 3; ++c)
-              W1[((m * 2 + h) * C1 + n) * 8 + c] = bf16_bits_rne(w1[((n * 3 + c) * 3 + dy) * 3 + dx]);
-        }
+  for (int dy = 0; dy < 4; ++dy)
+    for (int q = 0; q < 4; ++q)
+      for (int oc = 0; oc < C1; ++oc)
+        for (int u = 0; u < 4; ++u)
+          for (int c = 0; c < 3; ++c) {
+            const int ky = dy - (q >> 1), kx = u - (q & 1);
+            if (ky < 0 || ky > 2 || kx < 0 || kx > 2) continue;
+            const int n = 16 * q + oc, h = u >> 1, kk = 4 * (u & 1) + c;
+            W1[((dy * 2 + h) * 64 + n) * 8 + kk] = bf16_bits_rne(w1[((oc * 3 + c) * 3 + ky) * 3 + kx]);
+          }
   // conv2: tap t, K-half h = input channels 8h..8h+7
   uint16_t* W2 = reinterpret_cast<uint16_t*>(blob + OFF_W2);
   for (int t = 0; t < 9; ++t)
@@ -257,8 +256,8 @@ void pack_snm_blob(const float* params, uint8_t* blob) {
   std::memcpy(blob + OFF_B1, b1, C1 * 4);
   std::memcpy(blob + OFF_B2, b2, C2 * 4);
   std::memcpy(blob + OFF_BFC, bfc, 4);
-  float* F = reinterpret_cast<float*>(blob + OFF_WFC);
-  for (int i = 0; i < NF; ++i) F[i] = bf16_value(wfc[i]);
+  uint16_t* F = reinterpret_cast<uint16_t*>(blob + OFF_WFC);
+  for (int i = 0; i < NF; ++i) F[i] = bf16_bits_rne(wfc[i]);
 }
 
 // ------------------------------------------------------------------ batches
@@ -455,7 +454,7 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
 }
 
 // SNM grid: one persistent CTA per SM (the kernel holds all 512 TMEM columns), no more CTAs than frames.
-int snm_grid(const Batch* b) { return std::max(1, std::min(b->n, b->ctx->num_sms)); }
+int snm_grid(const Batch* b) { return std::max(1, std::min(b->n, kSnmCtasPerSm * b->ctx->num_sms)); }
 
 SddArgs make_sdd_args(Batch* b, int32_t i0, int32_t cnt) {
   SddArgs sa{};

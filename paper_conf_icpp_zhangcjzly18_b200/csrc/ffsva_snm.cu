@@ -8,27 +8,26 @@
 // to bf16, conv2 output and FC in fp32 (Q15).
 //
 // B200 mapping — implicit GEMM, no im2col, pooling folded into the N dimension:
-//   * GEMM rows are POOLED output pixels. For each of the four 2x2-pool positions q = (a, b) the conv
-//     output (2py+a, 2px+b) is one MMA chain into its own TMEM column group, so the max-pool is an in-register
-//     max over four column groups of the same TMEM lane (no cross-lane shuffles); bias and ReLU commute with
-//     max and are applied once after it.
-//   * Inputs live in shared memory as four parity planes (even/odd padded row x even/odd padded column),
-//     pixel-major with 8 channels per 16-byte row (one K-major no-swizzle core-matrix row). The input pixel
-//     of pooled row py, column px, pool position (a,b), tap (dy,dx) is (2py+a+dy, 2px+b+dx) = parity plane
-//     ((a+dy)&1, (b+dx)&1), plane pixel (py + (a+dy)>>1, px + (b+dx)>>1): a constant-stride view, so each tap
-//     of each pool position is the same UMMA descriptor shifted by a few bytes (SBO = 8 pixels = 128 B; plane
-//     rows are 32 (conv1) / 16 (conv2) pixels so rows continue the 128-B core-matrix stride).
-//   * conv1 (3 channels in 8 slots): two taps that sit in the two x-parity planes share one K=16 MMA (LBO =
-//     the plane distance); 24 MMAs (M128, N16) per tile x 7 tiles of 4 pooled rows x 32 px.
-//     conv2 (16 channels = two 8-channel planes, LBO = plane distance): 36 MMAs (M128, N32) per tile x 2 tiles
-//     of 8 pooled rows x 16 px.
+//   * GEMM rows are POOLED output pixels; a 2x2-pool's four conv outputs are four accumulator column groups of the
+//     same TMEM lane, so the max-pool is an in-register max over four column groups (no cross-lane shuffles); bias
+//     and ReLU commute with max and are applied once after it.
+//   * conv1: the A row of pooled pixel (py, px) is its 4x4 input patch (padded rows 2py..2py+3, columns
+//     2px..2px+3) x 4 channel slots (3 used); the four pool positions differ only in where their 3x3 kernel sits in
+//     the patch, so ONE A operand feeds N = 64 = 4 positions x 16 channels with per-position (zero-padded) weights:
+//     4 MMAs (M128 N64 K16, one per patch row) per tile of 4 pooled rows x 32 px instead of 24 narrow ones. The
+//     input lives in two row-parity planes of 64-px rows, 8 bytes per pixel, so a patch row of consecutive pooled
+//     pixels is a constant-stride view (rows 16 B apart, K-halves 16 B apart, 8-row groups 128 B apart): each
+//     patch row is the same UMMA descriptor moved by one plane row.
+//   * conv2 (16 channels = two 8-channel planes, LBO = plane distance): per pool position and tap one MMA
+//     (M128, N32) per tile x 2 tiles of 8 pooled rows x 16 px, A from four parity planes like conv1's patch rows.
 //   * conv1's epilogue writes bf16 pooled activations straight into conv2's parity planes; conv2's epilogue
-//     multiplies the pooled features by the FC weights in fp32 and reduces to one logit per frame.
-// One persistent CTA per SM (8 warps; warp w reads TMEM lane quadrant w%4, warp groups split the tiles), all
-// 512 TMEM columns; thread 0 issues every MMA and commits each tile to its own mbarrier so epilogues start as
-// soon as a tile lands. Work = dynamic-batch units (<= BatchSize survivors of one stream, split further when
-// the batch is small); the stream's 34 KB weight image is copied into shared memory once per unit (skipped when
-// the previous unit was the same stream), and the next frame's D50 image is prefetched with a bulk copy.
+//     multiplies the pooled features by the FC weights (bf16 values) in fp32 and reduces to one logit per frame.
+// Two persistent CTAs per SM (8 warps and 256 TMEM columns each: conv1 runs as two waves of <= 4 tiles, conv2's two
+// tiles reuse the columns), so one CTA's epilogues overlap the other's MMAs. MMAs are issued by a whole warp (one
+// elected lane) per warp group and committed per tile to its own mbarrier so epilogues start as soon as a tile lands.
+// Work = dynamic-batch units (<= BatchSize survivors of one stream, split further when the batch is small); the
+// stream's 26 KB weight image is copied into shared memory once per unit (skipped when the previous unit was the
+// same stream), and the next frame's D50 image is prefetched with a bulk copy.
 #include <cuda_bf16.h>
 
 #include "ffsva_internal.h"
@@ -39,26 +38,28 @@ namespace {
 using namespace snm;
 
 constexpr int kThreads = 256;
-// conv1 operand: 4 parity planes [ypar][xpar] x 27 rows x 32 px x 16 B (padded input 52x52, 3 of 8 channels)
-constexpr int A1_COLS = 32, A1_ROWS = 27;
-constexpr int A1_PLANE = A1_ROWS * A1_COLS * 16;            // 13824
-constexpr int A1_BYTES = 4 * A1_PLANE;                      // 55296
+// conv1 operand: 2 row-parity planes x 27 rows x 64 px x 8 B (padded input 52x52, 4 channel slots, 3 used)
+constexpr int A1_COLS = 64, A1_ROWS = 27;
+constexpr int A1_ROWB = A1_COLS * 8;                        // 512: pooled row -> next plane row = four 8-row groups
+constexpr int A1_PLANE = A1_ROWS * A1_ROWB;                 // 13824
+constexpr int A1_BYTES = 2 * A1_PLANE + 512;                // + tail read by junk columns of the last plane row
 // conv2 operand: 8 planes [ypar][xpar][chalf] x 14 rows x 16 px x 16 B (padded pooled conv1 27x27, 16 ch)
 constexpr int A2_COLS = 16, A2_ROWS = 14;
 constexpr int A2_PLANE = A2_ROWS * A2_COLS * 16;            // 3584
 constexpr int A2_BYTES = 8 * A2_PLANE + 512;                // + zero tail read by junk rows of the last tile
 constexpr int D50_BYTES = 7504;                             // staged D50 image (one frame)
 constexpr int OFF_A1 = 0;
-constexpr int OFF_A2 = OFF_A1 + A1_BYTES;                   // 55296
-constexpr int OFF_WB = OFF_A2 + A2_BYTES;                   // 84480
+constexpr int OFF_A2 = OFF_A1 + A1_BYTES;                   // 28160
+constexpr int OFF_WB = OFF_A2 + A2_BYTES;                   // 57344
 constexpr int OFF_IN = OFF_WB + BLOB_BYTES;                 // 2 staging buffers
 constexpr int OFF_LUT = OFF_IN + 2 * D50_BYTES;             // u16[256]: bf16 bits of (v - 128) / 128
 constexpr int OFF_RED = OFF_LUT + 512;
 constexpr int OFF_BAR = OFF_RED + 64;                       // 7 conv1 + 2 conv2 + 2 input mbarriers
 constexpr int OFF_TMEM = OFF_BAR + 16 * 8;
 constexpr int SMEM_BYTES = OFF_TMEM + 16;
-static_assert(SMEM_BYTES <= 227 * 1024, "shared memory budget");
-constexpr uint32_t kTmemCols = 512;
+static_assert(SMEM_BYTES <= 113 * 1024, "two CTAs per SM");
+static_assert(OFF_A2 % 16 == 0 && OFF_WB % 16 == 0 && OFF_IN % 16 == 0, "16-byte alignment");
+constexpr uint32_t kTmemCols = 256;
 
 constexpr int kTiles1 = 7;
 __constant__ int8_t c1_py0[kTiles1] = {0, 4, 8, 12, 16, 20, 21};  // last tile overlaps (idempotent writes)
@@ -174,8 +175,9 @@ __device__ __forceinline__ const uint8_t* d50_of(const SnmArgs& a, int f) {
 }
 
 // ---------------------------------------------------------------- input staging
-// D50 (50x50x3 u8, row-major) -> (v-128)/128 bf16 (C5, exact) into conv1's parity planes. Groups of 4 pixels =
-// 12 bytes = three aligned 32-bit shared loads; each channel through a 256-entry bf16 table.
+// D50 (50x50x3 u8, row-major) -> (v-128)/128 bf16 (C5, exact) into conv1's row-parity planes, one 8-byte pixel
+// (3 channels + a zero slot) per store. Groups of 4 pixels = 12 bytes = three aligned 32-bit shared loads; each
+// channel through a 256-entry bf16 table.
 __device__ __forceinline__ void convert_input(const uint8_t* d, uint8_t* A1, const uint16_t* lut) {
   constexpr int kGroups = snm::IN * snm::IN / 4;  // 625
   for (int g = threadIdx.x; g < kGroups; g += kThreads) {
@@ -189,35 +191,24 @@ __device__ __forceinline__ void convert_input(const uint8_t* d, uint8_t* A1, con
       const int p = 4 * g + q;
       const int y = p / snm::IN, x = p - y * snm::IN;
       const int Y = y + 1, X = x + 1;
-      const uint4 v = make_uint4((uint32_t)lut[b[3 * q]] | ((uint32_t)lut[b[3 * q + 1]] << 16),
-                                 (uint32_t)lut[b[3 * q + 2]], 0u, 0u);
-      *reinterpret_cast<uint4*>(A1 + ((Y & 1) * 2 + (X & 1)) * A1_PLANE + ((Y >> 1) * A1_COLS + (X >> 1)) * 16) = v;
+      const uint2 v = make_uint2((uint32_t)lut[b[3 * q]] | ((uint32_t)lut[b[3 * q + 1]] << 16), (uint32_t)lut[b[3 * q + 2]]);
+      *reinterpret_cast<uint2*>(A1 + (Y & 1) * A1_PLANE + (Y >> 1) * A1_ROWB + X * 8) = v;
     }
   }
 }
 
 // ---------------------------------------------------------------- MMA issue (one thread per warp group)
-__device__ __forceinline__ void issue_conv1_tile(uint32_t tmem, int t, uint32_t a1, uint32_t w1) {
+// conv1 tile t (pooled rows py0..py0+3 x 32 px) into TMEM columns col..col+63 ([pool position][16 channels]):
+// patch row dy of pooled row py is padded input row 2py + dy = plane (dy & 1), plane row py + (dy >> 1).
+__device__ __forceinline__ void issue_conv1_tile(uint32_t tmem, uint32_t col, int t, uint32_t a1, uint32_t w1) {
   const int py0 = c1_py0[t];
-  const uint32_t idesc = idesc_bf16(128, 16);
+  const uint32_t idesc = idesc_bf16(128, 64);
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    const int a = q >> 1, b = q & 1;
-    const uint32_t d = tmem + (uint32_t)(t * 64 + q * 16);
-#pragma unroll
-    for (int dy = 0; dy < 3; ++dy) {
-      const int ypar = (a + dy) & 1, roff = (a + dy) >> 1;
-      const uint32_t rowbase = a1 + (uint32_t)(ypar * 2 * A1_PLANE + (py0 + roff) * A1_COLS * 16);
-      // taps dx = 0, 1 (one in each x-parity plane) share one MMA: the x-even tap is the first K-half
-      const int coff = b;  // x-even tap sits one plane column further right when b = 1
-      const uint64_t ad_pair = umma_desc(rowbase + (uint32_t)(coff * 16), (uint32_t)(A1_PLANE - 16 * coff), 128);
-      const uint64_t bd_pair = umma_desc(w1 + (uint32_t)(((b * 3 + dy) * 2 + 0) * 512), C1 * 16, 128);
-      mma_bf16(d, ad_pair, bd_pair, idesc, dy > 0 ? 1u : 0u);
-      // tap dx = 2: x-parity b, plane column 1; second K-half carries zero weights
-      const uint64_t ad_one = umma_desc(rowbase + (uint32_t)(b * A1_PLANE + 16), 16, 128);
-      const uint64_t bd_one = umma_desc(w1 + (uint32_t)(((b * 3 + dy) * 2 + 1) * 512), C1 * 16, 128);
-      mma_bf16(d, ad_one, bd_one, idesc, 1u);
-    }
+  for (int dy = 0; dy < 4; ++dy) {
+    const uint32_t arow = a1 + (uint32_t)((dy & 1) * A1_PLANE + (py0 + (dy >> 1)) * A1_ROWB);
+    // K-halves = patch columns (0,1) and (2,1+2): 16 B apart; 8-row groups (8 pooled px) 128 B apart
+    mma_bf16(tmem + col, umma_desc(arow, 16, 128), umma_desc(w1 + (uint32_t)(dy * 2 * 64 * 16), 64 * 16, 128), idesc,
+             dy > 0 ? 1u : 0u);
   }
 }
 
@@ -241,10 +232,11 @@ __device__ __forceinline__ void issue_conv2_tile(uint32_t tmem, int u, uint32_t 
 
 // ---------------------------------------------------------------- epilogues
 // conv1 tile t: lane (quadrant qd, l) = pooled pixel (py0 + qd, l); bias, ReLU, bf16 into conv2's planes.
-__device__ __forceinline__ void conv1_epilogue(uint32_t tmem, int t, uint8_t* A2, const float* b1, uint16_t* dbg) {
+__device__ __forceinline__ void conv1_epilogue(uint32_t tmem, uint32_t col, int t, uint8_t* A2, const float* b1,
+                                               uint16_t* dbg) {
   const int qd = (threadIdx.x >> 5) & 3, l = threadIdx.x & 31;
   float v[16];
-  pooled16(tmem + ((uint32_t)(32 * qd) << 16), t * 64, 16, v);
+  pooled16(tmem + ((uint32_t)(32 * qd) << 16), (int)col, 16, v);
   const int py = c1_py0[t] + qd, px = l;
   if (px < P1) {
     uint32_t w[8];
@@ -263,7 +255,7 @@ __device__ __forceinline__ void conv1_epilogue(uint32_t tmem, int t, uint8_t* A2
 }
 
 // conv2 tile u: lane (qd, l) = pooled pixel (4u + 2qd + (l >> 4), l & 15); returns the FC partial sum.
-__device__ __forceinline__ float conv2_epilogue(uint32_t tmem, int u, const float* b2, const float* wfc, float* dbg) {
+__device__ __forceinline__ float conv2_epilogue(uint32_t tmem, int u, const float* b2, const uint16_t* wfc, float* dbg) {
   const int qd = (threadIdx.x >> 5) & 3, l = threadIdx.x & 31;
   const int py = 4 * u + 2 * qd + (l >> 4), px = l & 15;
   const bool own = px < P2 && (u == 0 ? py < 8 : py >= 8);
@@ -277,7 +269,7 @@ __device__ __forceinline__ float conv2_epilogue(uint32_t tmem, int u, const floa
       for (int i = 0; i < 16; ++i) {
         const int c = 16 * h + i;
         const float r = fmaxf(v[i] + b2[c], 0.f);
-        acc = fmaf(r, wfc[c * (P2 * P2) + py * P2 + px], acc);
+        acc = fmaf(r, __uint_as_float((uint32_t)wfc[c * (P2 * P2) + py * P2 + px] << 16), acc);
         if (dbg) dbg[c * (P2 * P2) + py * P2 + px] = r;
       }
     }
@@ -285,7 +277,7 @@ __device__ __forceinline__ float conv2_epilogue(uint32_t tmem, int u, const floa
   return acc;
 }
 
-__global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
+__global__ void __launch_bounds__(kThreads, kSnmCtasPerSm) snm_kernel(SnmArgs a) {
   extern __shared__ __align__(1024) uint8_t sm[];
   uint8_t* A1 = sm + OFF_A1;
   uint8_t* A2 = sm + OFF_A2;
@@ -320,7 +312,7 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
   const uint32_t w1 = smem_addr(WB + OFF_W1), w2 = smem_addr(WB + OFF_W2);
   const float* b1 = reinterpret_cast<const float*>(WB + OFF_B1);
   const float* b2 = reinterpret_cast<const float*>(WB + OFF_B2);
-  const float* wfc = reinterpret_cast<const float*>(WB + OFF_WFC);
+  const uint16_t* wfc = reinterpret_cast<const uint16_t*>(WB + OFF_WFC);
   uint32_t ph = 0;           // parity of the per-frame mbarriers (one phase per frame)
   uint32_t in_ph = 0;        // bit i: parity of input staging buffer i
   const uint8_t* loaded = nullptr;  // weight image currently in shared memory
@@ -359,20 +351,30 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
       fence_before();
       __syncthreads();  // frame j's conv1 operand (and the unit's weights) are in shared memory
 
-      // ---- conv1: 7 tiles, each warp group issues and drains its own (one commit per tile)
-      if (issuer) {
-        fence_after();
-        for (int t = grp; t < kTiles1; t += 2) {
-          issue_conv1_tile(tmem, t, a1, w1);
-          mma_commit(bar0 + 8 * t);
-        }
-      }
-      __syncwarp();
+      // ---- conv1: 7 tiles in two waves of TMEM columns (tile t -> columns (t % 4) * 64); each warp group issues
+      // and drains its own tiles (0, 2 | 4, 6 and 1, 3 | 5), one commit per tile. Wave B reuses wave A's columns of
+      // the same group once the whole group has read them (named barrier 1 + grp over its 128 threads).
       uint16_t* dbg1 = a.dbg_p1 ? a.dbg_p1 + (int64_t)j * (P1 * P1 * 16) : nullptr;
-      for (int t = grp; t < kTiles1; t += 2) {
-        mbar_wait(bar0 + 8 * t, ph);
-        fence_after();
-        conv1_epilogue(tmem, t, A2, b1, dbg1);
+#pragma unroll
+      for (int wave = 0; wave < 2; ++wave) {
+        if (issuer) {
+          fence_after();
+          for (int t = grp + 4 * wave; t < min(kTiles1, 4 * wave + 4); t += 2) {
+            issue_conv1_tile(tmem, (uint32_t)((t & 3) * 64), t, a1, w1);
+            mma_commit(bar0 + 8 * t);
+          }
+        }
+        __syncwarp();
+        for (int t = grp + 4 * wave; t < min(kTiles1, 4 * wave + 4); t += 2) {
+          mbar_wait(bar0 + 8 * t, ph);
+          fence_after();
+          conv1_epilogue(tmem, (uint32_t)((t & 3) * 64), t, A2, b1, dbg1);
+        }
+        if (wave == 0) {  // the group's wave-A columns are drained before its wave-B MMAs overwrite them
+          fence_before();
+          if (grp == 0) asm volatile("bar.sync 1, 128;" ::: "memory");
+          else asm volatile("bar.sync 2, 128;" ::: "memory");
+        }
       }
       fence_proxy_async();  // conv1's epilogue wrote conv2's operand through the generic proxy
       fence_before();
