@@ -313,7 +313,8 @@ __device__ __forceinline__ void st_async_u32(uint32_t raddr, uint32_t v, uint32_
                : "memory");
 }
 
-constexpr int kBulkThreads = 256;
+constexpr int kBulkThreads = 256;  // block size for rows of > 128 16-byte chunks; 128 threads for narrower rows
+                                   // (360p: twice the resident CTAs per SM for small per-CTA byte counts)
 constexpr int kBulkMaxStage = 160 * 1024;  // larger rows (e.g. 4K) take the register-streaming kernel
 
 template <bool kD100>
@@ -383,7 +384,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   for (int k = 0; k < 2; ++k) {
 #pragma unroll
     for (int j = 0; j < 8; ++j) acc[k][j] = 0u;
-    const int c = threadIdx.x + k * kBulkThreads;
+    const int c = threadIdx.x + k * (int)blockDim.x;
     if (c < nchunk) {
       const uint8_t* p = smem + 16 * c;
       int y = 0;
@@ -396,7 +397,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   uint16_t* colsum = reinterpret_cast<uint16_t*>(smem);
 #pragma unroll
   for (int k = 0; k < 2; ++k) {
-    const int c = threadIdx.x + k * kBulkThreads;
+    const int c = threadIdx.x + k * (int)blockDim.x;
     if (c < nchunk) store_colsum(reinterpret_cast<uint32_t*>(colsum), c, acc[k]);
   }
   __syncthreads();
@@ -405,7 +406,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   const int row3 = 3 * sdd_w;
   const int cellw = a.xbounds ? a.cellw : (W + sdd_w - 1) / sdd_w;  // widest cell (uniform over the CTA)
   uint32_t ssd_local = 0;
-  for (int o = threadIdx.x; o < row3; o += kBulkThreads) {
+  for (int o = threadIdx.x; o < row3; o += blockDim.x) {
     const int cx = o / 3, ch = o - 3 * cx;
     const int x0 = xb[cx], x1 = xb[cx + 1];
     const uint16_t* col = colsum + ch;
@@ -427,7 +428,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
     asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
     const uint32_t rbase = map_to_rank((uint32_t)__cvta_generic_to_shared(pair_in), 0);
     const uint32_t rbar = map_to_rank(bar_p, 0);
-    for (int o = threadIdx.x; o < half3; o += kBulkThreads) {
+    for (int o = threadIdx.x; o < half3; o += blockDim.x) {
       const int cx = o / 3, ch = o - 3 * cx;
       st_async_u32(rbase + 4u * (uint32_t)o, cell[6 * cx + ch] + cell[6 * cx + 3 + ch], rbar);
     }
@@ -436,7 +437,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
     const int64_t slot = a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f;
     uint8_t* d50row = a.d50 + slot * a.d50_stride + (int64_t)(r >> 1) * half3;
     mbar_wait_parity(bar_p, 0);
-    for (int o = threadIdx.x; o < half3; o += kBulkThreads) {
+    for (int o = threadIdx.x; o < half3; o += blockDim.x) {
       const int cx = o / 3, ch = o - 3 * cx;
       const uint32_t s = cell[6 * cx + ch] + cell[6 * cx + 3 + ch] + pair_in[o];
       const uint32_t n = (uint32_t)(xb[2 * cx + 2] - xb[2 * cx]) * (uint32_t)(yb - y0);
@@ -611,8 +612,9 @@ cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st) {
       else b.d50 += (int64_t)f0 * a.d50_stride;
       if (b.d100) b.d100 += (int64_t)f0 * a.sdd_w * a.sdd_h * 3;
       const dim3 grid((unsigned)a.sdd_h, (unsigned)cnt);
-      if (b.d100) sdd_bulk_kernel<true><<<grid, kBulkThreads, smem, st>>>(b);
-      else sdd_bulk_kernel<false><<<grid, kBulkThreads, smem, st>>>(b);
+      const int nt = a.max_chunks <= kBulkThreads / 2 ? kBulkThreads / 2 : kBulkThreads;
+      if (b.d100) sdd_bulk_kernel<true><<<grid, nt, smem, st>>>(b);
+      else sdd_bulk_kernel<false><<<grid, nt, smem, st>>>(b);
     }
     return cudaGetLastError();
   }
