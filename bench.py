@@ -419,7 +419,7 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
     for tok in args.online.split(","):
         tok = tok.strip()
         if tok == "auto":  # a ladder of fractions of the offline capacity, climbed until a count is not sustained
-            ladder = [max(31, int(f * value / 30)) for f in (0.55, 0.65, 0.75, 0.85)]
+            ladder = [max(31, int(f * value / 30)) for f in (0.55, 0.7, 0.85, 0.95)]
         elif tok:
             counts.append(int(tok))
     nc = len(sids)
@@ -431,24 +431,26 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
         refs.append(r)
     # full three-filter cascade (f1: SDD -> SNM -> T-YOLO, random-init T-YOLO weights) at these stream counts
     ty_counts = []
+    ty_ladder = []
     for tok in args.online_tyolo.split(","):
         tok = tok.strip()
-        if tok == "auto":  # the tick runs SDD, SNM and T-YOLO cycles serially; T-YOLO (~47 K frames/s) gets ~3 % of
-            ty_counts.append(max(31, int(0.1 * value / 30)))  # the frames at TOR 10 %
+        if tok == "auto":  # T-YOLO (~55 K frames/s) sees the SNM survivors, a few % of the frames at TOR 10 %:
+            ty_ladder = [max(31, int(f * value / 30)) for f in (0.1, 0.2, 0.3, 0.4)]  # climbed like the SDD+SNM one
         elif tok:
             ty_counts.append(int(tok))
     results = []
     opened = []
-    runs = [(S, False) for S in counts] + [(S, False) for S in ladder] + [(S, True) for S in ty_counts]
+    runs = ([(S, False) for S in counts] + [(S, False) for S in ladder] + [(S, True) for S in ty_counts] +
+            [(S, True) for S in ty_ladder])
     ty = None
-    if ty_counts:
+    if ty_counts or ty_ladder:
         import paper_conf_icpp_zhangcjzly18_b200 as ff
         ty = ff.Tyolo(ctx, synth.tyolo_weights(video.seed))
     ty_warm = False
-    ladder_failed = False
+    ladder_failed = ty_ladder_failed = False
     for S, with_ty in runs:
-        if S in ladder and not with_ty and ladder_failed:
-            continue  # the ladder stops at its first count that is not sustained
+        if (S in ladder and not with_ty and ladder_failed) or (S in ty_ladder and with_ty and ty_ladder_failed):
+            continue  # a ladder stops at its first count that is not sustained
         t_setup = time.perf_counter()
         while len(opened) < S:
             i = len(opened)
@@ -468,9 +470,12 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
         results.append(res)
         if S in ladder and not with_ty and not res["sustained"]:
             ladder_failed = True
+        if S in ty_ladder and with_ty and not res["sustained"]:
+            ty_ladder_failed = True
+    closed = set(id(st) for st in opened)
     for st in opened:
         st.close()
-        ctx.streams.remove(st)
+    ctx.streams = [st for st in ctx.streams if id(st) not in closed]  # (list.remove per stream is O(S^2))
     if ty is not None:
         ty.destroy()
     best = max([r["streams"] for r in results if r["sustained"] and "stages" not in r], default=0)
@@ -593,12 +598,12 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--online", default="30,auto",
                     help="comma-separated stream counts for the paced online validation (config m2); 'auto' = "
-                         "a ladder of 55/65/75/85%% of the measured frames/s / 30, climbed until a count is not "
+                         "a ladder of 55/70/85/95%% of the measured frames/s / 30, climbed until a count is not "
                          "sustained; empty to skip")
     ap.add_argument("--online-seconds", type=float, default=4.0)
     ap.add_argument("--online-tyolo", default="2000,auto",
                     help="stream counts for a paced run of the full cascade with the T-YOLO stage (f1); 'auto' = "
-                         "10%% of the measured frames/s / 30; empty to skip")
+                         "a ladder of 10/20/30/40%% of the measured frames/s / 30; empty to skip")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")

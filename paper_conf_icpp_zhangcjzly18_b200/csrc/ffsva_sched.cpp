@@ -66,7 +66,9 @@ struct ffsva_sched {
   unsigned long long* d_acc = nullptr;
   uint8_t* d_out = nullptr;   // ssd u64[cap] | logit f32[cap] | pass u8[cap] | snm_pass u8[cap] | snm_class u8[cap]
   uint8_t* h_out = nullptr;
-  std::deque<ffsva_event> pending;
+  // events not yet returned: pending[pend_head ..) (a vector with a consumed prefix, reset when drained)
+  std::vector<ffsva_event> pending;
+  size_t pend_head = 0;
   std::vector<sched::QFrame> adm;   // this cycle's SDD admissions, reused
   std::vector<sched::QFrame> flat;  // this cycle's SNM pops, reused
   std::vector<int32_t> starts;
@@ -445,6 +447,10 @@ FFSVA_API ffsva_status ffsva_sched_push(ffsva_sched* s, const ffsva_frame* frame
   for (int32_t i = 0; i < n; ++i) {  // validate everything before queueing anything
     ffsva_stream* st = frames[i].stream;
     if (!st || !frames[i].pixels) return fail(FFSVA_EINVAL, "frame without stream or pixels");
+    // an attached stream passed every check below when it attached (its descriptor is immutable, and a reference
+    // or SNM, once loaded, stays): consecutive frames of one stream are checked once
+    if (i > 0 && st == frames[i - 1].stream) continue;
+    if (st->ctx == s->ctx && s->lookup(st) >= 0) continue;
     if (st->ctx != s->ctx) return fail(FFSVA_EDEVICE, "stream lives on another device");
     if (!st->has_ref || !st->has_snm) return fail(FFSVA_ESTATE, "stream has no reference image or no SNM");
     if (st->desc.snm_w != snm::IN || st->desc.snm_h != snm::IN) return fail(FFSVA_EINVAL, "SNM grid must be 50x50");
@@ -510,8 +516,8 @@ FFSVA_API ffsva_status ffsva_sched_detach(ffsva_sched* s, ffsva_stream* st) {
   if (id < 0) return FFSVA_OK;
   const sched::StreamQ& q = s->pol.stream(id);
   if (!q.sdd.empty() || !q.snm.empty() || !q.ty.empty()) return fail(FFSVA_EAGAIN, "stream still has queued frames");
-  for (const ffsva_event& e : s->pending)
-    if (e.stream == st) return fail(FFSVA_EAGAIN, "stream still has unreported events");
+  for (size_t i = s->pend_head; i < s->pending.size(); ++i)
+    if (s->pending[i].stream == st) return fail(FFSVA_EAGAIN, "stream still has unreported events");
   if (s->inflight) {
     for (const sched::QFrame& q : s->f_adm)
       if (q.stream == id) return fail(FFSVA_EAGAIN, "stream has frames in flight");
@@ -626,9 +632,15 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
 
   ti.sdd_blocked = (int32_t)(s->pol.total_sdd_blocked() - blocked0);
   int32_t k = 0;
-  while (k < cap && !s->pending.empty()) {
-    events[k++] = s->pending.front();
-    s->pending.pop_front();
+  {
+    const size_t avail = s->pending.size() - s->pend_head;
+    k = (int32_t)std::min<size_t>((size_t)cap, avail);
+    if (k > 0) std::memcpy(events, s->pending.data() + s->pend_head, sizeof(ffsva_event) * (size_t)k);
+    s->pend_head += (size_t)k;
+    if (s->pend_head == s->pending.size()) {
+      s->pending.clear();
+      s->pend_head = 0;
+    }
   }
   *n_events = k;
   ti.sdd_queued = s->pol.queued_sdd();
@@ -637,7 +649,7 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
   ti.snm_blocked = (int32_t)(s->pol.total_snm_blocked() - snm_blocked0);
   ti.tyolo_ms = std::chrono::duration<float, std::milli>(t_ty1 - t_ty0).count();
   // in-flight frames count as pending events (they will be reported by a later tick)
-  ti.events_pending = (int64_t)s->pending.size() + (s->inflight ? (int64_t)(s->f_adm.size() + s->f_flat.size()) : 0);
+  ti.events_pending = (int64_t)(s->pending.size() - s->pend_head) + (s->inflight ? (int64_t)(s->f_adm.size() + s->f_flat.size()) : 0);
   const auto t_end = std::chrono::steady_clock::now();
   ti.sdd_ms = std::chrono::duration<float, std::milli>(t_snm0 - t_tick0).count();
   ti.snm_ms = std::chrono::duration<float, std::milli>(t_ty0 - t_snm0).count();

@@ -91,8 +91,10 @@ class Policy {
  public:
   int32_t add_stream(int32_t q_sdd, int32_t q_snm, int32_t batch, int32_t q_ty = 2) {
     int32_t id = -1;
-    for (int32_t i = 0; i < (int32_t)st_.size(); ++i)
-      if (!st_[i].live) { id = i; break; }
+    if (!free_ids_.empty()) {  // reuse a removed stream's id (O(1): attaching S streams is O(S), not O(S^2))
+      id = free_ids_.back();
+      free_ids_.pop_back();
+    }
     if (id < 0) {
       id = (int32_t)st_.size();
       st_.emplace_back();
@@ -122,6 +124,7 @@ class Policy {
     nq_snm_ -= (int64_t)s.snm.size();
     nq_ty_ -= (int64_t)s.ty.size();
     nsdd_[id] = nsnm_[id] = nty_[id] = 0;
+    if (s.live) free_ids_.push_back(id);
     s = StreamQ();
     return out;
   }
@@ -289,7 +292,8 @@ class Policy {
 
  private:
   std::vector<StreamQ> st_;
-  std::vector<int32_t> nsdd_, nsnm_, nty_;  // per-stream queue depths (compact mirror of the deques)
+  std::vector<int32_t> nsdd_, nsnm_, nty_;  // per-stream queue depths (compact mirror of the FIFOs)
+  std::vector<int32_t> free_ids_;           // ids of removed streams, reused by add_stream
   int64_t nq_sdd_ = 0, nq_snm_ = 0, nq_ty_ = 0;
   uint64_t tot_sdd_blocked_ = 0, tot_snm_blocked_ = 0;
   int32_t rr_ = 0;
