@@ -187,6 +187,15 @@ struct TyConvArgs {
   int32_t* counts;
 };
 cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st);
+// Layer 1 by patch views (ffsva_tyolo.cu): zero-bordered resize output [N][418][418][4] -> [N][208][208][16].
+struct TyL1Args {
+  const __nv_bfloat16* in;
+  __nv_bfloat16* out;
+  const uint8_t* w;          // 4 patch rows x [2 K-halves][64 n = 16q + oc][8 k = 4u + c] bf16 (8 KB)
+  const float* bias;         // [16]
+  int32_t N;
+};
+cudaError_t launch_tyolo_l1(const TyL1Args& a, int num_sms, cudaStream_t st);
 cudaError_t launch_tyolo_pool_s1(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C,
                                  cudaStream_t st);
 cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int32_t max_row_bytes, int32_t max_H,

@@ -464,7 +464,8 @@ __global__ void __launch_bounds__(kResizeThreads) tyolo_resize_kernel(const TyFr
     const int y0 = (int)(((uint32_t)oy * (uint32_t)fr.H) / (uint32_t)D);
     const int yh = (int)(((uint32_t)(oy + 1) * (uint32_t)fr.H) / (uint32_t)D);
     const int y1 = yh > y0 ? yh : y0 + 1;
-    __nv_bfloat16* orow = out + ((int64_t)f * D + oy) * D * 4;
+    // zero-bordered output [N][D+2][D+2][4] (layer 1 reads it by bulk copies; the border stays zero)
+    __nv_bfloat16* orow = out + (((int64_t)f * (D + 2) + oy + 1) * (D + 2) + 1) * 4;
     for (int ox = threadIdx.x; ox < D; ox += kResizeThreads) {
       const int2 xc = xcell[ox];
       uint32_t s0 = 0, s1 = 0, s2 = 0;
@@ -485,6 +486,139 @@ __global__ void __launch_bounds__(kResizeThreads) tyolo_resize_kernel(const TyFr
   }
 }
 
+// ---------------------------------------------------------------- layer 1 (3 -> 16, 3x3, 2x2/2 pool) by patch views
+// The first layer has 3 input channels: the generic kernel's per-row gathers (16 eight-byte pieces per pooled pixel)
+// bound it. Here its input is the zero-bordered resize output [N][418][418][4] bf16 (8 bytes per pixel), so a tile =
+// 128 consecutive pooled pixels of one pooled row needs four contiguous 2,064-byte input row segments (padded rows
+// 2oy .. 2oy+3 from column 2ox0), one bulk copy each, and NO im2col: the A row of pooled pixel ox is its 4x4 patch
+// x 4 channel slots, and patch row dy of consecutive pooled pixels is a constant-stride view of segment dy (rows 16 B
+// apart: two pixels per pooled step; K-halves 16 B apart; 8-row groups 128 B apart). One A operand feeds N = 64 =
+// 4 pool positions x 16 channels with per-position zero-padded 3x3 weights: 4 MMAs (M128 N64 K16) per tile.
+// Persistent, warp-specialised: warp 4 lane 0 copies segments through an S-stage ring, warp 5 issues the MMAs into
+// four TMEM accumulator buffers, warps 0-3 max-pool / bias / leaky / bf16 and store 32 B per pooled pixel.
+constexpr int kL1Pad = 418, kL1Out = 208;
+constexpr int kL1Seg = 258 * 8;                 // 2064 B: input columns 2ox0 .. 2ox0 + 257 of one padded row
+constexpr int kL1Stage = 4 * kL1Seg;            // 8256 B
+constexpr int kL1Stages = 8;
+constexpr int kL1Bufs = 4;                      // TMEM accumulators of 64 columns
+constexpr int kL1Threads = 192;
+constexpr int kL1WBytes = 4 * 2 * 64 * 16;      // 8192 B of packed weights
+constexpr int kL1Smem = kL1WBytes + kL1Stages * kL1Stage + 8 * (2 * kL1Stages + 2 * kL1Bufs + 1) + 16;
+
+__global__ void __launch_bounds__(kL1Threads, 2) tyolo_l1_kernel(TyL1Args a) {
+  extern __shared__ __align__(1024) uint8_t sm[];
+  uint8_t* Ws = sm;
+  uint8_t* Ss = sm + kL1WBytes;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(Ss + kL1Stages * kL1Stage);
+  uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 2 * kL1Stages + 2 * kL1Bufs + 1);
+  const uint32_t full0 = smem_addr(bars), empty0 = full0 + 8 * kL1Stages;
+  const uint32_t accf0 = empty0 + 8 * kL1Stages, acce0 = accf0 + 8 * kL1Bufs, wbar = acce0 + 8 * kL1Bufs;
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);
+  const int tiles = a.N * kL1Out * 2;  // (frame, pooled row, half of the row)
+
+  if (tid == 0) {
+    for (int s = 0; s < kL1Stages; ++s) {
+      mbar_init(full0 + 8 * s, 1);
+      mbar_init(empty0 + 8 * s, 1);
+    }
+    for (int b = 0; b < kL1Bufs; ++b) {
+      mbar_init(accf0 + 8 * b, 1);
+      mbar_init(acce0 + 8 * b, 128);
+    }
+    mbar_init(wbar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    mbar_expect_tx(wbar, kL1WBytes);
+    bulk_g2s(smem_addr(Ws), a.w, kL1WBytes, wbar);
+  }
+  if (warp == 5) tmem_alloc(smem_addr(s_tmem), kL1Bufs * 64);
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *s_tmem;
+
+  if (warp == 4) {
+    // ---------------- producer: four row segments per tile
+    if (lane == 0) {
+      int g = 0;
+      for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++g) {
+        const int n = t / (2 * kL1Out), rem = t - n * 2 * kL1Out, oy = rem >> 1, half = rem & 1;
+        const int s = g % kL1Stages;
+        const uint32_t bytes = half ? (uint32_t)(kL1Pad - 2 * 128) * 8 : (uint32_t)kL1Seg;
+        mbar_wait(empty0 + 8 * s, ((g / kL1Stages) & 1) ^ 1);
+        mbar_expect_tx(full0 + 8 * s, 4 * bytes);
+        const char* src = reinterpret_cast<const char*>(a.in) + (((int64_t)n * kL1Pad + 2 * oy) * kL1Pad + 256 * half) * 8;
+        for (int dy = 0; dy < 4; ++dy)
+          bulk_g2s(smem_addr(Ss + s * kL1Stage + dy * kL1Seg), src + (int64_t)dy * kL1Pad * 8, bytes, full0 + 8 * s);
+      }
+    }
+  } else if (warp == 5) {
+    // ---------------- MMA issue (whole warp, one elected lane)
+    mbar_wait(wbar, 0);
+    const uint32_t idesc = idesc_bf16(128, 64);
+    const uint64_t a_base = umma_desc(smem_addr(Ss), 16, 128), b_base = umma_desc(smem_addr(Ws), 64 * 16, 128);
+    int g = 0;
+    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++g) {
+      const int s = g % kL1Stages, b = g % kL1Bufs;
+      mbar_wait(acce0 + 8 * b, ((g / kL1Bufs) & 1) ^ 1);
+      mbar_wait(full0 + 8 * s, (g / kL1Stages) & 1);
+      fence_after();
+#pragma unroll
+      for (int dy = 0; dy < 4; ++dy)
+        mma_bf16(tmem + (uint32_t)(b * 64), a_base + (uint64_t)((s * kL1Stage + dy * kL1Seg) >> 4),
+                 b_base + (uint64_t)((dy * 2 * 64 * 16) >> 4), idesc, dy > 0 ? 1u : 0u);
+      mma_commit(empty0 + 8 * s);
+      mma_commit(accf0 + 8 * b);
+    }
+  } else {
+    // ---------------- epilogue (warps 0-3): TMEM lane = pooled pixel of the tile
+    const int qd = warp & 3, r = 32 * qd + lane;
+    float bias[16];
+#pragma unroll
+    for (int k = 0; k < 16; ++k) bias[k] = __ldg(a.bias + k);
+    int g = 0;
+    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++g) {
+      const int n = t / (2 * kL1Out), rem = t - n * 2 * kL1Out, oy = rem >> 1, half = rem & 1;
+      const int b = g % kL1Bufs;
+      mbar_wait(accf0 + 8 * b, (g / kL1Bufs) & 1);
+      fence_after();
+      uint32_t r0[16], r1[16], r2[16], r3[16];
+      const uint32_t trow = tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(b * 64);
+      tmem_ld16(trow, r0);
+      tmem_ld16(trow + 16, r1);
+      tmem_ld16(trow + 32, r2);
+      tmem_ld16(trow + 48, r3);
+      tmem_wait_ld2(r0, r1);
+      reg_fence2(r2, r3);
+      fence_before();
+      mbar_arrive(acce0 + 8 * b);  // the accumulator is in registers: the next tile may overwrite it
+      const int ox = 128 * half + r;
+      if (ox < kL1Out) {
+        uint32_t w[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          float x0 = fmaxf(fmaxf(__uint_as_float(r0[2 * k]), __uint_as_float(r1[2 * k])),
+                           fmaxf(__uint_as_float(r2[2 * k]), __uint_as_float(r3[2 * k]))) + bias[2 * k];
+          float x1 = fmaxf(fmaxf(__uint_as_float(r0[2 * k + 1]), __uint_as_float(r1[2 * k + 1])),
+                           fmaxf(__uint_as_float(r2[2 * k + 1]), __uint_as_float(r3[2 * k + 1]))) + bias[2 * k + 1];
+          x0 = x0 < 0.f ? 0.1f * x0 : x0;
+          x1 = x1 < 0.f ? 0.1f * x1 : x1;
+          w[k] = pack_bf16(x0, x1);
+        }
+        uint4* o = reinterpret_cast<uint4*>(a.out + (((int64_t)n * kL1Out + oy) * kL1Out + ox) * 16);
+        o[0] = make_uint4(w[0], w[1], w[2], w[3]);
+        o[1] = make_uint4(w[4], w[5], w[6], w[7]);
+      }
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == 5) {
+    fence_after();
+    tmem_dealloc(tmem, kL1Bufs * 64);
+  }
+}
+
 }  // namespace
 
 int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT) {
@@ -493,6 +627,10 @@ int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT) {
 
 cudaError_t tyolo_configure() {
   const int smem = 227 * 1024;
+  {
+    cudaError_t e = cudaFuncSetAttribute(tyolo_l1_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kL1Smem);
+    if (e != cudaSuccess) return e;
+  }
   cudaError_t e = cudaFuncSetAttribute(tyolo_conv_kernel<1, 4, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(tyolo_conv_kernel<1, 4, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -515,6 +653,13 @@ cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st) {
   else if (a.nq == 4) tyolo_conv_kernel<1, 4, false><<<grid, kConvThreads, smem, st>>>(a);
   else if (a.msub == 2) tyolo_conv_kernel<2, 1, false><<<grid, kConvThreads, smem, st>>>(a);
   else tyolo_conv_kernel<1, 1, false><<<grid, kConvThreads, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tyolo_l1(const TyL1Args& a, int num_sms, cudaStream_t st) {
+  const int tiles = a.N * kL1Out * 2;
+  const int grid = tiles < 2 * num_sms ? tiles : 2 * num_sms;
+  tyolo_l1_kernel<<<grid, kL1Threads, kL1Smem, st>>>(a);
   return cudaGetLastError();
 }
 

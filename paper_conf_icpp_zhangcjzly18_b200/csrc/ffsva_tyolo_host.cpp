@@ -52,6 +52,8 @@ struct ffsva_tyolo {
   // workspace for up to `cap` frames per chunk
   int cap = 0;
   __nv_bfloat16* d_act[2] = {nullptr, nullptr};
+  __nv_bfloat16* d_pad = nullptr;  // zero-bordered resize output [cap][418][418][4] (layer 1's input)
+  uint8_t* d_w1v = nullptr;        // layer 1 weights for the patch-view kernel (8 KB)
   float* d_raw = nullptr;
   int32_t* d_counts = nullptr;
   TyFrame* d_frames = nullptr;
@@ -153,6 +155,7 @@ ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
   const int cap = std::min(kMaxChunk, std::max(n, 16));
   cudaFree(m->d_act[0]);
   cudaFree(m->d_act[1]);
+  cudaFree(m->d_pad);
   cudaFree(m->d_raw);
   cudaFree(m->d_counts);
   cudaFree(m->d_frames);
@@ -162,8 +165,11 @@ ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
   size_t act = 0;  // largest activation per frame (bytes)
   act = std::max(act, (size_t)kIn * kIn * 4 * 2);
   for (int l = 0; l < 8; ++l) act = std::max(act, (size_t)m->L[l].Ho * m->L[l].Ho * m->L[l].Cout_pad * 2);
+  const size_t pad_bytes = (size_t)cap * (kIn + 2) * (kIn + 2) * 4 * 2;
   cudaError_t e = cudaMalloc(&m->d_act[0], act * cap);
   if (e == cudaSuccess) e = cudaMalloc(&m->d_act[1], act * cap);
+  if (e == cudaSuccess) e = cudaMalloc(&m->d_pad, pad_bytes);
+  if (e == cudaSuccess) e = cudaMemset(m->d_pad, 0, pad_bytes);  // the border is written once, here
   if (e == cudaSuccess) e = cudaMalloc(&m->d_raw, (size_t)cap * kGrid * kGrid * kHeadPad * 4);
   if (e == cudaSuccess) e = cudaMalloc(&m->d_counts, (size_t)cap * 4);
   if (e == cudaSuccess) e = cudaMalloc(&m->d_frames, (size_t)cap * sizeof(TyFrame));
@@ -229,12 +235,19 @@ ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, const int32_t*
   if (e == cudaSuccess) e = cudaMemsetAsync(m->d_counts, 0, 4 * (size_t)n, st);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO staging");
   if (ev) cudaEventRecord(ev[0], st);
-  if ((e = launch_tyolo_resize(m->d_frames, n, kIn, max_row, max_H, m->d_act[0], st)) != cudaSuccess)
+  if ((e = launch_tyolo_resize(m->d_frames, n, kIn, max_row, max_H, m->d_pad, st)) != cudaSuccess)
     return cuda_fail(ctx, e, "T-YOLO resize");
   g_launches += 1;
   if (ev) cudaEventRecord(ev[1], st);
-  int cur = 0;
-  for (int l = 0; l <= upto; ++l) {
+  int cur = -1;  // -1: the padded resize output
+  if (upto >= 0) {  // layer 1 by patch views of the padded input
+    const TyL1Args a1{m->d_pad, m->d_act[0], m->d_w1v, m->d_b + m->L[0].b_off, n};
+    if ((e = launch_tyolo_l1(a1, ctx->num_sms, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO layer 1");
+    g_launches += 1;
+    cur = 0;
+    if (ev) cudaEventRecord(ev[2], st);
+  }
+  for (int l = 1; l <= upto; ++l) {
     const TyConvArgs a = layer_args(m, l, n, m->d_act[cur], m->d_act[cur ^ 1], thresh);
     if ((e = launch_tyolo_conv(a, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO conv layer");
     g_launches += 1;
@@ -296,16 +309,32 @@ FFSVA_API ffsva_status ffsva_tyolo_load(int32_t device, const float* params, int
     std::memcpy(hb.data() + L.b_off, p + nw, sizeof(float) * L.Cout);
     p += nw + L.Cout;
   }
+  // layer 1 for the patch-view kernel: B of patch row dy = [K-half h][n = 16q + oc][k = 4(u & 1) + c], u = 2h + (k >> 2)
+  // the patch column; pool position q = (qa, qb) puts the 3x3 kernel at patch offset (qa, qb)
+  std::vector<uint16_t> w1v(4 * 2 * 64 * 8, 0);
+  for (int dy = 0; dy < 4; ++dy)
+    for (int q = 0; q < 4; ++q)
+      for (int oc = 0; oc < 16; ++oc)
+        for (int u = 0; u < 4; ++u)
+          for (int c = 0; c < 3; ++c) {
+            const int ky = dy - (q >> 1), kx = u - (q & 1);
+            if (ky < 0 || ky > 2 || kx < 0 || kx > 2) continue;
+            w1v[((dy * 2 + (u >> 1)) * 64 + 16 * q + oc) * 8 + 4 * (u & 1) + c] =
+                bf16_bits(params[((oc * 3 + c) * 3 + ky) * 3 + kx]);
+          }
   {
     std::lock_guard<std::mutex> lk(ctx->mu);
     DeviceGuard g(device);
     cudaError_t e = cudaMalloc(&m->d_w, wbytes);
+    if (e == cudaSuccess) e = cudaMalloc(&m->d_w1v, w1v.size() * 2);
+    if (e == cudaSuccess) e = cudaMemcpy(m->d_w1v, w1v.data(), w1v.size() * 2, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMalloc(&m->d_b, nb * 4);
     if (e == cudaSuccess) e = cudaMemcpy(m->d_w, hw.data(), wbytes, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMemcpy(m->d_b, hb.data(), nb * 4, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = tyolo_configure();
     if (e != cudaSuccess) {
       cudaFree(m->d_w);
+      cudaFree(m->d_w1v);
       cudaFree(m->d_b);
       ctx_release(ctx);
       return cuda_fail(nullptr, e, "ffsva_tyolo_load");
@@ -375,9 +404,17 @@ FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_fram
   cudaStream_t cs = (cudaStream_t)cuda_stream;
   int buf = 0;
   if ((st = run_chunk(m, frames, nullptr, n, layer, 0.2f, cs, nullptr, &buf)) != FFSVA_OK) return st;
-  const size_t bytes = layer < 0 ? (size_t)n * kIn * kIn * 4 * 2
-                                 : (size_t)n * m->L[layer].Ho * m->L[layer].Ho * m->L[layer].Cout_pad * 2;
-  cudaError_t e = cudaMemcpyAsync(out, m->d_act[buf], bytes, cudaMemcpyDeviceToHost, cs);
+  cudaError_t e = cudaSuccess;
+  if (buf < 0) {  // the resized input: the interior of the zero-bordered buffer
+    const size_t row = (size_t)kIn * 4 * 2, prow = (size_t)(kIn + 2) * 4 * 2;
+    for (int i = 0; i < n && e == cudaSuccess; ++i)
+      e = cudaMemcpy2DAsync(out + (size_t)i * kIn * kIn * 4, row,
+                            reinterpret_cast<const uint8_t*>(m->d_pad) + ((size_t)i * (kIn + 2) + 1) * prow + 4 * 2,
+                            prow, row, kIn, cudaMemcpyDeviceToHost, cs);
+  } else {
+    const size_t bytes = (size_t)n * m->L[layer].Ho * m->L[layer].Ho * m->L[layer].Cout_pad * 2;
+    e = cudaMemcpyAsync(out, m->d_act[buf], bytes, cudaMemcpyDeviceToHost, cs);
+  }
   if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
   if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_tyolo_layer_output");
   return FFSVA_OK;
@@ -428,6 +465,8 @@ FFSVA_API ffsva_status ffsva_tyolo_destroy(ffsva_tyolo* m) {
     cudaFree(m->d_b);
     cudaFree(m->d_act[0]);
     cudaFree(m->d_act[1]);
+    cudaFree(m->d_pad);
+    cudaFree(m->d_w1v);
     cudaFree(m->d_raw);
     cudaFree(m->d_counts);
     cudaFree(m->d_frames);
