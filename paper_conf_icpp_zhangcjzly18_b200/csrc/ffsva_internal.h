@@ -196,6 +196,10 @@ struct TyL1Args {
   int32_t N;
 };
 cudaError_t launch_tyolo_l1(const TyL1Args& a, int num_sms, cudaStream_t st);
+// Layer 2 by patch views: layer 1's planar zero-bordered output [N][210][2][2][105][8 ch] -> [N][104][104][32].
+// w: 16 (patch row, column) x [2 channel groups][128 n = 32q + oc][8 k] bf16 (64 KB).
+cudaError_t launch_tyolo_l2(const TyL1Args& a, int num_sms, cudaStream_t st);
+constexpr size_t kTyL2PadBytes = (size_t)210 * 4 * 105 * 16;  // per frame
 cudaError_t launch_tyolo_pool_s1(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C,
                                  cudaStream_t st);
 cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int32_t max_row_bytes, int32_t max_H,

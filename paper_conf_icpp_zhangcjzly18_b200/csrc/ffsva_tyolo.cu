@@ -497,6 +497,11 @@ __global__ void __launch_bounds__(kResizeThreads) tyolo_resize_kernel(const TyFr
 // Persistent, warp-specialised: warp 4 lane 0 copies segments through an S-stage ring, warp 5 issues the MMAs into
 // four TMEM accumulator buffers, warps 0-3 max-pool / bias / leaky / bf16 and store 32 B per pooled pixel.
 constexpr int kL1Pad = 418, kL1Out = 208;
+// layer 2's planar, zero-bordered input (= layer 1's output): [N][210 rows][2 column parities][2 channel groups]
+// [105 entries][16 B]
+constexpr int kL2Pad = 210, kL2Out = 104, kL2Entries = 105;
+constexpr int kL2Plane = kL2Entries * 16;       // 1680 B
+constexpr int kL2Row = 4 * kL2Plane;            // 6720 B
 constexpr int kL1Seg = 258 * 8;                 // 2064 B: input columns 2ox0 .. 2ox0 + 257 of one padded row
 constexpr int kL1Stage = 4 * kL1Seg;            // 8256 B
 constexpr int kL1Stages = 8;
@@ -605,9 +610,12 @@ __global__ void __launch_bounds__(kL1Threads, 2) tyolo_l1_kernel(TyL1Args a) {
           x1 = x1 < 0.f ? 0.1f * x1 : x1;
           w[k] = pack_bf16(x0, x1);
         }
-        uint4* o = reinterpret_cast<uint4*>(a.out + (((int64_t)n * kL1Out + oy) * kL1Out + ox) * 16);
-        o[0] = make_uint4(w[0], w[1], w[2], w[3]);
-        o[1] = make_uint4(w[4], w[5], w[6], w[7]);
+        // layer 2's planar input: padded pixel (Y, X) = (oy + 1, ox + 1), channel group g at plane (X & 1, g)
+        const int X = ox + 1;
+        uint8_t* o = reinterpret_cast<uint8_t*>(a.out) + ((int64_t)n * kL2Pad + oy + 1) * kL2Row +
+                     (X & 1) * 2 * kL2Plane + (X >> 1) * 16;
+        *reinterpret_cast<uint4*>(o) = make_uint4(w[0], w[1], w[2], w[3]);
+        *reinterpret_cast<uint4*>(o + kL2Plane) = make_uint4(w[4], w[5], w[6], w[7]);
       }
     }
   }
@@ -616,6 +624,136 @@ __global__ void __launch_bounds__(kL1Threads, 2) tyolo_l1_kernel(TyL1Args a) {
   if (warp == 5) {
     fence_after();
     tmem_dealloc(tmem, kL1Bufs * 64);
+  }
+}
+
+// ---------------------------------------------------------------- layer 2 (16 -> 32, 3x3, 2x2/2 pool) by patch views
+// Layer 1 writes its output zero-bordered and planar: padded row Y holds four planes (pixel-column parity p, channel
+// group g of 8) of 105 sixteen-byte entries (entry e = padded column 2e + p), so a padded row is one contiguous
+// 6,720-byte segment and, for patch column u, consecutive pooled pixels (columns 2ox + u) are consecutive entries of
+// plane (u & 1, g): a constant-stride view again (rows 16 B apart, the two channel groups one plane apart, 8-row
+// groups 128 B apart). A tile = one pooled row (104 pixels in 128 MMA rows), four segment copies; per patch row dy
+// and column u one MMA of K16 (16 channels) and N = 128 = 4 pool positions x 32 channels: 16 MMAs per tile.
+constexpr int kL2Stages = 5;
+constexpr int kL2Bufs = 4;                      // TMEM accumulators of 128 columns
+constexpr int kL2Threads = 192;
+constexpr int kL2WBytes = 16 * 2 * 128 * 16;    // 65,536 B: [dy][u][channel group][n][8]
+constexpr int kL2Stage = 4 * kL2Row;            // 26,880 B
+constexpr int kL2Smem = kL2WBytes + kL2Stages * kL2Stage + 512 + 8 * (2 * kL2Stages + 2 * kL2Bufs + 1) + 16;
+
+__global__ void __launch_bounds__(kL2Threads, 1) tyolo_l2_kernel(TyL1Args a) {
+  extern __shared__ __align__(1024) uint8_t sm[];
+  uint8_t* Ws = sm;
+  uint8_t* Ss = sm + kL2WBytes;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(Ss + kL2Stages * kL2Stage + 512);  // + tail read by junk rows
+  uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 2 * kL2Stages + 2 * kL2Bufs + 1);
+  const uint32_t full0 = smem_addr(bars), empty0 = full0 + 8 * kL2Stages;
+  const uint32_t accf0 = empty0 + 8 * kL2Stages, acce0 = accf0 + 8 * kL2Bufs, wbar = acce0 + 8 * kL2Bufs;
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);
+  const int tiles = a.N * kL2Out;  // (frame, pooled row)
+
+  if (tid == 0) {
+    for (int s = 0; s < kL2Stages; ++s) {
+      mbar_init(full0 + 8 * s, 1);
+      mbar_init(empty0 + 8 * s, 1);
+    }
+    for (int b = 0; b < kL2Bufs; ++b) {
+      mbar_init(accf0 + 8 * b, 1);
+      mbar_init(acce0 + 8 * b, 128);
+    }
+    mbar_init(wbar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    mbar_expect_tx(wbar, kL2WBytes);
+    bulk_g2s(smem_addr(Ws), a.w, kL2WBytes, wbar);
+  }
+  if (warp == 5) tmem_alloc(smem_addr(s_tmem), kL2Bufs * 128);
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *s_tmem;
+
+  if (warp == 4) {
+    if (lane == 0) {
+      int g = 0;
+      for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++g) {
+        const int n = t / kL2Out, oy = t - n * kL2Out;
+        const int s = g % kL2Stages;
+        mbar_wait(empty0 + 8 * s, ((g / kL2Stages) & 1) ^ 1);
+        mbar_expect_tx(full0 + 8 * s, kL2Stage);
+        // padded rows 2oy .. 2oy + 3 are contiguous: one copy of four segments
+        bulk_g2s(smem_addr(Ss + s * kL2Stage),
+                 reinterpret_cast<const char*>(a.in) + ((int64_t)n * kL2Pad + 2 * oy) * kL2Row, kL2Stage,
+                 full0 + 8 * s);
+      }
+    }
+  } else if (warp == 5) {
+    mbar_wait(wbar, 0);
+    const uint32_t idesc = idesc_bf16(128, 128);
+    const uint64_t a_base = umma_desc(smem_addr(Ss), kL2Plane, 128), b_base = umma_desc(smem_addr(Ws), 128 * 16, 128);
+    int g = 0;
+    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++g) {
+      const int s = g % kL2Stages, b = g % kL2Bufs;
+      mbar_wait(acce0 + 8 * b, ((g / kL2Bufs) & 1) ^ 1);
+      mbar_wait(full0 + 8 * s, (g / kL2Stages) & 1);
+      fence_after();
+#pragma unroll
+      for (int dy = 0; dy < 4; ++dy)
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          mma_bf16(tmem + (uint32_t)(b * 128),
+                   a_base + (uint64_t)((s * kL2Stage + dy * kL2Row + (u & 1) * 2 * kL2Plane + (u >> 1) * 16) >> 4),
+                   b_base + (uint64_t)(((dy * 4 + u) * 2 * 128 * 16) >> 4), idesc, (dy | u) ? 1u : 0u);
+      mma_commit(empty0 + 8 * s);
+      mma_commit(accf0 + 8 * b);
+    }
+  } else {
+    const int qd = warp & 3, r = 32 * qd + lane;
+    int g = 0;
+    for (int t = blockIdx.x; t < tiles; t += gridDim.x, ++g) {
+      const int n = t / kL2Out, oy = t - n * kL2Out;
+      const int b = g % kL2Bufs;
+      mbar_wait(accf0 + 8 * b, (g / kL2Bufs) & 1);
+      fence_after();
+      const uint32_t trow = tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(b * 128);
+      uint32_t w[16];
+#pragma unroll
+      for (int c0 = 0; c0 < 32; c0 += 16) {
+        uint32_t r0[16], r1[16], r2[16], r3[16];
+        tmem_ld16(trow + (uint32_t)c0, r0);
+        tmem_ld16(trow + (uint32_t)(32 + c0), r1);
+        tmem_ld16(trow + (uint32_t)(64 + c0), r2);
+        tmem_ld16(trow + (uint32_t)(96 + c0), r3);
+        tmem_wait_ld2(r0, r1);
+        reg_fence2(r2, r3);
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          float x0 = fmaxf(fmaxf(__uint_as_float(r0[2 * k]), __uint_as_float(r1[2 * k])),
+                           fmaxf(__uint_as_float(r2[2 * k]), __uint_as_float(r3[2 * k]))) + __ldg(a.bias + c0 + 2 * k);
+          float x1 = fmaxf(fmaxf(__uint_as_float(r0[2 * k + 1]), __uint_as_float(r1[2 * k + 1])),
+                           fmaxf(__uint_as_float(r2[2 * k + 1]), __uint_as_float(r3[2 * k + 1]))) +
+                     __ldg(a.bias + c0 + 2 * k + 1);
+          x0 = x0 < 0.f ? 0.1f * x0 : x0;
+          x1 = x1 < 0.f ? 0.1f * x1 : x1;
+          w[c0 / 2 + k] = pack_bf16(x0, x1);
+        }
+      }
+      fence_before();
+      mbar_arrive(acce0 + 8 * b);
+      if (r < kL2Out) {
+        uint4* o = reinterpret_cast<uint4*>(a.out + (((int64_t)n * kL2Out + oy) * kL2Out + r) * 32);
+        o[0] = make_uint4(w[0], w[1], w[2], w[3]);
+        o[1] = make_uint4(w[4], w[5], w[6], w[7]);
+        o[2] = make_uint4(w[8], w[9], w[10], w[11]);
+        o[3] = make_uint4(w[12], w[13], w[14], w[15]);
+      }
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == 5) {
+    fence_after();
+    tmem_dealloc(tmem, kL2Bufs * 128);
   }
 }
 
@@ -629,6 +767,7 @@ cudaError_t tyolo_configure() {
   const int smem = 227 * 1024;
   {
     cudaError_t e = cudaFuncSetAttribute(tyolo_l1_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kL1Smem);
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(tyolo_l2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kL2Smem);
     if (e != cudaSuccess) return e;
   }
   cudaError_t e = cudaFuncSetAttribute(tyolo_conv_kernel<1, 4, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -660,6 +799,13 @@ cudaError_t launch_tyolo_l1(const TyL1Args& a, int num_sms, cudaStream_t st) {
   const int tiles = a.N * kL1Out * 2;
   const int grid = tiles < 2 * num_sms ? tiles : 2 * num_sms;
   tyolo_l1_kernel<<<grid, kL1Threads, kL1Smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tyolo_l2(const TyL1Args& a, int num_sms, cudaStream_t st) {
+  const int tiles = a.N * kL2Out;
+  const int grid = tiles < num_sms ? tiles : num_sms;
+  tyolo_l2_kernel<<<grid, kL2Threads, kL2Smem, st>>>(a);
   return cudaGetLastError();
 }
 

@@ -54,6 +54,8 @@ struct ffsva_tyolo {
   __nv_bfloat16* d_act[2] = {nullptr, nullptr};
   __nv_bfloat16* d_pad = nullptr;  // zero-bordered resize output [cap][418][418][4] (layer 1's input)
   uint8_t* d_w1v = nullptr;        // layer 1 weights for the patch-view kernel (8 KB)
+  __nv_bfloat16* d_pad2 = nullptr; // layer 1's planar zero-bordered output (layer 2's input), kTyL2PadBytes per frame
+  uint8_t* d_w2v = nullptr;        // layer 2 weights for the patch-view kernel (64 KB)
   float* d_raw = nullptr;
   int32_t* d_counts = nullptr;
   TyFrame* d_frames = nullptr;
@@ -156,6 +158,7 @@ ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
   cudaFree(m->d_act[0]);
   cudaFree(m->d_act[1]);
   cudaFree(m->d_pad);
+  cudaFree(m->d_pad2);
   cudaFree(m->d_raw);
   cudaFree(m->d_counts);
   cudaFree(m->d_frames);
@@ -170,6 +173,8 @@ ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
   if (e == cudaSuccess) e = cudaMalloc(&m->d_act[1], act * cap);
   if (e == cudaSuccess) e = cudaMalloc(&m->d_pad, pad_bytes);
   if (e == cudaSuccess) e = cudaMemset(m->d_pad, 0, pad_bytes);  // the border is written once, here
+  if (e == cudaSuccess) e = cudaMalloc(&m->d_pad2, (size_t)cap * kTyL2PadBytes);
+  if (e == cudaSuccess) e = cudaMemset(m->d_pad2, 0, (size_t)cap * kTyL2PadBytes);
   if (e == cudaSuccess) e = cudaMalloc(&m->d_raw, (size_t)cap * kGrid * kGrid * kHeadPad * 4);
   if (e == cudaSuccess) e = cudaMalloc(&m->d_counts, (size_t)cap * 4);
   if (e == cudaSuccess) e = cudaMalloc(&m->d_frames, (size_t)cap * sizeof(TyFrame));
@@ -240,14 +245,21 @@ ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, const int32_t*
   g_launches += 1;
   if (ev) cudaEventRecord(ev[1], st);
   int cur = -1;  // -1: the padded resize output
-  if (upto >= 0) {  // layer 1 by patch views of the padded input
-    const TyL1Args a1{m->d_pad, m->d_act[0], m->d_w1v, m->d_b + m->L[0].b_off, n};
+  if (upto >= 0) {  // layer 1 by patch views of the padded input, into layer 2's planar padded input
+    const TyL1Args a1{m->d_pad, m->d_pad2, m->d_w1v, m->d_b + m->L[0].b_off, n};
     if ((e = launch_tyolo_l1(a1, ctx->num_sms, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO layer 1");
     g_launches += 1;
-    cur = 0;
+    cur = -2;  // -2: the planar layer-1 output
     if (ev) cudaEventRecord(ev[2], st);
   }
-  for (int l = 1; l <= upto; ++l) {
+  if (upto >= 1) {  // layer 2 by patch views
+    const TyL1Args a2{m->d_pad2, m->d_act[0], m->d_w2v, m->d_b + m->L[1].b_off, n};
+    if ((e = launch_tyolo_l2(a2, ctx->num_sms, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO layer 2");
+    g_launches += 1;
+    cur = 0;
+    if (ev) cudaEventRecord(ev[3], st);
+  }
+  for (int l = 2; l <= upto; ++l) {
     const TyConvArgs a = layer_args(m, l, n, m->d_act[cur], m->d_act[cur ^ 1], thresh);
     if ((e = launch_tyolo_conv(a, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO conv layer");
     g_launches += 1;
@@ -322,10 +334,27 @@ FFSVA_API ffsva_status ffsva_tyolo_load(int32_t device, const float* params, int
             w1v[((dy * 2 + (u >> 1)) * 64 + 16 * q + oc) * 8 + 4 * (u & 1) + c] =
                 bf16_bits(params[((oc * 3 + c) * 3 + ky) * 3 + kx]);
           }
+  // layer 2 for the patch-view kernel: B of (patch row dy, column u) = [channel group g][n = 32q + oc][8 channels]
+  std::vector<uint16_t> w2v(16 * 2 * 128 * 8, 0);
+  {
+    const float* w2 = params + 16 * 3 * 9 + 16;  // layer 2 follows layer 1's weights and biases
+    for (int dy = 0; dy < 4; ++dy)
+      for (int u = 0; u < 4; ++u)
+        for (int q = 0; q < 4; ++q) {
+          const int ky = dy - (q >> 1), kx = u - (q & 1);
+          if (ky < 0 || ky > 2 || kx < 0 || kx > 2) continue;
+          for (int oc = 0; oc < 32; ++oc)
+            for (int c = 0; c < 16; ++c)
+              w2v[(((dy * 4 + u) * 2 + (c >> 3)) * 128 + 32 * q + oc) * 8 + (c & 7)] =
+                  bf16_bits(w2[((oc * 16 + c) * 3 + ky) * 3 + kx]);
+        }
+  }
   {
     std::lock_guard<std::mutex> lk(ctx->mu);
     DeviceGuard g(device);
     cudaError_t e = cudaMalloc(&m->d_w, wbytes);
+    if (e == cudaSuccess) e = cudaMalloc(&m->d_w2v, w2v.size() * 2);
+    if (e == cudaSuccess) e = cudaMemcpy(m->d_w2v, w2v.data(), w2v.size() * 2, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMalloc(&m->d_w1v, w1v.size() * 2);
     if (e == cudaSuccess) e = cudaMemcpy(m->d_w1v, w1v.data(), w1v.size() * 2, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMalloc(&m->d_b, nb * 4);
@@ -335,6 +364,7 @@ FFSVA_API ffsva_status ffsva_tyolo_load(int32_t device, const float* params, int
     if (e != cudaSuccess) {
       cudaFree(m->d_w);
       cudaFree(m->d_w1v);
+      cudaFree(m->d_w2v);
       cudaFree(m->d_b);
       ctx_release(ctx);
       return cuda_fail(nullptr, e, "ffsva_tyolo_load");
@@ -405,7 +435,23 @@ FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_fram
   int buf = 0;
   if ((st = run_chunk(m, frames, nullptr, n, layer, 0.2f, cs, nullptr, &buf)) != FFSVA_OK) return st;
   cudaError_t e = cudaSuccess;
-  if (buf < 0) {  // the resized input: the interior of the zero-bordered buffer
+  if (buf == -2) {  // layer 1: unpack the planar zero-bordered buffer [n][210][parity][group][105][8] on the host
+    std::vector<uint16_t> pl((size_t)n * kTyL2PadBytes / 2);
+    e = cudaMemcpyAsync(pl.data(), m->d_pad2, pl.size() * 2, cudaMemcpyDeviceToHost, cs);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_tyolo_layer_output");
+    const size_t row = kTyL2PadBytes / 210 / 2, plane = row / 4;  // in bf16 elements
+    for (int i = 0; i < n; ++i)
+      for (int y = 0; y < 208; ++y)
+        for (int x = 0; x < 208; ++x)
+          for (int c = 0; c < 16; ++c) {
+            const int Y = y + 1, X = x + 1;
+            out[(((size_t)i * 208 + y) * 208 + x) * 16 + c] =
+                pl[((size_t)i * 210 + Y) * row + ((X & 1) * 2 + (c >> 3)) * plane + (X >> 1) * 8 + (c & 7)];
+          }
+    return FFSVA_OK;
+  }
+  if (buf == -1) {  // the resized input: the interior of the zero-bordered buffer
     const size_t row = (size_t)kIn * 4 * 2, prow = (size_t)(kIn + 2) * 4 * 2;
     for (int i = 0; i < n && e == cudaSuccess; ++i)
       e = cudaMemcpy2DAsync(out + (size_t)i * kIn * kIn * 4, row,
@@ -467,6 +513,8 @@ FFSVA_API ffsva_status ffsva_tyolo_destroy(ffsva_tyolo* m) {
     cudaFree(m->d_act[1]);
     cudaFree(m->d_pad);
     cudaFree(m->d_w1v);
+    cudaFree(m->d_pad2);
+    cudaFree(m->d_w2v);
     cudaFree(m->d_raw);
     cudaFree(m->d_counts);
     cudaFree(m->d_frames);
