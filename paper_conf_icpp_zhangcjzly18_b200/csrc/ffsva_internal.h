@@ -201,7 +201,21 @@ cudaError_t launch_tyolo_l1(const TyL1Args& a, int num_sms, cudaStream_t st);
 cudaError_t launch_tyolo_l2(const TyL1Args& a, int num_sms, cudaStream_t st);
 constexpr size_t kTyL2PadBytes = (size_t)210 * 4 * 105 * 16;  // per frame
 cudaError_t launch_tyolo_pool_s1(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C,
-                                 cudaStream_t st);
+                                 int64_t planar_stride, cudaStream_t st);
+// 13x13 layers by slab views (ffsva_tyolo.cu tyolo_slab_kernel). Slab layout of C channels: C/8 planes of `plane`
+// 16-byte entries, entry = frame * 225 + Y * 15 + X of the zero-bordered 15x15 grid; plane >= round_up(N * 225,
+// 256) + 64 (reads past the last frame stay inside the plane).
+inline int64_t tyolo_slab_plane(int32_t n) { return (int64_t)((n * 225 + 255) / 256) * 256 + 64; }
+struct TySlabArgs {
+  const __nv_bfloat16* in;   // slab layout, Cin channels
+  int64_t plane;             // entries per input plane
+  __nv_bfloat16* out;        // slab layout (out_plane > 0) or NHWC [N][13][13][Cout]
+  int64_t out_plane;
+  const uint8_t* wpk;        // the generic kernel's packing for this layer (NT = 256, K step = tap * Cin/64 + group)
+  const float* bias;
+  int32_t N, Cin, Cout;      // Cin % 64 == 0, Cout % 256 == 0
+};
+cudaError_t launch_tyolo_slab(const TySlabArgs& a, int num_sms, cudaStream_t st);
 cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int32_t max_row_bytes, int32_t max_H,
                                 __nv_bfloat16* out, cudaStream_t st);
 int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT);

@@ -364,7 +364,10 @@ __global__ void __launch_bounds__(kConvThreads, 1) tyolo_conv_kernel(TyConvArgs 
 // 2x2 max-pool with stride 1 and a -inf right/bottom border (Q30) on bf16 NHWC, 8 channels per thread. Applied
 // after the layer-6 convolution (bf16 rounding is monotone, so pooling the rounded values equals rounding the
 // pooled ones).
-__global__ void tyolo_pool_s1_kernel(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C) {
+// planar_stride > 0: write the 13x13 slab layout instead (plane c/8 at planar_stride entries, entry = frame * 225 +
+// (y + 1) * 15 + x + 1 of the zero-bordered 15x15 grid; see tyolo_slab_kernel)
+__global__ void tyolo_pool_s1_kernel(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C,
+                                     int64_t planar_stride) {
   const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int c8 = C >> 3;
   const int64_t total = (int64_t)n * H * H * c8;
@@ -393,7 +396,12 @@ __global__ void tyolo_pool_s1_kernel(const __nv_bfloat16* in, __nv_bfloat16* out
   o.y = *reinterpret_cast<uint32_t*>(&mx[1]);
   o.z = *reinterpret_cast<uint32_t*>(&mx[2]);
   o.w = *reinterpret_cast<uint32_t*>(&mx[3]);
-  *reinterpret_cast<uint4*>(out + p * C + 8 * cg) = o;
+  if (planar_stride > 0) {
+    const int64_t f = p / ((int64_t)H * H);
+    *reinterpret_cast<uint4*>(out + ((int64_t)cg * planar_stride + f * 225 + (y + 1) * 15 + x + 1) * 8) = o;
+  } else {
+    *reinterpret_cast<uint4*>(out + p * C + 8 * cg) = o;
+  }
 }
 
 // Q28 resize of each raw RGB8 frame to 416x416, x = v / 256 (Q29) as bf16 NHWC with a zero 4th channel. One CTA per
@@ -757,6 +765,171 @@ __global__ void __launch_bounds__(kL2Threads, 1) tyolo_l2_kernel(TyL1Args a) {
   }
 }
 
+// ---------------------------------------------------------------- 13x13 layers (3x3, no pool) by slab views
+// Input: zero-bordered "slab" layout: for every 8-channel group a plane of 16-byte entries, entry p = frame * 225 +
+// Y * 15 + X over the 15x15 padded grid (frames stacked). Output rows of the GEMM are the padded-grid entries p
+// themselves (rows with y or x >= 13 are computed and discarded: 169 of 225 useful), so tap (dy, dx) of consecutive
+// rows is the plane read at p + dy*15 + dx: a constant-stride UMMA view (rows 16 B apart, channel groups one plane
+// apart, 8-row groups 128 B apart). A tile job = 2 x 128 rows x 256 output channels; per 64-channel group one slab
+// of 160 entries x 8 planes per half is bulk-copied (16 copies) and feeds all nine taps, so the A operand costs
+// 40 KB per 9 K steps instead of a 32 KB im2col gather per step; B (the pre-packed weights of the generic kernel,
+// K step = tap * (Cin/64) + group) streams through a 4-stage ring. Warp 4 lane 0 copies, warp 5 issues MMAs,
+// warps 0-3 drain the accumulators (bias, leaky, bf16) into the next slab layout or NHWC.
+constexpr int kSlabEntries = 160;               // 128 rows + the largest tap offset (2 * 15 + 2) rounded up
+constexpr int kSlabPlaneBytes = kSlabEntries * 16;  // 2560
+constexpr int kSlabHalf = 8 * kSlabPlaneBytes;  // 20,480 B: one half's 64-channel slab
+constexpr int kSlabA = 2 * kSlabHalf;           // both halves
+constexpr int kSlabAStages = 2, kSlabBStages = 4;
+constexpr int kSlabBStage = 64 * 256 * 2;       // 32 KB: one K step of weights for a 256-wide N tile
+constexpr int kSlabThreads = 192;
+constexpr int kSlabSmem = kSlabAStages * kSlabA + kSlabBStages * kSlabBStage +
+                          8 * (2 * kSlabAStages + 2 * kSlabBStages + 2) + 16;
+
+__global__ void __launch_bounds__(kSlabThreads, 1) tyolo_slab_kernel(TySlabArgs a) {
+  extern __shared__ __align__(1024) uint8_t sm[];
+  uint8_t* As = sm;
+  uint8_t* Bs = sm + kSlabAStages * kSlabA;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(Bs + kSlabBStages * kSlabBStage);
+  uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 2 * kSlabAStages + 2 * kSlabBStages + 2);
+  const uint32_t fullA0 = smem_addr(bars), emptyA0 = fullA0 + 8 * kSlabAStages;
+  const uint32_t fullB0 = emptyA0 + 8 * kSlabAStages, emptyB0 = fullB0 + 8 * kSlabBStages;
+  const uint32_t accf = emptyB0 + 8 * kSlabBStages, acce = accf + 8;
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);
+  const int G = a.Cin >> 6;                       // 64-channel groups
+  const int n_nt = a.Cout >> 8;                   // 256-wide N tiles
+  const int m_tiles = (a.N * 225 + 255) >> 8;
+  const int jobs = m_tiles * n_nt;
+
+  if (tid == 0) {
+    for (int s = 0; s < kSlabAStages; ++s) {
+      mbar_init(fullA0 + 8 * s, 1);
+      mbar_init(emptyA0 + 8 * s, 1);
+    }
+    for (int s = 0; s < kSlabBStages; ++s) {
+      mbar_init(fullB0 + 8 * s, 1);
+      mbar_init(emptyB0 + 8 * s, 1);
+    }
+    mbar_init(accf, 1);
+    mbar_init(acce, 128);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 5) tmem_alloc(smem_addr(s_tmem), 512);
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *s_tmem;
+
+  if (warp == 4) {
+    // ---------------- producer: per job, G slabs (16 copies each) interleaved with 9 * G weight stages
+    if (lane == 0) {
+      int ga = 0, gb = 0;
+      for (int j = blockIdx.x; j < jobs; j += gridDim.x) {
+        const int mt = j / n_nt, nt = j - mt * n_nt;
+        const int64_t p0 = (int64_t)mt * 256;
+        for (int g = 0; g < G; ++g, ++ga) {
+          const int sa = ga % kSlabAStages;
+          mbar_wait(emptyA0 + 8 * sa, ((ga / kSlabAStages) & 1) ^ 1);
+          mbar_expect_tx(fullA0 + 8 * sa, kSlabA);
+          for (int h = 0; h < 2; ++h)
+            for (int pl = 0; pl < 8; ++pl)
+              bulk_g2s(smem_addr(As + sa * kSlabA + h * kSlabHalf + pl * kSlabPlaneBytes),
+                       reinterpret_cast<const char*>(a.in) + ((int64_t)(8 * g + pl) * a.plane + p0 + 128 * h) * 16,
+                       kSlabPlaneBytes, fullA0 + 8 * sa);
+          for (int t = 0; t < 9; ++t, ++gb) {
+            const int sb = gb % kSlabBStages;
+            mbar_wait(emptyB0 + 8 * sb, ((gb / kSlabBStages) & 1) ^ 1);
+            mbar_expect_tx(fullB0 + 8 * sb, kSlabBStage);
+            bulk_g2s(smem_addr(Bs + sb * kSlabBStage),
+                     a.wpk + ((int64_t)nt * 9 * G + t * G + g) * kSlabBStage, kSlabBStage, fullB0 + 8 * sb);
+          }
+        }
+      }
+    }
+  } else if (warp == 5) {
+    // ---------------- MMA issue
+    const uint32_t idesc = idesc_bf16(128, 256);
+    const uint64_t a_base = umma_desc(smem_addr(As), kSlabPlaneBytes, 128);
+    const uint64_t b_base = umma_desc(smem_addr(Bs), 256 * 16, 128);
+    int ga = 0, gb = 0, it = 0;
+    for (int j = blockIdx.x; j < jobs; j += gridDim.x, ++it) {
+      mbar_wait(acce, (it & 1) ^ 1);  // the epilogue has drained the accumulators
+      fence_after();
+      for (int g = 0; g < G; ++g, ++ga) {
+        const int sa = ga % kSlabAStages;
+        mbar_wait(fullA0 + 8 * sa, (ga / kSlabAStages) & 1);
+        for (int t = 0; t < 9; ++t, ++gb) {
+          const int sb = gb % kSlabBStages;
+          mbar_wait(fullB0 + 8 * sb, (gb / kSlabBStages) & 1);
+          fence_after();
+          const int toff = ((t / 3) * 15 + (t % 3)) * 16;  // tap (dy, dx): entries p + 15 dy + dx
+#pragma unroll
+          for (int h = 0; h < 2; ++h)
+#pragma unroll
+            for (int k = 0; k < 4; ++k)  // 16 channels = planes 2k, 2k + 1
+              mma_bf16(tmem + (uint32_t)(h * 256),
+                       a_base + (uint64_t)((sa * kSlabA + h * kSlabHalf + 2 * k * kSlabPlaneBytes + toff) >> 4),
+                       b_base + (uint64_t)((sb * kSlabBStage + k * 2 * 256 * 16) >> 4), idesc,
+                       (g | t | k) ? 1u : 0u);
+          mma_commit(emptyB0 + 8 * sb);
+        }
+        mma_commit(emptyA0 + 8 * sa);
+      }
+      mma_commit(accf);
+    }
+  } else {
+    // ---------------- epilogue (warps 0-3): lane = row of each half
+    const int qd = warp & 3, r = 32 * qd + lane;
+    int it = 0;
+    for (int j = blockIdx.x; j < jobs; j += gridDim.x, ++it) {
+      const int mt = j / n_nt, nt = j - mt * n_nt;
+      mbar_wait(accf, it & 1);
+      fence_after();
+      for (int h = 0; h < 2; ++h) {
+        const int64_t p = (int64_t)mt * 256 + 128 * h + r;
+        const int64_t f = p / 225;
+        const int q = (int)(p - f * 225), y = q / 15, x = q - 15 * (q / 15);
+        const bool valid = f < a.N && y < 13 && x < 13;
+        const uint32_t trow = tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(h * 256);
+        for (int c0 = 0; c0 < 256; c0 += 16) {
+          uint32_t rr[16];
+          tmem_ld16(trow + (uint32_t)c0, rr);
+          tmem_wait_ld(rr);
+          if (!valid) continue;
+          const int co = nt * 256 + c0;
+          uint32_t w[8];
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            float x0 = __uint_as_float(rr[2 * k]) + __ldg(a.bias + co + 2 * k);
+            float x1 = __uint_as_float(rr[2 * k + 1]) + __ldg(a.bias + co + 2 * k + 1);
+            x0 = x0 < 0.f ? 0.1f * x0 : x0;
+            x1 = x1 < 0.f ? 0.1f * x1 : x1;
+            w[k] = pack_bf16(x0, x1);
+          }
+          if (a.out_plane > 0) {  // next layer's slab layout: (y, x) -> padded (y + 1, x + 1)
+            const int64_t e = f * 225 + (y + 1) * 15 + x + 1;
+            *reinterpret_cast<uint4*>(a.out + ((int64_t)(co >> 3) * a.out_plane + e) * 8) = make_uint4(w[0], w[1], w[2], w[3]);
+            *reinterpret_cast<uint4*>(a.out + ((int64_t)((co >> 3) + 1) * a.out_plane + e) * 8) =
+                make_uint4(w[4], w[5], w[6], w[7]);
+          } else {
+            uint4* o = reinterpret_cast<uint4*>(a.out + (f * 169 + y * 13 + x) * a.Cout + co);
+            o[0] = make_uint4(w[0], w[1], w[2], w[3]);
+            o[1] = make_uint4(w[4], w[5], w[6], w[7]);
+          }
+        }
+      }
+      fence_before();
+      mbar_arrive(acce);
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == 5) {
+    fence_after();
+    tmem_dealloc(tmem, 512);
+  }
+}
+
 }  // namespace
 
 int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT) {
@@ -768,6 +941,8 @@ cudaError_t tyolo_configure() {
   {
     cudaError_t e = cudaFuncSetAttribute(tyolo_l1_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kL1Smem);
     if (e == cudaSuccess) e = cudaFuncSetAttribute(tyolo_l2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kL2Smem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(tyolo_slab_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSlabSmem);
     if (e != cudaSuccess) return e;
   }
   cudaError_t e = cudaFuncSetAttribute(tyolo_conv_kernel<1, 4, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -809,10 +984,16 @@ cudaError_t launch_tyolo_l2(const TyL1Args& a, int num_sms, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+cudaError_t launch_tyolo_slab(const TySlabArgs& a, int num_sms, cudaStream_t st) {
+  const int jobs = ((a.N * 225 + 255) / 256) * (a.Cout / 256);
+  tyolo_slab_kernel<<<jobs < num_sms ? jobs : num_sms, kSlabThreads, kSlabSmem, st>>>(a);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_tyolo_pool_s1(const __nv_bfloat16* in, __nv_bfloat16* out, int32_t n, int32_t H, int32_t C,
-                                 cudaStream_t st) {
+                                 int64_t planar_stride, cudaStream_t st) {
   const int64_t total = (int64_t)n * H * H * (C / 8);
-  tyolo_pool_s1_kernel<<<(unsigned)((total + 255) / 256), 256, 0, st>>>(in, out, n, H, C);
+  tyolo_pool_s1_kernel<<<(unsigned)((total + 255) / 256), 256, 0, st>>>(in, out, n, H, C, planar_stride);
   return cudaGetLastError();
 }
 

@@ -56,6 +56,8 @@ struct ffsva_tyolo {
   uint8_t* d_w1v = nullptr;        // layer 1 weights for the patch-view kernel (8 KB)
   __nv_bfloat16* d_pad2 = nullptr; // layer 1's planar zero-bordered output (layer 2's input), kTyL2PadBytes per frame
   uint8_t* d_w2v = nullptr;        // layer 2 weights for the patch-view kernel (64 KB)
+  __nv_bfloat16* d_slab[2] = {nullptr, nullptr};  // slab layouts of layer 7's (512 ch) and layer 8's (1024 ch) inputs
+  int64_t slab_plane = 0;          // entries per slab plane (fixed per workspace: the zero border must not move)
   float* d_raw = nullptr;
   int32_t* d_counts = nullptr;
   TyFrame* d_frames = nullptr;
@@ -159,6 +161,8 @@ ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
   cudaFree(m->d_act[1]);
   cudaFree(m->d_pad);
   cudaFree(m->d_pad2);
+  cudaFree(m->d_slab[0]);
+  cudaFree(m->d_slab[1]);
   cudaFree(m->d_raw);
   cudaFree(m->d_counts);
   cudaFree(m->d_frames);
@@ -175,6 +179,12 @@ ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
   if (e == cudaSuccess) e = cudaMemset(m->d_pad, 0, pad_bytes);  // the border is written once, here
   if (e == cudaSuccess) e = cudaMalloc(&m->d_pad2, (size_t)cap * kTyL2PadBytes);
   if (e == cudaSuccess) e = cudaMemset(m->d_pad2, 0, (size_t)cap * kTyL2PadBytes);
+  m->slab_plane = tyolo_slab_plane(cap);
+  for (int k = 0; k < 2 && e == cudaSuccess; ++k) {
+    const size_t bytes = (size_t)(k == 0 ? 512 : 1024) / 8 * (size_t)m->slab_plane * 16;
+    e = cudaMalloc(&m->d_slab[k], bytes);
+    if (e == cudaSuccess) e = cudaMemset(m->d_slab[k], 0, bytes);
+  }
   if (e == cudaSuccess) e = cudaMalloc(&m->d_raw, (size_t)cap * kGrid * kGrid * kHeadPad * 4);
   if (e == cudaSuccess) e = cudaMalloc(&m->d_counts, (size_t)cap * 4);
   if (e == cudaSuccess) e = cudaMalloc(&m->d_frames, (size_t)cap * sizeof(TyFrame));
@@ -260,16 +270,35 @@ ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, const int32_t*
     if (ev) cudaEventRecord(ev[3], st);
   }
   for (int l = 2; l <= upto; ++l) {
+    if (l == 6 || l == 7) {  // 13x13 layers 7 and 8 by slab views: slab 0 -> slab 1 -> NHWC
+      const Layer& L = m->L[l];
+      TySlabArgs sa{};
+      sa.in = m->d_slab[l - 6];
+      sa.plane = m->slab_plane;
+      sa.out = l == 6 ? m->d_slab[1] : m->d_act[0];
+      sa.out_plane = l == 6 ? m->slab_plane : 0;
+      sa.wpk = m->d_w + L.w_off;
+      sa.bias = m->d_b + L.b_off;
+      sa.N = n;
+      sa.Cin = L.Cin;
+      sa.Cout = L.Cout_pad;
+      if ((e = launch_tyolo_slab(sa, ctx->num_sms, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO slab layer");
+      g_launches += 1;
+      cur = l == 6 ? -4 : 0;  // -4: slab 1 (layer 7's output)
+      if (ev) cudaEventRecord(ev[2 + l], st);
+      continue;
+    }
     const TyConvArgs a = layer_args(m, l, n, m->d_act[cur], m->d_act[cur ^ 1], thresh);
     if ((e = launch_tyolo_conv(a, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO conv layer");
     g_launches += 1;
     cur ^= 1;
-    if (m->L[l].pool == 2) {  // 2x2/1 max-pool (Q30) back into the layer's input buffer
+    if (m->L[l].pool == 2) {  // 2x2/1 max-pool (Q30) into layer 7's slab input
       const Layer& L = m->L[l];
-      if ((e = launch_tyolo_pool_s1(m->d_act[cur], m->d_act[cur ^ 1], n, L.Ho, L.Cout_pad, st)) != cudaSuccess)
+      if ((e = launch_tyolo_pool_s1(m->d_act[cur], m->d_slab[0], n, L.Ho, L.Cout_pad, m->slab_plane, st)) !=
+          cudaSuccess)
         return cuda_fail(ctx, e, "T-YOLO 2x2/1 pool");
       g_launches += 1;
-      cur ^= 1;
+      cur = -3;  // -3: slab 0 (layer 6's pooled output)
     }
     if (ev) cudaEventRecord(ev[2 + l], st);
   }
@@ -451,6 +480,20 @@ FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_fram
           }
     return FFSVA_OK;
   }
+  if (buf == -3 || buf == -4) {  // layers 6 / 7: unpack a slab layout (planes of 8 channels, 15x15 padded grid)
+    const int C = buf == -3 ? 512 : 1024;
+    std::vector<uint16_t> sl((size_t)C / 8 * m->slab_plane * 8);
+    e = cudaMemcpyAsync(sl.data(), m->d_slab[buf == -3 ? 0 : 1], sl.size() * 2, cudaMemcpyDeviceToHost, cs);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_tyolo_layer_output");
+    for (int i = 0; i < n; ++i)
+      for (int y = 0; y < 13; ++y)
+        for (int x = 0; x < 13; ++x)
+          for (int c = 0; c < C; ++c)
+            out[(((size_t)i * 13 + y) * 13 + x) * C + c] =
+                sl[((size_t)(c >> 3) * m->slab_plane + (size_t)i * 225 + (y + 1) * 15 + x + 1) * 8 + (c & 7)];
+    return FFSVA_OK;
+  }
   if (buf == -1) {  // the resized input: the interior of the zero-bordered buffer
     const size_t row = (size_t)kIn * 4 * 2, prow = (size_t)(kIn + 2) * 4 * 2;
     for (int i = 0; i < n && e == cudaSuccess; ++i)
@@ -515,6 +558,8 @@ FFSVA_API ffsva_status ffsva_tyolo_destroy(ffsva_tyolo* m) {
     cudaFree(m->d_w1v);
     cudaFree(m->d_pad2);
     cudaFree(m->d_w2v);
+    cudaFree(m->d_slab[0]);
+    cudaFree(m->d_slab[1]);
     cudaFree(m->d_raw);
     cudaFree(m->d_counts);
     cudaFree(m->d_frames);
