@@ -211,9 +211,9 @@ struct TySlabArgs {
   int64_t plane;             // entries per input plane
   __nv_bfloat16* out;        // slab layout (out_plane > 0) or NHWC [N][13][13][Cout]
   int64_t out_plane;
-  const uint8_t* wpk;        // the generic kernel's packing for this layer (NT = 256, K step = tap * Cin/64 + group)
+  const uint8_t* wpk;        // the generic kernel's packing for this layer (NT = 128, K step = tap * Cin/64 + group)
   const float* bias;
-  int32_t N, Cin, Cout;      // Cin % 64 == 0, Cout % 256 == 0
+  int32_t N, Cin, Cout;      // Cin % 64 == 0, Cout % 128 == 0
 };
 cudaError_t launch_tyolo_slab(const TySlabArgs& a, int num_sms, cudaStream_t st);
 cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int32_t max_row_bytes, int32_t max_H,

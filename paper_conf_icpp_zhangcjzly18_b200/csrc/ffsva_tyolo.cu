@@ -770,34 +770,35 @@ __global__ void __launch_bounds__(kL2Threads, 1) tyolo_l2_kernel(TyL1Args a) {
 // Y * 15 + X over the 15x15 padded grid (frames stacked). Output rows of the GEMM are the padded-grid entries p
 // themselves (rows with y or x >= 13 are computed and discarded: 169 of 225 useful), so tap (dy, dx) of consecutive
 // rows is the plane read at p + dy*15 + dx: a constant-stride UMMA view (rows 16 B apart, channel groups one plane
-// apart, 8-row groups 128 B apart). A tile job = 2 x 128 rows x 256 output channels; per 64-channel group one slab
+// apart, 8-row groups 128 B apart). A tile job = 2 x 128 rows x 128 output channels (two TMEM accumulator buffers); per 64-channel group one slab
 // of 160 entries x 8 planes per half is bulk-copied (16 copies) and feeds all nine taps, so the A operand costs
-// 40 KB per 9 K steps instead of a 32 KB im2col gather per step; B (the pre-packed weights of the generic kernel,
-// K step = tap * (Cin/64) + group) streams through a 4-stage ring. Warp 4 lane 0 copies, warp 5 issues MMAs,
+// 40 KB per 9 K steps instead of a 32 KB im2col gather per step; B (the pre-packed weights of the generic kernel's
+// layout with NT = 128, K step = tap * (Cin/64) + group) streams through a 6-stage ring. Warp 4 lane 0 copies, warp 5 issues MMAs,
 // warps 0-3 drain the accumulators (bias, leaky, bf16) into the next slab layout or NHWC.
 constexpr int kSlabEntries = 160;               // 128 rows + the largest tap offset (2 * 15 + 2) rounded up
 constexpr int kSlabPlaneBytes = kSlabEntries * 16;  // 2560
 constexpr int kSlabHalf = 8 * kSlabPlaneBytes;  // 20,480 B: one half's 64-channel slab
 constexpr int kSlabA = 2 * kSlabHalf;           // both halves
-constexpr int kSlabAStages = 2, kSlabBStages = 4;
-constexpr int kSlabBStage = 64 * 256 * 2;       // 32 KB: one K step of weights for a 256-wide N tile
+constexpr int kSlabAStages = 2, kSlabBStages = 6;
+constexpr int kSlabNT = 128;                    // N tile: two accumulator buffers of 2 x 128 columns fit in TMEM
+constexpr int kSlabBStage = 64 * kSlabNT * 2;   // 16 KB: one K step of weights for a 128-wide N tile
 constexpr int kSlabThreads = 192;
 constexpr int kSlabSmem = kSlabAStages * kSlabA + kSlabBStages * kSlabBStage +
-                          8 * (2 * kSlabAStages + 2 * kSlabBStages + 2) + 16;
+                          8 * (2 * kSlabAStages + 2 * kSlabBStages + 4) + 16;
 
 __global__ void __launch_bounds__(kSlabThreads, 1) tyolo_slab_kernel(TySlabArgs a) {
   extern __shared__ __align__(1024) uint8_t sm[];
   uint8_t* As = sm;
   uint8_t* Bs = sm + kSlabAStages * kSlabA;
   uint64_t* bars = reinterpret_cast<uint64_t*>(Bs + kSlabBStages * kSlabBStage);
-  uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 2 * kSlabAStages + 2 * kSlabBStages + 2);
+  uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 2 * kSlabAStages + 2 * kSlabBStages + 4);
   const uint32_t fullA0 = smem_addr(bars), emptyA0 = fullA0 + 8 * kSlabAStages;
   const uint32_t fullB0 = emptyA0 + 8 * kSlabAStages, emptyB0 = fullB0 + 8 * kSlabBStages;
-  const uint32_t accf = emptyB0 + 8 * kSlabBStages, acce = accf + 8;
+  const uint32_t accf0 = emptyB0 + 8 * kSlabBStages, acce0 = accf0 + 16;  // two accumulator buffers
   const int tid = threadIdx.x, lane = tid & 31;
   const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);
   const int G = a.Cin >> 6;                       // 64-channel groups
-  const int n_nt = a.Cout >> 8;                   // 256-wide N tiles
+  const int n_nt = a.Cout / kSlabNT;
   const int m_tiles = (a.N * 225 + 255) >> 8;
   const int jobs = m_tiles * n_nt;
 
@@ -810,8 +811,10 @@ __global__ void __launch_bounds__(kSlabThreads, 1) tyolo_slab_kernel(TySlabArgs 
       mbar_init(fullB0 + 8 * s, 1);
       mbar_init(emptyB0 + 8 * s, 1);
     }
-    mbar_init(accf, 1);
-    mbar_init(acce, 128);
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(accf0 + 8 * b, 1);
+      mbar_init(acce0 + 8 * b, 128);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 5) tmem_alloc(smem_addr(s_tmem), 512);
@@ -848,12 +851,13 @@ __global__ void __launch_bounds__(kSlabThreads, 1) tyolo_slab_kernel(TySlabArgs 
     }
   } else if (warp == 5) {
     // ---------------- MMA issue
-    const uint32_t idesc = idesc_bf16(128, 256);
+    const uint32_t idesc = idesc_bf16(128, kSlabNT);
     const uint64_t a_base = umma_desc(smem_addr(As), kSlabPlaneBytes, 128);
-    const uint64_t b_base = umma_desc(smem_addr(Bs), 256 * 16, 128);
+    const uint64_t b_base = umma_desc(smem_addr(Bs), kSlabNT * 16, 128);
     int ga = 0, gb = 0, it = 0;
     for (int j = blockIdx.x; j < jobs; j += gridDim.x, ++it) {
-      mbar_wait(acce, (it & 1) ^ 1);  // the epilogue has drained the accumulators
+      const int ab = it & 1;
+      mbar_wait(acce0 + 8 * ab, ((it >> 1) & 1) ^ 1);  // the epilogue has drained this accumulator buffer
       fence_after();
       for (int g = 0; g < G; ++g, ++ga) {
         const int sa = ga % kSlabAStages;
@@ -867,15 +871,15 @@ __global__ void __launch_bounds__(kSlabThreads, 1) tyolo_slab_kernel(TySlabArgs 
           for (int h = 0; h < 2; ++h)
 #pragma unroll
             for (int k = 0; k < 4; ++k)  // 16 channels = planes 2k, 2k + 1
-              mma_bf16(tmem + (uint32_t)(h * 256),
+              mma_bf16(tmem + (uint32_t)(ab * 2 * kSlabNT + h * kSlabNT),
                        a_base + (uint64_t)((sa * kSlabA + h * kSlabHalf + 2 * k * kSlabPlaneBytes + toff) >> 4),
-                       b_base + (uint64_t)((sb * kSlabBStage + k * 2 * 256 * 16) >> 4), idesc,
+                       b_base + (uint64_t)((sb * kSlabBStage + k * 2 * kSlabNT * 16) >> 4), idesc,
                        (g | t | k) ? 1u : 0u);
           mma_commit(emptyB0 + 8 * sb);
         }
         mma_commit(emptyA0 + 8 * sa);
       }
-      mma_commit(accf);
+      mma_commit(accf0 + 8 * ab);
     }
   } else {
     // ---------------- epilogue (warps 0-3): lane = row of each half
@@ -883,20 +887,21 @@ __global__ void __launch_bounds__(kSlabThreads, 1) tyolo_slab_kernel(TySlabArgs 
     int it = 0;
     for (int j = blockIdx.x; j < jobs; j += gridDim.x, ++it) {
       const int mt = j / n_nt, nt = j - mt * n_nt;
-      mbar_wait(accf, it & 1);
+      const int ab = it & 1;
+      mbar_wait(accf0 + 8 * ab, (it >> 1) & 1);
       fence_after();
       for (int h = 0; h < 2; ++h) {
         const int64_t p = (int64_t)mt * 256 + 128 * h + r;
         const int64_t f = p / 225;
         const int q = (int)(p - f * 225), y = q / 15, x = q - 15 * (q / 15);
         const bool valid = f < a.N && y < 13 && x < 13;
-        const uint32_t trow = tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(h * 256);
-        for (int c0 = 0; c0 < 256; c0 += 16) {
+        const uint32_t trow = tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(ab * 2 * kSlabNT + h * kSlabNT);
+        for (int c0 = 0; c0 < kSlabNT; c0 += 16) {
           uint32_t rr[16];
           tmem_ld16(trow + (uint32_t)c0, rr);
           tmem_wait_ld(rr);
           if (!valid) continue;
-          const int co = nt * 256 + c0;
+          const int co = nt * kSlabNT + c0;
           uint32_t w[8];
 #pragma unroll
           for (int k = 0; k < 8; ++k) {
@@ -919,7 +924,7 @@ __global__ void __launch_bounds__(kSlabThreads, 1) tyolo_slab_kernel(TySlabArgs 
         }
       }
       fence_before();
-      mbar_arrive(acce);
+      mbar_arrive(acce0 + 8 * ab);
     }
   }
   fence_before();
@@ -985,7 +990,7 @@ cudaError_t launch_tyolo_l2(const TyL1Args& a, int num_sms, cudaStream_t st) {
 }
 
 cudaError_t launch_tyolo_slab(const TySlabArgs& a, int num_sms, cudaStream_t st) {
-  const int jobs = ((a.N * 225 + 255) / 256) * (a.Cout / 256);
+  const int jobs = ((a.N * 225 + 255) / 256) * (a.Cout / kSlabNT);
   tyolo_slab_kernel<<<jobs < num_sms ? jobs : num_sms, kSlabThreads, kSlabSmem, st>>>(a);
   return cudaGetLastError();
 }

@@ -89,6 +89,7 @@ void build_layers(ffsva_tyolo* m) {
     L.conv_pool = L.pool == 1 ? 1 : 0;
     L.nq = L.conv_pool ? 4 : 1;
     L.NT = std::min(L.Cout_pad, L.conv_pool ? 128 : 256);
+    if (l == 6 || l == 7) L.NT = 128;  // layers 7 and 8 run on the slab kernel (N tile 128)
     L.patch = L.conv_pool && L.Cp <= patch_cp ? 1 : 0;
     L.msub = L.conv_pool ? 1 : std::max(1, std::min(2, msub));
     if (L.patch) L.kchunks = 16 * L.Cp / 64 > 0 ? 16 * L.Cp / 64 : 1;  // 4x4 patch x Cp channels
