@@ -191,6 +191,7 @@ cudaError_t launch_tyolo_conv(const TyConvArgs& a, cudaStream_t st);
 struct TyL1Args {
   const __nv_bfloat16* in;
   __nv_bfloat16* out;
+  int64_t out_plane;         // layer 2: > 0 writes layer 3's parity slab (entries per plane), else NHWC
   const uint8_t* w;          // 4 patch rows x [2 K-halves][64 n = 16q + oc][8 k = 4u + c] bf16 (8 KB)
   const float* bias;         // [16]
   int32_t N;
@@ -216,6 +217,23 @@ struct TySlabArgs {
   int32_t N, Cin, Cout;      // Cin % 64 == 0, Cout % 128 == 0
 };
 cudaError_t launch_tyolo_slab(const TySlabArgs& a, int num_sms, cudaStream_t st);
+// Pool layers 3-5 by parity-slab views (tyolo_pslab_kernel). Parity slab of C channels on an H x H grid: planes
+// [C/8][Y parity][X parity] of `plane` 16-byte entries, entry = frame * Gp^2 + (Y >> 1) * Gp + (X >> 1) over the
+// zero-bordered (H+2)^2 grid, Gp = H/2 + 1; plane >= round_up(N * Gp^2, 128) + Gp + 16.
+inline int64_t tyolo_pslab_plane(int32_t n, int32_t Gp) {
+  return ((int64_t)n * Gp * Gp + 127) / 128 * 128 + Gp + 16;
+}
+struct TyPslabArgs {
+  const __nv_bfloat16* in;   // parity slab, Cin channels, grid Gp
+  int64_t plane;
+  __nv_bfloat16* out;        // next layer's parity slab (out_plane > 0, grid out_Gp) or NHWC [N][Gp-1][Gp-1][Cout]
+  int64_t out_plane;
+  int32_t out_Gp;
+  const uint8_t* wpk;        // [N tile of 64][64-channel group][tap][8-channel K group][64 n][8] bf16
+  const float* bias;
+  int32_t N, Cin, Cout, Gp;  // Cin 32 / 64 / 128 ..., Cout % 64 == 0
+};
+cudaError_t launch_tyolo_pslab(const TyPslabArgs& a, int num_sms, cudaStream_t st);
 cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int32_t max_row_bytes, int32_t max_H,
                                 __nv_bfloat16* out, cudaStream_t st);
 int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT);

@@ -749,11 +749,21 @@ __global__ void __launch_bounds__(kL2Threads, 1) tyolo_l2_kernel(TyL1Args a) {
       fence_before();
       mbar_arrive(acce0 + 8 * b);
       if (r < kL2Out) {
-        uint4* o = reinterpret_cast<uint4*>(a.out + (((int64_t)n * kL2Out + oy) * kL2Out + r) * 32);
-        o[0] = make_uint4(w[0], w[1], w[2], w[3]);
-        o[1] = make_uint4(w[4], w[5], w[6], w[7]);
-        o[2] = make_uint4(w[8], w[9], w[10], w[11]);
-        o[3] = make_uint4(w[12], w[13], w[14], w[15]);
+        if (a.out_plane > 0) {  // layer 3's parity-slab input (see tyolo_pslab_kernel): 32 channels, grid 53 x 53
+          const int Y = oy + 1, X = r + 1;
+          const int64_t e = (int64_t)n * 53 * 53 + (Y >> 1) * 53 + (X >> 1);
+          const int par = (Y & 1) * 2 + (X & 1);
+#pragma unroll
+          for (int cg = 0; cg < 4; ++cg)
+            *reinterpret_cast<uint4*>(a.out + (((int64_t)cg * 4 + par) * a.out_plane + e) * 8) =
+                make_uint4(w[4 * cg], w[4 * cg + 1], w[4 * cg + 2], w[4 * cg + 3]);
+        } else {
+          uint4* o = reinterpret_cast<uint4*>(a.out + (((int64_t)n * kL2Out + oy) * kL2Out + r) * 32);
+          o[0] = make_uint4(w[0], w[1], w[2], w[3]);
+          o[1] = make_uint4(w[4], w[5], w[6], w[7]);
+          o[2] = make_uint4(w[8], w[9], w[10], w[11]);
+          o[3] = make_uint4(w[12], w[13], w[14], w[15]);
+        }
       }
     }
   }
@@ -935,6 +945,191 @@ __global__ void __launch_bounds__(kSlabThreads, 1) tyolo_slab_kernel(TySlabArgs 
   }
 }
 
+// ---------------------------------------------------------------- pool layers 3-5 by parity-slab views
+// Input layout ("parity slab") of a layer with C channels on an H x H grid (H even), zero-bordered to (H+2)^2: for
+// every 8-channel group cg and padded-coordinate parity (Y & 1, X & 1) a plane of 16-byte entries, entry
+// e = frame * Gp^2 + (Y >> 1) * Gp + (X >> 1), Gp = (H + 2) / 2, planes ordered [cg][Y parity][X parity]. GEMM rows
+// are the entries e = (frame, py, px) of that Gp x Gp grid read as POOLED output pixels (py, px < H/2 useful: 96 % /
+// 93 % / 86 % for layers 3 / 4 / 5). For pool position (a, b) and tap (dy, dx) the input pixel is padded
+// (2py + a + dy, 2px + b + dx): plane parity ((a + dy) & 1, (b + dx) & 1) at entry e + ((a + dy) >> 1) * Gp +
+// ((b + dx) >> 1) — a constant-stride view for every (position, tap), so the four pool positions are four TMEM
+// accumulator chains fed from one staged slab (rows 16 B apart, channel groups four planes apart, 8-row groups
+// 128 B apart) and the 3x3 weights are shared by the chains. Per 64-channel group one slab of 128 + Gp + 2 entries
+// x 4 parities x 8 groups is bulk-copied (32 copies) and feeds 9 taps x 4 chains; weights (8 KB per tap and group,
+// N tile 64) stream through a ring. Warp 4 lane 0 copies, warp 5 issues, warps 0-3 max-pool / bias / leaky / bf16
+// into the next layer's parity slab or NHWC.
+constexpr int kPsBStages = 6;
+constexpr int kPsBStage = 64 * 64 * 2;          // 8 KB: one (tap, 64-channel group) of weights, N tile 64
+constexpr int kPsThreads = 192;
+constexpr int kPsMaxSlab = 96 * 1024;           // per A stage
+
+__host__ __device__ inline int ps_slab_entries(int Gp) { return (128 + Gp + 2 + 7) & ~7; }
+
+__global__ void __launch_bounds__(kPsThreads, 1) tyolo_pslab_kernel(TyPslabArgs a) {
+  extern __shared__ __align__(1024) uint8_t sm[];
+  const int Gp = a.Gp, SE = ps_slab_entries(Gp), SEB = SE * 16;
+  const int CG = a.Cin >= 64 ? 8 : a.Cin / 8;     // channel groups per slab (64 channels, or all of a smaller Cin)
+  const int G = a.Cin >= 64 ? a.Cin / 64 : 1;
+  const int slab_bytes = CG * 4 * SEB;
+  uint8_t* As = sm;
+  uint8_t* Bs = sm + 2 * slab_bytes;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(Bs + kPsBStages * kPsBStage);
+  uint32_t* s_tmem = reinterpret_cast<uint32_t*>(bars + 4 + 2 * kPsBStages + 4);
+  const uint32_t fullA0 = smem_addr(bars), emptyA0 = fullA0 + 16;
+  const uint32_t fullB0 = emptyA0 + 16, emptyB0 = fullB0 + 8 * kPsBStages;
+  const uint32_t accf0 = emptyB0 + 8 * kPsBStages, acce0 = accf0 + 16;
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);
+  const int n_nt = a.Cout / 64;
+  const int64_t entries = (int64_t)a.N * Gp * Gp;
+  const int m_tiles = (int)((entries + 127) / 128);
+  const int jobs = m_tiles * n_nt;
+  const int Ho = Gp - 1;
+
+  if (tid == 0) {
+    for (int s = 0; s < 2; ++s) {
+      mbar_init(fullA0 + 8 * s, 1);
+      mbar_init(emptyA0 + 8 * s, 1);
+    }
+    for (int s = 0; s < kPsBStages; ++s) {
+      mbar_init(fullB0 + 8 * s, 1);
+      mbar_init(emptyB0 + 8 * s, 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(accf0 + 8 * b, 1);
+      mbar_init(acce0 + 8 * b, 128);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 5) tmem_alloc(smem_addr(s_tmem), 512);
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *s_tmem;
+
+  if (warp == 4) {
+    if (lane == 0) {
+      int ga = 0, gb = 0;
+      for (int j = blockIdx.x; j < jobs; j += gridDim.x) {
+        const int mt = j / n_nt, nt = j - mt * n_nt;
+        const int64_t e0 = (int64_t)mt * 128;
+        for (int g = 0; g < G; ++g, ++ga) {
+          const int sa = ga & 1;
+          mbar_wait(emptyA0 + 8 * sa, ((ga >> 1) & 1) ^ 1);
+          mbar_expect_tx(fullA0 + 8 * sa, (uint32_t)slab_bytes);
+          for (int pl = 0; pl < CG * 4; ++pl)  // plane pl = cg * 4 + parity of this group
+            bulk_g2s(smem_addr(As + sa * slab_bytes + pl * SEB),
+                     reinterpret_cast<const char*>(a.in) + ((int64_t)(g * CG * 4 + pl) * a.plane + e0) * 16,
+                     (uint32_t)SEB, fullA0 + 8 * sa);
+          for (int t = 0; t < 9; ++t, ++gb) {
+            const int sb = gb % kPsBStages;
+            mbar_wait(emptyB0 + 8 * sb, ((gb / kPsBStages) & 1) ^ 1);
+            mbar_expect_tx(fullB0 + 8 * sb, kPsBStage);
+            bulk_g2s(smem_addr(Bs + sb * kPsBStage), a.wpk + (((int64_t)nt * G + g) * 9 + t) * kPsBStage, kPsBStage,
+                     fullB0 + 8 * sb);
+          }
+        }
+      }
+    }
+  } else if (warp == 5) {
+    const uint32_t idesc = idesc_bf16(128, 64);
+    const uint64_t a_base = umma_desc(smem_addr(As), 4 * SEB, 128);      // next channel group = 4 planes on
+    const uint64_t b_base = umma_desc(smem_addr(Bs), 64 * 16, 128);
+    const int ksteps = CG / 2;                                              // K16 steps per slab
+    int ga = 0, gb = 0, it = 0;
+    for (int j = blockIdx.x; j < jobs; j += gridDim.x, ++it) {
+      const int ab = it & 1;
+      mbar_wait(acce0 + 8 * ab, ((it >> 1) & 1) ^ 1);
+      fence_after();
+      for (int g = 0; g < G; ++g, ++ga) {
+        const int sa = ga & 1;
+        mbar_wait(fullA0 + 8 * sa, (ga >> 1) & 1);
+        for (int t = 0; t < 9; ++t, ++gb) {
+          const int sb = gb % kPsBStages;
+          mbar_wait(fullB0 + 8 * sb, (gb / kPsBStages) & 1);
+          fence_after();
+          const int dy = t / 3, dx = t - 3 * (t / 3);
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            const int ya = (q >> 1) + dy, xb = (q & 1) + dx;
+            const int par = (ya & 1) * 2 + (xb & 1), off = (ya >> 1) * Gp + (xb >> 1);
+            for (int k = 0; k < ksteps; ++k)
+              mma_bf16(tmem + (uint32_t)(ab * 256 + q * 64),
+                       a_base + (uint64_t)((sa * slab_bytes + (2 * k * 4 + par) * SEB + off * 16) >> 4),
+                       b_base + (uint64_t)((sb * kPsBStage + k * 2 * 64 * 16) >> 4), idesc, (g | t | k) ? 1u : 0u);
+          }
+          mma_commit(emptyB0 + 8 * sb);
+        }
+        mma_commit(emptyA0 + 8 * sa);
+      }
+      mma_commit(accf0 + 8 * ab);
+    }
+  } else {
+    const int qd = warp & 3, r = 32 * qd + lane;
+    int it = 0;
+    for (int j = blockIdx.x; j < jobs; j += gridDim.x, ++it) {
+      const int mt = j / n_nt, nt = j - mt * n_nt;
+      const int ab = it & 1;
+      mbar_wait(accf0 + 8 * ab, (it >> 1) & 1);
+      fence_after();
+      const int64_t e = (int64_t)mt * 128 + r;
+      const int64_t f = e / (Gp * Gp);
+      const int rem = (int)(e - f * Gp * Gp), py = rem / Gp, px = rem - Gp * (rem / Gp);
+      const bool valid = f < a.N && py < Ho && px < Ho;
+      const uint32_t trow = tmem + ((uint32_t)(32 * qd) << 16) + (uint32_t)(ab * 256);
+      for (int c0 = 0; c0 < 64; c0 += 16) {
+        uint32_t r0[16], r1[16], r2[16], r3[16];
+        tmem_ld16(trow + (uint32_t)c0, r0);
+        tmem_ld16(trow + (uint32_t)(64 + c0), r1);
+        tmem_ld16(trow + (uint32_t)(128 + c0), r2);
+        tmem_ld16(trow + (uint32_t)(192 + c0), r3);
+        tmem_wait_ld2(r0, r1);
+        reg_fence2(r2, r3);
+        if (!valid) continue;
+        const int co = nt * 64 + c0;
+        uint32_t w[8];
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          float x0 = fmaxf(fmaxf(__uint_as_float(r0[2 * k]), __uint_as_float(r1[2 * k])),
+                           fmaxf(__uint_as_float(r2[2 * k]), __uint_as_float(r3[2 * k]))) + __ldg(a.bias + co + 2 * k);
+          float x1 = fmaxf(fmaxf(__uint_as_float(r0[2 * k + 1]), __uint_as_float(r1[2 * k + 1])),
+                           fmaxf(__uint_as_float(r2[2 * k + 1]), __uint_as_float(r3[2 * k + 1]))) +
+                     __ldg(a.bias + co + 2 * k + 1);
+          x0 = x0 < 0.f ? 0.1f * x0 : x0;
+          x1 = x1 < 0.f ? 0.1f * x1 : x1;
+          w[k] = pack_bf16(x0, x1);
+        }
+        if (a.out_plane > 0) {  // the next layer's parity slab (grid Go = Ho / 2 + 1)
+          const int Go = a.out_Gp, Y = py + 1, X = px + 1;
+          const int64_t eo = f * Go * Go + (Y >> 1) * Go + (X >> 1);
+          const int par = (Y & 1) * 2 + (X & 1);
+          *reinterpret_cast<uint4*>(a.out + (((int64_t)(co >> 3) * 4 + par) * a.out_plane + eo) * 8) =
+              make_uint4(w[0], w[1], w[2], w[3]);
+          *reinterpret_cast<uint4*>(a.out + (((int64_t)((co >> 3) + 1) * 4 + par) * a.out_plane + eo) * 8) =
+              make_uint4(w[4], w[5], w[6], w[7]);
+        } else {
+          uint4* o = reinterpret_cast<uint4*>(a.out + ((f * Ho + py) * Ho + px) * a.Cout + co);
+          o[0] = make_uint4(w[0], w[1], w[2], w[3]);
+          o[1] = make_uint4(w[4], w[5], w[6], w[7]);
+        }
+      }
+      fence_before();
+      mbar_arrive(acce0 + 8 * ab);
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == 5) {
+    fence_after();
+    tmem_dealloc(tmem, 512);
+  }
+}
+
+int ps_smem_bytes(int Cin, int Gp) {
+  const int CG = Cin >= 64 ? 8 : Cin / 8;
+  return 2 * CG * 4 * ps_slab_entries(Gp) * 16 + kPsBStages * kPsBStage + 8 * (4 + 2 * kPsBStages + 4) + 16;
+}
+
 }  // namespace
 
 int tyolo_conv_smem_bytes(int stages, int a_tiles, int b_tiles, int NT) {
@@ -948,6 +1143,8 @@ cudaError_t tyolo_configure() {
     if (e == cudaSuccess) e = cudaFuncSetAttribute(tyolo_l2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kL2Smem);
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(tyolo_slab_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSlabSmem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(tyolo_pslab_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
     if (e != cudaSuccess) return e;
   }
   cudaError_t e = cudaFuncSetAttribute(tyolo_conv_kernel<1, 4, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -986,6 +1183,15 @@ cudaError_t launch_tyolo_l2(const TyL1Args& a, int num_sms, cudaStream_t st) {
   const int tiles = a.N * kL2Out;
   const int grid = tiles < num_sms ? tiles : num_sms;
   tyolo_l2_kernel<<<grid, kL2Threads, kL2Smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_tyolo_pslab(const TyPslabArgs& a, int num_sms, cudaStream_t st) {
+  const int smem = ps_smem_bytes(a.Cin, a.Gp);
+  if (smem > 227 * 1024 || a.Cout % 64 || (a.Cin < 64 && a.Cin % 16) || (a.Cin >= 64 && a.Cin % 64))
+    return cudaErrorInvalidValue;
+  const int64_t jobs = (((int64_t)a.N * a.Gp * a.Gp + 127) / 128) * (a.Cout / 64);
+  tyolo_pslab_kernel<<<(unsigned)(jobs < num_sms ? jobs : num_sms), kPsThreads, smem, st>>>(a);
   return cudaGetLastError();
 }
 

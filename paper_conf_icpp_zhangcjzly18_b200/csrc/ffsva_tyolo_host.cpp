@@ -17,6 +17,9 @@ constexpr int kIn = 416;      // T-YOLO input size (L169)
 constexpr int kGrid = 13;     // output grid (L171)
 constexpr int kHeadPad = 128; // 125 outputs padded to a 128-column tile
 constexpr int kMaxChunk = 256;
+// parity slabs of layers 3, 4, 5 (see TyPslabArgs): channels and grid size Gp = H/2 + 1 of their inputs
+constexpr int kPsC[3] = {32, 64, 128};
+constexpr int kPsGp[3] = {53, 27, 14};
 
 // tiny-yolo-voc: (Cin, Cout, kernel, pool after: 0 none, 1 2x2/2, 2 2x2/1)
 constexpr int kNet[9][4] = {{3, 16, 3, 1},     {16, 32, 3, 1},     {32, 64, 3, 1},
@@ -58,6 +61,9 @@ struct ffsva_tyolo {
   uint8_t* d_w2v = nullptr;        // layer 2 weights for the patch-view kernel (64 KB)
   __nv_bfloat16* d_slab[2] = {nullptr, nullptr};  // slab layouts of layer 7's (512 ch) and layer 8's (1024 ch) inputs
   int64_t slab_plane = 0;          // entries per slab plane (fixed per workspace: the zero border must not move)
+  __nv_bfloat16* d_ps[3] = {nullptr, nullptr, nullptr};  // parity slabs: inputs of layers 3, 4, 5
+  int64_t ps_plane[3] = {0, 0, 0};
+  uint8_t* d_wps[3] = {nullptr, nullptr, nullptr};       // layers 3-5 weights for the parity-slab kernel
   float* d_raw = nullptr;
   int32_t* d_counts = nullptr;
   TyFrame* d_frames = nullptr;
@@ -164,6 +170,7 @@ ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
   cudaFree(m->d_pad2);
   cudaFree(m->d_slab[0]);
   cudaFree(m->d_slab[1]);
+  for (auto& p : m->d_ps) cudaFree(p);
   cudaFree(m->d_raw);
   cudaFree(m->d_counts);
   cudaFree(m->d_frames);
@@ -181,6 +188,12 @@ ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
   if (e == cudaSuccess) e = cudaMalloc(&m->d_pad2, (size_t)cap * kTyL2PadBytes);
   if (e == cudaSuccess) e = cudaMemset(m->d_pad2, 0, (size_t)cap * kTyL2PadBytes);
   m->slab_plane = tyolo_slab_plane(cap);
+  for (int k = 0; k < 3 && e == cudaSuccess; ++k) {  // layers 3, 4, 5: C = 32, 64, 128 on grids 104, 52, 26
+    m->ps_plane[k] = tyolo_pslab_plane(cap, kPsGp[k]);
+    const size_t bytes = (size_t)(kPsC[k] / 8) * 4 * (size_t)m->ps_plane[k] * 16;
+    e = cudaMalloc(&m->d_ps[k], bytes);
+    if (e == cudaSuccess) e = cudaMemset(m->d_ps[k], 0, bytes);
+  }
   for (int k = 0; k < 2 && e == cudaSuccess; ++k) {
     const size_t bytes = (size_t)(k == 0 ? 512 : 1024) / 8 * (size_t)m->slab_plane * 16;
     e = cudaMalloc(&m->d_slab[k], bytes);
@@ -257,20 +270,42 @@ ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, const int32_t*
   if (ev) cudaEventRecord(ev[1], st);
   int cur = -1;  // -1: the padded resize output
   if (upto >= 0) {  // layer 1 by patch views of the padded input, into layer 2's planar padded input
-    const TyL1Args a1{m->d_pad, m->d_pad2, m->d_w1v, m->d_b + m->L[0].b_off, n};
+    const TyL1Args a1{m->d_pad, m->d_pad2, 0, m->d_w1v, m->d_b + m->L[0].b_off, n};
     if ((e = launch_tyolo_l1(a1, ctx->num_sms, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO layer 1");
     g_launches += 1;
     cur = -2;  // -2: the planar layer-1 output
     if (ev) cudaEventRecord(ev[2], st);
   }
   if (upto >= 1) {  // layer 2 by patch views
-    const TyL1Args a2{m->d_pad2, m->d_act[0], m->d_w2v, m->d_b + m->L[1].b_off, n};
+    const TyL1Args a2{m->d_pad2, m->d_ps[0], m->ps_plane[0], m->d_w2v, m->d_b + m->L[1].b_off, n};
     if ((e = launch_tyolo_l2(a2, ctx->num_sms, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO layer 2");
     g_launches += 1;
-    cur = 0;
+    cur = -10;  // -10 - k: parity slab k (layer 3 + k's input)
     if (ev) cudaEventRecord(ev[3], st);
   }
   for (int l = 2; l <= upto; ++l) {
+    if (l <= 4) {  // pool layers 3-5 by parity-slab views: slab 0 -> slab 1 -> slab 2 -> NHWC
+      const Layer& L = m->L[l];
+      const int k = l - 2;
+      TyPslabArgs pa{};
+      pa.in = m->d_ps[k];
+      pa.plane = m->ps_plane[k];
+      pa.out = l < 4 ? m->d_ps[k + 1] : m->d_act[0];
+      pa.out_plane = l < 4 ? m->ps_plane[k + 1] : 0;
+      pa.out_Gp = l < 4 ? kPsGp[k + 1] : 0;
+      pa.wpk = m->d_wps[k];
+      pa.bias = m->d_b + L.b_off;
+      pa.N = n;
+      pa.Cin = L.Cin;
+      pa.Cout = L.Cout_pad;
+      pa.Gp = kPsGp[k];
+      if ((e = launch_tyolo_pslab(pa, ctx->num_sms, st)) != cudaSuccess)
+        return cuda_fail(ctx, e, "T-YOLO parity-slab layer");
+      g_launches += 1;
+      cur = l < 4 ? -10 - (k + 1) : 0;
+      if (ev) cudaEventRecord(ev[2 + l], st);
+      continue;
+    }
     if (l == 6 || l == 7) {  // 13x13 layers 7 and 8 by slab views: slab 0 -> slab 1 -> NHWC
       const Layer& L = m->L[l];
       TySlabArgs sa{};
@@ -364,6 +399,32 @@ FFSVA_API ffsva_status ffsva_tyolo_load(int32_t device, const float* params, int
             w1v[((dy * 2 + (u >> 1)) * 64 + 16 * q + oc) * 8 + 4 * (u & 1) + c] =
                 bf16_bits(params[((oc * 3 + c) * 3 + ky) * 3 + kx]);
           }
+  // layers 3-5 for the parity-slab kernel: [N tile of 64][64-channel group][tap][8-channel K group][64 n][8] (K groups
+  // past Cin stay zero and are never read)
+  std::vector<uint16_t> wps[3];
+  {
+    const float* wl = params;
+    for (int l = 0; l < 5; ++l) {
+      const Layer& L = m->L[l];
+      if (l >= 2) {
+        const int G = std::max(1, L.Cin / 64), nts = L.Cout / 64;
+        std::vector<uint16_t>& v = wps[l - 2];
+        v.assign((size_t)nts * G * 9 * 8 * 64 * 8, 0);
+        for (int nt = 0; nt < nts; ++nt)
+          for (int g = 0; g < G; ++g)
+            for (int t = 0; t < 9; ++t)
+              for (int kg = 0; kg < 8; ++kg)
+                for (int nn = 0; nn < 64; ++nn)
+                  for (int ee = 0; ee < 8; ++ee) {
+                    const int c = 64 * g + 8 * kg + ee, oc = 64 * nt + nn;
+                    if (c >= L.Cin) continue;
+                    v[(((((size_t)nt * G + g) * 9 + t) * 8 + kg) * 64 + nn) * 8 + ee] =
+                        bf16_bits(wl[(((size_t)oc * L.Cin + c) * 3 + t / 3) * 3 + t % 3]);
+                  }
+      }
+      wl += (size_t)L.Cout * L.Cin * L.k * L.k + L.Cout;
+    }
+  }
   // layer 2 for the patch-view kernel: B of (patch row dy, column u) = [channel group g][n = 32q + oc][8 channels]
   std::vector<uint16_t> w2v(16 * 2 * 128 * 8, 0);
   {
@@ -383,6 +444,10 @@ FFSVA_API ffsva_status ffsva_tyolo_load(int32_t device, const float* params, int
     std::lock_guard<std::mutex> lk(ctx->mu);
     DeviceGuard g(device);
     cudaError_t e = cudaMalloc(&m->d_w, wbytes);
+    for (int k = 0; k < 3 && e == cudaSuccess; ++k) {
+      e = cudaMalloc(&m->d_wps[k], wps[k].size() * 2);
+      if (e == cudaSuccess) e = cudaMemcpy(m->d_wps[k], wps[k].data(), wps[k].size() * 2, cudaMemcpyHostToDevice);
+    }
     if (e == cudaSuccess) e = cudaMalloc(&m->d_w2v, w2v.size() * 2);
     if (e == cudaSuccess) e = cudaMemcpy(m->d_w2v, w2v.data(), w2v.size() * 2, cudaMemcpyHostToDevice);
     if (e == cudaSuccess) e = cudaMalloc(&m->d_w1v, w1v.size() * 2);
@@ -395,6 +460,7 @@ FFSVA_API ffsva_status ffsva_tyolo_load(int32_t device, const float* params, int
       cudaFree(m->d_w);
       cudaFree(m->d_w1v);
       cudaFree(m->d_w2v);
+      for (auto& p : m->d_wps) cudaFree(p);
       cudaFree(m->d_b);
       ctx_release(ctx);
       return cuda_fail(nullptr, e, "ffsva_tyolo_load");
@@ -481,6 +547,23 @@ FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_fram
           }
     return FFSVA_OK;
   }
+  if (buf <= -10) {  // parity slab k = -10 - buf: C = 32 / 64 / 128 channels of the H = 104 / 52 / 26 grid
+    const int k = -10 - buf, C = kPsC[k], Gp = kPsGp[k], H = 2 * (Gp - 1);
+    std::vector<uint16_t> ps((size_t)C / 8 * 4 * m->ps_plane[k] * 8);
+    e = cudaMemcpyAsync(ps.data(), m->d_ps[k], ps.size() * 2, cudaMemcpyDeviceToHost, cs);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
+    if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_tyolo_layer_output");
+    for (int i = 0; i < n; ++i)
+      for (int y = 0; y < H; ++y)
+        for (int x = 0; x < H; ++x)
+          for (int c = 0; c < C; ++c) {
+            const int Y = y + 1, X = x + 1;
+            const size_t pl = (size_t)(c >> 3) * 4 + (Y & 1) * 2 + (X & 1);
+            out[(((size_t)i * H + y) * H + x) * C + c] =
+                ps[(pl * m->ps_plane[k] + (size_t)i * Gp * Gp + (Y >> 1) * Gp + (X >> 1)) * 8 + (c & 7)];
+          }
+    return FFSVA_OK;
+  }
   if (buf == -3 || buf == -4) {  // layers 6 / 7: unpack a slab layout (planes of 8 channels, 15x15 padded grid)
     const int C = buf == -3 ? 512 : 1024;
     std::vector<uint16_t> sl((size_t)C / 8 * m->slab_plane * 8);
@@ -561,6 +644,8 @@ FFSVA_API ffsva_status ffsva_tyolo_destroy(ffsva_tyolo* m) {
     cudaFree(m->d_w2v);
     cudaFree(m->d_slab[0]);
     cudaFree(m->d_slab[1]);
+    for (auto& p : m->d_ps) cudaFree(p);
+    for (auto& p : m->d_wps) cudaFree(p);
     cudaFree(m->d_raw);
     cudaFree(m->d_counts);
     cudaFree(m->d_frames);
