@@ -226,8 +226,8 @@ inline int64_t tyolo_pslab_plane(int32_t n, int32_t Gp) {
 struct TyPslabArgs {
   const __nv_bfloat16* in;   // parity slab, Cin channels, grid Gp
   int64_t plane;
-  __nv_bfloat16* out;        // next layer's parity slab (out_plane > 0, grid out_Gp) or NHWC [N][Gp-1][Gp-1][Cout]
-  int64_t out_plane;
+  __nv_bfloat16* out;        // next layer's parity slab (out_plane > 0, grid out_Gp > 0), 13x13 slab (out_plane > 0,
+  int64_t out_plane;         // out_Gp < 0; tyolo_slab_kernel's layout) or NHWC [N][Gp-1][Gp-1][Cout] (out_plane 0)
   int32_t out_Gp;
   const uint8_t* wpk;        // [N tile of 64][64-channel group][tap][8-channel K group][64 n][8] bf16
   const float* bias;

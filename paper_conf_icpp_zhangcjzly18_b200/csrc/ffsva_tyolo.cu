@@ -1099,7 +1099,12 @@ __global__ void __launch_bounds__(kPsThreads, 1) tyolo_pslab_kernel(TyPslabArgs 
           x1 = x1 < 0.f ? 0.1f * x1 : x1;
           w[k] = pack_bf16(x0, x1);
         }
-        if (a.out_plane > 0) {  // the next layer's parity slab (grid Go = Ho / 2 + 1)
+        if (a.out_plane > 0 && a.out_Gp < 0) {  // 13x13 slab layout of tyolo_slab_kernel (padded 15 x 15 grid)
+          const int64_t eo = f * 225 + (py + 1) * 15 + px + 1;
+          *reinterpret_cast<uint4*>(a.out + ((int64_t)(co >> 3) * a.out_plane + eo) * 8) = make_uint4(w[0], w[1], w[2], w[3]);
+          *reinterpret_cast<uint4*>(a.out + ((int64_t)((co >> 3) + 1) * a.out_plane + eo) * 8) =
+              make_uint4(w[4], w[5], w[6], w[7]);
+        } else if (a.out_plane > 0) {  // the next layer's parity slab (grid Go = Ho / 2 + 1)
           const int Go = a.out_Gp, Y = py + 1, X = px + 1;
           const int64_t eo = f * Go * Go + (Y >> 1) * Go + (X >> 1);
           const int par = (Y & 1) * 2 + (X & 1);

@@ -59,7 +59,8 @@ struct ffsva_tyolo {
   uint8_t* d_w1v = nullptr;        // layer 1 weights for the patch-view kernel (8 KB)
   __nv_bfloat16* d_pad2 = nullptr; // layer 1's planar zero-bordered output (layer 2's input), kTyL2PadBytes per frame
   uint8_t* d_w2v = nullptr;        // layer 2 weights for the patch-view kernel (64 KB)
-  __nv_bfloat16* d_slab[2] = {nullptr, nullptr};  // slab layouts of layer 7's (512 ch) and layer 8's (1024 ch) inputs
+  __nv_bfloat16* d_slab[3] = {nullptr, nullptr, nullptr};  // slab layouts of the inputs of layers 7 (512 ch), 8 (1024)
+                                                            // and 6 (256 ch)
   int64_t slab_plane = 0;          // entries per slab plane (fixed per workspace: the zero border must not move)
   __nv_bfloat16* d_ps[3] = {nullptr, nullptr, nullptr};  // parity slabs: inputs of layers 3, 4, 5
   int64_t ps_plane[3] = {0, 0, 0};
@@ -95,7 +96,7 @@ void build_layers(ffsva_tyolo* m) {
     L.conv_pool = L.pool == 1 ? 1 : 0;
     L.nq = L.conv_pool ? 4 : 1;
     L.NT = std::min(L.Cout_pad, L.conv_pool ? 128 : 256);
-    if (l == 6 || l == 7) L.NT = 128;  // layers 7 and 8 run on the slab kernel (N tile 128)
+    if (l >= 5 && l <= 7) L.NT = 128;  // layers 6, 7 and 8 run on the slab kernel (N tile 128)
     L.patch = L.conv_pool && L.Cp <= patch_cp ? 1 : 0;
     L.msub = L.conv_pool ? 1 : std::max(1, std::min(2, msub));
     if (L.patch) L.kchunks = 16 * L.Cp / 64 > 0 ? 16 * L.Cp / 64 : 1;  // 4x4 patch x Cp channels
@@ -168,8 +169,7 @@ ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
   cudaFree(m->d_act[1]);
   cudaFree(m->d_pad);
   cudaFree(m->d_pad2);
-  cudaFree(m->d_slab[0]);
-  cudaFree(m->d_slab[1]);
+  for (auto& p : m->d_slab) cudaFree(p);
   for (auto& p : m->d_ps) cudaFree(p);
   cudaFree(m->d_raw);
   cudaFree(m->d_counts);
@@ -194,8 +194,8 @@ ffsva_status ensure_workspace(ffsva_tyolo* m, int n) {
     e = cudaMalloc(&m->d_ps[k], bytes);
     if (e == cudaSuccess) e = cudaMemset(m->d_ps[k], 0, bytes);
   }
-  for (int k = 0; k < 2 && e == cudaSuccess; ++k) {
-    const size_t bytes = (size_t)(k == 0 ? 512 : 1024) / 8 * (size_t)m->slab_plane * 16;
+  for (int k = 0; k < 3 && e == cudaSuccess; ++k) {
+    const size_t bytes = (size_t)(k == 0 ? 512 : k == 1 ? 1024 : 256) / 8 * (size_t)m->slab_plane * 16;
     e = cudaMalloc(&m->d_slab[k], bytes);
     if (e == cudaSuccess) e = cudaMemset(m->d_slab[k], 0, bytes);
   }
@@ -290,9 +290,9 @@ ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, const int32_t*
       TyPslabArgs pa{};
       pa.in = m->d_ps[k];
       pa.plane = m->ps_plane[k];
-      pa.out = l < 4 ? m->d_ps[k + 1] : m->d_act[0];
-      pa.out_plane = l < 4 ? m->ps_plane[k + 1] : 0;
-      pa.out_Gp = l < 4 ? kPsGp[k + 1] : 0;
+      pa.out = l < 4 ? m->d_ps[k + 1] : m->d_slab[2];  // layer 5 writes layer 6's 13x13 slab input
+      pa.out_plane = l < 4 ? m->ps_plane[k + 1] : m->slab_plane;
+      pa.out_Gp = l < 4 ? kPsGp[k + 1] : -15;
       pa.wpk = m->d_wps[k];
       pa.bias = m->d_b + L.b_off;
       pa.N = n;
@@ -302,7 +302,28 @@ ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, const int32_t*
       if ((e = launch_tyolo_pslab(pa, ctx->num_sms, st)) != cudaSuccess)
         return cuda_fail(ctx, e, "T-YOLO parity-slab layer");
       g_launches += 1;
-      cur = l < 4 ? -10 - (k + 1) : 0;
+      cur = l < 4 ? -10 - (k + 1) : -5;  // -5: slab 2 (layer 5's output)
+      if (ev) cudaEventRecord(ev[2 + l], st);
+      continue;
+    }
+    if (l == 5) {  // 13x13 layer 6 by slab views (slab 2 -> NHWC), then its 2x2/1 max-pool (Q30) into slab 0
+      const Layer& L = m->L[l];
+      TySlabArgs sa{};
+      sa.in = m->d_slab[2];
+      sa.plane = m->slab_plane;
+      sa.out = m->d_act[1];
+      sa.out_plane = 0;
+      sa.wpk = m->d_w + L.w_off;
+      sa.bias = m->d_b + L.b_off;
+      sa.N = n;
+      sa.Cin = L.Cin;
+      sa.Cout = L.Cout_pad;
+      if ((e = launch_tyolo_slab(sa, ctx->num_sms, st)) != cudaSuccess) return cuda_fail(ctx, e, "T-YOLO slab layer");
+      if ((e = launch_tyolo_pool_s1(m->d_act[1], m->d_slab[0], n, L.Ho, L.Cout_pad, m->slab_plane, st)) !=
+          cudaSuccess)
+        return cuda_fail(ctx, e, "T-YOLO 2x2/1 pool");
+      g_launches += 2;
+      cur = -3;  // -3: slab 0 (layer 6's pooled output)
       if (ev) cudaEventRecord(ev[2 + l], st);
       continue;
     }
@@ -564,10 +585,10 @@ FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_fram
           }
     return FFSVA_OK;
   }
-  if (buf == -3 || buf == -4) {  // layers 6 / 7: unpack a slab layout (planes of 8 channels, 15x15 padded grid)
-    const int C = buf == -3 ? 512 : 1024;
+  if (buf == -3 || buf == -4 || buf == -5) {  // layers 6 / 7 / 5: unpack a 13x13 slab (planes of 8 channels)
+    const int si = buf == -3 ? 0 : buf == -4 ? 1 : 2, C = si == 0 ? 512 : si == 1 ? 1024 : 256;
     std::vector<uint16_t> sl((size_t)C / 8 * m->slab_plane * 8);
-    e = cudaMemcpyAsync(sl.data(), m->d_slab[buf == -3 ? 0 : 1], sl.size() * 2, cudaMemcpyDeviceToHost, cs);
+    e = cudaMemcpyAsync(sl.data(), m->d_slab[si], sl.size() * 2, cudaMemcpyDeviceToHost, cs);
     if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
     if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_tyolo_layer_output");
     for (int i = 0; i < n; ++i)
@@ -642,8 +663,7 @@ FFSVA_API ffsva_status ffsva_tyolo_destroy(ffsva_tyolo* m) {
     cudaFree(m->d_w1v);
     cudaFree(m->d_pad2);
     cudaFree(m->d_w2v);
-    cudaFree(m->d_slab[0]);
-    cudaFree(m->d_slab[1]);
+    for (auto& p : m->d_slab) cudaFree(p);
     for (auto& p : m->d_ps) cudaFree(p);
     for (auto& p : m->d_wps) cudaFree(p);
     cudaFree(m->d_raw);
