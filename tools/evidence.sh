@@ -1,6 +1,7 @@
 #!/bin/bash
-# Round evidence on one B200: GPU tests, smoke, default bench (M2) + M3 / SNM / T-YOLO configs, ncu launch lists and
-# --set full captures (K1 M2/M3, K4, T-YOLO layers), sanitizers. Everything lands in gpurun_out/;
+# Round evidence on one B200: GPU tests, smoke, the default bench (M2 + paced online ladders), a bench line per
+# SURVEY §8(d) config (M1, M3, M4 sweep, M5) plus the SNM and T-YOLO stages, the reference arm, ncu launch lists and
+# --set full captures (K1 M2/M3, K4, T-YOLO view kernels), sanitizers. Everything lands in gpurun_out/;
 # tools/summarize_evidence.py turns it into profiles/<round>/.
 cd "$(dirname "$0")/.."
 mkdir -p gpurun_out
@@ -8,11 +9,13 @@ nvidia-smi > gpurun_out/nvidia-smi.txt 2>&1
 timeout 600 python __graft_entry__.py > gpurun_out/build.log 2>&1 || { echo BUILD FAILED; tail -30 gpurun_out/build.log; exit 1; }
 timeout 1500 python -m pytest tests -m gpu -q > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/pytest_gpu.log
 timeout 300 python __graft_entry__.py smoke > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"; tail -1 gpurun_out/smoke.log
-timeout 1500 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?"
-for CFG in m3 snm tyolo; do
+timeout 1800 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?"
+for CFG in m1 m3 m4_1 m4_10 m4_50 m5 snm tyolo; do
   timeout 900 python bench.py --config $CFG --steps ${STEPS:-200} --warmup 5 --online "" > gpurun_out/bench_$CFG.json 2> gpurun_out/bench_$CFG.err
   echo "bench $CFG rc=$?"
 done
+timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/bench_reference.json 2> gpurun_out/bench_reference.err
+echo "reference rc=$?"; cat gpurun_out/bench_reference.json | cut -c1-300
 for CFG in m2 m3; do
   timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"sdd|compact|snm" -s 60 -c 60 --csv \
     --log-file gpurun_out/launches_${CFG}.csv \
@@ -27,7 +30,13 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:snm_
 echo "ncu full k4 rc=$?"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:tyolo --csv --log-file gpurun_out/launches_tyolo.csv \
   python tools/tyolo_profile.py --frames 256 --iters 1 > /dev/null 2>&1; echo "ncu list tyolo rc=$?"
-LAYERS="1 2 8" bash tools/tyolo_ncu.sh
+# one capture per T-YOLO view kernel (profile run: 2 warm-up passes + 1; skip the warm-up launches of each kernel)
+for K in "tyolo_l1:2:l1" "tyolo_l2:2:l2" "tyolo_pslab:6:pslab_L3" "tyolo_slab:8:slab_L8" "tyolo_resize:2:resize"; do
+  IFS=: read KN SKIP NAME <<< "$K"
+  timeout 600 ncu --set full --clock-control none --import-source on -k regex:$KN -s $SKIP -c 1 -o gpurun_out/prof_tyolo_$NAME -f \
+    python tools/tyolo_profile.py --frames 256 --iters 1 > gpurun_out/ncu_tyolo_$NAME.log 2>&1
+  echo "ncu full $NAME rc=$?"
+done
 timeout 300 python tools/tyolo_profile.py --frames 256 --iters 10 > gpurun_out/tyolo_profile.log 2>&1
 for tool in memcheck synccheck racecheck; do
   timeout ${SAN_TIMEOUT:-1200} compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_run.py > gpurun_out/sanitize_$tool.log 2>&1

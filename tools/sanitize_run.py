@@ -1,4 +1,5 @@
-"""Small run through every kernel path (K1 bulk + stream variants, K3, K4, reference, online scheduler) for
+"""Small run through every kernel path (K1 bulk + stream variants, K2, K3, K4, reference, T-YOLO view kernels, online
+scheduler in synchronous and pipelined mode) for
 compute-sanitizer (memcheck / racecheck / synccheck / initcheck). Prints OK at the end."""
 import os
 import sys
@@ -60,6 +61,14 @@ def main():
     sched.set_tyolo(ty, num_tyolo=1)
     for t in range(6):
         sched.push([(streams[i % 2], d[i], i) for i in range(8)])
+        sched.tick(s)
+    sched.destroy()
+    # pipelined ticks (ffsva_sched_set_pipeline): kernels of cycle k overlap the host half of cycle k + 1
+    sched = Scheduler(ctx, max_frames_per_tick=4, snm_slots=16)
+    sched.set_pipeline(True)
+    for t in range(8):
+        if t < 6:
+            sched.push([(streams[i % 2], d[i], i) for i in range(8)])
         sched.tick(s)
     sched.destroy()
     ty.destroy()

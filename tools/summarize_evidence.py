@@ -28,6 +28,8 @@ OUT = os.path.join(ROOT, "gpurun_out")
 
 def short(name):
     for k, v in (("tyolo_conv", "K5 tyolo_conv"), ("tyolo_resize", "K5 tyolo_resize"), ("tyolo_pool", "K5 tyolo_pool_s1"),
+                 ("tyolo_l1", "K5a tyolo_l1"), ("tyolo_l2", "K5b tyolo_l2"), ("tyolo_pslab", "K5c tyolo_pslab"),
+                 ("tyolo_slab", "K5d tyolo_slab"),
                  ("sdd_prev", "K2 sdd_prev"), ("ref_update", "K2b ref_update"), ("sdd", "K1 sdd"),
                  ("compact", "K3 compact"), ("snm", "K4 snm")):
         if k in name:
@@ -61,9 +63,10 @@ def main():
     rnd = sys.argv[1] if len(sys.argv) > 1 else "r01"
     dst = os.path.join(ROOT, "profiles", rnd)
     os.makedirs(dst, exist_ok=True)
-    for f in ["bench.json", "bench.err", "bench_m3.json", "bench_snm.json", "bench_tyolo.json", "tyolo_profile.json",
-              "tyolo_profile.log", "pytest_gpu.log", "smoke.log", "nvidia-smi.txt"] + \
-            [os.path.basename(p) for p in glob.glob(os.path.join(OUT, "sanitize_*.log"))]:
+    for f in ["bench.json", "bench.err", "bench_reference.json", "tyolo_profile.json", "tyolo_profile.log",
+              "pytest_gpu.log", "smoke.log", "nvidia-smi.txt"] + \
+            [os.path.basename(p) for p in glob.glob(os.path.join(OUT, "sanitize_*.log"))] + \
+            [os.path.basename(p) for p in glob.glob(os.path.join(OUT, "bench_*.json"))]:
         p = os.path.join(OUT, f)
         if os.path.exists(p):
             shutil.copy(p, os.path.join(dst, f))
