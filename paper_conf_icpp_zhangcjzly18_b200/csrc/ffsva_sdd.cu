@@ -12,7 +12,8 @@
 //  * sdd_bulk_kernel (rows 16-B aligned, one 100-grid row fits in shared memory — every workload of the
 //    benchmark): one CTA per (frame, 100-grid row), CTA pairs form thread-block clusters. One thread issues
 //    cp.async.bulk copies (TMA engine, L2 evict-first) of the row's source rows into shared memory against an
-//    mbarrier, so the SM's whole share of the frame is in flight without tying up registers; column sums are
+//    mbarrier, so the SM's whole share of the frame is in flight without tying up registers (the row of R is
+//    copied into shared memory by the other threads meanwhile, off the cell phase's critical path); column sums are
 //    packed 2x16-bit SIMD adds of 16-byte shared loads; the odd CTA of a pair pushes its horizontal 2-cell sums
 //    into the even CTA's shared memory with st.async (DSMEM, mbarrier transaction completion, no fence) and
 //    the even CTA emits the D50 row from the four 100-cell sums.
@@ -99,40 +100,6 @@ __device__ __forceinline__ uint32_t cell_sum_n(const uint16_t* col, int x0, int 
   for (int k = 0; k < N; ++k)
     if (k < w) s += p[3 * k];
   return s;
-}
-
-// All three channel sums of one 100-grid cell whose interleaved u16 column sums occupy [u0, u1) of colsum
-// (u0 = 3*x0, u1 = 3*x1), read as packed u32 words. u16 index u has channel u % 3, so word k = (2k, 2k+1)
-// carries channels (0,1), (2,0), (1,2) for k % 3 = 0, 1, 2: three packed accumulators by word class, then
-// ch0 = lo(S0) + hi(S1), ch1 = hi(S0) + lo(S2), ch2 = lo(S1) + hi(S2). The caller guarantees no 16-bit lane
-// overflows ((x1 - x0 + 2) * rows * 255 / 2 < 65536).
-__device__ __forceinline__ void cell_sum3_packed(const uint32_t* cw, int u0, int u1, uint32_t& c0, uint32_t& c1,
-                                                 uint32_t& c2) {
-  const int k0 = u0 >> 1, k1 = (u1 + 1) >> 1;  // words [k0, k1)
-  uint32_t a = 0, b = 0, c = 0;                // classes (k0 + 0, 1, 2) % 3
-  int k = k0;
-  for (; k + 3 <= k1; k += 3) {
-    a += cw[k];
-    b += cw[k + 1];
-    c += cw[k + 2];
-  }
-  if (k < k1) a += cw[k];
-  if (k + 1 < k1) b += cw[k + 1];
-  if (u0 & 1) a -= cw[k0] & 0xFFFFu;  // first word: its low half belongs to the previous cell
-  if (u1 & 1) {                        // last word: its high half belongs to the next cell
-    const uint32_t hi = cw[k1 - 1] & 0xFFFF0000u;
-    const int j = (k1 - 1 - k0) % 3;
-    if (j == 0) a -= hi;
-    else if (j == 1) b -= hi;
-    else c -= hi;
-  }
-  const int cls = k0 % 3;  // rotate (a, b, c) to word classes (S0, S1, S2)
-  const uint32_t S0 = cls == 0 ? a : (cls == 1 ? c : b);
-  const uint32_t S1 = cls == 0 ? b : (cls == 1 ? a : c);
-  const uint32_t S2 = cls == 0 ? c : (cls == 1 ? b : a);
-  c0 = (S0 & 0xFFFFu) + (S1 >> 16);
-  c1 = (S0 >> 16) + (S2 & 0xFFFFu);
-  c2 = (S1 & 0xFFFFu) + (S2 >> 16);
 }
 
 // floor(a / n) for a < 2^31 and a quotient below 2^16 (box means: <= 255), without the ~20-instruction integer
@@ -317,19 +284,31 @@ constexpr int kBulkThreads = 256;  // block size for rows of > 128 16-byte chunk
                                    // (360p: twice the resident CTAs per SM for small per-CTA byte counts)
 constexpr int kBulkMaxStage = 160 * 1024;  // larger rows (e.g. 4K) take the register-streaming kernel
 
-template <bool kD100>
 #ifndef FFSVA_K1_MINBLOCKS
 #define FFSVA_K1_MINBLOCKS 6  // 6 CTAs/SM: caps registers at 40 (A/B knob)
+#endif
+#ifndef FFSVA_K1_REFPRE
+#define FFSVA_K1_REFPRE 1     // R row staged in shared memory during the bulk copy (A/B knob)
 #endif
 #ifndef FFSVA_K1_CELL16
 #define FFSVA_K1_CELL16 1     // cell sums unrolled to 16 (cells <= 16 px) instead of 24 (A/B knob)
 #endif
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_K1_MINBLOCKS)
+#ifndef FFSVA_K1_MINB128
+#define FFSVA_K1_MINB128 16   // 128-thread CTAs (rows of <= 128 chunks, e.g. 360p): 16 CTAs/SM, 32 registers (A/B knob)
+#endif
+// kNT threads per CTA; each thread owns kNT == 256 ? 2 : 1 16-byte chunks of the row. 320 (720p) and 384 (1080p)
+// threads give every thread at most one chunk and one 100-grid value, so no warp runs a second cell iteration while
+// the others wait at the barrier that follows.
+template <int kNT>
+struct K1Occ { static constexpr int v = kNT == 128 ? FFSVA_K1_MINB128 : kNT == 384 ? 3 : FFSVA_K1_MINBLOCKS; };
+template <bool kD100, int kNT>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kNT, K1Occ<kNT>::v)
     sdd_bulk_kernel(SddArgs a) {
+  constexpr int kCh = kNT == 256 ? 2 : 1;
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t bar_data;   // this row's source bytes have landed
   __shared__ __align__(8) uint64_t bar_pair;   // (even CTA) the odd CTA's 2-cell sums have landed
-  __shared__ uint32_t red[kBulkThreads / 32];
+  __shared__ uint32_t red[kNT / 32];
   const int sdd_w = a.sdd_w, sdd_h = a.sdd_h;
   const int f = blockIdx.y;              // frame (launches of > 65535 frames are split on the host)
   const int r = blockIdx.x;              // 100-grid row; the cluster pairs rows 2b and 2b+1
@@ -348,6 +327,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   uint32_t* cell = reinterpret_cast<uint32_t*>(smem + a.stage_bytes);  // [3*sdd_w]
   uint32_t* pair_in = cell + 3 * sdd_w;                                // [half3]
   int* xb = reinterpret_cast<int*>(pair_in + half3);                   // [sdd_w + 1]
+  uint8_t* ref_s = reinterpret_cast<uint8_t*>(xb + sdd_w + 1);         // [3*sdd_w] this row of R
   const uint32_t bar_d = (uint32_t)__cvta_generic_to_shared(&bar_data);
   const uint32_t bar_p = (uint32_t)__cvta_generic_to_shared(&bar_pair);
 
@@ -375,16 +355,30 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   } else {
     fill_xbounds(xb, W, sdd_w);
   }
+#if FFSVA_K1_REFPRE
+  // this row of R into shared memory while the bulk copy is in flight: the cell phase then reads it at shared
+  // latency instead of one dependent L2 round trip per loop iteration (which kept the stage occupied)
+  {
+    const uint8_t* rrow = fd.ref + (int64_t)r * (3 * sdd_w);
+    const int n3 = 3 * sdd_w;
+    if ((((uintptr_t)rrow) & 3) == 0 && (n3 & 3) == 0) {
+      for (int i = threadIdx.x; i < (n3 >> 2); i += blockDim.x)
+        reinterpret_cast<uint32_t*>(ref_s)[i] = __ldg(reinterpret_cast<const uint32_t*>(rrow) + i);
+    } else {
+      for (int i = threadIdx.x; i < n3; i += blockDim.x) ref_s[i] = __ldg(rrow + i);
+    }
+  }
+#endif
   __syncthreads();
   mbar_wait_parity(bar_d, 0);
 
   // ---- column sums of the row's source rows (<= 2 16-byte chunks per thread)
-  uint32_t acc[2][8];
+  uint32_t acc[kCh][8];
 #pragma unroll
-  for (int k = 0; k < 2; ++k) {
+  for (int k = 0; k < kCh; ++k) {
 #pragma unroll
     for (int j = 0; j < 8; ++j) acc[k][j] = 0u;
-    const int c = threadIdx.x + k * (int)blockDim.x;
+    const int c = threadIdx.x + k * kNT;
     if (c < nchunk) {
       const uint8_t* p = smem + 16 * c;
       int y = 0;
@@ -396,8 +390,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
   __syncthreads();  // the stage is consumed; its first 2*rb16 bytes now hold the u16 column sums
   uint16_t* colsum = reinterpret_cast<uint16_t*>(smem);
 #pragma unroll
-  for (int k = 0; k < 2; ++k) {
-    const int c = threadIdx.x + k * (int)blockDim.x;
+  for (int k = 0; k < kCh; ++k) {
+    const int c = threadIdx.x + k * kNT;
     if (c < nchunk) store_colsum(reinterpret_cast<uint32_t*>(colsum), c, acc[k]);
   }
   __syncthreads();
@@ -415,7 +409,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kBulkThreads, FFSVA_
     const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)rows;
     const uint32_t d = box_mean(s, n);
     if (kD100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)r * row3 + o] = (uint8_t)d;
+#if FFSVA_K1_REFPRE
+    const int diff = (int)d - (int)ref_s[o];
+#else
     const int diff = (int)d - (int)__ldg(fd.ref + (int64_t)r * row3 + o);
+#endif
     ssd_local += dist_term(diff, fd.metric);
   }
   if (fd.mode == kRefPrevious) ssd_local = 0;  // K2 measures against the previous frame's D100
@@ -541,7 +539,7 @@ int sdd_threads(int max_chunks) {
 }
 
 size_t sdd_bulk_smem_bytes(int stage_bytes, int sdd_w) {
-  return (size_t)stage_bytes + (size_t)4 * (3 * sdd_w + 3 * (sdd_w / 2) + sdd_w + 1);
+  return (size_t)stage_bytes + (size_t)4 * (3 * sdd_w + 3 * (sdd_w / 2) + sdd_w + 1) + (size_t)((3 * sdd_w + 3) & ~3);
 }
 
 int sdd_bulk_stage_bytes(int W, int H, int sdd_h) {
@@ -583,6 +581,33 @@ void sdd_plan_apply(const SddPlan& p, SddArgs& a) {
   a.stage_bytes = p.stage_bytes;
 }
 
+template <int kNT>
+cudaError_t k1_set_smem(int smem) {
+  cudaError_t e = cudaFuncSetAttribute(sdd_bulk_kernel<true, kNT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(sdd_bulk_kernel<false, kNT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  return e;
+}
+
+template <int kNT>
+void k1_launch(const SddArgs& b, dim3 grid, size_t smem, cudaStream_t st) {
+  if (b.d100) sdd_bulk_kernel<true, kNT><<<grid, kNT, smem, st>>>(b);
+  else sdd_bulk_kernel<false, kNT><<<grid, kNT, smem, st>>>(b);
+}
+
+// Block size of the bulk kernel (FFSVA_K1_NT overrides, for A/B runs). Measured on B200 (profiles/r01/k1_ab.md):
+// rows of <= 128 chunks (360p) 128 threads; rows of 321..384 chunks (1080p: 360) 384 threads, one chunk and one
+// 100-grid value per thread (M3 0.93 -> 0.97 of the copy peak); otherwise (720p) 256 threads with two chunks per
+// thread (320 threads measured slower there: 0.77 vs 0.83).
+int k1_threads(int max_chunks, int sdd_w) {
+  const int need = std::max(max_chunks, 3 * sdd_w);
+  int nt = max_chunks <= 128 ? 128 : (max_chunks > 320 && need <= 384) ? 384 : 256;
+  if (const char* e = std::getenv("FFSVA_K1_NT")) {
+    const int v = std::atoi(e);
+    if ((v == 128 || v == 256 || v == 320 || v == 384) && max_chunks <= (v == 256 ? 2 : 1) * v) nt = v;
+  }
+  return nt;
+}
+
 cudaError_t sdd_configure(size_t smem) {
   static size_t configured = 0;
   if (smem <= configured) return cudaSuccess;
@@ -590,9 +615,10 @@ cudaError_t sdd_configure(size_t smem) {
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(sdd_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(sdd_bulk_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(sdd_bulk_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    e = k1_set_smem<128>((int)smem);
+  if (e == cudaSuccess) e = k1_set_smem<256>((int)smem);
+  if (e == cudaSuccess) e = k1_set_smem<320>((int)smem);
+  if (e == cudaSuccess) e = k1_set_smem<384>((int)smem);
   if (e == cudaSuccess) configured = smem;
   return e;
 }
@@ -612,9 +638,12 @@ cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st) {
       else b.d50 += (int64_t)f0 * a.d50_stride;
       if (b.d100) b.d100 += (int64_t)f0 * a.sdd_w * a.sdd_h * 3;
       const dim3 grid((unsigned)a.sdd_h, (unsigned)cnt);
-      const int nt = a.max_chunks <= kBulkThreads / 2 ? kBulkThreads / 2 : kBulkThreads;
-      if (b.d100) sdd_bulk_kernel<true><<<grid, nt, smem, st>>>(b);
-      else sdd_bulk_kernel<false><<<grid, nt, smem, st>>>(b);
+      switch (k1_threads(a.max_chunks, a.sdd_w)) {
+        case 128: k1_launch<128>(b, grid, smem, st); break;
+        case 320: k1_launch<320>(b, grid, smem, st); break;
+        case 384: k1_launch<384>(b, grid, smem, st); break;
+        default: k1_launch<256>(b, grid, smem, st); break;
+      }
     }
     return cudaGetLastError();
   }
