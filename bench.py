@@ -198,8 +198,13 @@ def run_ours(args, cfg, ws, rank, local):
         planted[j] = expect
     ctx.stats(reset=True)
 
+    # consecutive steps alternate over --streams CUDA streams (different prepared batches, own buffers): step i+1's
+    # K1 starts while step i's K1 tail, K3 and K4 still run (the per-stream statistics are order-independent atomics)
+    nstr = max(1, min(args.streams, nbatches))
+    css = [cs] + [torch.cuda.Stream(device=dev) for _ in range(nstr - 1)]
+
     def step(i):
-        batches[i % nbatches].launch(cs)
+        batches[i % nbatches].launch(css[i % nstr])
 
     for i in range(args.warmup):
         step(i)
@@ -216,8 +221,14 @@ def run_ours(args, cfg, ws, rank, local):
         dist.barrier()
     with torch.cuda.stream(cs):
         e0.record(cs)
+        for s2 in css[1:]:
+            s2.wait_event(e0)
         for i in range(args.steps):
             step(args.warmup + i)
+        for s2 in css[1:]:  # the timed region ends when every stream's last step is done
+            ev = torch.cuda.Event()
+            ev.record(s2)
+            cs.wait_event(ev)
         # a8 reporting: per-stream statistics to a device tensor, all-gathered over NCCL when sharded
         ffb.ffsva_stats_copy(local, stats_dev.data_ptr(), S, False, False, cs.cuda_stream)
         if ws > 1:
@@ -297,7 +308,7 @@ def run_ours(args, cfg, ws, rank, local):
                              % (frames_per_step * fbytes / 1e9),
                        "parallelism": f"stream-sharded x{ws} (weak: {S} streams per GPU)",
                        "batch_size": BATCH, "delta_diff": DELTA, "c_low": C_LOW, "c_high": C_HIGH,
-                       "filter_degree": FD, "seed": cfg["seed"]},
+                       "filter_degree": FD, "seed": cfg["seed"], "cuda_streams": nstr},
             "sustained_streams_30fps": int(value // 30),
             "sdd_pass_per_step": m_avg,
             "roofline": {"bound": "hbm", "kernel": "K1 sdd_kernel (ingest + box downsample + SSD + threshold)",
@@ -592,6 +603,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--config", default="m2", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--streams", type=int, default=2,
+                    help="CUDA streams the timed steps alternate over (consecutive batches overlap)")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--cpu-frames", type=int, default=480)
     ap.add_argument("--no-e2e", action="store_true")
