@@ -293,7 +293,7 @@ def run_ours(args, cfg, ws, rank, local):
     # ---- online validation of "sustained 30-FPS streams" (paced arrivals through the online runtime)
     online = None
     if args.online and args.config == "m2":
-        online = online_validation(args, ctx, video, sids, pool, value, dev, cs)
+        online = online_validation(args, ctx, video, sids, pool, value / ws, dev, cs, ws)
 
     out = None
     if rank == 0:
@@ -418,10 +418,15 @@ def run_tyolo(args, cfg, ws, rank, local):
     return out
 
 
-def online_validation(args, ctx, video, sids, pool, value, dev, cs):
+def online_validation(args, ctx, video, sids, pool, value, dev, cs, ws=1):
     """Paced 30-FPS streams through the online runtime (feedback queue + dynamic batching, §4.3).
-    Stream i replays content stream i % len(sids) of the pool with its own reference image and SNM."""
+    Stream i replays content stream i % len(sids) of the pool with its own reference image and SNM.
+
+    N > 1: every rank runs the same per-GPU counts on its own GPU at the same time (streams are sharded, no frame
+    crosses GPUs); a count is sustained only if it is sustained on every rank (all-reduce MIN of the verdicts, so
+    the ranks also climb their ladders in lock step), and the whole-job count is N x the per-GPU count."""
     import torch
+    import torch.distributed as dist
 
     from paper_conf_icpp_zhangcjzly18_b200.online import run_paced
     from synth import synth
@@ -478,6 +483,12 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs):
         res = run_paced(ctx, opened[:S], [pool[i % nc] for i in range(S)], pool.shape[1], args.online_seconds,
                         cuda_stream=cs, tyolo=ty if with_ty else None, tick_s=0.010 if S < 10000 else 0.025)
         res["stream_setup_s"] = setup_s
+        if ws > 1:
+            ok = torch.tensor([1 if res["sustained"] else 0], dtype=torch.int32, device=dev)
+            dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+            res["sustained_this_rank"] = res["sustained"]
+            res["sustained"] = bool(ok.item())
+            res["streams_per_gpu"], res["streams"] = S, S * ws
         results.append(res)
         if S in ladder and not with_ty and not res["sustained"]:
             ladder_failed = True
