@@ -296,15 +296,13 @@ constexpr int kBulkMaxStage = 160 * 1024;  // larger rows (e.g. 4K) take the reg
 #ifndef FFSVA_K1_MINB128
 #define FFSVA_K1_MINB128 16   // 128-thread CTAs (rows of <= 128 chunks, e.g. 360p): 16 CTAs/SM, 32 registers (A/B knob)
 #endif
-// kNT threads per CTA; each thread owns kNT == 256 ? 2 : 1 16-byte chunks of the row. 320 (720p) and 384 (1080p)
-// threads give every thread at most one chunk and one 100-grid value, so no warp runs a second cell iteration while
-// the others wait at the barrier that follows.
-template <int kNT>
-struct K1Occ { static constexpr int v = kNT == 128 ? FFSVA_K1_MINB128 : kNT == 384 ? 3 : FFSVA_K1_MINBLOCKS; };
-template <bool kD100, int kNT>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kNT, K1Occ<kNT>::v)
+// kNT threads per CTA, each owning up to kCh 16-byte chunks of the row; kMinB resident CTAs per SM (register cap).
+// Variants (k1_threads): 128/1/16 for rows of <= 128 chunks (360p); 256/1/7 for <= 256 chunks (720p: 32 registers
+// and a 33 KB footprint, so seven CTAs fit an SM); 384/1/3 for 1080p rows (one chunk and one 100-grid value per
+// thread); 256/2/6 for everything else up to 512 chunks.
+template <bool kD100, int kNT, int kCh, int kMinB>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kNT, kMinB)
     sdd_bulk_kernel(SddArgs a) {
-  constexpr int kCh = kNT == 256 ? 2 : 1;
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) uint64_t bar_data;   // this row's source bytes have landed
   __shared__ __align__(8) uint64_t bar_pair;   // (even CTA) the odd CTA's 2-cell sums have landed
@@ -324,8 +322,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kNT, K1Occ<kNT>::v)
   const int y1 = ytab ? __ldg(a.ybounds + r + 1) : (int)(((uint32_t)(r + 1) * (uint32_t)H) / (uint32_t)sdd_h);
   const int rows = y1 - y0;
   const int half3 = 3 * (sdd_w >> 1);
-  uint32_t* cell = reinterpret_cast<uint32_t*>(smem + a.stage_bytes);  // [3*sdd_w]
-  uint32_t* pair_in = cell + 3 * sdd_w;                                // [half3]
+  // cell sums live in the stage behind the column sums (written only after the stage is consumed; the host sizes the
+  // stage >= 2*rb16 + 12*sdd_w), which keeps a 720p CTA at 33 KB
+  uint32_t* cell = reinterpret_cast<uint32_t*>(smem + 2 * rb16);        // [3*sdd_w]
+  uint32_t* pair_in = reinterpret_cast<uint32_t*>(smem + a.stage_bytes);  // [half3]
   int* xb = reinterpret_cast<int*>(pair_in + half3);                   // [sdd_w + 1]
   uint8_t* ref_s = reinterpret_cast<uint8_t*>(xb + sdd_w + 1);         // [3*sdd_w] this row of R
   const uint32_t bar_d = (uint32_t)__cvta_generic_to_shared(&bar_data);
@@ -539,7 +539,7 @@ int sdd_threads(int max_chunks) {
 }
 
 size_t sdd_bulk_smem_bytes(int stage_bytes, int sdd_w) {
-  return (size_t)stage_bytes + (size_t)4 * (3 * sdd_w + 3 * (sdd_w / 2) + sdd_w + 1) + (size_t)((3 * sdd_w + 3) & ~3);
+  return (size_t)stage_bytes + (size_t)4 * (3 * (sdd_w / 2) + sdd_w + 1) + (size_t)((3 * sdd_w + 3) & ~3);
 }
 
 int sdd_bulk_stage_bytes(int W, int H, int sdd_h) {
@@ -566,7 +566,8 @@ void sdd_plan_finish(SddPlan& p, int32_t sdd_w, int32_t sdd_h) {
   const bool pair_ok = p.vec16 && sdd_bulk_ok(p.max_chunks, p.pair_stage);
   p.variant = pair_ok && !(force && !std::strcmp(force, "stream")) ? kSddPair : kSddStream;
   if (p.variant == kSddPair) {
-    p.stage_bytes = p.pair_stage;
+    // the stage also holds the u16 column sums (2*rb16) followed by the u32 cell sums (12*sdd_w) once consumed
+    p.stage_bytes = std::max(p.pair_stage, 32 * p.max_chunks + 12 * sdd_w);
     p.smem = sdd_bulk_smem_bytes(p.pair_stage, sdd_w);
   } else {
     p.stage_bytes = 0;
@@ -581,31 +582,35 @@ void sdd_plan_apply(const SddPlan& p, SddArgs& a) {
   a.stage_bytes = p.stage_bytes;
 }
 
-template <int kNT>
+template <int kNT, int kCh, int kMinB>
 cudaError_t k1_set_smem(int smem) {
-  cudaError_t e = cudaFuncSetAttribute(sdd_bulk_kernel<true, kNT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e == cudaSuccess) e = cudaFuncSetAttribute(sdd_bulk_kernel<false, kNT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaError_t e = cudaFuncSetAttribute(sdd_bulk_kernel<true, kNT, kCh, kMinB>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(sdd_bulk_kernel<false, kNT, kCh, kMinB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             smem);
   return e;
 }
 
-template <int kNT>
+template <int kNT, int kCh, int kMinB>
 void k1_launch(const SddArgs& b, dim3 grid, size_t smem, cudaStream_t st) {
-  if (b.d100) sdd_bulk_kernel<true, kNT><<<grid, kNT, smem, st>>>(b);
-  else sdd_bulk_kernel<false, kNT><<<grid, kNT, smem, st>>>(b);
+  if (b.d100) sdd_bulk_kernel<true, kNT, kCh, kMinB><<<grid, kNT, smem, st>>>(b);
+  else sdd_bulk_kernel<false, kNT, kCh, kMinB><<<grid, kNT, smem, st>>>(b);
 }
 
-// Block size of the bulk kernel (FFSVA_K1_NT overrides, for A/B runs). Measured on B200 (profiles/r01/k1_ab.md):
-// rows of <= 128 chunks (360p) 128 threads; rows of 321..384 chunks (1080p: 360) 384 threads, one chunk and one
-// 100-grid value per thread (M3 0.93 -> 0.97 of the copy peak); otherwise (720p) 256 threads with two chunks per
-// thread (320 threads measured slower there: 0.77 vs 0.83).
-int k1_threads(int max_chunks, int sdd_w) {
+// K1 variant (block size) for a batch, measured on B200 (profiles/r01/k1_ab.md): rows of <= 128 16-byte chunks
+// (360p) 128 threads; <= 256 chunks (720p) 256 threads with one chunk each at 7 CTAs/SM; 321..384 chunks (1080p)
+// 384 threads (one chunk and one 100-grid value per thread: M3 0.93 -> 0.99 of the copy peak); otherwise 256
+// threads with two chunks each. FFSVA_K1_NT = 128 / 256 / 384 / 2562 (256 threads, two chunks) overrides (A/B).
+int k1_variant(int max_chunks, int sdd_w) {
   const int need = std::max(max_chunks, 3 * sdd_w);
-  int nt = max_chunks <= 128 ? 128 : (max_chunks > 320 && need <= 384) ? 384 : 256;
+  int v = max_chunks <= 128 ? 128 : max_chunks <= 256 ? 256 : (need <= 384) ? 384 : 2562;
   if (const char* e = std::getenv("FFSVA_K1_NT")) {
-    const int v = std::atoi(e);
-    if ((v == 128 || v == 256 || v == 320 || v == 384) && max_chunks <= (v == 256 ? 2 : 1) * v) nt = v;
+    const int o = std::atoi(e);
+    const int cap = o == 2562 ? 512 : o;
+    if ((o == 128 || o == 256 || o == 384 || o == 2562) && max_chunks <= cap) v = o;
   }
-  return nt;
+  return v;
 }
 
 cudaError_t sdd_configure(size_t smem) {
@@ -615,10 +620,10 @@ cudaError_t sdd_configure(size_t smem) {
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(sdd_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e == cudaSuccess)
-    e = k1_set_smem<128>((int)smem);
-  if (e == cudaSuccess) e = k1_set_smem<256>((int)smem);
-  if (e == cudaSuccess) e = k1_set_smem<320>((int)smem);
-  if (e == cudaSuccess) e = k1_set_smem<384>((int)smem);
+    e = k1_set_smem<128, 1, FFSVA_K1_MINB128>((int)smem);
+  if (e == cudaSuccess) e = k1_set_smem<256, 1, 7>((int)smem);
+  if (e == cudaSuccess) e = k1_set_smem<256, 2, FFSVA_K1_MINBLOCKS>((int)smem);
+  if (e == cudaSuccess) e = k1_set_smem<384, 1, 3>((int)smem);
   if (e == cudaSuccess) configured = smem;
   return e;
 }
@@ -638,11 +643,11 @@ cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st) {
       else b.d50 += (int64_t)f0 * a.d50_stride;
       if (b.d100) b.d100 += (int64_t)f0 * a.sdd_w * a.sdd_h * 3;
       const dim3 grid((unsigned)a.sdd_h, (unsigned)cnt);
-      switch (k1_threads(a.max_chunks, a.sdd_w)) {
-        case 128: k1_launch<128>(b, grid, smem, st); break;
-        case 320: k1_launch<320>(b, grid, smem, st); break;
-        case 384: k1_launch<384>(b, grid, smem, st); break;
-        default: k1_launch<256>(b, grid, smem, st); break;
+      switch (k1_variant(a.max_chunks, a.sdd_w)) {
+        case 128: k1_launch<128, 1, FFSVA_K1_MINB128>(b, grid, smem, st); break;
+        case 256: k1_launch<256, 1, 7>(b, grid, smem, st); break;
+        case 384: k1_launch<384, 1, 3>(b, grid, smem, st); break;
+        default: k1_launch<256, 2, FFSVA_K1_MINBLOCKS>(b, grid, smem, st); break;
       }
     }
     return cudaGetLastError();

@@ -39,6 +39,7 @@ for K in "tyolo_l1:2:l1" "tyolo_l2:2:l2" "tyolo_pslab:6:pslab_L3" "tyolo_slab:8:
 done
 timeout 300 python tools/tyolo_profile.py --frames 256 --iters 10 > gpurun_out/tyolo_profile.log 2>&1
 for tool in memcheck synccheck racecheck; do
-  timeout ${SAN_TIMEOUT:-1200} compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_run.py > gpurun_out/sanitize_$tool.log 2>&1
+  ARGS=""; [ $tool = racecheck ] && ARGS="--no-tyolo"
+  timeout ${SAN_TIMEOUT:-1200} compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_run.py $ARGS > gpurun_out/sanitize_$tool.log 2>&1
   echo "sanitize $tool rc=$?"; tail -2 gpurun_out/sanitize_$tool.log
 done
