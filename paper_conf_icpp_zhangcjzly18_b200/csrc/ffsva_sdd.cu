@@ -568,7 +568,7 @@ void sdd_plan_finish(SddPlan& p, int32_t sdd_w, int32_t sdd_h) {
   if (p.variant == kSddPair) {
     // the stage also holds the u16 column sums (2*rb16) followed by the u32 cell sums (12*sdd_w) once consumed
     p.stage_bytes = std::max(p.pair_stage, 32 * p.max_chunks + 12 * sdd_w);
-    p.smem = sdd_bulk_smem_bytes(p.pair_stage, sdd_w);
+    p.smem = sdd_bulk_smem_bytes(p.stage_bytes, sdd_w);
   } else {
     p.stage_bytes = 0;
     p.smem = sdd_smem_bytes(p.max_chunks, sdd_w);
@@ -614,8 +614,14 @@ int k1_variant(int max_chunks, int sdd_w) {
 }
 
 cudaError_t sdd_configure(size_t smem) {
-  static size_t configured = 0;
-  if (smem <= configured) return cudaSuccess;
+  // per device (the attribute is set on the current device); it is an upper bound for every later launch there, so
+  // it never goes below the 48 KB default
+  static size_t configured[64] = {};
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (dev < 0 || dev >= 64) dev = 0;
+  smem = std::max(smem, (size_t)48 * 1024);
+  if (smem <= configured[dev]) return cudaSuccess;
   cudaError_t e = cudaFuncSetAttribute(sdd_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(sdd_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -624,7 +630,7 @@ cudaError_t sdd_configure(size_t smem) {
   if (e == cudaSuccess) e = k1_set_smem<256, 1, 7>((int)smem);
   if (e == cudaSuccess) e = k1_set_smem<256, 2, FFSVA_K1_MINBLOCKS>((int)smem);
   if (e == cudaSuccess) e = k1_set_smem<384, 1, 3>((int)smem);
-  if (e == cudaSuccess) configured = smem;
+  if (e == cudaSuccess) configured[dev] = smem;
   return e;
 }
 

@@ -358,3 +358,37 @@ def test_full_size_config2_sampled(env):
     pb.destroy()
     for c in cams:
         c.st.close()
+
+
+def test_k1_shared_memory_limit_in_fresh_process():
+    """Regression: the first K1 launch of a process with tiny frames (128x100: a 3 KB footprint) must not lower
+    the kernels' dynamic shared-memory limit below what later, larger frames need (and vice versa). Run in a
+    fresh process so no earlier test has configured the kernels."""
+    import subprocess
+    import sys
+    import os
+    code = r'''
+import sys, torch
+sys.path.insert(0, sys.argv[1])
+import numpy as np
+import paper_conf_icpp_zhangcjzly18_b200 as ff
+from synth import synth
+from oracle import oracle as orc
+dev = torch.device("cuda:0"); ctx = ff.Context(dev)
+for (W, H) in ((128, 100), (1280, 720), (128, 100), (1920, 1080)):
+    v = synth.Video(seed=9, width=W, height=H, period=4, on_len=2)
+    st = ctx.open_stream(width=W, height=H, delta_diff=0.0)
+    refs = synth.frames(v, [0], [0], ref=True)
+    st.set_reference(torch.from_numpy(refs).to(dev)); st.snm_load(synth.snm_weights(9, 0))
+    host = synth.frames(v, [0] * 3, [0, 1, 2])
+    d = torch.from_numpy(host).to(dev)
+    r = ctx.filter_batch([(st, d[i], i) for i in range(3)])
+    R = orc.reference(refs, W, 100, 100)
+    for i in range(3):
+        assert int(r["ssd"][i]) == orc.ssd(orc.box_downsample(host[i], W, 100, 100), R), (W, i)
+    st.close()
+print("OK")
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, "-c", code, root], capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0 and "OK" in out.stdout, out.stdout + out.stderr
