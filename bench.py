@@ -435,7 +435,7 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs, ws=1):
     for tok in args.online.split(","):
         tok = tok.strip()
         if tok == "auto":  # a ladder of fractions of the offline capacity, climbed until a count is not sustained
-            ladder = [max(31, int(f * value / 30)) for f in (0.55, 0.7, 0.85, 0.95)]
+            ladder = [max(31, int(f * value / 30)) for f in (0.55, 0.7, 0.85, 0.9, 0.95)]
         elif tok:
             counts.append(int(tok))
     nc = len(sids)
@@ -451,7 +451,7 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs, ws=1):
     for tok in args.online_tyolo.split(","):
         tok = tok.strip()
         if tok == "auto":  # T-YOLO (~55 K frames/s) sees the SNM survivors, a few % of the frames at TOR 10 %:
-            ty_ladder = [max(31, int(f * value / 30)) for f in (0.1, 0.2, 0.3, 0.4)]  # climbed like the SDD+SNM one
+            ty_ladder = [max(31, int(f * value / 30)) for f in (0.1, 0.2, 0.3, 0.4, 0.5)]  # climbed like SDD+SNM's
         elif tok:
             ty_counts.append(int(tok))
     results = []
@@ -622,12 +622,12 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--online", default="30,auto",
                     help="comma-separated stream counts for the paced online validation (config m2); 'auto' = "
-                         "a ladder of 55/70/85/95%% of the measured frames/s / 30, climbed until a count is not "
+                         "a ladder of 55/70/85/90/95%% of the measured frames/s / 30, climbed until a count is not "
                          "sustained; empty to skip")
     ap.add_argument("--online-seconds", type=float, default=4.0)
     ap.add_argument("--online-tyolo", default="2000,auto",
                     help="stream counts for a paced run of the full cascade with the T-YOLO stage (f1); 'auto' = "
-                         "a ladder of 10/20/30/40%% of the measured frames/s / 30; empty to skip")
+                         "a ladder of 10/20/30/40/50%% of the measured frames/s / 30; empty to skip")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
