@@ -445,6 +445,119 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kNT, kMinB)
   ssd_commit(ssd_local, red, a, f, fd.slot, r == 0);
 }
 
+// ------------------------------------------------------------------ narrow rows: both rows of a pair in one CTA
+// For rows of <= 128 16-byte chunks (360p) the CTA-pair kernel's CTAs are short-lived enough that cluster dispatch
+// limits residency (ncu, M1: 38 % of warps active against 100 % possible). This variant gives one 256-thread CTA
+// both 100-grid rows 2b, 2b+1 of a 50-grid row: one bulk copy of their contiguous source rows, threads 0-127 take
+// row 2b and 128-255 row 2b+1 through the column and cell phases, and the D50 row is formed in shared memory (no
+// cluster, no DSMEM). Shared memory: stage (>= 4*rb16 + 24*sdd_w: the two u16 column-sum rows, then the u32 cell
+// sums of both rows once the stage is consumed) | xb[sdd_w + 1] | both rows of R.
+__global__ void __launch_bounds__(256, 8) sdd_band2_kernel_impl(SddArgs a, bool d100) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ __align__(8) uint64_t bar_data;
+  __shared__ uint32_t red[8];
+  const int sdd_w = a.sdd_w, sdd_h = a.sdd_h;
+  const int f = blockIdx.y;
+  const int b = blockIdx.x;  // 50-grid row: 100-grid rows 2b, 2b+1
+  const FrameDesc fd = a.frames[f];
+  const int W = fd.W, H = fd.H;
+  const int rb16 = (3 * W + 15) & ~15;
+  const int nchunk = rb16 >> 4;
+  const bool ytab = a.ybounds != nullptr;
+  const int r0 = 2 * b;
+  const int y0 = ytab ? __ldg(a.ybounds + r0) : (int)(((uint32_t)r0 * (uint32_t)H) / (uint32_t)sdd_h);
+  const int ym = ytab ? __ldg(a.ybounds + r0 + 1) : (int)(((uint32_t)(r0 + 1) * (uint32_t)H) / (uint32_t)sdd_h);
+  const int y1 = ytab ? __ldg(a.ybounds + r0 + 2) : (int)(((uint32_t)(r0 + 2) * (uint32_t)H) / (uint32_t)sdd_h);
+  const int rows = y1 - y0;
+  const int row3 = 3 * sdd_w, half3 = 3 * (sdd_w >> 1);
+  uint32_t* cell = reinterpret_cast<uint32_t*>(smem + 4 * rb16);          // [2][row3], in the consumed stage
+  int* xb = reinterpret_cast<int*>(smem + a.stage_bytes);                 // [sdd_w + 1]
+  uint8_t* ref_s = reinterpret_cast<uint8_t*>(xb + sdd_w + 1);            // [2][row3]
+  const uint32_t bar_d = (uint32_t)__cvta_generic_to_shared(&bar_data);
+
+  if (threadIdx.x == 0) {
+    mbar_init_cta(bar_d, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    mbar_expect_tx(bar_d, (uint32_t)(rows * rb16));
+    const uint32_t dst = (uint32_t)__cvta_generic_to_shared(smem);
+    const uint8_t* src = fd.pixels + (int64_t)y0 * fd.pitch;
+    if (fd.pitch == rb16) {
+      bulk_g2s(dst, src, (uint32_t)(rows * rb16), bar_d, pol);
+    } else {
+      for (int y = 0; y < rows; ++y) bulk_g2s(dst + y * rb16, src + (int64_t)y * fd.pitch, (uint32_t)rb16, bar_d, pol);
+    }
+  }
+  if (a.xbounds) {
+    for (int i = threadIdx.x; i <= sdd_w; i += blockDim.x) xb[i] = __ldg(a.xbounds + i);
+  } else {
+    fill_xbounds(xb, W, sdd_w);
+  }
+  {  // both rows of R (contiguous) while the copy is in flight
+    const uint8_t* rrow = fd.ref + (int64_t)r0 * row3;
+    const int n6 = 2 * row3;
+    if ((((uintptr_t)rrow) & 3) == 0 && (n6 & 3) == 0) {
+      for (int i = threadIdx.x; i < (n6 >> 2); i += blockDim.x)
+        reinterpret_cast<uint32_t*>(ref_s)[i] = __ldg(reinterpret_cast<const uint32_t*>(rrow) + i);
+    } else {
+      for (int i = threadIdx.x; i < n6; i += blockDim.x) ref_s[i] = __ldg(rrow + i);
+    }
+  }
+  __syncthreads();
+  mbar_wait_parity(bar_d, 0);
+
+  // ---- column sums: threads 0-127 over row 2b's source rows, 128-255 over row 2b+1's
+  const int h = threadIdx.x >> 7, c = threadIdx.x & 127;
+  const int ylo = h ? ym - y0 : 0, yhi = h ? rows : ym - y0;
+  uint32_t acc[8];
+#pragma unroll
+  for (int j = 0; j < 8; ++j) acc[j] = 0u;
+  if (c < nchunk) {
+    const uint8_t* p = smem + 16 * c;
+    int y = ylo;
+    for (; y + 1 < yhi; y += 2)
+      acc16x2(acc, *reinterpret_cast<const uint4*>(p + y * rb16), *reinterpret_cast<const uint4*>(p + (y + 1) * rb16));
+    if (y < yhi) acc16(acc, *reinterpret_cast<const uint4*>(p + y * rb16));
+  }
+  __syncthreads();  // the stage is consumed: [h * 2*rb16, (h+1) * 2*rb16) now holds row h's u16 column sums
+  if (c < nchunk) store_colsum(reinterpret_cast<uint32_t*>(smem + h * 2 * rb16), c, acc);
+  __syncthreads();
+
+  // ---- 100-grid cells of both rows: D100, distance vs R
+  const int cellw = a.xbounds ? a.cellw : (W + sdd_w - 1) / sdd_w;
+  uint32_t ssd_local = 0;
+  for (int o = threadIdx.x; o < 2 * row3; o += blockDim.x) {
+    const int sub = o >= row3;
+    const int rr = o - sub * row3;
+    const int cx = rr / 3, ch = rr - 3 * cx;
+    const int x0 = xb[cx], x1 = xb[cx + 1];
+    const uint16_t* col = reinterpret_cast<const uint16_t*>(smem + sub * 2 * rb16) + ch;
+    const uint32_t sum = cell_sum_w(col, x0, x1, cellw);
+    cell[o] = sum;
+    const uint32_t n = (uint32_t)(x1 - x0) * (uint32_t)(sub ? y1 - ym : ym - y0);
+    const uint32_t d = box_mean(sum, n);
+    if (d100) a.d100[(int64_t)f * sdd_h * row3 + (int64_t)(r0 + sub) * row3 + rr] = (uint8_t)d;
+    ssd_local += dist_term((int)d - (int)ref_s[o], fd.metric);
+  }
+  if (fd.mode == kRefPrevious) ssd_local = 0;  // K2 measures against the previous frame's D100
+  __syncthreads();
+
+  // ---- D50 row from the four 100-cell sums of each 50-cell
+  {
+    const int64_t slot = a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f;
+    uint8_t* d50row = a.d50 + slot * a.d50_stride + (int64_t)b * half3;
+    for (int o = threadIdx.x; o < half3; o += blockDim.x) {
+      const int cx = o / 3, ch = o - 3 * cx;
+      const uint32_t sum = cell[6 * cx + ch] + cell[6 * cx + 3 + ch] + cell[row3 + 6 * cx + ch] +
+                           cell[row3 + 6 * cx + 3 + ch];
+      const uint32_t n = (uint32_t)(xb[2 * cx + 2] - xb[2 * cx]) * (uint32_t)rows;
+      d50row[o] = (uint8_t)box_mean(sum, n);
+    }
+  }
+  ssd_commit(ssd_local, red, a, f, fd.slot, b == 0);
+}
+
 // Reference image R: one rounding of the mean over k frames x box. One thread per value.
 __global__ void reference_kernel(const uint8_t* __restrict__ frames, int32_t k, int64_t frame_stride, int32_t W,
                                  int32_t H, int64_t pitch, int32_t sdd_w, int32_t sdd_h, uint8_t* __restrict__ out) {
@@ -560,6 +673,13 @@ void sdd_plan_add(SddPlan& p, int32_t W, int32_t H, int64_t pitch, const void* p
   if ((pitch & 15) || ((uintptr_t)pixels & 15)) p.vec16 = false;
 }
 
+int k1_variant(int max_chunks, int sdd_w);
+constexpr int kK1Band2 = 1282;  // k1_variant id of sdd_band2_kernel_impl
+
+size_t sdd_band2_smem_bytes(int stage_bytes, int sdd_w) {
+  return (size_t)stage_bytes + (size_t)4 * (sdd_w + 1) + (size_t)((6 * sdd_w + 3) & ~3);
+}
+
 void sdd_plan_finish(SddPlan& p, int32_t sdd_w, int32_t sdd_h) {
   (void)sdd_h;
   const char* force = std::getenv("FFSVA_SDD_KERNEL");
@@ -567,8 +687,13 @@ void sdd_plan_finish(SddPlan& p, int32_t sdd_w, int32_t sdd_h) {
   p.variant = pair_ok && !(force && !std::strcmp(force, "stream")) ? kSddPair : kSddStream;
   if (p.variant == kSddPair) {
     // the stage also holds the u16 column sums (2*rb16) followed by the u32 cell sums (12*sdd_w) once consumed
-    p.stage_bytes = std::max(p.pair_stage, 32 * p.max_chunks + 12 * sdd_w);
-    p.smem = sdd_bulk_smem_bytes(p.stage_bytes, sdd_w);
+    if (k1_variant(p.max_chunks, sdd_w) == kK1Band2) {  // two rows' sources; then 2 x column sums + 2 x cells
+      p.stage_bytes = std::max(2 * p.pair_stage, 64 * p.max_chunks + 24 * sdd_w);
+      p.smem = sdd_band2_smem_bytes(p.stage_bytes, sdd_w);
+    } else {
+      p.stage_bytes = std::max(p.pair_stage, 32 * p.max_chunks + 12 * sdd_w);
+      p.smem = sdd_bulk_smem_bytes(p.stage_bytes, sdd_w);
+    }
   } else {
     p.stage_bytes = 0;
     p.smem = sdd_smem_bytes(p.max_chunks, sdd_w);
@@ -601,14 +726,15 @@ void k1_launch(const SddArgs& b, dim3 grid, size_t smem, cudaStream_t st) {
 // K1 variant (block size) for a batch, measured on B200 (profiles/r01/k1_ab.md): rows of <= 128 16-byte chunks
 // (360p) 128 threads; <= 256 chunks (720p) 256 threads with one chunk each at 7 CTAs/SM; 321..384 chunks (1080p)
 // 384 threads (one chunk and one 100-grid value per thread: M3 0.93 -> 0.99 of the copy peak); otherwise 256
-// threads with two chunks each. FFSVA_K1_NT = 128 / 256 / 384 / 2562 (256 threads, two chunks) overrides (A/B).
+// threads with two chunks each. Rows of <= 128 chunks run sdd_band2_kernel_impl (both rows of a pair in one CTA).
+// FFSVA_K1_NT = 128 (CTA pairs) / 1282 (band of two) / 256 / 384 / 2562 (256 threads, two chunks) overrides (A/B).
 int k1_variant(int max_chunks, int sdd_w) {
   const int need = std::max(max_chunks, 3 * sdd_w);
-  int v = max_chunks <= 128 ? 128 : max_chunks <= 256 ? 256 : (need <= 384) ? 384 : 2562;
+  int v = max_chunks <= 128 ? kK1Band2 : max_chunks <= 256 ? 256 : (need <= 384) ? 384 : 2562;
   if (const char* e = std::getenv("FFSVA_K1_NT")) {
     const int o = std::atoi(e);
-    const int cap = o == 2562 ? 512 : o;
-    if ((o == 128 || o == 256 || o == 384 || o == 2562) && max_chunks <= cap) v = o;
+    const int cap = o == 2562 ? 512 : o == kK1Band2 ? 128 : o;
+    if ((o == 128 || o == 256 || o == 384 || o == 2562 || o == kK1Band2) && max_chunks <= cap) v = o;
   }
   return v;
 }
@@ -630,6 +756,7 @@ cudaError_t sdd_configure(size_t smem) {
   if (e == cudaSuccess) e = k1_set_smem<256, 1, 7>((int)smem);
   if (e == cudaSuccess) e = k1_set_smem<256, 2, FFSVA_K1_MINBLOCKS>((int)smem);
   if (e == cudaSuccess) e = k1_set_smem<384, 1, 3>((int)smem);
+  if (e == cudaSuccess) e = cudaFuncSetAttribute(sdd_band2_kernel_impl, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e == cudaSuccess) configured[dev] = smem;
   return e;
 }
@@ -637,7 +764,9 @@ cudaError_t sdd_configure(size_t smem) {
 cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st) {
   if (a.n <= 0) return cudaSuccess;
   if (a.bulk) {
-    const size_t smem = sdd_bulk_smem_bytes(a.stage_bytes, a.sdd_w);
+    const int v = k1_variant(a.max_chunks, a.sdd_w);
+    const size_t smem = v == kK1Band2 ? sdd_band2_smem_bytes(a.stage_bytes, a.sdd_w)
+                                      : sdd_bulk_smem_bytes(a.stage_bytes, a.sdd_w);
     // grid (row, frame); gridDim.y <= 65535, so very large batches take several launches
     for (int32_t f0 = 0; f0 < a.n; f0 += 65535) {
       SddArgs b = a;
@@ -649,7 +778,10 @@ cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st) {
       else b.d50 += (int64_t)f0 * a.d50_stride;
       if (b.d100) b.d100 += (int64_t)f0 * a.sdd_w * a.sdd_h * 3;
       const dim3 grid((unsigned)a.sdd_h, (unsigned)cnt);
-      switch (k1_variant(a.max_chunks, a.sdd_w)) {
+      switch (v) {
+        case kK1Band2:
+          sdd_band2_kernel_impl<<<dim3((unsigned)(a.sdd_h / 2), (unsigned)cnt), 256, smem, st>>>(b, b.d100 != nullptr);
+          break;
         case 128: k1_launch<128, 1, FFSVA_K1_MINB128>(b, grid, smem, st); break;
         case 256: k1_launch<256, 1, 7>(b, grid, smem, st); break;
         case 384: k1_launch<384, 1, 3>(b, grid, smem, st); break;
