@@ -290,6 +290,9 @@ constexpr int kBulkMaxStage = 160 * 1024;  // larger rows (e.g. 4K) take the reg
 #ifndef FFSVA_K1_REFPRE
 #define FFSVA_K1_REFPRE 1     // R row staged in shared memory during the bulk copy (A/B knob)
 #endif
+#ifndef FFSVA_K1_EARLYBAR
+#define FFSVA_K1_EARLYBAR 1   // CTA barrier right after the mbarrier init, not after the x-bounds / R-row loads (A/B knob)
+#endif
 #ifndef FFSVA_K1_CELL16
 #define FFSVA_K1_CELL16 1     // cell sums unrolled to 16 (cells <= 16 px) instead of 24 (A/B knob)
 #endif
@@ -349,6 +352,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kNT, kMinB)
   }
   // publish the peer's mbarrier before any remote st.async (relaxed: no memory fence needed beyond
   // fence.mbarrier_init); the matching wait comes right before the DSMEM exchange
+#if FFSVA_K1_EARLYBAR
+  __syncthreads();  // publishes the mbarrier init only; the xb / R-row writes below are ordered by later barriers
+#endif
   asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
   if (a.xbounds) {  // set only for uniform-width batches
     for (int i = threadIdx.x; i <= sdd_w; i += blockDim.x) xb[i] = __ldg(a.xbounds + i);
@@ -369,7 +375,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kNT, kMinB)
     }
   }
 #endif
+#if !FFSVA_K1_EARLYBAR
   __syncthreads();
+#endif
   mbar_wait_parity(bar_d, 0);
 
   // ---- column sums of the row's source rows (<= 2 16-byte chunks per thread)
@@ -489,6 +497,9 @@ __global__ void __launch_bounds__(256, 8) sdd_band2_kernel_impl(SddArgs a, bool 
       for (int y = 0; y < rows; ++y) bulk_g2s(dst + y * rb16, src + (int64_t)y * fd.pitch, (uint32_t)rb16, bar_d, pol);
     }
   }
+#if FFSVA_K1_EARLYBAR
+  __syncthreads();  // publishes the mbarrier init only; the xb / R-row writes below are ordered by later barriers
+#endif
   if (a.xbounds) {
     for (int i = threadIdx.x; i <= sdd_w; i += blockDim.x) xb[i] = __ldg(a.xbounds + i);
   } else {
@@ -504,7 +515,9 @@ __global__ void __launch_bounds__(256, 8) sdd_band2_kernel_impl(SddArgs a, bool 
       for (int i = threadIdx.x; i < n6; i += blockDim.x) ref_s[i] = __ldg(rrow + i);
     }
   }
+#if !FFSVA_K1_EARLYBAR
   __syncthreads();
+#endif
   mbar_wait_parity(bar_d, 0);
 
   // ---- column sums: threads 0-127 over row 2b's source rows, 128-255 over row 2b+1's
