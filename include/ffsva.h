@@ -221,7 +221,9 @@ FFSVA_API ffsva_status ffsva_stats_copy(int32_t device, uint64_t* dst, int32_t m
  *           queue pops min(BatchSize, depth) frames and the SNM scores all pops in one launch. Frames whose fate
  *           is decided (dropped by SDD, or scored by SNM) are reported as events, oldest first; events beyond
  *           `cap` are kept for the next tick. Synchronous on cuda_stream.
- * The SNM stage feeds T-YOLO in the paper, which is out of scope: nothing blocks it here. Frames must stay valid
+ * Without a T-YOLO model attached nothing blocks the SNM stage; with one (ffsva_sched_set_tyolo, f1) SNM survivors
+ * wait in per-stream T-YOLO queues and the SNM stage skips a stream whose T-YOLO queue is over q_tyolo (L209).
+ * push validates every frame's pixels as device memory of the scheduler's device. Frames must stay valid
  * until their event is reported. Streams must be open on the scheduler's device and carry a reference and an
  * SNM; a stream is attached on its first push and must not be closed while it has queued frames. */
 typedef struct ffsva_sched ffsva_sched;

@@ -407,6 +407,7 @@ FFSVA_API ffsva_status ffsva_stream_export(ffsva_stream* s, void* dst, int64_t c
   std::lock_guard<std::mutex> lk(ctx->mu);
   DeviceGuard g(ctx->device);
   if (!dst_is_host) {
+    begin_ptr_checks(ctx);
     ffsva_status cs = check_device_ptr(ctx, dst, (size_t)total);
     if (cs != FFSVA_OK) return cs;
   }

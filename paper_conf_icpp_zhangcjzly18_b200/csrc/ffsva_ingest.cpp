@@ -49,7 +49,7 @@ extern "C" FFSVA_API ffsva_status ffsva_filter_batch_host(const ffsva_frame* fra
     ctx->ring_bytes = 0;
     if ((e = cudaMalloc(&ctx->d_ring, need)) != cudaSuccess) return cuda_fail(nullptr, e, "cudaMalloc(ring)");
     ctx->ring_bytes = need;
-    ctx->ranges.clear();
+    clear_ptr_cache(ctx);
   }
   // descriptors point into the ring (slot reuse is ordered by events below)
   std::vector<ffsva_frame> staged(frames, frames + n);

@@ -102,13 +102,63 @@ void ctx_release(DeviceCtx* c) {
   delete c;
 }
 
-// A device pointer must lie inside a device allocation of the context's device. Allocation ranges are cached
-// so a batch of frames from one pool costs one driver query.
+// A device pointer must lie inside a device allocation of the context's device. Allocation ranges are cached:
+// within one validation epoch (one API call) a batch of frames from one pool costs one driver query; a cached
+// range is re-confirmed with the driver (same base and size) the first time a new epoch uses it.
+namespace {
+using GetRange = CUresult (*)(CUdeviceptr*, size_t*, CUdeviceptr);
+GetRange driver_get_range() {
+  // driver entry point fetched through the runtime, so the library does not link libcuda (it must load on
+  // GPU-less hosts, where every compute call then reports FFSVA_ECUDA)
+  static GetRange fn = [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) != cudaSuccess) f = nullptr;
+    return (GetRange)f;
+  }();
+  return fn;
+}
+}  // namespace
+
+void begin_ptr_checks(DeviceCtx* ctx) {
+  std::lock_guard<std::mutex> lk(ctx->ranges_mu);
+  ++ctx->range_epoch;
+}
+
+void clear_ptr_cache(DeviceCtx* ctx) {
+  std::lock_guard<std::mutex> lk(ctx->ranges_mu);
+  ctx->ranges.clear();
+  ctx->range_mru = 0;
+}
+
 ffsva_status check_device_ptr(DeviceCtx* ctx, const void* p, size_t bytes) {
   if (!p) return fail(FFSVA_EINVAL, "NULL frame pointer");
   const uintptr_t a = (uintptr_t)p;
-  for (auto& r : ctx->ranges)
-    if (a >= r.first && a + bytes <= r.first + r.second) return FFSVA_OK;
+  GetRange get_range = driver_get_range();
+  {
+    std::lock_guard<std::mutex> lk(ctx->ranges_mu);
+    auto& R = ctx->ranges;
+    auto hit = [&](size_t i) { return a >= R[i].base && a + bytes <= R[i].base + R[i].size; };
+    size_t i = ctx->range_mru < R.size() && hit(ctx->range_mru) ? ctx->range_mru : R.size();
+    for (size_t j = 0; i == R.size() && j < R.size(); ++j)
+      if (hit(j)) i = j;
+    if (i < R.size()) {
+      if (R[i].epoch == ctx->range_epoch) {
+        ctx->range_mru = i;
+        return FFSVA_OK;
+      }
+      CUdeviceptr base = 0;
+      size_t size = 0;
+      if (get_range && get_range(&base, &size, (CUdeviceptr)a) == CUDA_SUCCESS && (uintptr_t)base == R[i].base &&
+          size == R[i].size) {
+        R[i].epoch = ctx->range_epoch;
+        ctx->range_mru = i;
+        return FFSVA_OK;
+      }
+      R.erase(R.begin() + (std::ptrdiff_t)i);  // freed or re-allocated since it was cached: full check below
+      ctx->range_mru = 0;
+    }
+  }
   cudaPointerAttributes attr;
   cudaError_t e = cudaPointerGetAttributes(&attr, p);
   if (e != cudaSuccess) {
@@ -118,21 +168,14 @@ ffsva_status check_device_ptr(DeviceCtx* ctx, const void* p, size_t bytes) {
   if (attr.type != cudaMemoryTypeDevice && attr.type != cudaMemoryTypeManaged)
     return fail(FFSVA_EINVAL, "pixels must be device memory (use ffsva_filter_batch_host for host frames)");
   if (attr.device != ctx->device) return fail(FFSVA_EDEVICE, "frame pixels live on another device");
-  // driver entry point fetched through the runtime, so the library does not link libcuda (it must load on
-  // GPU-less hosts, where every compute call then reports FFSVA_ECUDA)
-  using GetRange = CUresult (*)(CUdeviceptr*, size_t*, CUdeviceptr);
-  static GetRange get_range = [] {
-    void* fn = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q) != cudaSuccess) fn = nullptr;
-    return (GetRange)fn;
-  }();
   CUdeviceptr base = 0;
   size_t size = 0;
   if (get_range && get_range(&base, &size, (CUdeviceptr)a) == CUDA_SUCCESS) {
     if (a + bytes > (uintptr_t)base + size) return fail(FFSVA_EINVAL, "frame extends past its allocation");
+    std::lock_guard<std::mutex> lk(ctx->ranges_mu);
     if (ctx->ranges.size() >= 64) ctx->ranges.erase(ctx->ranges.begin());
-    ctx->ranges.emplace_back((uintptr_t)base, size);
+    ctx->ranges.push_back({(uintptr_t)base, size, ctx->range_epoch});
+    ctx->range_mru = ctx->ranges.size() - 1;
   }
   return FFSVA_OK;
 }
@@ -343,6 +386,7 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
   const StreamState* s0 = frames[0].stream;
   const int32_t sdd_w = s0->desc.sdd_w, sdd_h = s0->desc.sdd_h;
   SddPlan plan;
+  begin_ptr_checks(ctx);
   for (int32_t i = 0; i < n; ++i) {
     const StreamState* s = frames[i].stream;
     if (s->desc.sdd_w != sdd_w || s->desc.sdd_h != sdd_h)

@@ -85,8 +85,19 @@ struct DeviceCtx {
   uint8_t* d_ring = nullptr;
   size_t ring_bytes = 0;
   cudaStream_t copy_stream = nullptr;
-  // known device allocations [base, base + size) on this device (pointer validation cache)
-  std::vector<std::pair<uintptr_t, size_t>> ranges;
+  // known device allocations [base, base + size) on this device (pointer validation cache). Guarded by its own
+  // mutex: the online runtime validates pushed frames under the scheduler's lock, not the device lock. An entry is
+  // trusted only within the validation epoch that last confirmed it with the driver (begin_ptr_checks starts an
+  // epoch per API call), so a range the caller freed or re-allocated since is looked up again.
+  struct Range {
+    uintptr_t base;
+    size_t size;
+    uint64_t epoch;
+  };
+  std::mutex ranges_mu;
+  std::vector<Range> ranges;
+  uint64_t range_epoch = 1;
+  size_t range_mru = 0;
 };
 
 // device context registry
@@ -95,6 +106,8 @@ void ctx_release(DeviceCtx* ctx);                       // decrements; destroys 
 
 // helpers
 ffsva_status check_device_ptr(DeviceCtx* ctx, const void* p, size_t bytes);
+void begin_ptr_checks(DeviceCtx* ctx);   // new validation epoch: cached ranges are re-confirmed once on next use
+void clear_ptr_cache(DeviceCtx* ctx);
 ffsva_status ensure_stats(DeviceCtx* ctx, int32_t slots);
 uint64_t exact_threshold(double delta, uint64_t n_values);
 uint64_t exact_threshold_sq(double delta, uint64_t q);  // floor(delta^2 * q), exact (NRMSE, Q24)

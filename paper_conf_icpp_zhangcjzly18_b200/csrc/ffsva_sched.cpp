@@ -444,9 +444,18 @@ FFSVA_API ffsva_status ffsva_sched_destroy(ffsva_sched* s) {
 FFSVA_API ffsva_status ffsva_sched_push(ffsva_sched* s, const ffsva_frame* frames, int32_t n, uint8_t* accepted) {
   if (!s || n < 0 || (n > 0 && (!frames || !accepted))) return fail(FFSVA_EINVAL, "bad argument");
   std::lock_guard<std::mutex> lk(s->mu);
+  begin_ptr_checks(s->ctx);
   for (int32_t i = 0; i < n; ++i) {  // validate everything before queueing anything
     ffsva_stream* st = frames[i].stream;
     if (!st || !frames[i].pixels) return fail(FFSVA_EINVAL, "frame without stream or pixels");
+    if (st->ctx != s->ctx) return fail(FFSVA_EDEVICE, "stream lives on another device");
+    // every frame's bytes must be device memory of this device (K1's bulk copies and the T-YOLO resize read them);
+    // the range cache makes this one lookup per frame after the first of each allocation
+    {
+      const ffsva_stream_desc& d = st->desc;
+      ffsva_status cs = check_device_ptr(s->ctx, frames[i].pixels, (size_t)(d.height - 1) * d.row_pitch + 3 * d.width);
+      if (cs != FFSVA_OK) return cs;
+    }
     // an attached stream passed every check below when it attached (its descriptor is immutable, and a reference
     // or SNM, once loaded, stays): consecutive frames of one stream are checked once
     if (i > 0 && st == frames[i - 1].stream) continue;

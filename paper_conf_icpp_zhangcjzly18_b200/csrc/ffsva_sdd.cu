@@ -28,6 +28,7 @@
 #include <cstring>
 
 #include "ffsva_internal.h"
+#include "ffsva_ptx.h"
 
 namespace cg = cooperative_groups;
 
@@ -245,40 +246,10 @@ __global__ void __launch_bounds__(512) sdd_kernel(SddArgs a) {
 }
 
 // ------------------------------------------------------------------ bulk-async (TMA engine) + cluster variant
-__device__ __forceinline__ void mbar_init_cta(uint32_t bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait_parity(uint32_t bar, uint32_t parity) {
-  uint32_t done = 0;
-  while (!done) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}\n"
-        : "=r"(done)
-        : "r"(bar), "r"(parity)
-        : "memory");
-  }
-}
-__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar, uint64_t pol) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::
-          "r"(dst),
-      "l"(src), "r"(bytes), "r"(bar), "l"(pol)
-      : "memory");
-}
-__device__ __forceinline__ uint32_t map_to_rank(uint32_t saddr, uint32_t rank) {
-  uint32_t r;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(saddr), "r"(rank));
-  return r;
-}
-// Remote store of one u32 into a cluster peer's shared memory, completing bytes on the peer's mbarrier.
-__device__ __forceinline__ void st_async_u32(uint32_t raddr, uint32_t v, uint32_t rbar) {
-  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b32 [%0], %1, [%2];" ::"r"(raddr), "r"(v),
-               "r"(rbar)
-               : "memory");
-}
+// PTX wrappers: ffsva_ptx.h
+using ptx::map_to_rank;
+using ptx::mbar_expect_tx;
+using ptx::st_async_u32;
 
 constexpr int kBulkThreads = 256;  // block size for rows of > 128 16-byte chunks; 128 threads for narrower rows
                                    // (360p: twice the resident CTAs per SM for small per-CTA byte counts)
@@ -335,8 +306,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kNT, kMinB)
   const uint32_t bar_p = (uint32_t)__cvta_generic_to_shared(&bar_pair);
 
   if (threadIdx.x == 0) {
-    mbar_init_cta(bar_d, 1);
-    mbar_init_cta(bar_p, 1);
+    ptx::mbar_init(bar_d, 1);
+    ptx::mbar_init(bar_p, 1);
     if (rank == 0) mbar_expect_tx(bar_p, (uint32_t)(4 * half3));  // our own arrival + the peer's bytes
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     uint64_t pol;
@@ -345,9 +316,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kNT, kMinB)
     const uint32_t dst = (uint32_t)__cvta_generic_to_shared(smem);
     const uint8_t* src = fd.pixels + (int64_t)y0 * fd.pitch;
     if (fd.pitch == rb16) {
-      bulk_g2s(dst, src, (uint32_t)(rows * rb16), bar_d, pol);
+      ptx::bulk_g2s_hint(dst, src, (uint32_t)(rows * rb16), bar_d, pol);
     } else {
-      for (int y = 0; y < rows; ++y) bulk_g2s(dst + y * rb16, src + (int64_t)y * fd.pitch, (uint32_t)rb16, bar_d, pol);
+      for (int y = 0; y < rows; ++y) ptx::bulk_g2s_hint(dst + y * rb16, src + (int64_t)y * fd.pitch, (uint32_t)rb16, bar_d, pol);
     }
   }
   // publish the peer's mbarrier before any remote st.async (relaxed: no memory fence needed beyond
@@ -378,7 +349,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kNT, kMinB)
 #if !FFSVA_K1_EARLYBAR
   __syncthreads();
 #endif
-  mbar_wait_parity(bar_d, 0);
+  ptx::mbar_wait(bar_d, 0);
 
   // ---- column sums of the row's source rows (<= 2 16-byte chunks per thread)
   uint32_t acc[kCh][8];
@@ -442,7 +413,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kNT, kMinB)
     const int yb = ytab ? __ldg(a.ybounds + r + 2) : (int)(((uint32_t)(r + 2) * (uint32_t)H) / (uint32_t)sdd_h);
     const int64_t slot = a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f;
     uint8_t* d50row = a.d50 + slot * a.d50_stride + (int64_t)(r >> 1) * half3;
-    mbar_wait_parity(bar_p, 0);
+    ptx::mbar_wait(bar_p, 0);
     for (int o = threadIdx.x; o < half3; o += blockDim.x) {
       const int cx = o / 3, ch = o - 3 * cx;
       const uint32_t s = cell[6 * cx + ch] + cell[6 * cx + 3 + ch] + pair_in[o];
@@ -484,7 +455,7 @@ __global__ void __launch_bounds__(256, 8) sdd_band2_kernel_impl(SddArgs a, bool 
   const uint32_t bar_d = (uint32_t)__cvta_generic_to_shared(&bar_data);
 
   if (threadIdx.x == 0) {
-    mbar_init_cta(bar_d, 1);
+    ptx::mbar_init(bar_d, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     uint64_t pol;
     asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
@@ -492,9 +463,9 @@ __global__ void __launch_bounds__(256, 8) sdd_band2_kernel_impl(SddArgs a, bool 
     const uint32_t dst = (uint32_t)__cvta_generic_to_shared(smem);
     const uint8_t* src = fd.pixels + (int64_t)y0 * fd.pitch;
     if (fd.pitch == rb16) {
-      bulk_g2s(dst, src, (uint32_t)(rows * rb16), bar_d, pol);
+      ptx::bulk_g2s_hint(dst, src, (uint32_t)(rows * rb16), bar_d, pol);
     } else {
-      for (int y = 0; y < rows; ++y) bulk_g2s(dst + y * rb16, src + (int64_t)y * fd.pitch, (uint32_t)rb16, bar_d, pol);
+      for (int y = 0; y < rows; ++y) ptx::bulk_g2s_hint(dst + y * rb16, src + (int64_t)y * fd.pitch, (uint32_t)rb16, bar_d, pol);
     }
   }
 #if FFSVA_K1_EARLYBAR
@@ -518,7 +489,7 @@ __global__ void __launch_bounds__(256, 8) sdd_band2_kernel_impl(SddArgs a, bool 
 #if !FFSVA_K1_EARLYBAR
   __syncthreads();
 #endif
-  mbar_wait_parity(bar_d, 0);
+  ptx::mbar_wait(bar_d, 0);
 
   // ---- column sums: threads 0-127 over row 2b's source rows, 128-255 over row 2b+1's
   const int h = threadIdx.x >> 7, c = threadIdx.x & 127;
@@ -593,30 +564,34 @@ __global__ void reference_kernel(const uint8_t* __restrict__ frames, int32_t k, 
 // of the batch). One CTA per frame; 16-byte loads of two L2-resident 30 KB images (K1 wrote them just before).
 constexpr int kPrevThreads = 256;
 __global__ void __launch_bounds__(kPrevThreads) sdd_prev_kernel(PrevArgs a) {
-  __shared__ uint32_t red[kPrevThreads / 32];
+  __shared__ unsigned long long red[kPrevThreads / 32];
   const int f = a.pairs[2 * blockIdx.x], prev = a.pairs[2 * blockIdx.x + 1];
   const FrameDesc& fd = a.frames[f];
   const uint8_t* x = a.d100 + (int64_t)f * a.n_values;
   const uint8_t* r = prev >= 0 ? a.d100 + (int64_t)prev * a.n_values : fd.ref;
   const bool sad = fd.metric == kDistSad;
-  uint32_t acc = 0;
+  // u64 sums: one CTA covers a whole frame, and grids up to 4096x4096 would wrap a 32-bit sum (a 16-byte chunk's
+  // partial, <= 16 * 255^2, is the only 32-bit quantity)
+  unsigned long long acc = 0;
   const int nv16 = a.n_values >> 4;  // n_values = 3*sdd_w*sdd_h, sdd_w and sdd_h even: a multiple of 4 only
   if ((a.n_values & 15) == 0) {
     for (int i = threadIdx.x; i < nv16; i += kPrevThreads) {
       const uint4 u = reinterpret_cast<const uint4*>(x)[i], v = reinterpret_cast<const uint4*>(r)[i];
       const uint32_t uw[4] = {u.x, u.y, u.z, u.w}, vw[4] = {v.x, v.y, v.z, v.w};
+      uint32_t part = 0;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
         if (sad) {
-          acc = __vsadu4(uw[k], vw[k]) + acc;
+          part = __vsadu4(uw[k], vw[k]) + part;
         } else {
 #pragma unroll
           for (int b = 0; b < 4; ++b) {
             const int d = (int)((uw[k] >> (8 * b)) & 255u) - (int)((vw[k] >> (8 * b)) & 255u);
-            acc += (uint32_t)(d * d);
+            part += (uint32_t)(d * d);
           }
         }
       }
+      acc += part;
     }
   } else {
     for (int i = threadIdx.x; i < a.n_values; i += kPrevThreads) acc += dist_term((int)x[i] - (int)r[i], fd.metric);

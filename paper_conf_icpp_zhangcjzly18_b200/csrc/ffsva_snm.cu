@@ -31,6 +31,7 @@
 #include <cuda_bf16.h>
 
 #include "ffsva_internal.h"
+#include "ffsva_ptx.h"
 
 namespace ffsva {
 namespace {
@@ -64,87 +65,8 @@ constexpr uint32_t kTmemCols = 256;
 constexpr int kTiles1 = 7;
 __constant__ int8_t c1_py0[kTiles1] = {0, 4, 8, 12, 16, 20, 21};  // last tile overlaps (idempotent writes)
 
-// ---------------------------------------------------------------- PTX wrappers (sm_100a)
-__device__ __forceinline__ uint32_t smem_addr(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-
-// UMMA shared-memory descriptor, K-major, SWIZZLE_NONE: start, leading (K) byte offset, stride (M/N) byte
-// offset, all >> 4; version 1 (bits 46-47) for sm_100.
-__device__ __forceinline__ uint64_t umma_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
-  return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) |
-         ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) | (1ull << 46);
-}
-
-// Instruction descriptor kind::f16: D fp32 (bits 4-5 = 1), A bf16 (7-9 = 1), B bf16 (10-12 = 1), both
-// K-major, N >> 3 at bits 17-22, M >> 4 at bits 24-28.
-__host__ __device__ constexpr uint32_t idesc_bf16(int M, int N) {
-  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
-}
-
-// Issued by a whole warp with warp-uniform operands; elect.sync picks the one lane that issues (the same lane for
-// the MMAs and their commit). Warp-uniform descriptors stay in uniform registers: no per-MMA R2UR waterfall loop,
-// which made a single divergent issuing thread the bottleneck of this kernel.
-__device__ __forceinline__ void mma_bf16(uint32_t d_tmem, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
-  asm volatile(
-      "{\n\t.reg .pred p, e;\n\telect.sync _|e, 0xffffffff;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}\n" ::"r"(d_tmem),
-      "l"(a), "l"(b), "r"(idesc), "r"(acc));
-}
-
-__device__ __forceinline__ void mma_commit(uint32_t bar) {
-  asm volatile(
-      "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
-      "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}\n" ::"r"(bar)
-      : "memory");
-}
-
-__device__ __forceinline__ void fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
-
-__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
-}
-
-__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
-  uint32_t done = 0;
-  while (!done) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}\n"
-        : "=r"(done)
-        : "r"(bar), "r"(parity)
-        : "memory");
-  }
-}
-
-__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-}
-
-__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-               "l"(src), "r"(bytes), "r"(bar)
-               : "memory");
-}
-
-// 32 lanes x 16 columns of fp32 from TMEM (asynchronous: the registers are valid after tmem_wait)
-__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
-  asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
-      : "r"(taddr));
-}
-// tcgen05.wait::ld, with the loaded registers as in/out operands so no use can be scheduled above it
-__device__ __forceinline__ void tmem_wait(uint32_t (&r)[16], uint32_t (&s)[16]) {
-  asm volatile("tcgen05.wait::ld.sync.aligned;"
-               : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]), "+r"(r[6]), "+r"(r[7]),
-                 "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11]), "+r"(r[12]), "+r"(r[13]), "+r"(r[14]),
-                 "+r"(r[15]), "+r"(s[0]), "+r"(s[1]), "+r"(s[2]), "+r"(s[3]), "+r"(s[4]), "+r"(s[5]), "+r"(s[6]),
-                 "+r"(s[7]), "+r"(s[8]), "+r"(s[9]), "+r"(s[10]), "+r"(s[11]), "+r"(s[12]), "+r"(s[13]),
-                 "+r"(s[14]), "+r"(s[15])
-               :
-               : "memory");
-}
+// PTX wrappers (tcgen05 MMA / TMEM, mbarriers, bulk copies): ffsva_ptx.h
+using namespace ptx;
 
 // max over the four pool positions: 16 consecutive channels starting at column col of each position group
 __device__ __forceinline__ void pooled16(uint32_t taddr, int col, int group_cols, float (&v)[16]) {
@@ -153,17 +75,12 @@ __device__ __forceinline__ void pooled16(uint32_t taddr, int col, int group_cols
   tmem_ld16(taddr + (uint32_t)(col + group_cols), r1);
   tmem_ld16(taddr + (uint32_t)(col + 2 * group_cols), r2);
   tmem_ld16(taddr + (uint32_t)(col + 3 * group_cols), r3);
-  tmem_wait(r0, r1);
-  tmem_wait(r2, r3);
+  tmem_wait_ld2(r0, r1);
+  tmem_wait_ld2(r2, r3);
 #pragma unroll
   for (int i = 0; i < 16; ++i)
     v[i] = fmaxf(fmaxf(__uint_as_float(r0[i]), __uint_as_float(r1[i])),
                  fmaxf(__uint_as_float(r2[i]), __uint_as_float(r3[i])));
-}
-
-__device__ __forceinline__ uint32_t pack_bf16(float lo, float hi) {
-  __nv_bfloat162 h = __floats2bfloat162_rn(lo, hi);
-  return *reinterpret_cast<uint32_t*>(&h);
 }
 
 __device__ __forceinline__ uint32_t u8_to_bf16(uint32_t v) {  // (v - 128) / 128 is exact in bf16
@@ -448,11 +365,8 @@ __global__ void __launch_bounds__(kThreads, kSnmCtasPerSm) snm_kernel(SnmArgs a)
 int snm_smem_bytes() { return SMEM_BYTES; }
 
 cudaError_t snm_configure() {
-  static bool done = false;
-  if (done) return cudaSuccess;
-  cudaError_t e = cudaFuncSetAttribute(snm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
-  if (e == cudaSuccess) done = true;
-  return e;
+  // the attribute is per device: called by every device context's creation (on that device), never cached
+  return cudaFuncSetAttribute(snm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM_BYTES);
 }
 
 cudaError_t launch_snm(const SnmArgs& a, cudaStream_t st) {

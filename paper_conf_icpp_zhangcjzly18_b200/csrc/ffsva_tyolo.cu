@@ -1150,6 +1150,8 @@ cudaError_t tyolo_configure() {
       e = cudaFuncSetAttribute(tyolo_slab_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kSlabSmem);
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(tyolo_pslab_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    if (e == cudaSuccess)  // the default 48 KB limit also covers static and reserved memory
+      e = cudaFuncSetAttribute(tyolo_resize_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     if (e != cudaSuccess) return e;
   }
   cudaError_t e = cudaFuncSetAttribute(tyolo_conv_kernel<1, 4, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -1226,12 +1228,7 @@ cudaError_t launch_tyolo_resize(const TyFrame* frames, int32_t n, int32_t D, int
     while (R < D && span(R + 1) * rb16 <= 24 * 1024) ++R;
   const int stage = span(R) * rb16;
   if (D > kResizeMaxD || stage > 200 * 1024) return cudaErrorInvalidValue;
-  static bool configured = false;  // opt in once: the default 48 KB limit also covers static and reserved memory
-  if (!configured) {
-    cudaError_t e = cudaFuncSetAttribute(tyolo_resize_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-    if (e != cudaSuccess) return e;
-    configured = true;
-  }
+  // the >48 KB opt-in is set per device by tyolo_configure (every model load, on the model's device)
   const dim3 grid((unsigned)((D + R - 1) / R), (unsigned)n);
   tyolo_resize_kernel<<<grid, kResizeThreads, stage, st>>>(frames, D, R, stage, out);
   return cudaGetLastError();

@@ -365,6 +365,7 @@ ffsva_status run_chunk(ffsva_tyolo* m, const ffsva_frame* frames, const int32_t*
 
 ffsva_status validate(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n) {
   if (!m || n < 0 || (n > 0 && !frames)) return fail(FFSVA_EINVAL, "bad argument");
+  begin_ptr_checks(m->ctx);
   for (int32_t i = 0; i < n; ++i) {
     if (!frames[i].stream || !frames[i].pixels) return fail(FFSVA_EINVAL, "frame without stream or pixels");
     if (frames[i].stream->ctx != m->ctx) return fail(FFSVA_EDEVICE, "frame lives on another device");
@@ -496,10 +497,11 @@ FFSVA_API ffsva_status ffsva_tyolo_run(ffsva_tyolo* m, const ffsva_frame* frames
                                        float* raw, void* cuda_stream) {
   if (target_class < 0 || target_class >= 20) return fail(FFSVA_EINVAL, "target_class must be a VOC class 0..19");
   if (n > 0 && !counts && !pass && !raw) return fail(FFSVA_EINVAL, "no output requested");
+  if (!m) return fail(FFSVA_EINVAL, "bad argument");
+  DeviceCtx* ctx = m->ctx;
+  std::lock_guard<std::mutex> lk(ctx->mu);  // taken before validate(): it shares the device's pointer checks
   ffsva_status st = validate(m, frames, n);
   if (st != FFSVA_OK || n == 0) return st;
-  DeviceCtx* ctx = m->ctx;
-  std::lock_guard<std::mutex> lk(ctx->mu);
   DeviceGuard g(ctx->device);
   std::vector<int32_t> targets((size_t)n, target_class);
   return tyolo_run_unlocked(m, frames, n, targets.data(), thresh, number_of_objects, counts, pass, raw,
@@ -541,10 +543,11 @@ extern "C" {
 FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, int32_t layer,
                                                 uint16_t* out, void* cuda_stream) {
   if (layer < -1 || layer > 7 || !out) return fail(FFSVA_EINVAL, "layer must be -1 (resized input) .. 7");
+  if (!m) return fail(FFSVA_EINVAL, "bad argument");
+  DeviceCtx* ctx = m->ctx;
+  std::lock_guard<std::mutex> lk(ctx->mu);  // taken before validate(): it shares the device's pointer checks
   ffsva_status st = validate(m, frames, n);
   if (st != FFSVA_OK || n == 0) return st;
-  DeviceCtx* ctx = m->ctx;
-  std::lock_guard<std::mutex> lk(ctx->mu);
   DeviceGuard g(ctx->device);
   if (n > kMaxChunk) return fail(FFSVA_EINVAL, "at most 256 frames");
   if ((st = ensure_workspace(m, n)) != FFSVA_OK) return st;
@@ -617,11 +620,12 @@ FFSVA_API ffsva_status ffsva_tyolo_layer_output(ffsva_tyolo* m, const ffsva_fram
 FFSVA_API ffsva_status ffsva_tyolo_profile(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, int32_t iters,
                                            float* ms_out, void* cuda_stream) {
   if (iters < 1 || !ms_out) return fail(FFSVA_EINVAL, "bad argument");
+  if (!m) return fail(FFSVA_EINVAL, "bad argument");
+  DeviceCtx* ctx = m->ctx;
+  std::lock_guard<std::mutex> lk(ctx->mu);  // taken before validate(): it shares the device's pointer checks
   ffsva_status st = validate(m, frames, n);
   if (st != FFSVA_OK || n == 0) return st;
   if (n > kMaxChunk) return fail(FFSVA_EINVAL, "at most 256 frames per profiled chunk");
-  DeviceCtx* ctx = m->ctx;
-  std::lock_guard<std::mutex> lk(ctx->mu);
   DeviceGuard g(ctx->device);
   if ((st = ensure_workspace(m, n)) != FFSVA_OK) return st;
   cudaStream_t cs = (cudaStream_t)cuda_stream;
