@@ -64,6 +64,7 @@ CONFIGS = {
 }
 SNM_FLOP = 7_477_632  # algorithmic FLOP per survivor
 DELTA, C_LOW, C_HIGH, FD, BATCH = 24.0, 0.2, 0.8, 0.5, 30
+L_T = math.log(((C_HIGH - C_LOW) * FD + C_LOW) / (1 - ((C_HIGH - C_LOW) * FD + C_LOW)))  # Eq. (2) in logit space
 
 
 def dist_env():
@@ -134,7 +135,249 @@ def ncu_traffic(config_name: str):
     return None
 
 
+# ---------------------------------------------------------------------------------------------- distributed skeleton
+# The multi-rank plumbing every run goes through (one process per GPU): stream ownership, the timed
+# region (barrier + synchronize on both sides, the per-stream statistics all-gather inside it, max over ranks), the
+# gather latency and the one-GPU reference throughput for the scaling efficiency. It talks to an "engine" (the GPU
+# engine below; tests/test_bench_dist.py drives it with a host engine over gloo at world size 2):
+#   eng.device, eng.frames_per_step, eng.step(i), eng.join(), eng.sync(), eng.mark() -> token,
+#   eng.elapsed_ms(t0, t1), eng.stats() -> int64 tensor [rows, NSTAT] (equal rows on every rank),
+#   eng.solo_frames_per_step, eng.solo_step(i) (the N = 1 workload: the rank's own batches under weak scaling, the
+#   whole stream set under strong scaling), eng.start_clocks(), eng.stop_clocks() -> dict.
+
+def owned_streams(cfg, ws: int, rank: int):
+    """(global stream ids rank `rank` owns, rows of the gathered statistics per rank). Strong-scaling configs (M5)
+    split their streams contiguously (dist.shard_streams); the others give every rank its own streams (weak)."""
+    from paper_conf_icpp_zhangcjzly18_b200 import dist as fdist
+    if cfg.get("shard"):
+        return (list(fdist.shard_streams(cfg["streams"], ws, rank)),
+                max(len(fdist.shard_streams(cfg["streams"], ws, r)) for r in range(ws)))
+    return list(fdist.weak_streams(cfg["streams"], ws, rank)), cfg["streams"]
+
+
+def _world():
+    import torch.distributed as dist
+    return dist.get_world_size() if dist.is_available() and dist.is_initialized() else 1
+
+
+def _barrier():
+    import torch.distributed as dist
+    if _world() > 1:
+        dist.barrier()
+
+
+def _allreduce(x: float, op: str, device) -> float:
+    """all-reduce of one host number (op 'max' | 'min' | 'sum'); NCCL reduces on the device, gloo on the host."""
+    import torch
+    import torch.distributed as dist
+    if _world() == 1:
+        return float(x)
+    dev = device if dist.get_backend() == "nccl" else "cpu"
+    t = torch.tensor([float(x)], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op={"max": dist.ReduceOp.MAX, "min": dist.ReduceOp.MIN, "sum": dist.ReduceOp.SUM}[op])
+    return float(t.item())
+
+
+def timed_region(eng, steps: int, warmup: int):
+    """W untimed warm-up steps, then exactly K steps bracketed by a barrier + synchronize on both sides and timed on
+    the device; the per-stream statistics all-gather (NCCL all_gather_into_tensor, the run's one exchange) closes the
+    region. Returns (ms = max over ranks, total frames over ranks, gathered statistics, clocks)."""
+    from paper_conf_icpp_zhangcjzly18_b200 import dist as fdist
+    for i in range(warmup):
+        eng.step(i)
+    eng.sync()
+    _barrier()
+    eng.start_clocks()
+    eng.sync()
+    _barrier()
+    t0 = eng.mark()
+    for i in range(steps):
+        eng.step(warmup + i)
+    eng.join()
+    gathered = fdist.gather_stats(eng.stats())
+    t1 = eng.mark()
+    eng.sync()
+    _barrier()
+    clk = eng.stop_clocks()
+    ms_max = _allreduce(eng.elapsed_ms(t0, t1), "max", eng.device)
+    total = _allreduce(eng.frames_per_step * steps, "sum", eng.device)
+    return ms_max, int(total), gathered, clk
+
+
+def gather_us(eng, reps: int = 50) -> float:
+    """Device time of one statistics all-gather (the per-interval exchange of §8(e)), mean of `reps`, max over
+    ranks, in microseconds."""
+    from paper_conf_icpp_zhangcjzly18_b200 import dist as fdist
+    local = eng.stats()
+    fdist.gather_stats(local)
+    eng.sync()
+    _barrier()
+    t0 = eng.mark()
+    for _ in range(reps):
+        fdist.gather_stats(local)
+    t1 = eng.mark()
+    eng.sync()
+    return 1e3 * _allreduce(eng.elapsed_ms(t0, t1) / reps, "max", eng.device)
+
+
+def solo_fps(eng, steps: int, rank: int) -> float:
+    """Throughput of the N = 1 workload on one GPU (rank 0 alone while the other ranks wait), for the scaling
+    efficiency fps(G) / (G * fps(1)). Every rank returns rank 0's figure."""
+    fps = 0.0
+    eng.sync()
+    _barrier()
+    if rank == 0:
+        for i in range(2):
+            eng.solo_step(i)
+        eng.join()
+        eng.sync()
+        t0 = eng.mark()
+        for i in range(steps):
+            eng.solo_step(2 + i)
+        eng.join()
+        t1 = eng.mark()
+        eng.sync()
+        fps = eng.solo_frames_per_step * steps / (eng.elapsed_ms(t0, t1) / 1e3)
+    return _allreduce(fps, "max", eng.device)
+
+
+def scaling_fields(value: float, fps1: float, ws: int, g_us: float, gathered_rows: int, strong: bool) -> dict:
+    return {"kind": "strong" if strong else "weak", "n_gpus": ws, "fps_1gpu": fps1,
+            "efficiency": value / (ws * fps1) if fps1 > 0 else None,
+            "efficiency_def": "fps(G) / (G * fps(1)); fps(1) = the N = 1 workload timed on rank 0 of this run "
+                              "(strong: all streams on one GPU; weak: one rank's streams)",
+            "stats_gather_us": g_us, "stats_gather_rows": gathered_rows,
+            "stats_gather": "NCCL all_gather_into_tensor of the u64 per-stream table (device time, max over ranks)"}
+
+
 # ---------------------------------------------------------------------------------------------- our arm
+
+class GpuEngine:
+    """The bench's workload on one GPU: the rank's streams (reference + SNM each), a stream-major frame pool far
+    larger than L2, and prepared batches (one second of video of every owned stream each) replayed as CUDA graphs,
+    consecutive steps alternating over CUDA streams."""
+
+    def __init__(self, args, cfg, ws, rank, dev):
+        import torch
+
+        import paper_conf_icpp_zhangcjzly18_b200 as ff
+        from paper_conf_icpp_zhangcjzly18_b200 import ffsva as ffb
+        from synth import synth
+        self.torch, self.ffb, self.dev, self.device = torch, ffb, dev, dev
+        self.cfg, self.args, self.rank, self.ws = cfg, args, rank, ws
+        W, H, P = cfg["W"], cfg["H"], 3 * cfg["W"]
+        self.W, self.H, self.P, self.fbytes = W, H, P, H * P
+        self.sids, self.rows = owned_streams(cfg, ws, rank)
+        # strong scaling: rank 0 also holds the whole stream set (its shard is the prefix) for the N = 1 reference
+        self.strong = bool(cfg.get("shard"))
+        all_ids = list(range(cfg["streams"])) if (self.strong and ws > 1 and rank == 0) else self.sids
+        S_all, PF, SF = len(all_ids), cfg["pool_frames"], cfg["step_frames"]
+        self.video = synth.Video(seed=cfg["seed"], width=W, height=H, period=cfg["period"], on_len=cfg["on_len"])
+        self.ctx = ff.Context(dev)
+        self.delta = cfg.get("delta", DELTA)
+        self.streams = []
+        for s in all_ids:
+            st = self.ctx.open_stream(width=W, height=H, delta_diff=self.delta, c_low=C_LOW, c_high=C_HIGH,
+                                      filter_degree=FD, snm_batch=BATCH)
+            refs = torch.empty((32, H, P), dtype=torch.uint8, device=dev)
+            synth.frames_cuda(self.video, torch.full((32,), s, dtype=torch.int32, device=dev),
+                              torch.arange(32, dtype=torch.int64, device=dev), refs, self.fbytes, P, ref=True)
+            st.set_reference(refs)
+            del refs
+            st.snm_load(synth.snm_weights(cfg["seed"], s))
+            self.streams.append(st)
+        # frame pool: stream-major, pool[s][t]
+        self.pool = torch.empty((S_all, PF, H, P), dtype=torch.uint8, device=dev)
+        for k, s in enumerate(all_ids):
+            synth.frames_cuda(self.video, torch.full((PF,), s, dtype=torch.int32, device=dev),
+                              torch.arange(PF, dtype=torch.int64, device=dev), self.pool[k], self.fbytes, P)
+        torch.cuda.synchronize()
+        S = len(self.sids)
+        self.S, self.PF, self.SF = S, PF, SF
+        # prepared batches: batch j = frames [j*SF, (j+1)*SF) of every owned stream (one second of video)
+        self.nbatches = max(1, PF // SF)
+
+        def make(nstreams):
+            return [self.ctx.prepare([(self.streams[k], self.pool[k, j * SF + i], j * SF + i)
+                                      for k in range(nstreams) for i in range(SF)]) for j in range(self.nbatches)]
+        self.batches = make(S)
+        self.solo_batches = make(S_all) if S_all != S else self.batches
+        self.frames_per_step = S * SF
+        self.solo_frames_per_step = S_all * SF
+        self.planted = [sum(synth.planted(self.video, s, j * SF, (j + 1) * SF) for s in self.sids)
+                        for j in range(self.nbatches)]
+        self.cs = torch.cuda.Stream(device=dev)
+        nstr = max(1, min(args.streams, self.nbatches))
+        self.css = [self.cs] + [torch.cuda.Stream(device=dev) for _ in range(nstr - 1)]
+        self.stats_dev = torch.zeros((max(1, self.rows), ffb.NSTAT), dtype=torch.int64, device=dev)
+        self.clocks = None
+
+    # --- correctness gate before timing: SDD pass count == planted count on every batch (P8 at full size), and
+    # the fraction of survivors whose logit lies within the 2e-2 parity margin of the decision threshold
+    def gate(self):
+        near, surv = 0, 0
+        for j, b in enumerate(self.batches):
+            b.launch(self.cs)
+            r = b.fetch(self.cs)
+            expect = self.planted[j] if self.delta == DELTA else self.frames_per_step
+            if int(r["sdd_pass"].sum()) != expect:
+                raise RuntimeError(f"batch {j}: SDD passed {int(r['sdd_pass'].sum())} != expected {expect}")
+            self.planted[j] = expect
+            lg = r["logit"][r["sdd_pass"] == 1]
+            near += int((np.abs(lg - L_T) < 2e-2).sum())
+            surv += lg.size
+        self.ctx.stats(reset=True)
+        self.near_margin = {"fraction": near / surv if surv else 0.0, "survivors": surv, "margin": 2e-2,
+                            "bar": "< 0.10 (SURVEY.md §8(d): else the decision parity check is weak)"}
+        if surv and near / surv >= 0.10:
+            raise RuntimeError(f"{near}/{surv} survivors lie within 2e-2 of the SNM threshold (>= 10%)")
+
+    def step(self, i):
+        self.batches[i % self.nbatches].launch(self.css[i % len(self.css)])
+
+    def solo_step(self, i):
+        self.solo_batches[i % self.nbatches].launch(self.css[i % len(self.css)])
+
+    def join(self):  # the last step of every CUDA stream is done before the closing mark
+        for s2 in self.css[1:]:
+            ev = self.torch.cuda.Event()
+            ev.record(s2)
+            self.cs.wait_event(ev)
+
+    def sync(self):
+        self.torch.cuda.synchronize()
+
+    def mark(self):
+        e = self.torch.cuda.Event(enable_timing=True)
+        e.record(self.cs)
+        for s2 in self.css[1:]:  # later steps on the other streams start after this mark
+            s2.wait_event(e)
+        return e
+
+    def elapsed_ms(self, t0, t1):
+        t1.synchronize()
+        return t0.elapsed_time(t1)
+
+    def stats(self):
+        """a8: the owned streams' statistics rows (device table, stream slots in open order) -> stats_dev."""
+        n = min(self.S, self.rows)
+        self.ffb.ffsva_stats_copy(self.dev.index, self.stats_dev.data_ptr(), max(1, n), False, False,
+                                  self.cs.cuda_stream)
+        return self.stats_dev
+
+    def start_clocks(self):
+        self.clocks = ClockSampler(self.dev.index)
+        self.clocks.start()
+        time.sleep(0.3)
+
+    def stop_clocks(self):
+        return self.clocks.stop() if self.clocks else None
+
+    def close(self):
+        for b in {id(b): b for b in self.batches + self.solo_batches}.values():
+            b.destroy()
+        self.ctx.close()
+
 
 def run_ours(args, cfg, ws, rank, local):
     import torch
@@ -142,118 +385,29 @@ def run_ours(args, cfg, ws, rank, local):
 
     import paper_conf_icpp_zhangcjzly18_b200 as ff
     from paper_conf_icpp_zhangcjzly18_b200 import ffsva as ffb
-    from synth import synth
 
-    torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
-    if ws > 1:
-        dist.init_process_group("nccl", device_id=dev)
-    W, H, P = cfg["W"], cfg["H"], 3 * cfg["W"]
-    fbytes = H * P
-    if cfg.get("shard"):
-        lo, hi = rank * cfg["streams"] // ws, (rank + 1) * cfg["streams"] // ws
-        sids = list(range(lo, hi))
-    else:
-        sids = [rank * cfg["streams"] + s for s in range(cfg["streams"])]
-    S, PF, SF = len(sids), cfg["pool_frames"], cfg["step_frames"]
-    video = synth.Video(seed=cfg["seed"], width=W, height=H, period=cfg["period"], on_len=cfg["on_len"])
-    ctx = ff.Context(dev)
-    streams = []
-    for s in sids:
-        st = ctx.open_stream(width=W, height=H, delta_diff=cfg.get("delta", DELTA), c_low=C_LOW, c_high=C_HIGH,
-                             filter_degree=FD,
-                             snm_batch=BATCH)
-        refs = torch.empty((32, H, P), dtype=torch.uint8, device=dev)
-        synth.frames_cuda(video, torch.full((32,), s, dtype=torch.int32, device=dev),
-                          torch.arange(32, dtype=torch.int64, device=dev), refs, fbytes, P, ref=True)
-        st.set_reference(refs)
-        del refs
-        st.snm_load(synth.snm_weights(cfg["seed"], s))
-        streams.append(st)
-    # frame pool: stream-major, pool[s][t]
-    pool = torch.empty((S, PF, H, P), dtype=torch.uint8, device=dev)
-    for k, s in enumerate(sids):
-        synth.frames_cuda(video, torch.full((PF,), s, dtype=torch.int32, device=dev),
-                          torch.arange(PF, dtype=torch.int64, device=dev), pool[k], fbytes, P)
-    torch.cuda.synchronize()
-    # prepared batches: batch j = frames [j*SF, (j+1)*SF) of every stream (one second of video)
-    nbatches = max(1, PF // SF)
-    batches = []
-    for j in range(nbatches):
-        items = [(streams[k], pool[k, j * SF + i], j * SF + i) for k in range(S) for i in range(SF)]
-        batches.append(ctx.prepare(items))
-    frames_per_step = S * SF
-    planted = [sum(synth.planted(video, s, j * SF, (j + 1) * SF) for s in sids) for j in range(nbatches)]
-    cs = torch.cuda.Stream(device=dev)
-    stats_dev = torch.zeros((max(1, S), ffb.NSTAT), dtype=torch.int64, device=dev)
-    gathered = torch.zeros((ws * max(1, S), ffb.NSTAT), dtype=torch.int64, device=dev) if ws > 1 else None
-
-    # correctness gate before timing: SDD pass count == planted count on every batch (P8 at full size)
-    for j, b in enumerate(batches):
-        b.launch(cs)
-        r = b.fetch(cs)
-        expect = planted[j] if cfg.get("delta", DELTA) == DELTA else frames_per_step
-        if int(r["sdd_pass"].sum()) != expect:
-            raise RuntimeError(f"batch {j}: SDD passed {int(r['sdd_pass'].sum())} != expected {expect}")
-        planted[j] = expect
-    ctx.stats(reset=True)
-
-    # consecutive steps alternate over --streams CUDA streams (different prepared batches, own buffers): step i+1's
-    # K1 starts while step i's K1 tail, K3 and K4 still run (the per-stream statistics are order-independent atomics)
-    nstr = max(1, min(args.streams, nbatches))
-    css = [cs] + [torch.cuda.Stream(device=dev) for _ in range(nstr - 1)]
-
-    def step(i):
-        batches[i % nbatches].launch(css[i % nstr])
-
-    for i in range(args.warmup):
-        step(i)
-    torch.cuda.synchronize()
-    if ws > 1:
-        dist.barrier()
-    clocks = ClockSampler(local)
-    clocks.start()
-    time.sleep(0.3)
+    torch.cuda.set_device(dev)
+    eng = GpuEngine(args, cfg, ws, rank, dev)
+    eng.gate()
     launches0 = ff.ffsva_kernel_launches()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    torch.cuda.synchronize()
-    if ws > 1:
-        dist.barrier()
-    with torch.cuda.stream(cs):
-        e0.record(cs)
-        for s2 in css[1:]:
-            s2.wait_event(e0)
-        for i in range(args.steps):
-            step(args.warmup + i)
-        for s2 in css[1:]:  # the timed region ends when every stream's last step is done
-            ev = torch.cuda.Event()
-            ev.record(s2)
-            cs.wait_event(ev)
-        # a8 reporting: per-stream statistics to a device tensor, all-gathered over NCCL when sharded
-        ffb.ffsva_stats_copy(local, stats_dev.data_ptr(), S, False, False, cs.cuda_stream)
-        if ws > 1:
-            dist.all_gather_into_tensor(gathered, stats_dev)
-        e1.record(cs)
-    torch.cuda.synchronize()
+    ms_max, total_frames, gathered, clk = timed_region(eng, args.steps, args.warmup)
     launches = ff.ffsva_kernel_launches() - launches0
-    if ws > 1:
-        dist.barrier()
-    clk = clocks.stop()
-    ms = e0.elapsed_time(e1)
-    t = torch.tensor([ms], dtype=torch.float64, device=dev)
-    if ws > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms_max = float(t.item())
-    total_frames = frames_per_step * args.steps * ws
     value = total_frames / (ms_max / 1e3)
-    st_rows = stats_dev.cpu().numpy()
-    if int(st_rows[:, 0].sum()) != frames_per_step * (args.warmup + args.steps):
-        raise RuntimeError("per-stream frame counters disagree with the frames launched")
+    # the gathered table must account for every frame every rank launched (warm-up + timed steps)
+    g = gathered.cpu().numpy()
+    if int(g[:, 0].sum()) != int(_allreduce(eng.frames_per_step * (args.warmup + args.steps), "sum", dev)):
+        raise RuntimeError("gathered per-stream frame counters disagree with the frames launched")
+    g_us = gather_us(eng) if ws > 1 else 0.0
+    fps1 = solo_fps(eng, max(3, min(args.steps, 50)), rank) if ws > 1 else value
+    scaling = scaling_fields(value, fps1, ws, g_us, int(g.shape[0]), eng.strong)
 
     # ---- per-kernel device times (CUDA events on the launching stream) for the roofline
+    batches, nbatches, cs = eng.batches, eng.nbatches, eng.cs
     k_ms = ffb.ffsva_batch_profile([b.handle for b in batches], max(2, min(10, 30 // nbatches + 1)), cs.cuda_stream)
-    r_last = batches[0].fetch(cs)
-    m_avg = float(np.mean(planted))
+    m_avg = float(np.mean(eng.planted))
+    W, H, P, S, SF = eng.W, eng.H, eng.P, eng.S, eng.SF
+    frames_per_step = eng.frames_per_step
     k1_bytes = frames_per_step * (3 * W * H + 9) + m_avg * 7500
     hbm_peak, tf_peak, peak_kind = measured_peaks()
     achieved = k1_bytes / (k_ms[0] / 1e3) / 1e9
@@ -264,53 +418,59 @@ def run_ours(args, cfg, ws, rank, local):
     if not args.no_e2e:
         n_e2e = max(1, min(args.steps, args.e2e_steps))
         pinned = torch.empty((S, SF, H, P), dtype=torch.uint8).pin_memory()
-        pinned.copy_(pool[:, :SF].cpu())
-        items = [(streams[k], pinned[k, i].data_ptr(), i) for k in range(S) for i in range(SF)]
-        ctx.filter_batch(items, stream=cs, host=True)  # warm-up (ring allocation)
+        pinned.copy_(eng.pool[:S, :SF].cpu())
+        items = [(eng.streams[k], pinned[k, i].data_ptr(), i) for k in range(S) for i in range(SF)]
+        eng.ctx.filter_batch(items, stream=cs, host=True)  # warm-up (ring allocation)
         torch.cuda.synchronize()
-        if ws > 1:
-            dist.barrier()
+        _barrier()
         h0, h1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         h0.record(cs)
         for _ in range(n_e2e):
-            res = ctx.filter_batch(items, stream=cs, host=True)
+            eng.ctx.filter_batch(items, stream=cs, host=True)
         h1.record(cs)
         torch.cuda.synchronize()
-        te = torch.tensor([h0.elapsed_time(h1)], dtype=torch.float64, device=dev)
-        if ws > 1:
-            dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        e2e_val = frames_per_step * n_e2e * ws / (float(te.item()) / 1e3)
-        e2e = {"value": e2e_val, "unit": "frames/s", "h2d_bytes_per_step": int(frames_per_step * fbytes),
+        te = _allreduce(h0.elapsed_time(h1), "max", dev)
+        e2e_val = _allreduce(frames_per_step * n_e2e, "sum", dev) / (te / 1e3)
+        e2e = {"value": e2e_val, "unit": "frames/s", "h2d_bytes_per_step": int(frames_per_step * eng.fbytes),
                "d2h_bytes_per_step": int(frames_per_step * ffb.RESULT_DTYPE.itemsize), "steps": n_e2e,
                "path": "ffsva_filter_batch_host (pinned host frames -> 2-chunk device ring, copies overlapped "
                        "with K1)"}
         del pinned
 
     cpu = None
-    if rank == 0 and ws == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(cfg, video, sids, pool, args.cpu_frames)
+    if rank == 0 and not args.no_cpu_baseline:
+        if ws == 1:
+            cpu = cpu_baseline(cfg, eng.video, eng.sids, eng.pool, args.cpu_frames)
+        else:
+            cpu = {"kind": "oracle", "measured_at": "N = 1 only (the oracle is a host program: its figure does not "
+                                                   "change with the GPU count)"}
 
     # ---- online validation of "sustained 30-FPS streams" (paced arrivals through the online runtime)
     online = None
     if args.online and args.config == "m2":
-        online = online_validation(args, ctx, video, sids, pool, value / ws, dev, cs, ws)
+        online = online_validation(args, eng.ctx, eng.video, eng.sids, eng.pool[:S], value / ws, dev, cs, ws)
 
     out = None
     if rank == 0:
         out = {
             "metric": METRIC, "value": value, "unit": "frames/s", "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u8 (SDD) / bf16-fp32 (SNM)", "data": "synthetic",
+            "scaling": "strong" if eng.strong else "weak", "vs_baseline": None,
+            "dtype": "u8 (SDD) / bf16-fp32 (SNM)", "data": "synthetic",
             "config": {"workload": cfg["desc"], "config_id": args.config, "streams_per_gpu": S,
-                       "frames_per_step": frames_per_step * ws, "frame_bytes": fbytes,
-                       "pool_bytes_per_gpu": int(S * PF * fbytes),
+                       "frames_per_step": int(total_frames // args.steps), "frames_per_step_per_gpu": frames_per_step,
+                       "frame_bytes": eng.fbytes, "pool_bytes_per_gpu": int(S * eng.PF * eng.fbytes),
                        "l2": "inputs larger than L2: each step reads a different %.2f GB slice of the pool"
-                             % (frames_per_step * fbytes / 1e9),
-                       "parallelism": f"stream-sharded x{ws} (weak: {S} streams per GPU)",
+                             % (frames_per_step * eng.fbytes / 1e9),
+                       "parallelism": (f"stream-sharded x{ws} (strong: {cfg['streams']} streams split, {S} on rank 0)"
+                                       if eng.strong else f"stream-sharded x{ws} (weak: {S} streams per GPU)"),
+                       "dist_backend": args.dist_backend if ws > 1 else None,
                        "batch_size": BATCH, "delta_diff": DELTA, "c_low": C_LOW, "c_high": C_HIGH,
-                       "filter_degree": FD, "seed": cfg["seed"], "cuda_streams": nstr},
+                       "filter_degree": FD, "seed": cfg["seed"], "cuda_streams": len(eng.css)},
             "sustained_streams_30fps": int(value // 30),
             "sdd_pass_per_step": m_avg,
+            "snm_near_margin": eng.near_margin,
+            "multi_gpu": scaling,
             "roofline": {"bound": "hbm", "kernel": "K1 sdd_kernel (ingest + box downsample + SSD + threshold)",
                          "achieved": achieved, "peak": hbm_peak, "unit": "GB/s", "frac": achieved / hbm_peak,
                          "peak_source": peak_kind, "traffic": traffic,
@@ -332,11 +492,7 @@ def run_ours(args, cfg, ws, rank, local):
             out["sdd_roofline"] = out["roofline"]
             out["roofline"] = dict(out["snm_roofline"], kernel_ms=out["sdd_roofline"]["kernel_ms"],
                                    k4_share_of_step=k_ms[2] / max(1e-9, sum(k_ms)))
-    for b in batches:
-        b.destroy()
-    ctx.close()
-    if ws > 1:
-        dist.destroy_process_group()
+    eng.close()
     return out
 
 
@@ -484,10 +640,8 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs, ws=1):
                         cuda_stream=cs, tyolo=ty if with_ty else None, tick_s=0.010 if S < 10000 else 0.025)
         res["stream_setup_s"] = setup_s
         if ws > 1:
-            ok = torch.tensor([1 if res["sustained"] else 0], dtype=torch.int32, device=dev)
-            dist.all_reduce(ok, op=dist.ReduceOp.MIN)
             res["sustained_this_rank"] = res["sustained"]
-            res["sustained"] = bool(ok.item())
+            res["sustained"] = bool(_allreduce(1 if res["sustained"] else 0, "min", dev))
             res["streams_per_gpu"], res["streams"] = S, S * ws
         results.append(res)
         if S in ladder and not with_ty and not res["sustained"]:
@@ -650,6 +804,42 @@ def run_reference(args, cfg, ws, rank):
             "e2e": {"value": value, "unit": "frames/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
 
 
+def spawn_ranks(args) -> int:
+    """`python bench.py --gpus N` outside torchrun: build once here, then launch N ranks (one process per GPU) the
+    way the driver does, with the build step disabled in the children, and relay rank 0's output."""
+    import __graft_entry__ as ge
+    ge.build()
+    import socket
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    env = dict(os.environ, FFSVA_BENCH_PREBUILT="1")
+    return subprocess.call(cmd, env=env)
+
+
+def init_ranks(args, ws: int, rank: int, local: int):
+    """Process group + build order under torchrun: every rank joins the group first, rank 0 builds (unless the
+    launcher already did) while the others wait at a barrier, so no rank can load a half-written library."""
+    if ws > 1:
+        import torch
+        import torch.distributed as dist
+        if args.dist_backend == "nccl":
+            if torch.cuda.device_count() < ws:
+                raise SystemExit(f"--gpus {ws} with NCCL needs {ws} GPUs, found {torch.cuda.device_count()} "
+                                 f"(--dist-backend gloo shares GPUs between ranks, for testing the N > 1 path)")
+            torch.cuda.set_device(local)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
+    if os.environ.get("FFSVA_BENCH_PREBUILT") != "1" and rank == 0:
+        import __graft_entry__ as ge
+        ge.build()
+    _barrier()
+
+
 def main():
     ap = argparse.ArgumentParser(description=__doc__, formatter_class=argparse.RawDescriptionHelpFormatter)
     ap.add_argument("--gpus", type=int, default=1)
@@ -657,6 +847,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--config", default="m2", choices=sorted(CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend for N > 1 (gloo: ranks may share a GPU; a test mode)")
     ap.add_argument("--streams", type=int, default=2,
                     help="CUDA streams the timed steps alternate over (consecutive batches overlap)")
     ap.add_argument("--e2e-steps", type=int, default=5)
@@ -675,20 +867,27 @@ def main():
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
     ws, rank, local = dist_env()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(spawn_ranks(args))
+    if ws != args.gpus and "WORLD_SIZE" in os.environ:
+        ap.error(f"--gpus {args.gpus} but WORLD_SIZE={ws}")
     cfg = CONFIGS[args.config]
-    if args.impl == "reference":
+    if args.impl == "reference":  # the CPU oracle: rank 0 alone runs and prints it; the other ranks exit 0
         out = run_reference(args, cfg, ws, rank)
-    else:
-        import __graft_entry__ as ge
-        if rank == 0:
-            ge.build()
-        if ws > 1:
-            # other ranks wait for rank 0's build (the .so must exist before they load it)
-            while not os.path.exists(os.path.join(ROOT, "paper_conf_icpp_zhangcjzly18_b200", "lib", "libffsva.so")):
-                time.sleep(0.5)
-        out = run_tyolo(args, cfg, ws, rank, local) if args.config == "tyolo" else run_ours(args, cfg, ws, rank, local)
+        if out is not None:
+            print(json.dumps(out))
+        return
+    init_ranks(args, ws, rank, local)
+    if args.dist_backend == "gloo":
+        import torch
+        local = local % max(1, torch.cuda.device_count())
+    out = run_tyolo(args, cfg, ws, rank, local) if args.config == "tyolo" else run_ours(args, cfg, ws, rank, local)
     if rank == 0 and out is not None:
         print(json.dumps(out))
+    if ws > 1:
+        import torch.distributed as dist
+        _barrier()
+        dist.destroy_process_group()
 
 
 if __name__ == "__main__":

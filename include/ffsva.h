@@ -126,7 +126,12 @@ typedef struct {
   int32_t reserved;
 } ffsva_result;
 
-/* Counters per stream slot, ffsva_stats_copy() layout: u64[slots][FFSVA_NSTAT]. */
+/* Counters per stream slot, ffsva_stats_copy() layout: u64[slots][FFSVA_NSTAT] (a8; the per-filter frame ratios of
+ * PAPER.md L253 Fig. 5 and the arrival -> decision latency of the online runtime). Columns 0-7 are kept by the
+ * kernels (batch and online paths alike); columns 8-23 by the online runtime (ffsva_sched_*): a frame "arrives"
+ * when ffsva_sched_push accepts it and is "decided" when the tick that reports its event harvests it (dropped by
+ * SDD, scored by SNM, or counted by T-YOLO). Latency bins: bin 0 < 1 ms, bin k (1..12) in [2^(k-1), 2^k) ms,
+ * bin 13 >= 4096 ms. */
 enum {
   FFSVA_STAT_FRAMES = 0,   /* frames through SDD */
   FFSVA_STAT_SDD_PASS = 1, /* SDD survivors */
@@ -136,7 +141,10 @@ enum {
   FFSVA_STAT_CLASS1 = 5,
   FFSVA_STAT_CLASS2 = 6,
   FFSVA_STAT_SNM_BATCHES = 7, /* SNM weight loads = dynamic batches executed (L219) */
-  FFSVA_NSTAT = 8
+  FFSVA_STAT_DECIDED = 8,  /* online runtime: frames whose fate was reported (= sum of the latency bins) */
+  FFSVA_STAT_LAT_SUM_US = 9, /* online runtime: sum of their arrival -> decision latencies, microseconds */
+  FFSVA_STAT_LAT_BIN0 = 10, /* 14 latency bins, columns 10..23 */
+  FFSVA_NSTAT = 24
 };
 
 /* Create a stream (a camera) with its own SDD/SNM state on desc->device. The first stream of a device creates
@@ -281,6 +289,14 @@ FFSVA_API ffsva_status ffsva_sched_set_policy(ffsva_sched* s, int32_t policy);
  * off while a cycle is in flight returns FFSVA_EAGAIN (tick once more first). Errors: EINVAL. */
 FFSVA_API ffsva_status ffsva_sched_set_pipeline(ffsva_sched* s, int32_t on);
 
+/* Inspection (tests): the frames of the most recently launched cycle — its SDD admissions (stage 0) and its SNM
+ * pops (stage 1), in cycle order — with the 50x50x3 image each holds in the scheduler's device slot pool (the SNM's
+ * input: written by K1 when the frame was admitted, possibly several cycles earlier for a pop). Synchronous mode:
+ * the cycle of the last tick; pipelined mode: the cycle in flight (waited for), none if idle. Writes min(n, cap)
+ * entries: frames[k], stage[k], d50[k*7500 .. +7500) (host memory); *n = the cycle's frame count. */
+FFSVA_API ffsva_status ffsva_sched_inspect(ffsva_sched* s, ffsva_frame* frames, int32_t* stage, uint8_t* d50,
+                                           int32_t cap, int32_t* n);
+
 /* ---------------------------------------------------------------------------------------------------------
  * Admission control and stream re-forwarding between instances (§4.3.1: "when any queue of
  * T-YOLO or SNM is longer than its predefined threshold ... the corresponding video stream is re-forwarded to
@@ -291,7 +307,7 @@ FFSVA_API ffsva_status ffsva_sched_set_pipeline(ffsva_sched* s, int32_t on);
  *
  * Stream image: a self-contained byte image of a stream — its descriptor, thresholds, reference image R, packed
  * SNM weights and its per-stream statistics row — so the stream continues bit-identically elsewhere.
- *   ffsva_stream_image_bytes: size of s's image (57,152 B at the default 100x100 grid);
+ *   ffsva_stream_image_bytes: size of s's image (57,280 B at the default 100x100 grid);
  *   ffsva_stream_export: write the image to dst (host memory, or device memory on s's device when dst_is_host
  *     is 0 — e.g. a buffer about to be sent over NCCL); synchronous on cuda_stream;
  *   ffsva_stream_import: open a new stream on `device` from an image (host memory, or device memory on `device`

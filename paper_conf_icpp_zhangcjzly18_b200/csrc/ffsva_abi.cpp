@@ -1,5 +1,6 @@
 // ffsva_abi.cpp — the extern "C" entry points of include/ffsva.h: argument validation (always before any GPU
 // work), per-device locking, and dispatch into the runtime.
+#include <algorithm>
 #include <cmath>
 #include <cstring>
 #include <memory>
@@ -117,6 +118,8 @@ FFSVA_API ffsva_status ffsva_open_stream(const ffsva_stream_desc* desc, ffsva_st
     }
     // a fresh slot starts with zero statistics
     cudaMemset(ctx->d_stats + (size_t)s->slot * NSTAT, 0, sizeof(unsigned long long) * NSTAT);
+    std::lock_guard<std::mutex> lk(ctx->lat_mu);
+    std::fill_n(ctx->h_lat.begin() + (std::ptrdiff_t)s->slot * NLAT, NLAT, 0);
   }
   *out = s.release();
   return FFSVA_OK;
@@ -361,11 +364,28 @@ FFSVA_API ffsva_status ffsva_stats_copy(int32_t device, uint64_t* dst, int32_t m
     const int32_t ncopy = used < max_slots ? used : max_slots;
     cudaStream_t cs = (cudaStream_t)cuda_stream;
     cudaError_t e = cudaSuccess;
-    if (ncopy > 0)
-      e = cudaMemcpyAsync(dst, ctx->d_stats, sizeof(uint64_t) * NSTAT * ncopy,
-                          dst_is_host ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice, cs);
+    // kernel counters (device table, stride NSTAT) into columns 0..7, the online runtime's latency columns (host
+    // table, stride NLAT) into columns 8..23 of the FFSVA_NSTAT-wide rows
+    std::vector<uint64_t> lat;
+    {
+      std::lock_guard<std::mutex> lk2(ctx->lat_mu);
+      lat.assign(ctx->h_lat.begin(), ctx->h_lat.begin() + (std::ptrdiff_t)ncopy * NLAT);
+      if (reset) std::fill(ctx->h_lat.begin(), ctx->h_lat.end(), 0);
+    }
+    const size_t row = sizeof(uint64_t) * FFSVA_NSTAT;
+    if (ncopy > 0) {
+      e = cudaMemcpy2DAsync(dst, row, ctx->d_stats, sizeof(uint64_t) * NSTAT, sizeof(uint64_t) * NSTAT, (size_t)ncopy,
+                            dst_is_host ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice, cs);
+      if (e == cudaSuccess && !dst_is_host)  // pageable source: returns once the rows are staged
+        e = cudaMemcpy2DAsync(dst + NSTAT, row, lat.data(), sizeof(uint64_t) * NLAT, sizeof(uint64_t) * NLAT,
+                              (size_t)ncopy, cudaMemcpyHostToDevice, cs);
+    }
     if (e == cudaSuccess && reset) e = cudaMemsetAsync(ctx->d_stats, 0, sizeof(uint64_t) * NSTAT * ctx->stats_cap, cs);
-    if (e == cudaSuccess && dst_is_host) e = cudaStreamSynchronize(cs);
+    if (e == cudaSuccess && dst_is_host) {
+      e = cudaStreamSynchronize(cs);
+      for (int32_t i = 0; i < ncopy; ++i)
+        std::memcpy(dst + (size_t)i * FFSVA_NSTAT + NSTAT, lat.data() + (size_t)i * NLAT, sizeof(uint64_t) * NLAT);
+    }
     if (e != cudaSuccess) out = cuda_fail(ctx, e, "ffsva_stats_copy");
   }
   ctx_release(ctx);
@@ -375,7 +395,7 @@ FFSVA_API ffsva_status ffsva_stats_copy(int32_t device, uint64_t* dst, int32_t m
 // ---------------------------------------------------------------- stream images (re-forwarding)
 namespace {
 constexpr uint32_t kImageMagic = 0x56534646u;  // "FFSV"
-constexpr uint32_t kImageVersion = 3;  // 3: SNM image with patch-row conv1 operands and bf16 FC weights
+constexpr uint32_t kImageVersion = 4;  // 4: statistics row with the latency columns (FFSVA_NSTAT = 24)
 constexpr int64_t kImageHeader = 256;
 struct ImageHeader {
   uint32_t magic, version;
@@ -387,7 +407,7 @@ struct ImageHeader {
 static_assert(sizeof(ImageHeader) <= kImageHeader, "image header");
 int64_t al16(int64_t x) { return (x + 15) & ~(int64_t)15; }
 int64_t image_bytes(const ffsva_stream_desc& d) {
-  return kImageHeader + al16(3LL * d.sdd_w * d.sdd_h) + al16(snm::BLOB_BYTES) + 8LL * NSTAT;
+  return kImageHeader + al16(3LL * d.sdd_w * d.sdd_h) + al16(snm::BLOB_BYTES) + 8LL * FFSVA_NSTAT;
 }
 }  // namespace
 
@@ -419,7 +439,7 @@ FFSVA_API ffsva_status ffsva_stream_export(ffsva_stream* s, void* dst, int64_t c
   h.ref_sum_sq = s->ref_sum_sq;
   h.ref_bytes = 3LL * s->desc.sdd_w * s->desc.sdd_h;
   h.snm_bytes = snm::BLOB_BYTES;
-  h.stats_bytes = 8LL * NSTAT;
+  h.stats_bytes = 8LL * FFSVA_NSTAT;
   h.total = total;
   h.has_ref = s->has_ref;
   h.has_snm = s->has_snm;
@@ -433,7 +453,15 @@ FFSVA_API ffsva_status ffsva_stream_export(ffsva_stream* s, void* dst, int64_t c
   if (e == cudaSuccess) e = cudaMemcpyAsync(d + o_ref, s->d_ref, (size_t)h.ref_bytes, from_dev, cs);
   if (e == cudaSuccess) e = cudaMemcpyAsync(d + o_snm, s->d_snm, (size_t)h.snm_bytes, from_dev, cs);
   if (e == cudaSuccess)
-    e = cudaMemcpyAsync(d + o_st, ctx->d_stats + (size_t)s->slot * NSTAT, (size_t)h.stats_bytes, from_dev, cs);
+    e = cudaMemcpyAsync(d + o_st, ctx->d_stats + (size_t)s->slot * NSTAT, 8 * NSTAT, from_dev, cs);
+  std::vector<uint64_t> lat(NLAT);
+  {
+    std::lock_guard<std::mutex> lk2(ctx->lat_mu);
+    std::copy_n(ctx->h_lat.begin() + (std::ptrdiff_t)s->slot * NLAT, NLAT, lat.begin());
+  }
+  if (e == cudaSuccess)
+    e = cudaMemcpyAsync(d + o_st + 8 * NSTAT, lat.data(), 8 * NLAT,
+                        dst_is_host ? cudaMemcpyHostToHost : cudaMemcpyHostToDevice, cs);
   if (e == cudaSuccess) e = cudaStreamSynchronize(cs);  // hdr is a local buffer
   if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_stream_export");
   return FFSVA_OK;
@@ -456,7 +484,7 @@ FFSVA_API ffsva_status ffsva_stream_import(int32_t device, const void* src, int6
   if (h.magic != kImageMagic || h.version != kImageVersion) return fail(FFSVA_EINVAL, "not a stream image");
   h.desc.device = device;
   if (h.total != image_bytes(h.desc) || bytes < h.total || h.ref_bytes != 3LL * h.desc.sdd_w * h.desc.sdd_h ||
-      h.snm_bytes != snm::BLOB_BYTES || h.stats_bytes != 8LL * NSTAT)
+      h.snm_bytes != snm::BLOB_BYTES || h.stats_bytes != 8LL * FFSVA_NSTAT)
     return fail(FFSVA_EINVAL, "stream image sizes do not match its descriptor");
   ffsva_stream* s = nullptr;
   ffsva_status st = ffsva_open_stream(&h.desc, &s);  // validates the descriptor
@@ -471,7 +499,13 @@ FFSVA_API ffsva_status ffsva_stream_import(int32_t device, const void* src, int6
     const cudaMemcpyKind to_dev = src_is_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
     cudaError_t e = cudaMemcpy(s->d_ref, p + o_ref, (size_t)h.ref_bytes, to_dev);
     if (e == cudaSuccess) e = cudaMemcpy(s->d_snm, p + o_snm, (size_t)h.snm_bytes, to_dev);
-    if (e == cudaSuccess) e = cudaMemcpy(ctx->d_stats + (size_t)s->slot * NSTAT, p + o_st, (size_t)h.stats_bytes, to_dev);
+    if (e == cudaSuccess) e = cudaMemcpy(ctx->d_stats + (size_t)s->slot * NSTAT, p + o_st, 8 * NSTAT, to_dev);
+    if (e == cudaSuccess) {
+      std::vector<uint64_t> lat(NLAT);
+      e = cudaMemcpy(lat.data(), p + o_st + 8 * NSTAT, 8 * NLAT, src_is_host ? cudaMemcpyHostToHost : cudaMemcpyDeviceToHost);
+      std::lock_guard<std::mutex> lk2(ctx->lat_mu);
+      std::copy(lat.begin(), lat.end(), ctx->h_lat.begin() + (std::ptrdiff_t)s->slot * NLAT);
+    }
     if (e != cudaSuccess) {
       cuda_fail(ctx, e, "ffsva_stream_import");
       ok = false;

@@ -6,6 +6,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include "ffsva.h"
+
 namespace ffsva {
 
 // ------------------------------------------------------------------ per-frame descriptor (device, 64 B)
@@ -243,6 +245,8 @@ cudaError_t launch_fill_nan(float* p, int32_t n, cudaStream_t st);
 cudaError_t launch_reference(const uint8_t* frames, int32_t k, int64_t frame_stride, int32_t W, int32_t H,
                              int64_t pitch, int32_t sdd_w, int32_t sdd_h, uint8_t* out, cudaStream_t st);
 
-constexpr int NSTAT = 8;
+constexpr int NSTAT = 8;   // device statistics table stride (columns FFSVA_STAT_FRAMES .. FFSVA_STAT_SNM_BATCHES)
+constexpr int NLAT = 16;   // host latency columns per slot (FFSVA_STAT_DECIDED .. FFSVA_STAT_LAT_BIN0 + 13)
+static_assert(NSTAT + NLAT == FFSVA_NSTAT, "statistics row layout (include/ffsva.h)");
 
 }  // namespace ffsva

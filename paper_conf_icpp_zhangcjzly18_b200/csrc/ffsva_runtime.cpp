@@ -72,6 +72,7 @@ DeviceCtx* ctx_acquire(int device, ffsva_status* st) {
     c->device = device;
     c->num_sms = prop.multiProcessorCount;
     c->stats_cap = kMaxSlots;
+    c->h_lat.assign((size_t)kMaxSlots * NLAT, 0);
     if ((e = cudaMalloc(&c->d_stats, sizeof(unsigned long long) * NSTAT * kMaxSlots)) != cudaSuccess ||
         (e = cudaMemset(c->d_stats, 0, sizeof(unsigned long long) * NSTAT * kMaxSlots)) != cudaSuccess ||
         (e = cudaStreamCreateWithFlags(&c->copy_stream, cudaStreamNonBlocking)) != cudaSuccess ||
@@ -178,6 +179,23 @@ ffsva_status check_device_ptr(DeviceCtx* ctx, const void* p, size_t bytes) {
     ctx->range_mru = ctx->ranges.size() - 1;
   }
   return FFSVA_OK;
+}
+
+int latency_bin(int64_t us) {
+  if (us < 1000) return 0;
+  int k = 1;
+  for (int64_t ms = us / 1000; ms >= 2 && k < NLAT - 3; ms >>= 1) ++k;  // [2^(k-1), 2^k) ms -> k, capped at 13
+  return k;
+}
+
+void record_latency(DeviceCtx* ctx, int32_t slot, int64_t us) {
+  if (slot < 0 || slot >= ctx->stats_cap) return;
+  if (us < 0) us = 0;
+  std::lock_guard<std::mutex> lk(ctx->lat_mu);
+  uint64_t* row = ctx->h_lat.data() + (size_t)slot * NLAT;
+  row[0] += 1;
+  row[1] += (uint64_t)us;
+  row[2 + latency_bin(us)] += 1;
 }
 
 // ------------------------------------------------------------------ host arithmetic

@@ -77,7 +77,9 @@ struct DeviceCtx {
   int nstreams = 0;
   std::vector<int32_t> free_slots;
   int32_t next_slot = 0;
-  unsigned long long* d_stats = nullptr;  // [stats_cap][NSTAT]
+  unsigned long long* d_stats = nullptr;  // [stats_cap][NSTAT] (kernel counters)
+  std::mutex lat_mu;                      // guards h_lat (the online runtime records under its own lock)
+  std::vector<uint64_t> h_lat;            // [stats_cap][NLAT] (online arrival -> decision latency, a8)
   int32_t stats_cap = 0;
   bool sticky = false;
   Batch* scratch = nullptr;  // reusable batch for ffsva_filter_batch / ffsva_sdd_batch
@@ -109,6 +111,9 @@ ffsva_status check_device_ptr(DeviceCtx* ctx, const void* p, size_t bytes);
 void begin_ptr_checks(DeviceCtx* ctx);   // new validation epoch: cached ranges are re-confirmed once on next use
 void clear_ptr_cache(DeviceCtx* ctx);
 ffsva_status ensure_stats(DeviceCtx* ctx, int32_t slots);
+// a8: one decided frame of stream slot `slot` with arrival -> decision latency `us` (columns 8..23)
+void record_latency(DeviceCtx* ctx, int32_t slot, int64_t us);
+int latency_bin(int64_t us);
 uint64_t exact_threshold(double delta, uint64_t n_values);
 uint64_t exact_threshold_sq(double delta, uint64_t q);  // floor(delta^2 * q), exact (NRMSE, Q24)
 uint64_t stream_threshold(const ffsva_stream_desc& d, uint64_t ref_sum_sq);  // T of the stream's metric

@@ -22,6 +22,10 @@ using namespace ffsva;
 
 namespace {
 constexpr int64_t kD50Stride = 7504;
+int64_t now_us() {
+  return std::chrono::duration_cast<std::chrono::microseconds>(std::chrono::steady_clock::now().time_since_epoch())
+      .count();
+}
 size_t al256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 // Per-cycle staging: one pinned host block mirrored by one device block (a single H2D per stage).
@@ -220,6 +224,7 @@ void harvest_sdd(ffsva_sched* s, std::vector<sched::QFrame>& adm, int32_t na, ff
   const size_t n = (size_t)s->cap;
   const uint64_t* h_ssd = at<uint64_t>(s->h_out, 0);
   const uint8_t* h_pass = s->h_out + 12 * n;
+  const int64_t t_now = now_us();
   for (int32_t i = 0; i < na; ++i) {
     adm[i].ssd = h_ssd[i];
     s->pol.sdd_done(adm[i], h_pass[i] != 0);
@@ -236,6 +241,7 @@ void harvest_sdd(ffsva_sched* s, std::vector<sched::QFrame>& adm, int32_t na, ff
     ev.result.tyolo_count = -1;
     s->pending.push_back(ev);
     s->free_slots.push_back(adm[i].slot);
+    record_latency(s->ctx, ev.stream->slot, t_now - adm[i].t_push_us);
   }
 }
 
@@ -324,6 +330,7 @@ void harvest_snm(ffsva_sched* s, std::vector<sched::QFrame>& flat, int32_t m) {
   const float* h_logit = at<float>(s->h_out, 8 * n);
   const uint8_t* h_snm_pass = s->h_out + 13 * n;
   const uint8_t* h_snm_class = s->h_out + 14 * n;
+  const int64_t t_now = now_us();
   for (int32_t k = 0; k < m; ++k) {
     s->free_slots.push_back(flat[k].slot);
     flat[k].logit = h_logit[k];
@@ -340,6 +347,7 @@ void harvest_snm(ffsva_sched* s, std::vector<sched::QFrame>& flat, int32_t m) {
     ev.result.survivor_idx = -1;
     ev.result.tyolo_count = -1;
     s->pending.push_back(ev);
+    record_latency(s->ctx, ev.stream->slot, t_now - flat[k].t_push_us);
   }
 }
 
@@ -362,6 +370,7 @@ ffsva_status tyolo_cycle(ffsva_sched* s, cudaStream_t cs, ffsva_tick_info& ti) {
   ffsva_status ts = tyolo_run_unlocked(s->tyolo, fr.data(), nt, targets.data(), s->ty_thresh, 0, counts.data(),
                                        nullptr, nullptr, cs);
   if (ts != FFSVA_OK) return ts;
+  const int64_t t_now = now_us();
   for (int32_t i = 0; i < nt; ++i) {
     const ffsva_stream* st = s->by_id[tf[i].stream];
     ffsva_event ev{};
@@ -376,6 +385,7 @@ ffsva_status tyolo_cycle(ffsva_sched* s, cudaStream_t cs, ffsva_tick_info& ti) {
     ev.result.tyolo_count = counts[i];
     ev.result.tyolo_pass = counts[i] >= st->desc.number_of_objects ? 1 : 0;
     s->pending.push_back(ev);
+    record_latency(s->ctx, st->slot, t_now - tf[i].t_push_us);
   }
   return FFSVA_OK;
 }
@@ -472,6 +482,7 @@ FFSVA_API ffsva_status ffsva_sched_push(ffsva_sched* s, const ffsva_frame* frame
     if (st->desc.sdd_w != s->sdd_w || st->desc.sdd_h != s->sdd_h)
       return fail(FFSVA_EINVAL, "streams of one scheduler must share the SDD grid");
   }
+  const int64_t t_push = now_us();
   for (int32_t i = 0; i < n; ++i) {
     ffsva_stream* st = frames[i].stream;
     int32_t id = s->lookup(st);
@@ -485,6 +496,7 @@ FFSVA_API ffsva_status ffsva_sched_push(ffsva_sched* s, const ffsva_frame* frame
     sched::QFrame q;
     q.frame_no = frames[i].frame_no;
     q.pixels = frames[i].pixels;
+    q.t_push_us = t_push;
     accepted[i] = s->pol.push(id, q) ? 1 : 0;
   }
   return FFSVA_OK;
@@ -664,6 +676,41 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
   ti.snm_ms = std::chrono::duration<float, std::milli>(t_ty0 - t_snm0).count();
   ti.host_ms = std::chrono::duration<float, std::milli>(t_end - t_tick0).count();
   if (info) *info = ti;
+  return FFSVA_OK;
+}
+
+FFSVA_API ffsva_status ffsva_sched_inspect(ffsva_sched* s, ffsva_frame* frames, int32_t* stage, uint8_t* d50,
+                                           int32_t cap, int32_t* n) {
+  if (!s || !n || cap < 0 || (cap > 0 && (!frames || !stage || !d50))) return fail(FFSVA_EINVAL, "bad argument");
+  std::lock_guard<std::mutex> lk(s->mu);
+  DeviceCtx* ctx = s->ctx;
+  std::lock_guard<std::mutex> dlk(ctx->mu);
+  DeviceGuard g(ctx->device);
+  // the last launched cycle: synchronous mode keeps its admissions / pops in adm / flat; pipelined mode in f_adm /
+  // f_flat while in flight (their slots are freed only at the next tick's harvest)
+  const std::vector<sched::QFrame>* lists[2] = {&s->adm, &s->flat};
+  if (s->pipelined) {
+    if (!s->inflight) {
+      *n = 0;
+      return FFSVA_OK;
+    }
+    lists[0] = &s->f_adm;
+    lists[1] = &s->f_flat;
+  }
+  cudaError_t e = s->pipelined ? cudaEventSynchronize(s->done_ev) : cudaSuccess;
+  int32_t k = 0;
+  for (int st = 0; st < 2 && e == cudaSuccess; ++st)
+    for (const sched::QFrame& q : *lists[st]) {
+      if (k < cap) {
+        frames[k] = ffsva_frame{s->by_id[q.stream], (const uint8_t*)q.pixels, q.frame_no};
+        stage[k] = st;
+        e = cudaMemcpy(d50 + (size_t)k * 7500, s->d_pool + (size_t)q.slot * kD50Stride, 7500, cudaMemcpyDeviceToHost);
+        if (e != cudaSuccess) break;
+      }
+      ++k;
+    }
+  if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_inspect");
+  *n = k;
   return FFSVA_OK;
 }
 

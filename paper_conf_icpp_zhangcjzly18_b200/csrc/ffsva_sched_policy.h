@@ -46,6 +46,7 @@ struct QFrame {
   uint64_t ssd = 0;           // SDD distance, carried to the frame's final event
   float logit = 0.f;          // SNM result, carried through the T-YOLO queue
   uint8_t snm_class = 0;
+  int64_t t_push_us = 0;      // steady-clock microseconds when the push was accepted (a8 latency)
 };
 
 enum class BatchPolicy : int32_t { DYNAMIC = 0, FEEDBACK = 1, STATIC = 2 };

@@ -21,7 +21,11 @@ LIB_PATH = os.environ.get("FFSVA_LIB", os.path.join(_HERE, "lib", "libffsva.so")
 FFSVA_OK, FFSVA_EINVAL, FFSVA_ENOMEM, FFSVA_ECUDA, FFSVA_ESTATE, FFSVA_EAGAIN, FFSVA_EDEVICE = 0, -1, -2, -3, -4, -5, -6
 STATUS_NAMES = {0: "FFSVA_OK", -1: "FFSVA_EINVAL", -2: "FFSVA_ENOMEM", -3: "FFSVA_ECUDA", -4: "FFSVA_ESTATE",
                 -5: "FFSVA_EAGAIN", -6: "FFSVA_EDEVICE"}
-STAT_NAMES = ["frames", "sdd_pass", "snm_pass", "ssd_sum", "class0", "class1", "class2", "snm_batches"]
+STAT_NAMES = (["frames", "sdd_pass", "snm_pass", "ssd_sum", "class0", "class1", "class2", "snm_batches", "decided",
+               "lat_sum_us"] + [f"lat_bin{k}" for k in range(14)])  # include/ffsva.h FFSVA_STAT_*
+LAT_BIN0 = 10
+# latency bin k covers [LAT_EDGES_MS[k], LAT_EDGES_MS[k + 1]) milliseconds (bin 0 < 1 ms, bin 13 >= 4096 ms)
+LAT_EDGES_MS = [0.0] + [float(2 ** (k - 1)) for k in range(1, 14)] + [float("inf")]
 NSTAT = len(STAT_NAMES)
 
 # Every symbol include/ffsva.h declares (checked by tests/test_abi.py).
@@ -35,7 +39,7 @@ EXPORTS = ["ffsva_open_stream", "ffsva_set_reference", "ffsva_snm_load", "ffsva_
            "ffsva_stream_export",
            "ffsva_stream_import", "ffsva_sched_stream_load", "ffsva_sched_detach", "ffsva_tyolo_load",
            "ffsva_tyolo_run", "ffsva_tyolo_layer_output", "ffsva_tyolo_profile", "ffsva_tyolo_destroy",
-           "ffsva_sched_set_tyolo"]
+           "ffsva_sched_set_tyolo", "ffsva_sched_inspect"]
 
 
 class StreamDesc(ctypes.Structure):
@@ -146,6 +150,7 @@ def lib():
             "ffsva_tyolo_profile": [vp, vp, i32, i32, vp, vp],
             "ffsva_tyolo_destroy": [vp],
             "ffsva_sched_set_tyolo": [vp, vp, i32, ctypes.c_float],
+            "ffsva_sched_inspect": [vp, vp, vp, vp, i32, ctypes.POINTER(i32)],
         }
         for name, args in sig.items():
             fn = getattr(L, name)
@@ -545,6 +550,18 @@ class Scheduler:
             return False
         _check(r, "ffsva_sched_set_pipeline")
         return True
+
+    def inspect(self, cap: int = 1 << 16) -> dict:
+        """ffsva_sched_inspect: the last launched cycle's frames (stage 0 = SDD admission, 1 = SNM pop) and the
+        50x50x3 image each holds in the device slot pool."""
+        frames = np.zeros(max(1, cap), dtype=FRAME_DTYPE)
+        stage = np.zeros(max(1, cap), np.int32)
+        d50 = np.zeros((max(1, cap), 50, 50, 3), np.uint8)
+        n = ctypes.c_int32()
+        _check(lib().ffsva_sched_inspect(self.handle, frames.ctypes.data, stage.ctypes.data, d50.ctypes.data, cap,
+                                         ctypes.byref(n)), "ffsva_sched_inspect")
+        k = min(n.value, cap)
+        return {"frames": frames[:k], "stage": stage[:k], "d50": d50[:k], "n": n.value}
 
     def destroy(self) -> None:
         if self.handle:

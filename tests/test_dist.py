@@ -22,7 +22,7 @@ def test_shard_streams_partition():
 
 
 def test_summarize():
-    st = np.zeros((3, 8), np.int64)
+    st = np.zeros((3, 24), np.int64)
     st[:, 0] = [30, 30, 30]
     st[:, 1] = [3, 0, 6]
     st[:, 2] = [1, 0, 3]
@@ -33,6 +33,11 @@ def test_summarize():
     assert abs(s["sdd_pass_ratio"] - 0.1) < 1e-12 and abs(s["snm_pass_ratio"] - 4 / 9) < 1e-12
     assert abs(s["mean_mse"] - 10 / 90) < 1e-12
     assert s["snm_batches"] == 2
+    # latency columns (include/ffsva.h: 8 decided, 9 sum us, 10.. bins; bin 0 < 1 ms, bin k in [2^(k-1), 2^k) ms)
+    st[0, 8], st[0, 9], st[0, 10 + 0], st[0, 10 + 3] = 4, 3 * 500 + 5000, 3, 1   # 3 x 0.5 ms + 1 x 5 ms
+    s = fdist.summarize(st)
+    assert s["decided"] == 4 and abs(s["latency_mean_ms"] - 6.5 / 4) < 1e-12
+    assert s["latency_p50_ms_le"] == 1.0 and s["latency_p99_ms_le"] == 8.0
 
 
 def _free_port():

@@ -172,7 +172,7 @@ def test_snm_parity_interleaved_streams(env):
     surv = want["survivors"]
     assert surv.size == sum(synth.planted(c.video, c.sid, 0, 20) for c in cams)
     camlist = [c for c, _ in pairs]
-    err = check_snm(got["logit"], got["snm_pass"], got["snm_class"], want["logit"], camlist, surv, SNM_TOL)
+    err, nd = check_snm(got["logit"], got["snm_pass"], got["snm_class"], want["logit"], camlist, surv, SNM_TOL)
     want16 = oracle_for(pairs, bf16_emul=True)
     err16 = np.abs(got["logit"][surv] - want16["logit"][surv]).max()
     assert err16 <= SNM_TOL_BF16, err16
@@ -287,23 +287,32 @@ def test_prepared_batch_graph_replay_and_host_path(env):
 
 
 def test_stats_counters(env):
+    """a8 (L253 Fig. 5: per-filter frame ratios): the per-stream statistics rows against counts derived from the
+    ORACLE's per-frame results on the same frames (not from the GPU's own results). The SNM-pass and class counts
+    are exact unless an oracle logit lies within the 2e-2 margin of a threshold (asserted absent here)."""
     ff, ctx, dev = env
     cams = [Cam(ctx, synth.Video(seed=51, width=640, height=360, period=10, on_len=4), s, dev, snm_batch=3, k_ref=2)
             for s in range(2)]
     ctx.stats(reset=True)
     pairs = [(c, c.host_frames([t])[0]) for t in range(10) for c in cams]
-    got = _run_full(ctx, dev, pairs)
+    _run_full(ctx, dev, pairs)
     st = ctx.stats()
+    want = oracle_for(pairs)
     for c in cams:
         idx = np.array([i for i, (cc, _) in enumerate(pairs) if cc is c])
         row = st[c.st.slot]
+        surv = idx[want["sdd_pass"][idx] == 1]
+        lt = orc.logit(orc.tpre(f32(c.c_low), f32(c.c_high), f32(c.fd)))
+        for th in (lt, orc.logit(f32(c.c_low)), orc.logit(f32(c.c_high))):
+            assert np.all(np.abs(want["logit"][surv] - th) > SNM_TOL), "a logit within the margin: counts not exact"
         assert row[0] == idx.size
-        assert row[1] == got["sdd_pass"][idx].sum()
-        assert row[2] == got["snm_pass"][idx].sum()
-        assert row[3] == got["ssd"][idx].sum()
-        assert row[4] + row[5] + row[6] == got["sdd_pass"][idx].sum()
-        q = int(got["sdd_pass"][idx].sum())
-        assert row[7] == (q + 2) // 3  # dynamic batches of <= BatchSize 3 (L223)
+        assert row[1] == int(want["sdd_pass"][idx].sum()) == synth.planted(c.video, c.sid, 0, 10)
+        assert row[2] == int(want["snm_pass"][idx].sum())
+        assert row[3] == int(want["ssd"][idx].astype(np.uint64).sum())
+        for k in range(3):
+            assert row[4 + k] == int((want["snm_class"][surv] == k).sum())
+        assert row[7] == (surv.size + 2) // 3  # dynamic batches of <= BatchSize 3 (L223)
+        assert np.all(row[8:] == 0)  # latency columns belong to the online runtime
     for c in cams:
         c.st.close()
 
@@ -319,45 +328,6 @@ def test_synth_device_generator_matches_host(env):
     torch.cuda.synchronize()
     want = synth.frames(v, [0, 1, 2, 5], [0, 3, 4, 100])
     assert np.array_equal(out.cpu().numpy(), want)
-
-
-def test_full_size_config2_sampled(env):
-    """Config 2 at full size in the bench's launch configuration: 30 streams x 30 frames of 720p (one second of
-    video), prepared batch + graph replay. Property at full size: SDD pass count == planted count; sampled
-    frames checked element by element against the oracle."""
-    ff, ctx, dev = env
-    import torch
-    S, F, W, H = 30, 30, 1280, 720
-    v = synth.Video(seed=1002, width=W, height=H, period=300, on_len=30)
-    cams = [Cam(ctx, v, s, dev, k_ref=8, snm_batch=30) for s in range(S)]
-    sid = torch.arange(S, dtype=torch.int32, device=dev).repeat_interleave(F)
-    t0 = 120
-    ts = (torch.arange(F, dtype=torch.int64, device=dev) + t0).repeat(S)
-    pool = torch.empty((S * F, H, 3 * W), dtype=torch.uint8, device=dev)
-    synth.frames_cuda(v, sid, ts, pool, H * 3 * W, 3 * W)
-    torch.cuda.synchronize()
-    items = [(cams[i // F].st, pool[i], t0 + i % F) for i in range(S * F)]
-    pb = ctx.prepare(items)
-    s = torch.cuda.Stream()
-    pb.launch(s)
-    pb.launch(s)
-    got = pb.fetch(s)
-    planted = sum(synth.planted(v, k, t0, t0 + F) for k in range(S))
-    assert int(got["sdd_pass"].sum()) == planted
-    sid_h, ts_h = sid.cpu().numpy(), ts.cpu().numpy()
-    for i in range(S * F):
-        assert got["sdd_pass"][i] == int(synth.is_target(v, int(sid_h[i]), int(ts_h[i])))
-    sample = [i for i in range(S * F) if i % 61 == 0] + [int(i) for i in np.flatnonzero(got["sdd_pass"])[:8]]
-    for i in sample:
-        c = cams[i // F]
-        h = c.host_frames([int(ts_h[i])])[0]
-        w = oracle_for([(c, h)])
-        assert int(got["ssd"][i]) == int(w["ssd"][0])
-        if w["sdd_pass"][0]:
-            assert abs(got["logit"][i] - w["logit"][0]) <= SNM_TOL
-    pb.destroy()
-    for c in cams:
-        c.st.close()
 
 
 def test_k1_shared_memory_limit_in_fresh_process():

@@ -27,14 +27,18 @@ def env():
     ctx.close()
 
 
-@pytest.mark.parametrize("pipeline", [False, True])
-def test_online_feedback_queue_and_dynamic_batching(env, pipeline):
-    """Synchronous and pipelined ticks (ffsva_sched_set_pipeline): same per-frame results, every frame once."""
+@pytest.mark.parametrize("pipeline,W,H", [(False, 640, 360), (True, 640, 360), (False, 1280, 720),
+                                          (True, 1280, 720)])
+def test_online_feedback_queue_and_dynamic_batching(env, pipeline, W, H):
+    """Synchronous and pipelined ticks (ffsva_sched_set_pipeline): same per-frame results, every frame once. The
+    SNM's input in the online runtime is the device slot pool: after every tick, the image every admitted frame
+    got (K1 -> its slot) and the image every popped frame is scored from (possibly written cycles earlier) are read
+    back (ffsva_sched_inspect) and compared with the oracle's 50x50 resize byte for byte."""
     ff, ctx, dev = env
     import torch
     from paper_conf_icpp_zhangcjzly18_b200.ffsva import Scheduler
     q_sdd, q_snm, B = 2, 3, 1
-    v = synth.Video(seed=61, width=640, height=360, period=10, on_len=5)
+    v = synth.Video(seed=61, width=W, height=H, period=10, on_len=5)
     cams = []
     for s in range(3):
         c = Cam(ctx, v, s, dev, k_ref=2, snm_batch=B)
@@ -42,14 +46,18 @@ def test_online_feedback_queue_and_dynamic_batching(env, pipeline):
     # rebuild the streams with the online thresholds (Cam opens with the defaults)
     for c in cams:
         c.st.close()
-        c.st = ctx.open_stream(width=640, height=360, delta_diff=24.0, snm_batch=B, q_sdd=q_sdd, q_snm=q_snm)
+        c.st = ctx.open_stream(width=W, height=H, delta_diff=24.0, snm_batch=B, q_sdd=q_sdd, q_snm=q_snm)
         c.st.set_reference(torch.from_numpy(c.refs).to(dev))
         c.st.snm_load(c.params)
     T = 24
     host = {s: c.host_frames(list(range(T))) for s, c in enumerate(cams)}
     dev_frames = {s: torch.from_numpy(host[s]).to(dev) for s in host}
+    want_d50 = {(s, t): orc.box_downsample(host[s][t], W, 50, 50) for s in host for t in range(T)}
+    at_ptr = {dev_frames[s][t].data_ptr(): (s, t) for s in host for t in range(T)}
+    checked = {0: 0, 1: 0}
     sched = Scheduler(ctx, max_frames_per_tick=64, snm_slots=64)
     assert sched.set_pipeline(pipeline)
+    ctx.stats(reset=True)
     # pipelined: a cycle's survivors join the SNM queue one tick later, after the next admission check
     snm_slack = 6 if pipeline else 3
     handle_to_s = {c.st.handle: s for s, c in enumerate(cams)}
@@ -70,6 +78,13 @@ def test_online_feedback_queue_and_dynamic_batching(env, pipeline):
                     backlog[handle_to_s[st.handle]].remove(t)
         ev, info = sched.tick(cs)
         blocked += info["sdd_blocked"]
+        cyc = sched.inspect()
+        assert (cyc["stage"] == 0).sum() == info["admitted"] and (cyc["stage"] == 1).sum() == info["snm_scored"]
+        for fr, stg, img in zip(cyc["frames"], cyc["stage"], cyc["d50"]):
+            key = at_ptr[int(fr["pixels"])]
+            assert int(fr["frame_no"]) == key[1]
+            assert np.array_equal(img, want_d50[key]), ("slot-pool D50 differs", stg, key)
+            checked[int(stg)] += 1
         for c in cams:
             d_sdd, d_snm = sched.depth(c.st)
             assert d_sdd <= q_sdd + 1, "SDD queue grew past its threshold + 1"
@@ -83,11 +98,21 @@ def test_online_feedback_queue_and_dynamic_batching(env, pipeline):
             break
     sched.destroy()
     assert len(got) == 3 * T, f"{len(got)} of {3 * T} frames reported"
+    n_surv = sum(int(synth.is_target(v, s, t)) for s in range(3) for t in range(T))
+    assert checked[0] == 3 * T and checked[1] == n_surv > 0, checked  # every admission, every pop
+    # a8 statistics of the online runtime: kernel counters vs the oracle-derived schedule, and the latency
+    # histogram (one entry per reported frame; push -> report within this test's wall time)
+    st = ctx.stats()
+    for s_, c in enumerate(cams):
+        row = st[c.st.slot]
+        assert row[0] == T and row[1] == sum(int(synth.is_target(v, s_, t)) for t in range(T))
+        assert row[8] == T and int(row[10:24].sum()) == T, row
+        assert 0 < row[9] <= T * 600e6
     assert refused > 0, "the SDD-queue threshold never refused a push"
     assert blocked > 0, "the SNM-queue threshold never blocked the SDD stage"
     for (s, t), r in got.items():
         c = cams[s]
-        w = orc.filter_frames([host[s][t]], 640, [c.R], [24.0], [c.params], [f32(0.2)], [f32(0.8)], [f32(0.5)])
+        w = orc.filter_frames([host[s][t]], W, [c.R], [24.0], [c.params], [f32(0.2)], [f32(0.8)], [f32(0.5)])
         assert int(r["ssd"]) == int(w["ssd"][0]), (s, t)
         assert int(r["sdd_pass"]) == int(w["sdd_pass"][0]), (s, t)
         assert r["sdd_pass"] == int(synth.is_target(v, s, t))

@@ -210,3 +210,22 @@ def test_scheduler_rejects_previous_mode(env):
     assert L.ffsva_sched_push(h, fr, 1, acc) == ffb.FFSVA_EINVAL
     assert L.ffsva_sched_destroy(h) == ffb.FFSVA_OK
     cam.st.close()
+
+
+@pytest.mark.parametrize("metric", ["mse", "sad"])
+def test_previous_frame_mode_large_grid_no_wrap(env, metric):
+    """PREVIOUS mode on a 1000x1000 SDD grid (one CTA per frame in K2): a black frame after a white one gives
+    SSD = 3e6 * 255^2 = 1.95e11 (MSE) or 3e6 * 255 (SAD), far beyond 32 bits — the distance must not wrap."""
+    import torch
+    ff, ctx, dev = env
+    W = H = 1000
+    st = ctx.open_stream(width=W, height=H, delta_diff=0.0, sdd=(1000, 1000), ref_mode="previous", distance=metric)
+    white = np.full((H, 3 * W), 255, np.uint8)
+    st.set_reference(torch.from_numpy(white[None]).to(dev))
+    frames = torch.from_numpy(np.stack([np.zeros((H, 3 * W), np.uint8), white, white])).to(dev)
+    got = ctx.sdd_batch([(st, frames[i], i) for i in range(3)], want_d100=False)
+    n = 3 * W * H
+    big = n * (255 * 255 if metric == "mse" else 255)
+    assert [int(x) for x in got["ssd"]] == [big, big, 0]
+    assert [int(x) for x in got["sdd_pass"]] == [1, 1, 0]
+    st.close()
