@@ -241,13 +241,15 @@ def solo_fps(eng, steps: int, rank: int) -> float:
     return _allreduce(fps, "max", eng.device)
 
 
-def scaling_fields(value: float, fps1: float, ws: int, g_us: float, gathered_rows: int, strong: bool) -> dict:
+def scaling_fields(value: float, fps1: float, ws: int, g_us: float, gathered_rows: int, strong: bool,
+                   backend: str = "nccl") -> dict:
     return {"kind": "strong" if strong else "weak", "n_gpus": ws, "fps_1gpu": fps1,
             "efficiency": value / (ws * fps1) if fps1 > 0 else None,
             "efficiency_def": "fps(G) / (G * fps(1)); fps(1) = the N = 1 workload timed on rank 0 of this run "
                               "(strong: all streams on one GPU; weak: one rank's streams)",
             "stats_gather_us": g_us, "stats_gather_rows": gathered_rows,
-            "stats_gather": "NCCL all_gather_into_tensor of the u64 per-stream table (device time, max over ranks)"}
+            "stats_gather": ("NCCL all_gather_into_tensor" if backend == "nccl" else "gloo all_gather (host copies)")
+                            + " of the u64 per-stream table (device time, max over ranks)"}
 
 
 # ---------------------------------------------------------------------------------------------- our arm
@@ -390,6 +392,10 @@ def run_ours(args, cfg, ws, rank, local):
     torch.cuda.set_device(dev)
     eng = GpuEngine(args, cfg, ws, rank, dev)
     eng.gate()
+    # torch's current stream = the launching stream, so the statistics copy, the all-gather (NCCL orders its work
+    # after the current stream) and the closing timer mark are ordered on one stream
+    cur = torch.cuda.stream(eng.cs)
+    cur.__enter__()
     launches0 = ff.ffsva_kernel_launches()
     ms_max, total_frames, gathered, clk = timed_region(eng, args.steps, args.warmup)
     launches = ff.ffsva_kernel_launches() - launches0
@@ -400,7 +406,8 @@ def run_ours(args, cfg, ws, rank, local):
         raise RuntimeError("gathered per-stream frame counters disagree with the frames launched")
     g_us = gather_us(eng) if ws > 1 else 0.0
     fps1 = solo_fps(eng, max(3, min(args.steps, 50)), rank) if ws > 1 else value
-    scaling = scaling_fields(value, fps1, ws, g_us, int(g.shape[0]), eng.strong)
+    cur.__exit__(None, None, None)
+    scaling = scaling_fields(value, fps1, ws, g_us, int(g.shape[0]), eng.strong, args.dist_backend)
 
     # ---- per-kernel device times (CUDA events on the launching stream) for the roofline
     batches, nbatches, cs = eng.batches, eng.nbatches, eng.cs

@@ -147,3 +147,12 @@ def test_timed_region_world2_strong():
     assert tot0 == tot1 == 256 * 10 * 5                      # the whole stream set, split
     assert np.all(g0[:, 0] == 10 * 8) and np.array_equal(g0[:, 1], np.arange(256) * 8)
     assert _r0[-1]["kind"] == "strong"
+
+
+def test_timed_region_single_process_without_group():
+    """N = 1 (no process group at all): the same skeleton must run without torch.distributed initialised."""
+    eng = HostEngine(bench.CONFIGS["m2"], 1, 0, delay=0.001)
+    ms, total, gathered, _ = bench.timed_region(eng, steps=4, warmup=3)
+    assert total == 30 * 30 * 4 and ms >= 4.0
+    assert gathered.shape == (30, NSTAT) and np.all(gathered.numpy()[:, 0] == 30 * 7)
+    assert bench.gather_us(eng, reps=2) >= 0

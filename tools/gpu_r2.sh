@@ -11,11 +11,11 @@ if [ -z "$SKIP_TESTS" ]; then
   tail -30 gpurun_out/pytest_gpu.log
   timeout 300 python __graft_entry__.py smoke > gpurun_out/smoke.log 2>&1; echo "smoke rc=$?"; tail -3 gpurun_out/smoke.log
 fi
-B=${BENCH:---steps 40 --warmup 5 --online ""}
+B=${BENCH:---steps 40 --warmup 5 --online=}
 timeout 900 python bench.py $B > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?"
 cut -c1-1500 gpurun_out/bench.json; tail -5 gpurun_out/bench.err
 if [ -z "$SKIP_DIST" ]; then
-  timeout 900 python bench.py --gpus 2 --dist-backend gloo --steps 20 --warmup 3 --online "" --no-cpu-baseline \
+  timeout 900 python bench.py --gpus 2 --dist-backend gloo --steps 20 --warmup 3 --online= --no-cpu-baseline \
     > gpurun_out/bench_g2.json 2> gpurun_out/bench_g2.err; echo "bench g2 rc=$?"
   cut -c1-1500 gpurun_out/bench_g2.json; tail -5 gpurun_out/bench_g2.err
   timeout 900 python bench.py --gpus 2 --dist-backend gloo --config m5 --steps 10 --warmup 3 --no-cpu-baseline \
