@@ -93,6 +93,12 @@ class ClockSampler:
             return
         self.th = threading.Thread(target=self._read, daemon=True)
         self.th.start()
+        # nvidia-smi's NVML start-up stalls GPU work for tens of ms: the timed region starts only after its first
+        # sample (measured: a 40-step M1 region absorbed a ~100 ms stall otherwise)
+        t0 = time.perf_counter()
+        while not self.rows and time.perf_counter() - t0 < 10.0 and self.proc.poll() is None:
+            time.sleep(0.02)
+        time.sleep(0.25)
 
     def _read(self):
         for line in self.proc.stdout:
@@ -370,7 +376,6 @@ class GpuEngine:
     def start_clocks(self):
         self.clocks = ClockSampler(self.dev.index)
         self.clocks.start()
-        time.sleep(0.3)
 
     def stop_clocks(self):
         return self.clocks.stop() if self.clocks else None

@@ -71,6 +71,11 @@ struct SddArgs {
   const int32_t* ybounds;    // [sdd_h + 1] floor(i*uni_H/sdd_h) for frames of height uni_H, or nullptr
   int32_t uni_W, uni_H;
   int32_t cellw;             // widest 100-grid cell of uni_W-wide frames, ceil(uni_W / sdd_w) (0 if mixed)
+  bool seg;                  // bulk: the warp-segment pipeline kernel (narrow rows)
+  int32_t max_cellw;         // widest 100-grid cell over the batch
+  int32_t max_rows100;       // tallest 100-grid row (source rows) over the batch
+  int32_t magic_n;           // warp-segment kernel: entries of its box-area reciprocal table
+  int32_t min_cellw;         // narrowest 100-grid cell over the batch (floor(min W / sdd_w))
 };
 
 // K1 variant choice for one batch (sdd_plan_add per frame, then sdd_plan_finish): the bulk-async CTA-pair kernel
@@ -79,8 +84,12 @@ struct SddArgs {
 enum SddVariant : int32_t { kSddStream = 0, kSddPair = 1 };
 struct SddPlan {
   int32_t max_chunks = 1, pair_stage = 0;
+  int32_t seg_stage = 0;     // warp-segment kernel: max bytes of one 50-grid row's source rows
+  int32_t max_rows100 = 0, max_w = 0;  // tallest 100-grid row (source rows), widest frame
+  int32_t min_w = 0;         // narrowest frame
   bool vec16 = true;
   int32_t variant = kSddStream, stage_bytes = 0;
+  bool seg = false;
   size_t smem = 0;
 };
 void sdd_plan_add(SddPlan& p, int32_t W, int32_t H, int64_t pitch, const void* pixels, int32_t sdd_h);

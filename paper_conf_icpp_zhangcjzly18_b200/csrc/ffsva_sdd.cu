@@ -24,6 +24,7 @@
 #include <cooperative_groups.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 
@@ -542,6 +543,255 @@ __global__ void __launch_bounds__(256, 8) sdd_band2_kernel_impl(SddArgs a, bool 
   ssd_commit(ssd_local, red, a, f, fd.slot, b == 0);
 }
 
+// ------------------------------------------------------------------ narrow rows: warp-segment pipeline
+// K1 for rows of <= 128 16-byte chunks (360p) without CTA barriers. A persistent CTA = one producer warp + kG
+// groups of kSegWarps consumer warps; the producer bulk-copies the CTA's units (frame, 50-grid row = two 100-grid rows)
+// into a kNS-stage ring (full / empty mbarriers), group g consumes units g, g + kG, ... Within a group, warp w owns
+// a horizontal segment of the 50-grid row (50-cells [k0, k1), at most 10) and does all of its work alone:
+//   column phase — lane = 16-byte chunk of the segment's window (<= 32 chunks), packed 2 x 16-bit vertical sums of
+//                  each 100-grid row's source rows into a warp-private u16 column-sum row;
+//   cell phase   — lane = 100-grid cell of the segment, all three channels at once from u32 pairs of column sums
+//                  (absolute word w holds columns 2w, 2w+1, so w mod 3 fixes its channels: residue 0 = (c0, c1),
+//                  1 = (c2, c0), 2 = (c1, c2); a lone edge column is added alone), box means by multiply-high
+//                  (magic table: floor(2^32 / n) + 1, exact while sum * n < 2^32), D100 (optional), distance to R;
+//   D50          — each lane sums its cell over the two rows, the horizontal pair is one shuffle, even lanes emit
+//                  the 50-cell (Q8);
+// then lane 0 releases the stage (empty mbarrier, one arrival per warp). Warps only ever wait for data, never for
+// each other. The distance accumulates per lane over a warp's consecutive units of one frame and is reduced with one
+// atomic per warp and frame.
+constexpr int kSegWarps = 5;   // consumer warps per unit (half_w <= 50: at most 10 50-cells per warp)
+
+// kMinB CTAs per SM (register cap); a cell spans between kW0 and kW1 u32 words of column sums (kW0 loads need no
+// predicate); a 100-grid row has at most kMaxRows source rows. Boxes of one pixel are excluded by the host (the
+// magic table's n = 1 entry is not used).
+template <int kG, int kNS, int kMinB, int kW0, int kW1, int kMaxRows>
+__global__ void __launch_bounds__(32 * (kG * kSegWarps + 1), kMinB) sdd_seg_kernel(SddArgs a) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ __align__(8) uint64_t full[kNS], empty[kNS];
+  __shared__ int ybnd[kNS][3];  // source-row bounds of the unit's two 100-grid rows (frame rows)
+  __shared__ int unit_f[kNS], unit_b[kNS], unit_roff[kNS];
+  const int sdd_w = a.sdd_w, sdd_h = a.sdd_h, half_w = sdd_w >> 1;
+  constexpr int kCons = kG * kSegWarps;
+  // a stage = the unit's source rows, then (at r_base) the 16-byte aligned span holding its two rows of R
+  const int r_base = a.stage_bytes - ((6 * sdd_w + 31) & ~15);
+  uint8_t* stage = smem;                                                                    // [kNS][stage_bytes]
+  uint16_t* colsum = reinterpret_cast<uint16_t*>(smem + (size_t)kNS * a.stage_bytes);       // [kCons][2][512]
+  uint32_t* magic = reinterpret_cast<uint32_t*>(colsum + kCons * 2 * 512);                  // [magic_n]
+  const int nb = sdd_h >> 1;  // units per frame
+  const int64_t U = (int64_t)a.n * nb;
+  const int64_t u_begin = (int64_t)blockIdx.x * U / gridDim.x;
+  const int n_units = (int)((int64_t)(blockIdx.x + 1) * U / gridDim.x - u_begin);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+  if (threadIdx.x == 0) {
+    for (int st = 0; st < kNS; ++st) {
+      ptx::mbar_init((uint32_t)__cvta_generic_to_shared(&full[st]), 1);
+      ptx::mbar_init((uint32_t)__cvta_generic_to_shared(&empty[st]), kSegWarps);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  for (int n = threadIdx.x; n < a.magic_n; n += blockDim.x)
+    magic[n] = n > 1 ? 0xFFFFFFFFu / (uint32_t)n + 1u : (uint32_t)n;
+  __syncthreads();  // the only CTA barrier: mbarrier init + magic table
+
+  if (warp == kCons) {
+    // ---------------- producer warp (lane 0): the CTA's units in order through the stage ring
+    if (lane == 0) {
+      int fi = (int)(u_begin / nb), bi = (int)(u_begin - (int64_t)fi * nb);
+      uint64_t pol;
+      asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+      for (int i = 0; i < n_units; ++i) {
+        const int st = i % kNS;
+        if (i >= kNS) ptx::mbar_wait((uint32_t)__cvta_generic_to_shared(&empty[st]), (uint32_t)((i / kNS - 1) & 1));
+        const FrameDesc& fd = a.frames[fi];
+        const int H = fd.H, rb16 = (3 * fd.W + 15) & ~15;
+        int y[3];
+#pragma unroll
+        for (int j = 0; j < 3; ++j)
+          y[j] = a.ybounds ? __ldg(a.ybounds + 2 * bi + j) : (int)(((uint32_t)(2 * bi + j) * (uint32_t)H) / (uint32_t)sdd_h);
+        ybnd[st][0] = y[0];
+        ybnd[st][1] = y[1];
+        ybnd[st][2] = y[2];
+        unit_f[st] = fi;
+        unit_b[st] = bi;
+        if (bi == 0 && a.stats) atomicAdd(a.stats + (int64_t)fd.slot * NSTAT + 0, 1ull);
+        const int rows = y[2] - y[0];
+        // the unit's rows of R (L2-resident, 600 B at the default grid) ride along in the same stage
+        const int r0 = 2 * bi * 3 * sdd_w, r16 = r0 & ~15;
+        const int rbytes = (r0 - r16 + 6 * sdd_w + 15) & ~15;
+        unit_roff[st] = r0 - r16;
+        const uint32_t bar = (uint32_t)__cvta_generic_to_shared(&full[st]);
+        mbar_expect_tx(bar, (uint32_t)(rows * rb16 + rbytes));  // release: the unit's ybnd / unit_* writes above
+        const uint32_t dst = (uint32_t)__cvta_generic_to_shared(stage + (size_t)st * a.stage_bytes);
+        ptx::bulk_g2s_hint(dst + r_base, fd.ref + r16, (uint32_t)rbytes, bar, pol);
+        const uint8_t* src = fd.pixels + (int64_t)y[0] * fd.pitch;
+        if (fd.pitch == rb16) {
+          ptx::bulk_g2s_hint(dst, src, (uint32_t)(rows * rb16), bar, pol);
+        } else {
+          for (int yy = 0; yy < rows; ++yy)
+            ptx::bulk_g2s_hint(dst + yy * rb16, src + (int64_t)yy * fd.pitch, (uint32_t)rb16, bar, pol);
+        }
+        if (++bi == nb) {
+          bi = 0;
+          ++fi;
+        }
+      }
+    }
+    return;
+  }
+
+  // ---------------- consumer warps
+  const int g = warp / kSegWarps, ws = warp - g * kSegWarps;
+  const int k0 = ws * half_w / kSegWarps, k1 = (ws + 1) * half_w / kSegWarps;  // this warp's 50-cells
+  const int ncell = 2 * (k1 - k0);                                             // 100-cells per row
+  uint16_t* cs_w = colsum + (size_t)warp * 2 * 512;                            // [2][512] this warp's column sums
+  // per frame width (recomputed when it changes): the window's first chunk, this lane's cell's word range
+  int cur_w = -1, win_c0 = 0, win_n = 0;
+  int c_word = 0, c_nw = 0, c_q = 0, c_e0 = -1, c_e2 = -1;  // relative word index, count, residue, lone columns
+  uint32_t c_wd = 0, c_w50 = 0;                             // cell width, its 50-cell's width (pixels)
+  int cur_f = -1, cur_slot = 0;
+  uint8_t cur_mode = 0, cur_metric = 0;
+  const uint8_t* cur_ref = nullptr;
+  uint8_t* cur_d50 = nullptr;
+  uint32_t ssd_acc = 0;
+  const int cx = 2 * k0 + lane;  // this lane's 100-grid cell column (valid if lane < ncell)
+  const bool has_cell = lane < ncell;
+
+  for (int i = g; i < n_units; i += kG) {
+    const int st = i % kNS;
+    const uint32_t fb = (uint32_t)__cvta_generic_to_shared(&full[st]);
+    ptx::mbar_wait(fb, (uint32_t)((i / kNS) & 1));
+    const int f = unit_f[st], b = unit_b[st], roff = unit_roff[st];
+    const int y0 = ybnd[st][0], y1 = ybnd[st][1], y2 = ybnd[st][2];
+    if (f != cur_f) {  // warp-uniform
+      if (cur_f >= 0) {
+        uint32_t v = ssd_acc;
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+        if (lane == 0 && v) {
+          atomicAdd(a.acc_ssd + cur_f, (unsigned long long)v);
+          if (a.stats) atomicAdd(a.stats + (int64_t)cur_slot * NSTAT + 3, (unsigned long long)v);
+        }
+        ssd_acc = 0;
+      }
+      cur_f = f;
+      const FrameDesc& fd = a.frames[f];
+      cur_slot = fd.slot;
+      cur_mode = fd.mode;
+      cur_metric = fd.metric;
+      cur_ref = fd.ref;
+      cur_d50 = a.d50 + (a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f) * a.d50_stride;
+      const int W = fd.W;
+      if (W != cur_w) {
+        auto xbd = [&](int c) { return (int)(((uint32_t)c * (uint32_t)W) / (uint32_t)sdd_w); };
+        const int X0 = xbd(2 * k0), X1 = xbd(2 * k1);
+        win_c0 = (3 * X0) >> 4;
+        win_n = ((3 * X1 + 15) >> 4) - win_c0;
+        const int x0 = xbd(cx), x1 = xbd(cx + 1);
+        int s = 3 * x0, e = 3 * x1;  // absolute columns
+        c_e0 = (s & 1) ? s++ - 16 * win_c0 : -1;
+        c_e2 = (e & 1) ? --e - 16 * win_c0 : -1;
+        c_word = (s >> 1) - 8 * win_c0;
+        c_nw = (e - s) >> 1;
+        c_q = (s >> 1) % 3;
+        c_wd = (uint32_t)(x1 - x0);
+        c_w50 = (uint32_t)(xbd(2 * (k0 + (lane >> 1)) + 2) - xbd(2 * (k0 + (lane >> 1))));
+        cur_w = W;
+      }
+    }
+    const int rb16 = (3 * cur_w + 15) & ~15;
+    // R of this lane's cell in both rows, from the stage
+    uint32_t rv[2][3] = {{0, 0, 0}, {0, 0, 0}};
+    if (has_cell) {
+      const uint8_t* rp = stage + (size_t)st * a.stage_bytes + r_base + roff + cx * 3;
+#pragma unroll
+      for (int c = 0; c < 3; ++c) {
+        rv[0][c] = rp[c];
+        rv[1][c] = rp[3 * sdd_w + c];
+      }
+    }
+
+    // ---- column phase: lane = chunk of the window, both 100-grid rows
+    const uint8_t* sp = stage + (size_t)st * a.stage_bytes;
+    if (lane < win_n) {
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        const int ylo = (r ? y1 : y0) - y0, yn = (r ? y2 - y1 : y1 - y0);
+        const uint8_t* p = sp + 16 * (win_c0 + lane) + ylo * rb16;
+        uint32_t acc[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
+#pragma unroll
+        for (int yy = 0; yy < kMaxRows; yy += 2) {
+          if (yy + 1 < yn)
+            acc16x2(acc, *reinterpret_cast<const uint4*>(p + yy * rb16), *reinterpret_cast<const uint4*>(p + (yy + 1) * rb16));
+          else if (yy < yn)
+            acc16(acc, *reinterpret_cast<const uint4*>(p + yy * rb16));
+        }
+        store_colsum(reinterpret_cast<uint32_t*>(cs_w + r * 512), lane, acc);
+      }
+    }
+    __syncwarp();
+    // the stage is consumed by this warp
+    if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"((uint32_t)__cvta_generic_to_shared(&empty[st])) : "memory");
+
+    // ---- cell phase: lane = 100-grid cell, rows A then B; the 50-cell sums accumulate in the lane
+    uint32_t s50[3] = {0, 0, 0};
+    if (has_cell) {
+#pragma unroll
+      for (int r = 0; r < 2; ++r) {
+        const uint16_t* cs = cs_w + r * 512;
+        const uint32_t* w = reinterpret_cast<const uint32_t*>(cs) + c_word;
+        uint32_t bb[3] = {0u, 0u, 0u};
+#pragma unroll
+        for (int k = 0; k < kW1; ++k)
+          if (k < kW0 || k < c_nw) bb[k % 3] += w[k];
+        const uint32_t b0 = bb[0], b1 = bb[1], b2 = bb[2];
+        const uint32_t A0 = c_q == 0 ? b0 : (c_q == 1 ? b2 : b1);
+        const uint32_t A1 = c_q == 0 ? b1 : (c_q == 1 ? b0 : b2);
+        const uint32_t A2 = c_q == 0 ? b2 : (c_q == 1 ? b1 : b0);
+        const uint32_t c0 = (A0 & 0xFFFFu) + (A1 >> 16) + (c_e0 >= 0 ? (uint32_t)cs[c_e0] : 0u);
+        const uint32_t c1 = (A0 >> 16) + (A2 & 0xFFFFu);
+        const uint32_t c2 = (A1 & 0xFFFFu) + (A2 >> 16) + (c_e2 >= 0 ? (uint32_t)cs[c_e2] : 0u);
+        s50[0] += c0;
+        s50[1] += c1;
+        s50[2] += c2;
+        const uint32_t n = c_wd * (uint32_t)(r ? y2 - y1 : y1 - y0);
+        const uint32_t m = magic[n];
+        const uint32_t d0 = __umulhi(c0 + (n >> 1), m), d1 = __umulhi(c1 + (n >> 1), m), d2 = __umulhi(c2 + (n >> 1), m);
+        const int e0 = (int)d0 - (int)rv[r][0], e1 = (int)d1 - (int)rv[r][1], e2 = (int)d2 - (int)rv[r][2];
+        if (cur_mode != kRefPrevious) {  // PREVIOUS mode: K2 measures against the previous frame's D100
+          if (cur_metric == kDistSad) ssd_acc += (uint32_t)(abs(e0) + abs(e1) + abs(e2));
+          else ssd_acc += (uint32_t)(e0 * e0 + e1 * e1 + e2 * e2);
+        }
+        if (a.d100) {
+          uint8_t* o = a.d100 + (int64_t)cur_f * sdd_h * 3 * sdd_w + ((int64_t)(2 * b + r) * sdd_w + cx) * 3;
+          o[0] = (uint8_t)d0;
+          o[1] = (uint8_t)d1;
+          o[2] = (uint8_t)d2;
+        }
+      }
+    }
+    // ---- D50: horizontal pair (lanes 2m, 2m + 1) by one shuffle per channel; even lanes emit the 50-cell
+#pragma unroll
+    for (int c = 0; c < 3; ++c) s50[c] += __shfl_xor_sync(0xffffffffu, s50[c], 1);
+    if (has_cell && !(lane & 1)) {
+      const uint32_t n50 = c_w50 * (uint32_t)(y2 - y0);
+      const uint32_t m50 = magic[n50];
+      uint8_t* o = cur_d50 + ((int64_t)b * half_w + k0 + (lane >> 1)) * 3;
+#pragma unroll
+      for (int c = 0; c < 3; ++c) o[c] = (uint8_t)__umulhi(s50[c] + (n50 >> 1), m50);
+    }
+  }
+  if (cur_f >= 0) {
+    uint32_t v = ssd_acc;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+    if (lane == 0 && v) {
+      atomicAdd(a.acc_ssd + cur_f, (unsigned long long)v);
+      if (a.stats) atomicAdd(a.stats + (int64_t)cur_slot * NSTAT + 3, (unsigned long long)v);
+    }
+  }
+}
+
 // Reference image R: one rounding of the mean over k frames x box. One thread per value.
 __global__ void reference_kernel(const uint8_t* __restrict__ frames, int32_t k, int64_t frame_stride, int32_t W,
                                  int32_t H, int64_t pitch, int32_t sdd_w, int32_t sdd_h, uint8_t* __restrict__ out) {
@@ -658,11 +908,48 @@ void sdd_plan_add(SddPlan& p, int32_t W, int32_t H, int64_t pitch, const void* p
   const int rb16 = (3 * W + 15) & ~15;
   p.max_chunks = std::max(p.max_chunks, rb16 >> 4);
   p.pair_stage = std::max(p.pair_stage, sdd_bulk_stage_bytes(W, H, sdd_h));
+  // a 50-grid row (two 100-grid rows) spans at most ceil(2H / sdd_h) source rows
+  p.seg_stage = std::max(p.seg_stage, ((2 * H + sdd_h - 1) / sdd_h) * rb16);
+  p.max_rows100 = std::max(p.max_rows100, (H + sdd_h - 1) / sdd_h);
+  p.max_w = std::max(p.max_w, W);
+  p.min_w = p.min_w ? std::min(p.min_w, W) : W;
   if ((pitch & 15) || ((uintptr_t)pixels & 15)) p.vec16 = false;
 }
 
 int k1_variant(int max_chunks, int sdd_w);
-constexpr int kK1Band2 = 1282;  // k1_variant id of sdd_band2_kernel_impl
+constexpr int kK1Band2 = 1282;  // k1_variant id of sdd_band2_kernel_impl (rows of <= 128 chunks)
+
+int sdd_seg_magic_n(const SddPlan& p, int sdd_w) {  // largest box area + 1: a 50-grid cell of 2 x 2 100-grid cells
+  return 4 * p.max_rows100 * ((p.max_w + sdd_w - 1) / sdd_w) + 1;
+}
+
+// (groups of 5 consumer warps, stages) of the warp-segment kernel, measured on M1 (profiles/r02/k1_m1_ab.md):
+// 2 groups x 5 stages, two CTAs per SM; FFSVA_K1_SEG="g,ns" selects another instantiated pair (A/B)
+struct SegCfg {
+  int g, ns;
+};
+SegCfg seg_cfg() {
+  SegCfg c{2, 5};
+  if (const char* e = std::getenv("FFSVA_K1_SEG")) {
+    int g = 0, ns = 0;
+    if (std::sscanf(e, "%d,%d", &g, &ns) == 2 && ((g == 2 && ns == 5) || (g == 3 && ns == 8) || (g == 2 && ns == 4)))
+      c = SegCfg{g, ns};
+  }
+  return c;
+}
+size_t sdd_seg_smem_bytes(int stage_bytes, int magic_n) {
+  const SegCfg c = seg_cfg();
+  return (size_t)c.ns * stage_bytes + (size_t)c.g * kSegWarps * 2 * 512 * 2 + (size_t)4 * magic_n;
+}
+// The warp-segment kernel takes a narrow-row batch when: at most 10 50-cells per warp (half_w <= 50); a segment's
+// window of <= 32 chunks (cells of <= 8 px); packed 16-bit lanes that cannot overflow (every 100-cell channel sum
+// <= 65535); cells of >= 2 px (no one-pixel box: the magic table's n = 1 entry is not used); a unit that fits the stage
+// budget.
+bool sdd_seg_ok(const SddPlan& p, int sdd_w) {
+  const int cellw = (p.max_w + sdd_w - 1) / sdd_w;
+  return sdd_w / 2 <= 10 * kSegWarps && cellw <= 8 && (int64_t)p.max_rows100 * cellw * 255 <= 65535 &&
+         p.max_rows100 <= 16 && p.seg_stage <= 32 * 1024 && p.min_w >= 2 * sdd_w;
+}
 
 size_t sdd_band2_smem_bytes(int stage_bytes, int sdd_w) {
   return (size_t)stage_bytes + (size_t)4 * (sdd_w + 1) + (size_t)((6 * sdd_w + 3) & ~3);
@@ -674,8 +961,13 @@ void sdd_plan_finish(SddPlan& p, int32_t sdd_w, int32_t sdd_h) {
   const bool pair_ok = p.vec16 && sdd_bulk_ok(p.max_chunks, p.pair_stage);
   p.variant = pair_ok && !(force && !std::strcmp(force, "stream")) ? kSddPair : kSddStream;
   if (p.variant == kSddPair) {
-    // the stage also holds the u16 column sums (2*rb16) followed by the u32 cell sums (12*sdd_w) once consumed
-    if (k1_variant(p.max_chunks, sdd_w) == kK1Band2) {  // two rows' sources; then 2 x column sums + 2 x cells
+    const char* nt = std::getenv("FFSVA_K1_NT");  // 1282 keeps the one-CTA-per-band kernel (A/B)
+    if (k1_variant(p.max_chunks, sdd_w) == kK1Band2 && sdd_seg_ok(p, sdd_w) && !(nt && std::atoi(nt) == kK1Band2)) {
+      // source rows, then the 16-byte aligned span of the unit's two rows of R (the kernel's r_base)
+      p.stage_bytes = (p.seg_stage + ((6 * sdd_w + 31) & ~15) + 127) & ~127;
+      p.smem = sdd_seg_smem_bytes(p.stage_bytes, sdd_seg_magic_n(p, sdd_w));
+      p.seg = true;
+      } else if (k1_variant(p.max_chunks, sdd_w) == kK1Band2) {  // two rows' sources; then 2 x column sums + 2 x cells
       p.stage_bytes = std::max(2 * p.pair_stage, 64 * p.max_chunks + 24 * sdd_w);
       p.smem = sdd_band2_smem_bytes(p.stage_bytes, sdd_w);
     } else {
@@ -689,6 +981,11 @@ void sdd_plan_finish(SddPlan& p, int32_t sdd_w, int32_t sdd_h) {
 }
 
 void sdd_plan_apply(const SddPlan& p, SddArgs& a) {
+  a.seg = p.seg;
+  a.max_cellw = (p.max_w + a.sdd_w - 1) / a.sdd_w;
+  a.max_rows100 = p.max_rows100;
+  a.min_cellw = p.min_w / a.sdd_w;
+  a.magic_n = sdd_seg_magic_n(p, a.sdd_w);
   a.max_chunks = p.max_chunks;
   a.vec16 = p.vec16;
   a.bulk = p.variant == kSddPair;
@@ -727,6 +1024,18 @@ int k1_variant(int max_chunks, int sdd_w) {
   return v;
 }
 
+// warp-segment kernel instantiations: 360p (cells of 6-7 px = 8-10 words, 100-grid rows of 3-4 source rows) and a
+// general one (cells <= 8 px, <= 16 source rows)
+#define SEG_360(kG, kNS, kMinB) sdd_seg_kernel<kG, kNS, kMinB, 8, 10, 4>
+#define SEG_GEN(kG, kNS, kMinB) sdd_seg_kernel<kG, kNS, kMinB, 0, 12, 16>
+template <int kG, int kNS, int kMinB>
+cudaError_t seg_set_smem(int smem) {
+  cudaError_t e = cudaFuncSetAttribute(SEG_360(kG, kNS, kMinB), cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(SEG_GEN(kG, kNS, kMinB), cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  return e;
+}
+
 cudaError_t sdd_configure(size_t smem) {
   // per device (the attribute is set on the current device); it is an upper bound for every later launch there, so
   // it never goes below the 48 KB default
@@ -745,12 +1054,47 @@ cudaError_t sdd_configure(size_t smem) {
   if (e == cudaSuccess) e = k1_set_smem<256, 2, FFSVA_K1_MINBLOCKS>((int)smem);
   if (e == cudaSuccess) e = k1_set_smem<384, 1, 3>((int)smem);
   if (e == cudaSuccess) e = cudaFuncSetAttribute(sdd_band2_kernel_impl, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e == cudaSuccess) e = seg_set_smem<2, 5, 2>((int)smem);
+  if (e == cudaSuccess) e = seg_set_smem<3, 8, 1>((int)smem);
+  if (e == cudaSuccess) e = seg_set_smem<2, 4, 2>((int)smem);
   if (e == cudaSuccess) configured[dev] = smem;
   return e;
 }
 
+// Persistent grid of the warp-segment kernel: every SM filled to its occupancy.
+template <typename K>
+int seg_grid(K kernel, int threads, size_t smem, int64_t units) {
+  int dev = 0, sms = 0, per_sm = 1;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem) != cudaSuccess || per_sm < 1)
+    per_sm = 1;
+  return (int)std::max<int64_t>(1, std::min<int64_t>(units, (int64_t)sms * per_sm));
+}
+
+template <int kG, int kNS, int kMinB>
+void seg_launch(const SddArgs& a, size_t smem, int64_t units, cudaStream_t st) {
+  const int threads = 32 * (kG * kSegWarps + 1);
+  if (a.max_rows100 <= 4 && a.max_cellw <= 7 && a.min_cellw >= 6) {  // 360p
+    auto k = SEG_360(kG, kNS, kMinB);
+    k<<<seg_grid(k, threads, smem, units), threads, smem, st>>>(a);
+  } else {
+    auto k = SEG_GEN(kG, kNS, kMinB);
+    k<<<seg_grid(k, threads, smem, units), threads, smem, st>>>(a);
+  }
+}
+
 cudaError_t launch_sdd(const SddArgs& a, cudaStream_t st) {
   if (a.n <= 0) return cudaSuccess;
+  if (a.bulk && a.seg) {
+    const size_t smem = sdd_seg_smem_bytes(a.stage_bytes, a.magic_n);
+    const int64_t units = (int64_t)a.n * (a.sdd_h / 2);
+    const SegCfg c = seg_cfg();
+    if (c.g == 3) seg_launch<3, 8, 1>(a, smem, units, st);
+    else if (c.ns == 4) seg_launch<2, 4, 2>(a, smem, units, st);
+    else seg_launch<2, 5, 2>(a, smem, units, st);
+    return cudaGetLastError();
+  }
   if (a.bulk) {
     const int v = k1_variant(a.max_chunks, a.sdd_w);
     const size_t smem = v == kK1Band2 ? sdd_band2_smem_bytes(a.stage_bytes, a.sdd_w)
