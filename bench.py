@@ -499,6 +499,12 @@ def run_ours(args, cfg, ws, rank, local):
                              "peak_source": peak_kind, "survivors_per_s": m_avg / (k_ms[2] / 1e3) if k_ms[2] else 0},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
             "online": online,
+            "sustained_streams_validated": None if not online else {
+                "sdd_snm": online.get("max_sustained_streams_validated"),
+                "sdd_snm_tyolo": online.get("max_sustained_streams_validated_with_tyolo"),
+                "window_s": online.get("validation_window_s"),
+                "by_tor": {k: v["max_sustained_streams_validated"] for k, v in online.get("online_by_tor", {}).items()},
+                "by_tor_window_s": args.online_tor_confirm_seconds},
         }
         if args.config == "snm":  # K4 is this workload's dominant kernel: its tensor roofline is the line's
             out["sdd_roofline"] = out["roofline"]
@@ -590,22 +596,22 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs, ws=1):
     """Paced 30-FPS streams through the online runtime (feedback queue + dynamic batching, §4.3).
     Stream i replays content stream i % len(sids) of the pool with its own reference image and SNM.
 
+    Each ladder climbs fractions of the measured offline capacity with short rungs (--online-seconds) until a count is
+    not sustained, then confirms its best rung with a long paced run (--online-confirm-seconds, 30 s by default: the
+    §8(d) contract); if the confirmation fails, the rung below is confirmed instead. Ladders: SDD + SNM on the M2
+    content; the full SDD -> SNM -> T-YOLO cascade (f1); and the target-occurrence sweep of config M4 (TOR 1 / 10 /
+    50 %: the same backgrounds with 3 / 30 / 150 target frames per 300), confirmed over --online-tor-confirm-seconds.
+    The verdict of every run is online.sustained_verdict (p99 <= 1 s, >= 99 % of the window's arrivals decided, no
+    backlog growth over the last 10 s).
+
     N > 1: every rank runs the same per-GPU counts on its own GPU at the same time (streams are sharded, no frame
     crosses GPUs); a count is sustained only if it is sustained on every rank (all-reduce MIN of the verdicts, so
     the ranks also climb their ladders in lock step), and the whole-job count is N x the per-GPU count."""
     import torch
-    import torch.distributed as dist
 
     from paper_conf_icpp_zhangcjzly18_b200.online import run_paced
     from synth import synth
     W, H, P = video.width, video.height, 3 * video.width
-    counts, ladder = [], []
-    for tok in args.online.split(","):
-        tok = tok.strip()
-        if tok == "auto":  # a ladder of fractions of the offline capacity, climbed until a count is not sustained
-            ladder = [max(31, int(f * value / 30)) for f in (0.55, 0.7, 0.85, 0.9, 0.95)]
-        elif tok:
-            counts.append(int(tok))
     nc = len(sids)
     refs = []
     for k, s in enumerate(sids):
@@ -613,28 +619,11 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs, ws=1):
         synth.frames_cuda(video, torch.full((32,), s, dtype=torch.int32, device=dev),
                           torch.arange(32, dtype=torch.int64, device=dev), r, H * P, P, ref=True)
         refs.append(r)
-    # full three-filter cascade (f1: SDD -> SNM -> T-YOLO, random-init T-YOLO weights) at these stream counts
-    ty_counts = []
-    ty_ladder = []
-    for tok in args.online_tyolo.split(","):
-        tok = tok.strip()
-        if tok == "auto":  # T-YOLO (~55 K frames/s) sees the SNM survivors, a few % of the frames at TOR 10 %:
-            ty_ladder = [max(31, int(f * value / 30)) for f in (0.1, 0.2, 0.3, 0.4, 0.5)]  # climbed like SDD+SNM's
-        elif tok:
-            ty_counts.append(int(tok))
-    results = []
     opened = []
-    runs = ([(S, False) for S in counts] + [(S, False) for S in ladder] + [(S, True) for S in ty_counts] +
-            [(S, True) for S in ty_ladder])
     ty = None
-    if ty_counts or ty_ladder:
-        import paper_conf_icpp_zhangcjzly18_b200 as ff
-        ty = ff.Tyolo(ctx, synth.tyolo_weights(video.seed))
-    ty_warm = False
-    ladder_failed = ty_ladder_failed = False
-    for S, with_ty in runs:
-        if (S in ladder and not with_ty and ladder_failed) or (S in ty_ladder and with_ty and ty_ladder_failed):
-            continue  # a ladder stops at its first count that is not sustained
+    state = {"ty_warm": False}
+
+    def run(S, content, seconds, with_ty):
         t_setup = time.perf_counter()
         while len(opened) < S:
             i = len(opened)
@@ -644,34 +633,107 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs, ws=1):
             st.snm_load(synth.snm_weights(video.seed, 100000 + i))
             opened.append(st)
         setup_s = time.perf_counter() - t_setup
-        if with_ty and not ty_warm:  # outside the paced window: the first T-YOLO launches load their modules
-            ty.run([(opened[0], pool[0][t], t) for t in range(2)], target_class=14, thresh=0.2)
-            ty_warm = True
+        if with_ty and not state["ty_warm"]:  # outside the paced window: the first T-YOLO launches load their modules
+            ty.run([(opened[0], content[0][t], t) for t in range(2)], target_class=14, thresh=0.2)
+            state["ty_warm"] = True
         # cycles of 10 ms, 25 ms from 10 K streams on (the driver's per-cycle work over all cameras is amortised)
-        res = run_paced(ctx, opened[:S], [pool[i % nc] for i in range(S)], pool.shape[1], args.online_seconds,
+        res = run_paced(ctx, opened[:S], [content[i % nc] for i in range(S)], content.shape[1], seconds,
                         cuda_stream=cs, tyolo=ty if with_ty else None, tick_s=0.010 if S < 10000 else 0.025)
         res["stream_setup_s"] = setup_s
         if ws > 1:
             res["sustained_this_rank"] = res["sustained"]
             res["sustained"] = bool(_allreduce(1 if res["sustained"] else 0, "min", dev))
             res["streams_per_gpu"], res["streams"] = S, S * ws
-        results.append(res)
-        if S in ladder and not with_ty and not res["sustained"]:
-            ladder_failed = True
-        if S in ty_ladder and with_ty and not res["sustained"]:
-            ty_ladder_failed = True
+        return res
+
+    def climb(fracs, content, confirm_s, with_ty, bisect=2):
+        """Rungs at fractions of the offline capacity until one fails, then `bisect` halvings between the last
+        sustained and the failing fraction; the best sustained rung is confirmed with a long run (else the next
+        best). A short unrecorded run at the first rung's count warms the path first (allocations, first launches)."""
+        warm = run(max(31, int(fracs[0] * value / 30)), content, 2.0, with_ty)
+        rungs, ok, bad = [], [], None
+
+        def rung(f):
+            S = max(31, int(f * value / 30))
+            r = run(S, content, args.online_seconds, with_ty)
+            r["fraction_of_offline_capacity"] = f
+            rungs.append(r)
+            return r["sustained"], S
+
+        for f in fracs:
+            good, S = rung(f)
+            if not good:
+                bad = f
+                break
+            ok.append((f, S))
+        lo = ok[-1][0] if ok else 0.0
+        for _ in range(bisect if bad is not None else 0):
+            mid = (lo + bad) / 2
+            good, S = rung(mid)
+            if good:
+                ok.append((mid, S))
+                lo = mid
+            else:
+                bad = mid
+        best = sorted(ok, key=lambda t: t[1])
+        confirms, validated = [], 0
+        for _, S in reversed(best[-2:]):
+            r = run(S, content, confirm_s, with_ty)
+            confirms.append(r)
+            if r["sustained"]:
+                validated = S * ws
+                break
+        return {"rungs": rungs, "confirm": confirms, "max_sustained_streams_validated": validated,
+                "validation_window_s": confirm_s, "warmup_run": {k: warm[k] for k in ("streams", "seconds",
+                                                                                   "sustained")}}
+
+    out = {"policy": "q_sdd 2, q_snm 10, q_tyolo 2, BatchSize 30, num_t-yolo 4 (PAPER.md L173, L217, L219); "
+                     "sustained = p99 <= 1 s, >= 99 % of the window's arrivals decided, no backlog growth "
+                     "(online.sustained_verdict)"}
+    explicit = [int(t) for t in args.online.split(",") if t.strip() and t.strip() != "auto"]
+    out["runs"] = [run(S, pool, args.online_seconds, False) for S in explicit]
+    if "auto" in args.online:
+        lad = climb((0.55, 0.7, 0.85, 0.9, 0.95), pool, args.online_confirm_seconds, False)
+        out["sdd_snm"] = lad
+        out["max_sustained_streams_validated"] = lad["max_sustained_streams_validated"]
+        out["validation_window_s"] = lad["validation_window_s"]
+    if args.online_tyolo:
+        import paper_conf_icpp_zhangcjzly18_b200 as ff
+        ty = ff.Tyolo(ctx, synth.tyolo_weights(video.seed))
+        tyo = [int(t) for t in args.online_tyolo.split(",") if t.strip() and t.strip() != "auto"]
+        out["tyolo_runs"] = [run(S, pool, args.online_seconds, True) for S in tyo]
+        if "auto" in args.online_tyolo:  # T-YOLO (~100 K frames/s) sees the SNM survivors, a few % of the frames
+            lad = climb((0.1, 0.2, 0.3, 0.4, 0.5), pool, args.online_confirm_seconds, True)
+            out["sdd_snm_tyolo"] = lad
+            out["max_sustained_streams_validated_with_tyolo"] = lad["max_sustained_streams_validated"]
+    if args.online_tor:
+        # M4's target-occurrence sweep (SURVEY.md §8(d): S_max per TOR; the analogue of Fig. 6a, PAPER.md L255): the
+        # same backgrounds (so the same references) with TOR 1 / 10 / 50 % targets
+        by_tor = {}
+        for tok in args.online_tor.split(","):
+            tor = int(tok)
+            on_len = {1: 3, 10: 30, 50: 150}[tor]
+            if on_len == video.on_len:
+                content = pool
+            else:
+                v2 = synth.Video(seed=video.seed, width=W, height=H, period=video.period, on_len=on_len)
+                content = torch.empty_like(pool)
+                for k, s in enumerate(sids):
+                    synth.frames_cuda(v2, torch.full((pool.shape[1],), s, dtype=torch.int32, device=dev),
+                                      torch.arange(pool.shape[1], dtype=torch.int64, device=dev), content[k], H * P, P)
+            lad = climb((0.7, 0.85, 0.95), content, args.online_tor_confirm_seconds, False, bisect=1)
+            by_tor[f"{tor}%"] = {"max_sustained_streams_validated": lad["max_sustained_streams_validated"],
+                                 "validation_window_s": lad["validation_window_s"], "rungs": lad["rungs"],
+                                 "confirm": lad["confirm"]}
+            del content
+        out["online_by_tor"] = by_tor
     closed = set(id(st) for st in opened)
     for st in opened:
         st.close()
     ctx.streams = [st for st in ctx.streams if id(st) not in closed]  # (list.remove per stream is O(S^2))
     if ty is not None:
         ty.destroy()
-    best = max([r["streams"] for r in results if r["sustained"] and "stages" not in r], default=0)
-    best_ty = max([r["streams"] for r in results if r["sustained"] and "stages" in r], default=0)
-    return {"runs": results, "max_sustained_streams_validated": best,
-            "max_sustained_streams_validated_with_tyolo": best_ty,
-            "policy": "q_sdd 2, q_snm 10, q_tyolo 2, BatchSize 30, num_t-yolo 4 (PAPER.md L173, L217, L219); "
-                      "latency budget p99 <= 1 s"}
+    return out
 
 
 def _cpu_model() -> str:
@@ -871,8 +933,13 @@ def main():
                     help="comma-separated stream counts for the paced online validation (config m2); 'auto' = "
                          "a ladder of 55/70/85/90/95%% of the measured frames/s / 30, climbed until a count is not "
                          "sustained; empty to skip")
-    ap.add_argument("--online-seconds", type=float, default=4.0)
-    ap.add_argument("--online-tyolo", default="2000,auto",
+    ap.add_argument("--online-seconds", type=float, default=4.0, help="seconds per ladder rung")
+    ap.add_argument("--online-confirm-seconds", type=float, default=30.0,
+                    help="paced run that confirms a ladder's best rung (SURVEY.md §8(d): 30 s)")
+    ap.add_argument("--online-tor", default="1,10,50",
+                    help="target-occurrence sweep of the online ladder (config M4's TOR 1/10/50 %%); empty to skip")
+    ap.add_argument("--online-tor-confirm-seconds", type=float, default=10.0)
+    ap.add_argument("--online-tyolo", default="auto",
                     help="stream counts for a paced run of the full cascade with the T-YOLO stage (f1); 'auto' = "
                          "a ladder of 10/20/30/40/50%% of the measured frames/s / 30; empty to skip")
     args = ap.parse_args()
