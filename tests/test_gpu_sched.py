@@ -243,7 +243,7 @@ def test_online_three_stage_cascade_with_tyolo(env, pipeline):
     s, t = reached[0]
     want = orc.tyolo_forward(orc.resize(host[s][t], 640, 416, 416), params, bf16_emul=True)
     sc = orc.tyolo_scores(want, targets[s])
-    near = int((np.abs(sc - 0.2) <= 2e-2).sum())
+    near = int((np.abs(sc - 0.2) <= 0.75 * 0.03).sum())  # the score margin of test_gpu_tyolo.py (TAU_HEAD)
     assert abs(int(got[(s, t)]["tyolo_count"]) - orc.tyolo_count(want, targets[s], 0.2)) <= near
     for c in cams:
         c.st.close()

@@ -6,8 +6,9 @@ CPU oracle.
   own previous activation (bf16-rounded weights, fp64 accumulation, rounded to bf16) — isolates indexing,
   padding, pooling and packing bugs per layer; bar: |diff| <= 1 bf16 ulp of the value + 1e-3 absolute
   (fp32-vs-fp64 accumulation can flip one rounding);
-* the whole network vs orc.tyolo_forward (bf16 emulation) on full 416x416 frames; bar on the head outputs
-  derived in DESIGN.md (f1 parity), counts equal except boxes whose oracle score lies within 2e-2 of the threshold.
+* layer 9 (the 1x1 head) in isolation with a worst-case fp32-accumulation bar;
+* the whole network vs orc.tyolo_forward (bf16 emulation) on full 416x416 frames: absolute bar TAU_HEAD on the head
+  outputs, counts equal except boxes whose oracle score lies within the score margin that bar implies.
 """
 import numpy as np
 import pytest
@@ -110,6 +111,43 @@ def test_each_layer_against_oracle_ops(env, layer):
     st.close()
 
 
+def test_head_layer_against_oracle_op(env):
+    """Layer 9 (the 1x1 head, 1024 -> 125, fp32 outputs, no activation) in isolation: the GPU head on the GPU's own
+    layer-8 activation vs the oracle's conv1x1 with the bf16-rounded weights in fp64. The products of bf16 values are
+    exact in fp32, so the only differences are the fp32 accumulation over K = 1024 terms and the bias add: the
+    worst case is gamma_K = K * 2^-24 times sum |x w| (+ |b|) per output; the bar is twice that."""
+    ff, ctx, dev, ty, params = env
+    n = 2
+    st, host, d, items = _frames(ctx, dev, 1280, 720, n, seed=29, on_len=4)
+    x8 = ty.layer_output(items, 7)
+    got = ty.run(items, target_class=TARGET, raw=True)["raw"]
+    w, b = _layer_params(params, 8)
+    w = _round_bf16_fast(w).reshape(125, 1024)
+    compared = 0
+    for i in range(n):
+        x = np.transpose(x8[i].astype(np.float64), (2, 0, 1)).copy()
+        want = orc.conv1x1(x, w, b.astype(np.float64))
+        mag = orc.conv1x1(np.abs(x), np.abs(w)) + np.abs(b.astype(np.float64))[:, None, None]
+        g = np.transpose(got[i].astype(np.float64), (2, 0, 1))
+        bar = 2 * 1024 * 2.0 ** -24 * mag + 1e-6
+        err = np.abs(g - want)
+        assert np.all(err <= bar), f"head: max err {err.max():.3e}, worst err/bar {(err / bar).max():.2f}"
+        compared += err.size
+    assert compared == n * 125 * 13 * 13
+    st.close()
+
+
+# Whole-network bar (DESIGN.md §7, f1): the GPU and the bf16-emulating oracle round the same operands, so they differ
+# only where fp32 and fp64 accumulation land on different sides of a bf16 rounding boundary (~1-2 % of the values of a
+# layer, test_each_layer_against_oracle_ops); those 1-ulp flips propagate through the later layers, so no useful
+# worst-case bound exists. TAU_HEAD = 0.03 absolute on the 13x13x125 head is twice the largest difference measured
+# over 16 frames (0.0155, head values up to 4.7). A box score sigma(o) * softmax(z)_t moves by at most
+# (1/4 + 1/2) * TAU_HEAD to first order (sigma' <= 1/4; sum_j |d softmax_t / d z_j| = 2 p_t (1 - p_t) <= 1/2), so
+# counts must agree except for boxes whose oracle score lies within SCORE_MARGIN of the 0.2 threshold.
+TAU_HEAD = 0.03
+SCORE_MARGIN = 0.75 * TAU_HEAD
+
+
 def test_whole_network_against_oracle(env):
     """Two full 1280x720 frames with a planted object vs orc.tyolo_forward in bf16-emulation mode."""
     ff, ctx, dev, ty, params = env
@@ -121,10 +159,10 @@ def test_whole_network_against_oracle(env):
         want = orc.tyolo_forward(img, params, bf16_emul=True)
         g = got["raw"][i].astype(np.float64)
         err = np.abs(g - want)
-        scale = np.abs(want).max()
-        assert err.max() <= 2e-2 * max(1.0, scale), f"max |diff| {err.max():.3e} (scale {scale:.2f})"
-        sc = orc.tyolo_scores(want, TARGET)
-        near = np.abs(sc - 0.2) <= 2e-2
+        assert err.max() <= TAU_HEAD, f"max |diff| {err.max():.3e} > {TAU_HEAD}"
+        sc, sg = orc.tyolo_scores(want, TARGET), orc.tyolo_scores(g, TARGET)
+        assert np.abs(sc - sg).max() <= SCORE_MARGIN
+        near = np.abs(sc - 0.2) <= SCORE_MARGIN
         want_cnt = orc.tyolo_count(want, TARGET, 0.2)
         assert abs(int(got["counts"][i]) - want_cnt) <= int(near.sum()), (got["counts"][i], want_cnt, near.sum())
         if near.sum() == 0:

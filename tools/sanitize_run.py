@@ -13,7 +13,44 @@ from paper_conf_icpp_zhangcjzly18_b200.ffsva import Scheduler  # noqa: E402
 from synth import synth  # noqa: E402
 
 
+def minimal():
+    """--minimal (racecheck to completion): the narrow-row K1 (warp-segment pipeline), K3 and K4 on 8 frames of two
+    streams, the one-CTA-per-band K1 on 2 small frames, the CTA-pair K1 on one 720p frame, and two synchronous
+    scheduler ticks."""
+    dev = torch.device("cuda:0")
+    ctx = ff.Context(dev)
+    v = synth.Video(seed=5, width=640, height=360, period=4, on_len=2)
+    streams = []
+    for s in range(2):
+        st = ctx.open_stream(width=640, height=360, delta_diff=0.0 if s else 24.0, snm_batch=2)
+        st.set_reference(torch.from_numpy(synth.frames(v, [s] * 2, [0, 1], ref=True)).to(dev))
+        st.snm_load(synth.snm_weights(5, s, bias_std=0.1))
+        streams.append(st)
+    d = torch.from_numpy(synth.frames(v, [0, 1] * 4, [0, 0, 1, 1, 2, 2, 3, 3])).to(dev)
+    items = [(streams[i % 2], d[i], i) for i in range(8)]
+    r = ctx.filter_batch(items)
+    assert int(r["sdd_pass"][1::2].sum()) == 4  # delta 0: every frame of stream 1 reaches K4
+    for (W, H, n) in ((128, 100, 2), (1280, 720, 1)):
+        vb = synth.Video(seed=6, width=W, height=H, period=4, on_len=2)
+        sb = ctx.open_stream(width=W, height=H, delta_diff=0.0, snm_batch=2)
+        sb.set_reference(torch.from_numpy(synth.frames(vb, [0], [0], ref=True)).to(dev))
+        sb.snm_load(synth.snm_weights(6, 0))
+        db = torch.from_numpy(synth.frames(vb, [0] * n, list(range(n)))).to(dev)
+        ctx.filter_batch([(sb, db[i], i) for i in range(n)])
+        sb.close()
+    sched = Scheduler(ctx, max_frames_per_tick=8, snm_slots=16)
+    sched.push(items)
+    for _ in range(2):
+        sched.tick()
+    sched.destroy()
+    ctx.close()
+    torch.cuda.synchronize()
+    print("OK (minimal)")
+
+
 def main():
+    if "--minimal" in sys.argv:
+        return minimal()
     dev = torch.device("cuda:0")
     ctx = ff.Context(dev)
     v = synth.Video(seed=5, width=640, height=360, period=4, on_len=2)
