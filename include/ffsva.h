@@ -319,14 +319,17 @@ FFSVA_API ffsva_status ffsva_stream_export(ffsva_stream* s, void* dst, int64_t c
 FFSVA_API ffsva_status ffsva_stream_import(int32_t device, const void* src, int64_t bytes, int32_t src_is_host,
                                            ffsva_stream** out);
 
-/* Per-stream overload signals of the online runtime since the previous reset (L213): a stream is overloaded
- * when its SNM queue went over q_snm (the SDD stage had to skip it: sdd_blocked > 0) or its prefetcher was
- * refused (SDD queue over q_sdd: refused > 0). */
+/* Per-stream overload signals of the online runtime since the previous reset (L213: "when any queue of T-YOLO or
+ * SNM is longer than its predefined threshold ... the FFS-VA instance overloads"): a stream overloads its instance
+ * when its SNM queue went over q_snm (the SDD stage had to skip it: sdd_blocked > 0), its T-YOLO queue over q_tyolo
+ * (the SNM stage had to skip it: snm_blocked > 0) or its prefetcher was refused (SDD queue over q_sdd: refused > 0). */
 typedef struct {
   int32_t sdd_depth, snm_depth;   /* current queue depths (frames) */
   int32_t max_sdd, max_snm;       /* maxima since the reset */
   uint64_t pushed, refused;       /* frames accepted / refused by the SDD queue since the reset */
   uint64_t sdd_blocked;           /* SDD cycles that skipped the stream (SNM queue over q_snm) since the reset */
+  int32_t tyolo_depth, max_tyolo; /* T-YOLO queue depth now / maximum since the reset (f1 stage attached) */
+  uint64_t snm_blocked;           /* SNM cycles that skipped the stream (T-YOLO queue over q_tyolo) since the reset */
 } ffsva_stream_load;
 /* Attach the device's shared T-YOLO model (ffsva_tyolo_load) to the online runtime as its third stage (f1; NULL
  * detaches): SNM survivors then wait in per-stream T-YOLO queues; the SNM stage skips a stream while its T-YOLO

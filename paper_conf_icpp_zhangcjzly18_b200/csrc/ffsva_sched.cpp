@@ -526,6 +526,9 @@ FFSVA_API ffsva_status ffsva_sched_stream_load(ffsva_sched* s, ffsva_stream* st,
   out->pushed = q.pushed;
   out->refused = q.refused;
   out->sdd_blocked = q.sdd_blocked;
+  out->tyolo_depth = (int32_t)q.ty.size();
+  out->max_tyolo = q.max_ty;
+  out->snm_blocked = q.snm_blocked;
   if (reset) s->pol.reset_counters(id);
   return FFSVA_OK;
 }

@@ -95,7 +95,8 @@ class StreamLoad(ctypes.Structure):
     """ffsva_stream_load: per-stream overload signals of the online runtime."""
     _fields_ = [("sdd_depth", ctypes.c_int32), ("snm_depth", ctypes.c_int32), ("max_sdd", ctypes.c_int32),
                 ("max_snm", ctypes.c_int32), ("pushed", ctypes.c_uint64), ("refused", ctypes.c_uint64),
-                ("sdd_blocked", ctypes.c_uint64)]
+                ("sdd_blocked", ctypes.c_uint64), ("tyolo_depth", ctypes.c_int32), ("max_tyolo", ctypes.c_int32),
+                ("snm_blocked", ctypes.c_uint64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

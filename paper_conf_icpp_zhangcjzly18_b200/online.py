@@ -227,3 +227,87 @@ def run_unpaced(ctx, streams, content, n_content_frames, seconds, policy="dynami
             "snm_scored": int(scored), "snm_batches": int(pops),
             "mean_snm_batch": scored / pops if pops else 0.0}
 
+
+
+def run_controlled(ctx, owned, content, n_content_frames, n_cameras, seconds, spare_fps, interval_s=1.0,
+                   window_s=2.0, stage="sdd", fps=30.0, tick_s=0.010, cuda_stream=None, device=None, max_streams=64,
+                   q_snm_slots=4096):
+    """Paced cameras through one instance's online runtime with the f2 controller in the loop (PAPER.md L213, L225;
+    dist.Reforwarder). Every rank calls this at the same time with its own cameras (`owned`: global camera id ->
+    Stream; cameras 0..n_cameras-1 in all) and the content of every camera (`content[gid]`: device frames
+    [n_content_frames, H, pitch]) so a camera can continue wherever it is re-forwarded. Once per interval every rank
+    reports its measured stage rate and per-stream overload, the plan is computed identically everywhere and moves
+    are executed: the source stops its camera, ticks until the stream detaches, exports it; the target imports it
+    and continues the camera at the frame the source had reached. `fps` is one rate for every camera or a dict gid ->
+    frames/s. Returns this rank's decided frames per camera ({gid: {frame_no: result}}), the controller history and
+    the cameras it owns at the end."""
+    import torch
+
+    from .dist import Reforwarder
+    from .ffsva import FRAME_DTYPE, Scheduler
+
+    rate = {g: float(fps[g] if isinstance(fps, dict) else fps) for g in range(n_cameras)}
+    phase = {g: g * (1.0 / rate[g]) / max(1, n_cameras) for g in range(n_cameras)}
+    sched = Scheduler(ctx, max_frames_per_tick=max(256, 8 * n_cameras), snm_slots=q_snm_slots)
+    # images travel as device tensors whenever the process group is NCCL (dist._p2p_device), host tensors over gloo
+    dev = device if device is not None else torch.device("cuda", ctx.device)
+    rf = Reforwarder(ctx, sched, owned, spare_fps, window_s=window_s, stage=stage, device=dev)
+    next_frame = {g: 0 for g in owned}
+    decided = {}
+    by_handle = {}
+
+    def record(ev):
+        for e in ev:
+            g = by_handle[int(e["stream"])]
+            decided.setdefault(g, {})[int(e["frame_no"])] = e["result"].copy()
+
+    def drain(gid, st):  # the source side of a move: tick until the stream has left the scheduler
+        for _ in range(10000):
+            if sched.detach(st):
+                return
+            ev, _ = sched.tick(cuda_stream)
+            record(ev)
+        raise RuntimeError(f"camera {gid} never detached")
+
+    n_steps = int(round(seconds / interval_s))
+    steps = 0
+    try:
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        while steps < n_steps:
+            now = time.perf_counter()
+            el = now - t0
+            by_handle = {st.handle: g for g, st in owned.items()} | by_handle
+            items = []
+            for g, st in owned.items():
+                due = int(np.floor((el - phase[g]) * rate[g])) + 1
+                for k in range(next_frame[g], min(due, next_frame[g] + 3)):
+                    items.append((g, st, k))
+            if items:
+                fr = np.zeros(len(items), dtype=FRAME_DTYPE)
+                fr["stream"] = [st.handle for _, st, _ in items]
+                fr["pixels"] = [content[g][k % n_content_frames].data_ptr() for g, _, k in items]
+                fr["frame_no"] = [k for _, _, k in items]
+                acc = sched.push_array(fr)
+                for (g, _, k), a in zip(items, acc):
+                    if a and k == next_frame[g]:
+                        next_frame[g] = k + 1
+            ev, info = sched.tick(cuda_stream)
+            record(ev)
+            rf.on_tick(time.perf_counter() - t0, info)
+            if time.perf_counter() - t0 >= (steps + 1) * interval_s:
+                rf.step(time.perf_counter() - t0, interval_s, max_streams, detach=drain, next_frame=next_frame)
+                steps += 1
+                by_handle = {st.handle: g for g, st in owned.items()} | by_handle
+            rest = tick_s - (time.perf_counter() - now)
+            if rest > 0:
+                time.sleep(rest)
+        for _ in range(1000):  # drain what is still queued
+            ev, info = sched.tick(cuda_stream)
+            record(ev)
+            if info["sdd_queued"] == 0 and info["snm_queued"] == 0 and info["tyolo_queued"] == 0 and \
+                    info["events_pending"] == 0:
+                break
+    finally:
+        sched.destroy()
+    return {"decided": decided, "history": rf.history, "owned": sorted(owned)}

@@ -9,7 +9,7 @@ import socket
 import numpy as np
 import pytest
 
-from gpu_util import Cam
+from gpu_util import Cam, check_snm, oracle_for
 from synth import synth
 
 pytestmark = pytest.mark.gpu
@@ -57,6 +57,10 @@ def test_export_import_continues_identically(env, where, distance):
     r2 = ctx.filter_batch([(st2, d[i], i) for i in range(30)])
     _same(r1, r2)
     assert int(r1["sdd_pass"].sum()) > 0
+    # and the continued stream against the oracle (the imported R, thresholds and SNM are the exported ones)
+    want = oracle_for([(cam, host[i]) for i in range(30)])
+    assert np.array_equal(r2["ssd"], want["ssd"]) and np.array_equal(r2["sdd_pass"], want["sdd_pass"])
+    check_snm(r2["logit"], r2["snm_pass"], r2["snm_class"], want["logit"], [cam] * 30, want["survivors"])
     st2.close()
 
 
@@ -110,35 +114,48 @@ def _free_port():
 
 
 def _proc(rank, port, q):
+    """One instance of the f2 controller test (both processes on cuda:0, gloo: the box has one GPU; with NCCL the
+    same calls move the image as a device tensor)."""
     import torch
     import torch.distributed as dist
     import paper_conf_icpp_zhangcjzly18_b200 as ff
-    from paper_conf_icpp_zhangcjzly18_b200 import dist as fdist
+    from paper_conf_icpp_zhangcjzly18_b200.online import run_controlled
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=2)
     dev = torch.device("cuda:0")
     ctx = ff.Context(dev)
-    v = synth.Video(seed=95, width=640, height=360, period=6, on_len=2)
-    d = torch.from_numpy(synth.frames(v, [4] * 12, list(range(12)))).to(dev)
+    v = synth.Video(seed=95, width=640, height=360, period=2, on_len=2)  # every frame holds a target
+    NF = 12
+    content = {g: torch.from_numpy(synth.frames(v, [g] * NF, list(range(NF)))).to(dev) for g in range(3)}
     owned = {}
-    if rank == 0:
-        st = ctx.open_stream(width=640, height=360)
-        st.set_reference(torch.from_numpy(synth.frames(v, [4] * 4, list(range(4)), ref=True)).to(dev))
-        st.snm_load(synth.snm_weights(95, 4, bias_std=0.05))
-        owned[17] = st
-    before = ctx.filter_batch([(owned[17], d[i], i) for i in range(12)]) if rank == 0 else None
-    reports = fdist.gather_reports(0.95 if rank == 0 else 0.1, [(17, True, 1.0)] if rank == 0 else [], 4)
-    moves = fdist.plan_reforward(reports)
-    fdist.reforward(moves, owned, ctx, rank)
-    after = ctx.filter_batch([(owned[17], d[i], i) for i in range(12)]) if rank == 1 else None
-    q.put((rank, moves, sorted(owned), before, after))
+    for g in ((0, 1) if rank == 0 else (2,)):
+        # camera 0 (300 frames/s, every frame a target, BatchSize 1) overloads rank 0: its SNM queue goes over q_snm
+        st = ctx.open_stream(width=640, height=360, snm_batch=1 if g == 0 else 30, q_snm=2 if g == 0 else 10)
+        st.set_reference(torch.from_numpy(synth.frames(v, [g] * 4, list(range(4)), ref=True)).to(dev))
+        st.snm_load(synth.snm_weights(95, g, bias_std=0.05))
+        owned[g] = st
+    ctx.stats(reset=True)
+    out = run_controlled(ctx, owned, content, NF, 3, seconds=5.0, spare_fps=45.0, interval_s=1.0, window_s=2.0,
+                         fps={0: 300.0, 1: 30.0, 2: 30.0})
+    stats = ctx.stats()
+    rows = {g: stats[st.slot].copy() for g, st in owned.items()}
+    q.put((rank, out["history"], out["owned"], {g: sorted(d) for g, d in out["decided"].items()},
+           {g: {k: (int(r["ssd"]), int(r["sdd_pass"]), float(r["logit"])) for k, r in d.items()}
+            for g, d in out["decided"].items()}, rows))
+    for st in owned.values():
+        st.close()
     ctx.close()
     dist.destroy_process_group()
 
 
-def test_reforward_two_processes(env):
+def test_reforward_controller_two_processes(env):
+    """f2 in the online loop: rank 0 runs cameras 0 (300 frames/s) and 1 (30 frames/s) with
+    camera 0 overloading its SNM queue; rank 1 runs camera 2 at 30 frames/s, below the 45 frames/s spare level for
+    the whole 2-s window. The controller re-forwards camera 0 to rank 1, which continues it from the frame rank 0 reached; the
+    frames each side decided agree with the oracle; the stream's statistics row travels with it."""
     import torch.multiprocessing as mp
+    from oracle import oracle as orc
     mctx = mp.get_context("spawn")
     q = mctx.Queue()
     port = _free_port()
@@ -149,6 +166,21 @@ def test_reforward_two_processes(env):
     for p in procs:
         p.join(timeout=120)
         assert p.exitcode == 0
-    assert outs[0][1] == outs[1][1] == [(17, 0, 1)]
-    assert outs[0][2] == [] and outs[1][2] == [17]
-    _same(outs[0][3], outs[1][4])
+    moves = [m for h in outs[0][1] for m in h["moves"]]
+    assert moves == [(0, 0, 1)], outs[0][1] and [m for h in outs[1][1] for m in h["moves"]] == moves
+    assert outs[0][2] == [1] and outs[1][2] == [0, 2]
+    f0, f1 = outs[0][3].get(0, []), outs[1][3].get(0, [])
+    assert f0 and f1 and max(f0) < min(f1), "rank 1 continues camera 0 after the frames rank 0 decided"
+    assert set(f0) | set(f1) == set(range(max(f1) + 1)), "no frame of camera 0 lost in the handover"
+    # statistics row: the imported stream continued rank 0's counters
+    assert int(outs[1][5][0][0]) == len(f0) + len(f1)
+    # every decided frame of camera 0 (either side) against the oracle
+    v = synth.Video(seed=95, width=640, height=360, period=2, on_len=2)
+    R = orc.reference(synth.frames(v, [0] * 4, list(range(4)), ref=True), 640, 100, 100)
+    params = synth.snm_weights(95, 0, bias_std=0.05)
+    for side in (0, 1):
+        for k, (ssd, sp, lg) in list(outs[side][4][0].items())[::7]:
+            w = orc.filter_frames([synth.frame(v, 0, k % 12)], 640, [R], [24.0], [params], [np.float32(0.2)],
+                                  [np.float32(0.8)], [np.float32(0.5)])
+            assert ssd == int(w["ssd"][0]) and sp == int(w["sdd_pass"][0]) == 1
+            assert abs(lg - w["logit"][0]) <= 2e-2

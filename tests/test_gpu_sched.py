@@ -171,6 +171,16 @@ def test_fixed_size_batch_policies(env, policy):
     assert len(got) == 2 * T
     for (s, t), r in got.items():
         assert r["sdd_pass"] == int(synth.is_target(v, s, t)), (s, t)
+    # every frame against the oracle: the batch trigger changes timing only, never a frame's result (C8)
+    for s, c in enumerate(cams):
+        host = c.host_frames(list(range(T)))
+        w = orc.filter_frames(list(host), 640, [c.R] * T, [24.0] * T, [c.params] * T, [f32(0.2)] * T, [f32(0.8)] * T,
+                              [f32(0.5)] * T)
+        for t in range(T):
+            r = got[(s, t)]
+            assert int(r["ssd"]) == int(w["ssd"][t]) and int(r["sdd_pass"]) == int(w["sdd_pass"][t]), (s, t)
+            if w["sdd_pass"][t]:
+                assert abs(float(r["logit"]) - w["logit"][t]) <= SNM_TOL, (s, t)
     for c in cams:
         c.st.close()
 
