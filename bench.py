@@ -84,6 +84,10 @@ class ClockSampler:
         self.device, self.rows, self.proc, self.th = device, [], None, None
 
     def start(self):
+        if os.environ.get("FFSVA_BENCH_NO_CLOCKS") == "1":  # (diagnostics only: a line without clocks is rejected)
+            return
+        if os.environ.get("FFSVA_BENCH_CLOCKS") == "nvml":  # in-process NVML polling (A/B against nvidia-smi)
+            return self._start_nvml()
         try:
             self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
                                           "-lms", "200", "-i", str(self.device)], stdout=subprocess.PIPE,
@@ -93,8 +97,7 @@ class ClockSampler:
             return
         self.th = threading.Thread(target=self._read, daemon=True)
         self.th.start()
-        # nvidia-smi's NVML start-up stalls GPU work for tens of ms: the timed region starts only after its first
-        # sample (measured: a 40-step M1 region absorbed a ~100 ms stall otherwise)
+        # the timed region starts after nvidia-smi's first sample (its start-up is not part of the measurement)
         t0 = time.perf_counter()
         while not self.rows and time.perf_counter() - t0 < 10.0 and self.proc.poll() is None:
             time.sleep(0.02)
@@ -104,7 +107,29 @@ class ClockSampler:
         for line in self.proc.stdout:
             self.rows.append([x.strip() for x in line.split(",")])
 
+    def _start_nvml(self):
+        import pynvml
+        pynvml.nvmlInit()
+        h = pynvml.nvmlDeviceGetHandleByIndex(self.device)
+        self._stop = threading.Event()
+        bits = [pynvml.nvmlClocksEventReasonHwSlowdown, pynvml.nvmlClocksEventReasonHwThermalSlowdown,
+                pynvml.nvmlClocksEventReasonSwThermalSlowdown, pynvml.nvmlClocksEventReasonSwPowerCap]
+
+        def poll():
+            while not self._stop.is_set():
+                r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+                self.rows.append([str(self.device), str(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM)),
+                                  str(pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)), "", ""] +
+                                 ["Active" if r & b else "Not Active" for b in bits])
+                self._stop.wait(0.2)
+        self.th = threading.Thread(target=poll, daemon=True)
+        self.th.start()
+        time.sleep(0.25)
+
     def stop(self):
+        if getattr(self, "_stop", None) is not None:
+            self._stop.set()
+            self.th.join(timeout=2)
         if self.proc:
             self.proc.terminate()
             try:
@@ -197,14 +222,20 @@ def timed_region(eng, steps: int, warmup: int):
     eng.sync()
     _barrier()
     t0 = eng.mark()
+    marks = []
     for i in range(steps):
         eng.step(warmup + i)
+        if getattr(eng, "step_marks", False):
+            marks.append(eng.mark())
     eng.join()
     gathered = fdist.gather_stats(eng.stats())
     t1 = eng.mark()
     eng.sync()
     _barrier()
     clk = eng.stop_clocks()
+    if marks:  # diagnostics (FFSVA_BENCH_STEP_MARKS=1): the slowest step between consecutive marks
+        ts = [eng.elapsed_ms(t0, marks[0])] + [eng.elapsed_ms(a, b) for a, b in zip(marks, marks[1:])]
+        eng.step_ms = {"max": max(ts), "median": sorted(ts)[len(ts) // 2], "argmax": ts.index(max(ts))}
     ms_max = _allreduce(eng.elapsed_ms(t0, t1), "max", eng.device)
     total = _allreduce(eng.frames_per_step * steps, "sum", eng.device)
     return ms_max, int(total), gathered, clk
@@ -319,10 +350,13 @@ class GpuEngine:
         self.css = [self.cs] + [torch.cuda.Stream(device=dev) for _ in range(nstr - 1)]
         self.stats_dev = torch.zeros((max(1, self.rows), ffb.NSTAT), dtype=torch.int64, device=dev)
         self.clocks = None
+        self.step_marks = os.environ.get("FFSVA_BENCH_STEP_MARKS") == "1"
+        self.step_ms = None
 
     # --- correctness gate before timing: SDD pass count == planted count on every batch (P8 at full size), and
     # the fraction of survivors whose logit lies within the 2e-2 parity margin of the decision threshold
     def gate(self):
+        torch = self.torch
         near, surv = 0, 0
         for j, b in enumerate(self.batches):
             b.launch(self.cs)
@@ -335,6 +369,8 @@ class GpuEngine:
             near += int((np.abs(lg - L_T) < 2e-2).sum())
             surv += lg.size
         self.ctx.stats(reset=True)
+        self.stats()  # allocates the library's pinned statistics snapshot outside the timed region
+        torch.cuda.synchronize()
         self.near_margin = {"fraction": near / surv if surv else 0.0, "survivors": surv, "margin": 2e-2,
                             "bar": "< 0.10 (SURVEY.md §8(d): else the decision parity check is weak)"}
         if surv and near / surv >= 0.10:
@@ -498,6 +534,7 @@ def run_ours(args, cfg, ws, rank, local):
                              "frac": (m_avg * SNM_FLOP / (k_ms[2] / 1e3) / 1e12) / tf_peak if k_ms[2] > 0 else 0.0,
                              "peak_source": peak_kind, "survivors_per_s": m_avg / (k_ms[2] / 1e3) if k_ms[2] else 0},
             "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": int(launches), "clocks": clk,
+            **({"step_ms_diagnostic": eng.step_ms} if eng.step_ms else {}),
             "online": online,
             "sustained_streams_validated": None if not online else {
                 "sdd_snm": online.get("max_sustained_streams_validated"),

@@ -365,20 +365,33 @@ FFSVA_API ffsva_status ffsva_stats_copy(int32_t device, uint64_t* dst, int32_t m
     cudaStream_t cs = (cudaStream_t)cuda_stream;
     cudaError_t e = cudaSuccess;
     // kernel counters (device table, stride NSTAT) into columns 0..7, the online runtime's latency columns (host
-    // table, stride NLAT) into columns 8..23 of the FFSVA_NSTAT-wide rows
+    // table, stride NLAT) into columns 8..23 of the FFSVA_NSTAT-wide rows. Device destinations get the latency
+    // columns from a pinned snapshot, so the whole copy stays asynchronous on cs (no host synchronisation).
+    const size_t row = sizeof(uint64_t) * FFSVA_NSTAT;
     std::vector<uint64_t> lat;
-    {
+    uint64_t* snap = nullptr;
+    if (!dst_is_host && ncopy > 0) {
+      if (!ctx->h_lat_pinned) {
+        e = cudaMallocHost(&ctx->h_lat_pinned, sizeof(uint64_t) * NLAT * (size_t)ctx->stats_cap);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&ctx->lat_ev, cudaEventDisableTiming);
+      }
+      if (e == cudaSuccess) e = cudaEventSynchronize(ctx->lat_ev);  // the previous snapshot's copy has run
+      snap = ctx->h_lat_pinned;
+    }
+    if (e == cudaSuccess) {
       std::lock_guard<std::mutex> lk2(ctx->lat_mu);
-      lat.assign(ctx->h_lat.begin(), ctx->h_lat.begin() + (std::ptrdiff_t)ncopy * NLAT);
+      if (snap) std::copy(ctx->h_lat.begin(), ctx->h_lat.begin() + (std::ptrdiff_t)ncopy * NLAT, snap);
+      else lat.assign(ctx->h_lat.begin(), ctx->h_lat.begin() + (std::ptrdiff_t)ncopy * NLAT);
       if (reset) std::fill(ctx->h_lat.begin(), ctx->h_lat.end(), 0);
     }
-    const size_t row = sizeof(uint64_t) * FFSVA_NSTAT;
-    if (ncopy > 0) {
+    if (e == cudaSuccess && ncopy > 0) {
       e = cudaMemcpy2DAsync(dst, row, ctx->d_stats, sizeof(uint64_t) * NSTAT, sizeof(uint64_t) * NSTAT, (size_t)ncopy,
                             dst_is_host ? cudaMemcpyDeviceToHost : cudaMemcpyDeviceToDevice, cs);
-      if (e == cudaSuccess && !dst_is_host)  // pageable source: returns once the rows are staged
-        e = cudaMemcpy2DAsync(dst + NSTAT, row, lat.data(), sizeof(uint64_t) * NLAT, sizeof(uint64_t) * NLAT,
+      if (e == cudaSuccess && snap) {
+        e = cudaMemcpy2DAsync(dst + NSTAT, row, snap, sizeof(uint64_t) * NLAT, sizeof(uint64_t) * NLAT,
                               (size_t)ncopy, cudaMemcpyHostToDevice, cs);
+        if (e == cudaSuccess) e = cudaEventRecord(ctx->lat_ev, cs);
+      }
     }
     if (e == cudaSuccess && reset) e = cudaMemsetAsync(ctx->d_stats, 0, sizeof(uint64_t) * NSTAT * ctx->stats_cap, cs);
     if (e == cudaSuccess && dst_is_host) {

@@ -98,6 +98,8 @@ void ctx_release(DeviceCtx* c) {
   }
   cudaFree(c->d_stats);
   cudaFree(c->d_ring);
+  cudaFreeHost(c->h_lat_pinned);
+  if (c->lat_ev) cudaEventDestroy(c->lat_ev);
   cudaStreamDestroy(c->copy_stream);
   g_ctx[c->device] = nullptr;
   delete c;
@@ -401,6 +403,7 @@ static ffsva_status batch_alloc(DeviceCtx* ctx, Batch* b, int32_t cap, int32_t s
 
 ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, int32_t n, bool sdd_only,
                          bool want_d100, cudaStream_t st) {
+  NvtxRange r("ffsva batch: build (validate, plan, upload descriptors)");
   const StreamState* s0 = frames[0].stream;
   const int32_t sdd_w = s0->desc.sdd_w, sdd_h = s0->desc.sdd_h;
   SddPlan plan;
@@ -645,6 +648,7 @@ ffsva_status batch_profile(Batch* const* batches, int32_t nb, int32_t iters, flo
 }
 
 ffsva_status batch_run(Batch* b, cudaStream_t st, bool use_graph) {
+  NvtxRange r("ffsva batch: K1 -> K3 -> K4");
   DeviceCtx* ctx = b->ctx;
   if (b->n == 0) return FFSVA_OK;
   if (!use_graph || st == nullptr) {

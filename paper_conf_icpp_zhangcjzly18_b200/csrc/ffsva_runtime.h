@@ -6,6 +6,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "ffsva.h"
 #include "ffsva_internal.h"
 
@@ -80,6 +82,10 @@ struct DeviceCtx {
   unsigned long long* d_stats = nullptr;  // [stats_cap][NSTAT] (kernel counters)
   std::mutex lat_mu;                      // guards h_lat (the online runtime records under its own lock)
   std::vector<uint64_t> h_lat;            // [stats_cap][NLAT] (online arrival -> decision latency, a8)
+  // pinned snapshot of h_lat for ffsva_stats_copy into device memory: the copy stays asynchronous (no host sync on
+  // the caller's stream, e.g. inside a timed region); lat_ev guards the snapshot until its copy has run
+  uint64_t* h_lat_pinned = nullptr;
+  cudaEvent_t lat_ev = nullptr;
   int32_t stats_cap = 0;
   bool sticky = false;
   Batch* scratch = nullptr;  // reusable batch for ffsva_filter_batch / ffsva_sdd_batch
@@ -140,6 +146,12 @@ DeviceCtx* tyolo_device_ctx(const ffsva_tyolo* m);
 ffsva_status tyolo_run_unlocked(ffsva_tyolo* m, const ffsva_frame* frames, int32_t n, const int32_t* targets,
                                 float thresh, int32_t number_of_objects, int32_t* counts, uint8_t* pass, float* raw,
                                 cudaStream_t cs);
+
+// NVTX range (header-only NVTX3: a no-op unless a tool such as ncu / nsys injects itself)
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 // RAII device switch
 struct DeviceGuard {

@@ -15,6 +15,8 @@
 #include <unordered_map>
 #include <vector>
 
+#include <cstdlib>
+
 #include "ffsva_runtime.h"
 #include "ffsva_sched_policy.h"
 
@@ -87,11 +89,16 @@ struct ffsva_sched {
   ffsva_tyolo* tyolo = nullptr;
   float ty_thresh = 0.2f;
   std::vector<sched::QFrame> tyflat;
+  // per-stage CUDA graphs (updated in place tick to tick); FFSVA_SCHED_GRAPH=0 launches directly (A/B)
+  bool use_graph = true;
+  cudaGraphExec_t g_sdd = nullptr, g_snm = nullptr;
 };
 
 namespace {
 
 void sched_free(ffsva_sched* s) {
+  if (s->g_sdd) cudaGraphExecDestroy(s->g_sdd);
+  if (s->g_snm) cudaGraphExecDestroy(s->g_snm);
   if (s->done_ev) cudaEventDestroy(s->done_ev);
   cudaFree(s->d_pool);
   cudaFree(s->d_in);
@@ -133,6 +140,7 @@ struct SnmStage {
 // SDD admission (feedback: streams whose SNM queue is over q_snm wait) into host staging h: one D50 slot per
 // admitted frame, frame descriptors, per-stream segments (admitted frames arrive grouped by stream).
 SddStage prep_sdd(ffsva_sched* s, uint8_t* h, const Layout& L, std::vector<sched::QFrame>& adm) {
+  NvtxRange r("ffsva sched: SDD admission");
   SddStage sd;
   adm = s->pol.admit_sdd(s->max_frames, (int32_t)s->free_slots.size());
   sd.na = (int32_t)adm.size();
@@ -165,13 +173,12 @@ SddStage prep_sdd(ffsva_sched* s, uint8_t* h, const Layout& L, std::vector<sched
 
 // Upload the SDD staging (used parts only) into device region d, launch K1 (D50 into the slots) and K3 (threshold),
 // queue the D2H of distances and pass flags into h_out. Asynchronous on cs.
-cudaError_t launch_sdd_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layout& L, const SddStage& sd,
-                             cudaStream_t cs) {
+cudaError_t enqueue_sdd_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layout& L, const SddStage& sd,
+                              cudaStream_t cs) {
   DeviceCtx* ctx = s->ctx;
   const size_t n = (size_t)s->cap;
   const int32_t na = sd.na, nseg = sd.nseg;
-  cudaError_t e = sdd_configure(sd.plan.smem);
-  if (e == cudaSuccess) e = cudaMemcpyAsync(d + L.desc, h + L.desc, 64 * (size_t)na, cudaMemcpyHostToDevice, cs);
+  cudaError_t e = cudaMemcpyAsync(d + L.desc, h + L.desc, 64 * (size_t)na, cudaMemcpyHostToDevice, cs);
   if (e == cudaSuccess) e = cudaMemcpyAsync(d + L.index, h + L.index, 4 * (size_t)na, cudaMemcpyHostToDevice, cs);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(d + L.seg_lo, h + L.seg_lo, 4 * (size_t)(nseg + 1), cudaMemcpyHostToDevice, cs);
@@ -221,6 +228,7 @@ cudaError_t launch_sdd_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layou
 
 // SDD results (in h_out) of admissions adm[0, na): survivors join their SNM queue, dropped frames become events.
 void harvest_sdd(ffsva_sched* s, std::vector<sched::QFrame>& adm, int32_t na, ffsva_tick_info& ti) {
+  NvtxRange r("ffsva sched: SDD harvest");
   const size_t n = (size_t)s->cap;
   const uint64_t* h_ssd = at<uint64_t>(s->h_out, 0);
   const uint8_t* h_pass = s->h_out + 12 * n;
@@ -290,8 +298,8 @@ SnmStage prep_snm(ffsva_sched* s, uint8_t* h, const Layout& L, std::vector<sched
 
 // Upload the SNM staging into device region d, launch K4 on the popped frames' slots, queue the D2H of logits,
 // decisions and classes into h_out. Asynchronous on cs.
-cudaError_t launch_snm_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layout& L, const SnmStage& sn,
-                             cudaStream_t cs) {
+cudaError_t enqueue_snm_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layout& L, const SnmStage& sn,
+                              cudaStream_t cs) {
   const size_t n = (size_t)s->cap;
   const int32_t m = sn.m, nch = sn.nch;
   cudaError_t e = cudaMemcpyAsync(d + L.desc, h + L.desc, 64 * (size_t)m, cudaMemcpyHostToDevice, cs);
@@ -323,9 +331,56 @@ cudaError_t launch_snm_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layou
   return e;
 }
 
+// A stage's copies and kernels as a CUDA graph (SURVEY.md §3 "steady-state ticks are replayed as a captured CUDA
+// graph"): the tick's enqueue is captured, the stage's instantiated graph is updated in place when the topology
+// matches (only parameters change from tick to tick: counts, grids, staging offsets) or re-instantiated otherwise,
+// and launched as one unit. The legacy NULL stream cannot be captured: ticks on it enqueue directly.
+template <typename F>
+cudaError_t graph_launch(cudaGraphExec_t& exec, cudaStream_t cs, F&& enqueue) {
+  cudaGraph_t g = nullptr;
+  cudaError_t e = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal);
+  if (e != cudaSuccess) return e;
+  const cudaError_t fe = enqueue();
+  e = cudaStreamEndCapture(cs, &g);
+  if (fe != cudaSuccess) {
+    if (g) cudaGraphDestroy(g);
+    return fe;
+  }
+  if (e != cudaSuccess) return e;
+  if (exec) {
+    cudaGraphExecUpdateResultInfo info;
+    if (cudaGraphExecUpdate(exec, g, &info) != cudaSuccess) {  // topology changed: instantiate afresh
+      cudaGetLastError();
+      cudaGraphExecDestroy(exec);
+      exec = nullptr;
+    }
+  }
+  if (!exec) e = cudaGraphInstantiate(&exec, g, 0);
+  cudaGraphDestroy(g);
+  if (e == cudaSuccess) e = cudaGraphLaunch(exec, cs);
+  return e;
+}
+
+cudaError_t launch_sdd_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layout& L, const SddStage& sd,
+                             cudaStream_t cs) {
+  NvtxRange r("ffsva sched: SDD stage launch");
+  cudaError_t e = sdd_configure(sd.plan.smem);  // a function attribute: outside any capture
+  if (e != cudaSuccess) return e;
+  if (!s->use_graph || cs == nullptr) return enqueue_sdd_stage(s, h, d, L, sd, cs);
+  return graph_launch(s->g_sdd, cs, [&] { return enqueue_sdd_stage(s, h, d, L, sd, cs); });
+}
+
+cudaError_t launch_snm_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layout& L, const SnmStage& sn,
+                             cudaStream_t cs) {
+  NvtxRange r("ffsva sched: SNM stage launch");
+  if (!s->use_graph || cs == nullptr) return enqueue_snm_stage(s, h, d, L, sn, cs);
+  return graph_launch(s->g_snm, cs, [&] { return enqueue_snm_stage(s, h, d, L, sn, cs); });
+}
+
 // SNM results (in h_out) of pops flat[0, m): slots are freed; survivors with a T-YOLO stage wait in its queue,
 // every other frame becomes an event.
 void harvest_snm(ffsva_sched* s, std::vector<sched::QFrame>& flat, int32_t m) {
+  NvtxRange r("ffsva sched: SNM harvest");
   const size_t n = (size_t)s->cap;
   const float* h_logit = at<float>(s->h_out, 8 * n);
   const uint8_t* h_snm_pass = s->h_out + 13 * n;
@@ -355,6 +410,7 @@ void harvest_snm(ffsva_sched* s, std::vector<sched::QFrame>& flat, int32_t m) {
 // NumberofObjects per stream (L195). Synchronous on cs.
 ffsva_status tyolo_cycle(ffsva_sched* s, cudaStream_t cs, ffsva_tick_info& ti) {
   if (!s->tyolo) return FFSVA_OK;
+  NvtxRange r("ffsva sched: T-YOLO cycle");
   std::vector<sched::QFrame>& tf = s->tyflat;
   s->pol.pop_ty(tf);
   const int32_t nt = (int32_t)tf.size();
@@ -434,6 +490,7 @@ FFSVA_API ffsva_status ffsva_sched_create(int32_t device, int32_t max_frames_per
     return cuda_fail(nullptr, e, "ffsva_sched_create");
   }
   for (int32_t i = snm_slots - 1; i >= 0; --i) s->free_slots.push_back(i);
+  if (const char* g = std::getenv("FFSVA_SCHED_GRAPH")) s->use_graph = std::atoi(g) != 0;
   *out = s.release();
   return FFSVA_OK;
 }
@@ -584,6 +641,7 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
                                         int32_t* n_events, ffsva_tick_info* info) {
   if (!s || cap < 0 || (cap > 0 && !events) || !n_events) return fail(FFSVA_EINVAL, "bad argument");
   std::lock_guard<std::mutex> lk(s->mu);
+  NvtxRange nvtx_tick("ffsva_sched_tick");
   DeviceCtx* ctx = s->ctx;
   if (ctx->sticky) return fail(FFSVA_ECUDA, "device is in a sticky CUDA error state");
   std::lock_guard<std::mutex> dlk(ctx->mu);
