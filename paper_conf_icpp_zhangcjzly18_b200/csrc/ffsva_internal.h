@@ -39,16 +39,56 @@ constexpr int N_PARAMS = 27 * C1 + C1 + 9 * C1 * C2 + C2 + NF + 1;  // 9697
 // conv1 B operands, one per 4x4-patch row dy (the MMA's A rows are pooled pixels' 4x4 input patches, 4 channel
 // slots per pixel): N = 64 = [pool position q = 2a + b][16 output channels], K = 16 = [patch column u][4 channel
 // slots], value w1[oc][c][dy - a][u - b] where that tap exists (c < 3), else 0. Each is [2 K-halves][64 n][8 k] bf16.
+// Patch row 0 only reaches positions a = 0 (n < 32) and row 3 only a = 1 (n >= 32): those two MMAs use N = 32.
 constexpr int W1_MMAS = 4;
 constexpr int W1_BYTES = W1_MMAS * 2 * 64 * 16;     // 8192
-constexpr int W2_BYTES = 9 * 2 * C2 * 16;           // 9216: [tap][channel half][32 n][8] bf16
+// conv2 B operands, one per MMA of kConv2Mmas. The A operand of an MMA is one 3x3-window cell (Y', X') of the 4x4
+// patch around a pooled output pixel (Y', X' in 0..3, 16 input channels = K16); pool position (a, b) reads that cell
+// through tap (Y' - a, X' - b), so one A serves every position whose 3x3 window holds the cell: N = 32 x (positions
+// in one run of consecutive TMEM column groups, order kConv2Group). Each B is [2 K-halves][N][8] bf16.
+struct Conv2Mma {
+  int32_t cy, cx;   // patch cell (Y', X')
+  int32_t g0, ng;   // first TMEM column group (32 columns each) and number of groups (positions)
+  int32_t boff;     // byte offset of the B operand in the W2 region
+};
+// TMEM column group of pool position (a, b): (0,0) 0, (0,1) 1, (1,1) 2, (1,0) 3 — so the two-position cells of three
+// of the four edges are one contiguous run; the (0,0)+(1,0) cells (X' = 0) take two N = 32 MMAs.
+__host__ __device__ constexpr int conv2_group(int a, int b) { return a == 0 ? b : 3 - b; }
+constexpr int kConv2Mmas = 18;
+// MMA i of a conv2 tile (host packing and the kernel's issue loop, constant-folded there)
+__host__ __device__ constexpr Conv2Mma conv2_mma(int i) {
+  switch (i) {
+    // four-position cells first: the first MMA (accumulate = 0) initialises all 128 columns
+    case 0: return {1, 1, 0, 4, 0};
+    case 1: return {1, 2, 0, 4, 4096};
+    case 2: return {2, 1, 0, 4, 8192};
+    case 3: return {2, 2, 0, 4, 12288};
+    // two-position runs
+    case 4: return {0, 1, 0, 2, 16384};   // a = 0: (0,0) (0,1)
+    case 5: return {0, 2, 0, 2, 18432};
+    case 6: return {3, 1, 2, 2, 20480};   // a = 1: (1,1) (1,0)
+    case 7: return {3, 2, 2, 2, 22528};
+    case 8: return {1, 3, 1, 2, 24576};   // b = 1: (0,1) (1,1)
+    case 9: return {2, 3, 1, 2, 26624};
+    case 10: return {1, 0, 0, 1, 28672};  // b = 0: (0,0) | (1,0), not adjacent
+    case 11: return {1, 0, 3, 1, 29696};
+    case 12: return {2, 0, 0, 1, 30720};
+    case 13: return {2, 0, 3, 1, 31744};
+    // corners
+    case 14: return {0, 0, 0, 1, 32768};
+    case 15: return {0, 3, 1, 1, 33792};
+    case 16: return {3, 3, 2, 1, 34816};
+    default: return {3, 0, 3, 1, 35840};
+  }
+}
+constexpr int W2_BYTES = 36864;                     // 36 position-taps x 32 n x 32 B
 constexpr int OFF_W1 = 0;
 constexpr int OFF_W2 = OFF_W1 + W1_BYTES;           // 8192
-constexpr int OFF_B1 = OFF_W2 + W2_BYTES;           // 17408 (fp32[16])
-constexpr int OFF_B2 = OFF_B1 + C1 * 4;             // 17472 (fp32[32])
-constexpr int OFF_BFC = OFF_B2 + C2 * 4;            // 17600 (fp32[1] + pad to 16)
-constexpr int OFF_WFC = OFF_BFC + 16;               // 17616 (bf16[4608]: the weights are bf16 values, L159 Q15)
-constexpr int BLOB_BYTES = OFF_WFC + NF * 2;        // 26832
+constexpr int OFF_B1 = OFF_W2 + W2_BYTES;           // 45056 (fp32[16])
+constexpr int OFF_B2 = OFF_B1 + C1 * 4;             // 45120 (fp32[32])
+constexpr int OFF_BFC = OFF_B2 + C2 * 4;            // 45248 (fp32[1] + pad to 16)
+constexpr int OFF_WFC = OFF_BFC + 16;               // 45264: fp32 [8 channel quads][144 pixels][4] of bf16 values
+constexpr int BLOB_BYTES = OFF_WFC + NF * 4;        // 63696
 static_assert(BLOB_BYTES % 16 == 0, "blob must be 16-B granular");
 }  // namespace snm
 
@@ -141,13 +181,10 @@ struct SnmArgs {
   uint8_t* snm_pass;
   uint8_t* snm_class;
   unsigned long long* stats;
-  int32_t grid;
-  // debug taps (nullptr in production): pooled conv1 (bf16 as u16 [m][25][25][16]) and the pre-FC features
-  uint16_t* dbg_p1;
-  float* dbg_p2;             // [m][32][12][12]
+  int32_t grid;              // one CTA per SM at most: CTA c scores survivors [c*m/grid, (c+1)*m/grid) of work order
 };
 cudaError_t launch_snm(const SnmArgs& a, cudaStream_t st);
-constexpr int kSnmCtasPerSm = 2;  // K4 is persistent with two CTAs per SM (256 TMEM columns, < 113 KB smem each)
+constexpr int kSnmCtasPerSm = 1;  // K4 is persistent, one warp-specialised CTA per SM (all 512 TMEM columns, ~182 KB smem)
 int snm_smem_bytes();
 cudaError_t snm_configure();
 

@@ -309,18 +309,35 @@ void pack_snm_blob(const float* params, uint8_t* blob) {
             const int n = 16 * q + oc, h = u >> 1, kk = 4 * (u & 1) + c;
             W1[((dy * 2 + h) * 64 + n) * 8 + kk] = bf16_bits_rne(w1[((oc * 3 + c) * 3 + ky) * 3 + kx]);
           }
-  // conv2: tap t, K-half h = input channels 8h..8h+7
-  uint16_t* W2 = reinterpret_cast<uint16_t*>(blob + OFF_W2);
-  for (int t = 0; t < 9; ++t)
-    for (int h = 0; h < 2; ++h)
-      for (int n = 0; n < C2; ++n)
-        for (int c = 0; c < 8; ++c)
-          W2[((t * 2 + h) * C2 + n) * 8 + c] = bf16_bits_rne(w2[((n * C1 + 8 * h + c) * 3 + t / 3) * 3 + t % 3]);
+  // conv2: one B per MMA of conv2_mma (patch cell (Y', X')): row n = 32 * (group - g0) + oc holds the weights of pool
+  // position (a, b) of that group through tap (Y' - a, X' - b); K-half h = input channels 8h..8h+7.
+  for (int i = 0; i < kConv2Mmas; ++i) {
+    const Conv2Mma mm = conv2_mma(i);
+    uint16_t* B = reinterpret_cast<uint16_t*>(blob + OFF_W2 + mm.boff);
+    const int N = 32 * mm.ng;
+    for (int a = 0; a < 2; ++a)
+      for (int b = 0; b < 2; ++b) {
+        const int g = conv2_group(a, b) - mm.g0;
+        if (g < 0 || g >= mm.ng) continue;
+        const int ky = mm.cy - a, kx = mm.cx - b;
+        if (ky < 0 || ky > 2 || kx < 0 || kx > 2) std::abort();  // the table only lists taps that exist
+        for (int oc = 0; oc < C2; ++oc)
+          for (int h = 0; h < 2; ++h)
+            for (int c = 0; c < 8; ++c)
+              B[(h * N + 32 * g + oc) * 8 + c] = bf16_bits_rne(w2[((oc * C1 + 8 * h + c) * 3 + ky) * 3 + kx]);
+      }
+  }
   std::memcpy(blob + OFF_B1, b1, C1 * 4);
   std::memcpy(blob + OFF_B2, b2, C2 * 4);
   std::memcpy(blob + OFF_BFC, bfc, 4);
-  uint16_t* F = reinterpret_cast<uint16_t*>(blob + OFF_WFC);
-  for (int i = 0; i < NF; ++i) F[i] = bf16_bits_rne(wfc[i]);
+  // FC weights: bf16 values (Q15) held as fp32, [channel quad][pooled pixel][4] so a lane reads its pixel's 32 weights
+  // with eight 16-byte loads, consecutive lanes at consecutive addresses
+  float* F = reinterpret_cast<float*>(blob + OFF_WFC);
+  for (int c = 0; c < C2; ++c)
+    for (int p = 0; p < P2 * P2; ++p) {
+      const uint32_t bits = (uint32_t)bf16_bits_rne(wfc[c * P2 * P2 + p]) << 16;
+      std::memcpy(&F[((c >> 2) * P2 * P2 + p) * 4 + (c & 3)], &bits, 4);
+    }
 }
 
 // ------------------------------------------------------------------ batches

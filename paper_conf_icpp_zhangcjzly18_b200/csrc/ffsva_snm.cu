@@ -7,27 +7,33 @@
 // 4608->1 logit (Q9, Q11); input (v-128)/128 (Q10); bf16 operands, fp32 accumulation, pooled conv1 rounded
 // to bf16, conv2 output and FC in fp32 (Q15).
 //
-// B200 mapping — implicit GEMM, no im2col, pooling folded into the N dimension:
+// B200 mapping — implicit GEMMs, no im2col, pooling folded into the N dimension:
 //   * GEMM rows are POOLED output pixels; a 2x2-pool's four conv outputs are four accumulator column groups of the
-//     same TMEM lane, so the max-pool is an in-register max over four column groups (no cross-lane shuffles); bias
-//     and ReLU commute with max and are applied once after it.
-//   * conv1: the A row of pooled pixel (py, px) is its 4x4 input patch (padded rows 2py..2py+3, columns
+//     same TMEM lane, so the max-pool is an in-register max over four column groups; bias and ReLU commute with max
+//     and are applied once after it (max(v0..v3, -b) + b).
+//   * Cost model (tools/microbench/mma_rate.cu, one B200): an M128 K16 bf16 MMA costs 32 + N/4 clocks up to N = 128
+//     (shared-memory operand reads: the 4 KB A tile plus N x 32 B of B at 128 B/clk) and N/2 clocks beyond, so an MMA
+//     should read each A tile for as many output columns as possible.
+//   * conv1: the A row of pooled pixel (py, px) is its 4x4 input patch row dy (padded input row 2py + dy, columns
 //     2px..2px+3) x 4 channel slots (3 used); the four pool positions differ only in where their 3x3 kernel sits in
-//     the patch, so ONE A operand feeds N = 64 = 4 positions x 16 channels with per-position (zero-padded) weights:
-//     4 MMAs (M128 N64 K16, one per patch row) per tile of 4 pooled rows x 32 px instead of 24 narrow ones. The
-//     input lives in two row-parity planes of 64-px rows, 8 bytes per pixel, so a patch row of consecutive pooled
-//     pixels is a constant-stride view (rows 16 B apart, K-halves 16 B apart, 8-row groups 128 B apart): each
-//     patch row is the same UMMA descriptor moved by one plane row.
-//   * conv2 (16 channels = two 8-channel planes, LBO = plane distance): per pool position and tap one MMA
-//     (M128, N32) per tile x 2 tiles of 8 pooled rows x 16 px, A from four parity planes like conv1's patch rows.
+//     the patch, so ONE A operand feeds N = 4 positions x 16 channels: per 128-row tile two N = 64 MMAs (patch rows
+//     1, 2) and two N = 32 MMAs (row 0 reaches only positions a = 0, row 3 only a = 1). The input lives in two
+//     row-parity planes of 26 two-pixel entries per row, so GEMM row r = plane entry r: pooled pixel (r / 26, r % 26)
+//     and every patch row is a constant-stride view (rows 16 B apart, K-halves 16 B apart, 8-row groups 128 B apart):
+//     6 tiles cover the 25 x 25 pooled outputs (650 of 768 rows useful).
+//   * conv2: the 4x4 patch of a pooled output pixel has 16 cells; a cell's A view (16 channels = two 8-channel
+//     parity planes, rows = plane entries r, pooled pixel (r / 14, r % 14)) serves every pool position whose 3x3
+//     window holds it, so the 36 (position, tap) products of a tile take 18 MMAs (4 x N128, 6 x N64, 8 x N32,
+//     snm::conv2_mma) instead of 36 x N32; 2 tiles cover the 12 x 12 pooled outputs.
 //   * conv1's epilogue writes bf16 pooled activations straight into conv2's parity planes; conv2's epilogue
 //     multiplies the pooled features by the FC weights (bf16 values) in fp32 and reduces to one logit per frame.
-// Two persistent CTAs per SM (8 warps and 256 TMEM columns each: conv1 runs as two waves of <= 4 tiles, conv2's two
-// tiles reuse the columns), so one CTA's epilogues overlap the other's MMAs. MMAs are issued by a whole warp (one
-// elected lane) per warp group and committed per tile to its own mbarrier so epilogues start as soon as a tile lands.
-// Work = dynamic-batch units (<= BatchSize survivors of one stream, split further when the batch is small); the
-// stream's 26 KB weight image is copied into shared memory once per unit (skipped when the previous unit was the
-// same stream), and the next frame's D50 image is prefetched with a bulk copy.
+// One warp-specialised persistent CTA per SM (512 threads, all 512 TMEM columns), frames pipelined through
+// mbarrier rings: warp 0 stages each frame's D50 image (bulk copy) and the stream's weight image when the stream
+// changes; warps 4-7 convert D50 to conv1's bf16 operand (two buffers); warp 1 issues the MMAs (conv1 tiles into a
+// ring of four 64-column TMEM slots, conv2 tiles into two 128-column slots, frame j+1's conv1 interleaved with frame
+// j's conv2); warps 8-11 drain conv1 tiles into conv2's operand (two buffers); warps 12-15 drain conv2 tiles, apply
+// the FC and decide. CTA c scores the survivors [c*m/G, (c+1)*m/G) of the stream-major work order, so a stream's
+// weights are loaded once per CTA and per stream (a dynamic batch's frames are consecutive, L219).
 #include <cuda_bf16.h>
 
 #include "ffsva_internal.h"
@@ -37,299 +43,410 @@ namespace ffsva {
 namespace {
 
 using namespace snm;
-
-constexpr int kThreads = 256;
-// conv1 operand: 2 row-parity planes x 27 rows x 64 px x 8 B (padded input 52x52, 4 channel slots, 3 used)
-constexpr int A1_COLS = 64, A1_ROWS = 27;
-constexpr int A1_ROWB = A1_COLS * 8;                        // 512: pooled row -> next plane row = four 8-row groups
-constexpr int A1_PLANE = A1_ROWS * A1_ROWB;                 // 13824
-constexpr int A1_BYTES = 2 * A1_PLANE + 512;                // + tail read by junk columns of the last plane row
-// conv2 operand: 8 planes [ypar][xpar][chalf] x 14 rows x 16 px x 16 B (padded pooled conv1 27x27, 16 ch)
-constexpr int A2_COLS = 16, A2_ROWS = 14;
-constexpr int A2_PLANE = A2_ROWS * A2_COLS * 16;            // 3584
-constexpr int A2_BYTES = 8 * A2_PLANE + 512;                // + zero tail read by junk rows of the last tile
-constexpr int D50_BYTES = 7504;                             // staged D50 image (one frame)
-constexpr int OFF_A1 = 0;
-constexpr int OFF_A2 = OFF_A1 + A1_BYTES;                   // 28160
-constexpr int OFF_WB = OFF_A2 + A2_BYTES;                   // 57344
-constexpr int OFF_IN = OFF_WB + BLOB_BYTES;                 // 2 staging buffers
-constexpr int OFF_LUT = OFF_IN + 2 * D50_BYTES;             // u16[256]: bf16 bits of (v - 128) / 128
-constexpr int OFF_RED = OFF_LUT + 512;
-constexpr int OFF_BAR = OFF_RED + 64;                       // 7 conv1 + 2 conv2 + 2 input mbarriers
-constexpr int OFF_TMEM = OFF_BAR + 16 * 8;
-constexpr int SMEM_BYTES = OFF_TMEM + 16;
-static_assert(SMEM_BYTES <= 113 * 1024, "two CTAs per SM");
-static_assert(OFF_A2 % 16 == 0 && OFF_WB % 16 == 0 && OFF_IN % 16 == 0, "16-byte alignment");
-constexpr uint32_t kTmemCols = 256;
-
-constexpr int kTiles1 = 7;
-__constant__ int8_t c1_py0[kTiles1] = {0, 4, 8, 12, 16, 20, 21};  // last tile overlaps (idempotent writes)
-
-// PTX wrappers (tcgen05 MMA / TMEM, mbarriers, bulk copies): ffsva_ptx.h
 using namespace ptx;
 
-// max over the four pool positions: 16 consecutive channels starting at column col of each position group
-__device__ __forceinline__ void pooled16(uint32_t taddr, int col, int group_cols, float (&v)[16]) {
+constexpr int kThreads = 512;
+constexpr int NIN = 3;   // D50 staging ring
+constexpr int NI = 16;   // per-frame info ring (frames in flight between the producer and the conv2 epilogue)
+// conv1 operand: 2 row-parity planes x 26 rows x 26 entries (two padded pixels x 4 channel slots, 16 B)
+constexpr int A1_ROW = 26;                                  // entries per plane row
+constexpr int A1_PLANE = 26 * A1_ROW * 16;                  // 10816 B
+constexpr int A1_BYTES = 23552;                             // + tail read by junk rows of tile 5 (entry 1470 max)
+static_assert(A1_BYTES >= (A1_PLANE / 16 + 26 + 767 + 1 + 1) * 16, "conv1 operand tail");
+constexpr int kTiles1 = 6;
+// conv2 operand: 8 planes [ypar][xpar][chalf] x 14 rows x 14 entries of 8 channels (padded pooled conv1 27x27)
+constexpr int A2_COLS = 14;
+constexpr int A2_PLANE = 14 * A2_COLS * 16 + 32;            // 3168 B: the two column-parity planes of a channel half
+                                                            // are 2 * 3168 = 64 (mod 128) B apart, so the conv1
+                                                            // epilogue's stores of both parities do not share banks
+constexpr int A2_BYTES = 26512;                             // + tail read by junk rows of tile 1 (entry 1656 max)
+static_assert(A2_BYTES >= (7 * A2_PLANE / 16 + 255 + A2_COLS + 1 + 1) * 16, "conv2 operand tail");
+constexpr int D50_BYTES = 7504;                             // staged D50 image (one frame)
+
+constexpr int OFF_WB = 0;                                   // the stream's weight image (snm::BLOB_BYTES)
+constexpr int OFF_A1 = 63744;                               // 2 buffers
+constexpr int OFF_A2 = OFF_A1 + 2 * A1_BYTES;               // 110848, 2 buffers
+constexpr int OFF_IN = OFF_A2 + 2 * A2_BYTES;               // 163872, NIN stages
+constexpr int OFF_INFO = OFF_IN + NIN * D50_BYTES;          // 186384: int2 [NI] (frame, flags)
+constexpr int OFF_RED = OFF_INFO + NI * 8;                  // float [2][4]
+constexpr int OFF_BAR = OFF_RED + 32;
+// mbarriers (8 B each)
+constexpr int B_IN_FULL = 0, B_IN_EMPTY = B_IN_FULL + NIN, B_W_FULL = B_IN_EMPTY + NIN, B_W_EMPTY = B_W_FULL + 1,
+              B_INFO_EMPTY = B_W_EMPTY + 1, B_A1_FULL = B_INFO_EMPTY + NI, B_A1_EMPTY = B_A1_FULL + 2,
+              B_C1_FULL = B_A1_EMPTY + 2, B_C1_EMPTY = B_C1_FULL + 4, B_A2_FULL = B_C1_EMPTY + 4,
+              B_A2_EMPTY = B_A2_FULL + 2, B_C2_FULL = B_A2_EMPTY + 2, B_C2_EMPTY = B_C2_FULL + 2,
+              N_BARS = B_C2_EMPTY + 2;
+constexpr int OFF_TMEM = OFF_BAR + N_BARS * 8;
+constexpr int SMEM_BYTES = OFF_TMEM + 16;
+static_assert(OFF_A1 >= BLOB_BYTES && OFF_A1 % 128 == 0, "weight image fits");
+static_assert(OFF_A2 % 16 == 0 && OFF_IN % 16 == 0 && OFF_INFO % 16 == 0 && OFF_BAR % 8 == 0, "alignment");
+static_assert(SMEM_BYTES <= 227 * 1024, "one CTA per SM");
+constexpr uint32_t kTmemCols = 512;                         // conv1: 4 x 64 columns; conv2: 256 + 2 x 128
+constexpr uint32_t kC2Col = 256;
+
+// per-frame flags in the info ring
+constexpr int F_SEG_FIRST = 1, F_SEG_LAST = 2, F_POP_OPEN = 4;
+
+__device__ __forceinline__ float max3(float a, float b, float c) {
+  float d;
+  asm("max.f32 %0, %1, %2, %3;" : "=f"(d) : "f"(a), "f"(b), "f"(c));
+  return d;
+}
+// max over the four pool positions (16 consecutive channels from column col of each group), then bias and ReLU:
+// max_q(v_q + b) clamped at 0 == max(v_0, v_1, v_2, v_3, -b) + b (fp addition is monotone)
+__device__ __forceinline__ void pool_bias_relu16(uint32_t taddr, int col, int group_cols, const float* bias,
+                                                 float (&v)[16]) {
   uint32_t r0[16], r1[16], r2[16], r3[16];
   tmem_ld16(taddr + (uint32_t)col, r0);
   tmem_ld16(taddr + (uint32_t)(col + group_cols), r1);
   tmem_ld16(taddr + (uint32_t)(col + 2 * group_cols), r2);
   tmem_ld16(taddr + (uint32_t)(col + 3 * group_cols), r3);
   tmem_wait_ld2(r0, r1);
-  tmem_wait_ld2(r2, r3);
+  reg_fence2(r2, r3);
 #pragma unroll
-  for (int i = 0; i < 16; ++i)
-    v[i] = fmaxf(fmaxf(__uint_as_float(r0[i]), __uint_as_float(r1[i])),
-                 fmaxf(__uint_as_float(r2[i]), __uint_as_float(r3[i])));
-}
-
-__device__ __forceinline__ uint32_t u8_to_bf16(uint32_t v) {  // (v - 128) / 128 is exact in bf16
-  return (uint32_t)__bfloat16_as_ushort(__float2bfloat16_rn(((float)v - 128.0f) * 0.0078125f));
+  for (int i = 0; i < 16; ++i) {
+    const float b = bias[i];
+    v[i] = max3(max3(__uint_as_float(r0[i]), __uint_as_float(r1[i]), __uint_as_float(r2[i])), __uint_as_float(r3[i]),
+                -b) + b;
+  }
 }
 
 __device__ __forceinline__ const uint8_t* d50_of(const SnmArgs& a, int f) {
   return a.d50 + (a.d50_index ? (int64_t)__ldg(a.d50_index + f) : (int64_t)f) * a.d50_stride;
 }
 
-// ---------------------------------------------------------------- input staging
-// D50 (50x50x3 u8, row-major) -> (v-128)/128 bf16 (C5, exact) into conv1's row-parity planes, one 8-byte pixel
-// (3 channels + a zero slot) per store. Groups of 4 pixels = 12 bytes = three aligned 32-bit shared loads; each
-// channel through a 256-entry bf16 table.
-__device__ __forceinline__ void convert_input(const uint8_t* d, uint8_t* A1, const uint16_t* lut) {
-  constexpr int kGroups = snm::IN * snm::IN / 4;  // 625
-  for (int g = threadIdx.x; g < kGroups; g += kThreads) {
-    const uint32_t* w = reinterpret_cast<const uint32_t*>(d + 12 * g);
+// ---------------------------------------------------------------- MMA issue (warp 1, one elected lane)
+// conv1 tile t of the frame in A1 buffer a1 into TMEM columns d..d+63 ([a][b][16 channels]).
+__device__ __forceinline__ void issue_conv1_tile(uint32_t d, uint32_t a1, int t, uint32_t w1) {
+  const uint32_t id64 = idesc_bf16(128, 64), id32 = idesc_bf16(128, 32);
+  const uint32_t r0 = a1 + (uint32_t)(128 * t * 16);
+  // patch row dy: plane dy & 1, plane row offset dy >> 1 (26 entries)
+  const uint32_t row0 = r0, row1 = r0 + A1_PLANE, row2 = r0 + A1_ROW * 16, row3 = r0 + A1_PLANE + A1_ROW * 16;
+  mma_bf16(d, umma_desc(row1, 16, 128), umma_desc(w1 + 1 * 2048, 1024, 128), id64, 0u);
+  mma_bf16(d, umma_desc(row2, 16, 128), umma_desc(w1 + 2 * 2048, 1024, 128), id64, 1u);
+  mma_bf16(d, umma_desc(row0, 16, 128), umma_desc(w1 + 0 * 2048, 1024, 128), id32, 1u);
+  mma_bf16(d + 32, umma_desc(row3, 16, 128), umma_desc(w1 + 3 * 2048 + 512, 1024, 128), id32, 1u);
+}
+
+// conv2 tile u of the frame in A2 buffer a2 into TMEM columns d..d+127 ([group][32 channels]).
+__device__ __forceinline__ void issue_conv2_tile(uint32_t d, uint32_t a2, int u, uint32_t w2) {
+#pragma unroll
+  for (int i = 0; i < kConv2Mmas; ++i) {
+    const Conv2Mma mm = conv2_mma(i);
+    const uint32_t plane = (uint32_t)((((mm.cy & 1) * 2 + (mm.cx & 1)) * 2) * A2_PLANE);
+    const uint32_t start = (uint32_t)((128 * u + (mm.cy >> 1) * A2_COLS + (mm.cx >> 1)) * 16);
+    const int N = 32 * mm.ng;
+    mma_bf16(d + (uint32_t)(32 * mm.g0), umma_desc(a2 + plane + start, A2_PLANE, 128),
+             umma_desc(w2 + (uint32_t)mm.boff, (uint32_t)(N * 16), 128), idesc_bf16(128, N), i > 0 ? 1u : 0u);
+  }
+}
+
+// ---------------------------------------------------------------- input conversion (warps 4-7)
+// D50 (50x50x3 u8, row-major) -> (v-128)/128 bf16 (C5, exact) into conv1's row-parity planes. A thread writes one
+// 16-byte entry = padded columns (2e, 2e+1) = image columns (2e-1, 2e) of one row, 4 channel slots each (3 used);
+// its 6 source bytes are funnel-shifted out of two aligned words (lanes ~6 B apart: conflict-free loads, contiguous
+// 16-byte stores). bf16 of (v-128)/128 = high half of fma(2^23 + v, 1/128, -65537), 2^23 + v by one PRMT.
+__device__ __forceinline__ uint32_t bf16_hi_of_byte(uint32_t w, uint32_t k) {
+  return __float_as_uint(fmaf(__uint_as_float(__byte_perm(w, 0x4B000000u, 0x7440u | k)), 0.0078125f, -65537.0f));
+}
+__device__ __forceinline__ void convert_input(const uint8_t* d, uint8_t* A1, int t) {
+  constexpr int kEntries = IN * A1_ROW;  // 50 rows x 26 entries
+  for (int q = t; q < kEntries; q += 128) {
+    const int y = q / A1_ROW, e = q - y * A1_ROW;
+    // bytes [o, o + 6) of the image: columns 2e-1 and 2e (column -1 / 50 are the zero border)
+    const int o = y * 3 * IN + 6 * e - 3;
+    const int ob = o < 0 ? 0 : o & ~3;  // aligned base word (the first entry of row 0 starts before the image)
+    const uint32_t* w = reinterpret_cast<const uint32_t*>(d + ob);
     const uint32_t w0 = w[0], w1 = w[1], w2 = w[2];
-    const uint32_t b[12] = {w0 & 255u, (w0 >> 8) & 255u, (w0 >> 16) & 255u, w0 >> 24,
-                            w1 & 255u, (w1 >> 8) & 255u, (w1 >> 16) & 255u, w1 >> 24,
-                            w2 & 255u, (w2 >> 8) & 255u, (w2 >> 16) & 255u, w2 >> 24};
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const int p = 4 * g + q;
-      const int y = p / snm::IN, x = p - y * snm::IN;
-      const int Y = y + 1, X = x + 1;
-      const uint2 v = make_uint2((uint32_t)lut[b[3 * q]] | ((uint32_t)lut[b[3 * q + 1]] << 16), (uint32_t)lut[b[3 * q + 2]]);
-      *reinterpret_cast<uint2*>(A1 + (Y & 1) * A1_PLANE + (Y >> 1) * A1_ROWB + X * 8) = v;
+    const uint32_t sh = (uint32_t)(o - ob) * 8u;  // 0..24 bits (o >= ob except row 0, entry 0: handled below)
+    const uint32_t lo = __funnelshift_r(w0, w1, sh), hi = __funnelshift_r(w1, w2, sh);  // bytes o .. o+7
+    uint32_t c[6];
+    c[0] = bf16_hi_of_byte(lo, 0);
+    c[1] = bf16_hi_of_byte(lo, 1);
+    c[2] = bf16_hi_of_byte(lo, 2);
+    c[3] = bf16_hi_of_byte(lo, 3);
+    c[4] = bf16_hi_of_byte(hi, 0);
+    c[5] = bf16_hi_of_byte(hi, 1);
+    uint4 v = make_uint4(__byte_perm(c[0], c[1], 0x7632), c[2] >> 16, __byte_perm(c[3], c[4], 0x7632), c[5] >> 16);
+    if (e == 0) v.x = v.y = 0u;                   // column -1: left border
+    if (e == A1_ROW - 1) v.z = v.w = 0u;          // column 50: right border
+    if (o < 0) {                                  // row 0, entry 0: column 0 is bytes 0..2
+      v.z = __byte_perm(bf16_hi_of_byte(w0, 0), bf16_hi_of_byte(w0, 1), 0x7632);
+      v.w = bf16_hi_of_byte(w0, 2) >> 16;
     }
-  }
-}
-
-// ---------------------------------------------------------------- MMA issue (one thread per warp group)
-// conv1 tile t (pooled rows py0..py0+3 x 32 px) into TMEM columns col..col+63 ([pool position][16 channels]):
-// patch row dy of pooled row py is padded input row 2py + dy = plane (dy & 1), plane row py + (dy >> 1).
-__device__ __forceinline__ void issue_conv1_tile(uint32_t tmem, uint32_t col, int t, uint32_t a1, uint32_t w1) {
-  const int py0 = c1_py0[t];
-  const uint32_t idesc = idesc_bf16(128, 64);
-#pragma unroll
-  for (int dy = 0; dy < 4; ++dy) {
-    const uint32_t arow = a1 + (uint32_t)((dy & 1) * A1_PLANE + (py0 + (dy >> 1)) * A1_ROWB);
-    // K-halves = patch columns (0,1) and (2,1+2): 16 B apart; 8-row groups (8 pooled px) 128 B apart
-    mma_bf16(tmem + col, umma_desc(arow, 16, 128), umma_desc(w1 + (uint32_t)(dy * 2 * 64 * 16), 64 * 16, 128), idesc,
-             dy > 0 ? 1u : 0u);
-  }
-}
-
-__device__ __forceinline__ void issue_conv2_tile(uint32_t tmem, int u, uint32_t a2, uint32_t w2) {
-  const int py0 = 4 * u;
-  const uint32_t idesc = idesc_bf16(128, 32);
-#pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    const int a = q >> 1, b = q & 1;
-    const uint32_t d = tmem + (uint32_t)(u * 128 + q * 32);
-#pragma unroll
-    for (int tap = 0; tap < 9; ++tap) {
-      const int dy = tap / 3, dx = tap % 3;
-      const int ypar = (a + dy) & 1, roff = (a + dy) >> 1, xpar = (b + dx) & 1, coff = (b + dx) >> 1;
-      const uint32_t addr = a2 + (uint32_t)(((ypar * 2 + xpar) * 2) * A2_PLANE + ((py0 + roff) * A2_COLS + coff) * 16);
-      mma_bf16(d, umma_desc(addr, A2_PLANE, 128), umma_desc(w2 + (uint32_t)(tap * 2 * C2 * 16), C2 * 16, 128), idesc,
-               tap > 0 ? 1u : 0u);
-    }
+    const int Y = y + 1;
+    *reinterpret_cast<uint4*>(A1 + (Y & 1) * A1_PLANE + ((Y >> 1) * A1_ROW + e) * 16) = v;
   }
 }
 
 // ---------------------------------------------------------------- epilogues
-// conv1 tile t: lane (quadrant qd, l) = pooled pixel (py0 + qd, l); bias, ReLU, bf16 into conv2's planes.
-__device__ __forceinline__ void conv1_epilogue(uint32_t tmem, uint32_t col, int t, uint8_t* A2, const float* b1,
-                                               uint16_t* dbg) {
+// conv1 tile t, TMEM slot columns col: lane (quadrant qd, l) = GEMM row r = 128t + 32qd + l = pooled pixel
+// (r / 26, r % 26); bias, ReLU, bf16 into conv2's parity planes (border entries stay zero).
+__device__ __forceinline__ void conv1_epilogue(uint32_t tmem, uint32_t col, int t, uint8_t* A2, const float* b1) {
   const int qd = (threadIdx.x >> 5) & 3, l = threadIdx.x & 31;
   float v[16];
-  pooled16(tmem + ((uint32_t)(32 * qd) << 16), (int)col, 16, v);
-  const int py = c1_py0[t] + qd, px = l;
-  if (px < P1) {
+  pool_bias_relu16(tmem + ((uint32_t)(32 * qd) << 16), (int)col, 16, b1, v);
+  const int r = 128 * t + 32 * qd + l;
+  const int py = r / A1_ROW, px = r - py * A1_ROW;
+  if (py < P1 && px < P1) {
     uint32_t w[8];
 #pragma unroll
-    for (int i = 0; i < 8; ++i) w[i] = pack_bf16(fmaxf(v[2 * i] + b1[2 * i], 0.f), fmaxf(v[2 * i + 1] + b1[2 * i + 1], 0.f));
+    for (int i = 0; i < 8; ++i) w[i] = pack_bf16(v[2 * i], v[2 * i + 1]);
     const int Y = py + 1, X = px + 1;
     uint8_t* p = A2 + ((((Y & 1) * 2 + (X & 1)) * 2) * A2_PLANE + ((Y >> 1) * A2_COLS + (X >> 1)) * 16);
     *reinterpret_cast<uint4*>(p) = make_uint4(w[0], w[1], w[2], w[3]);
     *reinterpret_cast<uint4*>(p + A2_PLANE) = make_uint4(w[4], w[5], w[6], w[7]);
-    if (dbg) {
-      uint4* d = reinterpret_cast<uint4*>(dbg + (py * P1 + px) * 16);
-      d[0] = make_uint4(w[0], w[1], w[2], w[3]);
-      d[1] = make_uint4(w[4], w[5], w[6], w[7]);
-    }
   }
 }
 
-// conv2 tile u: lane (qd, l) = pooled pixel (4u + 2qd + (l >> 4), l & 15); returns the FC partial sum.
-__device__ __forceinline__ float conv2_epilogue(uint32_t tmem, int u, const float* b2, const uint16_t* wfc, float* dbg) {
+// conv2 tile u: lane (qd, l) = GEMM row r = 128u + 32qd + l = pooled pixel (r / 14, r % 14); returns the FC partial
+// sum over its 32 channels (0 for rows outside the 12 x 12 floor-pooled output).
+__device__ __forceinline__ float conv2_epilogue(uint32_t tmem, int u, const float* b2, const float* wfc) {
   const int qd = (threadIdx.x >> 5) & 3, l = threadIdx.x & 31;
-  const int py = 4 * u + 2 * qd + (l >> 4), px = l & 15;
-  const bool own = px < P2 && (u == 0 ? py < 8 : py >= 8);
+  const int r = 128 * u + 32 * qd + l;
+  const int py = r / A2_COLS, px = r - py * A2_COLS;
+  const bool own = py < P2 && px < P2;
+  const float4* wq = reinterpret_cast<const float4*>(wfc) + py * P2 + min(px, P2 - 1);  // in smem for every lane
   float acc = 0.f;
 #pragma unroll
   for (int h = 0; h < 2; ++h) {
     float v[16];
-    pooled16(tmem + ((uint32_t)(32 * qd) << 16), u * 128 + 16 * h, 32, v);
-    if (own) {
+    pool_bias_relu16(tmem + ((uint32_t)(32 * qd) << 16), (int)kC2Col + 128 * u + 16 * h, 32, b2 + 16 * h, v);
 #pragma unroll
-      for (int i = 0; i < 16; ++i) {
-        const int c = 16 * h + i;
-        const float r = fmaxf(v[i] + b2[c], 0.f);
-        acc = fmaf(r, __uint_as_float((uint32_t)wfc[c * (P2 * P2) + py * P2 + px] << 16), acc);
-        if (dbg) dbg[c * (P2 * P2) + py * P2 + px] = r;
-      }
+    for (int q = 0; q < 4; ++q) {
+      const float4 w = wq[(4 * h + q) * (P2 * P2)];
+      acc = fmaf(v[4 * q], w.x, acc);
+      acc = fmaf(v[4 * q + 1], w.y, acc);
+      acc = fmaf(v[4 * q + 2], w.z, acc);
+      acc = fmaf(v[4 * q + 3], w.w, acc);
     }
   }
-  return acc;
+  return own ? acc : 0.f;
 }
 
-__global__ void __launch_bounds__(kThreads, kSnmCtasPerSm) snm_kernel(SnmArgs a) {
+__global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
   extern __shared__ __align__(1024) uint8_t sm[];
-  uint8_t* A1 = sm + OFF_A1;
-  uint8_t* A2 = sm + OFF_A2;
+  const int m = a.counts[0];
+  const int j0 = (int)((int64_t)blockIdx.x * m / gridDim.x), j1 = (int)((int64_t)(blockIdx.x + 1) * m / gridDim.x);
+  const int S = j1 - j0;  // frames of this CTA (every role walks the same sequence)
+  if (S <= 0) return;
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0);  // warp-uniform (uniform registers)
   uint8_t* WB = sm + OFF_WB;
-  uint8_t* stage = sm + OFF_IN;
+  int2* info = reinterpret_cast<int2*>(sm + OFF_INFO);
   float* red = reinterpret_cast<float*>(sm + OFF_RED);
   uint32_t* s_tmem = reinterpret_cast<uint32_t*>(sm + OFF_TMEM);
-  __shared__ int s_chunk;
-  const int tid = threadIdx.x, lane = tid & 31;
-  const int warp = __shfl_sync(0xffffffffu, tid >> 5, 0), grp = warp >> 2;  // warp-uniform (uniform registers)
-  const uint32_t bar0 = smem_addr(sm + OFF_BAR);  // bar0 + 8*i: i < 7 conv1 tiles, 7..8 conv2 tiles, 9..10 input
-  const int n_chunks = a.counts[1];
-  if (n_chunks == 0) return;  // no survivors in this batch
+  const uint32_t bars = smem_addr(sm + OFF_BAR);
+  auto bar = [&](int i) { return bars + 8u * (uint32_t)i; };
 
-  for (int i = tid; i < (A1_BYTES + A2_BYTES) / 16; i += kThreads) reinterpret_cast<uint4*>(sm)[i] = make_uint4(0, 0, 0, 0);
-  uint16_t* lut = reinterpret_cast<uint16_t*>(sm + OFF_LUT);
-  lut[tid] = (uint16_t)u8_to_bf16((uint32_t)tid);  // kThreads == 256 entries
+  // zero both operand buffers of each GEMM (padding borders, the unused 4th channel slot, the junk-row tails)
+  for (int i = tid; i < (2 * A1_BYTES + 2 * A2_BYTES) / 16; i += kThreads)
+    reinterpret_cast<uint4*>(sm + OFF_A1)[i] = make_uint4(0, 0, 0, 0);
   if (tid == 0) {
-    for (int i = 0; i < 11; ++i) mbar_init(bar0 + 8 * i, 1);
+    for (int i = 0; i < NIN; ++i) {
+      mbar_init(bar(B_IN_FULL + i), 1);
+      mbar_init(bar(B_IN_EMPTY + i), 4);
+    }
+    mbar_init(bar(B_W_FULL), 1);
+    mbar_init(bar(B_W_EMPTY), 1);
+    for (int i = 0; i < NI; ++i) mbar_init(bar(B_INFO_EMPTY + i), 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(bar(B_A1_FULL + i), 4);
+      mbar_init(bar(B_A1_EMPTY + i), 1);
+      mbar_init(bar(B_A2_FULL + i), 4);
+      mbar_init(bar(B_A2_EMPTY + i), 1);
+      mbar_init(bar(B_C2_FULL + i), 2);
+      mbar_init(bar(B_C2_EMPTY + i), 4);
+    }
+    for (int i = 0; i < 4; ++i) {
+      mbar_init(bar(B_C1_FULL + i), 2);
+      mbar_init(bar(B_C1_EMPTY + i), 4);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_addr(s_tmem)),
-                 "r"(kTmemCols));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-  }
+  if (warp == 1) tmem_alloc(smem_addr(s_tmem), kTmemCols);
+  fence_proxy_async();  // the zeroed operand buffers are read by the tensor cores
   fence_before();
   __syncthreads();
   fence_after();
   const uint32_t tmem = *s_tmem;
-  const uint32_t a1 = smem_addr(A1), a2 = smem_addr(A2);
-  const uint32_t w1 = smem_addr(WB + OFF_W1), w2 = smem_addr(WB + OFF_W2);
-  const float* b1 = reinterpret_cast<const float*>(WB + OFF_B1);
-  const float* b2 = reinterpret_cast<const float*>(WB + OFF_B2);
-  const uint16_t* wfc = reinterpret_cast<const uint16_t*>(WB + OFF_WFC);
-  uint32_t ph = 0;           // parity of the per-frame mbarriers (one phase per frame)
-  uint32_t in_ph = 0;        // bit i: parity of input staging buffer i
-  const uint8_t* loaded = nullptr;  // weight image currently in shared memory
 
-  for (;;) {
-    if (tid == 0) s_chunk = atomicAdd(a.counts + 2, 1);
-    __syncthreads();
-    const int k = s_chunk;
-    if (k >= n_chunks) break;
-    const int start = a.chunks[k], end = a.chunks[k + 1];
-    const FrameDesc fd0 = a.frames[a.work[start]];
-    if (fd0.snm != loaded) {  // dynamic batch: one weight load per batch of this stream (L219)
-      const uint4* src = reinterpret_cast<const uint4*>(fd0.snm);
-      uint4* dst = reinterpret_cast<uint4*>(WB);
-      for (int i = tid; i < BLOB_BYTES / 16; i += kThreads) dst[i] = __ldg(src + i);
-      loaded = fd0.snm;
+  if (warp == 0) {
+    // ---------------- producer: per-frame info, D50 staging, the stream's weight image per segment
+    if (lane == 0) {
+      const uint32_t in0 = smem_addr(sm + OFF_IN);
+      int k = 0, nch = 0;  // chunk containing frame j (pop_start counting, online mode)
+      if (a.pop_start) {
+        nch = a.counts[1];
+        int lo = 0, hi = nch - 1;  // last k with chunks[k] <= j0
+        while (lo < hi) {
+          const int mid = (lo + hi + 1) >> 1;
+          if (__ldg(a.chunks + mid) <= j0) lo = mid;
+          else hi = mid - 1;
+        }
+        k = lo;
+      }
+      int f = __ldg(a.work + j0);
+      const uint8_t* snm = a.frames[f].snm;
+      const uint8_t* src = d50_of(a, f);
+      const uint8_t* prev = nullptr;
+      int g = -1;
+      for (int s = 0; s < S; ++s) {
+        const int j = j0 + s;
+        int fn = -1;
+        const uint8_t *snm_n = nullptr, *src_n = nullptr;
+        if (s + 1 < S) {  // one frame of lookahead: the next frame's stream decides this frame's segment end
+          fn = __ldg(a.work + j + 1);
+          snm_n = a.frames[fn].snm;
+          src_n = d50_of(a, fn);
+        }
+        const bool first = snm != prev, last = s + 1 == S || snm_n != snm;
+        int flags = (first ? F_SEG_FIRST : 0) | (last ? F_SEG_LAST : 0);
+        if (a.pop_start) {
+          while (k + 1 < nch && __ldg(a.chunks + k + 1) <= j) ++k;
+          if (__ldg(a.chunks + k) == j && a.pop_start[k]) flags |= F_POP_OPEN;
+        }
+        if (first) ++g;
+        if (s >= NI) mbar_wait_sleep(bar(B_INFO_EMPTY + s % NI), (uint32_t)((s / NI - 1) & 1));
+        info[s % NI] = make_int2(f, flags);
+        if (s >= NIN) mbar_wait_sleep(bar(B_IN_EMPTY + s % NIN), (uint32_t)((s / NIN - 1) & 1));
+        mbar_expect_tx(bar(B_IN_FULL + s % NIN), D50_BYTES);
+        bulk_g2s(in0 + (uint32_t)((s % NIN) * D50_BYTES), src, D50_BYTES, bar(B_IN_FULL + s % NIN));
+        if (first) {  // dynamic batch: one weight load per run of one stream's frames (L219)
+          if (g >= 1) mbar_wait_sleep(bar(B_W_EMPTY), (uint32_t)((g - 1) & 1));
+          mbar_expect_tx(bar(B_W_FULL), BLOB_BYTES);
+          constexpr int kPiece = 16384;
+          for (int o = 0; o < BLOB_BYTES; o += kPiece)
+            bulk_g2s(smem_addr(WB) + (uint32_t)o, snm + o, (uint32_t)min(kPiece, BLOB_BYTES - o), bar(B_W_FULL));
+        }
+        prev = snm;
+        f = fn;
+        snm = snm_n;
+        src = src_n;
+      }
     }
-    const float fc_bias = __ldg(reinterpret_cast<const float*>(fd0.snm + OFF_BFC));
-    uint32_t cnt_pass = 0, cnt_c0 = 0, cnt_c1 = 0, cnt_c2 = 0;
-    if (tid == 0) {  // stage the unit's first two D50 images
-      mbar_expect_tx(bar0 + 8 * 9, D50_BYTES);
-      bulk_g2s(smem_addr(stage), d50_of(a, a.work[start]), D50_BYTES, bar0 + 8 * 9);
-      if (start + 1 < end) {
-        mbar_expect_tx(bar0 + 8 * 10, D50_BYTES);
-        bulk_g2s(smem_addr(stage + D50_BYTES), d50_of(a, a.work[start + 1]), D50_BYTES, bar0 + 8 * 10);
-      }
-    }
-    mbar_wait(bar0 + 8 * 9, in_ph & 1u);
-    in_ph ^= 1u;
-    convert_input(stage, A1, lut);
-    fence_proxy_async();
-    const bool issuer = (warp & 3) == 0;  // warp 0 issues group 0's tiles, warp 4 group 1's (one elected lane)
-    for (int j = start; j < end; ++j) {
-      const int f = a.work[j];
-      const int buf = (j - start) & 1;
-      fence_before();
-      __syncthreads();  // frame j's conv1 operand (and the unit's weights) are in shared memory
-
-      // ---- conv1: 7 tiles in two waves of TMEM columns (tile t -> columns (t % 4) * 64); each warp group issues
-      // and drains its own tiles (0, 2 | 4, 6 and 1, 3 | 5), one commit per tile. Wave B reuses wave A's columns of
-      // the same group once the whole group has read them (named barrier 1 + grp over its 128 threads).
-      uint16_t* dbg1 = a.dbg_p1 ? a.dbg_p1 + (int64_t)j * (P1 * P1 * 16) : nullptr;
-#pragma unroll
-      for (int wave = 0; wave < 2; ++wave) {
-        if (issuer) {
-          fence_after();
-          for (int t = grp + 4 * wave; t < min(kTiles1, 4 * wave + 4); t += 2) {
-            issue_conv1_tile(tmem, (uint32_t)((t & 3) * 64), t, a1, w1);
-            mma_commit(bar0 + 8 * t);
-          }
-        }
-        __syncwarp();
-        for (int t = grp + 4 * wave; t < min(kTiles1, 4 * wave + 4); t += 2) {
-          mbar_wait(bar0 + 8 * t, ph);
-          fence_after();
-          conv1_epilogue(tmem, (uint32_t)((t & 3) * 64), t, A2, b1, dbg1);
-        }
-        if (wave == 0) {  // the group's wave-A columns are drained before its wave-B MMAs overwrite them
-          fence_before();
-          if (grp == 0) asm volatile("bar.sync 1, 128;" ::: "memory");
-          else asm volatile("bar.sync 2, 128;" ::: "memory");
-        }
-      }
-      fence_proxy_async();  // conv1's epilogue wrote conv2's operand through the generic proxy
-      fence_before();
-      __syncthreads();  // every conv1 tile has landed: conv1's operand is free again
-
-      // ---- conv2: one tile per warp group; while its MMAs run, stage frame j+1's conv1 operand
-      if (issuer) {
-        fence_after();
-        issue_conv2_tile(tmem, grp, a2, w2);
-        mma_commit(bar0 + 8 * (7 + grp));
-      }
-      __syncwarp();
-      if (j + 1 < end) {
-        const int nb = buf ^ 1;
-        mbar_wait(bar0 + 8 * (9 + nb), (in_ph >> nb) & 1u);
-        in_ph ^= 1u << nb;
-        convert_input(stage + nb * D50_BYTES, A1, lut);
-        fence_proxy_async();
-      }
-      if (tid == 0 && j + 2 < end) {  // frame j's staging buffer is consumed: prefetch frame j+2 into it
-        mbar_expect_tx(bar0 + 8 * (9 + buf), D50_BYTES);
-        bulk_g2s(smem_addr(stage + buf * D50_BYTES), d50_of(a, a.work[j + 2]), D50_BYTES, bar0 + 8 * (9 + buf));
-      }
-      mbar_wait(bar0 + 8 * (7 + grp), ph);
+  } else if (warp == 1) {
+    // ---------------- MMA issue: frame s's conv1 tiles interleaved with frame s-1's conv2 tiles
+    const uint32_t a1b = smem_addr(sm + OFF_A1), a2b = smem_addr(sm + OFF_A2);
+    const uint32_t w1 = smem_addr(WB + OFF_W1), w2 = smem_addr(WB + OFF_W2);
+    int g = -1;
+    auto c1 = [&](int s, int t) {
+      const int T = kTiles1 * s + t, slot = T & 3;
+      if (T >= 4) mbar_wait(bar(B_C1_EMPTY + slot), (uint32_t)(((T >> 2) - 1) & 1));
       fence_after();
-      float* dbg2 = a.dbg_p2 ? a.dbg_p2 + (int64_t)j * NF : nullptr;
-      float acc = conv2_epilogue(tmem, grp, b2, wfc, dbg2);
-      ph ^= 1u;
+      issue_conv1_tile(tmem + (uint32_t)(64 * slot), a1b + (uint32_t)((s & 1) * A1_BYTES), t, w1);
+      mma_commit(bar(B_C1_FULL + slot));
+      mbar_arrive_elect(bar(B_C1_FULL + slot));  // release: the epilogue warps may read this frame's info
+    };
+    auto c2 = [&](int s, int u) {
+      if (s >= 1) mbar_wait(bar(B_C2_EMPTY + u), (uint32_t)((s - 1) & 1));
+      fence_after();
+      issue_conv2_tile(tmem + kC2Col + (uint32_t)(128 * u), a2b + (uint32_t)((s & 1) * A2_BYTES), u, w2);
+      mma_commit(bar(B_C2_FULL + u));
+      mbar_arrive_elect(bar(B_C2_FULL + u));
+    };
+    auto wait_a2 = [&](int s) {
+      mbar_wait(bar(B_A2_FULL + (s & 1)), (uint32_t)((s >> 1) & 1));
+      fence_after();
+    };
+    for (int s = 0; s <= S; ++s) {
+      const bool have = s < S;
+      bool first = false;
+      if (have) {
+        mbar_wait(bar(B_A1_FULL + (s & 1)), (uint32_t)((s >> 1) & 1));
+        first = (info[s % NI].y & F_SEG_FIRST) != 0;
+      }
+      // the weight image of a new stream replaces the old one only after frame s-1's conv2 is drained, so that
+      // conv2 goes first at a stream change (and after the last frame)
+      const bool c2_first = s >= 1 && (!have || first);
+      if (c2_first) {
+        wait_a2(s - 1);
+        c2(s - 1, 0);
+        c2(s - 1, 1);
+        mma_commit(bar(B_A2_EMPTY + ((s - 1) & 1)));
+      }
+      if (!have) break;
+      if (first) {
+        ++g;
+        mbar_wait(bar(B_W_FULL), (uint32_t)(g & 1));
+      }
+      c1(s, 0);
+      c1(s, 1);
+      c1(s, 2);
+      c1(s, 3);
+      if (s >= 1 && !c2_first) {
+        wait_a2(s - 1);
+        c2(s - 1, 0);
+      }
+      c1(s, 4);
+      c1(s, 5);
+      mma_commit(bar(B_A1_EMPTY + (s & 1)));
+      if (s >= 1 && !c2_first) {
+        c2(s - 1, 1);
+        mma_commit(bar(B_A2_EMPTY + ((s - 1) & 1)));
+      }
+    }
+  } else if (warp >= 4 && warp < 8) {
+    // ---------------- D50 -> conv1 operand
+    const int t = tid - 128;
+    for (int s = 0; s < S; ++s) {
+      mbar_wait(bar(B_IN_FULL + s % NIN), (uint32_t)((s / NIN) & 1));
+      if (s >= 2) mbar_wait(bar(B_A1_EMPTY + (s & 1)), (uint32_t)(((s >> 1) - 1) & 1));
+      convert_input(sm + OFF_IN + (s % NIN) * D50_BYTES, sm + OFF_A1 + (s & 1) * A1_BYTES, t);
+      fence_proxy_async();
+      __syncwarp();
+      mbar_arrive_elect(bar(B_A1_FULL + (s & 1)));
+      mbar_arrive_elect(bar(B_IN_EMPTY + s % NIN));
+    }
+  } else if (warp >= 8 && warp < 12) {
+    // ---------------- conv1 epilogue -> conv2 operand
+    for (int s = 0; s < S; ++s) {
+      uint8_t* A2 = sm + OFF_A2 + (s & 1) * A2_BYTES;
+      if (s >= 2) mbar_wait(bar(B_A2_EMPTY + (s & 1)), (uint32_t)(((s >> 1) - 1) & 1));
+      float b1[16];
+      for (int t = 0; t < kTiles1; ++t) {
+        const int T = kTiles1 * s + t, slot = T & 3;
+        mbar_wait(bar(B_C1_FULL + slot), (uint32_t)((T >> 2) & 1));
+        fence_after();
+        if (t == 0) {
+#pragma unroll
+          for (int i = 0; i < 16; ++i) b1[i] = reinterpret_cast<const float*>(WB + OFF_B1)[i];
+        }
+        conv1_epilogue(tmem, (uint32_t)(64 * slot), t, A2, b1);
+        fence_before();
+        __syncwarp();
+        mbar_arrive_elect(bar(B_C1_EMPTY + slot));
+      }
+      fence_proxy_async();  // conv2's operand was written through the generic proxy
+      __syncwarp();
+      mbar_arrive_elect(bar(B_A2_FULL + (s & 1)));
+    }
+  } else if (warp >= 12) {
+    // ---------------- conv2 epilogue, FC, decision
+    const float* b2 = reinterpret_cast<const float*>(WB + OFF_B2);
+    const float* wfc = reinterpret_cast<const float*>(WB + OFF_WFC);
+    const int qd = warp & 3;
+    uint32_t cnt_pass = 0, cnt_c0 = 0, cnt_c1 = 0, cnt_c2 = 0, cnt_pop = 0;
+    for (int s = 0; s < S; ++s) {
+      float acc = 0.f;
+      for (int u = 0; u < 2; ++u) {
+        mbar_wait(bar(B_C2_FULL + u), (uint32_t)(s & 1));
+        fence_after();
+        acc += conv2_epilogue(tmem, u, b2, wfc);
+        fence_before();
+        __syncwarp();
+        mbar_arrive_elect(bar(B_C2_EMPTY + u));
+      }
 #pragma unroll
       for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
-      if (lane == 0) red[warp] = acc;
-      fence_before();
-      __syncthreads();
-      if (tid == 0) {
-        float logit = fc_bias;
-#pragma unroll
-        for (int w = 0; w < kThreads / 32; ++w) logit += red[w];
-        const FrameDesc fd = a.frames[f];
+      if (elect_one()) red[(s & 1) * 4 + qd] = acc;
+      asm volatile("bar.sync 1, 128;" ::: "memory");
+      if (warp == 12 && elect_one()) {
+        const int2 in = info[s % NI];
+        const int f = in.x;
+        const float* r = red + (s & 1) * 4;
+        const float logit = *reinterpret_cast<const float*>(WB + OFF_BFC) + ((r[0] + r[1]) + (r[2] + r[3]));
+        const FrameDesc& fd = a.frames[f];
         const uint8_t p = logit >= fd.L_t ? 1 : 0;
         const uint8_t cls = logit < fd.L_low ? 0 : (logit > fd.L_high ? 2 : 1);
         a.logit[f] = logit;
@@ -339,24 +456,29 @@ __global__ void __launch_bounds__(kThreads, kSnmCtasPerSm) snm_kernel(SnmArgs a)
         cnt_c0 += cls == 0;
         cnt_c1 += cls == 1;
         cnt_c2 += cls == 2;
+        cnt_pop += (in.y & F_POP_OPEN) ? 1 : 0;
+        if (in.y & F_SEG_LAST) {
+          if (a.stats) {
+            unsigned long long* st = a.stats + (int64_t)fd.slot * NSTAT;
+            atomicAdd(st + 2, (unsigned long long)cnt_pass);
+            atomicAdd(st + 4, (unsigned long long)cnt_c0);
+            atomicAdd(st + 5, (unsigned long long)cnt_c1);
+            atomicAdd(st + 6, (unsigned long long)cnt_c2);
+            if (cnt_pop) atomicAdd(st + 7, (unsigned long long)cnt_pop);
+          }
+          cnt_pass = cnt_c0 = cnt_c1 = cnt_c2 = cnt_pop = 0;
+          mbar_arrive(bar(B_W_EMPTY));  // this stream's weights are no longer read
+        }
+        mbar_arrive(bar(B_INFO_EMPTY + s % NI));
       }
     }
-    if (tid == 0 && a.stats) {
-      unsigned long long* st = a.stats + (int64_t)fd0.slot * NSTAT;
-      atomicAdd(st + 2, (unsigned long long)cnt_pass);
-      atomicAdd(st + 4, (unsigned long long)cnt_c0);
-      atomicAdd(st + 5, (unsigned long long)cnt_c1);
-      atomicAdd(st + 6, (unsigned long long)cnt_c2);
-      if (a.pop_start && a.pop_start[k]) atomicAdd(st + 7, 1ull);
-    }
-    __syncthreads();
   }
 
   fence_before();
   __syncthreads();
-  if (warp == 0) {
+  if (warp == 1) {
     fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
+    tmem_dealloc(tmem, kTmemCols);
   }
 }
 

@@ -48,7 +48,7 @@ def test_export_import_continues_identically(env, where, distance):
     r1 = ctx.filter_batch([(cam.st, d[i], i) for i in range(30)])
     stats_before = ctx.stats()[cam.st.slot].copy()
     n = cam.st.image_bytes()
-    assert n == 256 + 30000 + 26832 + 192  # header + R + packed SNM image (bf16 FC weights) + stats row (24 x u64)
+    assert n == 256 + 30000 + 63696 + 192  # header + R + packed SNM image (shared-memory image of K4) + stats row (24 x u64)
     img = cam.st.export() if where == "host" else cam.st.export(torch.empty(n, dtype=torch.uint8, device=dev))
     cam.st.close()
     st2 = ctx.import_stream(img)
