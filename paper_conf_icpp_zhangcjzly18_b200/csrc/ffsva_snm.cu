@@ -29,10 +29,10 @@
 //     multiplies the pooled features by the FC weights (bf16 values) in fp32 and reduces to one logit per frame.
 // One warp-specialised persistent CTA per SM (512 threads, all 512 TMEM columns), frames pipelined through
 // mbarrier rings: warp 0 stages each frame's D50 image (bulk copy) and the stream's weight image when the stream
-// changes; warps 4-7 convert D50 to conv1's bf16 operand (two buffers); warp 1 issues the MMAs (conv1 tiles into a
+// changes; warps 2-3 convert D50 to conv1's bf16 operand (two buffers); warp 1 issues the MMAs (conv1 tiles into a
 // ring of four 64-column TMEM slots, conv2 tiles into two 128-column slots, frame j+1's conv1 interleaved with frame
-// j's conv2); warps 8-11 drain conv1 tiles into conv2's operand (two buffers); warps 12-15 drain conv2 tiles, apply
-// the FC and decide. CTA c scores the survivors [c*m/G, (c+1)*m/G) of the stream-major work order, so a stream's
+// j's conv2); warps 4-7 and 8-11 drain the even and the odd conv1 tiles into conv2's operand (two buffers); warps
+// 12-15 drain conv2 tiles, apply the FC and decide. CTA c scores the survivors [c*m/G, (c+1)*m/G) of the stream-major work order, so a stream's
 // weights are loaded once per CTA and per stream (a dynamic batch's frames are consecutive, L219).
 #include <cuda_bf16.h>
 
@@ -45,8 +45,33 @@ namespace {
 using namespace snm;
 using namespace ptx;
 
+#ifndef FFSVA_K4_ABL
+#define FFSVA_K4_ABL 0  // A/B only (wrong results): 1 no conversion, 2 no conv1 epilogue, 4 no conv2 epilogue, 8 no MMAs
+#endif
+#ifndef FFSVA_K4_PROF
+#define FFSVA_K4_PROF 0  // A/B only: per-wait clock totals of CTA 0, printed at exit
+#endif
+#if FFSVA_K4_PROF
+}  // namespace
+}  // namespace ffsva
+#include <cstdio>
+namespace ffsva {
+namespace {
+__shared__ unsigned long long s_prof[16];
+#define KW(id, call)                                                        \
+  do {                                                                      \
+    const long long _t0 = clock64();                                        \
+    call;                                                                   \
+    if ((threadIdx.x & 31) == 0) atomicAdd(&s_prof[id], (unsigned long long)(clock64() - _t0)); \
+  } while (0)
+#else
+#define KW(id, call) call
+#endif
 constexpr int kThreads = 512;
 constexpr int NIN = 3;   // D50 staging ring
+constexpr int NA1 = 2;   // conv1 operand buffers
+constexpr int NA2 = 3;   // conv2 operand buffers (frames j-2 .. j: conv2 runs two frames behind conv1)
+constexpr int kConvWarps = 6;  // warps 2-7 convert
 constexpr int NI = 16;   // per-frame info ring (frames in flight between the producer and the conv2 epilogue)
 // conv1 operand: 2 row-parity planes x 26 rows x 26 entries (two padded pixels x 4 channel slots, 16 B)
 constexpr int A1_ROW = 26;                                  // entries per plane row
@@ -64,17 +89,17 @@ static_assert(A2_BYTES >= (7 * A2_PLANE / 16 + 255 + A2_COLS + 1 + 1) * 16, "con
 constexpr int D50_BYTES = 7504;                             // staged D50 image (one frame)
 
 constexpr int OFF_WB = 0;                                   // the stream's weight image (snm::BLOB_BYTES)
-constexpr int OFF_A1 = 63744;                               // 2 buffers
-constexpr int OFF_A2 = OFF_A1 + 2 * A1_BYTES;               // 110848, 2 buffers
-constexpr int OFF_IN = OFF_A2 + 2 * A2_BYTES;               // 163872, NIN stages
-constexpr int OFF_INFO = OFF_IN + NIN * D50_BYTES;          // 186384: int2 [NI] (frame, flags)
+constexpr int OFF_A1 = 63744;                               // NA1 buffers
+constexpr int OFF_A2 = OFF_A1 + NA1 * A1_BYTES;             // 110848, NA2 buffers
+constexpr int OFF_IN = OFF_A2 + NA2 * A2_BYTES;             // 190384, NIN stages
+constexpr int OFF_INFO = OFF_IN + NIN * D50_BYTES;          // 212896: int2 [NI] (frame, flags)
 constexpr int OFF_RED = OFF_INFO + NI * 8;                  // float [2][4]
 constexpr int OFF_BAR = OFF_RED + 32;
 // mbarriers (8 B each)
 constexpr int B_IN_FULL = 0, B_IN_EMPTY = B_IN_FULL + NIN, B_W_FULL = B_IN_EMPTY + NIN, B_W_EMPTY = B_W_FULL + 1,
-              B_INFO_EMPTY = B_W_EMPTY + 1, B_A1_FULL = B_INFO_EMPTY + NI, B_A1_EMPTY = B_A1_FULL + 2,
-              B_C1_FULL = B_A1_EMPTY + 2, B_C1_EMPTY = B_C1_FULL + 4, B_A2_FULL = B_C1_EMPTY + 4,
-              B_A2_EMPTY = B_A2_FULL + 2, B_C2_FULL = B_A2_EMPTY + 2, B_C2_EMPTY = B_C2_FULL + 2,
+              B_INFO_EMPTY = B_W_EMPTY + 1, B_A1_FULL = B_INFO_EMPTY + NI, B_A1_EMPTY = B_A1_FULL + NA1,
+              B_C1_FULL = B_A1_EMPTY + NA1, B_C1_EMPTY = B_C1_FULL + 4, B_A2_FULL = B_C1_EMPTY + 4,
+              B_A2_EMPTY = B_A2_FULL + NA2, B_C2_FULL = B_A2_EMPTY + NA2, B_C2_EMPTY = B_C2_FULL + 2,
               N_BARS = B_C2_EMPTY + 2;
 constexpr int OFF_TMEM = OFF_BAR + N_BARS * 8;
 constexpr int SMEM_BYTES = OFF_TMEM + 16;
@@ -141,7 +166,7 @@ __device__ __forceinline__ void issue_conv2_tile(uint32_t d, uint32_t a2, int u,
   }
 }
 
-// ---------------------------------------------------------------- input conversion (warps 4-7)
+// ---------------------------------------------------------------- input conversion (warps 2-3)
 // D50 (50x50x3 u8, row-major) -> (v-128)/128 bf16 (C5, exact) into conv1's row-parity planes. A thread writes one
 // 16-byte entry = padded columns (2e, 2e+1) = image columns (2e-1, 2e) of one row, 4 channel slots each (3 used);
 // its 6 source bytes are funnel-shifted out of two aligned words (lanes ~6 B apart: conflict-free loads, contiguous
@@ -151,7 +176,11 @@ __device__ __forceinline__ uint32_t bf16_hi_of_byte(uint32_t w, uint32_t k) {
 }
 __device__ __forceinline__ void convert_input(const uint8_t* d, uint8_t* A1, int t) {
   constexpr int kEntries = IN * A1_ROW;  // 50 rows x 26 entries
-  for (int q = t; q < kEntries; q += 128) {
+  constexpr int kStride = 32 * kConvWarps;
+#pragma unroll
+  for (int i = 0; i < (kEntries + kStride - 1) / kStride; ++i) {
+    const int q = t + i * kStride;
+    if (q >= kEntries) break;
     const int y = q / A1_ROW, e = q - y * A1_ROW;
     // bytes [o, o + 6) of the image: columns 2e-1 and 2e (column -1 / 50 are the zero border)
     const int o = y * 3 * IN + 6 * e - 3;
@@ -226,6 +255,10 @@ __device__ __forceinline__ float conv2_epilogue(uint32_t tmem, int u, const floa
 
 __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
   extern __shared__ __align__(1024) uint8_t sm[];
+#if FFSVA_K4_PROF
+  const long long t_start = clock64();
+  if (threadIdx.x < 16) s_prof[threadIdx.x] = 0;
+#endif
   const int m = a.counts[0];
   const int j0 = (int)((int64_t)blockIdx.x * m / gridDim.x), j1 = (int)((int64_t)(blockIdx.x + 1) * m / gridDim.x);
   const int S = j1 - j0;  // frames of this CTA (every role walks the same sequence)
@@ -240,21 +273,25 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
   auto bar = [&](int i) { return bars + 8u * (uint32_t)i; };
 
   // zero both operand buffers of each GEMM (padding borders, the unused 4th channel slot, the junk-row tails)
-  for (int i = tid; i < (2 * A1_BYTES + 2 * A2_BYTES) / 16; i += kThreads)
+  for (int i = tid; i < (NA1 * A1_BYTES + NA2 * A2_BYTES) / 16; i += kThreads)
     reinterpret_cast<uint4*>(sm + OFF_A1)[i] = make_uint4(0, 0, 0, 0);
   if (tid == 0) {
     for (int i = 0; i < NIN; ++i) {
       mbar_init(bar(B_IN_FULL + i), 1);
-      mbar_init(bar(B_IN_EMPTY + i), 4);
+      mbar_init(bar(B_IN_EMPTY + i), kConvWarps);
     }
     mbar_init(bar(B_W_FULL), 1);
     mbar_init(bar(B_W_EMPTY), 1);
     for (int i = 0; i < NI; ++i) mbar_init(bar(B_INFO_EMPTY + i), 1);
-    for (int i = 0; i < 2; ++i) {
-      mbar_init(bar(B_A1_FULL + i), 4);
+    for (int i = 0; i < NA1; ++i) {
+      mbar_init(bar(B_A1_FULL + i), kConvWarps);
       mbar_init(bar(B_A1_EMPTY + i), 1);
+    }
+    for (int i = 0; i < NA2; ++i) {
       mbar_init(bar(B_A2_FULL + i), 4);
       mbar_init(bar(B_A2_EMPTY + i), 1);
+    }
+    for (int i = 0; i < 2; ++i) {
       mbar_init(bar(B_C2_FULL + i), 2);
       mbar_init(bar(B_C2_EMPTY + i), 4);
     }
@@ -307,13 +344,13 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
           if (__ldg(a.chunks + k) == j && a.pop_start[k]) flags |= F_POP_OPEN;
         }
         if (first) ++g;
-        if (s >= NI) mbar_wait_sleep(bar(B_INFO_EMPTY + s % NI), (uint32_t)((s / NI - 1) & 1));
+        if (s >= NI) KW(0, mbar_wait_sleep(bar(B_INFO_EMPTY + s % NI), (uint32_t)((s / NI - 1) & 1)));
         info[s % NI] = make_int2(f, flags);
-        if (s >= NIN) mbar_wait_sleep(bar(B_IN_EMPTY + s % NIN), (uint32_t)((s / NIN - 1) & 1));
+        if (s >= NIN) KW(1, mbar_wait_sleep(bar(B_IN_EMPTY + s % NIN), (uint32_t)((s / NIN - 1) & 1)));
         mbar_expect_tx(bar(B_IN_FULL + s % NIN), D50_BYTES);
         bulk_g2s(in0 + (uint32_t)((s % NIN) * D50_BYTES), src, D50_BYTES, bar(B_IN_FULL + s % NIN));
         if (first) {  // dynamic batch: one weight load per run of one stream's frames (L219)
-          if (g >= 1) mbar_wait_sleep(bar(B_W_EMPTY), (uint32_t)((g - 1) & 1));
+          if (g >= 1) KW(2, mbar_wait_sleep(bar(B_W_EMPTY), (uint32_t)((g - 1) & 1)));
           mbar_expect_tx(bar(B_W_FULL), BLOB_BYTES);
           constexpr int kPiece = 16384;
           for (int o = 0; o < BLOB_BYTES; o += kPiece)
@@ -326,100 +363,99 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
       }
     }
   } else if (warp == 1) {
-    // ---------------- MMA issue: frame s's conv1 tiles interleaved with frame s-1's conv2 tiles
+    // ---------------- MMA issue: conv2 lags conv1 by two frames (frame s's conv1 tiles interleaved with frame s-2's
+    // conv2 tiles), so that every MMA's inputs were produced at least one conv2 tile earlier
     const uint32_t a1b = smem_addr(sm + OFF_A1), a2b = smem_addr(sm + OFF_A2);
     const uint32_t w1 = smem_addr(WB + OFF_W1), w2 = smem_addr(WB + OFF_W2);
     int g = -1;
     auto c1 = [&](int s, int t) {
       const int T = kTiles1 * s + t, slot = T & 3;
-      if (T >= 4) mbar_wait(bar(B_C1_EMPTY + slot), (uint32_t)(((T >> 2) - 1) & 1));
+      if (T >= 4) KW(3, mbar_wait(bar(B_C1_EMPTY + slot), (uint32_t)(((T >> 2) - 1) & 1)));
       fence_after();
-      issue_conv1_tile(tmem + (uint32_t)(64 * slot), a1b + (uint32_t)((s & 1) * A1_BYTES), t, w1);
+      if (!(FFSVA_K4_ABL & 8))
+        issue_conv1_tile(tmem + (uint32_t)(64 * slot), a1b + (uint32_t)((s % NA1) * A1_BYTES), t, w1);
       mma_commit(bar(B_C1_FULL + slot));
       mbar_arrive_elect(bar(B_C1_FULL + slot));  // release: the epilogue warps may read this frame's info
     };
     auto c2 = [&](int s, int u) {
-      if (s >= 1) mbar_wait(bar(B_C2_EMPTY + u), (uint32_t)((s - 1) & 1));
+      if (u == 0) {
+        KW(4, mbar_wait(bar(B_A2_FULL + s % NA2), (uint32_t)((s / NA2) & 1)));
+        fence_after();
+      }
+      if (s >= 1) KW(5, mbar_wait(bar(B_C2_EMPTY + u), (uint32_t)((s - 1) & 1)));
       fence_after();
-      issue_conv2_tile(tmem + kC2Col + (uint32_t)(128 * u), a2b + (uint32_t)((s & 1) * A2_BYTES), u, w2);
+      if (!(FFSVA_K4_ABL & 8))
+        issue_conv2_tile(tmem + kC2Col + (uint32_t)(128 * u), a2b + (uint32_t)((s % NA2) * A2_BYTES), u, w2);
       mma_commit(bar(B_C2_FULL + u));
       mbar_arrive_elect(bar(B_C2_FULL + u));
+      if (u == 1) mma_commit(bar(B_A2_EMPTY + s % NA2));
     };
-    auto wait_a2 = [&](int s) {
-      mbar_wait(bar(B_A2_FULL + (s & 1)), (uint32_t)((s >> 1) & 1));
-      fence_after();
-    };
-    for (int s = 0; s <= S; ++s) {
+    int nc2 = 0;  // next frame whose conv2 is not issued yet
+    for (int s = 0;; ++s) {
       const bool have = s < S;
       bool first = false;
       if (have) {
-        mbar_wait(bar(B_A1_FULL + (s & 1)), (uint32_t)((s >> 1) & 1));
+        KW(6, mbar_wait(bar(B_A1_FULL + s % NA1), (uint32_t)((s / NA1) & 1)));
         first = (info[s % NI].y & F_SEG_FIRST) != 0;
       }
-      // the weight image of a new stream replaces the old one only after frame s-1's conv2 is drained, so that
-      // conv2 goes first at a stream change (and after the last frame)
-      const bool c2_first = s >= 1 && (!have || first);
-      if (c2_first) {
-        wait_a2(s - 1);
-        c2(s - 1, 0);
-        c2(s - 1, 1);
-        mma_commit(bar(B_A2_EMPTY + ((s - 1) & 1)));
+      // a new stream's weight image replaces the old one only after every earlier frame's conv2 has been issued
+      // (and drained by the conv2 epilogue, which releases the image): drain the lag at a stream change and at the end
+      if (!have || (first && s > 0)) {
+        for (; nc2 < s; ++nc2) {
+          c2(nc2, 0);
+          c2(nc2, 1);
+        }
+        if (!have) break;
       }
-      if (!have) break;
       if (first) {
         ++g;
-        mbar_wait(bar(B_W_FULL), (uint32_t)(g & 1));
+        KW(7, mbar_wait(bar(B_W_FULL), (uint32_t)(g & 1)));
       }
+      const bool lag = nc2 <= s - 2;
       c1(s, 0);
       c1(s, 1);
       c1(s, 2);
       c1(s, 3);
-      if (s >= 1 && !c2_first) {
-        wait_a2(s - 1);
-        c2(s - 1, 0);
-      }
+      if (lag) c2(nc2, 0);
       c1(s, 4);
       c1(s, 5);
-      mma_commit(bar(B_A1_EMPTY + (s & 1)));
-      if (s >= 1 && !c2_first) {
-        c2(s - 1, 1);
-        mma_commit(bar(B_A2_EMPTY + ((s - 1) & 1)));
-      }
+      mma_commit(bar(B_A1_EMPTY + s % NA1));
+      if (lag) c2(nc2++, 1);
     }
-  } else if (warp >= 4 && warp < 8) {
+  } else if (warp >= 2 && warp < 2 + kConvWarps) {
     // ---------------- D50 -> conv1 operand
-    const int t = tid - 128;
+    const int t = tid - 64;
     for (int s = 0; s < S; ++s) {
-      mbar_wait(bar(B_IN_FULL + s % NIN), (uint32_t)((s / NIN) & 1));
-      if (s >= 2) mbar_wait(bar(B_A1_EMPTY + (s & 1)), (uint32_t)(((s >> 1) - 1) & 1));
-      convert_input(sm + OFF_IN + (s % NIN) * D50_BYTES, sm + OFF_A1 + (s & 1) * A1_BYTES, t);
+      KW(8, mbar_wait(bar(B_IN_FULL + s % NIN), (uint32_t)((s / NIN) & 1)));
+      if (s >= NA1) KW(9, mbar_wait(bar(B_A1_EMPTY + s % NA1), (uint32_t)((s / NA1 - 1) & 1)));
+      if (!(FFSVA_K4_ABL & 1)) convert_input(sm + OFF_IN + (s % NIN) * D50_BYTES, sm + OFF_A1 + (s % NA1) * A1_BYTES, t);
       fence_proxy_async();
       __syncwarp();
-      mbar_arrive_elect(bar(B_A1_FULL + (s & 1)));
+      mbar_arrive_elect(bar(B_A1_FULL + s % NA1));
       mbar_arrive_elect(bar(B_IN_EMPTY + s % NIN));
     }
   } else if (warp >= 8 && warp < 12) {
     // ---------------- conv1 epilogue -> conv2 operand
     for (int s = 0; s < S; ++s) {
-      uint8_t* A2 = sm + OFF_A2 + (s & 1) * A2_BYTES;
-      if (s >= 2) mbar_wait(bar(B_A2_EMPTY + (s & 1)), (uint32_t)(((s >> 1) - 1) & 1));
+      uint8_t* A2 = sm + OFF_A2 + (s % NA2) * A2_BYTES;
+      if (s >= NA2) KW(10, mbar_wait(bar(B_A2_EMPTY + s % NA2), (uint32_t)((s / NA2 - 1) & 1)));
       float b1[16];
       for (int t = 0; t < kTiles1; ++t) {
         const int T = kTiles1 * s + t, slot = T & 3;
-        mbar_wait(bar(B_C1_FULL + slot), (uint32_t)((T >> 2) & 1));
+        KW(11, mbar_wait(bar(B_C1_FULL + slot), (uint32_t)((T >> 2) & 1)));
         fence_after();
         if (t == 0) {
 #pragma unroll
           for (int i = 0; i < 16; ++i) b1[i] = reinterpret_cast<const float*>(WB + OFF_B1)[i];
         }
-        conv1_epilogue(tmem, (uint32_t)(64 * slot), t, A2, b1);
+        if (!(FFSVA_K4_ABL & 2)) conv1_epilogue(tmem, (uint32_t)(64 * slot), t, A2, b1);
         fence_before();
         __syncwarp();
         mbar_arrive_elect(bar(B_C1_EMPTY + slot));
       }
       fence_proxy_async();  // conv2's operand was written through the generic proxy
       __syncwarp();
-      mbar_arrive_elect(bar(B_A2_FULL + (s & 1)));
+      mbar_arrive_elect(bar(B_A2_FULL + s % NA2));
     }
   } else if (warp >= 12) {
     // ---------------- conv2 epilogue, FC, decision
@@ -430,9 +466,9 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
     for (int s = 0; s < S; ++s) {
       float acc = 0.f;
       for (int u = 0; u < 2; ++u) {
-        mbar_wait(bar(B_C2_FULL + u), (uint32_t)(s & 1));
+        KW(12, mbar_wait(bar(B_C2_FULL + u), (uint32_t)(s & 1)));
         fence_after();
-        acc += conv2_epilogue(tmem, u, b2, wfc);
+        if (!(FFSVA_K4_ABL & 4)) acc += conv2_epilogue(tmem, u, b2, wfc);
         fence_before();
         __syncwarp();
         mbar_arrive_elect(bar(B_C2_EMPTY + u));
@@ -440,7 +476,7 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
 #pragma unroll
       for (int off = 16; off > 0; off >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, off);
       if (elect_one()) red[(s & 1) * 4 + qd] = acc;
-      asm volatile("bar.sync 1, 128;" ::: "memory");
+      KW(13, asm volatile("bar.sync 1, 128;" ::: "memory"));
       if (warp == 12 && elect_one()) {
         const int2 in = info[s % NI];
         const int f = in.x;
@@ -476,6 +512,13 @@ __global__ void __launch_bounds__(kThreads, 1) snm_kernel(SnmArgs a) {
 
   fence_before();
   __syncthreads();
+#if FFSVA_K4_PROF
+  if (blockIdx.x == 0 && tid == 0) {
+    printf("K4PROF S=%d total=%lld", S, clock64() - t_start);
+    for (int i = 0; i < 14; ++i) printf(" w%d=%llu", i, s_prof[i]);
+    printf("\n");
+  }
+#endif
   if (warp == 1) {
     fence_after();
     tmem_dealloc(tmem, kTmemCols);
