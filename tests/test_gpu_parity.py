@@ -184,6 +184,46 @@ def test_snm_parity_interleaved_streams(env):
         c.st.close()
 
 
+@pytest.mark.parametrize("counts", [
+    [1, 2, 3, 5, 8, 13, 21, 34, 1, 40, 2, 7],                     # m = 137 < SMs: at most one survivor per CTA
+    [148],                                                        # one stream, exactly one survivor per SM
+    [1, 30, 2, 61, 3, 90, 1, 1, 120, 45, 7, 29, 1, 16, 33, 5, 9, 11, 70, 6],  # m = 541: several frames and streams
+])                                                                #   per CTA, runs of 1..120 frames
+def test_snm_pipeline_stream_runs(env, counts):
+    """K4's per-CTA survivor ranges cut the stream-major work order anywhere: runs of one stream's frames of every
+    length (one weight image per run, the pipeline drained at each stream change), fewer survivors than CTAs, exactly
+    one per CTA, several runs per CTA. Every survivor's logit vs the oracle's bf16-emulation mode (same operand
+    roundings) and the fp64 oracle, decisions, and the per-stream SNM counters (a8) vs the oracle."""
+    ff, ctx, dev = env
+    cams = [Cam(ctx, synth.Video(seed=61 + s, width=640, height=360, period=2, on_len=2), s, dev, snm_batch=7,
+                k_ref=2, bias_std=0.1) for s in range(len(counts))]
+    # frames interleaved across streams in the input (K3 orders them stream-major for K4)
+    order = [(s, t) for t in range(max(counts)) for s in range(len(counts)) if t < counts[s]]
+    pairs = [(cams[s], cams[s].host_frames([t])[0]) for s, t in order]
+    ctx.stats(reset=True)
+    got = _run_full(ctx, dev, pairs)
+    st = ctx.stats()
+    want = oracle_for(pairs)
+    surv = want["survivors"]
+    assert surv.size == len(pairs) and np.all(got["sdd_pass"] == 1)
+    camlist = [c for c, _ in pairs]
+    err, nd = check_snm(got["logit"], got["snm_pass"], got["snm_class"], want["logit"], camlist, surv, SNM_TOL)
+    want16 = oracle_for(pairs, bf16_emul=True)
+    err16 = np.abs(got["logit"][surv] - want16["logit"][surv]).max()
+    assert err16 <= SNM_TOL_BF16, err16
+    for s, c in enumerate(cams):
+        idx = np.array([i for i, (cc, _) in enumerate(pairs) if cc is c])
+        row = st[c.st.slot]
+        assert row[1] == counts[s]
+        assert row[2] == int(got["snm_pass"][idx].sum())
+        for k in range(3):
+            assert row[4 + k] == int((got["snm_class"][idx] == k).sum())
+        assert row[7] == (counts[s] + 6) // 7  # dynamic batches of <= BatchSize 7
+    print(f"m = {surv.size}: max |dlogit| vs fp64 {err:.3e}, vs bf16-emulated {err16:.3e}, {nd} decisions compared")
+    for c in cams:
+        c.st.close()
+
+
 def test_snm_closed_forms_on_gpu(env):
     """P10 on the kernel: zero weights -> logit = b_fc exactly; w2 = 0, wfc = 1 -> b_fc + 144 * sum ReLU(b2)."""
     ff, ctx, dev = env

@@ -38,10 +38,6 @@ for K in "tyolo_l1:2:l1" "tyolo_l2:2:l2" "tyolo_pslab:6:pslab_L3" "tyolo_slab:8:
   echo "ncu full $NAME rc=$?"
 done
 timeout 300 python tools/tyolo_profile.py --frames 256 --iters 10 > gpurun_out/tyolo_profile.log 2>&1
-# racecheck of the whole run does not finish within 25 min on this box (see profiles/r01/sanitize_racecheck.log);
-# RACECHECK=1 adds it
-for tool in memcheck synccheck ${RACECHECK:+racecheck}; do
-  ARGS=""; [ $tool = racecheck ] && ARGS="--no-tyolo"
-  timeout ${SAN_TIMEOUT:-1200} compute-sanitizer --tool $tool --error-exitcode 9 python tools/sanitize_run.py $ARGS > gpurun_out/sanitize_$tool.log 2>&1
-  echo "sanitize $tool rc=$?"; tail -2 gpurun_out/sanitize_$tool.log
-done
+# compute-sanitizer is closed on this GPU pool (runs under it left GPUs needing a reset; see
+# profiles/r02/sanitize_closed.log): the K4 pipeline is covered instead by the stream-run parity test and its own
+# bounds (static_asserts on every shared-memory region and operand tail)
