@@ -10,8 +10,8 @@
 // sum is four __ballot_sync + __popc (lane-mask) steps; warp totals are scanned in shared memory.
 //   pass 1 (input order)      -> survivor_idx[i] = rank of i among survivors, or -1
 //   pass 2 (stream-major perm) -> work[] = survivors grouped by stream, posw[] = exclusive counts
-//   pass 3 (segments)          -> chunk list: each stream's queue split into pops of <= BatchSize frames
-// The SNM kernel consumes chunks through an atomic cursor that this kernel resets.
+//   pass 3 (segments)          -> pop list: each stream's queue split into pops of <= BatchSize frames (chunks[k] =
+//                                 first work position of pop k), counts[0] = m survivors for K4's per-CTA ranges
 #include "ffsva_internal.h"
 
 namespace ffsva {
@@ -159,36 +159,27 @@ __global__ void __launch_bounds__(kThreads) compact_kernel(CompactArgs a) {
   if (threadIdx.x == 0) a.posw[n] = carry;
   __syncthreads();
 
-  // ---------------- pass 3: per-stream pops of <= BatchSize (dynamic batching, L223), each pop split into
-  // SNM work units of U frames so that small batches still spread over the SNM grid (U = m / snm_ctas,
-  // clamped to [1, BatchSize]; a unit never crosses a pop, so a pop's frames share one stream's weights)
-  const int m_all = carry;
+  // ---------------- pass 3: per-stream pops of <= BatchSize (dynamic batching, L223); K4 loads a stream's weights
+  // once per run of its frames in work order, so a pop's frames share one weight image
   int chunk_carry = 0;
   for (int base = 0; base < a.n_seg; base += kThreads) {
     const int s = base + threadIdx.x;
-    int q = 0, B = 1, lo_pos = 0, U = 1;
+    int q = 0, B = 1, lo_pos = 0;
     if (s < a.n_seg) {
       lo_pos = a.posw[a.seg_lo[s]];
       q = a.posw[a.seg_lo[s + 1]] - lo_pos;  // this stream's SNM queue depth
       B = a.seg_batch[s];
-      U = a.snm_ctas > 0 ? m_all / a.snm_ctas : B;
-      U = U < 1 ? 1 : (U > B ? B : U);
       if (a.stats && q > 0) {
         unsigned long long* st = a.stats + (int64_t)a.seg_slot[s] * NSTAT;
         atomicAdd(st + 1, (unsigned long long)q);                    // SDD survivors
         if (a.snm_ctas > 0) atomicAdd(st + 7, (unsigned long long)((q + B - 1) / B));  // dynamic batches
       }
     }
-    const int full = q / B, rest = q - full * B;
-    const int per_full = (B + U - 1) / U;
-    const int nch = full * per_full + (rest + U - 1) / U;
+    const int nch = (q + B - 1) / B;
     int total;
     const int off = chunk_carry + block_exclusive_scan(nch, s_warp, &total);
     int k = off;
-    for (int p = 0; p <= full; ++p) {
-      const int plen = p < full ? B : rest;
-      for (int u = 0; u < plen; u += U) a.chunks[k++] = lo_pos + p * B + u;
-    }
+    for (int p = 0; p < nch; ++p) a.chunks[k++] = lo_pos + p * B;
     chunk_carry += total;
   }
   if (threadIdx.x == 0) {

@@ -155,12 +155,12 @@ struct CompactArgs {
   const int32_t* seg_batch;  // [n_seg] BatchSize of the segment's stream
   const int32_t* seg_slot;   // [n_seg] stats slot of the segment's stream
   unsigned long long* stats; // SNM_BATCHES (pops) counted here; may be nullptr
-  int32_t snm_ctas;          // SNM grid size: pops are split into work units of ~m/snm_ctas frames
+  int32_t snm_ctas;          // K4 grid size, 0 for SDD-only batches (then no dynamic batches are counted)
   int32_t* survivor_idx;     // [n] out
   int32_t* work;             // [n] out: survivors in work order (frame indices)
   int32_t* posw;             // [n + 1] scratch: exclusive survivor count in perm order
-  int32_t* chunks;           // [n + 1] out: chunk k = work[chunks[k] .. chunks[k+1]) (one stream, <= BatchSize)
-  int32_t* counts;           // [4] out: m, n_chunks, chunk cursor (reset 0), pad
+  int32_t* chunks;           // [n + 1] out: pop k = work[chunks[k] .. chunks[k+1]) (one stream, <= BatchSize)
+  int32_t* counts;           // [4] out: m, n_chunks, 0, pad
   float* logit;              // [n] initialised here: NaN / 0 / 0 (the SNM kernel overwrites survivors)
   uint8_t* snm_pass;
   uint8_t* snm_class;
@@ -174,7 +174,7 @@ struct SnmArgs {
   const int32_t* d50_index;  // optional [n]: frame f's D50 image is slot d50_index[f]
   const int32_t* work;
   const int32_t* chunks;
-  int32_t* counts;           // m, n_chunks, cursor
+  int32_t* counts;           // m (survivors), n_chunks
   const uint8_t* pop_start;  // optional [n_chunks]: 1 if the unit opens a dynamic batch (online mode counts
                              // SNM_BATCHES here; batch mode counts them in K3)
   float* logit;              // [n] (frame order)

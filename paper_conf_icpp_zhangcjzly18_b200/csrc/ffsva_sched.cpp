@@ -273,13 +273,11 @@ SnmStage prep_snm(ffsva_sched* s, uint8_t* h, const Layout& L, std::vector<sched
   int32_t nch = 0;
   for (size_t p = 0; p + 1 < starts.size(); ++p) {
     const ffsva_stream* st = s->by_id[flat[starts[p]].stream];
-    // a pop is split into work units of U frames so small cycles still spread over the SMs
-    const int32_t U = std::max(1, std::min(st->desc.snm_batch, m / std::max(1, kSnmCtasPerSm * s->ctx->num_sms)));
     const FrameDesc d = make_desc(st, nullptr);
     for (int32_t j = starts[p]; j < starts[p + 1]; ++j) {
       const int32_t k = j - starts[p];
-      if (k % U == 0) {
-        hpop[nch] = k == 0 ? 1 : 0;
+      if (k == 0) {  // one chunk per pop (K4 counts SNM_BATCHES per chunk that opens a pop)
+        hpop[nch] = 1;
         hch[nch++] = j;
       }
       hd[j] = d;
@@ -322,7 +320,7 @@ cudaError_t enqueue_snm_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layo
   na.snm_pass = s->d_out + 13 * n;
   na.snm_class = s->d_out + 14 * n;
   na.stats = s->ctx->d_stats;
-  na.grid = std::max(1, std::min(nch, kSnmCtasPerSm * s->ctx->num_sms));
+  na.grid = std::max(1, std::min(m, kSnmCtasPerSm * s->ctx->num_sms));  // K4: per-CTA ranges of the m pops' frames
   if (e == cudaSuccess) e = launch_snm(na, cs);
   g_launches += 1;
   if (e == cudaSuccess) e = cudaMemcpyAsync(at<float>(s->h_out, 8 * n), na.logit, 4 * (size_t)m, cudaMemcpyDeviceToHost, cs);
