@@ -32,7 +32,7 @@ size_t al256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 // Per-cycle staging: one pinned host block mirrored by one device block (a single H2D per stage).
 struct Layout {
-  size_t desc, index, work, chunks, counts, seg_lo, seg_batch, seg_slot, pop_start, total;
+  size_t desc, index, work, chunks, counts, seg_lo, seg_batch, seg_slot, pop_start, xb, yb, total;
   explicit Layout(size_t n) {
     size_t o = 0;
     desc = o; o += al256(64 * n);
@@ -44,6 +44,8 @@ struct Layout {
     seg_batch = o; o += al256(4 * n);
     seg_slot = o; o += al256(4 * n);
     pop_start = o; o += al256(n);
+    xb = o; o += al256(4 * 4097);  // cell boundary tables of a cycle whose frames share W / H (grids <= 4096)
+    yb = o; o += al256(4 * 4097);
     total = o;
   }
 };
@@ -71,7 +73,8 @@ struct ffsva_sched {
   int32_t *d_perm = nullptr, *d_posw = nullptr, *d_surv = nullptr;
   unsigned long long* d_acc = nullptr;
   uint8_t* d_out = nullptr;   // ssd u64[cap] | logit f32[cap] | pass u8[cap] | snm_pass u8[cap] | snm_class u8[cap]
-  uint8_t* h_out = nullptr;
+  uint8_t* h_out = nullptr;   // 2 result buffers (15 * cap bytes each): a cycle's D2H lands in h_out + hb * 15 * cap
+  uint8_t* h_out_cur = nullptr;  // the launching cycle's result buffer (enqueue_*_stage)
   // events not yet returned: pending[pend_head ..) (a vector with a consumed prefix, reset when drained)
   std::vector<ffsva_event> pending;
   size_t pend_head = 0;
@@ -79,11 +82,13 @@ struct ffsva_sched {
   std::vector<sched::QFrame> flat;  // this cycle's SNM pops, reused
   std::vector<int32_t> starts;
   // pipelined mode (ffsva_sched_set_pipeline): the kernels tick k launches are harvested by tick k + 1, so the
-  // caller's work between ticks and the next cycle's host preparation overlap them. Host staging is double
-  // buffered (hb), the device staging holds separate SDD and SNM regions.
+  // caller's work between ticks and the next cycle's host preparation overlap them. Host staging and host result
+  // buffers are double buffered (hb; the in-flight cycle's is f_hb), the device staging holds separate SDD and SNM
+  // regions (stream order separates consecutive cycles). Without a T-YOLO stage tick k launches cycle k before it
+  // waits for and harvests cycle k-1, so the GPU never idles on the harvest.
   bool pipelined = false, inflight = false;
-  int32_t hb = 0;
-  cudaEvent_t done_ev = nullptr;
+  int32_t hb = 0, f_hb = 0;
+  cudaEvent_t ev[2] = {nullptr, nullptr};  // ev[b]: the cycle launched with buffers b has finished
   std::vector<sched::QFrame> f_adm, f_flat;  // the in-flight cycle's admissions and pops
   // T-YOLO stage (f1): the device's shared model, its per-cycle extraction and score threshold
   ffsva_tyolo* tyolo = nullptr;
@@ -99,7 +104,8 @@ namespace {
 void sched_free(ffsva_sched* s) {
   if (s->g_sdd) cudaGraphExecDestroy(s->g_sdd);
   if (s->g_snm) cudaGraphExecDestroy(s->g_snm);
-  if (s->done_ev) cudaEventDestroy(s->done_ev);
+  for (cudaEvent_t e : s->ev)
+    if (e) cudaEventDestroy(e);
   cudaFree(s->d_pool);
   cudaFree(s->d_in);
   cudaFree(s->d_mem);
@@ -131,6 +137,7 @@ T* at(uint8_t* base, size_t off) { return reinterpret_cast<T*>(base + off); }
 // ---------------------------------------------------------------- cycle phases (shared by both tick modes)
 struct SddStage {
   int32_t na = 0, nseg = 0, sdd_w = 0, sdd_h = 0;
+  int32_t uni_W = -1, uni_H = -1;  // the admitted frames' common width / height (-1: mixed)
   SddPlan plan;
 };
 struct SnmStage {
@@ -168,6 +175,23 @@ SddStage prep_sdd(ffsva_sched* s, uint8_t* h, const Layout& L, std::vector<sched
   }
   hseg[sd.nseg] = sd.na;
   sdd_plan_finish(sd.plan, sd.sdd_w, sd.sdd_h);
+  // cell boundary tables (C1) when every admitted frame has the same width / height: K1 then reads its row and
+  // column bounds without waiting for its frame descriptor (as prepared batches do)
+  sd.uni_W = s->by_id[adm[0].stream]->desc.width;
+  sd.uni_H = s->by_id[adm[0].stream]->desc.height;
+  for (int32_t i = 1; i < sd.na && (sd.uni_W > 0 || sd.uni_H > 0); ++i) {
+    const ffsva_stream_desc& d = s->by_id[adm[i].stream]->desc;
+    if (d.width != sd.uni_W) sd.uni_W = -1;
+    if (d.height != sd.uni_H) sd.uni_H = -1;
+  }
+  if (sd.uni_W > 0) {
+    int32_t* hxb = at<int32_t>(h, L.xb);
+    for (int32_t i = 0; i <= sd.sdd_w; ++i) hxb[i] = (int32_t)(((int64_t)i * sd.uni_W) / sd.sdd_w);
+  }
+  if (sd.uni_H > 0) {
+    int32_t* hyb = at<int32_t>(h, L.yb);
+    for (int32_t i = 0; i <= sd.sdd_h; ++i) hyb[i] = (int32_t)(((int64_t)i * sd.uni_H) / sd.sdd_h);
+  }
   return sd;
 }
 
@@ -186,6 +210,10 @@ cudaError_t enqueue_sdd_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layo
     e = cudaMemcpyAsync(d + L.seg_batch, h + L.seg_batch, 4 * (size_t)nseg, cudaMemcpyHostToDevice, cs);
   if (e == cudaSuccess)
     e = cudaMemcpyAsync(d + L.seg_slot, h + L.seg_slot, 4 * (size_t)nseg, cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess && sd.uni_W > 0)
+    e = cudaMemcpyAsync(d + L.xb, h + L.xb, 4 * (size_t)(sd.sdd_w + 1), cudaMemcpyHostToDevice, cs);
+  if (e == cudaSuccess && sd.uni_H > 0)
+    e = cudaMemcpyAsync(d + L.yb, h + L.yb, 4 * (size_t)(sd.sdd_h + 1), cudaMemcpyHostToDevice, cs);
   SddArgs sa{};
   sa.frames = at<FrameDesc>(d, L.desc);
   sa.n = na;
@@ -197,6 +225,11 @@ cudaError_t enqueue_sdd_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layo
   sa.acc_ssd = s->d_acc;
   sa.stats = ctx->d_stats;
   sdd_plan_apply(sd.plan, sa);
+  sa.uni_W = sd.uni_W;
+  sa.uni_H = sd.uni_H;
+  sa.cellw = sd.uni_W > 0 ? (sd.uni_W + sd.sdd_w - 1) / sd.sdd_w : 0;
+  sa.xbounds = sd.uni_W > 0 ? at<int32_t>(d, L.xb) : nullptr;
+  sa.ybounds = sd.uni_H > 0 ? at<int32_t>(d, L.yb) : nullptr;
   if (e == cudaSuccess) e = launch_sdd(sa, cs);
   CompactArgs ca{};  // threshold + per-stream SDD-pass stats; no SNM work units (snm_ctas = 0)
   ca.frames = sa.frames;
@@ -221,17 +254,19 @@ cudaError_t enqueue_sdd_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layo
   ca.snm_class = s->d_out + 14 * n;
   if (e == cudaSuccess) e = launch_compact(ca, cs);
   g_launches += 2;
-  if (e == cudaSuccess) e = cudaMemcpyAsync(at<uint64_t>(s->h_out, 0), ca.ssd, 8 * (size_t)na, cudaMemcpyDeviceToHost, cs);
-  if (e == cudaSuccess) e = cudaMemcpyAsync(s->h_out + 12 * n, ca.pass, (size_t)na, cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(at<uint64_t>(s->h_out_cur, 0), ca.ssd, 8 * (size_t)na, cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(s->h_out_cur + 12 * n, ca.pass, (size_t)na, cudaMemcpyDeviceToHost, cs);
   return e;
 }
 
-// SDD results (in h_out) of admissions adm[0, na): survivors join their SNM queue, dropped frames become events.
-void harvest_sdd(ffsva_sched* s, std::vector<sched::QFrame>& adm, int32_t na, ffsva_tick_info& ti) {
+// SDD results (in result buffer hout) of admissions adm[0, na): survivors join their SNM queue, dropped frames
+// become events.
+void harvest_sdd(ffsva_sched* s, const uint8_t* hout, std::vector<sched::QFrame>& adm, int32_t na,
+                 ffsva_tick_info& ti) {
   NvtxRange r("ffsva sched: SDD harvest");
   const size_t n = (size_t)s->cap;
-  const uint64_t* h_ssd = at<uint64_t>(s->h_out, 0);
-  const uint8_t* h_pass = s->h_out + 12 * n;
+  const uint64_t* h_ssd = reinterpret_cast<const uint64_t*>(hout);
+  const uint8_t* h_pass = hout + 12 * n;
   const int64_t t_now = now_us();
   for (int32_t i = 0; i < na; ++i) {
     adm[i].ssd = h_ssd[i];
@@ -323,9 +358,9 @@ cudaError_t enqueue_snm_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layo
   na.grid = std::max(1, std::min(m, kSnmCtasPerSm * s->ctx->num_sms));  // K4: per-CTA ranges of the m pops' frames
   if (e == cudaSuccess) e = launch_snm(na, cs);
   g_launches += 1;
-  if (e == cudaSuccess) e = cudaMemcpyAsync(at<float>(s->h_out, 8 * n), na.logit, 4 * (size_t)m, cudaMemcpyDeviceToHost, cs);
-  if (e == cudaSuccess) e = cudaMemcpyAsync(s->h_out + 13 * n, na.snm_pass, (size_t)m, cudaMemcpyDeviceToHost, cs);
-  if (e == cudaSuccess) e = cudaMemcpyAsync(s->h_out + 14 * n, na.snm_class, (size_t)m, cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(at<float>(s->h_out_cur, 8 * n), na.logit, 4 * (size_t)m, cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(s->h_out_cur + 13 * n, na.snm_pass, (size_t)m, cudaMemcpyDeviceToHost, cs);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(s->h_out_cur + 14 * n, na.snm_class, (size_t)m, cudaMemcpyDeviceToHost, cs);
   return e;
 }
 
@@ -375,14 +410,14 @@ cudaError_t launch_snm_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layou
   return graph_launch(s->g_snm, cs, [&] { return enqueue_snm_stage(s, h, d, L, sn, cs); });
 }
 
-// SNM results (in h_out) of pops flat[0, m): slots are freed; survivors with a T-YOLO stage wait in its queue,
-// every other frame becomes an event.
-void harvest_snm(ffsva_sched* s, std::vector<sched::QFrame>& flat, int32_t m) {
+// SNM results (in result buffer hout) of pops flat[0, m): slots are freed; survivors with a T-YOLO stage wait in its
+// queue, every other frame becomes an event.
+void harvest_snm(ffsva_sched* s, const uint8_t* hout, std::vector<sched::QFrame>& flat, int32_t m) {
   NvtxRange r("ffsva sched: SNM harvest");
   const size_t n = (size_t)s->cap;
-  const float* h_logit = at<float>(s->h_out, 8 * n);
-  const uint8_t* h_snm_pass = s->h_out + 13 * n;
-  const uint8_t* h_snm_class = s->h_out + 14 * n;
+  const float* h_logit = reinterpret_cast<const float*>(hout + 8 * n);
+  const uint8_t* h_snm_pass = hout + 13 * n;
+  const uint8_t* h_snm_class = hout + 14 * n;
   const int64_t t_now = now_us();
   for (int32_t k = 0; k < m; ++k) {
     s->free_slots.push_back(flat[k].slot);
@@ -468,8 +503,10 @@ FFSVA_API ffsva_status ffsva_sched_create(int32_t device, int32_t max_frames_per
   if (e == cudaSuccess) e = cudaMalloc(&s->d_pool, (size_t)snm_slots * kD50Stride);
   if (e == cudaSuccess) e = cudaMalloc(&s->d_in, 2 * L.total);       // SDD region | SNM region
   if (e == cudaSuccess) e = cudaMallocHost(&s->h_in, 4 * L.total);   // 2 buffers x (SDD | SNM)
-  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&s->done_ev, cudaEventDisableTiming);
-  if (e == cudaSuccess) e = cudaMallocHost(&s->h_out, 15 * n);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&s->ev[0], cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaEventCreateWithFlags(&s->ev[1], cudaEventDisableTiming);
+  if (e == cudaSuccess) e = cudaMallocHost(&s->h_out, 2 * 15 * n);
+  s->h_out_cur = s->h_out;
   if (e == cudaSuccess) {
     uint8_t* b = (uint8_t*)s->d_mem;
     s->d_perm = at<int32_t>(b, o_perm);
@@ -654,17 +691,19 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
   ffsva_status st = FFSVA_OK;
   std::chrono::steady_clock::time_point t_snm0, t_ty0;
 
+  const size_t out_bytes = 15 * (size_t)s->cap;
   if (!s->pipelined) {
     // ---------------- synchronous cycle: SDD (launch, wait, harvest), then SNM on the updated queues
     uint8_t* hs = s->h_in;
     uint8_t* hn = s->h_in + L.total;
+    s->h_out_cur = s->h_out;
     SddStage sd = prep_sdd(s, hs, L, s->adm);
     ti.admitted = sd.na;
     if (sd.na > 0) {
       cudaError_t e = launch_sdd_stage(s, hs, d_sdd, L, sd, cs);
       if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
       if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (SDD cycle)");
-      harvest_sdd(s, s->adm, sd.na, ti);
+      harvest_sdd(s, s->h_out, s->adm, sd.na, ti);
     }
     t_snm0 = std::chrono::steady_clock::now();
     SnmStage sn = prep_snm(s, hn, L, s->flat, s->starts, ti);
@@ -672,38 +711,55 @@ FFSVA_API ffsva_status ffsva_sched_tick(ffsva_sched* s, void* cuda_stream, ffsva
       cudaError_t e = launch_snm_stage(s, hn, d_snm, L, sn, cs);
       if (e == cudaSuccess) e = cudaStreamSynchronize(cs);
       if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (SNM cycle)");
-      harvest_snm(s, s->flat, sn.m);
+      harvest_snm(s, s->h_out, s->flat, sn.m);
     }
     t_ty0 = std::chrono::steady_clock::now();
     if ((st = tyolo_cycle(s, cs, ti)) != FFSVA_OK) return st;
   } else {
-    // ---------------- pipelined cycle: prepare this cycle on the host while the previous one runs, then harvest
-    // the previous one, run the T-YOLO cycle on its survivors, and launch this one without waiting for it
+    // ---------------- pipelined cycle: prepare this cycle on the host while the previous one runs; without a
+    // T-YOLO stage launch it at once, then wait for and harvest the previous one (its results are in the other
+    // result buffer); with one, harvest first (the T-YOLO cycle runs on the previous cycle's SNM survivors before
+    // this cycle's kernels are queued behind it)
     uint8_t* hs = s->h_in + (size_t)(2 * s->hb) * L.total;
     uint8_t* hn = hs + L.total;
     SddStage sd = prep_sdd(s, hs, L, s->adm);
     ti.admitted = sd.na;
     SnmStage sn = prep_snm(s, hn, L, s->flat, s->starts, ti);
+    const bool launch = sd.na > 0 || sn.m > 0;
+    auto launch_cycle = [&]() -> cudaError_t {
+      s->h_out_cur = s->h_out + (size_t)s->hb * out_bytes;
+      cudaError_t e = cudaSuccess;
+      if (sd.na > 0) e = launch_sdd_stage(s, hs, d_sdd, L, sd, cs);
+      if (e == cudaSuccess && sn.m > 0) e = launch_snm_stage(s, hn, d_snm, L, sn, cs);
+      if (e == cudaSuccess) e = cudaEventRecord(s->ev[s->hb], cs);
+      return e;
+    };
+    const bool early = launch && s->tyolo == nullptr;
+    if (early) {
+      cudaError_t e = launch_cycle();
+      if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (launch)");
+    }
     if (s->inflight) {
-      cudaError_t e = cudaEventSynchronize(s->done_ev);
+      cudaError_t e = cudaEventSynchronize(s->ev[s->f_hb]);
       if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (in-flight cycle)");
-      harvest_sdd(s, s->f_adm, (int32_t)s->f_adm.size(), ti);
-      harvest_snm(s, s->f_flat, (int32_t)s->f_flat.size());
+      const uint8_t* hout = s->h_out + (size_t)s->f_hb * out_bytes;
+      harvest_sdd(s, hout, s->f_adm, (int32_t)s->f_adm.size(), ti);
+      harvest_snm(s, hout, s->f_flat, (int32_t)s->f_flat.size());
       s->inflight = false;
     }
     t_snm0 = std::chrono::steady_clock::now();
     t_ty0 = t_snm0;
     if ((st = tyolo_cycle(s, cs, ti)) != FFSVA_OK) return st;
-    if (sd.na > 0 || sn.m > 0) {
-      cudaError_t e = cudaSuccess;
-      if (sd.na > 0) e = launch_sdd_stage(s, hs, d_sdd, L, sd, cs);
-      if (e == cudaSuccess && sn.m > 0) e = launch_snm_stage(s, hn, d_snm, L, sn, cs);
-      if (e == cudaSuccess) e = cudaEventRecord(s->done_ev, cs);
-      if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (launch)");
+    if (launch) {
+      if (!early) {
+        cudaError_t e = launch_cycle();
+        if (e != cudaSuccess) return cuda_fail(ctx, e, "ffsva_sched_tick (launch)");
+      }
       s->f_adm.swap(s->adm);
       s->f_adm.resize((size_t)sd.na);
       s->f_flat.swap(s->flat);
       s->f_flat.resize((size_t)sn.m);
+      s->f_hb = s->hb;
       s->inflight = true;
       s->hb ^= 1;
     }
@@ -756,7 +812,7 @@ FFSVA_API ffsva_status ffsva_sched_inspect(ffsva_sched* s, ffsva_frame* frames, 
     lists[0] = &s->f_adm;
     lists[1] = &s->f_flat;
   }
-  cudaError_t e = s->pipelined ? cudaEventSynchronize(s->done_ev) : cudaSuccess;
+  cudaError_t e = s->pipelined ? cudaEventSynchronize(s->ev[s->f_hb]) : cudaSuccess;
   int32_t k = 0;
   for (int st = 0; st < 2 && e == cudaSuccess; ++st)
     for (const sched::QFrame& q : *lists[st]) {
