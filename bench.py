@@ -730,7 +730,7 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs, ws=1):
     explicit = [int(t) for t in args.online.split(",") if t.strip() and t.strip() != "auto"]
     out["runs"] = [run(S, pool, args.online_seconds, False) for S in explicit]
     if "auto" in args.online:
-        lad = climb((0.55, 0.7, 0.85, 0.9, 0.95), pool, args.online_confirm_seconds, False)
+        lad = climb((0.55, 0.7, 0.85, 0.9, 0.95, 1.0), pool, args.online_confirm_seconds, False)
         out["sdd_snm"] = lad
         out["max_sustained_streams_validated"] = lad["max_sustained_streams_validated"]
         out["validation_window_s"] = lad["validation_window_s"]
@@ -968,7 +968,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--online", default="30,auto",
                     help="comma-separated stream counts for the paced online validation (config m2); 'auto' = "
-                         "a ladder of 55/70/85/90/95%% of the measured frames/s / 30, climbed until a count is not "
+                         "a ladder of 55/70/85/90/95/100%% of the measured frames/s / 30, climbed until a count is not "
                          "sustained; empty to skip")
     ap.add_argument("--online-seconds", type=float, default=4.0, help="seconds per ladder rung")
     ap.add_argument("--online-confirm-seconds", type=float, default=30.0,
