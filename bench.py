@@ -333,17 +333,20 @@ class GpuEngine:
         torch.cuda.synchronize()
         S = len(self.sids)
         self.S, self.PF, self.SF = S, PF, SF
-        # prepared batches: batch j = frames [j*SF, (j+1)*SF) of every owned stream (one second of video)
-        self.nbatches = max(1, PF // SF)
+        # prepared batches: batch j = frames [j*SF, (j+1)*SF) of every owned stream (one second of video); a pool of
+        # exactly one batch (M1, M5) gets one prepared copy per CUDA stream (same frames, own buffers), so consecutive
+        # steps overlap like the other configs' (each step still runs K1 -> K3 -> K4 on all of its frames)
+        uniq = max(1, PF // SF)
+        self.nbatches = uniq if uniq > 1 else max(1, args.streams)
 
         def make(nstreams):
-            return [self.ctx.prepare([(self.streams[k], self.pool[k, j * SF + i], j * SF + i)
+            return [self.ctx.prepare([(self.streams[k], self.pool[k, (j % uniq) * SF + i], (j % uniq) * SF + i)
                                       for k in range(nstreams) for i in range(SF)]) for j in range(self.nbatches)]
         self.batches = make(S)
         self.solo_batches = make(S_all) if S_all != S else self.batches
         self.frames_per_step = S * SF
         self.solo_frames_per_step = S_all * SF
-        self.planted = [sum(synth.planted(self.video, s, j * SF, (j + 1) * SF) for s in self.sids)
+        self.planted = [sum(synth.planted(self.video, s, (j % uniq) * SF, (j % uniq + 1) * SF) for s in self.sids)
                         for j in range(self.nbatches)]
         self.cs = torch.cuda.Stream(device=dev)
         nstr = max(1, min(args.streams, self.nbatches))
