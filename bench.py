@@ -511,8 +511,9 @@ def run_ours(args, cfg, ws, rank, local):
             "config": {"workload": cfg["desc"], "config_id": args.config, "streams_per_gpu": S,
                        "frames_per_step": int(total_frames // args.steps), "frames_per_step_per_gpu": frames_per_step,
                        "frame_bytes": eng.fbytes, "pool_bytes_per_gpu": int(S * eng.PF * eng.fbytes),
-                       "l2": "inputs larger than L2: each step reads a different %.2f GB slice of the pool"
-                             % (frames_per_step * eng.fbytes / 1e9),
+                       "l2": ("inputs larger than L2: each step reads a different %.2f GB slice of the pool"
+                              % (frames_per_step * eng.fbytes / 1e9) if eng.PF > eng.SF else
+                              "inputs larger than L2: each step reads the whole %.2f GB pool" % (S * eng.PF * eng.fbytes / 1e9)),
                        "parallelism": (f"stream-sharded x{ws} (strong: {cfg['streams']} streams split, {S} on rank 0)"
                                        if eng.strong else f"stream-sharded x{ws} (weak: {S} streams per GPU)"),
                        "dist_backend": args.dist_backend if ws > 1 else None,
