@@ -231,7 +231,7 @@ cudaError_t enqueue_sdd_stage(ffsva_sched* s, uint8_t* h, uint8_t* d, const Layo
   sa.xbounds = sd.uni_W > 0 ? at<int32_t>(d, L.xb) : nullptr;
   sa.ybounds = sd.uni_H > 0 ? at<int32_t>(d, L.yb) : nullptr;
   if (e == cudaSuccess) e = launch_sdd(sa, cs);
-  CompactArgs ca{};  // threshold + per-stream SDD-pass stats; no SNM work units (snm_ctas = 0)
+  CompactArgs ca{};  // threshold + per-stream SDD-pass stats; the SNM stage forms its own pops (snm_ctas = 0)
   ca.frames = sa.frames;
   ca.acc_ssd = s->d_acc;
   ca.ssd = at<uint64_t>(s->d_out, 0);
