@@ -664,9 +664,9 @@ def online_validation(args, ctx, video, sids, pool, value, dev, cs, ws=1):
     ty = None
     state = {"ty_warm": False}
 
-    # a device context holds at most 131,072 streams (the statistics table's rows): the ladders stop below it,
-    # leaving room for the benchmark's own streams
-    s_cap = 131072 - 512
+    # a device context holds at most 65,536 streams (the statistics table's rows; FrameDesc.slot is 16-bit): the
+    # ladders stop below it, leaving room for the benchmark's own streams
+    s_cap = 65536 - 512
 
     def run(S, content, seconds, with_ty):
         S = min(S, s_cap)

@@ -20,9 +20,9 @@ struct FrameDesc {
   int32_t W, H;            // raw size
   float L_t;               // logit threshold for t_pre (Eq. (2)); pass iff logit >= L_t
   float L_low, L_high;     // logit(c_low), logit(c_high) for the class (L159)
-  uint32_t slot : 24;      // stream slot (stats row; < kMaxSlots per device)
-  uint32_t metric : 4;     // SDD distance: kDistMse / kDistSad / kDistNrmse (ffsva_distance)
-  uint32_t mode : 4;       // SDD reference: kRefBackground / kRefPrevious (ffsva_ref_mode)
+  uint16_t slot;           // stream slot (stats row; < 65536 slots per device)
+  uint8_t metric;          // SDD distance: kDistMse / kDistSad / kDistNrmse (ffsva_distance)
+  uint8_t mode;            // SDD reference: kRefBackground / kRefPrevious (ffsva_ref_mode)
 };
 constexpr uint8_t kDistMse = 0, kDistSad = 1, kDistNrmse = 2;
 constexpr uint8_t kRefBackground = 0, kRefPrevious = 1;

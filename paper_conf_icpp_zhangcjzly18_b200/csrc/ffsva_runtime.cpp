@@ -15,7 +15,7 @@ std::atomic<uint64_t> g_launches{0};
 static thread_local std::string t_err;
 static std::mutex g_mu;
 static DeviceCtx* g_ctx[64] = {nullptr};
-constexpr int32_t kMaxSlots = 131072;  // stats table rows = streams per device (fixed: graphs never see a realloc)
+constexpr int32_t kMaxSlots = 65536;  // stats table rows per device (fixed so graphs never see a realloc)
 
 void set_error(const std::string& msg) { t_err = msg; }
 const char* last_error() { return t_err.c_str(); }
@@ -470,7 +470,7 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
     d.L_t = s->L_t;
     d.L_low = s->L_low;
     d.L_high = s->L_high;
-    d.slot = (uint32_t)s->slot;
+    d.slot = (uint16_t)s->slot;
     d.metric = (uint8_t)s->desc.distance;
     d.mode = (uint8_t)s->desc.ref_mode;
     hperm[i] = i;
@@ -504,7 +504,7 @@ ffsva_status batch_build(DeviceCtx* ctx, Batch* b, const ffsva_frame* frames, in
         prev = it->second;
         it->second = i;
       } else {
-        last.emplace_back((int32_t)hd[i].slot, i);
+        last.emplace_back(hd[i].slot, i);
       }
       hpm[2 * npm] = i;
       hpm[2 * npm + 1] = prev;

@@ -125,7 +125,7 @@ FrameDesc make_desc(const ffsva_stream* st, const void* pixels) {
   d.L_t = st->L_t;
   d.L_low = st->L_low;
   d.L_high = st->L_high;
-  d.slot = (uint32_t)st->slot;
+  d.slot = (uint16_t)st->slot;
   d.metric = (uint8_t)st->desc.distance;
   d.mode = (uint8_t)st->desc.ref_mode;
   return d;
